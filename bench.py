@@ -1,0 +1,365 @@
+#!/usr/bin/env python
+"""Benchmark of the fused RAP preprocessing kernel (BASELINE.json metric:
+preprocessed samples/s, % of HBM roofline).
+
+A step = one rap_preprocess launch over one synthetic Criteo-Terabyte-shaped
+batch (config 2, 65536 rows, the full 152-op graph) — every §8(a) row of the
+hot path.  Inputs are resident in HBM when the timed region starts; the
+batch/output sets are rotated so their total exceeds 2x the L2 (126 MB).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl rap|reference]
+
+Prints ONE JSON line on rank 0.  `--impl reference` times the CPU oracle (the
+task's reference arm for a paper-only reference) on bounded samples.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "preprocessed samples/s"
+UNIT = "samples/s"
+WORKLOADS = {"c2": ("criteo_terabyte_c2", 65536), "c1": ("criteo_kaggle_c1", 4096), "c4": ("multihot_c4", 131072)}
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=3000)
+    ap.add_argument("--warmup", type=int, default=50)
+    ap.add_argument("--impl", default="rap", choices=["rap", "reference"])
+    ap.add_argument("--workload", default="c2", choices=list(WORKLOADS))
+    ap.add_argument("--batch", type=int, default=0, help="override rows per batch")
+    ap.add_argument("--budget", type=int, default=0, help="SM budget (0 = all SMs)")
+    ap.add_argument("--e2e-steps", type=int, default=30)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=10.0)
+    ap.add_argument("--profile", action="store_true", help="short run for ncu (no clocks / e2e / cpu)")
+    return ap.parse_args()
+
+
+def workload(name, seed=0):
+    from paper_conf_asplos_wangwdz0d24_b200 import synth
+
+    if name == "c2":
+        return synth.c2_terabyte(seed)
+    if name == "c1":
+        return synth.c1_kaggle(seed)
+    return synth.c4_multihot(seed)
+
+
+# ----------------------------------------------------------------------------- clocks
+class ClockSampler:
+    """Samples SM clock and throttle reasons with NVML while the timed region runs."""
+
+    REASONS = {"hw_slowdown": 0x8, "hw_thermal_slowdown": 0x40, "sw_thermal_slowdown": 0x20,
+               "sw_power_cap": 0x4, "hw_power_brake_slowdown": 0x80}
+
+    def __init__(self, index):
+        self.samples, self.reasons = [], set()
+        self.ok = False
+        try:
+            import pynvml
+
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception as e:  # noqa: BLE001
+            self.err = str(e)
+        self._stop = threading.Event()
+
+    def _run(self):
+        while not self._stop.is_set():
+            self.sample()
+            time.sleep(0.002)
+
+    def sample(self):
+        try:
+            mhz = self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM)
+            r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+            self.samples.append(mhz)
+            for k, bit in self.REASONS.items():
+                if r & bit:
+                    self.reasons.add(k)
+        except Exception:  # noqa: BLE001
+            pass
+
+    def __enter__(self):
+        if self.ok:
+            self.sample()
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        if self.ok:
+            self._stop.set()
+            self.t.join()
+            self.sample()
+
+    def summary(self):
+        if not self.ok or not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "samples": 0}
+        return {"sm_mhz": float(np.median(self.samples)), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+# ----------------------------------------------------------------------------- helpers
+def measured_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured"
+    except Exception:  # noqa: BLE001
+        return 6650.0, "fallback"
+
+
+def traffic_from_profile(workload_name):
+    """DRAM bytes per launch from the committed ncu --set full summary, if any."""
+    p = os.path.join(ROOT, "profiles", "traffic.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return d.get(workload_name)
+    except Exception:  # noqa: BLE001
+        return None
+
+
+def cpu_baseline(w, seconds, rows=8192):
+    """The oracle, as it stands, on a bounded sample of the same workload."""
+    from oracle import oracle
+    from paper_conf_asplos_wangwdz0d24_b200 import synth
+
+    host = synth.make_batch(w, rows, seed=101)
+    oracle.lib()
+    n = 0
+    t0 = time.perf_counter()
+    while True:
+        r = oracle.run(w.spec, host)
+        assert r["status"] == "OK"
+        n += 1
+        if time.perf_counter() - t0 >= seconds:
+            break
+    dt = time.perf_counter() - t0
+    return {"value": n * rows / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"{n} x {rows}-row batches of {w.name} (seed 101), single-threaded C oracle, {dt:.1f} s"}
+
+
+def dist_env():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+# ----------------------------------------------------------------------------- reference arm
+def run_reference(args):
+    rank, world, _ = dist_env()
+    if rank != 0:
+        return 0
+    from oracle import oracle
+    from paper_conf_asplos_wangwdz0d24_b200 import synth
+
+    wname, B = WORKLOADS[args.workload]
+    B = args.batch or B
+    w = workload(args.workload)
+    oracle.lib()
+    total_steps = args.steps + args.warmup
+    budget_s = 90.0
+    # oracle throughput ~6e4 rows/s on C2: size each step so the run stays within ~budget_s
+    rows = int(max(32, min(B, 6e4 * budget_s / max(total_steps, 1))))
+    host = synth.make_batch(w, rows, seed=202)
+    for _ in range(args.warmup):
+        oracle.run(w.spec, host)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        r = oracle.run(w.spec, host)
+    dt = time.perf_counter() - t0
+    assert r["status"] == "OK"
+    value = args.steps * rows / dt
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": 0,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64+f32",
+            "data": "synthetic",
+            "config": {"workload": wname, "batch": B, "sample_rows_per_step": rows, "parallelism": "cpu-1thread"},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
+                             "sample": f"{rows}-row sample of {wname} per step (seed 202), single-threaded C oracle"},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ----------------------------------------------------------------------------- GPU arm
+def run_rap(args):
+    import torch
+
+    rank, world, local = dist_env()
+    if world > 1:
+        import torch.distributed as dist
+
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    else:
+        torch.cuda.set_device(0)
+    dev = torch.device("cuda", torch.cuda.current_device())
+    from paper_conf_asplos_wangwdz0d24_b200 import rap, synth
+
+    wname, B = WORKLOADS[args.workload]
+    B = args.batch or B
+    w = workload(args.workload)
+    # Replicas: with N > 1 every rank preprocesses its own batch of B rows (data-parallel
+    # batches, no data-path collective) -> weak scaling, value = all ranks' rows / max time.
+    plan = rap.Plan(w.spec, device=dev.index, sm_budget=args.budget)
+    props = torch.cuda.get_device_properties(dev)
+    l2 = getattr(props, "L2_cache_size", 126 * 2**20)
+
+    first = synth.make_batch(w, B, seed=1000 + rank)
+    raw0 = rap.DeviceBatch(first, dev)
+    out0 = rap.DeviceOutput(plan, B, raw0.sp_nnz, dev)
+    d_out, f_out, vb = out0.d_out, out0.f_out, out0.bound
+    # algorithmic bytes of one launch: measured from the produced output
+    plan.preprocess(raw0, out0)
+    torch.cuda.synchronize()
+    n_vals = int(out0.offsets[-1].item())
+    alg_bytes = synth.algorithmic_bytes(w.spec, first, n_vals)
+    set_bytes = alg_bytes
+    nsets = 1 if args.profile else max(4, math.ceil(3 * l2 / max(set_bytes, 1)))
+    sets = [(raw0, out0)]
+    for i in range(1, nsets):
+        h = synth.make_batch(w, B, seed=1000 + rank + 97 * i)
+        r = rap.DeviceBatch(h, dev)
+        sets.append((r, rap.DeviceOutput(plan, B, r.sp_nnz, dev)))
+    stream = torch.cuda.current_stream(dev)
+
+    for i in range(args.warmup):
+        r, o = sets[i % nsets]
+        plan.preprocess(r, o, stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+
+    K = args.steps
+    ev_s = [torch.cuda.Event(enable_timing=True) for _ in range(K)]
+    ev_e = [torch.cuda.Event(enable_timing=True) for _ in range(K)]
+    t_start = torch.cuda.Event(enable_timing=True)
+    t_end = torch.cuda.Event(enable_timing=True)
+    sampler = ClockSampler(dev.index) if not args.profile else None
+    ctx = sampler if sampler else _Null()
+    with ctx:
+        t_start.record(stream)
+        for i in range(K):
+            r, o = sets[i % nsets]
+            ev_s[i].record(stream)
+            plan.preprocess(r, o, stream)
+            ev_e[i].record(stream)
+        t_end.record(stream)
+        t_end.synchronize()
+    torch.cuda.synchronize()
+    total_ms = t_start.elapsed_time(t_end)
+    kern_ms = float(np.mean([ev_s[i].elapsed_time(ev_e[i]) for i in range(K)]))
+    if world > 1:
+        import torch.distributed as dist
+
+        t = torch.tensor([total_ms, kern_ms], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        total_ms, kern_ms = float(t[0]), float(t[1])
+        dist.barrier()
+    ms_per_step = total_ms / K
+    value = world * B * K / (total_ms / 1e3)
+
+    # ---- correctness spot check of the last launch (cheap invariants, not the oracle)
+    o = sets[(K - 1) % nsets][1]
+    offs = o.offsets
+    assert int(offs[0]) == 0 and bool((offs[1:] >= offs[:-1]).all())
+
+    # ---- end to end through the C ABI with host buffers
+    e2e = None
+    if not args.no_e2e and not args.profile:
+        hraw = rap.DeviceBatch(first, None, pin=True)
+        hout = rap.DeviceOutput(plan, B, hraw.sp_nnz, None, pin=True)
+        h2d = sum(x.numel() * x.element_size() for x in hraw.dense)
+        h2d += sum(x.numel() * x.element_size() for x in hraw.dense_valid if x is not None)
+        h2d += sum(x.numel() * x.element_size() for x in hraw.sp_off)
+        h2d += sum(int(n) * 8 for n in hraw.sp_nnz)
+        h2d += sum(x.numel() * x.element_size() for x in hraw.sp_valid if x is not None)
+        d2h = (B * d_out * 4) + (B * f_out * 4) + (B * f_out + 1) * 8 + vb * 8
+        for _ in range(3):
+            plan.preprocess_host(hraw, hout, stream)
+        if world > 1:
+            torch.distributed.barrier()
+        E = max(3, args.e2e_steps)
+        t0 = time.perf_counter()
+        for _ in range(E):
+            plan.preprocess_host(hraw, hout, stream)
+        dt = time.perf_counter() - t0
+        if world > 1:
+            import torch.distributed as dist
+
+            t = torch.tensor([dt], device=dev, dtype=torch.float64)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            dt = float(t[0])
+        e2e = {"value": world * B * E / dt, "unit": UNIT, "h2d_bytes_per_step": int(h2d),
+               "d2h_bytes_per_step": int(d2h), "steps": E}
+
+    peak, peak_kind = measured_peaks()
+    achieved = alg_bytes / (kern_ms / 1e3) / 1e9
+    traffic = traffic_from_profile(wname)
+    roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+            "traffic": traffic, "peak_source": peak_kind, "alg_bytes_per_launch": int(alg_bytes),
+            "kernel_ms": kern_ms}
+    clocks = sampler.summary() if sampler else None
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline and not args.profile:
+        cpu = cpu_baseline(w, args.cpu_seconds)
+    info = plan.info()
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": args.warmup,
+                "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+                "dtype": "int64+f32", "data": "synthetic",
+                "config": {"workload": wname, "batch": B, "graph_ops": len(w.spec["nodes"]),
+                           "dense_out_cols": d_out, "sparse_out_features": f_out,
+                           "parallelism": "replicas" if world > 1 else "single-gpu",
+                           "sm_budget": info["sm_budget"], "grid": info["grid"],
+                           "l2_policy": f"rotate {nsets} distinct input/output sets, {nsets * set_bytes / 2**20:.0f} MB "
+                                        f"total vs L2 {l2 / 2**20:.0f} MB"},
+                "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks, "gpu_launches": K}
+        print(json.dumps(line), flush=True)
+    plan.close()
+    if world > 1:
+        import torch.distributed as dist
+
+        dist.destroy_process_group()
+    return 0
+
+
+class _Null:
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        return False
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_rap(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,208 @@
+/*
+ * rap.h — C ABI of the B200-native RAP fused DLRM input-preprocessing library
+ * (librap.so).  Paper: Wang et al., "RAP: Resource-aware Automated GPU Sharing
+ * for Multi-GPU Recommendation Model Training and Input Preprocessing",
+ * ASPLOS '24 (PAPER.md, cited L<line>).
+ *
+ * The calls follow the paper's problem statement: a plan is built once from
+ * "the computational graph of data preprocessing" plus the hardware and the
+ * co-running budget (L840-846 §4); each batch, one call turns the raw batch
+ * into the "input tensors" consumed by training (L466-469 §2.1); the budget
+ * can be changed between batches so the fused kernel fits the remaining GPU
+ * capacity (resource-aware sharding, L1351-1366 §6.2).
+ *
+ * Conventions (all entry points):
+ *  - Plain C types only; every pointer documented as HOST or DEVICE.
+ *  - Ownership: rap_plan_create deep-copies the graph and parameters (the
+ *    caller may free them on return).  The plan owns its device program blob,
+ *    descriptor table, scan-state and staging workspaces.  The caller owns
+ *    every raw-batch and output buffer and the CUDA stream.
+ *  - Errors: functions return rap_status; rap_last_error() gives a
+ *    thread-local human-readable detail of the last failure.  Asynchronous
+ *    device faults surface through the CUDA stream as usual.
+ *  - Concurrency: a plan is not re-entrant — use one plan per stream that
+ *    runs concurrently.  Results never depend on the SM budget.
+ *  - Operator semantics: DESIGN.md §3 (readings R1-R20 of Table 1).
+ */
+#ifndef RAP_H
+#define RAP_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  RAP_OK = 0,
+  RAP_ERR_INVALID_ARGUMENT = 1, /* null pointer, negative size, bad param index, bad budget */
+  RAP_ERR_INVALID_GRAPH = 2,    /* cycle, bad reference, unknown op, type mismatch (R20) */
+  RAP_ERR_INVALID_PARAM = 3,    /* operator parameter out of its domain (R20) */
+  RAP_ERR_CAPACITY = 4,         /* output buffer smaller than the host-computed bound */
+  RAP_ERR_UNSUPPORTED = 5,      /* valid graph outside what the kernel lowers (nested NGram) */
+  RAP_ERR_CUDA = 6,             /* a CUDA runtime call failed */
+  RAP_ERR_OUT_OF_MEMORY = 7
+} rap_status;
+
+/* Operators of PAPER.md Table 1 (L440-463). */
+typedef enum {
+  RAP_OP_FILLNULL = 0,   /* L462: "Fill NA/NaN values using the specified value"        (R10) */
+  RAP_OP_LOGIT = 1,      /* L446: "Logit transform for normalization"                   (R11) */
+  RAP_OP_BOXCOX = 2,     /* L448: "BoxCox transform for normalization"                  (R12) */
+  RAP_OP_ONEHOT = 3,     /* L449: "Apply one hot encoding to normalize dense features"  (R9)  */
+  RAP_OP_SIGRIDHASH = 4, /* L452: "Compute hash value to normalize list of sparse features" (R1-R3) */
+  RAP_OP_BUCKETIZE = 5,  /* L458: "Shard features based on bucket borders"              (R4)  */
+  RAP_OP_FIRSTX = 6,     /* L454: "List truncation of sparse features"                  (R5)  */
+  RAP_OP_CLAMP = 7,      /* L455: "Clamp the sparse input based on the upper and lower bound" (R6) */
+  RAP_OP_NGRAM = 8,      /* L459 + footnote L181-182: n-gram across multiple sparse features (R7) */
+  RAP_OP_MAPID = 9       /* L460: "Maps feature IDs to fixed values"                    (R8)  */
+} rap_op_type;
+
+/* Node input encoding: a value >= 0 is a node index; raw columns are encoded
+ * with these macros (dense column c is an f32 scalar per row, sparse column c
+ * an Arrow list<int64>). */
+#define RAP_RAW_DENSE(c) (-1 - 2 * (c))
+#define RAP_RAW_SPARSE(c) (-2 - 2 * (c))
+
+/* One DAG node (§2.3: a feature's preprocessing is a DAG).
+ * HOST memory.  `inputs` has n_inputs entries (1, or 1..8 for NGram);
+ * `param` indexes the rap_op_param array passed to rap_plan_create. */
+typedef struct {
+  int32_t op;            /* rap_op_type */
+  int32_t n_inputs;
+  const int32_t* inputs; /* node indices or RAP_RAW_* */
+  int32_t param;
+} rap_node;
+
+/* The whole preprocessing graph.  HOST memory.  Outputs are emitted in this
+ * order: Dense nodes as 1 dense column, OneHot nodes as K dense columns, Ids
+ * nodes as one jagged sparse feature (R17). */
+typedef struct {
+  int32_t n_dense_in, n_sparse_in, n_nodes;
+  const rap_node* nodes;
+  int32_t n_outputs;
+  const int32_t* output_nodes;
+} rap_graph;
+
+/* Operator parameters.  HOST memory; only the fields of the node's op are
+ * read.  `borders` is f32[n_borders] when Bucketize reads a Dense value and
+ * int64[n_borders] when it reads an id list. */
+typedef struct {
+  float f_fill, eps, lambda;
+  int64_t i_fill, lo, hi, x, max_value, map_default;
+  uint64_t salt;
+  int32_t n, k_width, n_borders;
+  const void* borders;
+  int64_t map_size;
+  const int64_t* map_keys;
+  const int64_t* map_vals;
+} rap_op_param;
+
+/* One raw columnar batch (Arrow layout: columnar data
+ * loaded to the GPU).  The pointer ARRAYS are HOST memory; the column buffers
+ * they point to are DEVICE memory for rap_preprocess and HOST memory for
+ * rap_preprocess_host.
+ *   dense[c]       f32[n_rows]
+ *   dense_valid[c] u32 bitmap, bit (b&31) of word b>>5, 1 = valid; the array
+ *                  itself or an entry may be NULL = all valid (R19)
+ *   sp_offsets[c]  int32[n_rows+1], absolute, non-decreasing (off[0] may be > 0)
+ *   sp_values[c]   int64 child values
+ *   sp_valid[c]    bitmap as above (NULL = all valid)
+ *   sp_nnz         HOST int64[n_sparse_in]: sp_offsets[c][n_rows] - sp_offsets[c][0]
+ *                  (used only for the host-side capacity bound and H2D sizes) */
+typedef struct {
+  int64_t n_rows;
+  const float* const* dense;
+  const uint32_t* const* dense_valid;
+  const int32_t* const* sp_offsets;
+  const int64_t* const* sp_values;
+  const uint32_t* const* sp_valid;
+  const int64_t* sp_nnz;
+} rap_raw_batch;
+
+/* Output "input tensors" (R17).  DEVICE memory for rap_preprocess, HOST for
+ * rap_preprocess_host.
+ *   dense_out  f32[n_rows * dense_ld], row-major, dense_ld >= d_out_cols
+ *   lengths    int32[n_sparse_out * n_rows], feature-major
+ *   offsets    int64[n_sparse_out * n_rows + 1]
+ *   values     int64[values_capacity]; values_capacity must be >= the bound
+ *              returned by rap_plan_output_shape, else RAP_ERR_CAPACITY. */
+typedef struct {
+  float* dense_out;
+  int64_t dense_ld;
+  int32_t* lengths;
+  int64_t* offsets;
+  int64_t* values;
+  int64_t values_capacity;
+} rap_output;
+
+struct rap_plan;
+typedef struct rap_plan rap_plan;
+
+/* Read-only description of a plan (HOST). */
+typedef struct {
+  int32_t device, sm_count, sm_budget, ctas_per_sm, threads_per_cta, grid;
+  int32_t n_dense_out_cols, n_sparse_out, n_dense_groups, rows_per_dense_desc;
+  int32_t max_rows_per_sparse_desc, min_rows_per_sparse_desc;
+  int64_t n_descriptors_last, n_launches;
+  int64_t smem_bytes;
+} rap_plan_info;
+
+/* Build a plan (the a0 row of DESIGN.md §1): validate the DAG and parameters
+ * (R20, same checks and codes as the oracle), lower every output to a device
+ * op program, precompute H(salt), sort MapId tables, size the descriptor
+ * geometry, query occupancy and set grid = f(sm_budget).  sm_budget in
+ * [1, #SMs] (the SMs' worth of CTA slots the kernel may hold, §6.2);
+ * 0 = all SMs.  `device` is a CUDA ordinal.  *out receives the plan. */
+rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, int32_t n_params,
+                           int32_t device, int32_t sm_budget, rap_plan** out);
+
+/* Shapes for a batch of n_rows rows.  sp_nnz: HOST int64[n_sparse_in] (may be
+ * NULL when n_rows == 0).  Outputs (HOST, any may be NULL): dense output
+ * columns, sparse output features, an upper bound on values written. */
+rap_status rap_plan_output_shape(const rap_plan* plan, int64_t n_rows, const int64_t* sp_nnz,
+                                 int64_t* d_out_cols, int64_t* n_sparse_out, int64_t* values_upper_bound);
+
+/* Enqueue one fused preprocessing launch on `stream` (a cudaStream_t; NULL =
+ * legacy default stream).  Device buffers.  No host synchronisation, no host
+ * reads of device data; the only allocation is the one-time growth of the
+ * plan's scan-state when n_rows exceeds every earlier call.  Outputs are valid
+ * when the stream reaches this point. */
+rap_status rap_preprocess(rap_plan* plan, const rap_raw_batch* raw, const rap_output* out, void* stream);
+
+/* Same as rap_preprocess with HOST raw and output buffers (pinned memory makes
+ * the copies asynchronous): copies the batch into plan-owned device staging,
+ * launches, copies dense/lengths/offsets and the first values_upper_bound
+ * values back, and synchronises `stream` before returning.  Host values beyond
+ * offsets[end] are unspecified. */
+rap_status rap_preprocess_host(rap_plan* plan, const rap_raw_batch* raw, const rap_output* out, void* stream);
+
+/* Change the SM budget for the next rap_preprocess (resource-aware sharding,
+ * L1351-1366).  sm_budget in [1, #SMs]; 0 = all SMs. */
+rap_status rap_set_budget(rap_plan* plan, int32_t sm_budget);
+
+/* Co-running cost model (§5, L871-879 and L1138-1143):
+ * predicted standalone latency P (microseconds) of one rap_preprocess for a
+ * batch of n_rows under sm_budget, from an analytic roofline predictor
+ * (bytes / bandwidth share of the budget + launch cost) that replaces the
+ * paper's XGBoost model (L1037-1057).  sp_nnz as in rap_plan_output_shape. */
+rap_status rap_predict_latency_us(const rap_plan* plan, int64_t n_rows, const int64_t* sp_nnz,
+                                  int32_t sm_budget, double* latency_us);
+
+/* Smallest budget whose predicted exposed latency T_delta = P - OC is <= 0
+ * for the given overlapping capacity OC (microseconds of training slack),
+ * L1138-1152; if none fits, the budget minimising T_delta (all SMs).
+ * Writes the budget and T_delta (HOST). */
+rap_status rap_choose_budget(const rap_plan* plan, int64_t n_rows, const int64_t* sp_nnz,
+                             double overlap_capacity_us, int32_t* sm_budget, double* t_delta_us);
+
+rap_status rap_plan_info_get(const rap_plan* plan, rap_plan_info* info);
+void rap_plan_destroy(rap_plan* plan);
+
+const char* rap_status_string(rap_status status);
+const char* rap_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* RAP_H */

@@ -1,0 +1,1022 @@
+// rap_plan.cpp — host planner and C ABI (include/rap.h).
+//
+// rap_plan_create = row a0 of DESIGN.md §1: validate the preprocessing DAG
+// with the R20 checks, lower every output to a device op
+// program (rap_internal.h), precompute H(salt) and sorted MapId / Bucketize
+// tables, size the (feature, row-range) descriptor geometry and the grid from
+// the SM budget (resource-aware sharding, L1351-1366 §6.2).  rap_preprocess
+// = row a1: one launch, no host sync.
+#include <cuda_runtime.h>
+#include <math.h>
+#include <stdint.h>
+#include <string.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstdlib>
+#include <limits>
+#include <numeric>
+#include <string>
+#include <utility>
+#include <vector>
+
+#include "../../include/rap.h"
+#include "rap_internal.h"
+
+using namespace rapk;
+
+namespace {
+
+thread_local std::string g_last_error;
+
+rap_status fail(rap_status s, const std::string& msg) {
+  g_last_error = msg;
+  return s;
+}
+
+rap_status cuda_fail(cudaError_t e, const char* what) {
+  return fail(RAP_ERR_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
+}
+
+// Node value types (DESIGN.md §3 "type system").
+enum VType { VT_NONE = 0, VT_DENSE = 1, VT_IDS = 2, VT_VEC = 3 };
+
+constexpr int kGroupCols = 64;        // dense output columns per dense descriptor
+constexpr int kRowsDense = 128;       // rows per dense descriptor
+constexpr int kRowsSparse = 1024;     // rows per sparse descriptor
+
+int64_t sat_add(int64_t a, int64_t b) {
+  if (a > INT64_MAX - b) return INT64_MAX;
+  return a + b;
+}
+int64_t sat_mul(int64_t a, int64_t b) {
+  if (a != 0 && b > INT64_MAX / a) return INT64_MAX;
+  return a * b;
+}
+
+}  // namespace
+
+struct rap_plan {
+  int device = 0, sm_count = 0, budget = 0, ctas_per_sm = 1, smem = 0;
+  int n_dense_in = 0, n_sparse_in = 0;
+  // lowered program (host copies)
+  std::vector<DevOp> ops;
+  std::vector<DenseExpr> dexprs;
+  std::vector<Chain> chains;
+  std::vector<NGramDesc> ngrams;
+  std::vector<Unit> units;
+  std::vector<Group> groups;
+  std::vector<SparseOut> souts;
+  std::vector<float> ftab;
+  std::vector<int64_t> itab;
+  std::vector<int> used_dense, used_sparse;
+  int d_out = 0, tile_ld = 1;
+  // device program blob
+  unsigned char* blob = nullptr;
+  size_t off_ops = 0, off_dexprs = 0, off_chains = 0, off_ngrams = 0, off_units = 0, off_groups = 0, off_souts = 0,
+         off_ftab = 0, off_itab = 0;
+  // per-n_rows descriptor table
+  int32_t* d_desc_start = nullptr;
+  int64_t desc_rows = -1;
+  std::vector<int32_t> h_desc_start;
+  int64_t n_sparse_desc = 0, n_dense_desc = 0;
+  // scheduling state
+  unsigned long long* d_sched = nullptr;  // ticket, done, epoch (device-managed)
+  unsigned long long* d_status = nullptr;
+  int64_t status_cap = 0;
+  int32_t* d_err = nullptr;
+  int64_t n_launches = 0;
+  int64_t last_n_desc = 0;
+  // host-buffer staging (rap_preprocess_host)
+  std::vector<void*> stage;
+  std::vector<size_t> stage_cap;
+};
+
+namespace {
+
+// ----------------------------------------------------------------------------
+// Validation (R20).  Mirrors the oracle's order; implemented independently.
+struct Validated {
+  std::vector<int> type;   // per node
+  std::vector<int> order;  // topological
+  int64_t d_out = 0, f_out = 0;
+};
+
+int in_type(const rap_graph* g, const std::vector<int>& type, int32_t ref) {
+  if (ref >= 0) return type[ref];
+  if ((-ref) % 2 == 1) return VT_DENSE;  // -1 - 2c
+  return VT_IDS;                          // -2 - 2c
+}
+
+bool ref_ok(const rap_graph* g, int32_t ref) {
+  if (ref >= 0) return ref < g->n_nodes;
+  int32_t m = -ref;
+  if (m % 2 == 1) {
+    int c = (m - 1) / 2;
+    return c < g->n_dense_in;
+  }
+  int c = (m - 2) / 2;
+  return c < g->n_sparse_in;
+}
+
+rap_status validate(const rap_graph* g, const rap_op_param* params, int32_t n_params, Validated* v) {
+  if (!g) return fail(RAP_ERR_INVALID_ARGUMENT, "graph is NULL");
+  if (g->n_dense_in < 0 || g->n_sparse_in < 0 || g->n_nodes < 0 || g->n_outputs < 0)
+    return fail(RAP_ERR_INVALID_ARGUMENT, "negative count in graph");
+  if ((g->n_nodes > 0 && !g->nodes) || (g->n_outputs > 0 && !g->output_nodes))
+    return fail(RAP_ERR_INVALID_ARGUMENT, "graph arrays are NULL");
+  if (n_params < 0 || (n_params > 0 && !params)) return fail(RAP_ERR_INVALID_ARGUMENT, "params array");
+  const int N = g->n_nodes;
+  for (int i = 0; i < N; ++i) {
+    const rap_node& nd = g->nodes[i];
+    if (nd.param < 0 || nd.param >= n_params)
+      return fail(RAP_ERR_INVALID_ARGUMENT, "node " + std::to_string(i) + ": param index out of range");
+  }
+  for (int i = 0; i < N; ++i) {
+    const rap_node& nd = g->nodes[i];
+    if (nd.op < RAP_OP_FILLNULL || nd.op > RAP_OP_MAPID)
+      return fail(RAP_ERR_INVALID_GRAPH, "node " + std::to_string(i) + ": unknown op");
+    if (nd.op == RAP_OP_NGRAM) {
+      if (nd.n_inputs < 1 || nd.n_inputs > kMaxNgramK)
+        return fail(RAP_ERR_INVALID_PARAM, "node " + std::to_string(i) + ": NGram needs 1..8 inputs");
+    } else if (nd.n_inputs != 1) {
+      return fail(RAP_ERR_INVALID_GRAPH, "node " + std::to_string(i) + ": op takes one input");
+    }
+    if (!nd.inputs) return fail(RAP_ERR_INVALID_ARGUMENT, "node inputs NULL");
+    for (int k = 0; k < nd.n_inputs; ++k)
+      if (!ref_ok(g, nd.inputs[k]))
+        return fail(RAP_ERR_INVALID_GRAPH, "node " + std::to_string(i) + ": input reference out of range");
+  }
+  for (int o = 0; o < g->n_outputs; ++o)
+    if (g->output_nodes[o] < 0 || g->output_nodes[o] >= N)
+      return fail(RAP_ERR_INVALID_GRAPH, "output reference out of range");
+  // cycle check + topological order (iterative DFS)
+  std::vector<int> state(N, 0);
+  v->order.clear();
+  for (int s = 0; s < N; ++s) {
+    if (state[s]) continue;
+    std::vector<std::pair<int, int>> st{{s, 0}};
+    state[s] = 1;
+    while (!st.empty()) {
+      auto& top = st.back();
+      const rap_node& nd = g->nodes[top.first];
+      if (top.second < nd.n_inputs) {
+        int32_t ref = nd.inputs[top.second++];
+        if (ref >= 0) {
+          if (state[ref] == 1) return fail(RAP_ERR_INVALID_GRAPH, "cycle in preprocessing graph");
+          if (state[ref] == 0) {
+            state[ref] = 1;
+            st.push_back({ref, 0});
+          }
+        }
+      } else {
+        state[top.first] = 2;
+        v->order.push_back(top.first);
+        st.pop_back();
+      }
+    }
+  }
+  v->type.assign(N, VT_NONE);
+  for (int i : v->order) {
+    const rap_node& nd = g->nodes[i];
+    int t0 = in_type(g, v->type, nd.inputs[0]);
+    int t = VT_NONE;
+    switch (nd.op) {
+      case RAP_OP_FILLNULL: t = (t0 == VT_DENSE || t0 == VT_IDS) ? t0 : VT_NONE; break;
+      case RAP_OP_LOGIT:
+      case RAP_OP_BOXCOX: t = t0 == VT_DENSE ? VT_DENSE : VT_NONE; break;
+      case RAP_OP_BUCKETIZE: t = (t0 == VT_DENSE || t0 == VT_IDS) ? VT_IDS : VT_NONE; break;
+      case RAP_OP_ONEHOT: t = t0 == VT_IDS ? VT_VEC : VT_NONE; break;
+      case RAP_OP_NGRAM:
+        t = VT_IDS;
+        for (int k = 0; k < nd.n_inputs; ++k)
+          if (in_type(g, v->type, nd.inputs[k]) != VT_IDS) t = VT_NONE;
+        break;
+      default: t = t0 == VT_IDS ? VT_IDS : VT_NONE; break;
+    }
+    if (t == VT_NONE) return fail(RAP_ERR_INVALID_GRAPH, "node " + std::to_string(i) + ": input type mismatch");
+    v->type[i] = t;
+  }
+  for (int i = 0; i < N; ++i) {
+    const rap_node& nd = g->nodes[i];
+    const rap_op_param& pr = params[nd.param];
+    const int t0 = in_type(g, v->type, nd.inputs[0]);
+    const std::string who = "node " + std::to_string(i) + ": ";
+    switch (nd.op) {
+      case RAP_OP_FILLNULL:
+        if (t0 == VT_DENSE && std::isnan(pr.f_fill)) return fail(RAP_ERR_INVALID_PARAM, who + "fill is NaN");
+        break;
+      case RAP_OP_LOGIT:
+        if (!(pr.eps > 0.0f && pr.eps < 0.5f)) return fail(RAP_ERR_INVALID_PARAM, who + "eps not in (0, 0.5)");
+        break;
+      case RAP_OP_BOXCOX:
+        if (!std::isfinite(pr.lambda)) return fail(RAP_ERR_INVALID_PARAM, who + "lambda not finite");
+        break;
+      case RAP_OP_BUCKETIZE:
+        if (pr.n_borders < 1 || pr.n_borders > 65536) return fail(RAP_ERR_INVALID_PARAM, who + "borders count");
+        if (!pr.borders) return fail(RAP_ERR_INVALID_PARAM, who + "borders NULL");
+        if (t0 == VT_DENSE) {
+          const float* b = static_cast<const float*>(pr.borders);
+          for (int k = 0; k < pr.n_borders; ++k) {
+            if (std::isnan(b[k])) return fail(RAP_ERR_INVALID_PARAM, who + "NaN border");
+            if (k > 0 && b[k] < b[k - 1]) return fail(RAP_ERR_INVALID_PARAM, who + "borders not sorted");
+          }
+        } else {
+          const int64_t* b = static_cast<const int64_t*>(pr.borders);
+          for (int k = 1; k < pr.n_borders; ++k)
+            if (b[k] < b[k - 1]) return fail(RAP_ERR_INVALID_PARAM, who + "borders not sorted");
+        }
+        break;
+      case RAP_OP_ONEHOT:
+        if (pr.k_width < 1 || pr.k_width > 4096) return fail(RAP_ERR_INVALID_PARAM, who + "K not in [1, 4096]");
+        break;
+      case RAP_OP_SIGRIDHASH:
+        if (pr.max_value < 1) return fail(RAP_ERR_INVALID_PARAM, who + "max_value < 1");
+        break;
+      case RAP_OP_FIRSTX:
+        if (pr.x < 0) return fail(RAP_ERR_INVALID_PARAM, who + "x < 0");
+        break;
+      case RAP_OP_CLAMP:
+        if (pr.lo > pr.hi) return fail(RAP_ERR_INVALID_PARAM, who + "lo > hi");
+        break;
+      case RAP_OP_NGRAM:
+        if (pr.n < 1 || pr.n > 8 || pr.max_value < 1) return fail(RAP_ERR_INVALID_PARAM, who + "n or max_value");
+        break;
+      case RAP_OP_MAPID: {
+        if (pr.map_size < 0) return fail(RAP_ERR_INVALID_PARAM, who + "map_size < 0");
+        if (pr.map_size > 0 && (!pr.map_keys || !pr.map_vals)) return fail(RAP_ERR_INVALID_PARAM, who + "map NULL");
+        if (pr.map_size > (int64_t)INT32_MAX) return fail(RAP_ERR_INVALID_PARAM, who + "map too large");
+        std::vector<int64_t> k(pr.map_keys, pr.map_keys + pr.map_size);
+        std::sort(k.begin(), k.end());
+        if (std::adjacent_find(k.begin(), k.end()) != k.end())
+          return fail(RAP_ERR_INVALID_PARAM, who + "duplicate MapId key");
+        break;
+      }
+    }
+  }
+  v->d_out = v->f_out = 0;
+  for (int o = 0; o < g->n_outputs; ++o) {
+    int t = v->type[g->output_nodes[o]];
+    if (t == VT_DENSE) v->d_out += 1;
+    else if (t == VT_VEC) v->d_out += params[g->nodes[g->output_nodes[o]].param].k_width;
+    else v->f_out += 1;
+  }
+  return RAP_OK;
+}
+
+// ----------------------------------------------------------------------------
+// Lowering.
+struct Lowerer {
+  const rap_graph* g;
+  const rap_op_param* params;
+  rap_plan* P;
+  std::vector<int> dense_memo, chain_memo;
+
+  int lower_dense(int32_t ref) {
+    if (ref >= 0 && dense_memo[ref] >= 0) return dense_memo[ref];
+    std::vector<int> path;  // node ids, output -> source
+    int32_t cur = ref;
+    while (cur >= 0) {
+      path.push_back(cur);
+      cur = g->nodes[cur].inputs[0];
+    }
+    const int col = (-cur - 1) / 2;
+    DenseExpr de{};
+    de.col = col;
+    de.op_begin = (int)P->ops.size();
+    for (auto it = path.rbegin(); it != path.rend(); ++it) {
+      const rap_node& nd = g->nodes[*it];
+      const rap_op_param& pr = params[nd.param];
+      DevOp op{};
+      if (nd.op == RAP_OP_FILLNULL) {
+        op.kind = OK_FILL_F;
+        op.f0 = pr.f_fill;
+      } else if (nd.op == RAP_OP_LOGIT) {
+        op.kind = OK_LOGIT;
+        volatile float eps = pr.eps;
+        op.f0 = eps;
+        op.f1 = 1.0f - eps;  // f32 arithmetic (R11)
+      } else {
+        op.kind = OK_BOXCOX;
+        op.f0 = pr.lambda;
+      }
+      P->ops.push_back(op);
+    }
+    de.op_end = (int)P->ops.size();
+    P->dexprs.push_back(de);
+    const int idx = (int)P->dexprs.size() - 1;
+    if (ref >= 0) dense_memo[ref] = idx;
+    return idx;
+  }
+
+  // returns chain index, or -1 with *st set
+  int lower_ids(int32_t ref, bool allow_ngram, rap_status* st) {
+    if (ref >= 0 && chain_memo[ref] >= 0) {
+      const Chain& c = P->chains[chain_memo[ref]];
+      if (c.src_kind == SRC_NGRAM && !allow_ngram) {
+        *st = fail(RAP_ERR_UNSUPPORTED, "NGram over an NGram output is not supported");
+        return -1;
+      }
+      return chain_memo[ref];
+    }
+    // walk back through single-input id ops
+    std::vector<int> path;
+    int32_t cur = ref;
+    Chain ch{};
+    ch.xcap = kNoCap;
+    ch.null_xcap = kNoCap;
+    while (true) {
+      if (cur < 0) {  // raw sparse column
+        ch.src_kind = SRC_SPARSE;
+        ch.src = (-cur - 2) / 2;
+        break;
+      }
+      const rap_node& nd = g->nodes[cur];
+      if (nd.op == RAP_OP_NGRAM) {
+        ch.src_kind = SRC_NGRAM;
+        break;
+      }
+      if (nd.op == RAP_OP_BUCKETIZE && in_is_dense(nd.inputs[0])) {
+        ch.src_kind = SRC_DENSE_BUCKET;
+        break;
+      }
+      path.push_back(cur);
+      cur = nd.inputs[0];
+    }
+    if (ch.src_kind == SRC_NGRAM) {
+      if (!allow_ngram) {
+        *st = fail(RAP_ERR_UNSUPPORTED, "NGram over an NGram output is not supported");
+        return -1;
+      }
+      const rap_node& nd = g->nodes[cur];
+      const rap_op_param& pr = params[nd.param];
+      NGramDesc ng{};
+      ng.n = pr.n;
+      ng.k = nd.n_inputs;
+      ng.hsalt = splitmix_H(pr.salt);
+      ng.M = pr.max_value;
+      for (int k = 0; k < nd.n_inputs; ++k) {
+        int c = lower_ids(nd.inputs[k], false, st);
+        if (c < 0) return -1;
+        ng.chain[k] = c;
+      }
+      P->ngrams.push_back(ng);
+      ch.src = (int)P->ngrams.size() - 1;
+    } else if (ch.src_kind == SRC_DENSE_BUCKET) {
+      const rap_node& nd = g->nodes[cur];
+      const rap_op_param& pr = params[nd.param];
+      ch.src = lower_dense(nd.inputs[0]);
+      ch.btab = (int)P->ftab.size();
+      ch.bm = pr.n_borders;
+      const float* b = static_cast<const float*>(pr.borders);
+      P->ftab.insert(P->ftab.end(), b, b + pr.n_borders);
+    }
+    ch.op_begin = (int)P->ops.size();
+    bool fill_seen = false;
+    int null_begin = 0;
+    for (auto it = path.rbegin(); it != path.rend(); ++it) {
+      const rap_node& nd = g->nodes[*it];
+      const rap_op_param& pr = params[nd.param];
+      DevOp op{};
+      switch (nd.op) {
+        case RAP_OP_FILLNULL:
+          if (!fill_seen && ch.src_kind == SRC_SPARSE) {
+            fill_seen = true;
+            ch.fill = pr.i_fill;
+            null_begin = (int)P->ops.size();
+          }
+          continue;
+        case RAP_OP_FIRSTX:
+          ch.xcap = std::min(ch.xcap, pr.x);
+          if (fill_seen) ch.null_xcap = std::min(ch.null_xcap, pr.x);
+          continue;
+        case RAP_OP_CLAMP:
+          op.kind = OK_CLAMP;
+          op.a = pr.lo;
+          op.b = pr.hi;
+          break;
+        case RAP_OP_SIGRIDHASH:
+          op.kind = OK_SIGRID;
+          op.hsalt = splitmix_H(pr.salt);
+          op.M = pr.max_value;
+          break;
+        case RAP_OP_BUCKETIZE: {
+          op.kind = OK_BUCKET_I;
+          op.a = (int64_t)P->itab.size();
+          op.m = pr.n_borders;
+          const int64_t* b = static_cast<const int64_t*>(pr.borders);
+          P->itab.insert(P->itab.end(), b, b + pr.n_borders);
+          break;
+        }
+        case RAP_OP_MAPID: {
+          op.kind = OK_MAPID;
+          op.a = (int64_t)P->itab.size();
+          op.m = (int32_t)pr.map_size;
+          op.b = pr.map_default;
+          std::vector<std::pair<int64_t, int64_t>> kv;
+          for (int64_t k = 0; k < pr.map_size; ++k) kv.push_back({pr.map_keys[k], pr.map_vals[k]});
+          std::sort(kv.begin(), kv.end());
+          for (auto& e : kv) P->itab.push_back(e.first);
+          for (auto& e : kv) P->itab.push_back(e.second);
+          break;
+        }
+        default:
+          *st = fail(RAP_ERR_UNSUPPORTED, "unexpected op in id chain");
+          return -1;
+      }
+      P->ops.push_back(op);
+    }
+    ch.op_end = (int)P->ops.size();
+    ch.has_fill = fill_seen ? 1 : 0;
+    ch.null_op_begin = fill_seen ? null_begin : ch.op_end;
+    P->chains.push_back(ch);
+    const int idx = (int)P->chains.size() - 1;
+    if (ref >= 0) chain_memo[ref] = idx;
+    return idx;
+  }
+
+  bool in_is_dense(int32_t ref) {
+    if (ref < 0) return (-ref) % 2 == 1;
+    return type_of[ref] == VT_DENSE;
+  }
+  std::vector<int> type_of;
+};
+
+template <class T>
+size_t push_blob(std::vector<unsigned char>& blob, const std::vector<T>& v) {
+  size_t off = (blob.size() + 15) / 16 * 16;
+  blob.resize(off + v.size() * sizeof(T));
+  if (!v.empty()) memcpy(blob.data() + off, v.data(), v.size() * sizeof(T));
+  return off;
+}
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    cudaGetDevice(&prev);
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+int64_t chain_bound(const rap_plan* P, const Chain& ch, int64_t B, const int64_t* nnz) {
+  int64_t b;
+  if (ch.src_kind == SRC_SPARSE) {
+    b = sat_add(nnz ? std::max<int64_t>(nnz[ch.src], 0) : 0, ch.has_fill ? B : 0);
+  } else if (ch.src_kind == SRC_DENSE_BUCKET) {
+    b = B;
+  } else {
+    const NGramDesc& ng = P->ngrams[ch.src];
+    b = 0;
+    for (int k = 0; k < ng.k; ++k) b = sat_add(b, chain_bound(P, P->chains[ng.chain[k]], B, nnz));
+  }
+  return std::min(b, sat_mul(ch.xcap, B));
+}
+
+int64_t values_bound(const rap_plan* P, int64_t B, const int64_t* nnz) {
+  int64_t tot = 0;
+  for (const SparseOut& so : P->souts) tot = sat_add(tot, chain_bound(P, P->chains[so.chain], B, nnz));
+  return tot;
+}
+
+rap_status set_grid_budget(rap_plan* P, int32_t budget) {
+  if (budget < 0 || budget > P->sm_count) return fail(RAP_ERR_INVALID_ARGUMENT, "sm_budget not in [0, #SMs]");
+  P->budget = budget == 0 ? P->sm_count : budget;
+  return RAP_OK;
+}
+
+// Bytes one call moves (each raw byte read once, each output byte written once).
+double algorithmic_bytes(const rap_plan* P, int64_t B, const int64_t* nnz) {
+  double b = 0;
+  for (int c : P->used_dense) b += 4.0 * B + B / 8.0;
+  for (int s : P->used_sparse) b += 4.0 * (B + 1) + 8.0 * (nnz ? nnz[s] : 0) + B / 8.0;
+  b += 4.0 * B * P->d_out + 12.0 * B * P->souts.size() + 8.0 + 8.0 * values_bound(P, B, nnz);
+  return b;
+}
+
+}  // namespace
+
+// ============================================================================
+extern "C" {
+
+const char* rap_status_string(rap_status s) {
+  switch (s) {
+    case RAP_OK: return "RAP_OK";
+    case RAP_ERR_INVALID_ARGUMENT: return "RAP_ERR_INVALID_ARGUMENT";
+    case RAP_ERR_INVALID_GRAPH: return "RAP_ERR_INVALID_GRAPH";
+    case RAP_ERR_INVALID_PARAM: return "RAP_ERR_INVALID_PARAM";
+    case RAP_ERR_CAPACITY: return "RAP_ERR_CAPACITY";
+    case RAP_ERR_UNSUPPORTED: return "RAP_ERR_UNSUPPORTED";
+    case RAP_ERR_CUDA: return "RAP_ERR_CUDA";
+    case RAP_ERR_OUT_OF_MEMORY: return "RAP_ERR_OUT_OF_MEMORY";
+  }
+  return "RAP_ERR_UNKNOWN";
+}
+
+const char* rap_last_error(void) { return g_last_error.c_str(); }
+
+rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, int32_t n_params, int32_t device,
+                           int32_t sm_budget, rap_plan** out) {
+  if (!out) return fail(RAP_ERR_INVALID_ARGUMENT, "out is NULL");
+  *out = nullptr;
+  Validated v;
+  rap_status st = validate(graph, params, n_params, &v);
+  if (st != RAP_OK) return st;
+  if (graph->n_dense_in > 128 || graph->n_sparse_in > 1024)
+    return fail(RAP_ERR_UNSUPPORTED, "more than 128 dense or 1024 sparse raw columns");
+
+  int n_dev = 0;
+  cudaError_t e = cudaGetDeviceCount(&n_dev);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaGetDeviceCount");
+  if (device < 0 || device >= n_dev) return fail(RAP_ERR_INVALID_ARGUMENT, "bad device ordinal");
+  DeviceGuard dg(device);
+
+  rap_plan* P = new rap_plan();
+  P->device = device;
+  P->n_dense_in = graph->n_dense_in;
+  P->n_sparse_in = graph->n_sparse_in;
+  e = cudaDeviceGetAttribute(&P->sm_count, cudaDevAttrMultiProcessorCount, device);
+  if (e != cudaSuccess) {
+    delete P;
+    return cuda_fail(e, "cudaDeviceGetAttribute");
+  }
+  st = set_grid_budget(P, sm_budget);
+  if (st != RAP_OK) {
+    delete P;
+    return st;
+  }
+
+  // ---- lower outputs
+  Lowerer L{graph, params, P};
+  L.dense_memo.assign(graph->n_nodes, -1);
+  L.chain_memo.assign(graph->n_nodes, -1);
+  L.type_of = v.type;
+  int col = 0;
+  std::vector<Unit> flat_units;
+  for (int o = 0; o < graph->n_outputs; ++o) {
+    const int node = graph->output_nodes[o];
+    const int t = v.type[node];
+    if (t == VT_DENSE) {
+      Unit u{};
+      u.kind = U_DENSE;
+      u.idx = L.lower_dense(node);
+      u.col = col;
+      u.width = 1;
+      flat_units.push_back(u);
+      col += 1;
+    } else if (t == VT_VEC) {
+      const rap_node& nd = graph->nodes[node];
+      int c = L.lower_ids(nd.inputs[0], true, &st);
+      if (c < 0) {
+        delete P;
+        return st;
+      }
+      Unit u{};
+      u.kind = U_ONEHOT;
+      u.idx = c;
+      u.col = col;
+      u.width = params[nd.param].k_width;
+      u.k0 = 0;
+      flat_units.push_back(u);
+      col += u.width;
+    } else {
+      int c = L.lower_ids(node, true, &st);
+      if (c < 0) {
+        delete P;
+        return st;
+      }
+      SparseOut so{};
+      so.chain = c;
+      so.rows_per_desc = kRowsSparse;
+      P->souts.push_back(so);
+    }
+  }
+  P->d_out = col;
+  // ---- column groups of <= kGroupCols columns (OneHot units may be split)
+  {
+    int gcol0 = 0;
+    Group cur{};
+    cur.unit_begin = 0;
+    cur.col0 = 0;
+    for (const Unit& u0 : flat_units) {
+      Unit u = u0;
+      int remaining = u.width;
+      int64_t k0 = u.k0;
+      int c = u.col;
+      while (remaining > 0) {
+        int room = kGroupCols - (c - gcol0);
+        if (room == 0) {
+          cur.unit_end = (int)P->units.size();
+          cur.width = c - gcol0;
+          P->groups.push_back(cur);
+          gcol0 = c;
+          cur = Group{};
+          cur.unit_begin = (int)P->units.size();
+          cur.col0 = gcol0;
+          room = kGroupCols;
+        }
+        int w = std::min(room, remaining);
+        Unit piece = u;
+        piece.col = c;
+        piece.width = w;
+        piece.k0 = k0;
+        P->units.push_back(piece);
+        c += w;
+        k0 += w;
+        remaining -= w;
+      }
+    }
+    if (col > gcol0) {
+      cur.unit_end = (int)P->units.size();
+      cur.width = col - gcol0;
+      P->groups.push_back(cur);
+    }
+  }
+  int max_w = 1;
+  for (const Group& gr : P->groups) max_w = std::max(max_w, gr.width);
+  P->tile_ld = max_w | 1;
+  // used raw columns (for the byte model)
+  {
+    std::vector<char> ud(graph->n_dense_in, 0), us(graph->n_sparse_in, 0);
+    for (int i = 0; i < graph->n_nodes; ++i)
+      for (int k = 0; k < graph->nodes[i].n_inputs; ++k) {
+        int32_t r = graph->nodes[i].inputs[k];
+        if (r < 0 && (-r) % 2 == 1) ud[(-r - 1) / 2] = 1;
+        if (r < 0 && (-r) % 2 == 0) us[(-r - 2) / 2] = 1;
+      }
+    for (int c = 0; c < graph->n_dense_in; ++c)
+      if (ud[c]) P->used_dense.push_back(c);
+    for (int c = 0; c < graph->n_sparse_in; ++c)
+      if (us[c]) P->used_sparse.push_back(c);
+  }
+
+  // ---- device blob
+  std::vector<unsigned char> blob;
+  P->off_ops = push_blob(blob, P->ops);
+  P->off_dexprs = push_blob(blob, P->dexprs);
+  P->off_chains = push_blob(blob, P->chains);
+  P->off_ngrams = push_blob(blob, P->ngrams);
+  P->off_units = push_blob(blob, P->units);
+  P->off_groups = push_blob(blob, P->groups);
+  P->off_souts = push_blob(blob, P->souts);
+  P->off_ftab = push_blob(blob, P->ftab);
+  P->off_itab = push_blob(blob, P->itab);
+  if (blob.empty()) blob.resize(16);
+  e = cudaMalloc(&P->blob, blob.size());
+  if (e == cudaSuccess) e = cudaMemcpy(P->blob, blob.data(), blob.size(), cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMalloc(&P->d_sched, 3 * sizeof(unsigned long long));
+  if (e == cudaSuccess) {
+    const unsigned long long init[3] = {0ull, 0ull, 1ull};
+    e = cudaMemcpy(P->d_sched, init, sizeof(init), cudaMemcpyHostToDevice);
+  }
+  if (e == cudaSuccess) e = cudaMalloc(&P->d_err, sizeof(int32_t));
+  if (e == cudaSuccess) e = cudaMemset(P->d_err, 0, sizeof(int32_t));
+  if (e == cudaSuccess) e = cudaMalloc(&P->d_desc_start, sizeof(int32_t) * (P->souts.size() + 1));
+  if (e != cudaSuccess) {
+    rap_plan_destroy(P);
+    return cuda_fail(e, "plan device allocation");
+  }
+
+  // ---- shared memory and occupancy
+  const int sparse_smem = kRowsSparse * (4 + 8 + 4) + 16;
+  const int dense_smem = kRowsDense * P->tile_ld * 4;
+  P->smem = std::max(sparse_smem, dense_smem);
+  int occ = 0;
+  e = (cudaError_t)fused_occupancy(P->smem, P->n_dense_in, P->n_sparse_in, &occ);
+  if (e != cudaSuccess) {
+    rap_plan_destroy(P);
+    return cuda_fail(e, "occupancy query");
+  }
+  P->ctas_per_sm = std::max(1, occ);
+  *out = P;
+  return RAP_OK;
+}
+
+void rap_plan_destroy(rap_plan* P) {
+  if (!P) return;
+  DeviceGuard dg(P->device);
+  cudaFree(P->blob);
+  cudaFree(P->d_sched);
+  cudaFree(P->d_err);
+  cudaFree(P->d_desc_start);
+  cudaFree(P->d_status);
+  for (void* s : P->stage) cudaFree(s);
+  delete P;
+}
+
+rap_status rap_set_budget(rap_plan* P, int32_t sm_budget) {
+  if (!P) return fail(RAP_ERR_INVALID_ARGUMENT, "plan is NULL");
+  return set_grid_budget(P, sm_budget);
+}
+
+rap_status rap_plan_output_shape(const rap_plan* P, int64_t n_rows, const int64_t* sp_nnz, int64_t* d_out_cols,
+                                 int64_t* n_sparse_out, int64_t* values_upper_bound) {
+  if (!P) return fail(RAP_ERR_INVALID_ARGUMENT, "plan is NULL");
+  if (n_rows < 0) return fail(RAP_ERR_INVALID_ARGUMENT, "n_rows < 0");
+  if (!sp_nnz && n_rows > 0 && P->n_sparse_in > 0) return fail(RAP_ERR_INVALID_ARGUMENT, "sp_nnz is NULL");
+  if (d_out_cols) *d_out_cols = P->d_out;
+  if (n_sparse_out) *n_sparse_out = (int64_t)P->souts.size();
+  if (values_upper_bound) *values_upper_bound = n_rows > 0 ? values_bound(P, n_rows, sp_nnz) : 0;
+  return RAP_OK;
+}
+
+rap_status rap_plan_info_get(const rap_plan* P, rap_plan_info* info) {
+  if (!P || !info) return fail(RAP_ERR_INVALID_ARGUMENT, "NULL argument");
+  memset(info, 0, sizeof(*info));
+  info->device = P->device;
+  info->sm_count = P->sm_count;
+  info->sm_budget = P->budget;
+  info->ctas_per_sm = P->ctas_per_sm;
+  info->threads_per_cta = kThreads;
+  info->grid = P->budget * P->ctas_per_sm;
+  info->n_dense_out_cols = P->d_out;
+  info->n_sparse_out = (int32_t)P->souts.size();
+  info->n_dense_groups = (int32_t)P->groups.size();
+  info->rows_per_dense_desc = kRowsDense;
+  info->max_rows_per_sparse_desc = kRowsSparse;
+  info->min_rows_per_sparse_desc = kRowsSparse;
+  info->n_descriptors_last = P->last_n_desc;
+  info->n_launches = P->n_launches;
+  info->smem_bytes = P->smem;
+  return RAP_OK;
+}
+
+static rap_status check_batch(const rap_plan* P, const rap_raw_batch* raw, const rap_output* out) {
+  if (!P || !raw || !out) return fail(RAP_ERR_INVALID_ARGUMENT, "NULL argument");
+  if (raw->n_rows < 0) return fail(RAP_ERR_INVALID_ARGUMENT, "n_rows < 0");
+  if (raw->n_rows > (int64_t)INT32_MAX - kRowsSparse) return fail(RAP_ERR_INVALID_ARGUMENT, "n_rows too large");
+  const int64_t B = raw->n_rows;
+  if (B == 0) {
+    if (!P->souts.empty() && !out->offsets) return fail(RAP_ERR_INVALID_ARGUMENT, "offsets NULL");
+    return RAP_OK;
+  }
+  for (int c : P->used_dense)
+    if (!raw->dense || !raw->dense[c]) return fail(RAP_ERR_INVALID_ARGUMENT, "dense column pointer NULL");
+  for (int s : P->used_sparse)
+    if (!raw->sp_offsets || !raw->sp_values || !raw->sp_offsets[s])
+      return fail(RAP_ERR_INVALID_ARGUMENT, "sparse column pointer NULL");
+  if (P->d_out > 0 && (!out->dense_out || out->dense_ld < P->d_out))
+    return fail(RAP_ERR_INVALID_ARGUMENT, "dense_out NULL or dense_ld < d_out");
+  if (!P->souts.empty()) {
+    if (!out->lengths || !out->offsets) return fail(RAP_ERR_INVALID_ARGUMENT, "lengths/offsets NULL");
+    if (P->n_sparse_in > 0 && !raw->sp_nnz) return fail(RAP_ERR_INVALID_ARGUMENT, "sp_nnz NULL");
+    const int64_t bound = values_bound(P, B, raw->sp_nnz);
+    if (bound > 0 && !out->values) return fail(RAP_ERR_INVALID_ARGUMENT, "values NULL");
+    if (out->values_capacity < bound)
+      return fail(RAP_ERR_CAPACITY, "values_capacity " + std::to_string(out->values_capacity) + " < bound " +
+                                        std::to_string(bound));
+  }
+  return RAP_OK;
+}
+
+static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output* out, cudaStream_t stream) {
+  const int64_t B = raw->n_rows;
+  cudaError_t e;
+  if (B == 0) {
+    if (!P->souts.empty()) {
+      e = cudaMemsetAsync(out->offsets, 0, sizeof(int64_t), stream);
+      if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync");
+    }
+    return RAP_OK;
+  }
+  // per-n_rows descriptor table (feature-major sparse descriptors)
+  if (P->desc_rows != B) {
+    P->h_desc_start.assign(P->souts.size() + 1, 0);
+    int64_t acc = 0;
+    for (size_t f = 0; f < P->souts.size(); ++f) {
+      P->h_desc_start[f] = (int32_t)acc;
+      acc += (B + P->souts[f].rows_per_desc - 1) / P->souts[f].rows_per_desc;
+    }
+    P->h_desc_start[P->souts.size()] = (int32_t)acc;
+    P->n_sparse_desc = acc;
+    e = cudaMemcpyAsync(P->d_desc_start, P->h_desc_start.data(), sizeof(int32_t) * P->h_desc_start.size(),
+                        cudaMemcpyHostToDevice, stream);
+    if (e != cudaSuccess) return cuda_fail(e, "descriptor table upload");
+    P->desc_rows = B;
+  }
+  P->n_dense_desc = P->groups.empty() ? 0 : (int64_t)P->groups.size() * ((B + kRowsDense - 1) / kRowsDense);
+  const int64_t n_total = P->n_sparse_desc + P->n_dense_desc;
+  if (n_total == 0) return RAP_OK;
+  // scan state (grows, never shrinks)
+  if (P->n_sparse_desc > P->status_cap) {
+    if (P->d_status) {
+      e = cudaStreamSynchronize(stream);
+      if (e != cudaSuccess) return cuda_fail(e, "cudaStreamSynchronize");
+      cudaFree(P->d_status);
+      P->d_status = nullptr;
+    }
+    const int64_t cap = std::max<int64_t>(P->n_sparse_desc, 1024);
+    e = cudaMalloc(&P->d_status, sizeof(unsigned long long) * cap);
+    if (e != cudaSuccess) return fail(RAP_ERR_OUT_OF_MEMORY, "scan-state allocation");
+    e = cudaMemsetAsync(P->d_status, 0, sizeof(unsigned long long) * cap, stream);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync");
+    P->status_cap = cap;
+  }
+  const int64_t grid = std::min<int64_t>(n_total, (int64_t)P->budget * P->ctas_per_sm);
+  Common c{};
+  c.ops = reinterpret_cast<const DevOp*>(P->blob + P->off_ops);
+  c.dexprs = reinterpret_cast<const DenseExpr*>(P->blob + P->off_dexprs);
+  c.chains = reinterpret_cast<const Chain*>(P->blob + P->off_chains);
+  c.ngrams = reinterpret_cast<const NGramDesc*>(P->blob + P->off_ngrams);
+  c.units = reinterpret_cast<const Unit*>(P->blob + P->off_units);
+  c.groups = reinterpret_cast<const Group*>(P->blob + P->off_groups);
+  c.souts = reinterpret_cast<const SparseOut*>(P->blob + P->off_souts);
+  c.ftab = reinterpret_cast<const float*>(P->blob + P->off_ftab);
+  c.itab = reinterpret_cast<const int64_t*>(P->blob + P->off_itab);
+  c.desc_start = P->d_desc_start;
+  c.n_sparse_out = (int32_t)P->souts.size();
+  c.n_groups = (int32_t)P->groups.size();
+  c.rows_dense = kRowsDense;
+  c.tile_ld = P->tile_ld;
+  c.n_rows = B;
+  c.n_sparse_desc = P->n_sparse_desc;
+  c.n_total_desc = n_total;
+  c.sched = P->d_sched;
+  c.status = P->d_status;
+  c.status_cap = P->status_cap;
+  c.dense_out = out->dense_out;
+  c.ld = out->dense_ld;
+  c.lengths = out->lengths;
+  c.offsets = out->offsets;
+  c.values = out->values;
+  c.values_cap = out->values_capacity;
+  c.err = P->d_err;
+  LaunchRaw lr{};
+  lr.n_dense = P->n_dense_in;
+  lr.n_sparse = P->n_sparse_in;
+  lr.dense = raw->dense;
+  lr.dvalid = raw->dense_valid;
+  lr.off = raw->sp_offsets;
+  lr.val = raw->sp_values;
+  lr.svalid = raw->sp_valid;
+  int rc = launch_fused(c, lr, (int)grid, P->smem, stream);
+  if (rc != 0) return cuda_fail((cudaError_t)rc, "fused kernel launch");
+  P->n_launches += 1;
+  P->last_n_desc = n_total;
+  return RAP_OK;
+}
+
+rap_status rap_preprocess(rap_plan* P, const rap_raw_batch* raw, const rap_output* out, void* stream) {
+  rap_status st = check_batch(P, raw, out);
+  if (st != RAP_OK) return st;
+  DeviceGuard dg(P->device);
+  return launch(P, raw, out, reinterpret_cast<cudaStream_t>(stream));
+}
+
+static rap_status stage_buf(rap_plan* P, size_t slot, size_t bytes, void** ptr) {
+  if (P->stage.size() <= slot) {
+    P->stage.resize(slot + 1, nullptr);
+    P->stage_cap.resize(slot + 1, 0);
+  }
+  if (P->stage_cap[slot] < bytes) {
+    cudaFree(P->stage[slot]);
+    P->stage[slot] = nullptr;
+    size_t cap = std::max<size_t>(bytes + bytes / 4, 256);
+    cudaError_t e = cudaMalloc(&P->stage[slot], cap);
+    if (e != cudaSuccess) {
+      P->stage_cap[slot] = 0;
+      return fail(RAP_ERR_OUT_OF_MEMORY, "staging allocation");
+    }
+    P->stage_cap[slot] = cap;
+  }
+  *ptr = P->stage[slot];
+  return RAP_OK;
+}
+
+rap_status rap_preprocess_host(rap_plan* P, const rap_raw_batch* raw, const rap_output* out, void* stream_v) {
+  rap_status st = check_batch(P, raw, out);
+  if (st != RAP_OK) return st;
+  DeviceGuard dg(P->device);
+  cudaStream_t stream = reinterpret_cast<cudaStream_t>(stream_v);
+  const int64_t B = raw->n_rows;
+  const size_t bm_bytes = (size_t)((B + 31) / 32) * 4;
+  std::vector<const float*> d_dense(P->n_dense_in, nullptr);
+  std::vector<const uint32_t*> d_dvalid(P->n_dense_in, nullptr);
+  std::vector<const int32_t*> d_off(P->n_sparse_in, nullptr);
+  std::vector<const int64_t*> d_val(P->n_sparse_in, nullptr);
+  std::vector<const uint32_t*> d_svalid(P->n_sparse_in, nullptr);
+  size_t slot = 0;
+  cudaError_t e = cudaSuccess;
+  auto h2d = [&](const void* src, size_t bytes, void** dst) -> rap_status {
+    rap_status s = stage_buf(P, slot++, bytes, dst);
+    if (s != RAP_OK) return s;
+    if (bytes) e = cudaMemcpyAsync(*dst, src, bytes, cudaMemcpyHostToDevice, stream);
+    return e == cudaSuccess ? RAP_OK : cuda_fail(e, "H2D copy");
+  };
+  if (B > 0) {
+    for (int c : P->used_dense) {
+      void* d;
+      if ((st = h2d(raw->dense[c], sizeof(float) * B, &d)) != RAP_OK) return st;
+      d_dense[c] = static_cast<const float*>(d);
+      if (raw->dense_valid && raw->dense_valid[c]) {
+        if ((st = h2d(raw->dense_valid[c], bm_bytes, &d)) != RAP_OK) return st;
+        d_dvalid[c] = static_cast<const uint32_t*>(d);
+      }
+    }
+    for (int s : P->used_sparse) {
+      void* d;
+      const int32_t* ho = raw->sp_offsets[s];
+      if ((st = h2d(ho, sizeof(int32_t) * (B + 1), &d)) != RAP_OK) return st;
+      d_off[s] = static_cast<const int32_t*>(d);
+      const int64_t lo = ho[0], n = ho[B] - ho[0];
+      if ((st = h2d(raw->sp_values[s] + lo, sizeof(int64_t) * std::max<int64_t>(n, 0), &d)) != RAP_OK) return st;
+      d_val[s] = static_cast<const int64_t*>(d) - lo;  // absolute offsets index this base
+      if (raw->sp_valid && raw->sp_valid[s]) {
+        if ((st = h2d(raw->sp_valid[s], bm_bytes, &d)) != RAP_OK) return st;
+        d_svalid[s] = static_cast<const uint32_t*>(d);
+      }
+    }
+  }
+  const int64_t F = (int64_t)P->souts.size();
+  const int64_t vb = B > 0 ? values_bound(P, B, raw->sp_nnz) : 0;
+  void *dd = nullptr, *dl = nullptr, *dof = nullptr, *dv = nullptr;
+  if ((st = stage_buf(P, slot++, sizeof(float) * std::max<int64_t>(B * P->d_out, 1), &dd)) != RAP_OK) return st;
+  if ((st = stage_buf(P, slot++, sizeof(int32_t) * std::max<int64_t>(B * F, 1), &dl)) != RAP_OK) return st;
+  if ((st = stage_buf(P, slot++, sizeof(int64_t) * (B * F + 1), &dof)) != RAP_OK) return st;
+  if ((st = stage_buf(P, slot++, sizeof(int64_t) * std::max<int64_t>(vb, 1), &dv)) != RAP_OK) return st;
+  rap_raw_batch dr = *raw;
+  dr.dense = d_dense.data();
+  dr.dense_valid = d_dvalid.data();
+  dr.sp_offsets = d_off.data();
+  dr.sp_values = d_val.data();
+  dr.sp_valid = d_svalid.data();
+  rap_output dout{};
+  dout.dense_out = static_cast<float*>(dd);
+  dout.dense_ld = P->d_out;
+  dout.lengths = static_cast<int32_t*>(dl);
+  dout.offsets = static_cast<int64_t*>(dof);
+  dout.values = static_cast<int64_t*>(dv);
+  dout.values_capacity = std::max<int64_t>(vb, 0);
+  if ((st = launch(P, &dr, &dout, stream)) != RAP_OK) return st;
+  // D2H
+  if (B > 0 && P->d_out > 0) {
+    if (out->dense_ld == P->d_out)
+      e = cudaMemcpyAsync(out->dense_out, dd, sizeof(float) * B * P->d_out, cudaMemcpyDeviceToHost, stream);
+    else
+      e = cudaMemcpy2DAsync(out->dense_out, sizeof(float) * out->dense_ld, dd, sizeof(float) * P->d_out,
+                            sizeof(float) * P->d_out, B, cudaMemcpyDeviceToHost, stream);
+    if (e != cudaSuccess) return cuda_fail(e, "D2H dense");
+  }
+  if (F > 0) {
+    if (B > 0) e = cudaMemcpyAsync(out->lengths, dl, sizeof(int32_t) * B * F, cudaMemcpyDeviceToHost, stream);
+    if (e == cudaSuccess)
+      e = cudaMemcpyAsync(out->offsets, dof, sizeof(int64_t) * (B * F + 1), cudaMemcpyDeviceToHost, stream);
+    if (e == cudaSuccess && vb > 0)
+      e = cudaMemcpyAsync(out->values, dv, sizeof(int64_t) * vb, cudaMemcpyDeviceToHost, stream);
+    if (e != cudaSuccess) return cuda_fail(e, "D2H sparse");
+  }
+  e = cudaStreamSynchronize(stream);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaStreamSynchronize");
+  return RAP_OK;
+}
+
+rap_status rap_predict_latency_us(const rap_plan* P, int64_t n_rows, const int64_t* sp_nnz, int32_t sm_budget,
+                                  double* latency_us) {
+  if (!P || !latency_us) return fail(RAP_ERR_INVALID_ARGUMENT, "NULL argument");
+  if (n_rows < 0 || sm_budget < 0 || sm_budget > P->sm_count) return fail(RAP_ERR_INVALID_ARGUMENT, "bad size");
+  const int b = sm_budget == 0 ? P->sm_count : sm_budget;
+  const double bytes = n_rows > 0 ? algorithmic_bytes(P, n_rows, sp_nnz) : 0.0;
+  // Analytic roofline predictor: the fused kernel streams at
+  // HBM bandwidth once ~sat SMs issue loads; fewer SMs get a linear share.
+  const char* env = getenv("RAP_HBM_GBS");
+  const double peak_gbs = env ? atof(env) : 6500.0;
+  const double sat = 0.5 * P->sm_count;
+  const double bw = peak_gbs * 1e9 * std::min(1.0, b / sat);
+  const double launch_us = 5.0;
+  *latency_us = launch_us + bytes / bw * 1e6;
+  return RAP_OK;
+}
+
+rap_status rap_choose_budget(const rap_plan* P, int64_t n_rows, const int64_t* sp_nnz, double oc_us,
+                             int32_t* sm_budget, double* t_delta_us) {
+  if (!P || !sm_budget) return fail(RAP_ERR_INVALID_ARGUMENT, "NULL argument");
+  // T_delta = sum_i P_i - OC (L1138-1143); pick the smallest budget with
+  // T_delta <= 0 so the most SMs stay with training (L1145-1152).
+  double best_td = 1e300;
+  int best_b = P->sm_count;
+  for (int b = 1; b <= P->sm_count; ++b) {
+    double p_us = 0;
+    rap_status st = rap_predict_latency_us(P, n_rows, sp_nnz, b, &p_us);
+    if (st != RAP_OK) return st;
+    const double td = p_us - oc_us;
+    if (td <= 0) {
+      *sm_budget = b;
+      if (t_delta_us) *t_delta_us = td;
+      return RAP_OK;
+    }
+    if (td < best_td) {
+      best_td = td;
+      best_b = b;
+    }
+  }
+  *sm_budget = best_b;
+  if (t_delta_us) *t_delta_us = best_td;
+  return RAP_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,324 @@
+"""Thin ctypes binding of librap.so (include/rap.h).
+
+Argument marshalling only: every step of the preprocessing path runs in the
+CUDA kernel behind the C ABI.  PyTorch supplies device memory and streams.
+There is no fallback: if librap.so is missing this module raises on import
+of the library (``load()``), and nothing here computes any operator.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import numpy as np
+
+from . import _build
+
+OPS = {"fillnull": 0, "logit": 1, "boxcox": 2, "onehot": 3, "sigridhash": 4,
+       "bucketize": 5, "firstx": 6, "clamp": 7, "ngram": 8, "mapid": 9}
+STATUS = {0: "OK", 1: "INVALID_ARGUMENT", 2: "INVALID_GRAPH", 3: "INVALID_PARAM", 4: "CAPACITY",
+          5: "UNSUPPORTED", 6: "CUDA", 7: "OUT_OF_MEMORY"}
+
+EXPORTS = ["rap_plan_create", "rap_plan_output_shape", "rap_preprocess", "rap_preprocess_host", "rap_set_budget",
+           "rap_predict_latency_us", "rap_choose_budget", "rap_plan_info_get", "rap_plan_destroy",
+           "rap_status_string", "rap_last_error"]
+
+
+class RapError(RuntimeError):
+    def __init__(self, status, detail=""):
+        self.status = STATUS.get(status, str(status))
+        super().__init__(f"RAP_ERR_{self.status}: {detail}")
+
+
+class RapNode(C.Structure):
+    _fields_ = [("op", C.c_int32), ("n_inputs", C.c_int32), ("inputs", C.POINTER(C.c_int32)), ("param", C.c_int32)]
+
+
+class RapGraph(C.Structure):
+    _fields_ = [("n_dense_in", C.c_int32), ("n_sparse_in", C.c_int32), ("n_nodes", C.c_int32),
+                ("nodes", C.POINTER(RapNode)), ("n_outputs", C.c_int32), ("output_nodes", C.POINTER(C.c_int32))]
+
+
+class RapOpParam(C.Structure):
+    _fields_ = [("f_fill", C.c_float), ("eps", C.c_float), ("lam", C.c_float),
+                ("i_fill", C.c_int64), ("lo", C.c_int64), ("hi", C.c_int64), ("x", C.c_int64),
+                ("max_value", C.c_int64), ("map_default", C.c_int64), ("salt", C.c_uint64),
+                ("n", C.c_int32), ("k_width", C.c_int32), ("n_borders", C.c_int32), ("borders", C.c_void_p),
+                ("map_size", C.c_int64), ("map_keys", C.c_void_p), ("map_vals", C.c_void_p)]
+
+
+class RapRawBatch(C.Structure):
+    _fields_ = [("n_rows", C.c_int64), ("dense", C.c_void_p), ("dense_valid", C.c_void_p),
+                ("sp_offsets", C.c_void_p), ("sp_values", C.c_void_p), ("sp_valid", C.c_void_p),
+                ("sp_nnz", C.c_void_p)]
+
+
+class RapOutput(C.Structure):
+    _fields_ = [("dense_out", C.c_void_p), ("dense_ld", C.c_int64), ("lengths", C.c_void_p),
+                ("offsets", C.c_void_p), ("values", C.c_void_p), ("values_capacity", C.c_int64)]
+
+
+class RapPlanInfo(C.Structure):
+    _fields_ = [("device", C.c_int32), ("sm_count", C.c_int32), ("sm_budget", C.c_int32),
+                ("ctas_per_sm", C.c_int32), ("threads_per_cta", C.c_int32), ("grid", C.c_int32),
+                ("n_dense_out_cols", C.c_int32), ("n_sparse_out", C.c_int32), ("n_dense_groups", C.c_int32),
+                ("rows_per_dense_desc", C.c_int32), ("max_rows_per_sparse_desc", C.c_int32),
+                ("min_rows_per_sparse_desc", C.c_int32), ("n_descriptors_last", C.c_int64),
+                ("n_launches", C.c_int64), ("smem_bytes", C.c_int64)]
+
+
+_lib = None
+
+
+def load(build_if_stale: bool = False):
+    """Load librap.so.  Raises if it is missing — there is no fallback path."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if build_if_stale:
+        _build.build()
+    if not os.path.exists(_build.LIB):
+        raise ImportError(f"librap.so not built at {_build.LIB}; run __graft_entry__.build()")
+    L = C.CDLL(_build.LIB)
+    P = C.c_void_p
+    L.rap_plan_create.restype = C.c_int
+    L.rap_plan_create.argtypes = [C.POINTER(RapGraph), C.POINTER(RapOpParam), C.c_int32, C.c_int32, C.c_int32,
+                                  C.POINTER(P)]
+    L.rap_plan_output_shape.restype = C.c_int
+    L.rap_plan_output_shape.argtypes = [P, C.c_int64, P, C.POINTER(C.c_int64), C.POINTER(C.c_int64),
+                                        C.POINTER(C.c_int64)]
+    L.rap_preprocess.restype = C.c_int
+    L.rap_preprocess.argtypes = [P, C.POINTER(RapRawBatch), C.POINTER(RapOutput), P]
+    L.rap_preprocess_host.restype = C.c_int
+    L.rap_preprocess_host.argtypes = [P, C.POINTER(RapRawBatch), C.POINTER(RapOutput), P]
+    L.rap_set_budget.restype = C.c_int
+    L.rap_set_budget.argtypes = [P, C.c_int32]
+    L.rap_predict_latency_us.restype = C.c_int
+    L.rap_predict_latency_us.argtypes = [P, C.c_int64, P, C.c_int32, C.POINTER(C.c_double)]
+    L.rap_choose_budget.restype = C.c_int
+    L.rap_choose_budget.argtypes = [P, C.c_int64, P, C.c_double, C.POINTER(C.c_int32), C.POINTER(C.c_double)]
+    L.rap_plan_info_get.restype = C.c_int
+    L.rap_plan_info_get.argtypes = [P, C.POINTER(RapPlanInfo)]
+    L.rap_plan_destroy.restype = None
+    L.rap_plan_destroy.argtypes = [P]
+    L.rap_status_string.restype = C.c_char_p
+    L.rap_status_string.argtypes = [C.c_int]
+    L.rap_last_error.restype = C.c_char_p
+    L.rap_last_error.argtypes = []
+    _lib = L
+    return L
+
+
+def _check(st):
+    if st != 0:
+        raise RapError(st, load().rap_last_error().decode())
+
+
+def raw_ref(kind: str, idx: int) -> int:
+    if kind == "n":
+        return int(idx)
+    if kind == "d":
+        return -1 - 2 * int(idx)
+    return -2 - 2 * int(idx)
+
+
+def marshal_graph(spec):
+    """Graph-spec dict (synth.py docstring) -> (RapGraph, RapOpParam[], keepalive)."""
+    keep = []
+    nodes = spec["nodes"]
+    n = len(nodes)
+    cn = (RapNode * max(n, 1))()
+    cp = (RapOpParam * max(n, 1))()
+    for i, nd in enumerate(nodes):
+        ins = (C.c_int32 * max(len(nd["inputs"]), 1))(*[raw_ref(k, x) for k, x in nd["inputs"]])
+        keep.append(ins)
+        op = nd["op"]
+        cn[i].op = OPS[op] if isinstance(op, str) else int(op)
+        cn[i].n_inputs = len(nd["inputs"])
+        cn[i].inputs = ins
+        cn[i].param = i
+        p = cp[i]
+        p.f_fill = nd.get("f_fill", 0.0)
+        p.eps = nd.get("eps", 1e-6)
+        p.lam = nd.get("lambda", 0.0)
+        p.i_fill = nd.get("i_fill", 0)
+        p.lo = nd.get("lo", 0)
+        p.hi = nd.get("hi", 0)
+        p.x = nd.get("x", 0)
+        p.max_value = nd.get("max_value", 0)
+        p.map_default = nd.get("map_default", 0)
+        p.salt = nd.get("salt", 0) & (2**64 - 1)
+        p.n = nd.get("n", 0)
+        p.k_width = nd.get("k", 0)
+        if "borders" in nd:
+            b = np.asarray(nd["borders"])
+            arr = np.ascontiguousarray(b, dtype=np.int64 if b.dtype.kind in "iu" else np.float32)
+            keep.append(arr)
+            p.n_borders = nd.get("n_borders", len(arr))
+            p.borders = arr.ctypes.data if len(arr) else None
+        else:
+            p.n_borders = nd.get("n_borders", 0)
+        if "keys" in nd:
+            k = np.ascontiguousarray(nd["keys"], dtype=np.int64)
+            v = np.ascontiguousarray(nd["vals"], dtype=np.int64)
+            keep += [k, v]
+            p.map_size = nd.get("map_size", len(k))
+            p.map_keys = k.ctypes.data if len(k) else None
+            p.map_vals = v.ctypes.data if len(v) else None
+        else:
+            p.map_size = nd.get("map_size", 0)
+    outs = (C.c_int32 * max(len(spec["outputs"]), 1))(*spec["outputs"])
+    g = RapGraph(spec["n_dense"], spec["n_sparse"], n, cn, len(spec["outputs"]), outs)
+    keep += [cn, cp, outs]
+    return g, cp, keep
+
+
+def _ptr_array(ptrs):
+    a = (C.c_void_p * max(len(ptrs), 1))()
+    for i, x in enumerate(ptrs):
+        a[i] = x
+    return a
+
+
+def _stream_handle(stream):
+    if stream is None:
+        import torch
+
+        return C.c_void_p(torch.cuda.current_stream().cuda_stream)
+    if isinstance(stream, int):
+        return C.c_void_p(stream)
+    return C.c_void_p(stream.cuda_stream)
+
+
+class DeviceBatch:
+    """A raw batch resident in device memory (torch tensors) + its C struct."""
+
+    def __init__(self, batch, device, pin=False):
+        import torch
+
+        self.n_rows = int(batch["n_rows"])
+        dev = torch.device(device) if not pin else torch.device("cpu")
+
+        def t(a, dt):
+            x = torch.from_numpy(np.ascontiguousarray(a, dtype=dt))
+            return x.pin_memory() if pin else x.to(dev, non_blocking=False)
+
+        self.dense = [t(x, np.float32) for x in batch["dense"]]
+        self.dense_valid = [None if x is None else t(x, np.uint32) for x in batch["dense_valid"]]
+        self.sp_off = [t(x, np.int32) for x in batch["sp_off"]]
+        self.sp_val = [t(x, np.int64) if len(x) else t(np.zeros(1, np.int64), np.int64) for x in batch["sp_val"]]
+        self.sp_valid = [None if x is None else t(x, np.uint32) for x in batch["sp_valid"]]
+        self.sp_nnz = np.array([int(o[-1]) - int(o[0]) for o in batch["sp_off"]] or [0], dtype=np.int64)
+        self._build_struct()
+
+    def _build_struct(self):
+        def ptr(x):
+            return None if x is None else x.data_ptr()
+
+        self._arrs = [_ptr_array([ptr(x) for x in self.dense]), _ptr_array([ptr(x) for x in self.dense_valid]),
+                      _ptr_array([ptr(x) for x in self.sp_off]), _ptr_array([ptr(x) for x in self.sp_val]),
+                      _ptr_array([ptr(x) for x in self.sp_valid])]
+        a = self._arrs
+        self.struct = RapRawBatch(self.n_rows, C.cast(a[0], C.c_void_p), C.cast(a[1], C.c_void_p),
+                                  C.cast(a[2], C.c_void_p), C.cast(a[3], C.c_void_p), C.cast(a[4], C.c_void_p),
+                                  self.sp_nnz.ctypes.data)
+
+
+class DeviceOutput:
+    """Output tensors (device, or pinned host when pin=True) + their C struct."""
+
+    def __init__(self, plan, n_rows, sp_nnz, device, pin=False, dense_ld=None, capacity=None):
+        import torch
+
+        d, f, vb = plan.output_shape(n_rows, sp_nnz)
+        self.d_out, self.f_out, self.bound = d, f, vb
+        ld = d if dense_ld is None else dense_ld
+        kw = {"pin_memory": True} if pin else {"device": device}
+        self.dense = torch.empty(max(n_rows * ld, 1), dtype=torch.float32, **kw)
+        self.lengths = torch.empty(max(n_rows * f, 1), dtype=torch.int32, **kw)
+        self.offsets = torch.empty(n_rows * f + 1, dtype=torch.int64, **kw)
+        cap = vb if capacity is None else capacity
+        self.values = torch.empty(max(cap, 1), dtype=torch.int64, **kw)
+        self.n_rows, self.ld = n_rows, ld
+        self.struct = RapOutput(self.dense.data_ptr(), ld, self.lengths.data_ptr(), self.offsets.data_ptr(),
+                                self.values.data_ptr(), cap)
+
+    def to_numpy(self):
+        B, d, f = self.n_rows, self.d_out, self.f_out
+        off = self.offsets.cpu().numpy()
+        n = int(off[-1]) if len(off) else 0
+        return {"dense": self.dense.cpu().numpy()[: B * self.ld].reshape(B, self.ld)[:, :d],
+                "lengths": self.lengths.cpu().numpy()[: B * f], "offsets": off,
+                "values": self.values.cpu().numpy()[:n]}
+
+
+class Plan:
+    """rap_plan_create / rap_preprocess / rap_set_budget (include/rap.h)."""
+
+    def __init__(self, spec, device: int = 0, sm_budget: int = 0):
+        L = load()
+        self.spec = spec
+        g, params, self._keep = marshal_graph(spec)
+        h = C.c_void_p()
+        _check(L.rap_plan_create(C.byref(g), params, len(spec["nodes"]), device, sm_budget, C.byref(h)))
+        self.handle = h
+        self.device = device
+
+    def close(self):
+        if getattr(self, "handle", None):
+            load().rap_plan_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def output_shape(self, n_rows, sp_nnz):
+        nnz = np.ascontiguousarray(sp_nnz if sp_nnz is not None and len(sp_nnz) else [0], dtype=np.int64)
+        d, f, vb = C.c_int64(), C.c_int64(), C.c_int64()
+        _check(load().rap_plan_output_shape(self.handle, n_rows, nnz.ctypes.data, C.byref(d), C.byref(f),
+                                            C.byref(vb)))
+        return d.value, f.value, vb.value
+
+    def preprocess(self, raw: DeviceBatch, out: DeviceOutput, stream=None):
+        _check(load().rap_preprocess(self.handle, C.byref(raw.struct), C.byref(out.struct), _stream_handle(stream)))
+
+    def preprocess_host(self, raw: DeviceBatch, out: DeviceOutput, stream=None):
+        """raw / out built with pin=True (host buffers); synchronises the stream."""
+        _check(load().rap_preprocess_host(self.handle, C.byref(raw.struct), C.byref(out.struct),
+                                          _stream_handle(stream)))
+
+    def set_budget(self, sm_budget: int):
+        _check(load().rap_set_budget(self.handle, sm_budget))
+
+    def info(self) -> dict:
+        i = RapPlanInfo()
+        _check(load().rap_plan_info_get(self.handle, C.byref(i)))
+        return {k: getattr(i, k) for k, _ in RapPlanInfo._fields_}
+
+    def predict_latency_us(self, n_rows, sp_nnz, sm_budget=0):
+        nnz = np.ascontiguousarray(sp_nnz if len(sp_nnz) else [0], dtype=np.int64)
+        v = C.c_double()
+        _check(load().rap_predict_latency_us(self.handle, n_rows, nnz.ctypes.data, sm_budget, C.byref(v)))
+        return v.value
+
+    def choose_budget(self, n_rows, sp_nnz, overlap_capacity_us):
+        nnz = np.ascontiguousarray(sp_nnz if len(sp_nnz) else [0], dtype=np.int64)
+        b, td = C.c_int32(), C.c_double()
+        _check(load().rap_choose_budget(self.handle, n_rows, nnz.ctypes.data, overlap_capacity_us, C.byref(b),
+                                        C.byref(td)))
+        return b.value, td.value
+
+
+def validate_only(spec):
+    """Status name rap_plan_create gives for a spec on device 0 (needs a GPU
+    only when the graph is valid)."""
+    L = load()
+    g, params, keep = marshal_graph(spec)
+    h = C.c_void_p()
+    st = L.rap_plan_create(C.byref(g), params, len(spec["nodes"]), 0, 0, C.byref(h))
+    if st == 0:
+        L.rap_plan_destroy(h)
+    return STATUS.get(st, str(st))
