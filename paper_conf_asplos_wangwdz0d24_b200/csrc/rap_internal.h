@@ -3,9 +3,15 @@
 // nothing here is shared with oracle/.
 //
 // A plan lowers every output of the preprocessing DAG to
-// a small "op program": a source (raw sparse column, dense expression then
-// Bucketize, or NGram) followed by elementwise id ops, with FirstX folded into
-// a length cap and FillNull into a null-row rule.
+// a flattened, position-independent program that a CTA copies into shared
+// memory in one coalesced burst before it processes a descriptor:
+//  - SProg, one per sparse output: an id-list chain (source = raw sparse
+//    column, dense expression + Bucketize, or NGram over up to 8 source
+//    chains), elementwise id ops, FirstX folded into a length cap and FillNull
+//    into a null-row rule, plus an optional staged Bucketize border table;
+//  - DProg, one per dense column group: the dense expressions and OneHot
+//    units that produce up to kGroupCols adjacent output columns.
+// DESIGN.md §7 describes the layout.
 #pragma once
 #include <stdint.h>
 
@@ -17,19 +23,30 @@
 
 namespace rapk {
 
-constexpr int kThreads = 256;        // threads per CTA
-constexpr int kMaxNgramK = 8;        // NGram sources (R7: 1 <= k <= 8)
+constexpr int kThreads = 256;          // threads per CTA
+constexpr int kMaxNgramK = 8;          // NGram sources (R7: 1 <= k <= 8)
 constexpr int64_t kNoCap = INT64_MAX;
+constexpr int kVBuf = 2048;            // output ids a sparse descriptor stages in smem
+constexpr int kRowsSparseMax = 1024;   // rows per sparse descriptor (upper bound)
+constexpr int kNgSlots = 1024;         // NGram (source, row) slots per descriptor: k * rows <= kNgSlots
+constexpr int kMaxStagedOps = 32;      // ops carried inside an SProg
+constexpr int kStageTab = 1024;        // int64 Bucketize borders staged with an SProg
+constexpr int kGroupCols = 64;         // dense output columns per column group
+constexpr int kMaxDenseOps = 96;       // ops carried inside a DProg
+constexpr int kDenseTabF = 256;        // f32 borders carried inside a DProg
+constexpr int kDenseTileBytes = 40960; // dense row-major tile budget (smem)
 
 // Elementwise op kinds.  Dense ops act on an f32 scalar, id ops on int64.
 enum OpKind : int32_t {
-  OK_FILL_F = 0,   // dense FillNull: NaN -> f0                          (R10)
-  OK_LOGIT = 1,    // f0 = lo = eps, f1 = hi = 1 - eps (f32)            (R11)
-  OK_BOXCOX = 2,   // f0 = lambda                                        (R12)
-  OK_CLAMP = 3,    // a = lo, b = hi                                     (R6)
-  OK_SIGRID = 4,   // hsalt = H(salt), M                                 (R3)
-  OK_BUCKET_I = 5, // itab[a .. a+m) sorted int64 borders                (R4)
-  OK_MAPID = 6     // itab[a .. a+m) sorted keys, itab[a+m ..) vals, b = default (R8)
+  OK_FILL_F = 0,    // dense FillNull: NaN -> f0                                  (R10)
+  OK_LOGIT = 1,     // f0 = lo = eps, f1 = hi = 1 - eps (f32)                     (R11)
+  OK_BOXCOX = 2,    // f0 = lambda                                                (R12)
+  OK_CLAMP = 3,     // a = lo, b = hi                                             (R6)
+  OK_SIGRID = 4,    // hsalt = H(salt), M                                         (R3)
+  OK_BUCKET_I = 5,  // global itab[a .. a+m) sorted int64 borders                 (R4)
+  OK_MAPID = 6,     // open-addressing table of 2^m (key, val) slots at itab[a ..),
+                    // b = default, M = 1 if INT64_MIN is a key (its value in hsalt) (R8)
+  OK_BUCKET_S = 7   // borders staged with the program: table[a .. a+m)          (R4)
 };
 
 struct DevOp {
@@ -42,69 +59,82 @@ struct DevOp {
 
 enum SrcKind : int32_t { SRC_SPARSE = 0, SRC_DENSE_BUCKET = 1, SRC_NGRAM = 2 };
 
-// Dense expression: raw dense column -> ops[op_begin, op_end) (all dense ops).
-struct DenseExpr {
-  int32_t col, op_begin, op_end, pad;
-};
-
-// Id-list chain.  Valid rows: out = ops[op_begin,op_end)(src[j]) for
-// j < min(L, xcap).  Null rows of a SRC_SPARSE source: if has_fill the list
-// is [fill] passed through ops[null_op_begin, op_end) and capped at
-// null_xcap, otherwise empty (R14).
+// Id-list chain (op indices are local to the program that holds it).
+// Valid rows: out = ops[op_begin,op_end)(src[j]) for j < min(L, xcap).
+// Null rows of a SRC_SPARSE source: with has_fill the list is [fill] passed
+// through ops[null_op_begin, op_end) and capped at null_xcap, otherwise empty
+// (R14).  SRC_DENSE_BUCKET: src = raw dense column, dense ops
+// [dop_begin, dop_end), f32 borders ftab[btab .. btab+bm) (global).
 struct Chain {
-  int32_t src_kind, src;        // sparse column | dense expr | ngram index
+  int32_t src_kind, src;
   int32_t op_begin, op_end;
   int32_t null_op_begin, has_fill;
   int64_t xcap, null_xcap;
   int64_t fill;
-  int32_t btab, bm;             // SRC_DENSE_BUCKET: f32 borders ftab[btab .. btab+bm)
+  int32_t btab, bm;
+  int32_t dop_begin, dop_end;
 };
 
 struct NGramDesc {
   int32_t n, k;
-  uint64_t hsalt;               // H(salt)
+  uint64_t hsalt;  // H(salt)
   int64_t M;
-  int32_t chain[kMaxNgramK];
+  int32_t chain[kMaxNgramK];  // host-side chain indices (unused on the device)
 };
 
-enum UnitKind : int32_t { U_DENSE = 0, U_ONEHOT = 1 };
-
-// A dense output unit inside a column group: one Dense column, or the
-// columns [col, col+width) of a OneHot, holding ids [k0, k0+width).
-struct Unit {
-  int32_t kind, idx, col, width;
-  int64_t k0;
+struct SProg {
+  Chain ch;
+  Chain src[kMaxNgramK];
+  NGramDesc ng;
+  int32_t n_ops;       // ops used
+  int32_t tab_len;     // staged int64 table entries (OK_BUCKET_S)
+  int32_t global_ops;  // 1: op indices refer to Common::ops (program too large to stage)
+  int32_t pad;
+  int64_t tab_off;     // itab offset of the staged table
+  DevOp ops[kMaxStagedOps];
 };
 
-// Column group: the dense output columns [col0, col0+width) one dense
-// descriptor writes for its row block.
-struct Group {
-  int32_t unit_begin, unit_end, col0, width;
+enum UnitKind : int32_t { U_DENSE = 0, U_ONEHOT_DB = 1, U_ONEHOT_G = 2 };
+
+// A dense output unit of a column group: one Dense column (U_DENSE), or the
+// columns [col, col+width) of a OneHot holding ids [k0, k0+width) —
+// U_ONEHOT_DB when its list is a dense Bucketize (id ops [iop_begin, iop_end),
+// cap xcap), U_ONEHOT_G (any other list) through the SProg oprogs[prog].
+// gops = 1: op indices / borders refer to Common::ops / Common::ftab.
+struct DUnit {
+  int32_t kind, col, width, src_col;
+  int32_t op_begin, op_end;
+  int32_t btab, bm;
+  int32_t iop_begin, iop_end;
+  int32_t prog, gops;
+  int64_t k0, xcap;
 };
 
-struct SparseOut {
-  int32_t chain, rows_per_desc;
+struct DProg {
+  int32_t n_units, width, col0, any_onehot;
+  int32_t n_ops, n_ftab, pad0, pad1;
+  DUnit units[kGroupCols];
+  DevOp ops[kMaxDenseOps];
+  float ftab[kDenseTabF];
 };
 
 // Non-array kernel parameters.
 struct Common {
-  const DevOp* ops;
-  const DenseExpr* dexprs;
-  const Chain* chains;
-  const NGramDesc* ngrams;
-  const Unit* units;
-  const Group* groups;
-  const SparseOut* souts;
+  const SProg* sprogs;        // [n_sparse_out]
+  const SProg* oprogs;        // OneHot generic programs
+  const DProg* dprogs;        // [n_groups]
+  const DevOp* ops;           // global op array (programs too large to stage)
   const float* ftab;
   const int64_t* itab;
-  const int32_t* desc_start;    // [n_sparse_out + 1] for this n_rows
+  const int32_t* desc_start;  // [n_sparse_out + 1] for this n_rows
+  const int32_t* rows_per_desc;  // [n_sparse_out]
   int32_t n_sparse_out, n_groups, rows_dense, tile_ld;
   int64_t n_rows, n_sparse_desc, n_total_desc;
   // sched[0] = ticket counter, sched[1] = CTAs done, sched[2] = epoch.  The
   // last CTA to finish resets the counters and advances the epoch, so the
   // launch parameters are identical from call to call (CUDA-graph replayable).
   unsigned long long* sched;
-  unsigned long long* status;   // decoupled look-back words, one per sparse descriptor
+  unsigned long long* status;  // decoupled look-back words, one per sparse descriptor
   int64_t status_cap;
   float* dense_out;
   int64_t ld;
@@ -141,6 +171,8 @@ RAP_HD uint64_t splitmix_H(uint64_t x) {
 
 // Launch entry implemented in rap_kernel.cu.  Returns a cudaError_t value.
 int launch_fused(const Common& c, const LaunchRaw& raw, int grid, int smem_bytes, void* stream);
+// Dynamic shared memory the kernel needs for a dense tile of tile_bytes.
+int fused_smem_bytes(int tile_bytes);
 // Occupancy query: CTAs per SM for the given dynamic smem.
 int fused_occupancy(int smem_bytes, int n_dense, int n_sparse, int* ctas_per_sm);
 

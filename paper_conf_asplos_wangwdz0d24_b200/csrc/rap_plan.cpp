@@ -42,9 +42,17 @@ rap_status cuda_fail(cudaError_t e, const char* what) {
 // Node value types (DESIGN.md §3 "type system").
 enum VType { VT_NONE = 0, VT_DENSE = 1, VT_IDS = 2, VT_VEC = 3 };
 
-constexpr int kGroupCols = 64;        // dense output columns per dense descriptor
-constexpr int kRowsDense = 128;       // rows per dense descriptor
-constexpr int kRowsSparse = 1024;     // rows per sparse descriptor
+// Host-only intermediate form of the lowering (the device sees SProg / DProg).
+struct DenseExpr {
+  int32_t col, op_begin, op_end, pad;
+};
+enum HUnitKind { HU_DENSE = 0, HU_ONEHOT = 1 };
+struct Unit {  // one dense output: a Dense node (idx = dense expr) or a OneHot (idx = chain)
+  int32_t kind, idx, col, width;
+};
+struct SparseOut {
+  int32_t chain, rows_per_desc;
+};
 
 int64_t sat_add(int64_t a, int64_t b) {
   if (a > INT64_MAX - b) return INT64_MAX;
@@ -65,21 +73,22 @@ struct rap_plan {
   std::vector<DenseExpr> dexprs;
   std::vector<Chain> chains;
   std::vector<NGramDesc> ngrams;
-  std::vector<Unit> units;
-  std::vector<Group> groups;
   std::vector<SparseOut> souts;
   std::vector<float> ftab;
   std::vector<int64_t> itab;
   std::vector<int> used_dense, used_sparse;
-  int d_out = 0, tile_ld = 1;
+  // flattened device programs
+  std::vector<SProg> sprogs, oprogs;
+  std::vector<DProg> dprogs;
+  int d_out = 0, rows_dense = 256;
   // device program blob
   unsigned char* blob = nullptr;
-  size_t off_ops = 0, off_dexprs = 0, off_chains = 0, off_ngrams = 0, off_units = 0, off_groups = 0, off_souts = 0,
-         off_ftab = 0, off_itab = 0;
+  size_t off_ops = 0, off_sprogs = 0, off_oprogs = 0, off_dprogs = 0, off_ftab = 0, off_itab = 0;
   // per-n_rows descriptor table
   int32_t* d_desc_start = nullptr;
+  int32_t* d_rows_per_desc = nullptr;
   int64_t desc_rows = -1;
-  std::vector<int32_t> h_desc_start;
+  std::vector<int32_t> h_desc_start, h_rows_per_desc;
   int64_t n_sparse_desc = 0, n_dense_desc = 0;
   // scheduling state
   unsigned long long* d_sched = nullptr;  // ticket, done, epoch (device-managed)
@@ -366,7 +375,10 @@ struct Lowerer {
     } else if (ch.src_kind == SRC_DENSE_BUCKET) {
       const rap_node& nd = g->nodes[cur];
       const rap_op_param& pr = params[nd.param];
-      ch.src = lower_dense(nd.inputs[0]);
+      const DenseExpr& de = P->dexprs[lower_dense(nd.inputs[0])];
+      ch.src = de.col;  // raw dense column; its dense ops precede the bucketize
+      ch.dop_begin = de.op_begin;
+      ch.dop_end = de.op_end;
       ch.btab = (int)P->ftab.size();
       ch.bm = pr.n_borders;
       const float* b = static_cast<const float*>(pr.borders);
@@ -410,15 +422,31 @@ struct Lowerer {
           break;
         }
         case RAP_OP_MAPID: {
+          // open-addressing hash table: 2^lg slots, load <= 1/2, Fibonacci
+          // hashing, linear probing; INT64_MIN marks an empty slot
           op.kind = OK_MAPID;
-          op.a = (int64_t)P->itab.size();
-          op.m = (int32_t)pr.map_size;
           op.b = pr.map_default;
-          std::vector<std::pair<int64_t, int64_t>> kv;
-          for (int64_t k = 0; k < pr.map_size; ++k) kv.push_back({pr.map_keys[k], pr.map_vals[k]});
-          std::sort(kv.begin(), kv.end());
-          for (auto& e : kv) P->itab.push_back(e.first);
-          for (auto& e : kv) P->itab.push_back(e.second);
+          int lg = 4;
+          while ((int64_t(1) << lg) < 2 * pr.map_size) ++lg;
+          const int64_t cap = int64_t(1) << lg;
+          if (P->itab.size() % 2) P->itab.push_back(0);  // 16-byte aligned slots
+          op.a = (int64_t)P->itab.size();
+          op.m = lg;
+          P->itab.resize(P->itab.size() + 2 * cap, 0);
+          int64_t* tab = P->itab.data() + op.a;
+          for (int64_t k = 0; k < cap; ++k) tab[2 * k] = INT64_MIN;
+          for (int64_t k = 0; k < pr.map_size; ++k) {
+            const int64_t key = pr.map_keys[k];
+            if (key == INT64_MIN) {
+              op.M = 1;
+              op.hsalt = (uint64_t)pr.map_vals[k];
+              continue;
+            }
+            uint64_t i = ((uint64_t)key * 0x9E3779B97F4A7C15ull) >> (64 - lg);
+            while (tab[2 * i] != INT64_MIN) i = (i + 1) & (uint64_t)(cap - 1);
+            tab[2 * i] = key;
+            tab[2 * i + 1] = pr.map_vals[k];
+          }
           break;
         }
         default:
@@ -478,6 +506,20 @@ int64_t chain_bound(const rap_plan* P, const Chain& ch, int64_t B, const int64_t
   return std::min(b, sat_mul(ch.xcap, B));
 }
 
+double expected_len(const rap_plan* P, const Chain& ch, int64_t B, const int64_t* nnz) {
+  double e;
+  if (ch.src_kind == SRC_SPARSE) {
+    e = (nnz && B > 0 ? (double)std::max<int64_t>(nnz[ch.src], 0) / (double)B : 1.0) + (ch.has_fill ? 1.0 : 0.0);
+  } else if (ch.src_kind == SRC_DENSE_BUCKET) {
+    e = 1.0;
+  } else {
+    const NGramDesc& ng = P->ngrams[ch.src];
+    e = 0;
+    for (int k = 0; k < ng.k; ++k) e += expected_len(P, P->chains[ng.chain[k]], B, nnz);
+  }
+  return std::min(e, (double)ch.xcap);
+}
+
 int64_t values_bound(const rap_plan* P, int64_t B, const int64_t* nnz) {
   int64_t tot = 0;
   for (const SparseOut& so : P->souts) tot = sat_add(tot, chain_bound(P, P->chains[so.chain], B, nnz));
@@ -497,6 +539,163 @@ double algorithmic_bytes(const rap_plan* P, int64_t B, const int64_t* nnz) {
   for (int s : P->used_sparse) b += 4.0 * (B + 1) + 8.0 * (nnz ? nnz[s] : 0) + B / 8.0;
   b += 4.0 * B * P->d_out + 12.0 * B * P->souts.size() + 8.0 + 8.0 * values_bound(P, B, nnz);
   return b;
+}
+
+// ----------------------------------------------------------------------------
+// Flattened device programs (rap_internal.h).
+
+// SProg of an id chain: the chain (and an NGram's source chains) with their
+// ops copied in and rebased; the first Bucketize border tables that fit are
+// staged next to the program.  Programs with more than kMaxStagedOps ops keep
+// global op indices.
+SProg make_sprog(rap_plan* P, int chain_idx) {
+  SProg sp;
+  memset(&sp, 0, sizeof(sp));
+  sp.ch = P->chains[chain_idx];
+  int nsrc = 0;
+  if (sp.ch.src_kind == SRC_NGRAM) {
+    sp.ng = P->ngrams[sp.ch.src];
+    nsrc = sp.ng.k;
+    for (int k = 0; k < nsrc; ++k) sp.src[k] = P->chains[sp.ng.chain[k]];
+  }
+  int total = 0;
+  for (int c = 0; c <= nsrc; ++c) {
+    const Chain& cc = c == 0 ? sp.ch : sp.src[c - 1];
+    total += cc.op_end - cc.op_begin;
+    if (cc.src_kind == SRC_DENSE_BUCKET) total += cc.dop_end - cc.dop_begin;
+  }
+  if (total > kMaxStagedOps) {
+    sp.global_ops = 1;
+    return sp;
+  }
+  int pos = 0;
+  for (int c = 0; c <= nsrc; ++c) {
+    Chain& cc = c == 0 ? sp.ch : sp.src[c - 1];
+    if (cc.src_kind == SRC_DENSE_BUCKET) {
+      const int n = cc.dop_end - cc.dop_begin;
+      for (int k = 0; k < n; ++k) sp.ops[pos + k] = P->ops[cc.dop_begin + k];
+      cc.dop_begin = pos;
+      cc.dop_end = pos + n;
+      pos += n;
+    }
+    const int n = cc.op_end - cc.op_begin;
+    for (int k = 0; k < n; ++k) sp.ops[pos + k] = P->ops[cc.op_begin + k];
+    cc.null_op_begin = pos + (cc.null_op_begin - cc.op_begin);
+    cc.op_begin = pos;
+    cc.op_end = pos + n;
+    pos += n;
+  }
+  sp.n_ops = pos;
+  std::vector<int64_t> tab;
+  for (int o = 0; o < pos; ++o) {
+    DevOp& op = sp.ops[o];
+    if (op.kind == OK_BUCKET_I && (int)tab.size() + op.m <= kStageTab) {
+      const int64_t local = (int64_t)tab.size();
+      tab.insert(tab.end(), P->itab.begin() + op.a, P->itab.begin() + op.a + op.m);
+      op.kind = OK_BUCKET_S;
+      op.a = local;
+    }
+  }
+  if (!tab.empty()) {
+    if (P->itab.size() % 2) P->itab.push_back(0);  // 16-byte aligned for the staging copy
+    sp.tab_off = (int64_t)P->itab.size();
+    sp.tab_len = (int32_t)tab.size();
+    P->itab.insert(P->itab.end(), tab.begin(), tab.end());
+  }
+  return sp;
+}
+
+// DProgs: dense outputs packed left to right into column groups of at most
+// kGroupCols columns, kMaxDenseOps ops and kDenseTabF borders (a OneHot may
+// be split across groups).
+void build_dprogs(rap_plan* P, const std::vector<Unit>& flat) {
+  std::vector<int> oprog_of(P->chains.size(), -1);
+  DProg cur;
+  memset(&cur, 0, sizeof(cur));
+  auto close = [&](int end_col) {
+    if (cur.n_units == 0) return;
+    cur.width = end_col - cur.col0;
+    P->dprogs.push_back(cur);
+    memset(&cur, 0, sizeof(cur));
+  };
+  for (const Unit& u : flat) {
+    // what one piece of this unit needs inside a DProg
+    int need_ops = 0, need_tab = 0, kind = U_DENSE;
+    const DenseExpr* de = nullptr;
+    const Chain* ch = nullptr;
+    if (u.kind == HU_DENSE) {
+      de = &P->dexprs[u.idx];
+      need_ops = de->op_end - de->op_begin;
+    } else {
+      ch = &P->chains[u.idx];
+      if (ch->src_kind == SRC_DENSE_BUCKET) {
+        kind = U_ONEHOT_DB;
+        need_ops = (ch->dop_end - ch->dop_begin) + (ch->op_end - ch->op_begin);
+        need_tab = ch->bm;
+      } else {
+        kind = U_ONEHOT_G;
+        if (oprog_of[u.idx] < 0) {
+          oprog_of[u.idx] = (int)P->oprogs.size();
+          P->oprogs.push_back(make_sprog(P, u.idx));
+        }
+      }
+    }
+    const bool global = need_ops > kMaxDenseOps || need_tab > kDenseTabF;
+    if (global) need_ops = need_tab = 0;
+    int c = u.col, remaining = u.width;
+    int64_t k0 = 0;
+    while (remaining > 0) {
+      if (cur.n_units == 0) cur.col0 = c;
+      if (c - cur.col0 >= kGroupCols || cur.n_units == kGroupCols || cur.n_ops + need_ops > kMaxDenseOps ||
+          cur.n_ftab + need_tab > kDenseTabF) {
+        close(c);
+        cur.col0 = c;
+      }
+      const int w = std::min(kGroupCols - (c - cur.col0), remaining);
+      DUnit du;
+      memset(&du, 0, sizeof(du));
+      du.kind = kind;
+      du.col = c - cur.col0;
+      du.width = w;
+      du.k0 = k0;
+      du.gops = global ? 1 : 0;
+      auto copy_ops = [&](int b, int e, int32_t* ob, int32_t* oe) {
+        if (global) {
+          *ob = b;
+          *oe = e;
+          return;
+        }
+        *ob = cur.n_ops;
+        for (int k = b; k < e; ++k) cur.ops[cur.n_ops++] = P->ops[k];
+        *oe = cur.n_ops;
+      };
+      if (kind == U_DENSE) {
+        du.src_col = de->col;
+        copy_ops(de->op_begin, de->op_end, &du.op_begin, &du.op_end);
+      } else if (kind == U_ONEHOT_DB) {
+        du.src_col = ch->src;
+        du.xcap = ch->xcap;
+        copy_ops(ch->dop_begin, ch->dop_end, &du.op_begin, &du.op_end);
+        copy_ops(ch->op_begin, ch->op_end, &du.iop_begin, &du.iop_end);
+        du.bm = ch->bm;
+        if (global) {
+          du.btab = ch->btab;
+        } else {
+          du.btab = cur.n_ftab;
+          for (int k = 0; k < ch->bm; ++k) cur.ftab[cur.n_ftab++] = P->ftab[ch->btab + k];
+        }
+      } else {
+        du.prog = oprog_of[u.idx];
+        du.xcap = ch->xcap;
+      }
+      cur.units[cur.n_units++] = du;
+      if (kind != U_DENSE) cur.any_onehot = 1;
+      c += w;
+      k0 += w;
+      remaining -= w;
+    }
+  }
+  close(P->d_out);
 }
 
 }  // namespace
@@ -563,7 +762,7 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
     const int t = v.type[node];
     if (t == VT_DENSE) {
       Unit u{};
-      u.kind = U_DENSE;
+      u.kind = HU_DENSE;
       u.idx = L.lower_dense(node);
       u.col = col;
       u.width = 1;
@@ -577,11 +776,10 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
         return st;
       }
       Unit u{};
-      u.kind = U_ONEHOT;
+      u.kind = HU_ONEHOT;
       u.idx = c;
       u.col = col;
       u.width = params[nd.param].k_width;
-      u.k0 = 0;
       flat_units.push_back(u);
       col += u.width;
     } else {
@@ -592,54 +790,20 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
       }
       SparseOut so{};
       so.chain = c;
-      so.rows_per_desc = kRowsSparse;
+      so.rows_per_desc = kRowsSparseMax;
       P->souts.push_back(so);
     }
   }
   P->d_out = col;
-  // ---- column groups of <= kGroupCols columns (OneHot units may be split)
+  // ---- flattened device programs
+  for (const SparseOut& so : P->souts) P->sprogs.push_back(make_sprog(P, so.chain));
+  build_dprogs(P, flat_units);
   {
-    int gcol0 = 0;
-    Group cur{};
-    cur.unit_begin = 0;
-    cur.col0 = 0;
-    for (const Unit& u0 : flat_units) {
-      Unit u = u0;
-      int remaining = u.width;
-      int64_t k0 = u.k0;
-      int c = u.col;
-      while (remaining > 0) {
-        int room = kGroupCols - (c - gcol0);
-        if (room == 0) {
-          cur.unit_end = (int)P->units.size();
-          cur.width = c - gcol0;
-          P->groups.push_back(cur);
-          gcol0 = c;
-          cur = Group{};
-          cur.unit_begin = (int)P->units.size();
-          cur.col0 = gcol0;
-          room = kGroupCols;
-        }
-        int w = std::min(room, remaining);
-        Unit piece = u;
-        piece.col = c;
-        piece.width = w;
-        piece.k0 = k0;
-        P->units.push_back(piece);
-        c += w;
-        k0 += w;
-        remaining -= w;
-      }
-    }
-    if (col > gcol0) {
-      cur.unit_end = (int)P->units.size();
-      cur.width = col - gcol0;
-      P->groups.push_back(cur);
-    }
+    int max_w = 1;
+    for (const DProg& dp : P->dprogs) max_w = std::max(max_w, dp.width);
+    const int rows = kDenseTileBytes / ((max_w | 1) * 4);
+    P->rows_dense = std::max(32, std::min(256, rows / 32 * 32));
   }
-  int max_w = 1;
-  for (const Group& gr : P->groups) max_w = std::max(max_w, gr.width);
-  P->tile_ld = max_w | 1;
   // used raw columns (for the byte model)
   {
     std::vector<char> ud(graph->n_dense_in, 0), us(graph->n_sparse_in, 0);
@@ -658,12 +822,9 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
   // ---- device blob
   std::vector<unsigned char> blob;
   P->off_ops = push_blob(blob, P->ops);
-  P->off_dexprs = push_blob(blob, P->dexprs);
-  P->off_chains = push_blob(blob, P->chains);
-  P->off_ngrams = push_blob(blob, P->ngrams);
-  P->off_units = push_blob(blob, P->units);
-  P->off_groups = push_blob(blob, P->groups);
-  P->off_souts = push_blob(blob, P->souts);
+  P->off_sprogs = push_blob(blob, P->sprogs);
+  P->off_oprogs = push_blob(blob, P->oprogs);
+  P->off_dprogs = push_blob(blob, P->dprogs);
   P->off_ftab = push_blob(blob, P->ftab);
   P->off_itab = push_blob(blob, P->itab);
   if (blob.empty()) blob.resize(16);
@@ -677,15 +838,16 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
   if (e == cudaSuccess) e = cudaMalloc(&P->d_err, sizeof(int32_t));
   if (e == cudaSuccess) e = cudaMemset(P->d_err, 0, sizeof(int32_t));
   if (e == cudaSuccess) e = cudaMalloc(&P->d_desc_start, sizeof(int32_t) * (P->souts.size() + 1));
+  if (e == cudaSuccess) e = cudaMalloc(&P->d_rows_per_desc, sizeof(int32_t) * (P->souts.size() + 1));
   if (e != cudaSuccess) {
     rap_plan_destroy(P);
     return cuda_fail(e, "plan device allocation");
   }
 
   // ---- shared memory and occupancy
-  const int sparse_smem = kRowsSparse * (4 + 8 + 4) + 16;
-  const int dense_smem = kRowsDense * P->tile_ld * 4;
-  P->smem = std::max(sparse_smem, dense_smem);
+  int max_w = 1;
+  for (const DProg& dp : P->dprogs) max_w = std::max(max_w, dp.width);
+  P->smem = fused_smem_bytes(P->rows_dense * (max_w | 1) * 4);
   int occ = 0;
   e = (cudaError_t)fused_occupancy(P->smem, P->n_dense_in, P->n_sparse_in, &occ);
   if (e != cudaSuccess) {
@@ -704,6 +866,7 @@ void rap_plan_destroy(rap_plan* P) {
   cudaFree(P->d_sched);
   cudaFree(P->d_err);
   cudaFree(P->d_desc_start);
+  cudaFree(P->d_rows_per_desc);
   cudaFree(P->d_status);
   for (void* s : P->stage) cudaFree(s);
   delete P;
@@ -736,10 +899,15 @@ rap_status rap_plan_info_get(const rap_plan* P, rap_plan_info* info) {
   info->grid = P->budget * P->ctas_per_sm;
   info->n_dense_out_cols = P->d_out;
   info->n_sparse_out = (int32_t)P->souts.size();
-  info->n_dense_groups = (int32_t)P->groups.size();
-  info->rows_per_dense_desc = kRowsDense;
-  info->max_rows_per_sparse_desc = kRowsSparse;
-  info->min_rows_per_sparse_desc = kRowsSparse;
+  info->n_dense_groups = (int32_t)P->dprogs.size();
+  info->rows_per_dense_desc = P->rows_dense;
+  int rmax = 0, rmin = INT32_MAX;
+  for (const SparseOut& so : P->souts) {
+    rmax = std::max(rmax, so.rows_per_desc);
+    rmin = std::min(rmin, so.rows_per_desc);
+  }
+  info->max_rows_per_sparse_desc = rmax;
+  info->min_rows_per_sparse_desc = P->souts.empty() ? 0 : rmin;
   info->n_descriptors_last = P->last_n_desc;
   info->n_launches = P->n_launches;
   info->smem_bytes = P->smem;
@@ -749,7 +917,7 @@ rap_status rap_plan_info_get(const rap_plan* P, rap_plan_info* info) {
 static rap_status check_batch(const rap_plan* P, const rap_raw_batch* raw, const rap_output* out) {
   if (!P || !raw || !out) return fail(RAP_ERR_INVALID_ARGUMENT, "NULL argument");
   if (raw->n_rows < 0) return fail(RAP_ERR_INVALID_ARGUMENT, "n_rows < 0");
-  if (raw->n_rows > (int64_t)INT32_MAX - kRowsSparse) return fail(RAP_ERR_INVALID_ARGUMENT, "n_rows too large");
+  if (raw->n_rows > (int64_t)INT32_MAX - kRowsSparseMax) return fail(RAP_ERR_INVALID_ARGUMENT, "n_rows too large");
   const int64_t B = raw->n_rows;
   if (B == 0) {
     if (!P->souts.empty() && !out->offsets) return fail(RAP_ERR_INVALID_ARGUMENT, "offsets NULL");
@@ -784,22 +952,48 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
     }
     return RAP_OK;
   }
-  // per-n_rows descriptor table (feature-major sparse descriptors)
-  if (P->desc_rows != B) {
-    P->h_desc_start.assign(P->souts.size() + 1, 0);
-    int64_t acc = 0;
+  // per-call descriptor table (feature-major sparse descriptors).  Rows per
+  // descriptor are chosen so a descriptor's output ids fit the kVBuf staging
+  // buffer at the expected list length (the work-descriptor table).
+  {
+    bool changed = P->desc_rows != B;
     for (size_t f = 0; f < P->souts.size(); ++f) {
-      P->h_desc_start[f] = (int32_t)acc;
-      acc += (B + P->souts[f].rows_per_desc - 1) / P->souts[f].rows_per_desc;
+      const double e = expected_len(P, P->chains[P->souts[f].chain], B, raw->sp_nnz);
+      int R = kRowsSparseMax;
+      while (R > 32 && R * std::max(e, 1.0) > 0.75 * kVBuf) R >>= 1;
+      const Chain& ch = P->chains[P->souts[f].chain];
+      if (ch.src_kind == SRC_NGRAM)
+        while (R * P->ngrams[ch.src].k > kNgSlots) R >>= 1;
+      if (R != P->souts[f].rows_per_desc) {
+        P->souts[f].rows_per_desc = R;
+        changed = true;
+      }
     }
-    P->h_desc_start[P->souts.size()] = (int32_t)acc;
-    P->n_sparse_desc = acc;
-    e = cudaMemcpyAsync(P->d_desc_start, P->h_desc_start.data(), sizeof(int32_t) * P->h_desc_start.size(),
-                        cudaMemcpyHostToDevice, stream);
-    if (e != cudaSuccess) return cuda_fail(e, "descriptor table upload");
-    P->desc_rows = B;
+    if (changed) {
+      P->h_desc_start.assign(P->souts.size() + 1, 0);
+      int64_t acc = 0;
+      for (size_t f = 0; f < P->souts.size(); ++f) {
+        P->h_desc_start[f] = (int32_t)acc;
+        acc += (B + P->souts[f].rows_per_desc - 1) / P->souts[f].rows_per_desc;
+      }
+      P->h_desc_start[P->souts.size()] = (int32_t)acc;
+      P->n_sparse_desc = acc;
+      e = cudaMemcpyAsync(P->d_desc_start, P->h_desc_start.data(), sizeof(int32_t) * P->h_desc_start.size(),
+                          cudaMemcpyHostToDevice, stream);
+      if (e == cudaSuccess)
+      {
+        std::vector<int32_t> rpd(P->souts.size() + 1, 0);
+        for (size_t f = 0; f < P->souts.size(); ++f) rpd[f] = P->souts[f].rows_per_desc;
+        P->h_rows_per_desc = rpd;
+        if (e == cudaSuccess)
+          e = cudaMemcpyAsync(P->d_rows_per_desc, P->h_rows_per_desc.data(), sizeof(int32_t) * rpd.size(),
+                              cudaMemcpyHostToDevice, stream);
+      }
+      if (e != cudaSuccess) return cuda_fail(e, "descriptor table upload");
+      P->desc_rows = B;
+    }
   }
-  P->n_dense_desc = P->groups.empty() ? 0 : (int64_t)P->groups.size() * ((B + kRowsDense - 1) / kRowsDense);
+  P->n_dense_desc = P->dprogs.empty() ? 0 : (int64_t)P->dprogs.size() * ((B + P->rows_dense - 1) / P->rows_dense);
   const int64_t n_total = P->n_sparse_desc + P->n_dense_desc;
   if (n_total == 0) return RAP_OK;
   // scan state (grows, never shrinks)
@@ -820,19 +1014,16 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
   const int64_t grid = std::min<int64_t>(n_total, (int64_t)P->budget * P->ctas_per_sm);
   Common c{};
   c.ops = reinterpret_cast<const DevOp*>(P->blob + P->off_ops);
-  c.dexprs = reinterpret_cast<const DenseExpr*>(P->blob + P->off_dexprs);
-  c.chains = reinterpret_cast<const Chain*>(P->blob + P->off_chains);
-  c.ngrams = reinterpret_cast<const NGramDesc*>(P->blob + P->off_ngrams);
-  c.units = reinterpret_cast<const Unit*>(P->blob + P->off_units);
-  c.groups = reinterpret_cast<const Group*>(P->blob + P->off_groups);
-  c.souts = reinterpret_cast<const SparseOut*>(P->blob + P->off_souts);
+  c.sprogs = reinterpret_cast<const SProg*>(P->blob + P->off_sprogs);
+  c.oprogs = reinterpret_cast<const SProg*>(P->blob + P->off_oprogs);
+  c.dprogs = reinterpret_cast<const DProg*>(P->blob + P->off_dprogs);
   c.ftab = reinterpret_cast<const float*>(P->blob + P->off_ftab);
   c.itab = reinterpret_cast<const int64_t*>(P->blob + P->off_itab);
   c.desc_start = P->d_desc_start;
   c.n_sparse_out = (int32_t)P->souts.size();
-  c.n_groups = (int32_t)P->groups.size();
-  c.rows_dense = kRowsDense;
-  c.tile_ld = P->tile_ld;
+  c.n_groups = (int32_t)P->dprogs.size();
+  c.rows_dense = P->rows_dense;
+  c.rows_per_desc = P->d_rows_per_desc;
   c.n_rows = B;
   c.n_sparse_desc = P->n_sparse_desc;
   c.n_total_desc = n_total;
