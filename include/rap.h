@@ -197,6 +197,14 @@ rap_status rap_choose_budget(const rap_plan* plan, int64_t n_rows, const int64_t
                              double overlap_capacity_us, int32_t* sm_budget, double* t_delta_us);
 
 rap_status rap_plan_info_get(const rap_plan* plan, rap_plan_info* info);
+
+/* Profiling aid.  enable = 1: the following rap_preprocess calls record 8
+ * uint64 stamps per descriptor (slot 0 = %globaltimer at descriptor start,
+ * slots 1..7 = clock64 at phase boundaries) for up to `cap` descriptors.
+ * enable = 0: synchronise the device and copy the stamps of the last call to
+ * HOST host_out (uint64[cap * 8]); *n_desc receives that call's descriptor
+ * count.  enable = -1: stop recording and free the buffer. */
+rap_status rap_debug_trace(rap_plan* plan, int32_t enable, uint64_t* host_out, int64_t cap, int64_t* n_desc);
 void rap_plan_destroy(rap_plan* plan);
 
 const char* rap_status_string(rap_status status);

@@ -34,7 +34,11 @@ constexpr int kStageTab = 1024;        // int64 Bucketize borders staged with an
 constexpr int kGroupCols = 64;         // dense output columns per column group
 constexpr int kMaxDenseOps = 96;       // ops carried inside a DProg
 constexpr int kDenseTabF = 256;        // f32 borders carried inside a DProg
-constexpr int kDenseTileBytes = 40960; // dense row-major tile budget (smem)
+constexpr int kDenseTileBytes = 28672; // dense row-major tile budget (smem)
+constexpr int kDenseInBytes = 12288;   // dense input columns staged per descriptor (smem)
+constexpr int kInVals = 2048;          // child ids of a sparse descriptor staged in smem
+constexpr int kInOff = 1088;           // staged offsets (all sources of a descriptor)
+constexpr int kInBm = 128;             // staged validity words (all sources)
 
 // Elementwise op kinds.  Dense ops act on an f32 scalar, id ops on int64.
 enum OpKind : int32_t {
@@ -82,10 +86,30 @@ struct NGramDesc {
   int32_t chain[kMaxNgramK];  // host-side chain indices (unused on the device)
 };
 
+// Canonical pipeline: a SRC_SPARSE chain whose id ops are an
+// ordered subset of Clamp -> MapId -> SigridHash -> Bucketize (each at most
+// once, MapId without an INT64_MIN key) runs through a specialised,
+// register-resident code path instead of the op interpreter.  mask bits:
+// 1 Clamp, 2 MapId, 4 SigridHash, 8 Bucketize; null_mask = the stages a
+// filled null row goes through.  For an NGram output the same form describes
+// the post-hash ops.
+enum CanonBit : int32_t { CB_CLAMP = 1, CB_MAPID = 2, CB_SIGRID = 4, CB_BUCKET = 8 };
+struct Canon {
+  int32_t ok, mask, null_mask, map_m;
+  int32_t bk_m, pad;
+  int64_t lo, hi;          // Clamp
+  int64_t map_a, map_def;  // MapId: itab offset of the table, default
+  uint64_t hs;             // SigridHash: H(salt)
+  int64_t M;
+  int64_t bk_a;            // Bucketize: absolute itab offset of the borders
+};
+
 struct SProg {
   Chain ch;
   Chain src[kMaxNgramK];
   NGramDesc ng;
+  Canon cn;                  // the output chain (post-hash ops for an NGram)
+  Canon src_cn[kMaxNgramK];  // NGram sources
   int32_t n_ops;       // ops used
   int32_t tab_len;     // staged int64 table entries (OK_BUCKET_S)
   int32_t global_ops;  // 1: op indices refer to Common::ops (program too large to stage)
@@ -101,22 +125,51 @@ enum UnitKind : int32_t { U_DENSE = 0, U_ONEHOT_DB = 1, U_ONEHOT_G = 2 };
 // U_ONEHOT_DB when its list is a dense Bucketize (id ops [iop_begin, iop_end),
 // cap xcap), U_ONEHOT_G (any other list) through the SProg oprogs[prog].
 // gops = 1: op indices / borders refer to Common::ops / Common::ftab.
+// slot: index of src_col in DProg::cols (the staged input columns).
 struct DUnit {
   int32_t kind, col, width, src_col;
   int32_t op_begin, op_end;
   int32_t btab, bm;
   int32_t iop_begin, iop_end;
   int32_t prog, gops;
+  int32_t slot, pad;
   int64_t k0, xcap;
 };
 
 struct DProg {
   int32_t n_units, width, col0, any_onehot;
-  int32_t n_ops, n_ftab, pad0, pad1;
+  int32_t n_ops, n_ftab, n_cols, pad1;
+  int32_t cols[kGroupCols];  // distinct raw dense columns read by the group
   DUnit units[kGroupCols];
   DevOp ops[kMaxDenseOps];
   float ftab[kDenseTabF];
 };
+
+// Work decomposition of one launch.  Sparse tiles are
+// (output f, 128-row range rt), numbered feature-major t = f * T + rt, which
+// is also the order of the jagged scan (R17).  The planner's cost model cuts
+// [0, S) into one contiguous chunk per CTA and deals out the dense blocks
+// (128 rows x one column group) so every CTA gets about the same estimated
+// work.  CTA i then: (1) computes the output lengths of its chunk (one warp per
+// tile) and their chunk-local exclusive prefix; (2) publishes the chunk total;
+// (3) runs its dense blocks; (4) obtains its chunk base by a decoupled
+// look-back over CTAs < i (usually already resolved thanks to (3)); (5) writes
+// offsets and ids of its chunk.  No grid barrier.
+constexpr int kMaxCtas = 2048;        // look-back words / partition entries a plan allocates
+constexpr int kTileRows = 128;        // rows of a sparse tile (4 groups of 32)
+constexpr int kDenseBlockRows = 128;  // rows of a dense block (CTA unit)
+
+// Per-CTA partition: sparse tiles [s0(i), s0(i+1)), dense blocks [d0(i), d0(i+1)).
+struct Part {
+  int32_t s0, d0;
+};
+
+// Look-back status word: [63:44] epoch, [43:42] flag, [41:0] value.
+constexpr int kEpochShift = 44;
+constexpr int kFlagShift = 42;
+constexpr unsigned long long kValueMask = (1ull << 42) - 1;
+constexpr unsigned long long kFlagAgg = 1, kFlagPrefix = 2;
+constexpr unsigned long long kEpochMax = (1ull << 20) - 1;
 
 // Non-array kernel parameters.
 struct Common {
@@ -126,16 +179,18 @@ struct Common {
   const DevOp* ops;           // global op array (programs too large to stage)
   const float* ftab;
   const int64_t* itab;
-  const int32_t* desc_start;  // [n_sparse_out + 1] for this n_rows
-  const int32_t* rows_per_desc;  // [n_sparse_out]
-  int32_t n_sparse_out, n_groups, rows_dense, tile_ld;
-  int64_t n_rows, n_sparse_desc, n_total_desc;
-  // sched[0] = ticket counter, sched[1] = CTAs done, sched[2] = epoch.  The
-  // last CTA to finish resets the counters and advances the epoch, so the
-  // launch parameters are identical from call to call (CUDA-graph replayable).
+  int32_t n_sparse_out, n_groups;
+  int64_t n_rows;
+  int64_t tiles_per_feature;  // T = ceil(n_rows / kTileRows)
+  int64_t n_sparse_tiles;     // S = n_sparse_out * T
+  int64_t n_dense_tiles;      // n_groups * ceil(n_rows / kDenseBlockRows)
+  const Part* part;           // [gridDim.x + 1]
+  // sched[0] = CTAs done, sched[1] = epoch of the look-back words; the last
+  // CTA advances the epoch, so launch parameters are identical from call to
+  // call (CUDA-graph replayable).
   unsigned long long* sched;
-  unsigned long long* status;  // decoupled look-back words, one per sparse descriptor
-  int64_t status_cap;
+  unsigned long long* status;  // [gridDim.x] look-back words, one per CTA chunk
+  int64_t* tile_sum;           // [S] tile length sums -> chunk-local exclusive prefixes
   float* dense_out;
   int64_t ld;
   int32_t* lengths;
@@ -143,7 +198,12 @@ struct Common {
   int64_t* values;
   int64_t values_cap;
   int32_t* err;
+  // profiling aid (rap_debug_trace): kTracePts globaltimer stamps per CTA
+  unsigned long long* trace;
+  int64_t trace_cap;
 };
+
+constexpr int kTracePts = 8;
 
 struct LaunchRaw {
   int32_t n_dense, n_sparse;
@@ -154,13 +214,6 @@ struct LaunchRaw {
   const uint32_t* const* svalid;
 };
 
-// Status word of the look-back: [63:44] epoch, [43:42] flag, [41:0] value.
-constexpr int kEpochShift = 44;
-constexpr int kFlagShift = 42;
-constexpr unsigned long long kValueMask = (1ull << 42) - 1;
-constexpr unsigned long long kFlagAgg = 1, kFlagPrefix = 2;
-constexpr unsigned long long kEpochMax = (1ull << 20) - 1;
-
 // ---- hash (reading R1/R2), product-side implementation ----
 RAP_HD uint64_t splitmix_H(uint64_t x) {
   uint64_t z = x + 0x9E3779B97F4A7C15ull;
@@ -169,10 +222,12 @@ RAP_HD uint64_t splitmix_H(uint64_t x) {
   return z ^ (z >> 31);
 }
 
-// Launch entry implemented in rap_kernel.cu.  Returns a cudaError_t value.
+// Launch entry implemented in rap_kernel.cu (cooperative launch: all CTAs
+// co-resident, so the look-back never waits on an unscheduled CTA).
+// Returns a cudaError_t value.
 int launch_fused(const Common& c, const LaunchRaw& raw, int grid, int smem_bytes, void* stream);
-// Dynamic shared memory the kernel needs for a dense tile of tile_bytes.
-int fused_smem_bytes(int tile_bytes);
+// Dynamic shared memory per CTA for dense groups up to max_width columns.
+int fused_smem_bytes(int max_width);
 // Occupancy query: CTAs per SM for the given dynamic smem.
 int fused_occupancy(int smem_bytes, int n_dense, int n_sparse, int* ctas_per_sm);
 

@@ -1,18 +1,25 @@
 // rap_kernel.cu — the fused, persistent sm_100a preprocessing kernel.
 //
-// One launch processes a whole raw batch (§6.1: horizontal
-// fusion of the per-feature kernels; here every op of every feature runs in a
-// single persistent kernel, so the chains are fused vertically as well and no
-// intermediate touches HBM).  CTAs pull (feature, row-range) descriptors from
-// an atomic ticket counter and copy the descriptor's flattened program
-// (rap_internal.h) into shared memory in one burst.  Sparse descriptors come
-// first, in feature-major order, and build the jagged offsets with a block
-// scan plus a decoupled look-back across descriptors.  The
-// look-back is deferred: a descriptor publishes its aggregate right after the
-// length pass, computes its ids into shared memory, and only then asks for
-// its prefix.  Dense descriptors transpose columnar input to the row-major
-// MLP input through shared memory.  The grid is capped by the SM budget
-// (§6.2).
+// One cooperative launch processes a whole raw batch (§6.1
+// L1161-1174: horizontal fusion of the per-feature kernels; here every op of
+// every feature runs in one persistent kernel, so the chains are fused
+// vertically as well and no intermediate touches HBM).  The jagged offsets
+// are a global exclusive scan over (feature, row) in feature-major order
+// (R17), so the launch runs in three phases separated by two self-resetting
+// grid barriers:
+//   phase 1  every warp computes the output lengths of 128-row sparse tiles
+//            (closed form from the Arrow offsets and validity words), writes
+//            them, and records one length sum per tile;
+//   phase 2  every CTA scans its chunk of tile sums;
+//   phase 3  CTAs take work units by ticket: a dense column-group block
+//            (inputs staged by cp.async.bulk onto an mbarrier, evaluated
+//            (row, unit)-parallel into a row-major smem tile, float4 stores),
+//            or 8 consecutive sparse tiles of one feature, one per warp, each
+//            writing its offsets and ids at positions known from phase 2.
+// Warps work on their own tiles without CTA barriers; loads of a tile are
+// issued together (4 row groups per lane) so each warp keeps several
+// independent memory requests in flight.  The grid is capped by the SM
+// budget (§6.2).
 //
 // Operator semantics: DESIGN.md §3 readings R1-R20 (Table 1).
 // Nothing here is tensor-core work: the path is integer ALU + a few SFU
@@ -38,13 +45,10 @@ struct KParams {
 };
 
 constexpr int kWarps = kThreads / 32;
+constexpr int kGroups = kTileRows / 32;  // row groups of a sparse tile (one row per lane each)
+constexpr int kMaxGrid = 2048;           // look-back words allocated by the plan
 
 __host__ __device__ constexpr int align_up(int x, int a) { return (x + a - 1) / a * a; }
-
-// Shared-memory carve-up.  Sparse and dense descriptors reuse the same bytes.
-constexpr int kSProgBytes = align_up((int)sizeof(SProg), 16);
-constexpr int kSparseSmem = kSProgBytes + 8 * kStageTab + 8 * kVBuf + 3 * 4 * kRowsSparseMax + 2 * 4 * kNgSlots;
-constexpr int kDProgBytes = align_up((int)sizeof(DProg), 16);
 
 // ----------------------------------------------------------------------------
 // Scalar helpers.
@@ -53,9 +57,56 @@ __device__ __forceinline__ uint64_t reduce_M(uint64_t h, int64_t M) {  // R2
   return __umul64hi(h, (uint64_t)M);
 }
 
-__device__ __forceinline__ uint32_t bitmap_word(const uint32_t* bm, int64_t r) {
-  return bm == nullptr ? 0xffffffffu : __ldg(bm + (r >> 5));
+__device__ __forceinline__ unsigned long long ld_acquire(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
 }
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+
+// Profiling aid: per-CTA phase stamps (%globaltimer), thread 0 only, enabled
+// when the plan allocated a trace buffer (rap_debug_trace).
+__device__ __forceinline__ void trace_stamp(const Common& c, int k) {
+  if (c.trace != nullptr && threadIdx.x == 0 && (int64_t)blockIdx.x < c.trace_cap) {
+    unsigned long long v;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(v));
+    c.trace[(int64_t)blockIdx.x * kTracePts + k] = v;
+  }
+}
+
+// ---- mbarrier + bulk async copies (TMA engine, non-tensor form) ----
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+
+__device__ __forceinline__ void mbar_arrive_expect(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n"
+      "RAP_WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra RAP_WAIT_%=;\n}" ::"r"(smem_u32(bar)),
+      "r"(phase)
+      : "memory");
+}
+
+// bytes: multiple of 16; dst, src: 16-byte aligned.
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   smem_u32(dst)),
+               "l"(src), "r"(bytes), "r"(smem_u32(bar))
+               : "memory");
+}
+
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 
 __device__ __forceinline__ unsigned long long ld_relaxed(const unsigned long long* p) {
   unsigned long long v;
@@ -67,192 +118,22 @@ __device__ __forceinline__ void st_relaxed(unsigned long long* p, unsigned long 
   asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
-// Upper bound = #{i : b[i] <= x} for sorted borders (R4; NaN -> 0).  Works on
-// shared or global memory (generic pointer).
-template <class T>
-__device__ __forceinline__ int64_t upper_bound(const T* b, int m, T x) {
-  int lo = 0, n = m;
-  while (n > 0) {
-    const int half = n >> 1;
-    if (b[lo + half] <= x) {
-      lo += half + 1;
-      n -= half + 1;
-    } else {
-      n = half;
-    }
-  }
-  return lo;
-}
-
-// MapId (R8) through an open-addressing table built by the planner:
-// 2^m slots of (key, value), empty key = INT64_MIN, Fibonacci hashing,
-// linear probing.  A real INT64_MIN key is carried in the op itself.
-__device__ __forceinline__ int64_t map_lookup(const DevOp& op, const int64_t* itab, int64_t x) {
-  if (x == INT64_MIN) return op.M ? (int64_t)op.hsalt : op.b;
-  const longlong2* t = reinterpret_cast<const longlong2*>(itab + op.a);
-  const uint32_t mask = (1u << op.m) - 1u;
-  uint32_t i = (uint32_t)(((uint64_t)x * 0x9E3779B97F4A7C15ull) >> (64 - op.m));
-  while (true) {
-    const longlong2 kv = __ldg(t + i);
-    if (kv.x == x) return kv.y;
-    if (kv.x == INT64_MIN) return op.b;
-    i = (i + 1) & mask;
-  }
-}
-
-__device__ __forceinline__ int64_t apply_id_ops(const DevOp* ops, const int64_t* itab, const int64_t* stab,
-                                                int64_t v, int o0, int o1) {
-  for (int o = o0; o < o1; ++o) {
-    const DevOp& op = ops[o];
-    switch (op.kind) {
-      case OK_CLAMP:  // R6
-        v = v < op.a ? op.a : v;
-        v = v > op.b ? op.b : v;
-        break;
-      case OK_SIGRID:  // R3: reduce(H(H(salt) ^ x), M)
-        v = (int64_t)reduce_M(splitmix_H(op.hsalt ^ (uint64_t)v), op.M);
-        break;
-      case OK_BUCKET_S:
-        v = upper_bound(stab + op.a, op.m, v);
-        break;
-      case OK_BUCKET_I:
-        v = upper_bound(itab + op.a, op.m, v);
-        break;
-      default:  // OK_MAPID
-        v = map_lookup(op, itab, v);
-        break;
-    }
-  }
-  return v;
-}
-
-// Dense ops (R10-R12) in f32.
-__device__ __forceinline__ float apply_dense_ops(const DevOp* ops, float x, int o0, int o1) {
-  for (int o = o0; o < o1; ++o) {
-    const DevOp& op = ops[o];
-    if (op.kind == OK_FILL_F) {
-      if (isnan(x)) x = op.f0;
-    } else if (op.kind == OK_LOGIT) {
-      const float z = x < op.f0 ? op.f0 : (x > op.f1 ? op.f1 : x);
-      x = logf(__fdiv_rn(z, __fsub_rn(1.0f, z)));
-    } else {  // OK_BOXCOX
-      const float lam = op.f0;
-      if (lam == 0.0f) {
-        x = logf(x);
-      } else {
-        const float u = __fmul_rn(lam, logf(x));
-        x = __fdiv_rn(expm1f(u), lam);
-      }
-    }
-  }
-  return x;
-}
-
-// Raw dense value with the R14 null rule (null slot -> NaN).
-template <class P>
-__device__ __forceinline__ float dense_raw(const P& p, int col, int64_t row) {
-  const uint32_t w = bitmap_word(p.dvalid[col], row);
-  const float x = __ldg(p.dense[col] + row);
-  return ((w >> (row & 31)) & 1u) ? x : __int_as_float(0x7fc00000);
-}
-
-// ----------------------------------------------------------------------------
-// Id-list chains.
-
-// Source list of a chain for one row: returns the output length and the first
-// child index (start >= 0), -1 for a filled null row, -2 for a dense bucket.
-template <class P>
-__device__ __forceinline__ int32_t leaf_len(const P& p, const Chain& ch, int64_t row, int32_t* start) {
-  if (ch.src_kind == SRC_SPARSE) {
-    const int s = ch.src;
-    const uint32_t w = bitmap_word(p.svalid[s], row);
-    const int32_t a = __ldg(p.off[s] + row), b = __ldg(p.off[s] + row + 1);
-    if ((w >> (row & 31)) & 1u) {
-      *start = a;
-      return (int32_t)min((int64_t)max(b - a, 0), ch.xcap);  // R5 FirstX as a cap
-    }
-    *start = -1;
-    return ch.has_fill ? (int32_t)min((int64_t)1, ch.null_xcap) : 0;  // R10 / R14
-  }
-  *start = -2;  // SRC_DENSE_BUCKET: always a length-1 list (R4)
-  return (int32_t)min((int64_t)1, ch.xcap);
-}
-
-template <class P>
-__device__ __forceinline__ int64_t leaf_value(const P& p, const DevOp* ops, const int64_t* stab, const Chain& ch,
-                                              int32_t start, int64_t row, int32_t j) {
-  if (start >= 0)
-    return apply_id_ops(ops, p.c.itab, stab, __ldg(p.val[ch.src] + start + j), ch.op_begin, ch.op_end);
-  if (start == -1) return apply_id_ops(ops, p.c.itab, stab, ch.fill, ch.null_op_begin, ch.op_end);
-  const float x = apply_dense_ops(ops, dense_raw(p, ch.src, row), ch.dop_begin, ch.dop_end);
-  return apply_id_ops(ops, p.c.itab, stab, upper_bound(p.c.ftab + ch.btab, ch.bm, x), ch.op_begin, ch.op_end);
-}
-
-__device__ __forceinline__ const DevOp* prog_ops(const SProg& pg, const DevOp* gops) {
-  return pg.global_ops ? gops : pg.ops;
-}
-
-// Whole-chain length / element for any source kind (NGram sources
-// recomputed from global memory), used by the OneHot generic unit.
-template <class P>
-__device__ int32_t chain_len_g(const P& p, const SProg& pg, int64_t row, int32_t* st, int32_t* sl) {
-  if (pg.ch.src_kind != SRC_NGRAM) return leaf_len(p, pg.ch, row, st);
-  int tot = 0;
-  for (int c = 0; c < pg.ng.k; ++c) {
-    sl[c] = leaf_len(p, pg.src[c], row, st + c);
-    tot += sl[c];
-  }
-  return (int32_t)min((int64_t)max(tot - pg.ng.n + 1, 0), pg.ch.xcap);
-}
-
-template <class P>
-__device__ int64_t ngram_window(const P& p, const SProg& pg, const DevOp* ops, const int64_t* stab, const int32_t* st,
-                                const int32_t* sl, int stride, int64_t row, int32_t j) {
-  // R7: h = H(salt); h = H(h ^ c[j+q]) for q < n; reduce(h, M)
-  const NGramDesc& ng = pg.ng;
-  uint64_t h = ng.hsalt;
-  int c = 0;
-  int32_t pos = j;
-  int32_t lc = sl[0];
-  for (int q = 0; q < ng.n; ++q) {
-    while (pos >= lc) {
-      pos -= lc;
-      ++c;
-      lc = sl[c * stride];
-    }
-    const int64_t e = leaf_value(p, ops, stab, pg.src[c], st[c * stride], row, pos);
-    h = splitmix_H(h ^ (uint64_t)e);
-    ++pos;
-  }
-  return apply_id_ops(ops, p.c.itab, stab, (int64_t)reduce_M(h, ng.M), pg.ch.op_begin, pg.ch.op_end);
-}
-
-template <class P>
-__device__ int64_t chain_elem_g(const P& p, const SProg& pg, const int64_t* stab, const int32_t* st,
-                                const int32_t* sl, int64_t row, int32_t j) {
-  const DevOp* ops = prog_ops(pg, p.c.ops);
-  if (pg.ch.src_kind != SRC_NGRAM) return leaf_value(p, ops, stab, pg.ch, st[0], row, j);
-  return ngram_window(p, pg, ops, stab, st, sl, 1, row, j);
-}
-
-// ----------------------------------------------------------------------------
 __device__ __forceinline__ long long warp_sum64(long long v) {
 #pragma unroll
   for (int d = 16; d >= 1; d >>= 1) v += __shfl_xor_sync(0xffffffffu, v, d);
   return v;
 }
 
-// Decoupled look-back (warp 0).  Each lane inspects 4 predecessor words, so
-// one round trip covers 128 descriptors.  Walking from the nearest
-// predecessor down, aggregates are summed until the first inclusive prefix;
-// only an unpublished word on that path makes the warp wait (the part before
-// it is banked).  Returns the exclusive prefix, publishes the inclusive one.
+// Decoupled look-back over the chunk totals of CTAs < slot (warp 0).  Each
+// lane inspects 4 predecessor words, so one round trip covers 128 chunks;
+// walking from the nearest predecessor down, totals are summed until the
+// first inclusive prefix, and only an unpublished word on that path makes the
+// warp wait.  Returns the exclusive prefix and publishes the inclusive one.
 __device__ long long lookback(unsigned long long* status, long long slot, long long agg, unsigned long long epoch,
                               int lane) {
   const unsigned long long tag = epoch << kEpochShift;
   long long excl = 0;
   long long top = slot - 1;
-  int spins = 0;
   while (top >= 0) {
     unsigned long long w[4];
     int flag[4];
@@ -288,303 +169,812 @@ __device__ long long lookback(unsigned long long* status, long long slot, long l
     }
     if (fkind == (int)kFlagPrefix) break;
     top -= 4 * fl + fq;  // wait on the first unpublished predecessor
-    if (++spins > 2) __nanosleep(32);
   }
   if (lane == 0) st_relaxed(status + slot, tag | (kFlagPrefix << kFlagShift) | (unsigned long long)(excl + agg));
   return excl;
 }
 
-// Warp-cooperative 16-byte copy global -> shared.
-__device__ __forceinline__ void warp_copy16(void* dst, const void* src, int bytes, int lane) {
-  const int4* s = reinterpret_cast<const int4*>(src);
-  int4* d = reinterpret_cast<int4*>(dst);
-  const int n = bytes >> 4;
-  for (int k = lane; k < n; k += 32) d[k] = __ldg(s + k);
+// Upper bound = #{i : b[i] <= x} for sorted borders (R4; NaN -> 0).
+template <class T>
+__device__ __forceinline__ int64_t upper_bound(const T* b, int m, T x) {
+  int lo = 0, n = m;
+  while (n > 0) {
+    const int half = n >> 1;
+    if (__ldg(b + lo + half) <= x) {
+      lo += half + 1;
+      n -= half + 1;
+    } else {
+      n = half;
+    }
+  }
+  return lo;
 }
 
-struct SparseSmem {
-  SProg* prog;
-  int64_t* tab;    // [kStageTab] staged Bucketize borders
-  int64_t* vals;   // [kVBuf] staged output ids
-  int32_t* len;    // [R] output length per row
-  int32_t* excl;   // [R] exclusive prefix within the descriptor
-  int32_t* start;  // [R] first child index (-1 filled null row, -2 computed)
-  int32_t* ngs;    // [kNgSlots] NGram: per (source, row) start
-  int32_t* ngl;    // [kNgSlots] NGram: per (source, row) length
+__device__ __forceinline__ int64_t upper_bound_s(const float* b, int m, float x) {  // shared-memory borders
+  int lo = 0, n = m;
+  while (n > 0) {
+    const int half = n >> 1;
+    if (b[lo + half] <= x) {
+      lo += half + 1;
+      n -= half + 1;
+    } else {
+      n = half;
+    }
+  }
+  return lo;
+}
+
+// MapId (R8) through an open-addressing table built by the planner:
+// 2^m slots of (key, value), empty key = INT64_MIN, Fibonacci hashing,
+// linear probing.  A real INT64_MIN key is carried in the op (M = 1, hsalt).
+__device__ __forceinline__ int64_t map_lookup(const int64_t* itab, int64_t a, int m, int64_t dflt, int has_min,
+                                              int64_t min_val, int64_t x) {
+  if (x == INT64_MIN) return has_min ? min_val : dflt;
+  const longlong2* t = reinterpret_cast<const longlong2*>(itab + a);
+  const uint32_t mask = (1u << m) - 1u;
+  uint32_t i = (uint32_t)(((uint64_t)x * 0x9E3779B97F4A7C15ull) >> (64 - m));
+  while (true) {
+    const longlong2 kv = __ldg(t + i);
+    if (kv.x == x) return kv.y;
+    if (kv.x == INT64_MIN) return dflt;
+    i = (i + 1) & mask;
+  }
+}
+
+// One id op; kind is warp-uniform, so this is a predicated if-chain.  The
+// staged-table form (OK_BUCKET_S) indexes the plan's int64 pool at tab_off.
+__device__ __forceinline__ int64_t apply_id_op(const DevOp& op, const int64_t* itab, int64_t tab_off, int64_t v) {
+  const int kind = op.kind;
+  if (kind == OK_SIGRID) return (int64_t)reduce_M(splitmix_H(op.hsalt ^ (uint64_t)v), op.M);  // R3
+  if (kind == OK_CLAMP) {                                                                       // R6
+    v = v < op.a ? op.a : v;
+    return v > op.b ? op.b : v;
+  }
+  if (kind == OK_BUCKET_S) return upper_bound(itab + tab_off + op.a, op.m, v);  // R4
+  if (kind == OK_BUCKET_I) return upper_bound(itab + op.a, op.m, v);
+  return map_lookup(itab, op.a, op.m, op.b, (int)op.M, (int64_t)op.hsalt, v);  // R8
+}
+
+__device__ __forceinline__ int64_t apply_id_ops(const DevOp* ops, const int64_t* itab, int64_t tab_off, int64_t v,
+                                                int o0, int o1) {
+  for (int o = o0; o < o1; ++o) v = apply_id_op(ops[o], itab, tab_off, v);
+  return v;
+}
+
+// Register-resident pipeline of up to kPipe id ops (loaded once per tile;
+// the ops are warp-uniform): per element the op itself plus a uniform branch.
+constexpr int kPipe = 3;
+struct Pipe {
+  int n;
+  int km[kPipe];  // kind | m << 8
+  int64_t p0[kPipe], p1[kPipe];
 };
 
-__device__ __forceinline__ SparseSmem carve_sparse(unsigned char* smem) {
-  SparseSmem s;
-  int o = 0;
-  s.prog = reinterpret_cast<SProg*>(smem + o);
-  o += kSProgBytes;
-  s.tab = reinterpret_cast<int64_t*>(smem + o);
-  o += 8 * kStageTab;
-  s.vals = reinterpret_cast<int64_t*>(smem + o);
-  o += 8 * kVBuf;
-  s.len = reinterpret_cast<int32_t*>(smem + o);
-  o += 4 * kRowsSparseMax;
-  s.excl = reinterpret_cast<int32_t*>(smem + o);
-  o += 4 * kRowsSparseMax;
-  s.start = reinterpret_cast<int32_t*>(smem + o);
-  o += 4 * kRowsSparseMax;
-  s.ngs = reinterpret_cast<int32_t*>(smem + o);
-  o += 4 * kNgSlots;
-  s.ngl = reinterpret_cast<int32_t*>(smem + o);
-  return s;
+__device__ __forceinline__ bool pipe_ok(const DevOp* ops, int o0, int o1) {
+  if (o1 - o0 > kPipe) return false;
+  for (int o = o0; o < o1; ++o)
+    if (ops[o].kind == OK_MAPID && ops[o].M) return false;
+  return true;
 }
 
-// Warp 0: feature of ticket t by a 32-ary search over desc_start (one round
-// trip for <= 32 features, two for <= 1024), then the program copy.
-template <class P>
-__device__ int locate_and_stage(const P& p, long long t, const SparseSmem& sm) {
-  const int lane = threadIdx.x & 31;
-  int lo = 0, hi = p.c.n_sparse_out;
-  while (hi - lo > 1) {
-    const int step = (hi - lo + 31) >> 5;
-    const int idx = lo + lane * step;
-    const bool ok = idx < hi && __ldg(p.c.desc_start + idx) <= t;
-    const unsigned m = __ballot_sync(0xffffffffu, ok);
-    const int k = 31 - __clz(m);
-    lo += k * step;
-    hi = min(hi, lo + step);
-  }
-  const int f = lo;
-  const SProg* g = p.c.sprogs + f;
-  warp_copy16(sm.prog, g, kSProgBytes, lane);
-  __syncwarp();
-  const int tl = sm.prog->tab_len;
-  if (tl > 0) warp_copy16(sm.tab, p.c.itab + sm.prog->tab_off, align_up(8 * tl, 16), lane);
-  return f;
-}
-
-// Value of output element j of local row i.
-template <class P>
-__device__ __forceinline__ int64_t sparse_value(const P& p, const SProg& pg, const DevOp* ops, const SparseSmem& sm,
-                                                int R, int64_t r0, int i, int32_t j) {
-  if (pg.ch.src_kind != SRC_NGRAM) return leaf_value(p, ops, sm.tab, pg.ch, sm.start[i], r0 + i, j);
-  return ngram_window(p, pg, ops, sm.tab, sm.ngs + i, sm.ngl + i, R, r0 + i, j);
-}
-
-// Elements of a descriptor, one warp per 32-row group, emitted into shared
-// memory or straight to the output (dst already offset by the base).
-template <class P>
-__device__ void emit_values(const P& p, const SProg& pg, const DevOp* ops, const SparseSmem& sm, int R, int64_t r0,
-                            int nr, int64_t* dst, long long dst_limit) {
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const int ngroups = (nr + 31) / 32;
-  for (int g = warp; g < ngroups; g += kWarps) {
-    const int i = g * 32 + lane;
-    const bool has = i < nr;
-    const int len = has ? sm.len[i] : 0;
-    const int ex = has ? sm.excl[i] : 0;
-    const int gbase = __shfl_sync(0xffffffffu, ex, 0);
-    const int lastlane = min(31, nr - 1 - g * 32);
-    int lex = ex - gbase;
-    const int T = __shfl_sync(0xffffffffu, lex + len, lastlane);
-    if (!has) lex = INT_MAX;
-    int64_t* out = dst + gbase;
-    const long long lim = dst_limit - gbase;
-    if (__all_sync(0xffffffffu, !has || len == 1)) {
-      if (has && lane < lim) out[lane] = sparse_value(p, pg, ops, sm, R, r0, i, 0);
-      continue;
+__device__ __forceinline__ void load_pipe(Pipe& pp, const DevOp* ops, int o0, int o1, int64_t tab_off) {
+  pp.n = o1 - o0;
+#pragma unroll
+  for (int k = 0; k < kPipe; ++k) {
+    pp.km[k] = -1;
+    pp.p0[k] = pp.p1[k] = 0;
+    if (k < pp.n) {
+      const DevOp& op = ops[o0 + k];
+      pp.km[k] = op.kind | (op.m << 8);
+      if (op.kind == OK_SIGRID) {
+        pp.p0[k] = (int64_t)op.hsalt;
+        pp.p1[k] = op.M;
+      } else {
+        pp.p0[k] = op.kind == OK_BUCKET_S ? tab_off + op.a : op.a;
+        pp.p1[k] = op.b;
+      }
     }
+  }
+}
+
+__device__ __forceinline__ int64_t run_pipe(const Pipe& pp, const int64_t* itab, int64_t v, int k0) {
+#pragma unroll
+  for (int k = 0; k < kPipe; ++k) {
+    if (k >= k0 && k < pp.n) {
+      const int kind = pp.km[k] & 0xff, m = pp.km[k] >> 8;
+      if (kind == OK_SIGRID) {
+        v = (int64_t)reduce_M(splitmix_H((uint64_t)pp.p0[k] ^ (uint64_t)v), pp.p1[k]);
+      } else if (kind == OK_CLAMP) {
+        v = v < pp.p0[k] ? pp.p0[k] : v;
+        v = v > pp.p1[k] ? pp.p1[k] : v;
+      } else if (kind == OK_MAPID) {
+        v = map_lookup(itab, pp.p0[k], m, pp.p1[k], 0, 0, v);
+      } else {  // OK_BUCKET_S / OK_BUCKET_I: p0 = absolute itab offset
+        v = upper_bound(itab + pp.p0[k], m, v);
+      }
+    }
+  }
+  return v;
+}
+
+// Canonical pipeline (rap_internal.h): the stages present in MASK, in the
+// fixed order Clamp -> MapId -> SigridHash -> Bucketize; `active` selects the
+// stages of this element (all for a valid row, null_mask for a filled row).
+template <int MASK>
+__device__ __forceinline__ int64_t canon_apply(const Canon& q, const int64_t* itab, int64_t v, int active) {
+  if ((MASK & CB_CLAMP) && (active & CB_CLAMP)) {  // R6
+    v = v < q.lo ? q.lo : v;
+    v = v > q.hi ? q.hi : v;
+  }
+  if ((MASK & CB_MAPID) && (active & CB_MAPID)) v = map_lookup(itab, q.map_a, q.map_m, q.map_def, 0, 0, v);  // R8
+  if ((MASK & CB_SIGRID) && (active & CB_SIGRID))
+    v = (int64_t)reduce_M(splitmix_H(q.hs ^ (uint64_t)v), q.M);                    // R3
+  if ((MASK & CB_BUCKET) && (active & CB_BUCKET)) v = upper_bound(itab + q.bk_a, q.bk_m, v);  // R4
+  return v;
+}
+
+// Calls body.template operator()<MASK>() for the runtime mask (16 cases).
+#define RAP_CANON_DISPATCH(mask, CALL)   \
+  switch ((mask) & 15) {                 \
+    case 0: CALL(0); break;              \
+    case 1: CALL(1); break;              \
+    case 2: CALL(2); break;              \
+    case 3: CALL(3); break;              \
+    case 4: CALL(4); break;              \
+    case 5: CALL(5); break;              \
+    case 6: CALL(6); break;              \
+    case 7: CALL(7); break;              \
+    case 8: CALL(8); break;              \
+    case 9: CALL(9); break;              \
+    case 10: CALL(10); break;            \
+    case 11: CALL(11); break;            \
+    case 12: CALL(12); break;            \
+    case 13: CALL(13); break;            \
+    case 14: CALL(14); break;            \
+    default: CALL(15); break;            \
+  }
+
+// Dense ops (R10-R12) in f32.
+__device__ __forceinline__ float apply_dense_ops(const DevOp* ops, float x, int o0, int o1) {
+  for (int o = o0; o < o1; ++o) {
+    const DevOp& op = ops[o];
+    if (op.kind == OK_FILL_F) {
+      if (isnan(x)) x = op.f0;
+    } else if (op.kind == OK_LOGIT) {
+      const float z = x < op.f0 ? op.f0 : (x > op.f1 ? op.f1 : x);
+      x = logf(__fdiv_rn(z, __fsub_rn(1.0f, z)));
+    } else {  // OK_BOXCOX
+      const float lam = op.f0;
+      if (lam == 0.0f) {
+        x = logf(x);
+      } else {
+        const float u = __fmul_rn(lam, logf(x));
+        x = __fdiv_rn(expm1f(u), lam);
+      }
+    }
+  }
+  return x;
+}
+
+// Raw dense value from global memory with the R14 null rule (null -> NaN).
+template <class P>
+__device__ __forceinline__ float dense_raw(const P& p, int col, int64_t row) {
+  const uint32_t* bm = p.dvalid[col];
+  const uint32_t w = bm == nullptr ? 0xffffffffu : __ldg(bm + (row >> 5));
+  const float x = __ldg(p.dense[col] + row);
+  return ((w >> (row & 31)) & 1u) ? x : __int_as_float(0x7fc00000);
+}
+
+// ----------------------------------------------------------------------------
+// Id-list sources.  For one row: the output length of a chain and the first
+// child index (start >= 0), -1 for a filled null row (R10), -2 for a dense
+// bucket (computed from the dense column).
+
+struct RowIn {  // raw row data of one SRC_SPARSE source
+  int32_t a, b;
+  uint32_t w;  // validity word of the row's 32-row group
+};
+
+template <class P>
+__device__ __forceinline__ RowIn load_row(const P& p, const Chain& ch, int64_t row, bool in) {
+  RowIn r{0, 0, 0u};
+  if (in && ch.src_kind == SRC_SPARSE) {
+    const int32_t* off = p.off[ch.src];
+    const uint32_t* bm = p.svalid[ch.src];
+    r.a = __ldg(off + row);
+    r.b = __ldg(off + row + 1);
+    r.w = bm == nullptr ? 0xffffffffu : __ldg(bm + (row >> 5));
+  }
+  return r;
+}
+
+__device__ __forceinline__ int32_t row_len(const Chain& ch, const RowIn& r, int lane, bool in, int32_t* start) {
+  if (!in) {
+    *start = -1;
+    return 0;
+  }
+  if (ch.src_kind != SRC_SPARSE) {
+    *start = -2;  // SRC_DENSE_BUCKET: a length-1 list (R4)
+    return (int32_t)min((int64_t)1, ch.xcap);
+  }
+  if ((r.w >> lane) & 1u) {
+    *start = r.a;
+    return (int32_t)min((int64_t)max(r.b - r.a, 0), ch.xcap);  // R5 FirstX as a cap
+  }
+  *start = -1;
+  return ch.has_fill ? (int32_t)min((int64_t)1, ch.null_xcap) : 0;  // R10 / R14
+}
+
+// Element j of a source list (generic interpreter path).
+template <class P>
+__device__ __forceinline__ int64_t src_value(const P& p, const DevOp* ops, int64_t tab_off, const Chain& ch,
+                                             int32_t start, int64_t row, int32_t j) {
+  if (start >= 0) return apply_id_ops(ops, p.c.itab, tab_off, __ldg(p.val[ch.src] + start + j), ch.op_begin, ch.op_end);
+  if (start == -1) return apply_id_ops(ops, p.c.itab, tab_off, ch.fill, ch.null_op_begin, ch.op_end);
+  const float x = apply_dense_ops(ops, dense_raw(p, ch.src, row), ch.dop_begin, ch.dop_end);
+  return apply_id_ops(ops, p.c.itab, tab_off, upper_bound(p.c.ftab + ch.btab, ch.bm, x), ch.op_begin, ch.op_end);
+}
+
+__device__ __forceinline__ const DevOp* prog_ops(const SProg& pg, const DevOp* gops) {
+  return pg.global_ops ? gops : pg.ops;
+}
+
+// NGram window j (R7): h = H(salt); h = H(h ^ c[j+q]) for q < n; then the
+// chain's post ops on reduce(h, M).  st[c * stride] / sl[c * stride]:
+// per-source start / length of the row.
+template <class P>
+__device__ __noinline__ int64_t ngram_window(const P& p, const SProg& pg, const DevOp* ops, const int32_t* st,
+                                             const int32_t* sl, int stride, int64_t row, int32_t j) {
+  const int n = pg.ng.n;
+  uint64_t h = pg.ng.hsalt;
+  int c = 0;
+  int32_t pos = j;
+  for (int q = 0; q < n; ++q) {
+    while (pos >= sl[c * stride]) {
+      pos -= sl[c * stride];
+      ++c;
+    }
+    const int64_t e = src_value(p, ops, pg.tab_off, pg.src[c], st[c * stride], row, pos);
+    h = splitmix_H(h ^ (uint64_t)e);
+    ++pos;
+  }
+  return apply_id_ops(ops, p.c.itab, pg.tab_off, (int64_t)reduce_M(h, pg.ng.M), pg.ch.op_begin, pg.ch.op_end);
+}
+
+__device__ __forceinline__ int warp_incl_scan(int v, int lane) {
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const int y = __shfl_up_sync(0xffffffffu, v, d);
+    if (lane >= d) v += y;
+  }
+  return v;
+}
+
+// ----------------------------------------------------------------------------
+// Phase 1: output lengths of sparse tile (f, rt) -> lengths[], tile_sum[].
+template <class P>
+__device__ void length_tile(const P& p, int f, int64_t rt, int lane) {
+  const SProg& pg = p.c.sprogs[f];
+  const int64_t B = p.c.n_rows;
+  const int64_t r0 = rt * kTileRows;
+  int32_t* lengths = p.c.lengths + (int64_t)f * B;
+  int sum = 0;
+  if (pg.ch.src_kind != SRC_NGRAM) {
+    const Chain ch = pg.ch;
+    RowIn in[kGroups];
+#pragma unroll
+    for (int g = 0; g < kGroups; ++g) {
+      const int64_t row = r0 + 32 * g + lane;
+      in[g] = load_row(p, ch, row, row < B);
+    }
+#pragma unroll
+    for (int g = 0; g < kGroups; ++g) {
+      const int64_t row = r0 + 32 * g + lane;
+      int32_t st;
+      const int32_t len = row_len(ch, in[g], lane, row < B, &st);
+      if (row < B) lengths[row] = len;
+      sum += len;
+    }
+  } else {
+    const int k = pg.ng.k, n = pg.ng.n;
+    const int64_t xcap = pg.ch.xcap;
+    for (int g = 0; g < kGroups; ++g) {
+      const int64_t row = r0 + 32 * g + lane;
+      const bool inr = row < B;
+      RowIn in[kMaxNgramK];
+#pragma unroll
+      for (int c = 0; c < kMaxNgramK; ++c)
+        if (c < k) in[c] = load_row(p, pg.src[c], row, inr);
+      int tot = 0;
+#pragma unroll
+      for (int c = 0; c < kMaxNgramK; ++c) {
+        if (c < k) {
+          int32_t st;
+          tot += row_len(pg.src[c], in[c], lane, inr, &st);
+        }
+      }
+      const int32_t len = inr ? (int32_t)min((int64_t)max(tot - n + 1, 0), xcap) : 0;
+      if (inr) lengths[row] = len;
+      sum += len;
+    }
+  }
+#pragma unroll
+  for (int d = 16; d >= 1; d >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, d);
+  if (lane == 0) p.c.tile_sum[(int64_t)f * p.c.tiles_per_feature + rt] = sum;
+}
+
+// ----------------------------------------------------------------------------
+// Phase 3: offsets and ids of sparse tile (f, rt), whose first output id goes
+// to values[base].
+template <class P>
+__device__ __noinline__ void value_group_general(const P& p, int f, int64_t row0, int lane, int32_t mylen,
+                                                 int32_t myst, int32_t lx, long long gbase);
+template <class P>
+__device__ __noinline__ void value_tile_ngram(const P& p, int f, int64_t rt, int lane, long long base,
+                                              int32_t* scr);
+
+// Specialised tile of a canonical SRC_SPARSE chain (mask MASK).
+template <int MASK, class P>
+__device__ __noinline__ void value_tile_canon(const P& p, int f, int64_t rt, int lane, long long base) {
+  const SProg& pg = p.c.sprogs[f];
+  const Canon q = pg.cn;
+  const int src = pg.ch.src;
+  const int has_fill = pg.ch.has_fill;
+  const int64_t xcap = pg.ch.xcap, null_xcap = pg.ch.null_xcap, fill = pg.ch.fill;
+  const int64_t B = p.c.n_rows;
+  const int64_t r0 = rt * kTileRows;
+  int64_t* offsets = p.c.offsets + (int64_t)f * B;
+  int64_t* values = p.c.values;
+  const long long cap = p.c.values_cap;
+  const int64_t* itab = p.c.itab;
+  const int32_t* off = p.off[src];
+  const uint32_t* bm = p.svalid[src];
+  const int64_t* val = p.val[src];
+  int32_t a[kGroups], b[kGroups];
+  uint32_t w[kGroups];
+#pragma unroll
+  for (int g = 0; g < kGroups; ++g) {  // all row loads of the tile first
+    const int64_t row = r0 + 32 * g + lane;
+    const bool in = row < B;
+    a[g] = in ? __ldg(off + row) : 0;
+    b[g] = in ? __ldg(off + row + 1) : 0;
+    w[g] = (in && bm) ? __ldg(bm + (row >> 5)) : 0xffffffffu;
+  }
+  int32_t len[kGroups], lex[kGroups];
+  long long gb[kGroups];
+  bool valid[kGroups];
+  bool all1 = true;
+  long long run = base;
+#pragma unroll
+  for (int g = 0; g < kGroups; ++g) {
+    const int64_t row = r0 + 32 * g + lane;
+    valid[g] = (w[g] >> lane) & 1u;
+    int32_t l = valid[g] ? (int32_t)min((int64_t)max(b[g] - a[g], 0), xcap)
+                         : (has_fill ? (int32_t)min((int64_t)1, null_xcap) : 0);  // R5, R10, R14
+    if (row >= B) l = 0;
+    len[g] = l;
+    all1 &= l <= 1;
+    const int incl = warp_incl_scan(l, lane);
+    lex[g] = incl - l;
+    gb[g] = run;
+    run += __shfl_sync(0xffffffffu, incl, 31);
+    if (row < B) offsets[row] = gb[g] + lex[g];
+  }
+  if (f == p.c.n_sparse_out - 1 && rt == p.c.tiles_per_feature - 1 && lane == 0) {
+    p.c.offsets[(int64_t)p.c.n_sparse_out * B] = run;  // total, R17
+    if (run > cap) atomicExch(p.c.err, 1);
+  }
+  if (__all_sync(0xffffffffu, all1)) {
+    // at most one id per row: every lane owns its rows' output slots
+    int64_t raw[kGroups];
+#pragma unroll
+    for (int g = 0; g < kGroups; ++g) raw[g] = (len[g] == 1 && valid[g]) ? __ldg(val + a[g]) : fill;
+#pragma unroll
+    for (int g = 0; g < kGroups; ++g) {
+      if (len[g] == 1) {
+        const int64_t v = canon_apply<MASK>(q, itab, raw[g], valid[g] ? 15 : q.null_mask);
+        const long long pos = gb[g] + lex[g];
+        if (pos < cap) values[pos] = v;
+      }
+    }
+    return;
+  }
+  // multi-id rows: elements in output order, the owning row found by a
+  // 5-step shuffle search over the lanes' exclusive prefixes
+#pragma unroll 1
+  for (int g = 0; g < kGroups; ++g) {
+    const int T = __shfl_sync(0xffffffffu, lex[g] + len[g], 31);
+    const int mylex = (r0 + 32 * g + lane < B) ? lex[g] : INT_MAX;
+    const int32_t mystart = valid[g] ? a[g] : -1;
     for (int eb = 0; eb < T; eb += 32) {
       const int e = eb + lane;
       int r = 0;
 #pragma unroll
       for (int step = 16; step >= 1; step >>= 1) {
-        const int c = __shfl_sync(0xffffffffu, lex, r + step);
+        const int c = __shfl_sync(0xffffffffu, mylex, r + step);
         if (c <= e) r += step;
       }
-      const int lex_r = __shfl_sync(0xffffffffu, lex, r);
-      if (e < T && e < lim) out[e] = sparse_value(p, pg, ops, sm, R, r0, g * 32 + r, e - lex_r);
+      const int lex_r = __shfl_sync(0xffffffffu, mylex, r);
+      const int32_t st_r = __shfl_sync(0xffffffffu, mystart, r);
+      if (e < T) {
+        const int64_t x = st_r >= 0 ? __ldg(val + st_r + (e - lex_r)) : fill;
+        const int64_t v = canon_apply<MASK>(q, itab, x, st_r >= 0 ? 15 : q.null_mask);
+        const long long pos = gb[g] + e;
+        if (pos < cap) values[pos] = v;
+      }
     }
   }
 }
 
-// ----------------------------------------------------------------------------
-// Sparse descriptor: (output feature f, rows [r0, r0+nr)).
 template <class P>
-__device__ void sparse_desc(const P& p, long long t, unsigned long long epoch, unsigned char* smem, long long* s_warp,
-                            long long* s_bcast, int* s_f) {
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const SparseSmem sm = carve_sparse(smem);
-  if (warp == 0) {
-    const int f = locate_and_stage(p, t, sm);
-    if (lane == 0) *s_f = f;
-  }
-  __syncthreads();
-  const int f = *s_f;
-  const SProg& pg = *sm.prog;
+__device__ void value_tile(const P& p, int f, int64_t rt, int lane, long long base, int32_t* scr) {
+  const SProg& pg = p.c.sprogs[f];
   const DevOp* ops = prog_ops(pg, p.c.ops);
-  const int R = __ldg(p.c.rows_per_desc + f);
   const int64_t B = p.c.n_rows;
-  const int64_t r0 = (t - __ldg(p.c.desc_start + f)) * (int64_t)R;
-  const int nr = (int)min((int64_t)R, B - r0);
-
-  // Phase A: closed-form output length of every row (a3).  Each thread owns
-  // `per` consecutive rows; all loads of a row are issued together.
-  const int per = (R + kThreads - 1) / kThreads;
-  const int i0 = tid * per;
-  int local = 0;
-  if (pg.ch.src_kind != SRC_NGRAM) {
-#pragma unroll 4
-    for (int k = 0; k < per; ++k) {
-      const int i = i0 + k;
-      if (i < nr) {
-        int32_t st;
-        const int32_t len = leaf_len(p, pg.ch, r0 + i, &st);
-        sm.len[i] = len;
-        sm.start[i] = st;
-        local += len;
-      }
-    }
-  } else {
-    for (int k = 0; k < per; ++k) {
-      const int i = i0 + k;
-      if (i < nr) {
-        int tot = 0;
-#pragma unroll 4
-        for (int c = 0; c < pg.ng.k; ++c) {
-          int32_t st;
-          const int32_t lc = leaf_len(p, pg.src[c], r0 + i, &st);
-          sm.ngs[c * R + i] = st;
-          sm.ngl[c * R + i] = lc;
-          tot += lc;
-        }
-        const int32_t len = (int32_t)min((int64_t)max(tot - pg.ng.n + 1, 0), pg.ch.xcap);
-        sm.len[i] = len;
-        local += len;
-      }
-    }
-  }
-  // Phase B: block exclusive scan (warp shuffle + smem); aggregate published early.
-  int incl = local;
-#pragma unroll
-  for (int d = 1; d < 32; d <<= 1) {
-    const int y = __shfl_up_sync(0xffffffffu, incl, d);
-    if (lane >= d) incl += y;
-  }
-  if (lane == 31) s_warp[warp] = incl;
-  __syncthreads();
-  if (warp == 0) {
-    const long long w = lane < kWarps ? s_warp[lane] : 0;
-    long long wi = w;
-#pragma unroll
-    for (int d = 1; d < kWarps; d <<= 1) {
-      const long long y = __shfl_up_sync(0xffffffffu, wi, d);
-      if (lane >= d) wi += y;
-    }
-    const long long agg = __shfl_sync(0xffffffffu, wi, kWarps - 1);
-    if (lane < kWarps) s_warp[lane] = wi - w;
-    if (lane == 0) {
-      s_bcast[1] = agg;
-      const unsigned long long tag = epoch << kEpochShift;
-      st_relaxed(p.c.status + t, tag | ((t == 0 ? kFlagPrefix : kFlagAgg) << kFlagShift) | (unsigned long long)agg);
-    }
-  }
-  __syncthreads();
-  {
-    int run = (int)s_warp[warp] + incl - local;
-    for (int k = 0; k < per; ++k) {
-      const int i = i0 + k;
-      if (i < nr) {
-        sm.excl[i] = run;
-        run += sm.len[i];
-      }
-    }
-  }
-  const long long agg = s_bcast[1];
-  __syncthreads();
-
-  const bool staged = agg <= kVBuf;
-  if (staged) {
-    // Phase E (ids into shared memory) while predecessors resolve their prefixes.
-    emit_values(p, pg, ops, sm, R, r0, nr, sm.vals, LLONG_MAX);
-  }
-  // Phase C: decoupled look-back (slot = ticket).
-  if (warp == 0) {
-    const long long excl = t == 0 ? 0 : lookback(p.c.status, t, agg, epoch, lane);
-    if (lane == 0) s_bcast[0] = excl;
-  }
-  __syncthreads();
-  const long long base = s_bcast[0];
-
-  // Phase D: lengths / offsets (feature-major, R17), then the ids.
-  const int64_t fB = (int64_t)f * B + r0;
-  for (int i = tid; i < nr; i += kThreads) {
-    p.c.lengths[fB + i] = sm.len[i];
-    p.c.offsets[fB + i] = base + sm.excl[i];
-  }
-  if (tid == 0) {
-    if (t == p.c.n_sparse_desc - 1) p.c.offsets[(int64_t)p.c.n_sparse_out * B] = base + agg;
-    if (base + agg > p.c.values_cap) atomicExch(p.c.err, 1);
-  }
+  const int64_t r0 = rt * kTileRows;
+  int64_t* offsets = p.c.offsets + (int64_t)f * B;
+  int64_t* values = p.c.values;
   const long long cap = p.c.values_cap;
-  if (staged) {
-    int64_t* out = p.c.values + base;
-    const int lim = (int)min(agg, cap - base);
-    for (int k = tid; k < lim; k += kThreads) out[k] = sm.vals[k];
-  } else {
-    emit_values(p, pg, ops, sm, R, r0, nr, p.c.values + base, cap - base);
+  const int64_t* itab = p.c.itab;
+
+  const int canon = __ldg(&pg.cn.ok) && __ldg(&pg.ch.src_kind) == SRC_SPARSE;
+  if (canon) {
+    const int mask = __ldg(&pg.cn.mask);
+#define RAP_VT_CALL(M) value_tile_canon<M>(p, f, rt, lane, base)
+    RAP_CANON_DISPATCH(mask, RAP_VT_CALL)
+#undef RAP_VT_CALL
+    return;
+  }
+  if (pg.ch.src_kind != SRC_NGRAM) {
+    const Chain ch = pg.ch;
+    // all row loads of the tile first (kGroups independent requests per lane)
+    RowIn in[kGroups];
+#pragma unroll
+    for (int g = 0; g < kGroups; ++g) {
+      const int64_t row = r0 + 32 * g + lane;
+      in[g] = load_row(p, ch, row, row < B);
+    }
+    int32_t len[kGroups], st[kGroups], lex[kGroups];
+    long long gb[kGroups];
+    bool all1 = true;
+    long long run = base;
+#pragma unroll
+    for (int g = 0; g < kGroups; ++g) {
+      const int64_t row = r0 + 32 * g + lane;
+      len[g] = row_len(ch, in[g], lane, row < B, &st[g]);
+      all1 &= len[g] <= 1;
+      const int incl = warp_incl_scan(len[g], lane);
+      lex[g] = incl - len[g];
+      gb[g] = run;
+      run += __shfl_sync(0xffffffffu, incl, 31);
+      if (row < B) offsets[row] = gb[g] + lex[g];
+    }
+    if (f == p.c.n_sparse_out - 1 && rt == p.c.tiles_per_feature - 1 && lane == 0) {
+      p.c.offsets[(int64_t)p.c.n_sparse_out * B] = run;  // total, R17
+      if (run > cap) atomicExch(p.c.err, 1);
+    }
+    const bool use_pipe = ch.src_kind == SRC_SPARSE && pipe_ok(ops, ch.op_begin, ch.op_end);
+    Pipe pipe;
+    if (use_pipe) load_pipe(pipe, ops, ch.op_begin, ch.op_end, pg.tab_off);
+    const int null_k0 = ch.null_op_begin - ch.op_begin;
+    if (__all_sync(0xffffffffu, all1)) {
+      // one id per row at most: every lane owns its rows' output slots
+      int64_t raw[kGroups];
+#pragma unroll
+      for (int g = 0; g < kGroups; ++g)
+        raw[g] = (len[g] == 1 && st[g] >= 0) ? __ldg(p.val[ch.src] + st[g]) : ch.fill;
+#pragma unroll
+      for (int g = 0; g < kGroups; ++g) {
+        if (len[g] == 1) {
+          const int64_t row = r0 + 32 * g + lane;
+          int64_t v;
+          if (use_pipe) {
+            v = run_pipe(pipe, itab, raw[g], st[g] >= 0 ? 0 : null_k0);
+          } else {
+            v = src_value(p, ops, pg.tab_off, ch, st[g], row, 0);
+          }
+          const long long pos = gb[g] + lex[g];
+          if (pos < cap) values[pos] = v;
+        }
+      }
+      return;
+    }
+    // general (multi-id rows): elements in output order, per row group
+#pragma unroll 1
+    for (int g = 0; g < kGroups; ++g) value_group_general(p, f, r0 + 32 * g, lane, len[g], st[g], lex[g], gb[g]);
+    return;
+  }
+  value_tile_ngram(p, f, rt, lane, base, scr);
+}
+
+// Ids of one 32-row group with multi-id rows: elements in output order, the
+// owning row found by a 5-step shuffle search over the lanes' exclusive prefixes.
+template <class P>
+__device__ __noinline__ void value_group_general(const P& p, int f, int64_t row0, int lane, int32_t mylen,
+                                                 int32_t myst, int32_t lx, long long gbase) {
+  const SProg& pg = p.c.sprogs[f];
+  const DevOp* ops = prog_ops(pg, p.c.ops);
+  const Chain& ch = pg.ch;
+  const long long cap = p.c.values_cap;
+  const bool use_pipe = ch.src_kind == SRC_SPARSE && pipe_ok(ops, ch.op_begin, ch.op_end);
+  Pipe pipe;
+  if (use_pipe) load_pipe(pipe, ops, ch.op_begin, ch.op_end, pg.tab_off);
+  const int null_k0 = ch.null_op_begin - ch.op_begin;
+  const int T = __shfl_sync(0xffffffffu, lx + mylen, 31);
+  const int mylex = (row0 + lane < p.c.n_rows) ? lx : INT_MAX;
+  for (int eb = 0; eb < T; eb += 32) {
+    const int e = eb + lane;
+    int r = 0;
+#pragma unroll
+    for (int step = 16; step >= 1; step >>= 1) {
+      const int c = __shfl_sync(0xffffffffu, mylex, r + step);
+      if (c <= e) r += step;
+    }
+    const int lex_r = __shfl_sync(0xffffffffu, mylex, r);
+    const int32_t st_r = __shfl_sync(0xffffffffu, myst, r);
+    if (e < T) {
+      const int32_t j = e - lex_r;
+      int64_t v;
+      if (use_pipe) {
+        const int64_t x = st_r >= 0 ? __ldg(p.val[ch.src] + st_r + j) : ch.fill;
+        v = run_pipe(pipe, p.c.itab, x, st_r >= 0 ? 0 : null_k0);
+      } else {
+        v = src_value(p, ops, pg.tab_off, ch, st_r, row0 + r, j);
+      }
+      const long long pos = gbase + e;
+      if (pos < cap) p.c.values[pos] = v;
+    }
+  }
+}
+
+// NGram feature tile (R7): per row the k source lists, windows over their
+// concatenation.
+template <class P>
+__device__ __noinline__ void value_tile_ngram(const P& p, int f, int64_t rt, int lane, long long base,
+                                              int32_t* scr) {
+  const SProg& pg = p.c.sprogs[f];
+  const DevOp* ops = prog_ops(pg, p.c.ops);
+  const int64_t B = p.c.n_rows;
+  const int64_t r0 = rt * kTileRows;
+  int64_t* offsets = p.c.offsets + (int64_t)f * B;
+  int64_t* values = p.c.values;
+  const long long cap = p.c.values_cap;
+
+  // NGram feature (R7): per row the k source lists, windows over their
+  // concatenation.  Per-source (start, length) of the warp's 32 rows live in
+  // warp-private shared memory: scr[c*32 + lane] / scr[(kMaxNgramK + c)*32 + lane].
+  const int k = pg.ng.k, n = pg.ng.n;
+  const int64_t xcap = pg.ch.xcap;
+  int32_t* st_s = scr;
+  int32_t* sl_s = scr + kMaxNgramK * 32;
+  int64_t* ev_s = reinterpret_cast<int64_t*>(scr + 2 * kMaxNgramK * 32);  // [c][lane] element ids
+  const int64_t* itab = p.c.itab;
+  // canonical fast path: every source (and the post-hash ops) canonical
+  bool canon_all = pg.cn.ok;
+  for (int c = 0; c < k; ++c) canon_all &= pg.src_cn[c].ok != 0;
+  long long run = base;
+#pragma unroll 1
+  for (int g = 0; g < kGroups; ++g) {
+    const int64_t row = r0 + 32 * g + lane;
+    const bool inr = row < B;
+    RowIn in[kMaxNgramK];
+#pragma unroll
+    for (int c = 0; c < kMaxNgramK; ++c)
+      if (c < k) in[c] = load_row(p, pg.src[c], row, inr);
+    int tot = 0, slmax = 0;
+#pragma unroll
+    for (int c = 0; c < kMaxNgramK; ++c) {
+      if (c < k) {
+        int32_t st;
+        const int32_t sl = row_len(pg.src[c], in[c], lane, inr, &st);
+        st_s[c * 32 + lane] = st;
+        sl_s[c * 32 + lane] = sl;
+        tot += sl;
+        slmax = max(slmax, sl);
+        if (canon_all) ev_s[c * 32 + lane] = (sl >= 1 && st >= 0) ? __ldg(p.val[pg.src[c].src] + st) : pg.src[c].fill;
+      }
+    }
+    __syncwarp();
+    const int32_t len = inr ? (int32_t)min((int64_t)max(tot - n + 1, 0), xcap) : 0;
+    const int incl = warp_incl_scan(len, lane);
+    const int lx = incl - len;
+    const int T = __shfl_sync(0xffffffffu, incl, 31);
+    if (inr) offsets[row] = run + lx;
+    if (canon_all && __all_sync(0xffffffffu, slmax <= 1)) {
+      // single-id sources: run each source's canonical pipeline once per row,
+      // then hash the windows from the staged ids
+      unsigned present = 0;
+      for (int c = 0; c < k; ++c) {
+        const Canon qc = pg.src_cn[c];
+        const int sl = sl_s[c * 32 + lane];
+        if (sl == 1) {
+          present |= 1u << c;
+          const int act = st_s[c * 32 + lane] >= 0 ? 15 : qc.null_mask;
+          int64_t x = ev_s[c * 32 + lane];
+#define RAP_NG_CALL(M) x = canon_apply<M>(qc, itab, x, act)
+          RAP_CANON_DISPATCH(qc.mask, RAP_NG_CALL)
+#undef RAP_NG_CALL
+          ev_s[c * 32 + lane] = x;
+        }
+      }
+      const Canon qp = pg.cn;
+      for (int j = 0; j < len; ++j) {
+        uint64_t h = pg.ng.hsalt;  // R7: h = H(salt); h = H(h ^ c[j+q])
+        int seen = 0, q = 0;
+        for (int c = 0; c < k && q < n; ++c) {
+          if ((present >> c) & 1u) {
+            if (seen >= j) {
+              h = splitmix_H(h ^ (uint64_t)ev_s[c * 32 + lane]);
+              ++q;
+            }
+            ++seen;
+          }
+        }
+        int64_t v = (int64_t)reduce_M(h, pg.ng.M);
+#define RAP_NP_CALL(M) v = canon_apply<M>(qp, itab, v, 15)
+        RAP_CANON_DISPATCH(qp.mask, RAP_NP_CALL)
+#undef RAP_NP_CALL
+        const long long pos = run + lx + j;
+        if (pos < cap) values[pos] = v;
+      }
+    } else if (__all_sync(0xffffffffu, len <= 1)) {
+      if (len == 1) {
+        const long long pos = run + lx;
+        const int64_t v = ngram_window(p, pg, ops, st_s + lane, sl_s + lane, 32, row, 0);
+        if (pos < cap) values[pos] = v;
+      }
+    } else {
+      const int mylex = inr ? lx : INT_MAX;
+      for (int eb = 0; eb < T; eb += 32) {
+        const int e = eb + lane;
+        int r = 0;
+#pragma unroll
+        for (int step = 16; step >= 1; step >>= 1) {
+          const int c = __shfl_sync(0xffffffffu, mylex, r + step);
+          if (c <= e) r += step;
+        }
+        const int lex_r = __shfl_sync(0xffffffffu, mylex, r);
+        if (e < T) {
+          const int64_t v = ngram_window(p, pg, ops, st_s + r, sl_s + r, 32, r0 + 32 * g + r, e - lex_r);
+          const long long pos = run + e;
+          if (pos < cap) values[pos] = v;
+        }
+      }
+    }
+    __syncwarp();
+    run += T;
+  }
+  if (f == p.c.n_sparse_out - 1 && rt == p.c.tiles_per_feature - 1 && lane == 0) {
+    p.c.offsets[(int64_t)p.c.n_sparse_out * B] = run;
+    if (run > cap) atomicExch(p.c.err, 1);
   }
 }
 
 // ----------------------------------------------------------------------------
-// Dense descriptor: (row block, column group) -> row-major tile via smem (a2).
+// Dense block: kDenseBlockRows rows of one column group -> row-major tile via
+// smem (a2).  Inputs staged with bulk copies on the CTA mbarrier.
+struct CtaState {
+  uint64_t bar;
+  long long ticket;
+  int staged, phase;
+};
+
+constexpr int kDProgBytes = align_up((int)sizeof(DProg), 16);
+
+__host__ __device__ constexpr int dense_in_bytes() { return 16 * kDenseBlockRows * 4 + 16 * 8 * 4; }
+
+// OneHot over a generic id list (sparse list, NGram windows): set the columns
+// of the ids in [k0, k0+width) in the row's tile slice (R9).
 template <class P>
-__device__ void dense_desc(const P& p, long long t, unsigned char* smem) {
+__device__ __noinline__ void onehot_generic(const P& p, const DUnit& un, int64_t row, float* trow) {
+  const SProg& og = p.c.oprogs[un.prog];
+  const DevOp* gops = prog_ops(og, p.c.ops);
+  const int ln = (int)(row & 31);
+  int32_t st[kMaxNgramK], sl[kMaxNgramK];
+  if (og.ch.src_kind != SRC_NGRAM) {
+    const RowIn ri = load_row(p, og.ch, row, true);
+    const int32_t L = row_len(og.ch, ri, ln, true, &st[0]);
+    for (int32_t j = 0; j < L; ++j) {
+      const int64_t d = src_value(p, gops, og.tab_off, og.ch, st[0], row, j) - un.k0;
+      if (d >= 0 && d < un.width) trow[un.col + (int)d] = 1.0f;
+    }
+    return;
+  }
+  int tot = 0;
+  for (int c = 0; c < og.ng.k; ++c) {
+    const RowIn ri = load_row(p, og.src[c], row, true);
+    sl[c] = row_len(og.src[c], ri, ln, true, &st[c]);
+    tot += sl[c];
+  }
+  const int32_t L = (int32_t)min((int64_t)max(tot - og.ng.n + 1, 0), og.ch.xcap);
+  for (int32_t j = 0; j < L; ++j) {
+    const int64_t d = ngram_window(p, og, gops, st, sl, 1, row, j) - un.k0;
+    if (d >= 0 && d < un.width) trow[un.col + (int)d] = 1.0f;
+  }
+}
+
+template <class P>
+__device__ void dense_block(const P& p, int gi, int64_t rb, unsigned char* smem, CtaState& cs) {
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const int gi = (int)(t % p.c.n_groups);
-  const long long rb = t / p.c.n_groups;
   DProg* dp = reinterpret_cast<DProg*>(smem);
-  float* tile = reinterpret_cast<float*>(smem + kDProgBytes);
+  float* din = reinterpret_cast<float*>(smem + kDProgBytes);  // [16][kDenseBlockRows]
+  uint32_t* dbm = reinterpret_cast<uint32_t*>(smem + kDProgBytes + 16 * kDenseBlockRows * 4);  // [16][8]
+  float* tile = reinterpret_cast<float*>(smem + kDProgBytes + dense_in_bytes());
+  const int64_t B = p.c.n_rows;
+  const int64_t r0 = rb * kDenseBlockRows;
+  const int nr = (int)min((int64_t)kDenseBlockRows, B - r0);
+  const int nw = (nr + 31) >> 5;
   if (warp == 0) {
-    // header + used units, used ops, used borders
     const DProg* g = p.c.dprogs + gi;
-    const int nu = __ldg(&g->n_units), no = __ldg(&g->n_ops), nf = __ldg(&g->n_ftab);
-    warp_copy16(dp, g, align_up((int)offsetof(DProg, units) + nu * (int)sizeof(DUnit), 16), lane);
-    warp_copy16(dp->ops, g->ops, align_up(no * (int)sizeof(DevOp), 16), lane);
-    warp_copy16(dp->ftab, g->ftab, align_up(nf * 4, 16), lane);
+    const int nu = __ldg(&g->n_units), no = __ldg(&g->n_ops), nf = __ldg(&g->n_ftab), nc = __ldg(&g->n_cols);
+    const int col = lane < nc ? __ldg(&g->cols[lane]) : 0;
+    const bool aligned = lane >= nc || ((reinterpret_cast<uintptr_t>(p.dense[col] + r0) & 15) == 0 &&
+                                        (p.dvalid[col] == nullptr ||
+                                         (reinterpret_cast<uintptr_t>(p.dvalid[col] + (r0 >> 5)) & 15) == 0));
+    const bool stage = __all_sync(0xffffffffu, aligned) && (nr & 3) == 0 && nc <= 16;
+    if (stage) {
+      const uint32_t bytes_v = (uint32_t)nr * 4, bytes_b = (uint32_t)align_up(nw * 4, 16);
+      uint32_t total = 0;
+      if (lane < nc) total = bytes_v + (p.dvalid[col] ? bytes_b : 0);
+#pragma unroll
+      for (int d = 16; d >= 1; d >>= 1) total += __shfl_xor_sync(0xffffffffu, total, d);
+      if (lane == 0) {
+        fence_proxy_async();
+        mbar_arrive_expect(&cs.bar, total);
+      }
+      __syncwarp();
+      if (lane < nc) {
+        bulk_g2s(din + lane * kDenseBlockRows, p.dense[col] + r0, bytes_v, &cs.bar);
+        if (p.dvalid[col]) bulk_g2s(dbm + lane * 8, p.dvalid[col] + (r0 >> 5), bytes_b, &cs.bar);
+      }
+    }
+    if (lane == 0) cs.staged = stage ? 1 : 0;
+    const int4* src = reinterpret_cast<const int4*>(g);
+    int4* dst = reinterpret_cast<int4*>(dp);
+    const int n_hdr = align_up((int)offsetof(DProg, units) + nu * (int)sizeof(DUnit), 16) >> 4;
+    for (int k = lane; k < n_hdr; k += 32) dst[k] = __ldg(src + k);
+    const int4* so = reinterpret_cast<const int4*>(g->ops);
+    int4* d2 = reinterpret_cast<int4*>(dp->ops);
+    for (int k = lane; k < (align_up(no * (int)sizeof(DevOp), 16) >> 4); k += 32) d2[k] = __ldg(so + k);
+    const int4* sf = reinterpret_cast<const int4*>(g->ftab);
+    int4* d3 = reinterpret_cast<int4*>(dp->ftab);
+    for (int k = lane; k < (align_up(nf * 4, 16) >> 4); k += 32) d3[k] = __ldg(sf + k);
   }
   __syncthreads();
-  const int64_t B = p.c.n_rows;
-  const int64_t r0 = rb * (int64_t)p.c.rows_dense;
-  const int nr = (int)min((int64_t)p.c.rows_dense, B - r0);
   const int W = dp->width;
   const int LD = W | 1;  // odd row pitch: conflict-free column writes
-  if (dp->any_onehot) {
+  if (dp->any_onehot)
     for (int i = tid; i < nr * LD; i += kThreads) tile[i] = 0.0f;
-    __syncthreads();
-  }
+  const bool staged = cs.staged;
+  if (staged) mbar_wait(&cs.bar, cs.phase);
+  __syncthreads();
   const int nu = dp->n_units;
-  for (int r = tid; r < nr; r += kThreads) {
+  // (row, unit) pairs over all threads, unit-major so a warp shares its unit
+  for (int idx = tid; idx < nr * nu; idx += kThreads) {
+    const int u = idx / nr, r = idx - u * nr;
     const int64_t row = r0 + r;
-    for (int u = 0; u < nu; ++u) {
-      const DUnit& un = dp->units[u];
-      const DevOp* uops = un.gops ? p.c.ops : dp->ops;
-      if (un.kind == U_DENSE) {
-        tile[r * LD + un.col] = apply_dense_ops(uops, dense_raw(p, un.src_col, row), un.op_begin, un.op_end);
-      } else if (un.kind == U_ONEHOT_DB) {
-        if (un.xcap > 0) {
-          const float* uft = un.gops ? p.c.ftab : dp->ftab;
-          const float x = apply_dense_ops(uops, dense_raw(p, un.src_col, row), un.op_begin, un.op_end);
-          const int64_t id = apply_id_ops(uops, p.c.itab, nullptr, upper_bound(uft + un.btab, un.bm, x),
-                                          un.iop_begin, un.iop_end);
-          const int64_t d = id - un.k0;
-          if (d >= 0 && d < un.width) tile[r * LD + un.col + (int)d] = 1.0f;
-        }
-      } else {  // U_ONEHOT_G: generic list (R9), program read from global memory
-        const SProg& pg = p.c.oprogs[un.prog];
-        const int64_t* stab = p.c.itab + pg.tab_off;
-        int32_t st[kMaxNgramK], sl[kMaxNgramK];
-        const int32_t L = chain_len_g(p, pg, row, st, sl);
-        for (int32_t j = 0; j < L; ++j) {
-          const int64_t d = chain_elem_g(p, pg, stab, st, sl, row, j) - un.k0;
-          if (d >= 0 && d < un.width) tile[r * LD + un.col + (int)d] = 1.0f;
-        }
-      }
+    const DUnit& un = dp->units[u];
+    const DevOp* uops = un.gops ? p.c.ops : dp->ops;
+    if (un.kind == U_ONEHOT_G) {  // generic list (R9), program from global memory
+      onehot_generic(p, un, row, tile + r * LD);
+      continue;
+    }
+    float x;
+    if (staged) {
+      const uint32_t w = p.dvalid[un.src_col] ? dbm[un.slot * 8 + (r >> 5)] : 0xffffffffu;
+      x = ((w >> (r & 31)) & 1u) ? din[un.slot * kDenseBlockRows + r] : __int_as_float(0x7fc00000);
+    } else {
+      x = dense_raw(p, un.src_col, row);
+    }
+    x = apply_dense_ops(uops, x, un.op_begin, un.op_end);
+    if (un.kind == U_DENSE) {
+      tile[r * LD + un.col] = x;
+    } else if (un.xcap > 0) {  // U_ONEHOT_DB
+      const float* uft = un.gops ? p.c.ftab : dp->ftab;
+      const int64_t bidx = un.gops ? upper_bound(uft + un.btab, un.bm, x) : upper_bound_s(uft + un.btab, un.bm, x);
+      const int64_t id = apply_id_ops(uops, p.c.itab, 0, bidx, un.iop_begin, un.iop_end);
+      const int64_t d = id - un.k0;
+      if (d >= 0 && d < un.width) tile[r * LD + un.col + (int)d] = 1.0f;
     }
   }
   __syncthreads();
@@ -603,59 +993,118 @@ __device__ void dense_desc(const P& p, long long t, unsigned char* smem) {
     for (int r = warp; r < nr; r += kWarps)
       for (int cc = lane; cc < W; cc += 32) out[r * ld + cc] = tile[r * LD + cc];
   }
+  if (tid == 0 && staged) cs.phase ^= 1;
 }
 
+// ----------------------------------------------------------------------------
+#ifndef RAP_MIN_CTAS
+#define RAP_MIN_CTAS 4
+#endif
 template <int MD, int MS>
-__global__ void __launch_bounds__(kThreads, 4) rap_fused_kernel(const __grid_constant__ KParams<MD, MS> p) {
-  extern __shared__ __align__(16) unsigned char smem[];
-  __shared__ long long s_ticket;
+__global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const __grid_constant__ KParams<MD, MS> p) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  __shared__ CtaState cs;
+  __shared__ long long s_wtot[kWarps];
+  __shared__ long long s_bcast[2];
   __shared__ unsigned long long s_epoch;
   __shared__ int s_last;
-  __shared__ int s_f;
-  __shared__ long long s_warp[kWarps];
-  __shared__ long long s_bcast[2];
-  const int tid = threadIdx.x;
-  unsigned long long* sched = p.c.sched;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int64_t T = p.c.tiles_per_feature;
+  const Part pa = p.c.part[blockIdx.x], pb = p.c.part[blockIdx.x + 1];
+  const int32_t s0 = pa.s0, s1 = pb.s0, d0 = pa.d0, d1 = pb.d0;
   if (tid == 0) {
-    s_epoch = ld_relaxed(sched + 2);
-    s_ticket = (long long)atomicAdd(sched, 1ull);
+    mbar_init(&cs.bar, 1);
+    cs.phase = 0;
+    s_epoch = ld_relaxed(p.c.sched + 1);
+  }
+  trace_stamp(p.c, 0);
+
+  // (1) output lengths of the chunk's sparse tiles, one warp per tile
+  for (int32_t t = s0 + warp; t < s1; t += kWarps) {
+    const uint32_t f = (uint32_t)t / (uint32_t)T;
+    length_tile(p, (int)f, (int64_t)t - (int64_t)f * T, lane);
   }
   __syncthreads();
-  const unsigned long long epoch = s_epoch;
-  long long t = s_ticket;
-  while (t < p.c.n_total_desc) {
-    unsigned long long nxt = 0;
-    if (tid == 0) nxt = atomicAdd(sched, 1ull);  // prefetch the next ticket
-    if (t < p.c.n_sparse_desc) {
-      sparse_desc(p, t, epoch, smem, s_warp, s_bcast, &s_f);
-    } else {
-      dense_desc(p, t - p.c.n_sparse_desc, smem);
+  trace_stamp(p.c, 1);
+  // chunk-local exclusive scan of the tile sums (in place)
+  long long carry = 0;
+  for (int32_t b0 = s0; b0 < s1; b0 += kThreads) {
+    const int32_t i = b0 + tid;
+    const long long v = i < s1 ? p.c.tile_sum[i] : 0;
+    long long incl = v;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const long long y = __shfl_up_sync(0xffffffffu, incl, d);
+      if (lane >= d) incl += y;
     }
+    if (lane == 31) s_wtot[warp] = incl;
     __syncthreads();
-    if (tid == 0) s_ticket = (long long)nxt;
+    long long wpre = 0, btot = 0;
+#pragma unroll
+    for (int q = 0; q < kWarps; ++q) {
+      const long long w = s_wtot[q];
+      if (q < warp) wpre += w;
+      btot += w;
+    }
+    if (i < s1) p.c.tile_sum[i] = carry + wpre + incl - v;
+    carry += btot;
     __syncthreads();
-    t = s_ticket;
   }
-  // The last CTA out resets the ticket / done counters and advances the epoch
-  // (clearing the look-back words when the 20-bit epoch wraps).
+  // (2) publish the chunk total right away (R17 scan across CTAs)
+  const unsigned long long epoch = s_epoch;
+  if (tid == 0) {
+    const unsigned long long tag = epoch << kEpochShift;
+    st_relaxed(p.c.status + blockIdx.x,
+               tag | ((blockIdx.x == 0 ? kFlagPrefix : kFlagAgg) << kFlagShift) | (unsigned long long)carry);
+  }
+  trace_stamp(p.c, 2);
+
+  // (3) dense blocks (no dependency on the scan)
+  for (int32_t d = d0; d < d1; ++d) {
+    const uint32_t gi = (uint32_t)d % (uint32_t)p.c.n_groups;
+    dense_block(p, (int)gi, (int64_t)((uint32_t)d / (uint32_t)p.c.n_groups), smem, cs);
+    __syncthreads();
+  }
+  trace_stamp(p.c, 3);
+
+  // (4) chunk base by decoupled look-back over CTAs < blockIdx.x
+  if (warp == 0) {
+    const long long excl = blockIdx.x == 0 ? 0 : lookback(p.c.status, blockIdx.x, carry, epoch, lane);
+    if (lane == 0) s_bcast[0] = excl;
+  }
+  __syncthreads();
+  const long long cbase = s_bcast[0];
+  trace_stamp(p.c, 4);
+
+  // (5) offsets and ids of the chunk's tiles, one warp per tile
+  {
+    // warp-private scratch in the (dense-block) dynamic smem
+    int32_t* scr = reinterpret_cast<int32_t*>(smem) + warp * (4 * kMaxNgramK * 32);
+    for (int32_t t = s0 + warp; t < s1; t += kWarps) {
+      const uint32_t f = (uint32_t)t / (uint32_t)T;
+      value_tile(p, (int)f, (int64_t)t - (int64_t)f * T, lane, cbase + p.c.tile_sum[t], scr);
+    }
+  }
+  trace_stamp(p.c, 5);
+
+  // The last CTA out advances the epoch of the look-back words (clearing
+  // them when the 20-bit epoch wraps) and resets the done counter.
+  __syncthreads();
   if (tid == 0) {
     __threadfence();
-    const unsigned long long prev = atomicAdd(sched + 1, 1ull);
+    const unsigned long long prev = atomicAdd(p.c.sched, 1ull);
     s_last = (prev == (unsigned long long)gridDim.x - 1) ? 1 : 0;
     if (s_last) __threadfence();
   }
   __syncthreads();
   if (s_last) {
     const bool wrap = epoch >= kEpochMax;
-    if (wrap) {
-      for (long long i = tid; i < p.c.status_cap; i += kThreads) p.c.status[i] = 0ull;
-      __threadfence();
-    }
+    if (wrap)
+      for (int i = tid; i < (int)gridDim.x; i += kThreads) p.c.status[i] = 0ull;
     __syncthreads();
     if (tid == 0) {
-      sched[0] = 0ull;
-      sched[1] = 0ull;
-      sched[2] = wrap ? 1ull : epoch + 1ull;
+      p.c.sched[0] = 0ull;
+      p.c.sched[1] = wrap ? 1ull : epoch + 1ull;
       __threadfence();
     }
   }
@@ -682,20 +1131,34 @@ static int launch_t(const Common& c, const LaunchRaw& raw, int grid, int smem, c
     p.val[i] = raw.val[i];
     p.svalid[i] = raw.svalid ? raw.svalid[i] : nullptr;
   }
-  rap_fused_kernel<MD, MS><<<grid, kThreads, smem, st>>>(p);
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(kThreads);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeCooperative;  // co-residency for the grid barriers
+  attr[0].val.cooperative = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  cudaError_t e = cudaLaunchKernelEx(&cfg, rap_fused_kernel<MD, MS>, p);
+  if (e != cudaSuccess) return (int)e;
   return (int)cudaGetLastError();
 }
 
 int launch_fused(const Common& c, const LaunchRaw& raw, int grid, int smem_bytes, void* stream) {
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  if (grid > kMaxGrid) return (int)cudaErrorInvalidValue;
   if (raw.n_dense <= 32 && raw.n_sparse <= 64) return launch_t<32, 64>(c, raw, grid, smem_bytes, st);
   if (raw.n_dense <= 128 && raw.n_sparse <= 1024) return launch_t<128, 1024>(c, raw, grid, smem_bytes, st);
   return (int)cudaErrorInvalidValue;
 }
 
-int fused_smem_bytes(int tile_bytes) {
-  const int dense = kDProgBytes + align_up(tile_bytes, 16);
-  return dense > kSparseSmem ? dense : kSparseSmem;
+int fused_smem_bytes(int max_width) {
+  const int tile = kDenseBlockRows * (max_width | 1) * 4;
+  const int dense = kDProgBytes + dense_in_bytes() + align_up(tile, 16);
+  const int ngram_scratch = kWarps * 4 * kMaxNgramK * 32 * 4;  // value_tile_ngram warp scratch
+  return dense > ngram_scratch ? dense : ngram_scratch;
 }
 
 int fused_occupancy(int smem_bytes, int n_dense, int n_sparse, int* ctas_per_sm) {

@@ -85,18 +85,22 @@ struct rap_plan {
   unsigned char* blob = nullptr;
   size_t off_ops = 0, off_sprogs = 0, off_oprogs = 0, off_dprogs = 0, off_ftab = 0, off_itab = 0;
   // per-n_rows descriptor table
-  int32_t* d_desc_start = nullptr;
-  int32_t* d_rows_per_desc = nullptr;
-  int64_t desc_rows = -1;
-  std::vector<int32_t> h_desc_start, h_rows_per_desc;
-  int64_t n_sparse_desc = 0, n_dense_desc = 0;
+  int64_t* d_tile_sum = nullptr;   // per sparse tile length sums (scan scratch)
+  int64_t tile_cap = 0;
+  // per-CTA partition (cost model), cached by its key
+  Part* d_part = nullptr;
+  std::vector<Part> h_part;
+  std::vector<double> key_part;
+  std::vector<double> sparse_row_cost, dense_row_cost;
   // scheduling state
-  unsigned long long* d_sched = nullptr;  // ticket, done, epoch (device-managed)
-  unsigned long long* d_status = nullptr;
-  int64_t status_cap = 0;
+  unsigned long long* d_sched = nullptr;   // CTAs done, look-back epoch
+  unsigned long long* d_status = nullptr;  // look-back words, one per CTA
   int32_t* d_err = nullptr;
   int64_t n_launches = 0;
   int64_t last_n_desc = 0;
+  // profiling aid (rap_debug_trace)
+  unsigned long long* d_trace = nullptr;
+  int64_t trace_cap = 0;
   // host-buffer staging (rap_preprocess_host)
   std::vector<void*> stage;
   std::vector<size_t> stage_cap;
@@ -544,6 +548,36 @@ double algorithmic_bytes(const rap_plan* P, int64_t B, const int64_t* nnz) {
 // ----------------------------------------------------------------------------
 // Flattened device programs (rap_internal.h).
 
+// Canonical form of a chain's id ops (rap_internal.h); ok = 0 when the ops
+// are not an ordered subset of Clamp -> MapId -> SigridHash -> Bucketize.
+// post = true: the chain is an NGram output (its ops follow the hash).
+Canon make_canon(const DevOp* ops, const Chain& ch, int64_t tab_off, bool post) {
+  Canon c;
+  memset(&c, 0, sizeof(c));
+  if (!post && ch.src_kind != SRC_SPARSE) return c;
+  int stage = 0;
+  for (int o = ch.op_begin; o < ch.op_end; ++o) {
+    const DevOp& op = ops[o];
+    int s, bit;
+    switch (op.kind) {
+      case OK_CLAMP: s = 0; bit = CB_CLAMP; c.lo = op.a; c.hi = op.b; break;
+      case OK_MAPID:
+        if (op.M) return Canon{};  // INT64_MIN key: interpreter
+        s = 1; bit = CB_MAPID; c.map_a = op.a; c.map_m = op.m; c.map_def = op.b; break;
+      case OK_SIGRID: s = 2; bit = CB_SIGRID; c.hs = op.hsalt; c.M = op.M; break;
+      case OK_BUCKET_I: s = 3; bit = CB_BUCKET; c.bk_a = op.a; c.bk_m = op.m; break;
+      case OK_BUCKET_S: s = 3; bit = CB_BUCKET; c.bk_a = tab_off + op.a; c.bk_m = op.m; break;
+      default: return Canon{};
+    }
+    if (s < stage) return Canon{};
+    stage = s + 1;
+    c.mask |= bit;
+    if (o >= ch.null_op_begin) c.null_mask |= bit;
+  }
+  c.ok = 1;
+  return c;
+}
+
 // SProg of an id chain: the chain (and an NGram's source chains) with their
 // ops copied in and rebased; the first Bucketize border tables that fit are
 // staged next to the program.  Programs with more than kMaxStagedOps ops keep
@@ -602,6 +636,9 @@ SProg make_sprog(rap_plan* P, int chain_idx) {
     sp.tab_len = (int32_t)tab.size();
     P->itab.insert(P->itab.end(), tab.begin(), tab.end());
   }
+  const DevOp* ops = sp.global_ops ? P->ops.data() : sp.ops;
+  sp.cn = make_canon(ops, sp.ch, sp.tab_off, sp.ch.src_kind == SRC_NGRAM);
+  for (int k = 0; k < nsrc; ++k) sp.src_cn[k] = make_canon(ops, sp.src[k], sp.tab_off, false);
   return sp;
 }
 
@@ -669,11 +706,19 @@ void build_dprogs(rap_plan* P, const std::vector<Unit>& flat) {
         for (int k = b; k < e; ++k) cur.ops[cur.n_ops++] = P->ops[k];
         *oe = cur.n_ops;
       };
+      auto slot_of = [&](int col) {
+        for (int k = 0; k < cur.n_cols; ++k)
+          if (cur.cols[k] == col) return k;
+        cur.cols[cur.n_cols] = col;
+        return cur.n_cols++;
+      };
       if (kind == U_DENSE) {
         du.src_col = de->col;
+        du.slot = slot_of(de->col);
         copy_ops(de->op_begin, de->op_end, &du.op_begin, &du.op_end);
       } else if (kind == U_ONEHOT_DB) {
         du.src_col = ch->src;
+        du.slot = slot_of(ch->src);
         du.xcap = ch->xcap;
         copy_ops(ch->dop_begin, ch->dop_end, &du.op_begin, &du.op_end);
         copy_ops(ch->op_begin, ch->op_end, &du.iop_begin, &du.iop_end);
@@ -790,7 +835,7 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
       }
       SparseOut so{};
       so.chain = c;
-      so.rows_per_desc = kRowsSparseMax;
+      so.rows_per_desc = kTileRows;
       P->souts.push_back(so);
     }
   }
@@ -799,9 +844,12 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
   for (const SparseOut& so : P->souts) P->sprogs.push_back(make_sprog(P, so.chain));
   build_dprogs(P, flat_units);
   {
-    int max_w = 1;
-    for (const DProg& dp : P->dprogs) max_w = std::max(max_w, dp.width);
-    const int rows = kDenseTileBytes / ((max_w | 1) * 4);
+    int max_w = 1, max_cols = 1;
+    for (const DProg& dp : P->dprogs) {
+      max_w = std::max(max_w, dp.width);
+      max_cols = std::max(max_cols, dp.n_cols);
+    }
+    const int rows = std::min(kDenseTileBytes / ((max_w | 1) * 4), kDenseInBytes / (max_cols * 4));
     P->rows_dense = std::max(32, std::min(256, rows / 32 * 32));
   }
   // used raw columns (for the byte model)
@@ -830,15 +878,16 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
   if (blob.empty()) blob.resize(16);
   e = cudaMalloc(&P->blob, blob.size());
   if (e == cudaSuccess) e = cudaMemcpy(P->blob, blob.data(), blob.size(), cudaMemcpyHostToDevice);
-  if (e == cudaSuccess) e = cudaMalloc(&P->d_sched, 3 * sizeof(unsigned long long));
+  if (e == cudaSuccess) e = cudaMalloc(&P->d_sched, 2 * sizeof(unsigned long long));
   if (e == cudaSuccess) {
-    const unsigned long long init[3] = {0ull, 0ull, 1ull};
+    const unsigned long long init[2] = {0ull, 1ull};
     e = cudaMemcpy(P->d_sched, init, sizeof(init), cudaMemcpyHostToDevice);
   }
+  if (e == cudaSuccess) e = cudaMalloc(&P->d_status, sizeof(unsigned long long) * kMaxCtas);
+  if (e == cudaSuccess) e = cudaMemset(P->d_status, 0, sizeof(unsigned long long) * kMaxCtas);
+  if (e == cudaSuccess) e = cudaMalloc(&P->d_part, sizeof(Part) * (kMaxCtas + 1));
   if (e == cudaSuccess) e = cudaMalloc(&P->d_err, sizeof(int32_t));
   if (e == cudaSuccess) e = cudaMemset(P->d_err, 0, sizeof(int32_t));
-  if (e == cudaSuccess) e = cudaMalloc(&P->d_desc_start, sizeof(int32_t) * (P->souts.size() + 1));
-  if (e == cudaSuccess) e = cudaMalloc(&P->d_rows_per_desc, sizeof(int32_t) * (P->souts.size() + 1));
   if (e != cudaSuccess) {
     rap_plan_destroy(P);
     return cuda_fail(e, "plan device allocation");
@@ -847,7 +896,7 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
   // ---- shared memory and occupancy
   int max_w = 1;
   for (const DProg& dp : P->dprogs) max_w = std::max(max_w, dp.width);
-  P->smem = fused_smem_bytes(P->rows_dense * (max_w | 1) * 4);
+  P->smem = fused_smem_bytes(max_w);
   int occ = 0;
   e = (cudaError_t)fused_occupancy(P->smem, P->n_dense_in, P->n_sparse_in, &occ);
   if (e != cudaSuccess) {
@@ -864,10 +913,11 @@ void rap_plan_destroy(rap_plan* P) {
   DeviceGuard dg(P->device);
   cudaFree(P->blob);
   cudaFree(P->d_sched);
-  cudaFree(P->d_err);
-  cudaFree(P->d_desc_start);
-  cudaFree(P->d_rows_per_desc);
   cudaFree(P->d_status);
+  cudaFree(P->d_part);
+  cudaFree(P->d_err);
+  cudaFree(P->d_tile_sum);
+  cudaFree(P->d_trace);
   for (void* s : P->stage) cudaFree(s);
   delete P;
 }
@@ -888,6 +938,37 @@ rap_status rap_plan_output_shape(const rap_plan* P, int64_t n_rows, const int64_
   return RAP_OK;
 }
 
+rap_status rap_debug_trace(rap_plan* P, int32_t enable, uint64_t* host_out, int64_t cap, int64_t* n_desc) {
+  if (!P) return fail(RAP_ERR_INVALID_ARGUMENT, "plan is NULL");
+  DeviceGuard dg(P->device);
+  cudaError_t e = cudaSuccess;
+  if (enable == 1) {
+    if (cap <= 0) return fail(RAP_ERR_INVALID_ARGUMENT, "cap <= 0");
+    e = cudaDeviceSynchronize();
+    if (e == cudaSuccess && P->trace_cap < cap) {
+      cudaFree(P->d_trace);
+      P->d_trace = nullptr;
+      P->trace_cap = 0;
+      e = cudaMalloc(&P->d_trace, sizeof(unsigned long long) * kTracePts * cap);
+      if (e == cudaSuccess) P->trace_cap = cap;
+    }
+    if (e == cudaSuccess) e = cudaMemset(P->d_trace, 0, sizeof(unsigned long long) * kTracePts * P->trace_cap);
+  } else if (enable == 0) {
+    if (!host_out) return fail(RAP_ERR_INVALID_ARGUMENT, "host_out is NULL");
+    e = cudaDeviceSynchronize();
+    const int64_t n = std::min(cap, std::min(P->trace_cap, P->last_n_desc));
+    if (e == cudaSuccess && n > 0)
+      e = cudaMemcpy(host_out, P->d_trace, sizeof(unsigned long long) * kTracePts * n, cudaMemcpyDeviceToHost);
+    if (n_desc) *n_desc = P->last_n_desc;
+  } else {
+    e = cudaDeviceSynchronize();
+    cudaFree(P->d_trace);
+    P->d_trace = nullptr;
+    P->trace_cap = 0;
+  }
+  return e == cudaSuccess ? RAP_OK : cuda_fail(e, "rap_debug_trace");
+}
+
 rap_status rap_plan_info_get(const rap_plan* P, rap_plan_info* info) {
   if (!P || !info) return fail(RAP_ERR_INVALID_ARGUMENT, "NULL argument");
   memset(info, 0, sizeof(*info));
@@ -900,7 +981,7 @@ rap_status rap_plan_info_get(const rap_plan* P, rap_plan_info* info) {
   info->n_dense_out_cols = P->d_out;
   info->n_sparse_out = (int32_t)P->souts.size();
   info->n_dense_groups = (int32_t)P->dprogs.size();
-  info->rows_per_dense_desc = P->rows_dense;
+  info->rows_per_dense_desc = kDenseBlockRows;
   int rmax = 0, rmin = INT32_MAX;
   for (const SparseOut& so : P->souts) {
     rmax = std::max(rmax, so.rows_per_desc);
@@ -917,7 +998,7 @@ rap_status rap_plan_info_get(const rap_plan* P, rap_plan_info* info) {
 static rap_status check_batch(const rap_plan* P, const rap_raw_batch* raw, const rap_output* out) {
   if (!P || !raw || !out) return fail(RAP_ERR_INVALID_ARGUMENT, "NULL argument");
   if (raw->n_rows < 0) return fail(RAP_ERR_INVALID_ARGUMENT, "n_rows < 0");
-  if (raw->n_rows > (int64_t)INT32_MAX - kRowsSparseMax) return fail(RAP_ERR_INVALID_ARGUMENT, "n_rows too large");
+  if (raw->n_rows > (int64_t)INT32_MAX - kTileRows) return fail(RAP_ERR_INVALID_ARGUMENT, "n_rows too large");
   const int64_t B = raw->n_rows;
   if (B == 0) {
     if (!P->souts.empty() && !out->offsets) return fail(RAP_ERR_INVALID_ARGUMENT, "offsets NULL");
@@ -942,6 +1023,123 @@ static rap_status check_batch(const rap_plan* P, const rap_raw_batch* raw, const
   return RAP_OK;
 }
 
+// ----------------------------------------------------------------------------
+// Cost model of the fused kernel (lane-instructions per row).
+// It plays the role of the paper's preprocessing latency predictor
+// (L1037-1057) for the intra-kernel schedule: the partition gives every CTA
+// about the same predicted work.
+static double op_cost(const DevOp& op) {
+  switch (op.kind) {
+    case OK_CLAMP: return 8;
+    case OK_SIGRID: return 40;
+    case OK_MAPID: return 30;
+    case OK_BUCKET_I:
+    case OK_BUCKET_S: return 4 + 6 * std::log2((double)op.m + 1);
+    case OK_FILL_F: return 3;
+    case OK_LOGIT: return 40;
+    default: return 70;  // OK_BOXCOX
+  }
+}
+
+static double chain_ops_cost(const rap_plan* P, const Chain& ch) {
+  double c = 0;
+  for (int o = ch.op_begin; o < ch.op_end; ++o) c += op_cost(P->ops[o]);
+  if (ch.src_kind == SRC_DENSE_BUCKET) {
+    for (int o = ch.dop_begin; o < ch.dop_end; ++o) c += op_cost(P->ops[o]);
+    c += 4 + 6 * std::log2((double)ch.bm + 1);
+  }
+  return c;
+}
+
+static double sparse_row_cost(const rap_plan* P, const Chain& ch, int64_t B, const int64_t* nnz) {
+  if (ch.src_kind != SRC_NGRAM) return 40 + expected_len(P, ch, B, nnz) * (8 + chain_ops_cost(P, ch));
+  const NGramDesc& ng = P->ngrams[ch.src];
+  double c = 40, lens = 0, elem = 0;
+  for (int k = 0; k < ng.k; ++k) {
+    const Chain& s = P->chains[ng.chain[k]];
+    const double e = expected_len(P, s, B, nnz);
+    lens += e;
+    elem += e * (8 + chain_ops_cost(P, s));
+    c += 15;
+  }
+  const double windows = std::min((double)ch.xcap, std::max(0.0, lens - ng.n + 1));
+  return c + windows * (ng.n * (elem / std::max(lens, 1.0) + 35) + 10 + chain_ops_cost(P, ch));
+}
+
+static double dense_row_cost(const rap_plan* P, const DProg& dp) {
+  double c = 0;
+  for (int u = 0; u < dp.n_units; ++u) {
+    const DUnit& un = dp.units[u];
+    const DevOp* ops = un.gops ? P->ops.data() : dp.ops;
+    c += 12;
+    if (un.kind == U_ONEHOT_G) {
+      c += 100;
+      continue;
+    }
+    for (int o = un.op_begin; o < un.op_end; ++o) c += op_cost(ops[o]);
+    if (un.kind == U_ONEHOT_DB) {
+      c += 10 + 6 * std::log2((double)un.bm + 1);
+      for (int o = un.iop_begin; o < un.iop_end; ++o) c += op_cost(ops[o]);
+    }
+  }
+  return c + 2.0 * dp.width;
+}
+
+// Per-CTA partition of the launch: contiguous chunks of the feature-major
+// sparse tile sequence plus an even share of the dense blocks, balanced by
+// the cost model.  Recomputed (and uploaded) only when its key changes.
+static rap_status update_partition(rap_plan* P, int64_t B, const int64_t* nnz, int G, cudaStream_t stream) {
+  const int64_t F = (int64_t)P->souts.size();
+  const int64_t T = (B + kTileRows - 1) / kTileRows;
+  const int64_t Tb = (B + kDenseBlockRows - 1) / kDenseBlockRows;
+  std::vector<double> key{(double)B, (double)G};
+  for (const SparseOut& so : P->souts)  // mean list lengths, quantised to 1/16
+    key.push_back(std::round(16.0 * expected_len(P, P->chains[so.chain], B, nnz)));
+  if (key == P->key_part) return RAP_OK;
+  std::vector<double> tile_cost(F), dense_cost(P->dprogs.size());
+  double total = 0;
+  for (int64_t f = 0; f < F; ++f) {
+    tile_cost[f] = kTileRows * sparse_row_cost(P, P->chains[P->souts[f].chain], B, nnz);
+    total += tile_cost[f] * T;
+  }
+  for (size_t g = 0; g < P->dprogs.size(); ++g) {
+    dense_cost[g] = kDenseBlockRows * dense_row_cost(P, P->dprogs[g]);
+    total += dense_cost[g] * Tb;
+  }
+  const int64_t D = (int64_t)P->dprogs.size() * Tb;
+  const int64_t S = F * T;
+  std::vector<Part> part(G + 1);
+  std::vector<double> sbudget(G);
+  double sparse_total = 0, sb_total = 0;
+  for (int64_t f = 0; f < F; ++f) sparse_total += tile_cost[f] * T;
+  for (int i = 0; i <= G; ++i) part[i].d0 = (int32_t)((int64_t)i * D / G);
+  for (int i = 0; i < G; ++i) {
+    double dc = 0;
+    for (int32_t d = part[i].d0; d < part[i + 1].d0; ++d) dc += dense_cost[d % (int64_t)P->dprogs.size()];
+    sbudget[i] = std::max(0.0, total / G - dc);
+    sb_total += sbudget[i];
+  }
+  const double scale = sb_total > 0 ? sparse_total / sb_total : 0;
+  double want = 0, cum = 0;
+  int64_t t = 0;
+  for (int i = 0; i < G; ++i) {
+    part[i].s0 = (int32_t)t;
+    want += sbudget[i] * scale;
+    while (t < S) {
+      const double c = tile_cost[t / T];
+      if (cum + 0.5 * c > want) break;
+      cum += c;
+      ++t;
+    }
+  }
+  part[G].s0 = (int32_t)S;
+  P->h_part = part;
+  cudaError_t e = cudaMemcpyAsync(P->d_part, P->h_part.data(), sizeof(Part) * (G + 1), cudaMemcpyHostToDevice, stream);
+  if (e != cudaSuccess) return cuda_fail(e, "partition upload");
+  P->key_part = key;
+  return RAP_OK;
+}
+
 static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output* out, cudaStream_t stream) {
   const int64_t B = raw->n_rows;
   cudaError_t e;
@@ -952,66 +1150,27 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
     }
     return RAP_OK;
   }
-  // per-call descriptor table (feature-major sparse descriptors).  Rows per
-  // descriptor are chosen so a descriptor's output ids fit the kVBuf staging
-  // buffer at the expected list length (the work-descriptor table).
-  {
-    bool changed = P->desc_rows != B;
-    for (size_t f = 0; f < P->souts.size(); ++f) {
-      const double e = expected_len(P, P->chains[P->souts[f].chain], B, raw->sp_nnz);
-      int R = kRowsSparseMax;
-      while (R > 32 && R * std::max(e, 1.0) > 0.75 * kVBuf) R >>= 1;
-      const Chain& ch = P->chains[P->souts[f].chain];
-      if (ch.src_kind == SRC_NGRAM)
-        while (R * P->ngrams[ch.src].k > kNgSlots) R >>= 1;
-      if (R != P->souts[f].rows_per_desc) {
-        P->souts[f].rows_per_desc = R;
-        changed = true;
-      }
-    }
-    if (changed) {
-      P->h_desc_start.assign(P->souts.size() + 1, 0);
-      int64_t acc = 0;
-      for (size_t f = 0; f < P->souts.size(); ++f) {
-        P->h_desc_start[f] = (int32_t)acc;
-        acc += (B + P->souts[f].rows_per_desc - 1) / P->souts[f].rows_per_desc;
-      }
-      P->h_desc_start[P->souts.size()] = (int32_t)acc;
-      P->n_sparse_desc = acc;
-      e = cudaMemcpyAsync(P->d_desc_start, P->h_desc_start.data(), sizeof(int32_t) * P->h_desc_start.size(),
-                          cudaMemcpyHostToDevice, stream);
-      if (e == cudaSuccess)
-      {
-        std::vector<int32_t> rpd(P->souts.size() + 1, 0);
-        for (size_t f = 0; f < P->souts.size(); ++f) rpd[f] = P->souts[f].rows_per_desc;
-        P->h_rows_per_desc = rpd;
-        if (e == cudaSuccess)
-          e = cudaMemcpyAsync(P->d_rows_per_desc, P->h_rows_per_desc.data(), sizeof(int32_t) * rpd.size(),
-                              cudaMemcpyHostToDevice, stream);
-      }
-      if (e != cudaSuccess) return cuda_fail(e, "descriptor table upload");
-      P->desc_rows = B;
-    }
-  }
-  P->n_dense_desc = P->dprogs.empty() ? 0 : (int64_t)P->dprogs.size() * ((B + P->rows_dense - 1) / P->rows_dense);
-  const int64_t n_total = P->n_sparse_desc + P->n_dense_desc;
-  if (n_total == 0) return RAP_OK;
-  // scan state (grows, never shrinks)
-  if (P->n_sparse_desc > P->status_cap) {
-    if (P->d_status) {
+  // Work decomposition: 128-row sparse tiles per output,
+  // 128-row dense blocks per column group; one length sum per sparse tile.
+  const int64_t F = (int64_t)P->souts.size();
+  const int64_t T = (B + kTileRows - 1) / kTileRows;
+  const int64_t n_sparse_tiles = F * T;
+  const int64_t n_dense = P->dprogs.empty() ? 0 : (int64_t)P->dprogs.size() * ((B + kDenseBlockRows - 1) / kDenseBlockRows);
+  if (n_sparse_tiles == 0 && n_dense == 0) return RAP_OK;
+  const int64_t grid = std::min<int64_t>((int64_t)P->budget * P->ctas_per_sm, kMaxCtas);
+  rap_status st;
+  if (n_sparse_tiles > P->tile_cap) {  // scan scratch (grows, never shrinks)
+    if (P->d_tile_sum) {
       e = cudaStreamSynchronize(stream);
       if (e != cudaSuccess) return cuda_fail(e, "cudaStreamSynchronize");
-      cudaFree(P->d_status);
-      P->d_status = nullptr;
+      cudaFree(P->d_tile_sum);
+      P->d_tile_sum = nullptr;
     }
-    const int64_t cap = std::max<int64_t>(P->n_sparse_desc, 1024);
-    e = cudaMalloc(&P->d_status, sizeof(unsigned long long) * cap);
-    if (e != cudaSuccess) return fail(RAP_ERR_OUT_OF_MEMORY, "scan-state allocation");
-    e = cudaMemsetAsync(P->d_status, 0, sizeof(unsigned long long) * cap, stream);
-    if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync");
-    P->status_cap = cap;
+    const int64_t cap = std::max<int64_t>(n_sparse_tiles, 4096);
+    e = cudaMalloc(&P->d_tile_sum, sizeof(int64_t) * cap);
+    if (e != cudaSuccess) return fail(RAP_ERR_OUT_OF_MEMORY, "scan scratch allocation");
+    P->tile_cap = cap;
   }
-  const int64_t grid = std::min<int64_t>(n_total, (int64_t)P->budget * P->ctas_per_sm);
   Common c{};
   c.ops = reinterpret_cast<const DevOp*>(P->blob + P->off_ops);
   c.sprogs = reinterpret_cast<const SProg*>(P->blob + P->off_sprogs);
@@ -1019,17 +1178,17 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
   c.dprogs = reinterpret_cast<const DProg*>(P->blob + P->off_dprogs);
   c.ftab = reinterpret_cast<const float*>(P->blob + P->off_ftab);
   c.itab = reinterpret_cast<const int64_t*>(P->blob + P->off_itab);
-  c.desc_start = P->d_desc_start;
-  c.n_sparse_out = (int32_t)P->souts.size();
+  c.n_sparse_out = (int32_t)F;
   c.n_groups = (int32_t)P->dprogs.size();
-  c.rows_dense = P->rows_dense;
-  c.rows_per_desc = P->d_rows_per_desc;
   c.n_rows = B;
-  c.n_sparse_desc = P->n_sparse_desc;
-  c.n_total_desc = n_total;
+  c.tiles_per_feature = T;
+  c.n_sparse_tiles = n_sparse_tiles;
+  c.n_dense_tiles = n_dense;
+  if ((st = update_partition(P, B, raw->sp_nnz, (int)grid, stream)) != RAP_OK) return st;
+  c.part = P->d_part;
   c.sched = P->d_sched;
   c.status = P->d_status;
-  c.status_cap = P->status_cap;
+  c.tile_sum = P->d_tile_sum;
   c.dense_out = out->dense_out;
   c.ld = out->dense_ld;
   c.lengths = out->lengths;
@@ -1037,6 +1196,9 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
   c.values = out->values;
   c.values_cap = out->values_capacity;
   c.err = P->d_err;
+  c.trace = P->d_trace;
+  c.trace_cap = P->trace_cap;
+  const int64_t n_total = n_sparse_tiles + n_dense;
   LaunchRaw lr{};
   lr.n_dense = P->n_dense_in;
   lr.n_sparse = P->n_sparse_in;

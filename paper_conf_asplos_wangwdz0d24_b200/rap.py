@@ -20,7 +20,7 @@ STATUS = {0: "OK", 1: "INVALID_ARGUMENT", 2: "INVALID_GRAPH", 3: "INVALID_PARAM"
           5: "UNSUPPORTED", 6: "CUDA", 7: "OUT_OF_MEMORY"}
 
 EXPORTS = ["rap_plan_create", "rap_plan_output_shape", "rap_preprocess", "rap_preprocess_host", "rap_set_budget",
-           "rap_predict_latency_us", "rap_choose_budget", "rap_plan_info_get", "rap_plan_destroy",
+           "rap_predict_latency_us", "rap_choose_budget", "rap_plan_info_get", "rap_debug_trace", "rap_plan_destroy",
            "rap_status_string", "rap_last_error"]
 
 
@@ -99,6 +99,8 @@ def load(build_if_stale: bool = False):
     L.rap_choose_budget.argtypes = [P, C.c_int64, P, C.c_double, C.POINTER(C.c_int32), C.POINTER(C.c_double)]
     L.rap_plan_info_get.restype = C.c_int
     L.rap_plan_info_get.argtypes = [P, C.POINTER(RapPlanInfo)]
+    L.rap_debug_trace.restype = C.c_int
+    L.rap_debug_trace.argtypes = [P, C.c_int32, P, C.c_int64, C.POINTER(C.c_int64)]
     L.rap_plan_destroy.restype = None
     L.rap_plan_destroy.argtypes = [P]
     L.rap_status_string.restype = C.c_char_p
@@ -297,6 +299,19 @@ class Plan:
         i = RapPlanInfo()
         _check(load().rap_plan_info_get(self.handle, C.byref(i)))
         return {k: getattr(i, k) for k, _ in RapPlanInfo._fields_}
+
+    def trace_enable(self, cap: int):
+        _check(load().rap_debug_trace(self.handle, 1, None, cap, None))
+
+    def trace_read(self, cap: int):
+        """Stamps of the last call: uint64 [n_desc, 8] (profiling aid)."""
+        buf = np.zeros((cap, 8), dtype=np.uint64)
+        n = C.c_int64()
+        _check(load().rap_debug_trace(self.handle, 0, buf.ctypes.data, cap, C.byref(n)))
+        return buf[: min(cap, n.value)]
+
+    def trace_disable(self):
+        _check(load().rap_debug_trace(self.handle, -1, None, 0, None))
 
     def predict_latency_us(self, n_rows, sp_nnz, sm_budget=0):
         nnz = np.ascontiguousarray(sp_nnz if len(sp_nnz) else [0], dtype=np.int64)

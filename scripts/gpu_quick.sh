@@ -1,8 +1,18 @@
 #!/bin/bash
-# build + gpu tests + bench + one ncu --set full capture of the fused kernel
+# build + gpu tests + bench + trace + one ncu --set full capture
 mkdir -p gpurun_out
 python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1
 timeout 900 python -m pytest tests -x -q -m gpu > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_gpu.log
-timeout 600 python bench.py ${BENCH_ARGS} > gpurun_out/bench.json 2> gpurun_out/bench.err
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:rap_fused -s 5 -c 1 -o gpurun_out/prof -f python bench.py --profile --steps 8 --warmup 5 ${BENCH_ARGS} > gpurun_out/ncu_full.log 2>&1
-tail -3 gpurun_out/pytest_gpu.log; cat gpurun_out/bench.json
+tail -3 gpurun_out/pytest_gpu.log
+grep -E "^FAILED|^E  " gpurun_out/pytest_gpu.log | head -8
+timeout 600 python bench.py --no-cpu-baseline ${BENCH_ARGS} > gpurun_out/bench.json 2> gpurun_out/bench.err
+python -c "import json; d=json.load(open('gpurun_out/bench.json')); print('kernel_us', d['roofline']['kernel_ms']*1e3, 'frac', d['roofline']['frac'], 'e2e', d['e2e']['value'])" 2>&1 | tail -1
+tail -2 gpurun_out/bench.err
+timeout 300 python scripts/trace.py 2>&1 | tail -7
+timeout 300 python scripts/probe.py 2>&1 | tail -8
+for v in ${VARIANTS}; do
+  RAP_NVCC_FLAGS="$v" python -c "from paper_conf_asplos_wangwdz0d24_b200 import _build; _build.build(force=True)"
+  echo "variant [$v]: $(timeout 300 python bench.py --no-e2e --no-cpu-baseline --steps 2000 | python -c 'import json,sys; d=json.loads(sys.stdin.read()); print(d["roofline"]["kernel_ms"]*1e3, "us", d["roofline"]["frac"])')"
+done
+python -c "from paper_conf_asplos_wangwdz0d24_b200 import _build; _build.build(force=True)"
+[ -z "$NO_NCU" ] && timeout 900 ncu --set full --clock-control none --import-source on -k regex:rap_fused -s 5 -c 1 -o gpurun_out/prof -f python bench.py --profile --steps 8 --warmup 5 ${BENCH_ARGS} > gpurun_out/ncu_full.log 2>&1

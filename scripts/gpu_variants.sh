@@ -1,0 +1,12 @@
+#!/bin/bash
+# build variants of librap.so and bench each (plus gpu tests on the default)
+mkdir -p gpurun_out
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1
+timeout 900 python -m pytest tests -x -q -m gpu > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_gpu.log
+tail -2 gpurun_out/pytest_gpu.log
+for v in "" ${VARIANTS}; do
+  RAP_NVCC_FLAGS="$v" python -c "from paper_conf_asplos_wangwdz0d24_b200 import _build; _build.build(force=True)"
+  echo "variant [$v]: $(timeout 300 python bench.py --no-e2e --no-cpu-baseline --steps 2000 | python -c 'import json,sys; d=json.loads(sys.stdin.read()); print(d["roofline"]["kernel_ms"]*1e3, "us", d["roofline"]["frac"])')"
+done
+python -c "from paper_conf_asplos_wangwdz0d24_b200 import _build; _build.build(force=True)"
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:rap_fused -s 5 -c 1 -o gpurun_out/prof -f python bench.py --profile --steps 8 --warmup 5 > gpurun_out/ncu_full.log 2>&1
