@@ -148,18 +148,21 @@ struct DProg {
 // Work decomposition of one launch.  Sparse tiles are
 // (output f, 128-row range rt), numbered feature-major t = f * T + rt, which
 // is also the order of the jagged scan (R17).  The planner's cost model cuts
-// [0, S) into one contiguous chunk per CTA and deals out the dense blocks
-// (128 rows x one column group) so every CTA gets about the same estimated
-// work.  CTA i then: (1) computes the output lengths of its chunk (one warp per
-// tile) and their chunk-local exclusive prefix; (2) publishes the chunk total;
-// (3) runs its dense blocks; (4) obtains its chunk base by a decoupled
-// look-back over CTAs < i (usually already resolved thanks to (3)); (5) writes
-// offsets and ids of its chunk.  No grid barrier.
+// [0, S) into one contiguous chunk per CTA for the length pass (cost ~ source
+// columns read).  CTA i then: (1) computes the output lengths of its chunk
+// (one warp per tile, tiles taken from a CTA-local counter) and their
+// chunk-local exclusive prefixes, tagged with i, into tile_sum; (2) publishes
+// the chunk total; (3) CTA 0 / warp 0 scans all chunk totals into per-chunk
+// prefixes and raises a scan-done word; (4) every CTA takes dense blocks
+// (128 rows x one column group) from a global queue; (5) every warp takes
+// value tiles from a global queue and writes offsets and ids at
+// prefix[chunk(t)] + tile_sum[t].  No grid barrier; the queues balance the
+// heavy phases whatever the cost model's error.
 constexpr int kMaxCtas = 2048;        // look-back words / partition entries a plan allocates
 constexpr int kTileRows = 128;        // rows of a sparse tile (4 groups of 32)
 constexpr int kDenseBlockRows = 128;  // rows of a dense block (CTA unit)
 
-// Per-CTA partition: sparse tiles [s0(i), s0(i+1)), dense blocks [d0(i), d0(i+1)).
+// Per-CTA partition of the length pass: sparse tiles [s0(i), s0(i+1)); d0 unused (0).
 struct Part {
   int32_t s0, d0;
 };
@@ -185,12 +188,13 @@ struct Common {
   int64_t n_sparse_tiles;     // S = n_sparse_out * T
   int64_t n_dense_tiles;      // n_groups * ceil(n_rows / kDenseBlockRows)
   const Part* part;           // [gridDim.x + 1]
-  // sched[0] = CTAs done, sched[1] = epoch of the look-back words; the last
-  // CTA advances the epoch, so launch parameters are identical from call to
-  // call (CUDA-graph replayable).
+  // sched[0] = CTAs done, sched[1] = epoch of the status words, sched[2] =
+  // dense-block queue head, sched[3] = value-tile queue head; the last CTA
+  // resets the heads and advances the epoch, so launch parameters are
+  // identical from call to call (CUDA-graph replayable).
   unsigned long long* sched;
-  unsigned long long* status;  // [gridDim.x] look-back words, one per CTA chunk
-  int64_t* tile_sum;           // [S] tile length sums -> chunk-local exclusive prefixes
+  unsigned long long* status;  // [kMaxCtas] chunk totals, then [kMaxCtas] chunk prefixes (+ scan-done word)
+  int64_t* tile_sum;           // [S] tile length sums -> ([63:48] chunk, [47:0] chunk-local exclusive prefix)
   float* dense_out;
   int64_t ld;
   int32_t* lengths;

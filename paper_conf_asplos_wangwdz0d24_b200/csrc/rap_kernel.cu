@@ -47,6 +47,8 @@ struct KParams {
 constexpr int kWarps = kThreads / 32;
 constexpr int kGroups = kTileRows / 32;  // row groups of a sparse tile (one row per lane each)
 constexpr int kMaxGrid = 2048;           // look-back words allocated by the plan
+constexpr int kCidShift = 48;             // tile_sum: [63:48] chunk (CTA) id, [47:0] chunk-local prefix
+constexpr unsigned long long kLocalMask = (1ull << kCidShift) - 1;
 
 __host__ __device__ constexpr int align_up(int x, int a) { return (x + a - 1) / a * a; }
 
@@ -122,56 +124,6 @@ __device__ __forceinline__ long long warp_sum64(long long v) {
 #pragma unroll
   for (int d = 16; d >= 1; d >>= 1) v += __shfl_xor_sync(0xffffffffu, v, d);
   return v;
-}
-
-// Decoupled look-back over the chunk totals of CTAs < slot (warp 0).  Each
-// lane inspects 4 predecessor words, so one round trip covers 128 chunks;
-// walking from the nearest predecessor down, totals are summed until the
-// first inclusive prefix, and only an unpublished word on that path makes the
-// warp wait.  Returns the exclusive prefix and publishes the inclusive one.
-__device__ long long lookback(unsigned long long* status, long long slot, long long agg, unsigned long long epoch,
-                              int lane) {
-  const unsigned long long tag = epoch << kEpochShift;
-  long long excl = 0;
-  long long top = slot - 1;
-  while (top >= 0) {
-    unsigned long long w[4];
-    int flag[4];
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      const long long idx = top - 4 * lane - q;
-      w[q] = idx >= 0 ? ld_relaxed(status + idx) : 0ull;
-      flag[q] = idx >= 0 ? (((w[q] >> kEpochShift) == epoch) ? (int)((w[q] >> kFlagShift) & 3ull) : 0)
-                         : (int)kFlagPrefix;
-    }
-    int qstop = 4;  // first slot (descending) that is unpublished or a prefix
-#pragma unroll
-    for (int q = 3; q >= 0; --q)
-      if (flag[q] != (int)kFlagAgg) qstop = q;
-    const unsigned smask = __ballot_sync(0xffffffffu, qstop < 4);
-    const int fl = smask ? __ffs(smask) - 1 : 32;
-    const int fq = __shfl_sync(0xffffffffu, qstop, fl & 31);
-    int mykind = 0;
-#pragma unroll
-    for (int q = 0; q < 4; ++q)
-      if (q == qstop) mykind = flag[q];
-    const int fkind = __shfl_sync(0xffffffffu, mykind, fl & 31);
-    long long v = 0;
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      const bool take = lane < fl || (lane == fl && (q < fq || (q == fq && fkind == (int)kFlagPrefix)));
-      if (take) v += (long long)(w[q] & kValueMask);
-    }
-    excl += warp_sum64(v);
-    if (smask == 0) {
-      top -= 128;
-      continue;
-    }
-    if (fkind == (int)kFlagPrefix) break;
-    top -= 4 * fl + fq;  // wait on the first unpublished predecessor
-  }
-  if (lane == 0) st_relaxed(status + slot, tag | (kFlagPrefix << kFlagShift) | (unsigned long long)(excl + agg));
-  return excl;
 }
 
 // Upper bound = #{i : b[i] <= x} for sorted borders (R4; NaN -> 0).
@@ -451,29 +403,102 @@ __device__ __forceinline__ int warp_incl_scan(int v, int lane) {
 }
 
 // ----------------------------------------------------------------------------
+// Sparse tiles with 4 consecutive rows per lane (rows r0 + 4*lane + k): one
+// 16-byte offsets load, one validity word, 16-byte length / offset stores.
+
+// Per-feature state a warp keeps in registers across its tiles.
+struct FeatCtx {
+  int f, kind, src, has_fill, canon, mask;
+  int64_t xcap, null_xcap, fill;
+  Canon q;
+};
+
+template <class P>
+__device__ __forceinline__ void load_ctx(const P& p, int f, FeatCtx& x) {
+  const SProg& pg = p.c.sprogs[f];
+  x.f = f;
+  x.kind = pg.ch.src_kind;
+  x.src = pg.ch.src;
+  x.has_fill = pg.ch.has_fill;
+  x.xcap = pg.ch.xcap;
+  x.null_xcap = pg.ch.null_xcap;
+  x.fill = pg.ch.fill;
+  x.q = pg.cn;
+  x.canon = x.q.ok && x.kind == SRC_SPARSE;
+  x.mask = x.q.mask;
+}
+
+// Arrow offsets of rows r0+4*lane .. +4 and the validity word of those rows.
+struct Quad {
+  int32_t a[5];
+  uint32_t w;
+};
+
+__device__ __forceinline__ Quad load_quad(const int32_t* off, const uint32_t* bm, int64_t r0, int lane, int64_t B,
+                                          bool aligned) {
+  Quad q;
+  const int64_t row = r0 + 4 * lane;
+  if (aligned && row + 4 <= B) {
+    const int4 v = __ldg(reinterpret_cast<const int4*>(off + row));
+    q.a[0] = v.x;
+    q.a[1] = v.y;
+    q.a[2] = v.z;
+    q.a[3] = v.w;
+    q.a[4] = __ldg(off + row + 4);
+  } else {
+#pragma unroll
+    for (int k = 0; k < 5; ++k) q.a[k] = row + k <= B ? __ldg(off + row + k) : 0;
+  }
+  q.w = (bm != nullptr && row < B) ? __ldg(bm + (row >> 5)) : 0xffffffffu;
+  return q;
+}
+
+// Output length of row k of the quad (R5 FirstX cap, R10 fill, R14 null).
+__device__ __forceinline__ int32_t quad_len(const Quad& q, int k, int lane, int64_t row, int64_t B, int64_t xcap,
+                                            int has_fill, int64_t null_xcap) {
+  if (row >= B) return 0;
+  if ((q.w >> ((4 * lane + k) & 31)) & 1u) return (int32_t)min((int64_t)max(q.a[k + 1] - q.a[k], 0), xcap);
+  return has_fill ? (int32_t)min((int64_t)1, null_xcap) : 0;
+}
+
+__device__ __forceinline__ bool quad_valid(const Quad& q, int k, int lane) {
+  return (q.w >> ((4 * lane + k) & 31)) & 1u;
+}
+
 // Phase 1: output lengths of sparse tile (f, rt) -> lengths[], tile_sum[].
 template <class P>
-__device__ void length_tile(const P& p, int f, int64_t rt, int lane) {
+__device__ void length_tile(const P& p, const FeatCtx& fc, int64_t rt, int lane) {
+  const int f = fc.f;
   const SProg& pg = p.c.sprogs[f];
   const int64_t B = p.c.n_rows;
   const int64_t r0 = rt * kTileRows;
   int32_t* lengths = p.c.lengths + (int64_t)f * B;
   int sum = 0;
-  if (pg.ch.src_kind != SRC_NGRAM) {
-    const Chain ch = pg.ch;
-    RowIn in[kGroups];
+  if (fc.kind == SRC_SPARSE) {
+    const int32_t* off = p.off[fc.src];
+    const Quad q = load_quad(off, p.svalid[fc.src], r0, lane, B, (reinterpret_cast<uintptr_t>(off) & 15) == 0);
+    int32_t l[4];
 #pragma unroll
-    for (int g = 0; g < kGroups; ++g) {
-      const int64_t row = r0 + 32 * g + lane;
-      in[g] = load_row(p, ch, row, row < B);
+    for (int k = 0; k < 4; ++k) {
+      l[k] = quad_len(q, k, lane, r0 + 4 * lane + k, B, fc.xcap, fc.has_fill, fc.null_xcap);
+      sum += l[k];
     }
+    const int64_t row = r0 + 4 * lane;
+    int32_t* lp = lengths + row;
+    if (row + 4 <= B && (reinterpret_cast<uintptr_t>(lp) & 15) == 0) {
+      *reinterpret_cast<int4*>(lp) = make_int4(l[0], l[1], l[2], l[3]);
+    } else {
+#pragma unroll
+      for (int k = 0; k < 4; ++k)
+        if (row + k < B) lp[k] = l[k];
+    }
+  } else if (fc.kind == SRC_DENSE_BUCKET) {
 #pragma unroll
     for (int g = 0; g < kGroups; ++g) {
       const int64_t row = r0 + 32 * g + lane;
-      int32_t st;
-      const int32_t len = row_len(ch, in[g], lane, row < B, &st);
+      const int32_t len = (int32_t)min((int64_t)1, fc.xcap);
       if (row < B) lengths[row] = len;
-      sum += len;
+      sum += row < B ? len : 0;
     }
   } else {
     const int k = pg.ng.k, n = pg.ng.n;
@@ -513,101 +538,95 @@ template <class P>
 __device__ __noinline__ void value_tile_ngram(const P& p, int f, int64_t rt, int lane, long long base,
                                               int32_t* scr);
 
-// Specialised tile of a canonical SRC_SPARSE chain (mask MASK).
+// Specialised tile of a canonical SRC_SPARSE chain (mask MASK); the lane
+// owns rows r0 + 4*lane + k, so its output ids are contiguous.
 template <int MASK, class P>
-__device__ __noinline__ void value_tile_canon(const P& p, int f, int64_t rt, int lane, long long base) {
-  const SProg& pg = p.c.sprogs[f];
-  const Canon q = pg.cn;
-  const int src = pg.ch.src;
-  const int has_fill = pg.ch.has_fill;
-  const int64_t xcap = pg.ch.xcap, null_xcap = pg.ch.null_xcap, fill = pg.ch.fill;
+__device__ __noinline__ void value_tile_canon(const P& p, const FeatCtx& fc, int64_t rt, int lane, long long base) {
+  const Canon& q = fc.q;
+  const int f = fc.f;
   const int64_t B = p.c.n_rows;
   const int64_t r0 = rt * kTileRows;
-  int64_t* offsets = p.c.offsets + (int64_t)f * B;
+  const int64_t row = r0 + 4 * lane;
   int64_t* values = p.c.values;
   const long long cap = p.c.values_cap;
   const int64_t* itab = p.c.itab;
-  const int32_t* off = p.off[src];
-  const uint32_t* bm = p.svalid[src];
-  const int64_t* val = p.val[src];
-  int32_t a[kGroups], b[kGroups];
-  uint32_t w[kGroups];
+  const int32_t* off = p.off[fc.src];
+  const int64_t* val = p.val[fc.src];
+  const Quad qd = load_quad(off, p.svalid[fc.src], r0, lane, B, (reinterpret_cast<uintptr_t>(off) & 15) == 0);
+  int32_t l[4], e[4];
+  int tot = 0;
 #pragma unroll
-  for (int g = 0; g < kGroups; ++g) {  // all row loads of the tile first
-    const int64_t row = r0 + 32 * g + lane;
-    const bool in = row < B;
-    a[g] = in ? __ldg(off + row) : 0;
-    b[g] = in ? __ldg(off + row + 1) : 0;
-    w[g] = (in && bm) ? __ldg(bm + (row >> 5)) : 0xffffffffu;
+  for (int k = 0; k < 4; ++k) {
+    l[k] = quad_len(qd, k, lane, row + k, B, fc.xcap, fc.has_fill, fc.null_xcap);
+    e[k] = tot;
+    tot += l[k];
   }
-  int32_t len[kGroups], lex[kGroups];
-  long long gb[kGroups];
-  bool valid[kGroups];
-  bool all1 = true;
-  long long run = base;
+  const int incl = warp_incl_scan(tot, lane);
+  const int L = incl - tot;  // lane exclusive prefix within the tile
+  const long long lb = base + L;
+  // offsets (R17), 16-byte stores when aligned
+  int64_t* op = p.c.offsets + (int64_t)f * B + row;
+  if (row + 4 <= B && (reinterpret_cast<uintptr_t>(op) & 15) == 0) {
+    reinterpret_cast<longlong2*>(op)[0] = make_longlong2(lb + e[0], lb + e[1]);
+    reinterpret_cast<longlong2*>(op)[1] = make_longlong2(lb + e[2], lb + e[3]);
+  } else {
 #pragma unroll
-  for (int g = 0; g < kGroups; ++g) {
-    const int64_t row = r0 + 32 * g + lane;
-    valid[g] = (w[g] >> lane) & 1u;
-    int32_t l = valid[g] ? (int32_t)min((int64_t)max(b[g] - a[g], 0), xcap)
-                         : (has_fill ? (int32_t)min((int64_t)1, null_xcap) : 0);  // R5, R10, R14
-    if (row >= B) l = 0;
-    len[g] = l;
-    all1 &= l <= 1;
-    const int incl = warp_incl_scan(l, lane);
-    lex[g] = incl - l;
-    gb[g] = run;
-    run += __shfl_sync(0xffffffffu, incl, 31);
-    if (row < B) offsets[row] = gb[g] + lex[g];
+    for (int k = 0; k < 4; ++k)
+      if (row + k < B) op[k] = lb + e[k];
   }
-  if (f == p.c.n_sparse_out - 1 && rt == p.c.tiles_per_feature - 1 && lane == 0) {
-    p.c.offsets[(int64_t)p.c.n_sparse_out * B] = run;  // total, R17
-    if (run > cap) atomicExch(p.c.err, 1);
+  const int T = __shfl_sync(0xffffffffu, incl, 31);
+  if (f == p.c.n_sparse_out - 1 && rt == p.c.tiles_per_feature - 1 && lane == 31) {
+    p.c.offsets[(int64_t)p.c.n_sparse_out * B] = base + T;  // total, R17
+    if (base + T > cap) atomicExch(p.c.err, 1);
   }
-  if (__all_sync(0xffffffffu, all1)) {
-    // at most one id per row: every lane owns its rows' output slots
-    int64_t raw[kGroups];
+  if (__all_sync(0xffffffffu, l[0] <= 1 && l[1] <= 1 && l[2] <= 1 && l[3] <= 1)) {
+    // at most one id per row: all raw ids first, then the pipelines
+    int64_t raw[4];
 #pragma unroll
-    for (int g = 0; g < kGroups; ++g) raw[g] = (len[g] == 1 && valid[g]) ? __ldg(val + a[g]) : fill;
+    for (int k = 0; k < 4; ++k) raw[k] = (l[k] == 1 && quad_valid(qd, k, lane)) ? __ldg(val + qd.a[k]) : fc.fill;
 #pragma unroll
-    for (int g = 0; g < kGroups; ++g) {
-      if (len[g] == 1) {
-        const int64_t v = canon_apply<MASK>(q, itab, raw[g], valid[g] ? 15 : q.null_mask);
-        const long long pos = gb[g] + lex[g];
+    for (int k = 0; k < 4; ++k) {
+      if (l[k] == 1) {
+        const int64_t v = canon_apply<MASK>(q, itab, raw[k], quad_valid(qd, k, lane) ? 15 : q.null_mask);
+        const long long pos = lb + e[k];
         if (pos < cap) values[pos] = v;
       }
     }
     return;
   }
-  // multi-id rows: elements in output order, the owning row found by a
-  // 5-step shuffle search over the lanes' exclusive prefixes
-#pragma unroll 1
-  for (int g = 0; g < kGroups; ++g) {
-    const int T = __shfl_sync(0xffffffffu, lex[g] + len[g], 31);
-    const int mylex = (r0 + 32 * g + lane < B) ? lex[g] : INT_MAX;
-    const int32_t mystart = valid[g] ? a[g] : -1;
-    for (int eb = 0; eb < T; eb += 32) {
-      const int e = eb + lane;
-      int r = 0;
+  // multi-id rows: elements in output order; owning lane by a 5-step shuffle
+  // search over the lane prefixes, then the row within the lane
+  const int mylex = L;
+  for (int eb = 0; eb < T; eb += 32) {
+    const int ee = eb + lane;
+    int r = 0;
 #pragma unroll
-      for (int step = 16; step >= 1; step >>= 1) {
-        const int c = __shfl_sync(0xffffffffu, mylex, r + step);
-        if (c <= e) r += step;
-      }
-      const int lex_r = __shfl_sync(0xffffffffu, mylex, r);
-      const int32_t st_r = __shfl_sync(0xffffffffu, mystart, r);
-      if (e < T) {
-        const int64_t x = st_r >= 0 ? __ldg(val + st_r + (e - lex_r)) : fill;
-        const int64_t v = canon_apply<MASK>(q, itab, x, st_r >= 0 ? 15 : q.null_mask);
-        const long long pos = gb[g] + e;
-        if (pos < cap) values[pos] = v;
-      }
+    for (int step = 16; step >= 1; step >>= 1) {
+      const int c = __shfl_sync(0xffffffffu, mylex, r + step);
+      if (c <= ee) r += step;
+    }
+    const int in_lane = ee - __shfl_sync(0xffffffffu, mylex, r);
+    const int e1 = __shfl_sync(0xffffffffu, e[1], r), e2 = __shfl_sync(0xffffffffu, e[2], r),
+              e3 = __shfl_sync(0xffffffffu, e[3], r);
+    const int k = in_lane >= e3 ? 3 : (in_lane >= e2 ? 2 : (in_lane >= e1 ? 1 : 0));
+    const int ek = k == 3 ? e3 : (k == 2 ? e2 : (k == 1 ? e1 : 0));
+    const int32_t a0 = __shfl_sync(0xffffffffu, qd.a[0], r), a1 = __shfl_sync(0xffffffffu, qd.a[1], r),
+                  a2 = __shfl_sync(0xffffffffu, qd.a[2], r), a3 = __shfl_sync(0xffffffffu, qd.a[3], r);
+    const uint32_t wr = __shfl_sync(0xffffffffu, qd.w, r);
+    const int32_t ak = k == 3 ? a3 : (k == 2 ? a2 : (k == 1 ? a1 : a0));
+    const bool vk = (wr >> ((4 * r + k) & 31)) & 1u;
+    if (ee < T) {
+      const int64_t x = vk ? __ldg(val + ak + (in_lane - ek)) : fc.fill;
+      const int64_t v = canon_apply<MASK>(q, itab, x, vk ? 15 : q.null_mask);
+      const long long pos = base + ee;
+      if (pos < cap) values[pos] = v;
     }
   }
 }
 
 template <class P>
-__device__ void value_tile(const P& p, int f, int64_t rt, int lane, long long base, int32_t* scr) {
+__device__ void value_tile(const P& p, const FeatCtx& fc, int64_t rt, int lane, long long base, int32_t* scr) {
+  const int f = fc.f;
   const SProg& pg = p.c.sprogs[f];
   const DevOp* ops = prog_ops(pg, p.c.ops);
   const int64_t B = p.c.n_rows;
@@ -617,11 +636,9 @@ __device__ void value_tile(const P& p, int f, int64_t rt, int lane, long long ba
   const long long cap = p.c.values_cap;
   const int64_t* itab = p.c.itab;
 
-  const int canon = __ldg(&pg.cn.ok) && __ldg(&pg.ch.src_kind) == SRC_SPARSE;
-  if (canon) {
-    const int mask = __ldg(&pg.cn.mask);
-#define RAP_VT_CALL(M) value_tile_canon<M>(p, f, rt, lane, base)
-    RAP_CANON_DISPATCH(mask, RAP_VT_CALL)
+  if (fc.canon) {
+#define RAP_VT_CALL(M) value_tile_canon<M>(p, fc, rt, lane, base)
+    RAP_CANON_DISPATCH(fc.mask, RAP_VT_CALL)
 #undef RAP_VT_CALL
     return;
   }
@@ -1008,21 +1025,33 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
   __shared__ long long s_bcast[2];
   __shared__ unsigned long long s_epoch;
   __shared__ int s_last;
+  __shared__ int s_next[1];  // CTA-local length-tile counter
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int64_t T = p.c.tiles_per_feature;
   const Part pa = p.c.part[blockIdx.x], pb = p.c.part[blockIdx.x + 1];
-  const int32_t s0 = pa.s0, s1 = pb.s0, d0 = pa.d0, d1 = pb.d0;
+  const int32_t s0 = pa.s0, s1 = pb.s0;
   if (tid == 0) {
     mbar_init(&cs.bar, 1);
     cs.phase = 0;
     s_epoch = ld_relaxed(p.c.sched + 1);
+    s_next[0] = 0;
   }
+  __syncthreads();
   trace_stamp(p.c, 0);
 
   // (1) output lengths of the chunk's sparse tiles, one warp per tile
-  for (int32_t t = s0 + warp; t < s1; t += kWarps) {
-    const uint32_t f = (uint32_t)t / (uint32_t)T;
-    length_tile(p, (int)f, (int64_t)t - (int64_t)f * T, lane);
+  // Warps take tiles from a CTA-local counter (tile costs differ by feature:
+  // NGram tiles cost several plain ones).
+  FeatCtx fc;
+  fc.f = -1;
+  while (true) {
+    int t = 0;
+    if (lane == 0) t = s0 + atomicAdd(&s_next[0], 1);
+    t = __shfl_sync(0xffffffffu, t, 0);
+    if (t >= s1) break;
+    const int f = (int)((uint32_t)t / (uint32_t)T);
+    if (f != fc.f) load_ctx(p, f, fc);  // a chunk spans few features: cached per warp
+    length_tile(p, fc, (int64_t)t - (int64_t)f * T, lane);
   }
   __syncthreads();
   trace_stamp(p.c, 1);
@@ -1046,43 +1075,98 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
       if (q < warp) wpre += w;
       btot += w;
     }
-    if (i < s1) p.c.tile_sum[i] = carry + wpre + incl - v;
+    if (i < s1) p.c.tile_sum[i] = (int64_t)(((unsigned long long)blockIdx.x << kCidShift) | (unsigned long long)(carry + wpre + incl - v));
     carry += btot;
     __syncthreads();
   }
-  // (2) publish the chunk total right away (R17 scan across CTAs)
+  // (2) publish the chunk total; the chunk's tile prefixes (tile_sum) are
+  // released before it
   const unsigned long long epoch = s_epoch;
+  const unsigned long long tag = epoch << kEpochShift;
+  const int G = (int)gridDim.x;
+  unsigned long long* pref = p.c.status + kMaxCtas;  // [G] chunk prefixes, [G] = scan-done word
   if (tid == 0) {
-    const unsigned long long tag = epoch << kEpochShift;
-    st_relaxed(p.c.status + blockIdx.x,
-               tag | ((blockIdx.x == 0 ? kFlagPrefix : kFlagAgg) << kFlagShift) | (unsigned long long)carry);
+    __threadfence();
+    st_relaxed(p.c.status + blockIdx.x, tag | (kFlagAgg << kFlagShift) | (unsigned long long)carry);
   }
   trace_stamp(p.c, 2);
 
-  // (3) dense blocks (no dependency on the scan)
-  for (int32_t d = d0; d < d1; ++d) {
+  // (3) CTA 0 / warp 0 scans the chunk totals once all are published (one
+  // round trip per poll) and writes every chunk's exclusive prefix, then the
+  // scan-done word.
+  if (blockIdx.x == 0 && warp == 0) {
+    const int per = (G + 31) / 32;  // lane owns chunks [lane*per, lane*per + per)
+    while (true) {
+      bool ready = true;
+      for (int j = 0; j < per; ++j) {
+        const int i = lane * per + j;
+        if (i < G) ready &= (ld_relaxed(p.c.status + i) >> kEpochShift) == epoch;
+      }
+      if (__all_sync(0xffffffffu, ready)) break;
+      __nanosleep(100);
+    }
+    __threadfence();
+    long long own = 0;
+    for (int j = 0; j < per; ++j) {
+      const int i = lane * per + j;
+      if (i < G) own += (long long)(ld_relaxed(p.c.status + i) & kValueMask);
+    }
+    long long incl = own;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const long long y = __shfl_up_sync(0xffffffffu, incl, d);
+      if (lane >= d) incl += y;
+    }
+    long long run = incl - own;
+    for (int j = 0; j < per; ++j) {
+      const int i = lane * per + j;
+      if (i < G) {
+        st_relaxed(pref + i, tag | (unsigned long long)run);
+        run += (long long)(ld_relaxed(p.c.status + i) & kValueMask);
+      }
+    }
+    __syncwarp();
+    if (lane == 31) {
+      __threadfence();
+      st_relaxed(pref + G, tag | (unsigned long long)run);  // scan done; value = grand total
+    }
+  }
+
+  // (4) dense blocks from a global queue (CTA units, no dependency on the scan)
+  while (true) {
+    if (tid == 0) s_bcast[1] = (long long)atomicAdd(p.c.sched + 2, 1ull);
+    __syncthreads();
+    const long long d = s_bcast[1];
+    __syncthreads();
+    if (d >= p.c.n_dense_tiles) break;
     const uint32_t gi = (uint32_t)d % (uint32_t)p.c.n_groups;
     dense_block(p, (int)gi, (int64_t)((uint32_t)d / (uint32_t)p.c.n_groups), smem, cs);
     __syncthreads();
   }
   trace_stamp(p.c, 3);
 
-  // (4) chunk base by decoupled look-back over CTAs < blockIdx.x
-  if (warp == 0) {
-    const long long excl = blockIdx.x == 0 ? 0 : lookback(p.c.status, blockIdx.x, carry, epoch, lane);
-    if (lane == 0) s_bcast[0] = excl;
-  }
-  __syncthreads();
-  const long long cbase = s_bcast[0];
-  trace_stamp(p.c, 4);
-
-  // (5) offsets and ids of the chunk's tiles, one warp per tile
+  // (5) sparse value tiles from a global queue (warp units), once the scan is
+  // done; tile base = chunk prefix + chunk-local tile prefix
   {
-    // warp-private scratch in the (dense-block) dynamic smem
+    if (lane == 0) {
+      while ((ld_relaxed(pref + G) >> kEpochShift) != epoch) __nanosleep(64);
+    }
+    __syncwarp();
+    __threadfence();
+    trace_stamp(p.c, 4);
     int32_t* scr = reinterpret_cast<int32_t*>(smem) + warp * (4 * kMaxNgramK * 32);
-    for (int32_t t = s0 + warp; t < s1; t += kWarps) {
-      const uint32_t f = (uint32_t)t / (uint32_t)T;
-      value_tile(p, (int)f, (int64_t)t - (int64_t)f * T, lane, cbase + p.c.tile_sum[t], scr);
+    const int64_t S = p.c.n_sparse_tiles;
+    while (true) {
+      long long t = 0;
+      if (lane == 0) t = (long long)atomicAdd(p.c.sched + 3, 1ull);
+      t = __shfl_sync(0xffffffffu, t, 0);
+      if (t >= S) break;
+      const int f = (int)((uint64_t)t / (uint64_t)T);
+      if (f != fc.f) load_ctx(p, f, fc);
+      const unsigned long long ts = (unsigned long long)p.c.tile_sum[t];
+      const int cid = (int)(ts >> kCidShift);
+      const long long base = (long long)(ld_relaxed(pref + cid) & kValueMask) + (long long)(ts & kLocalMask);
+      value_tile(p, fc, (int64_t)t - (int64_t)f * T, lane, base, scr);
     }
   }
   trace_stamp(p.c, 5);
@@ -1100,10 +1184,15 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
   if (s_last) {
     const bool wrap = epoch >= kEpochMax;
     if (wrap)
-      for (int i = tid; i < (int)gridDim.x; i += kThreads) p.c.status[i] = 0ull;
+      for (int i = tid; i <= (int)gridDim.x; i += kThreads) {
+        p.c.status[i] = 0ull;
+        p.c.status[kMaxCtas + i] = 0ull;
+      }
     __syncthreads();
     if (tid == 0) {
       p.c.sched[0] = 0ull;
+      p.c.sched[2] = 0ull;
+      p.c.sched[3] = 0ull;
       p.c.sched[1] = wrap ? 1ull : epoch + 1ull;
       __threadfence();
     }

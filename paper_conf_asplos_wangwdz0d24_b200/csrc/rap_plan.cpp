@@ -878,13 +878,13 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
   if (blob.empty()) blob.resize(16);
   e = cudaMalloc(&P->blob, blob.size());
   if (e == cudaSuccess) e = cudaMemcpy(P->blob, blob.data(), blob.size(), cudaMemcpyHostToDevice);
-  if (e == cudaSuccess) e = cudaMalloc(&P->d_sched, 2 * sizeof(unsigned long long));
+  if (e == cudaSuccess) e = cudaMalloc(&P->d_sched, 4 * sizeof(unsigned long long));
   if (e == cudaSuccess) {
-    const unsigned long long init[2] = {0ull, 1ull};
+    const unsigned long long init[4] = {0ull, 1ull, 0ull, 0ull};
     e = cudaMemcpy(P->d_sched, init, sizeof(init), cudaMemcpyHostToDevice);
   }
-  if (e == cudaSuccess) e = cudaMalloc(&P->d_status, sizeof(unsigned long long) * kMaxCtas);
-  if (e == cudaSuccess) e = cudaMemset(P->d_status, 0, sizeof(unsigned long long) * kMaxCtas);
+  if (e == cudaSuccess) e = cudaMalloc(&P->d_status, sizeof(unsigned long long) * 2 * kMaxCtas);
+  if (e == cudaSuccess) e = cudaMemset(P->d_status, 0, sizeof(unsigned long long) * 2 * kMaxCtas);
   if (e == cudaSuccess) e = cudaMalloc(&P->d_part, sizeof(Part) * (kMaxCtas + 1));
   if (e == cudaSuccess) e = cudaMalloc(&P->d_err, sizeof(int32_t));
   if (e == cudaSuccess) e = cudaMemset(P->d_err, 0, sizeof(int32_t));
@@ -1085,46 +1085,32 @@ static double dense_row_cost(const rap_plan* P, const DProg& dp) {
   return c + 2.0 * dp.width;
 }
 
-// Per-CTA partition of the launch: contiguous chunks of the feature-major
-// sparse tile sequence plus an even share of the dense blocks, balanced by
-// the cost model.  Recomputed (and uploaded) only when its key changes.
-static rap_status update_partition(rap_plan* P, int64_t B, const int64_t* nnz, int G, cudaStream_t stream) {
+// Per-CTA partition of the length pass: contiguous chunks of the
+// feature-major sparse tile sequence with about the same number of source
+// columns to read (a length tile reads one offsets column per source).  The
+// dense blocks and value tiles are not partitioned: they come from the
+// kernel's global queues.  Recomputed (and uploaded) only when B or the grid
+// changes.
+static rap_status update_partition(rap_plan* P, int64_t B, int G, cudaStream_t stream) {
   const int64_t F = (int64_t)P->souts.size();
   const int64_t T = (B + kTileRows - 1) / kTileRows;
-  const int64_t Tb = (B + kDenseBlockRows - 1) / kDenseBlockRows;
   std::vector<double> key{(double)B, (double)G};
-  for (const SparseOut& so : P->souts)  // mean list lengths, quantised to 1/16
-    key.push_back(std::round(16.0 * expected_len(P, P->chains[so.chain], B, nnz)));
   if (key == P->key_part) return RAP_OK;
-  std::vector<double> tile_cost(F), dense_cost(P->dprogs.size());
+  std::vector<double> tile_cost(F);
   double total = 0;
   for (int64_t f = 0; f < F; ++f) {
-    tile_cost[f] = kTileRows * sparse_row_cost(P, P->chains[P->souts[f].chain], B, nnz);
+    const Chain& ch = P->chains[P->souts[f].chain];
+    tile_cost[f] = 1.0 + (ch.src_kind == SRC_NGRAM ? (double)P->ngrams[ch.src].k : 1.0);
     total += tile_cost[f] * T;
   }
-  for (size_t g = 0; g < P->dprogs.size(); ++g) {
-    dense_cost[g] = kDenseBlockRows * dense_row_cost(P, P->dprogs[g]);
-    total += dense_cost[g] * Tb;
-  }
-  const int64_t D = (int64_t)P->dprogs.size() * Tb;
   const int64_t S = F * T;
   std::vector<Part> part(G + 1);
-  std::vector<double> sbudget(G);
-  double sparse_total = 0, sb_total = 0;
-  for (int64_t f = 0; f < F; ++f) sparse_total += tile_cost[f] * T;
-  for (int i = 0; i <= G; ++i) part[i].d0 = (int32_t)((int64_t)i * D / G);
-  for (int i = 0; i < G; ++i) {
-    double dc = 0;
-    for (int32_t d = part[i].d0; d < part[i + 1].d0; ++d) dc += dense_cost[d % (int64_t)P->dprogs.size()];
-    sbudget[i] = std::max(0.0, total / G - dc);
-    sb_total += sbudget[i];
-  }
-  const double scale = sb_total > 0 ? sparse_total / sb_total : 0;
   double want = 0, cum = 0;
   int64_t t = 0;
   for (int i = 0; i < G; ++i) {
     part[i].s0 = (int32_t)t;
-    want += sbudget[i] * scale;
+    part[i].d0 = 0;
+    want += total / G;
     while (t < S) {
       const double c = tile_cost[t / T];
       if (cum + 0.5 * c > want) break;
@@ -1133,6 +1119,7 @@ static rap_status update_partition(rap_plan* P, int64_t B, const int64_t* nnz, i
     }
   }
   part[G].s0 = (int32_t)S;
+  part[G].d0 = 0;
   P->h_part = part;
   cudaError_t e = cudaMemcpyAsync(P->d_part, P->h_part.data(), sizeof(Part) * (G + 1), cudaMemcpyHostToDevice, stream);
   if (e != cudaSuccess) return cuda_fail(e, "partition upload");
@@ -1184,7 +1171,7 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
   c.tiles_per_feature = T;
   c.n_sparse_tiles = n_sparse_tiles;
   c.n_dense_tiles = n_dense;
-  if ((st = update_partition(P, B, raw->sp_nnz, (int)grid, stream)) != RAP_OK) return st;
+  if ((st = update_partition(P, B, (int)grid, stream)) != RAP_OK) return st;
   c.part = P->d_part;
   c.sched = P->d_sched;
   c.status = P->d_status;

@@ -2,7 +2,7 @@
 """Per-CTA phase timing of one launch (rap_debug_trace; dev tool).
 
 Stamps (%globaltimer, ns): 0 start, 1 lengths done, 2 chunk total published,
-3 dense blocks done, 4 look-back done, 5 values done.
+3 dense queue drained, 4 scan-done seen, 5 value queue drained.
 """
 import os
 import sys
@@ -13,7 +13,7 @@ import torch  # noqa: F401
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_asplos_wangwdz0d24_b200 import rap, synth  # noqa: E402
 
-NAMES = ["start", "lengths", "published", "dense", "lookback", "values"]
+NAMES = ["start", "lengths", "published", "dense", "scanwait", "values"]
 
 
 def main():
