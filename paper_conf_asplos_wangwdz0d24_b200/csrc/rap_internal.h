@@ -147,32 +147,13 @@ struct DProg {
 
 // Work decomposition of one launch.  Sparse tiles are
 // (output f, 128-row range rt), numbered feature-major t = f * T + rt, which
-// is also the order of the jagged scan (R17).  The planner's cost model cuts
-// [0, S) into one contiguous chunk per CTA for the length pass (cost ~ source
-// columns read).  CTA i then: (1) computes the output lengths of its chunk
-// (one warp per tile, tiles taken from a CTA-local counter) and their
-// chunk-local exclusive prefixes, tagged with i, into tile_sum; (2) publishes
-// the chunk total; (3) CTA 0 / warp 0 scans all chunk totals into per-chunk
-// prefixes and raises a scan-done word; (4) every CTA takes dense blocks
-// (128 rows x one column group) from a global queue; (5) every warp takes
-// value tiles from a global queue and writes offsets and ids at
-// prefix[chunk(t)] + tile_sum[t].  No grid barrier; the queues balance the
-// heavy phases whatever the cost model's error.
-constexpr int kMaxCtas = 2048;        // look-back words / partition entries a plan allocates
+// is also the order of the jagged scan (R17).  Warps take sparse tiles from a
+// global queue in that order and resolve each tile's base by a decoupled
+// look-back over per-tile status words; CTAs then take dense blocks (128 rows
+// x one column group) from a second queue.  No grid barrier.
+constexpr int kMaxCtas = 2048;        // grid cap
 constexpr int kTileRows = 128;        // rows of a sparse tile (4 groups of 32)
 constexpr int kDenseBlockRows = 128;  // rows of a dense block (CTA unit)
-
-// Per-CTA partition of the length pass: sparse tiles [s0(i), s0(i+1)); d0 unused (0).
-struct Part {
-  int32_t s0, d0;
-};
-
-// Look-back status word: [63:44] epoch, [43:42] flag, [41:0] value.
-constexpr int kEpochShift = 44;
-constexpr int kFlagShift = 42;
-constexpr unsigned long long kValueMask = (1ull << 42) - 1;
-constexpr unsigned long long kFlagAgg = 1, kFlagPrefix = 2;
-constexpr unsigned long long kEpochMax = (1ull << 20) - 1;
 
 // Non-array kernel parameters.
 struct Common {
@@ -187,14 +168,12 @@ struct Common {
   int64_t tiles_per_feature;  // T = ceil(n_rows / kTileRows)
   int64_t n_sparse_tiles;     // S = n_sparse_out * T
   int64_t n_dense_tiles;      // n_groups * ceil(n_rows / kDenseBlockRows)
-  const Part* part;           // [gridDim.x + 1]
-  // sched[0] = CTAs done, sched[1] = epoch of the status words, sched[2] =
-  // dense-block queue head, sched[3] = value-tile queue head; the last CTA
-  // resets the heads and advances the epoch, so launch parameters are
-  // identical from call to call (CUDA-graph replayable).
+  // sched[0] = CTAs done, sched[1] = launch epoch, sched[2] = dense-block
+  // queue head, sched[3] = sparse-tile queue head; the last CTA resets the
+  // heads and advances the epoch, so launch parameters are identical from
+  // call to call (CUDA-graph replayable).
   unsigned long long* sched;
-  unsigned long long* status;  // [kMaxCtas] chunk totals, then [kMaxCtas] chunk prefixes (+ scan-done word)
-  int64_t* tile_sum;           // [S] tile length sums -> ([63:48] chunk, [47:0] chunk-local exclusive prefix)
+  unsigned long long* status;  // [S] look-back words, one per sparse tile
   float* dense_out;
   int64_t ld;
   int32_t* lengths;
@@ -226,8 +205,8 @@ RAP_HD uint64_t splitmix_H(uint64_t x) {
   return z ^ (z >> 31);
 }
 
-// Launch entry implemented in rap_kernel.cu (cooperative launch: all CTAs
-// co-resident, so the look-back never waits on an unscheduled CTA).
+// Launch entry implemented in rap_kernel.cu (a tile only waits on tiles
+// already taken from the queue, so no co-residency is required).
 // Returns a cudaError_t value.
 int launch_fused(const Common& c, const LaunchRaw& raw, int grid, int smem_bytes, void* stream);
 // Dynamic shared memory per CTA for dense groups up to max_width columns.

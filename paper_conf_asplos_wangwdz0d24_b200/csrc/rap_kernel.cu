@@ -1,25 +1,22 @@
 // rap_kernel.cu — the fused, persistent sm_100a preprocessing kernel.
 //
-// One cooperative launch processes a whole raw batch (§6.1
-// L1161-1174: horizontal fusion of the per-feature kernels; here every op of
-// every feature runs in one persistent kernel, so the chains are fused
-// vertically as well and no intermediate touches HBM).  The jagged offsets
-// are a global exclusive scan over (feature, row) in feature-major order
-// (R17), so the launch runs in three phases separated by two self-resetting
-// grid barriers:
-//   phase 1  every warp computes the output lengths of 128-row sparse tiles
-//            (closed form from the Arrow offsets and validity words), writes
-//            them, and records one length sum per tile;
-//   phase 2  every CTA scans its chunk of tile sums;
-//   phase 3  CTAs take work units by ticket: a dense column-group block
-//            (inputs staged by cp.async.bulk onto an mbarrier, evaluated
-//            (row, unit)-parallel into a row-major smem tile, float4 stores),
-//            or 8 consecutive sparse tiles of one feature, one per warp, each
-//            writing its offsets and ids at positions known from phase 2.
-// Warps work on their own tiles without CTA barriers; loads of a tile are
-// issued together (4 row groups per lane) so each warp keeps several
-// independent memory requests in flight.  The grid is capped by the SM
-// budget (§6.2).
+// One launch processes a whole raw batch (§6.1:
+// horizontal fusion of the per-feature kernels; here every op of every
+// feature runs in one persistent kernel, so the chains are fused vertically
+// as well and no intermediate touches HBM).  The jagged offsets are a global
+// exclusive scan over (feature, row) in feature-major order (R17), done in a
+// single pass with a decoupled look-back:
+//   (1) warps take 128-row sparse tiles from a global queue in scan order;
+//       a tile computes its output lengths (closed form from the Arrow
+//       offsets and validity words), publishes their sum, computes its ids
+//       (base-independent), resolves its base from its predecessors' words,
+//       then stores lengths, offsets and ids;
+//   (2) CTAs take dense column-group blocks from a second queue (inputs
+//       staged by cp.async.bulk onto an mbarrier, evaluated (row, unit)-
+//       parallel into a row-major smem tile, float4 stores).
+// No grid barrier and no cross-CTA wait other than the look-back; queue
+// order = scan order, so a tile only ever waits on tiles already taken.  The
+// grid is capped by the SM budget (§6.2).
 //
 // Operator semantics: DESIGN.md §3 readings R1-R20 (Table 1).
 // Nothing here is tensor-core work: the path is integer ALU + a few SFU
@@ -46,9 +43,13 @@ struct KParams {
 
 constexpr int kWarps = kThreads / 32;
 constexpr int kGroups = kTileRows / 32;  // row groups of a sparse tile (one row per lane each)
-constexpr int kMaxGrid = 2048;           // look-back words allocated by the plan
-constexpr int kCidShift = 48;             // tile_sum: [63:48] chunk (CTA) id, [47:0] chunk-local prefix
-constexpr unsigned long long kLocalMask = (1ull << kCidShift) - 1;
+constexpr int kNgScratch = kWarps * 4 * kMaxNgramK * 32 * 4;  // NGram warp scratch (smem, sparse phase)
+// Look-back word: [63:44] epoch, [43:42] flag, [41:0] value.
+constexpr int kEpochShift = 44;
+constexpr int kFlagShift = 42;
+constexpr unsigned long long kValueMask = (1ull << 42) - 1;
+constexpr unsigned long long kFlagAgg = 1, kFlagPrefix = 2;
+constexpr unsigned long long kEpochMax = (1ull << 20) - 1;
 
 __host__ __device__ constexpr int align_up(int x, int a) { return (x + a - 1) / a * a; }
 
@@ -403,6 +404,52 @@ __device__ __forceinline__ int warp_incl_scan(int v, int lane) {
 }
 
 // ----------------------------------------------------------------------------
+// Single-pass jagged scan (R17) over the feature-major sparse tile sequence:
+// decoupled look-back.  Tile t publishes its length total (AGG) as soon as it
+// is known, and later resolves its exclusive prefix by summing its
+// predecessors' words, 32 per round trip, back to the nearest inclusive
+// prefix (PREF), which it then publishes for itself.  Words carry the
+// launch epoch, so they never need clearing between launches.
+struct TileRef {
+  unsigned long long* status;
+  long long t;
+  unsigned long long tag;  // epoch << kEpochShift
+};
+
+__device__ __forceinline__ void publish_agg(const TileRef& tr, long long T, int lane) {
+  if (lane == 0) st_relaxed(tr.status + tr.t, tr.tag | (kFlagAgg << kFlagShift) | (unsigned long long)T);
+}
+
+__device__ __forceinline__ long long tile_lookback(const TileRef& tr, long long T, int lane) {
+  const unsigned long long epoch = tr.tag >> kEpochShift;
+  long long excl = 0;
+  long long top = tr.t - 1;
+  while (top >= 0) {
+    const long long idx = top - lane;
+    unsigned long long w = 0;
+    unsigned pm, take;
+    while (true) {
+      int fl = (int)kFlagPrefix;  // before tile 0: an inclusive prefix of 0
+      w = 0;
+      if (idx >= 0) {
+        w = ld_relaxed(tr.status + idx);
+        fl = (w >> kEpochShift) == epoch ? (int)((w >> kFlagShift) & 3ull) : 0;
+      }
+      pm = __ballot_sync(0xffffffffu, fl == (int)kFlagPrefix);
+      const unsigned zm = __ballot_sync(0xffffffffu, fl == 0);
+      take = pm ? ((pm & (0u - pm)) << 1) - 1u : 0xffffffffu;  // lanes up to the nearest prefix
+      if ((zm & take) == 0) break;
+      __nanosleep(32);
+    }
+    excl += warp_sum64(((take >> lane) & 1u) ? (long long)(w & kValueMask) : 0ll);
+    if (pm) break;
+    top -= 32;
+  }
+  if (lane == 0) st_relaxed(tr.status + tr.t, tr.tag | (kFlagPrefix << kFlagShift) | (unsigned long long)(excl + T));
+  return excl;
+}
+
+// ----------------------------------------------------------------------------
 // Sparse tiles with 4 consecutive rows per lane (rows r0 + 4*lane + k): one
 // 16-byte offsets load, one validity word, 16-byte length / offset stores.
 
@@ -465,69 +512,6 @@ __device__ __forceinline__ bool quad_valid(const Quad& q, int k, int lane) {
   return (q.w >> ((4 * lane + k) & 31)) & 1u;
 }
 
-// Phase 1: output lengths of sparse tile (f, rt) -> lengths[], tile_sum[].
-template <class P>
-__device__ void length_tile(const P& p, const FeatCtx& fc, int64_t rt, int lane) {
-  const int f = fc.f;
-  const SProg& pg = p.c.sprogs[f];
-  const int64_t B = p.c.n_rows;
-  const int64_t r0 = rt * kTileRows;
-  int32_t* lengths = p.c.lengths + (int64_t)f * B;
-  int sum = 0;
-  if (fc.kind == SRC_SPARSE) {
-    const int32_t* off = p.off[fc.src];
-    const Quad q = load_quad(off, p.svalid[fc.src], r0, lane, B, (reinterpret_cast<uintptr_t>(off) & 15) == 0);
-    int32_t l[4];
-#pragma unroll
-    for (int k = 0; k < 4; ++k) {
-      l[k] = quad_len(q, k, lane, r0 + 4 * lane + k, B, fc.xcap, fc.has_fill, fc.null_xcap);
-      sum += l[k];
-    }
-    const int64_t row = r0 + 4 * lane;
-    int32_t* lp = lengths + row;
-    if (row + 4 <= B && (reinterpret_cast<uintptr_t>(lp) & 15) == 0) {
-      *reinterpret_cast<int4*>(lp) = make_int4(l[0], l[1], l[2], l[3]);
-    } else {
-#pragma unroll
-      for (int k = 0; k < 4; ++k)
-        if (row + k < B) lp[k] = l[k];
-    }
-  } else if (fc.kind == SRC_DENSE_BUCKET) {
-#pragma unroll
-    for (int g = 0; g < kGroups; ++g) {
-      const int64_t row = r0 + 32 * g + lane;
-      const int32_t len = (int32_t)min((int64_t)1, fc.xcap);
-      if (row < B) lengths[row] = len;
-      sum += row < B ? len : 0;
-    }
-  } else {
-    const int k = pg.ng.k, n = pg.ng.n;
-    const int64_t xcap = pg.ch.xcap;
-    for (int g = 0; g < kGroups; ++g) {
-      const int64_t row = r0 + 32 * g + lane;
-      const bool inr = row < B;
-      RowIn in[kMaxNgramK];
-#pragma unroll
-      for (int c = 0; c < kMaxNgramK; ++c)
-        if (c < k) in[c] = load_row(p, pg.src[c], row, inr);
-      int tot = 0;
-#pragma unroll
-      for (int c = 0; c < kMaxNgramK; ++c) {
-        if (c < k) {
-          int32_t st;
-          tot += row_len(pg.src[c], in[c], lane, inr, &st);
-        }
-      }
-      const int32_t len = inr ? (int32_t)min((int64_t)max(tot - n + 1, 0), xcap) : 0;
-      if (inr) lengths[row] = len;
-      sum += len;
-    }
-  }
-#pragma unroll
-  for (int d = 16; d >= 1; d >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, d);
-  if (lane == 0) p.c.tile_sum[(int64_t)f * p.c.tiles_per_feature + rt] = sum;
-}
-
 // ----------------------------------------------------------------------------
 // Phase 3: offsets and ids of sparse tile (f, rt), whose first output id goes
 // to values[base].
@@ -535,13 +519,30 @@ template <class P>
 __device__ __noinline__ void value_group_general(const P& p, int f, int64_t row0, int lane, int32_t mylen,
                                                  int32_t myst, int32_t lx, long long gbase);
 template <class P>
-__device__ __noinline__ void value_tile_ngram(const P& p, int f, int64_t rt, int lane, long long base,
+__device__ __noinline__ void value_tile_ngram(const P& p, int f, int64_t rt, int lane, const TileRef& tr,
                                               int32_t* scr);
+
+// Lengths (int4) and offsets (2 x longlong2) of the lane's 4 rows.
+__device__ __forceinline__ void store_quad(int32_t* lp, int64_t* op, int64_t row, int64_t B, const int32_t* l,
+                                           long long lb, const int32_t* e) {
+  if (row + 4 <= B && (reinterpret_cast<uintptr_t>(lp) & 15) == 0 && (reinterpret_cast<uintptr_t>(op) & 15) == 0) {
+    *reinterpret_cast<int4*>(lp) = make_int4(l[0], l[1], l[2], l[3]);
+    reinterpret_cast<longlong2*>(op)[0] = make_longlong2(lb + e[0], lb + e[1]);
+    reinterpret_cast<longlong2*>(op)[1] = make_longlong2(lb + e[2], lb + e[3]);
+  } else {
+#pragma unroll
+    for (int k = 0; k < 4; ++k)
+      if (row + k < B) {
+        lp[k] = l[k];
+        op[k] = lb + e[k];
+      }
+  }
+}
 
 // Specialised tile of a canonical SRC_SPARSE chain (mask MASK); the lane
 // owns rows r0 + 4*lane + k, so its output ids are contiguous.
 template <int MASK, class P>
-__device__ __noinline__ void value_tile_canon(const P& p, const FeatCtx& fc, int64_t rt, int lane, long long base) {
+__device__ __noinline__ void value_tile_canon(const P& p, const FeatCtx& fc, int64_t rt, int lane, const TileRef& tr) {
   const Canon& q = fc.q;
   const int f = fc.f;
   const int64_t B = p.c.n_rows;
@@ -563,36 +564,38 @@ __device__ __noinline__ void value_tile_canon(const P& p, const FeatCtx& fc, int
   }
   const int incl = warp_incl_scan(tot, lane);
   const int L = incl - tot;  // lane exclusive prefix within the tile
-  const long long lb = base + L;
-  // offsets (R17), 16-byte stores when aligned
+  const int T = __shfl_sync(0xffffffffu, incl, 31);
+  publish_agg(tr, T, lane);
+  const bool last = f == p.c.n_sparse_out - 1 && rt == p.c.tiles_per_feature - 1;
+  int32_t* lp = p.c.lengths + (int64_t)f * B + row;
   int64_t* op = p.c.offsets + (int64_t)f * B + row;
-  if (row + 4 <= B && (reinterpret_cast<uintptr_t>(op) & 15) == 0) {
-    reinterpret_cast<longlong2*>(op)[0] = make_longlong2(lb + e[0], lb + e[1]);
-    reinterpret_cast<longlong2*>(op)[1] = make_longlong2(lb + e[2], lb + e[3]);
-  } else {
+  if (__all_sync(0xffffffffu, l[0] <= 1 && l[1] <= 1 && l[2] <= 1 && l[3] <= 1)) {
+    // at most one id per row: the ids are computed before the base is known
+    int64_t v[4];
+#pragma unroll
+    for (int k = 0; k < 4; ++k) v[k] = (l[k] == 1 && quad_valid(qd, k, lane)) ? __ldg(val + qd.a[k]) : fc.fill;
 #pragma unroll
     for (int k = 0; k < 4; ++k)
-      if (row + k < B) op[k] = lb + e[k];
-  }
-  const int T = __shfl_sync(0xffffffffu, incl, 31);
-  if (f == p.c.n_sparse_out - 1 && rt == p.c.tiles_per_feature - 1 && lane == 31) {
-    p.c.offsets[(int64_t)p.c.n_sparse_out * B] = base + T;  // total, R17
-    if (base + T > cap) atomicExch(p.c.err, 1);
-  }
-  if (__all_sync(0xffffffffu, l[0] <= 1 && l[1] <= 1 && l[2] <= 1 && l[3] <= 1)) {
-    // at most one id per row: all raw ids first, then the pipelines
-    int64_t raw[4];
-#pragma unroll
-    for (int k = 0; k < 4; ++k) raw[k] = (l[k] == 1 && quad_valid(qd, k, lane)) ? __ldg(val + qd.a[k]) : fc.fill;
+      if (l[k] == 1) v[k] = canon_apply<MASK>(q, itab, v[k], quad_valid(qd, k, lane) ? 15 : q.null_mask);
+    const long long base = tile_lookback(tr, T, lane);
+    const long long lb = base + L;
+    store_quad(lp, op, row, B, l, lb, e);
 #pragma unroll
     for (int k = 0; k < 4; ++k) {
-      if (l[k] == 1) {
-        const int64_t v = canon_apply<MASK>(q, itab, raw[k], quad_valid(qd, k, lane) ? 15 : q.null_mask);
-        const long long pos = lb + e[k];
-        if (pos < cap) values[pos] = v;
-      }
+      const long long pos = lb + e[k];
+      if (l[k] == 1 && pos < cap) values[pos] = v[k];
+    }
+    if (last && lane == 31) {
+      p.c.offsets[(int64_t)p.c.n_sparse_out * B] = base + T;  // total, R17
+      if (base + T > cap) atomicExch(p.c.err, 1);
     }
     return;
+  }
+  const long long base = tile_lookback(tr, T, lane);
+  store_quad(lp, op, row, B, l, base + L, e);
+  if (last && lane == 31) {
+    p.c.offsets[(int64_t)p.c.n_sparse_out * B] = base + T;
+    if (base + T > cap) atomicExch(p.c.err, 1);
   }
   // multi-id rows: elements in output order; owning lane by a 5-step shuffle
   // search over the lane prefixes, then the row within the lane
@@ -624,84 +627,99 @@ __device__ __noinline__ void value_tile_canon(const P& p, const FeatCtx& fc, int
   }
 }
 
+// Tile of any other SRC_SPARSE / SRC_DENSE_BUCKET chain (op interpreter).
 template <class P>
-__device__ void value_tile(const P& p, const FeatCtx& fc, int64_t rt, int lane, long long base, int32_t* scr) {
-  const int f = fc.f;
+__device__ __noinline__ void value_tile_generic(const P& p, int f, int64_t rt, int lane, const TileRef& tr) {
   const SProg& pg = p.c.sprogs[f];
   const DevOp* ops = prog_ops(pg, p.c.ops);
   const int64_t B = p.c.n_rows;
   const int64_t r0 = rt * kTileRows;
   int64_t* offsets = p.c.offsets + (int64_t)f * B;
+  int32_t* lengths = p.c.lengths + (int64_t)f * B;
   int64_t* values = p.c.values;
   const long long cap = p.c.values_cap;
   const int64_t* itab = p.c.itab;
+  const Chain ch = pg.ch;
+  // all row loads of the tile first (kGroups independent requests per lane)
+  RowIn in[kGroups];
+#pragma unroll
+  for (int g = 0; g < kGroups; ++g) {
+    const int64_t row = r0 + 32 * g + lane;
+    in[g] = load_row(p, ch, row, row < B);
+  }
+  int32_t len[kGroups], st[kGroups], lex[kGroups], gb[kGroups];
+  bool all1 = true;
+  int run = 0;  // tile-relative
+#pragma unroll
+  for (int g = 0; g < kGroups; ++g) {
+    const int64_t row = r0 + 32 * g + lane;
+    len[g] = row_len(ch, in[g], lane, row < B, &st[g]);
+    all1 &= len[g] <= 1;
+    const int incl = warp_incl_scan(len[g], lane);
+    lex[g] = incl - len[g];
+    gb[g] = run;
+    run += __shfl_sync(0xffffffffu, incl, 31);
+  }
+  publish_agg(tr, run, lane);
+  const bool use_pipe = ch.src_kind == SRC_SPARSE && pipe_ok(ops, ch.op_begin, ch.op_end);
+  Pipe pipe;
+  if (use_pipe) load_pipe(pipe, ops, ch.op_begin, ch.op_end, pg.tab_off);
+  const int null_k0 = ch.null_op_begin - ch.op_begin;
+  all1 = __all_sync(0xffffffffu, all1);
+  int64_t v1[kGroups];
+  if (all1) {
+    // one id per row at most: ids computed before the base is known
+#pragma unroll
+    for (int g = 0; g < kGroups; ++g)
+      v1[g] = (len[g] == 1 && st[g] >= 0) ? __ldg(p.val[ch.src] + st[g]) : ch.fill;
+#pragma unroll
+    for (int g = 0; g < kGroups; ++g) {
+      if (len[g] == 1) {
+        const int64_t row = r0 + 32 * g + lane;
+        v1[g] = use_pipe ? run_pipe(pipe, itab, v1[g], st[g] >= 0 ? 0 : null_k0)
+                         : src_value(p, ops, pg.tab_off, ch, st[g], row, 0);
+      }
+    }
+  }
+  const long long base = tile_lookback(tr, run, lane);
+#pragma unroll
+  for (int g = 0; g < kGroups; ++g) {
+    const int64_t row = r0 + 32 * g + lane;
+    if (row < B) {
+      lengths[row] = len[g];
+      offsets[row] = base + gb[g] + lex[g];
+    }
+  }
+  if (f == p.c.n_sparse_out - 1 && rt == p.c.tiles_per_feature - 1 && lane == 0) {
+    p.c.offsets[(int64_t)p.c.n_sparse_out * B] = base + run;  // total, R17
+    if (base + run > cap) atomicExch(p.c.err, 1);
+  }
+  if (all1) {
+#pragma unroll
+    for (int g = 0; g < kGroups; ++g) {
+      const long long pos = base + gb[g] + lex[g];
+      if (len[g] == 1 && pos < cap) values[pos] = v1[g];
+    }
+    return;
+  }
+  // general (multi-id rows): elements in output order, per row group
+#pragma unroll 1
+  for (int g = 0; g < kGroups; ++g)
+    value_group_general(p, f, r0 + 32 * g, lane, len[g], st[g], lex[g], base + gb[g]);
+}
 
+template <class P>
+__device__ __forceinline__ void value_tile(const P& p, const FeatCtx& fc, int64_t rt, int lane, const TileRef& tr,
+                                           int32_t* scr) {
   if (fc.canon) {
-#define RAP_VT_CALL(M) value_tile_canon<M>(p, fc, rt, lane, base)
+#define RAP_VT_CALL(M) value_tile_canon<M>(p, fc, rt, lane, tr)
     RAP_CANON_DISPATCH(fc.mask, RAP_VT_CALL)
 #undef RAP_VT_CALL
-    return;
+  } else if (fc.kind == SRC_NGRAM) {
+    value_tile_ngram(p, fc.f, rt, lane, tr, scr);
+  } else {
+    value_tile_generic(p, fc.f, rt, lane, tr);
   }
-  if (pg.ch.src_kind != SRC_NGRAM) {
-    const Chain ch = pg.ch;
-    // all row loads of the tile first (kGroups independent requests per lane)
-    RowIn in[kGroups];
-#pragma unroll
-    for (int g = 0; g < kGroups; ++g) {
-      const int64_t row = r0 + 32 * g + lane;
-      in[g] = load_row(p, ch, row, row < B);
-    }
-    int32_t len[kGroups], st[kGroups], lex[kGroups];
-    long long gb[kGroups];
-    bool all1 = true;
-    long long run = base;
-#pragma unroll
-    for (int g = 0; g < kGroups; ++g) {
-      const int64_t row = r0 + 32 * g + lane;
-      len[g] = row_len(ch, in[g], lane, row < B, &st[g]);
-      all1 &= len[g] <= 1;
-      const int incl = warp_incl_scan(len[g], lane);
-      lex[g] = incl - len[g];
-      gb[g] = run;
-      run += __shfl_sync(0xffffffffu, incl, 31);
-      if (row < B) offsets[row] = gb[g] + lex[g];
-    }
-    if (f == p.c.n_sparse_out - 1 && rt == p.c.tiles_per_feature - 1 && lane == 0) {
-      p.c.offsets[(int64_t)p.c.n_sparse_out * B] = run;  // total, R17
-      if (run > cap) atomicExch(p.c.err, 1);
-    }
-    const bool use_pipe = ch.src_kind == SRC_SPARSE && pipe_ok(ops, ch.op_begin, ch.op_end);
-    Pipe pipe;
-    if (use_pipe) load_pipe(pipe, ops, ch.op_begin, ch.op_end, pg.tab_off);
-    const int null_k0 = ch.null_op_begin - ch.op_begin;
-    if (__all_sync(0xffffffffu, all1)) {
-      // one id per row at most: every lane owns its rows' output slots
-      int64_t raw[kGroups];
-#pragma unroll
-      for (int g = 0; g < kGroups; ++g)
-        raw[g] = (len[g] == 1 && st[g] >= 0) ? __ldg(p.val[ch.src] + st[g]) : ch.fill;
-#pragma unroll
-      for (int g = 0; g < kGroups; ++g) {
-        if (len[g] == 1) {
-          const int64_t row = r0 + 32 * g + lane;
-          int64_t v;
-          if (use_pipe) {
-            v = run_pipe(pipe, itab, raw[g], st[g] >= 0 ? 0 : null_k0);
-          } else {
-            v = src_value(p, ops, pg.tab_off, ch, st[g], row, 0);
-          }
-          const long long pos = gb[g] + lex[g];
-          if (pos < cap) values[pos] = v;
-        }
-      }
-      return;
-    }
-    // general (multi-id rows): elements in output order, per row group
-#pragma unroll 1
-    for (int g = 0; g < kGroups; ++g) value_group_general(p, f, r0 + 32 * g, lane, len[g], st[g], lex[g], gb[g]);
-    return;
-  }
-  value_tile_ngram(p, f, rt, lane, base, scr);
 }
 
 // Ids of one 32-row group with multi-id rows: elements in output order, the
@@ -747,15 +765,56 @@ __device__ __noinline__ void value_group_general(const P& p, int f, int64_t row0
 // NGram feature tile (R7): per row the k source lists, windows over their
 // concatenation.
 template <class P>
-__device__ __noinline__ void value_tile_ngram(const P& p, int f, int64_t rt, int lane, long long base,
+__device__ __noinline__ void value_tile_ngram(const P& p, int f, int64_t rt, int lane, const TileRef& tr,
                                               int32_t* scr) {
   const SProg& pg = p.c.sprogs[f];
   const DevOp* ops = prog_ops(pg, p.c.ops);
   const int64_t B = p.c.n_rows;
   const int64_t r0 = rt * kTileRows;
   int64_t* offsets = p.c.offsets + (int64_t)f * B;
+  int32_t* lengths = p.c.lengths + (int64_t)f * B;
   int64_t* values = p.c.values;
   const long long cap = p.c.values_cap;
+  // pass 1: the tile's output length total (quad layout: 4 rows per lane,
+  // every source's offsets requested before any is used), published at once
+  long long base;
+  {
+    int32_t tot4[4] = {0, 0, 0, 0};
+#pragma unroll 1
+    for (int c0 = 0; c0 < pg.ng.k; c0 += 4) {  // 4 sources' offsets in flight at a time
+      Quad qs[4];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const int c = c0 + j;
+        if (c < pg.ng.k && pg.src[c].src_kind == SRC_SPARSE) {
+          const int32_t* off = p.off[pg.src[c].src];
+          qs[j] = load_quad(off, p.svalid[pg.src[c].src], r0, lane, B, (reinterpret_cast<uintptr_t>(off) & 15) == 0);
+        }
+      }
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const int c = c0 + j;
+        if (c < pg.ng.k) {
+          const Chain& sc = pg.src[c];
+#pragma unroll
+          for (int q = 0; q < 4; ++q) {
+            const int64_t row = r0 + 4 * lane + q;
+            if (sc.src_kind == SRC_SPARSE)
+              tot4[q] += quad_len(qs[j], q, lane, row, B, sc.xcap, sc.has_fill, sc.null_xcap);
+            else
+              tot4[q] += row < B ? (int32_t)min((int64_t)1, sc.xcap) : 0;
+          }
+        }
+      }
+    }
+    int sum = 0;
+#pragma unroll
+    for (int q = 0; q < 4; ++q)
+      if (r0 + 4 * lane + q < B) sum += (int32_t)min((int64_t)max(tot4[q] - pg.ng.n + 1, 0), pg.ch.xcap);
+    const long long T = warp_sum64(sum);
+    publish_agg(tr, T, lane);
+    base = tile_lookback(tr, T, lane);
+  }
 
   // NGram feature (R7): per row the k source lists, windows over their
   // concatenation.  Per-source (start, length) of the warp's 32 rows live in
@@ -796,7 +855,10 @@ __device__ __noinline__ void value_tile_ngram(const P& p, int f, int64_t rt, int
     const int incl = warp_incl_scan(len, lane);
     const int lx = incl - len;
     const int T = __shfl_sync(0xffffffffu, incl, 31);
-    if (inr) offsets[row] = run + lx;
+    if (inr) {
+      lengths[row] = len;
+      offsets[row] = run + lx;
+    }
     if (canon_all && __all_sync(0xffffffffu, slmax <= 1)) {
       // single-id sources: run each source's canonical pipeline once per row,
       // then hash the windows from the staged ids
@@ -1021,141 +1083,28 @@ template <int MD, int MS>
 __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const __grid_constant__ KParams<MD, MS> p) {
   extern __shared__ __align__(128) unsigned char smem[];
   __shared__ CtaState cs;
-  __shared__ long long s_wtot[kWarps];
-  __shared__ long long s_bcast[2];
+  __shared__ long long s_item;
   __shared__ unsigned long long s_epoch;
   __shared__ int s_last;
-  __shared__ int s_next[1];  // CTA-local length-tile counter
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const int64_t T = p.c.tiles_per_feature;
-  const Part pa = p.c.part[blockIdx.x], pb = p.c.part[blockIdx.x + 1];
-  const int32_t s0 = pa.s0, s1 = pb.s0;
   if (tid == 0) {
     mbar_init(&cs.bar, 1);
     cs.phase = 0;
     s_epoch = ld_relaxed(p.c.sched + 1);
-    s_next[0] = 0;
   }
   __syncthreads();
   trace_stamp(p.c, 0);
-
-  // (1) output lengths of the chunk's sparse tiles, one warp per tile
-  // Warps take tiles from a CTA-local counter (tile costs differ by feature:
-  // NGram tiles cost several plain ones).
-  FeatCtx fc;
-  fc.f = -1;
-  while (true) {
-    int t = 0;
-    if (lane == 0) t = s0 + atomicAdd(&s_next[0], 1);
-    t = __shfl_sync(0xffffffffu, t, 0);
-    if (t >= s1) break;
-    const int f = (int)((uint32_t)t / (uint32_t)T);
-    if (f != fc.f) load_ctx(p, f, fc);  // a chunk spans few features: cached per warp
-    length_tile(p, fc, (int64_t)t - (int64_t)f * T, lane);
-  }
-  __syncthreads();
-  trace_stamp(p.c, 1);
-  // chunk-local exclusive scan of the tile sums (in place)
-  long long carry = 0;
-  for (int32_t b0 = s0; b0 < s1; b0 += kThreads) {
-    const int32_t i = b0 + tid;
-    const long long v = i < s1 ? p.c.tile_sum[i] : 0;
-    long long incl = v;
-#pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-      const long long y = __shfl_up_sync(0xffffffffu, incl, d);
-      if (lane >= d) incl += y;
-    }
-    if (lane == 31) s_wtot[warp] = incl;
-    __syncthreads();
-    long long wpre = 0, btot = 0;
-#pragma unroll
-    for (int q = 0; q < kWarps; ++q) {
-      const long long w = s_wtot[q];
-      if (q < warp) wpre += w;
-      btot += w;
-    }
-    if (i < s1) p.c.tile_sum[i] = (int64_t)(((unsigned long long)blockIdx.x << kCidShift) | (unsigned long long)(carry + wpre + incl - v));
-    carry += btot;
-    __syncthreads();
-  }
-  // (2) publish the chunk total; the chunk's tile prefixes (tile_sum) are
-  // released before it
   const unsigned long long epoch = s_epoch;
-  const unsigned long long tag = epoch << kEpochShift;
-  const int G = (int)gridDim.x;
-  unsigned long long* pref = p.c.status + kMaxCtas;  // [G] chunk prefixes, [G] = scan-done word
-  if (tid == 0) {
-    __threadfence();
-    st_relaxed(p.c.status + blockIdx.x, tag | (kFlagAgg << kFlagShift) | (unsigned long long)carry);
-  }
-  trace_stamp(p.c, 2);
 
-  // (3) CTA 0 / warp 0 scans the chunk totals once all are published (one
-  // round trip per poll) and writes every chunk's exclusive prefix, then the
-  // scan-done word.
-  if (blockIdx.x == 0 && warp == 0) {
-    const int per = (G + 31) / 32;  // lane owns chunks [lane*per, lane*per + per)
-    while (true) {
-      bool ready = true;
-      for (int j = 0; j < per; ++j) {
-        const int i = lane * per + j;
-        if (i < G) ready &= (ld_relaxed(p.c.status + i) >> kEpochShift) == epoch;
-      }
-      if (__all_sync(0xffffffffu, ready)) break;
-      __nanosleep(100);
-    }
-    __threadfence();
-    long long own = 0;
-    for (int j = 0; j < per; ++j) {
-      const int i = lane * per + j;
-      if (i < G) own += (long long)(ld_relaxed(p.c.status + i) & kValueMask);
-    }
-    long long incl = own;
-#pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-      const long long y = __shfl_up_sync(0xffffffffu, incl, d);
-      if (lane >= d) incl += y;
-    }
-    long long run = incl - own;
-    for (int j = 0; j < per; ++j) {
-      const int i = lane * per + j;
-      if (i < G) {
-        st_relaxed(pref + i, tag | (unsigned long long)run);
-        run += (long long)(ld_relaxed(p.c.status + i) & kValueMask);
-      }
-    }
-    __syncwarp();
-    if (lane == 31) {
-      __threadfence();
-      st_relaxed(pref + G, tag | (unsigned long long)run);  // scan done; value = grand total
-    }
-  }
-
-  // (4) dense blocks from a global queue (CTA units, no dependency on the scan)
-  while (true) {
-    if (tid == 0) s_bcast[1] = (long long)atomicAdd(p.c.sched + 2, 1ull);
-    __syncthreads();
-    const long long d = s_bcast[1];
-    __syncthreads();
-    if (d >= p.c.n_dense_tiles) break;
-    const uint32_t gi = (uint32_t)d % (uint32_t)p.c.n_groups;
-    dense_block(p, (int)gi, (int64_t)((uint32_t)d / (uint32_t)p.c.n_groups), smem, cs);
-    __syncthreads();
-  }
-  trace_stamp(p.c, 3);
-
-  // (5) sparse value tiles from a global queue (warp units), once the scan is
-  // done; tile base = chunk prefix + chunk-local tile prefix
+  // (1) sparse tiles (warp units) from a global queue, in scan order
   {
-    if (lane == 0) {
-      while ((ld_relaxed(pref + G) >> kEpochShift) != epoch) __nanosleep(64);
-    }
-    __syncwarp();
-    __threadfence();
-    trace_stamp(p.c, 4);
+    FeatCtx fc;
+    fc.f = -1;
     int32_t* scr = reinterpret_cast<int32_t*>(smem) + warp * (4 * kMaxNgramK * 32);
-    const int64_t S = p.c.n_sparse_tiles;
+    const int64_t S = p.c.n_sparse_tiles, T = p.c.tiles_per_feature;
+    TileRef tr;
+    tr.status = p.c.status;
+    tr.tag = epoch << kEpochShift;
     while (true) {
       long long t = 0;
       if (lane == 0) t = (long long)atomicAdd(p.c.sched + 3, 1ull);
@@ -1163,16 +1112,29 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
       if (t >= S) break;
       const int f = (int)((uint64_t)t / (uint64_t)T);
       if (f != fc.f) load_ctx(p, f, fc);
-      const unsigned long long ts = (unsigned long long)p.c.tile_sum[t];
-      const int cid = (int)(ts >> kCidShift);
-      const long long base = (long long)(ld_relaxed(pref + cid) & kValueMask) + (long long)(ts & kLocalMask);
-      value_tile(p, fc, (int64_t)t - (int64_t)f * T, lane, base, scr);
+      tr.t = t;
+      value_tile(p, fc, (int64_t)t - (int64_t)f * T, lane, tr, scr);
     }
   }
-  trace_stamp(p.c, 5);
+  trace_stamp(p.c, 1);
+  __syncthreads();
 
-  // The last CTA out advances the epoch of the look-back words (clearing
-  // them when the 20-bit epoch wraps) and resets the done counter.
+  // (2) dense blocks (CTA units) from a second global queue
+  while (true) {
+    if (tid == 0) s_item = (long long)atomicAdd(p.c.sched + 2, 1ull);
+    __syncthreads();
+    const long long d = s_item;
+    __syncthreads();
+    if (d >= p.c.n_dense_tiles) break;
+    const uint32_t gi = (uint32_t)d % (uint32_t)p.c.n_groups;
+    dense_block(p, (int)gi, (int64_t)((uint32_t)d / (uint32_t)p.c.n_groups), smem, cs);
+    __syncthreads();
+  }
+  trace_stamp(p.c, 2);
+
+  // The last CTA out resets the queue heads and advances the epoch of the
+  // look-back words (clearing them when the 20-bit epoch wraps), so launch
+  // parameters are identical from call to call (CUDA-graph replayable).
   __syncthreads();
   if (tid == 0) {
     __threadfence();
@@ -1184,10 +1146,7 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
   if (s_last) {
     const bool wrap = epoch >= kEpochMax;
     if (wrap)
-      for (int i = tid; i <= (int)gridDim.x; i += kThreads) {
-        p.c.status[i] = 0ull;
-        p.c.status[kMaxCtas + i] = 0ull;
-      }
+      for (int64_t i = tid; i < p.c.n_sparse_tiles; i += kThreads) p.c.status[i] = 0ull;
     __syncthreads();
     if (tid == 0) {
       p.c.sched[0] = 0ull;
@@ -1225,11 +1184,7 @@ static int launch_t(const Common& c, const LaunchRaw& raw, int grid, int smem, c
   cfg.blockDim = dim3(kThreads);
   cfg.dynamicSmemBytes = smem;
   cfg.stream = st;
-  cudaLaunchAttribute attr[1];
-  attr[0].id = cudaLaunchAttributeCooperative;  // co-residency for the grid barriers
-  attr[0].val.cooperative = 1;
-  cfg.attrs = attr;
-  cfg.numAttrs = 1;
+  cfg.numAttrs = 0;
   cudaError_t e = cudaLaunchKernelEx(&cfg, rap_fused_kernel<MD, MS>, p);
   if (e != cudaSuccess) return (int)e;
   return (int)cudaGetLastError();
@@ -1237,7 +1192,7 @@ static int launch_t(const Common& c, const LaunchRaw& raw, int grid, int smem, c
 
 int launch_fused(const Common& c, const LaunchRaw& raw, int grid, int smem_bytes, void* stream) {
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
-  if (grid > kMaxGrid) return (int)cudaErrorInvalidValue;
+  if (grid > kMaxCtas) return (int)cudaErrorInvalidValue;
   if (raw.n_dense <= 32 && raw.n_sparse <= 64) return launch_t<32, 64>(c, raw, grid, smem_bytes, st);
   if (raw.n_dense <= 128 && raw.n_sparse <= 1024) return launch_t<128, 1024>(c, raw, grid, smem_bytes, st);
   return (int)cudaErrorInvalidValue;
@@ -1246,8 +1201,7 @@ int launch_fused(const Common& c, const LaunchRaw& raw, int grid, int smem_bytes
 int fused_smem_bytes(int max_width) {
   const int tile = kDenseBlockRows * (max_width | 1) * 4;
   const int dense = kDProgBytes + dense_in_bytes() + align_up(tile, 16);
-  const int ngram_scratch = kWarps * 4 * kMaxNgramK * 32 * 4;  // value_tile_ngram warp scratch
-  return dense > ngram_scratch ? dense : ngram_scratch;
+  return dense > kNgScratch ? dense : kNgScratch;
 }
 
 int fused_occupancy(int smem_bytes, int n_dense, int n_sparse, int* ctas_per_sm) {

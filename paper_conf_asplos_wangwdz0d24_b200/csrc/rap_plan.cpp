@@ -85,16 +85,12 @@ struct rap_plan {
   unsigned char* blob = nullptr;
   size_t off_ops = 0, off_sprogs = 0, off_oprogs = 0, off_dprogs = 0, off_ftab = 0, off_itab = 0;
   // per-n_rows descriptor table
-  int64_t* d_tile_sum = nullptr;   // per sparse tile length sums (scan scratch)
-  int64_t tile_cap = 0;
   // per-CTA partition (cost model), cached by its key
-  Part* d_part = nullptr;
-  std::vector<Part> h_part;
-  std::vector<double> key_part;
   std::vector<double> sparse_row_cost, dense_row_cost;
   // scheduling state
   unsigned long long* d_sched = nullptr;   // CTAs done, look-back epoch
-  unsigned long long* d_status = nullptr;  // look-back words, one per CTA
+  unsigned long long* d_status = nullptr;  // look-back words, one per sparse tile (grows)
+  int64_t status_cap = 0;
   int32_t* d_err = nullptr;
   int64_t n_launches = 0;
   int64_t last_n_desc = 0;
@@ -878,14 +874,11 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
   if (blob.empty()) blob.resize(16);
   e = cudaMalloc(&P->blob, blob.size());
   if (e == cudaSuccess) e = cudaMemcpy(P->blob, blob.data(), blob.size(), cudaMemcpyHostToDevice);
-  if (e == cudaSuccess) e = cudaMalloc(&P->d_sched, 4 * sizeof(unsigned long long));
+  if (e == cudaSuccess) e = cudaMalloc(&P->d_sched, 8 * sizeof(unsigned long long));
   if (e == cudaSuccess) {
-    const unsigned long long init[4] = {0ull, 1ull, 0ull, 0ull};
+    const unsigned long long init[8] = {0ull, 0ull, 0ull, 0ull, 0ull, 0ull, 0ull, 0ull};
     e = cudaMemcpy(P->d_sched, init, sizeof(init), cudaMemcpyHostToDevice);
   }
-  if (e == cudaSuccess) e = cudaMalloc(&P->d_status, sizeof(unsigned long long) * 2 * kMaxCtas);
-  if (e == cudaSuccess) e = cudaMemset(P->d_status, 0, sizeof(unsigned long long) * 2 * kMaxCtas);
-  if (e == cudaSuccess) e = cudaMalloc(&P->d_part, sizeof(Part) * (kMaxCtas + 1));
   if (e == cudaSuccess) e = cudaMalloc(&P->d_err, sizeof(int32_t));
   if (e == cudaSuccess) e = cudaMemset(P->d_err, 0, sizeof(int32_t));
   if (e != cudaSuccess) {
@@ -914,9 +907,7 @@ void rap_plan_destroy(rap_plan* P) {
   cudaFree(P->blob);
   cudaFree(P->d_sched);
   cudaFree(P->d_status);
-  cudaFree(P->d_part);
   cudaFree(P->d_err);
-  cudaFree(P->d_tile_sum);
   cudaFree(P->d_trace);
   for (void* s : P->stage) cudaFree(s);
   delete P;
@@ -1085,48 +1076,6 @@ static double dense_row_cost(const rap_plan* P, const DProg& dp) {
   return c + 2.0 * dp.width;
 }
 
-// Per-CTA partition of the length pass: contiguous chunks of the
-// feature-major sparse tile sequence with about the same number of source
-// columns to read (a length tile reads one offsets column per source).  The
-// dense blocks and value tiles are not partitioned: they come from the
-// kernel's global queues.  Recomputed (and uploaded) only when B or the grid
-// changes.
-static rap_status update_partition(rap_plan* P, int64_t B, int G, cudaStream_t stream) {
-  const int64_t F = (int64_t)P->souts.size();
-  const int64_t T = (B + kTileRows - 1) / kTileRows;
-  std::vector<double> key{(double)B, (double)G};
-  if (key == P->key_part) return RAP_OK;
-  std::vector<double> tile_cost(F);
-  double total = 0;
-  for (int64_t f = 0; f < F; ++f) {
-    const Chain& ch = P->chains[P->souts[f].chain];
-    tile_cost[f] = 1.0 + (ch.src_kind == SRC_NGRAM ? (double)P->ngrams[ch.src].k : 1.0);
-    total += tile_cost[f] * T;
-  }
-  const int64_t S = F * T;
-  std::vector<Part> part(G + 1);
-  double want = 0, cum = 0;
-  int64_t t = 0;
-  for (int i = 0; i < G; ++i) {
-    part[i].s0 = (int32_t)t;
-    part[i].d0 = 0;
-    want += total / G;
-    while (t < S) {
-      const double c = tile_cost[t / T];
-      if (cum + 0.5 * c > want) break;
-      cum += c;
-      ++t;
-    }
-  }
-  part[G].s0 = (int32_t)S;
-  part[G].d0 = 0;
-  P->h_part = part;
-  cudaError_t e = cudaMemcpyAsync(P->d_part, P->h_part.data(), sizeof(Part) * (G + 1), cudaMemcpyHostToDevice, stream);
-  if (e != cudaSuccess) return cuda_fail(e, "partition upload");
-  P->key_part = key;
-  return RAP_OK;
-}
-
 static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output* out, cudaStream_t stream) {
   const int64_t B = raw->n_rows;
   cudaError_t e;
@@ -1138,25 +1087,27 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
     return RAP_OK;
   }
   // Work decomposition: 128-row sparse tiles per output,
-  // 128-row dense blocks per column group; one length sum per sparse tile.
+  // 128-row dense blocks per column group; one look-back word per sparse tile.
   const int64_t F = (int64_t)P->souts.size();
   const int64_t T = (B + kTileRows - 1) / kTileRows;
   const int64_t n_sparse_tiles = F * T;
   const int64_t n_dense = P->dprogs.empty() ? 0 : (int64_t)P->dprogs.size() * ((B + kDenseBlockRows - 1) / kDenseBlockRows);
   if (n_sparse_tiles == 0 && n_dense == 0) return RAP_OK;
   const int64_t grid = std::min<int64_t>((int64_t)P->budget * P->ctas_per_sm, kMaxCtas);
-  rap_status st;
-  if (n_sparse_tiles > P->tile_cap) {  // scan scratch (grows, never shrinks)
-    if (P->d_tile_sum) {
+  if (n_sparse_tiles > P->status_cap) {  // look-back words (grow, never shrink; zero = no epoch)
+    if (P->d_status) {
       e = cudaStreamSynchronize(stream);
       if (e != cudaSuccess) return cuda_fail(e, "cudaStreamSynchronize");
-      cudaFree(P->d_tile_sum);
-      P->d_tile_sum = nullptr;
+      cudaFree(P->d_status);
+      P->d_status = nullptr;
+      P->status_cap = 0;
     }
     const int64_t cap = std::max<int64_t>(n_sparse_tiles, 4096);
-    e = cudaMalloc(&P->d_tile_sum, sizeof(int64_t) * cap);
-    if (e != cudaSuccess) return fail(RAP_ERR_OUT_OF_MEMORY, "scan scratch allocation");
-    P->tile_cap = cap;
+    e = cudaMalloc(&P->d_status, sizeof(unsigned long long) * cap);
+    if (e != cudaSuccess) return fail(RAP_ERR_OUT_OF_MEMORY, "look-back word allocation");
+    e = cudaMemsetAsync(P->d_status, 0, sizeof(unsigned long long) * cap, stream);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync");
+    P->status_cap = cap;
   }
   Common c{};
   c.ops = reinterpret_cast<const DevOp*>(P->blob + P->off_ops);
@@ -1171,11 +1122,8 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
   c.tiles_per_feature = T;
   c.n_sparse_tiles = n_sparse_tiles;
   c.n_dense_tiles = n_dense;
-  if ((st = update_partition(P, B, (int)grid, stream)) != RAP_OK) return st;
-  c.part = P->d_part;
   c.sched = P->d_sched;
   c.status = P->d_status;
-  c.tile_sum = P->d_tile_sum;
   c.dense_out = out->dense_out;
   c.ld = out->dense_ld;
   c.lengths = out->lengths;

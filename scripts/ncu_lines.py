@@ -70,6 +70,28 @@ def main():
     print(f"{'line':32s} {'stall%':>7s} {'winstr%':>8s} {'winstr':>12s}")
     for k, v in sorted(agg.items(), key=lambda kv: -kv[1][0])[:top]:
         print(f"{k:32s} {100 * v[0] / max(tot[0], 1):7.2f} {100 * v[1] / max(tot[1], 1):8.2f} {v[1]:12d}")
+    src = os.environ.get("SRC")  # optional: per-function totals (function = last definition above the line)
+    if src:
+        starts = []
+        for i, ln in enumerate(open(src).read().splitlines(), 1):
+            m = re.match(r"^(?:__device__|__global__|template|static|[a-z_]+ )[^;{]*?([A-Za-z_0-9]+)\(", ln)
+            if m and not ln.startswith("template"):
+                starts.append((i, m.group(1)))
+        fn = collections.defaultdict(lambda: [0, 0])
+        for k, v in agg.items():
+            f = "?"
+            if k and k.split(":")[0] == os.environ.get("SRCNAME", os.path.basename(src)):
+                n = int(k.split(":")[1])
+                for i, name in starts:
+                    if i <= n:
+                        f = name
+            elif k:
+                f = k.split(":")[0]
+            fn[f][0] += v[0]
+            fn[f][1] += v[1]
+        print(f"\n{'function':32s} {'stall%':>7s} {'winstr%':>8s}")
+        for k, v in sorted(fn.items(), key=lambda kv: -kv[1][1])[:top]:
+            print(f"{k:32s} {100 * v[0] / max(tot[0], 1):7.2f} {100 * v[1] / max(tot[1], 1):8.2f}")
 
 
 if __name__ == "__main__":

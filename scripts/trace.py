@@ -1,8 +1,8 @@
 #!/usr/bin/env python
 """Per-CTA phase timing of one launch (rap_debug_trace; dev tool).
 
-Stamps (%globaltimer, ns): 0 start, 1 lengths done, 2 chunk total published,
-3 dense queue drained, 4 scan-done seen, 5 value queue drained.
+Stamps (%globaltimer, ns): 0 start, 1 sparse-tile queue drained, 2 dense
+queue drained.
 """
 import os
 import sys
@@ -13,7 +13,7 @@ import torch  # noqa: F401
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_asplos_wangwdz0d24_b200 import rap, synth  # noqa: E402
 
-NAMES = ["start", "lengths", "published", "dense", "scanwait", "values"]
+NAMES = ["start", "sparse", "dense"]
 
 
 def main():
@@ -38,9 +38,9 @@ def main():
         plan.preprocess(raw, out)
     tr = plan.trace_read(4096)[: info["grid"]].astype(np.int64)
     t0 = tr[:, 0].min()
-    rel = (tr[:, :6] - t0) / 1e3
-    print(f"{os.environ.get('KEEP', 'all')}: grid {info['grid']}  kernel span {rel[:, 5].max():.2f} us")
-    for k in range(1, 6):
+    rel = (tr[:, :3] - t0) / 1e3
+    print(f"{os.environ.get('KEEP', 'all')}: grid {info['grid']}  kernel span {rel[:, 2].max():.2f} us")
+    for k in range(1, 3):
         d = rel[:, k] - rel[:, k - 1]
         print(f"  {NAMES[k - 1]:>9s}->{NAMES[k]:<9s} median {np.median(d):7.2f}  min {d.min():7.2f}  "
               f"max {d.max():7.2f}   (abs end: median {np.median(rel[:, k]):7.2f} max {rel[:, k].max():7.2f})")
