@@ -145,12 +145,14 @@ struct DProg {
   float ftab[kDenseTabF];
 };
 
-// Work decomposition of one launch.  Sparse tiles are
-// (output f, 128-row range rt), numbered feature-major t = f * T + rt, which
-// is also the order of the jagged scan (R17).  Warps take sparse tiles from a
-// global queue in that order and resolve each tile's base by a decoupled
-// look-back over per-tile status words; CTAs then take dense blocks (128 rows
-// x one column group) from a second queue.  No grid barrier.
+// Work decomposition of one launch.  Units are the sparse
+// tiles (output f, 128-row range rt), numbered feature-major t = f * T + rt
+// (the order of the jagged scan, R17), followed by the dense blocks (128 rows
+// x one column group).  The host splits the unit sequence into one
+// contiguous, cost-balanced range per CTA (Common::part); a CTA sums its
+// sparse tiles' output lengths, publishes that aggregate, runs its dense
+// blocks, adds its predecessors' aggregates and then writes its tiles.  No
+// grid barrier, no per-tile look-back.
 constexpr int kMaxCtas = 2048;        // grid cap
 constexpr int kTileRows = 128;        // rows of a sparse tile (4 groups of 32)
 constexpr int kDenseBlockRows = 128;  // rows of a dense block (CTA unit)
@@ -168,12 +170,13 @@ struct Common {
   int64_t tiles_per_feature;  // T = ceil(n_rows / kTileRows)
   int64_t n_sparse_tiles;     // S = n_sparse_out * T
   int64_t n_dense_tiles;      // n_groups * ceil(n_rows / kDenseBlockRows)
-  // sched[0] = CTAs done, sched[1] = launch epoch, sched[2] = dense-block
-  // queue head, sched[3] = sparse-tile queue head; the last CTA resets the
-  // heads and advances the epoch, so launch parameters are identical from
-  // call to call (CUDA-graph replayable).
+  // sched[0] = CTAs done, sched[1] = launch epoch, sched[2] = rank counter
+  // (arrival order); the last CTA resets the counters and advances the
+  // epoch, so launch parameters are identical from call to call (CUDA-graph
+  // replayable).
   unsigned long long* sched;
-  unsigned long long* status;  // [S] look-back words, one per sparse tile
+  const int64_t* part;         // [grid + 1] unit range of each CTA rank
+  unsigned long long* agg;     // [kMaxCtas] per-rank aggregate words (epoch-tagged)
   float* dense_out;
   int64_t ld;
   int32_t* lengths;
@@ -186,7 +189,7 @@ struct Common {
   int64_t trace_cap;
 };
 
-constexpr int kTracePts = 8;
+constexpr int kTracePts = 16;
 
 struct LaunchRaw {
   int32_t n_dense, n_sparse;
@@ -205,8 +208,8 @@ RAP_HD uint64_t splitmix_H(uint64_t x) {
   return z ^ (z >> 31);
 }
 
-// Launch entry implemented in rap_kernel.cu (a tile only waits on tiles
-// already taken from the queue, so no co-residency is required).
+// Launch entry implemented in rap_kernel.cu (a CTA only waits on CTAs that
+// took a lower rank, i.e. are already resident: no co-residency is required).
 // Returns a cudaError_t value.
 int launch_fused(const Common& c, const LaunchRaw& raw, int grid, int smem_bytes, void* stream);
 // Dynamic shared memory per CTA for dense groups up to max_width columns.

@@ -44,12 +44,11 @@ struct KParams {
 constexpr int kWarps = kThreads / 32;
 constexpr int kGroups = kTileRows / 32;  // row groups of a sparse tile (one row per lane each)
 constexpr int kNgScratch = kWarps * 4 * kMaxNgramK * 32 * 4;  // NGram warp scratch (smem, sparse phase)
-// Look-back word: [63:44] epoch, [43:42] flag, [41:0] value.
+// Aggregate word of a CTA: [63:44] tag = launch epoch + 1 (0 = never
+// written), [43:0] the CTA's output length total.
 constexpr int kEpochShift = 44;
-constexpr int kFlagShift = 42;
-constexpr unsigned long long kValueMask = (1ull << 42) - 1;
-constexpr unsigned long long kFlagAgg = 1, kFlagPrefix = 2;
-constexpr unsigned long long kEpochMax = (1ull << 20) - 1;
+constexpr unsigned long long kValueMask = (1ull << kEpochShift) - 1;
+constexpr unsigned long long kEpochMax = (1ull << 20) - 2;
 
 __host__ __device__ constexpr int align_up(int x, int a) { return (x + a - 1) / a * a; }
 
@@ -77,6 +76,16 @@ __device__ __forceinline__ void trace_stamp(const Common& c, int k) {
     unsigned long long v;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(v));
     c.trace[(int64_t)blockIdx.x * kTracePts + k] = v;
+  }
+}
+
+// Profiling aid: clock64 at slot k of this CTA's trace row, once per launch
+// (first call wins), after the value `dep` is available.
+__device__ __forceinline__ void trace_clk(const Common& c, int k, long long dep) {
+  if (c.trace != nullptr && threadIdx.x == 0 && (int64_t)blockIdx.x < c.trace_cap) {
+    asm volatile("" ::"l"(dep));
+    unsigned long long* slot = c.trace + (int64_t)blockIdx.x * kTracePts + k;
+    if (*slot == 0) *slot = clock64();
   }
 }
 
@@ -250,42 +259,101 @@ __device__ __forceinline__ int64_t run_pipe(const Pipe& pp, const int64_t* itab,
   return v;
 }
 
-// Canonical pipeline (rap_internal.h): the stages present in MASK, in the
-// fixed order Clamp -> MapId -> SigridHash -> Bucketize; `active` selects the
-// stages of this element (all for a valid row, null_mask for a filled row).
-template <int MASK>
-__device__ __forceinline__ int64_t canon_apply(const Canon& q, const int64_t* itab, int64_t v, int active) {
-  if ((MASK & CB_CLAMP) && (active & CB_CLAMP)) {  // R6
-    v = v < q.lo ? q.lo : v;
-    v = v > q.hi ? q.hi : v;
+// Batched forms for N independent elements: every step issues N independent
+// loads before any is consumed (memory-level parallelism instead of N
+// serial probe chains).
+template <int N>
+__device__ __forceinline__ void map_lookup_n(const int64_t* itab, int64_t a, int m, int64_t dflt, int64_t (&v)[N],
+                                             unsigned act) {  // R8, no INT64_MIN key
+  const longlong2* t = reinterpret_cast<const longlong2*>(itab + a);
+  const uint32_t mask = (1u << m) - 1u;
+  uint32_t idx[N];
+  longlong2 kv[N];
+#pragma unroll
+  for (int j = 0; j < N; ++j) {
+    idx[j] = (uint32_t)(((uint64_t)v[j] * 0x9E3779B97F4A7C15ull) >> (64 - m));
+    kv[j] = ((act >> j) & 1u) ? __ldg(t + idx[j]) : make_longlong2(INT64_MIN, 0);
   }
-  if ((MASK & CB_MAPID) && (active & CB_MAPID)) v = map_lookup(itab, q.map_a, q.map_m, q.map_def, 0, 0, v);  // R8
-  if ((MASK & CB_SIGRID) && (active & CB_SIGRID))
-    v = (int64_t)reduce_M(splitmix_H(q.hs ^ (uint64_t)v), q.M);                    // R3
-  if ((MASK & CB_BUCKET) && (active & CB_BUCKET)) v = upper_bound(itab + q.bk_a, q.bk_m, v);  // R4
-  return v;
+#pragma unroll
+  for (int j = 0; j < N; ++j) {
+    if (!((act >> j) & 1u)) continue;
+    if (v[j] == INT64_MIN) {
+      v[j] = dflt;
+      continue;
+    }
+    while (true) {
+      if (kv[j].x == v[j]) {
+        v[j] = kv[j].y;
+        break;
+      }
+      if (kv[j].x == INT64_MIN) {
+        v[j] = dflt;
+        break;
+      }
+      idx[j] = (idx[j] + 1) & mask;
+      kv[j] = __ldg(t + idx[j]);
+    }
+  }
 }
 
-// Calls body.template operator()<MASK>() for the runtime mask (16 cases).
-#define RAP_CANON_DISPATCH(mask, CALL)   \
-  switch ((mask) & 15) {                 \
-    case 0: CALL(0); break;              \
-    case 1: CALL(1); break;              \
-    case 2: CALL(2); break;              \
-    case 3: CALL(3); break;              \
-    case 4: CALL(4); break;              \
-    case 5: CALL(5); break;              \
-    case 6: CALL(6); break;              \
-    case 7: CALL(7); break;              \
-    case 8: CALL(8); break;              \
-    case 9: CALL(9); break;              \
-    case 10: CALL(10); break;            \
-    case 11: CALL(11); break;            \
-    case 12: CALL(12); break;            \
-    case 13: CALL(13); break;            \
-    case 14: CALL(14); break;            \
-    default: CALL(15); break;            \
+// #{i : b[i] <= x} over sorted b[0..m), m >= 1, branchless with a uniform
+// step count (R4).
+template <int N>
+__device__ __forceinline__ void upper_bound_n(const int64_t* b, int m, int64_t (&v)[N], unsigned act) {
+  int base[N];
+#pragma unroll
+  for (int j = 0; j < N; ++j) base[j] = 0;
+  int n = m;
+  while (n > 1) {
+    const int half = n >> 1;
+#pragma unroll
+    for (int j = 0; j < N; ++j) base[j] += (__ldg(b + base[j] + half) <= v[j]) ? half : 0;
+    n -= half;
   }
+#pragma unroll
+  for (int j = 0; j < N; ++j)
+    if ((act >> j) & 1u) v[j] = base[j] + (__ldg(b + base[j]) <= v[j] ? 1 : 0);
+}
+
+// Canonical pipeline (rap_internal.h) over N elements: the stages in q.mask,
+// in the fixed order Clamp -> MapId -> SigridHash -> Bucketize.  act[j] =
+// element j is processed; full[j] = it runs every stage (a valid row) rather
+// than q.null_mask (a filled null, R10).  The mask is warp-uniform, so the
+// stage tests are uniform branches (one code copy, no per-mask variants:
+// instruction-cache footprint matters more than the tests).
+template <int N>
+__device__ __forceinline__ void canon_apply_n(const Canon& q, const int64_t* itab, int64_t (&v)[N], unsigned act,
+                                              unsigned full) {
+  // element j runs stage X iff act bit j and (full bit j or X in null_mask)
+  const unsigned nul = act & ~full;
+  if (q.mask & CB_CLAMP) {  // R6
+    const unsigned on = (q.null_mask & CB_CLAMP) ? act : (act & full);
+#pragma unroll
+    for (int j = 0; j < N; ++j)
+      if ((on >> j) & 1u) {
+        v[j] = v[j] < q.lo ? q.lo : v[j];
+        v[j] = v[j] > q.hi ? q.hi : v[j];
+      }
+  }
+  if (q.mask & CB_MAPID)  // R8
+    map_lookup_n<N>(itab, q.map_a, q.map_m, q.map_def, v, (q.null_mask & CB_MAPID) ? act : (act & full));
+  if (q.mask & CB_SIGRID) {  // R3
+    const unsigned on = (q.null_mask & CB_SIGRID) ? act : (act & full);
+#pragma unroll
+    for (int j = 0; j < N; ++j)
+      if ((on >> j) & 1u) v[j] = (int64_t)reduce_M(splitmix_H(q.hs ^ (uint64_t)v[j]), q.M);
+  }
+  if (q.mask & CB_BUCKET)  // R4
+    upper_bound_n<N>(itab + q.bk_a, q.bk_m, v, (q.null_mask & CB_BUCKET) ? act : (act & full));
+  (void)nul;
+}
+
+// One element through the canonical pipeline (not inlined: cold paths).
+__device__ __noinline__ int64_t canon1(const Canon& q, const int64_t* itab, int64_t x, bool full) {
+  int64_t v[1] = {x};
+  canon_apply_n<1>(q, itab, v, 1u, full ? 1u : 0u);
+  return v[0];
+}
 
 // Dense ops (R10-R12) in f32.
 __device__ __forceinline__ float apply_dense_ops(const DevOp* ops, float x, int o0, int o1) {
@@ -404,75 +472,45 @@ __device__ __forceinline__ int warp_incl_scan(int v, int lane) {
 }
 
 // ----------------------------------------------------------------------------
-// Single-pass jagged scan (R17) over the feature-major sparse tile sequence:
-// decoupled look-back.  Tile t publishes its length total (AGG) as soon as it
-// is known, and later resolves its exclusive prefix by summing its
-// predecessors' words, 32 per round trip, back to the nearest inclusive
-// prefix (PREF), which it then publishes for itself.  Words carry the
-// launch epoch, so they never need clearing between launches.
-struct TileRef {
-  unsigned long long* status;
-  long long t;
-  unsigned long long tag;  // epoch << kEpochShift
-};
-
-__device__ __forceinline__ void publish_agg(const TileRef& tr, long long T, int lane) {
-  if (lane == 0) st_relaxed(tr.status + tr.t, tr.tag | (kFlagAgg << kFlagShift) | (unsigned long long)T);
-}
-
-__device__ __forceinline__ long long tile_lookback(const TileRef& tr, long long T, int lane) {
-  const unsigned long long epoch = tr.tag >> kEpochShift;
-  long long excl = 0;
-  long long top = tr.t - 1;
-  while (top >= 0) {
-    const long long idx = top - lane;
-    unsigned long long w = 0;
-    unsigned pm, take;
-    while (true) {
-      int fl = (int)kFlagPrefix;  // before tile 0: an inclusive prefix of 0
-      w = 0;
-      if (idx >= 0) {
-        w = ld_relaxed(tr.status + idx);
-        fl = (w >> kEpochShift) == epoch ? (int)((w >> kFlagShift) & 3ull) : 0;
-      }
-      pm = __ballot_sync(0xffffffffu, fl == (int)kFlagPrefix);
-      const unsigned zm = __ballot_sync(0xffffffffu, fl == 0);
-      take = pm ? ((pm & (0u - pm)) << 1) - 1u : 0xffffffffu;  // lanes up to the nearest prefix
-      if ((zm & take) == 0) break;
-      __nanosleep(32);
-    }
-    excl += warp_sum64(((take >> lane) & 1u) ? (long long)(w & kValueMask) : 0ll);
-    if (pm) break;
-    top -= 32;
-  }
-  if (lane == 0) st_relaxed(tr.status + tr.t, tr.tag | (kFlagPrefix << kFlagShift) | (unsigned long long)(excl + T));
-  return excl;
-}
-
-// ----------------------------------------------------------------------------
-// Sparse tiles with 4 consecutive rows per lane (rows r0 + 4*lane + k): one
-// 16-byte offsets load, one validity word, 16-byte length / offset stores.
-
-// Per-feature state a warp keeps in registers across its tiles.
+// Jagged scan (R17) over the feature-major sparse tile sequence.  Each CTA
+// owns a contiguous, cost-balanced range of it (host partition, DESIGN.md
+// §7) and splits it into one contiguous sub-range per warp.  Phase L sums
+// every sub-range's output lengths (closed form from the Arrow offsets) and
+// publishes the CTA aggregate; after its dense blocks the CTA adds its
+// predecessors' aggregates (one parallel read, no chained look-back), so
+// every warp knows the base of its sub-range before it stores anything and
+// then walks its tiles with a running base: a tile function takes its base
+// and returns its output length total.
+// Per-feature dispatch state a warp keeps in registers across its tiles.
+enum TileKind : int { TK_CANON = 0, TK_NGRAM_FAST = 1, TK_NGRAM = 2, TK_GENERIC = 3 };
 struct FeatCtx {
-  int f, kind, src, has_fill, canon, mask;
+  int f, kind, sk, src, has_fill;
   int64_t xcap, null_xcap, fill;
-  Canon q;
+  Canon q;  // canonical pipeline (TK_CANON), in registers
 };
 
 template <class P>
 __device__ __forceinline__ void load_ctx(const P& p, int f, FeatCtx& x) {
   const SProg& pg = p.c.sprogs[f];
-  x.f = f;
-  x.kind = pg.ch.src_kind;
-  x.src = pg.ch.src;
-  x.has_fill = pg.ch.has_fill;
-  x.xcap = pg.ch.xcap;
-  x.null_xcap = pg.ch.null_xcap;
-  x.fill = pg.ch.fill;
+  const Chain ch = pg.ch;  // one burst of independent loads
   x.q = pg.cn;
-  x.canon = x.q.ok && x.kind == SRC_SPARSE;
-  x.mask = x.q.mask;
+  x.f = f;
+  x.sk = ch.src_kind;
+  x.src = ch.src;
+  x.has_fill = ch.has_fill;
+  x.xcap = ch.xcap;
+  x.null_xcap = ch.null_xcap;
+  x.fill = ch.fill;
+  if (x.sk == SRC_SPARSE) {
+    x.kind = x.q.ok ? TK_CANON : TK_GENERIC;
+  } else if (x.sk == SRC_NGRAM) {
+    const int k = pg.ng.k;
+    bool fast = x.q.ok && k <= 4;
+    for (int c = 0; c < k; ++c) fast = fast && pg.src_cn[c].ok && pg.src[c].src_kind == SRC_SPARSE;
+    x.kind = fast ? TK_NGRAM_FAST : TK_NGRAM;
+  } else {
+    x.kind = TK_GENERIC;
+  }
 }
 
 // Arrow offsets of rows r0+4*lane .. +4 and the validity word of those rows.
@@ -519,8 +557,8 @@ template <class P>
 __device__ __noinline__ void value_group_general(const P& p, int f, int64_t row0, int lane, int32_t mylen,
                                                  int32_t myst, int32_t lx, long long gbase);
 template <class P>
-__device__ __noinline__ void value_tile_ngram(const P& p, int f, int64_t rt, int lane, const TileRef& tr,
-                                              int32_t* scr);
+__device__ __noinline__ long long value_tile_ngram(const P& p, int f, int64_t rt, int lane, long long base,
+                                                   int32_t* scr);
 
 // Lengths (int4) and offsets (2 x longlong2) of the lane's 4 rows.
 __device__ __forceinline__ void store_quad(int32_t* lp, int64_t* op, int64_t row, int64_t B, const int32_t* l,
@@ -539,10 +577,11 @@ __device__ __forceinline__ void store_quad(int32_t* lp, int64_t* op, int64_t row
   }
 }
 
-// Specialised tile of a canonical SRC_SPARSE chain (mask MASK); the lane
-// owns rows r0 + 4*lane + k, so its output ids are contiguous.
-template <int MASK, class P>
-__device__ __noinline__ void value_tile_canon(const P& p, const FeatCtx& fc, int64_t rt, int lane, const TileRef& tr) {
+// Tile of a canonical SRC_SPARSE chain; the lane owns rows r0 + 4*lane + k,
+// so its output ids are contiguous.
+template <class P>
+__device__ __forceinline__ long long value_tile_canon(const P& p, const FeatCtx& fc, int64_t rt, int lane,
+                                                      long long base) {
   const Canon& q = fc.q;
   const int f = fc.f;
   const int64_t B = p.c.n_rows;
@@ -553,7 +592,9 @@ __device__ __noinline__ void value_tile_canon(const P& p, const FeatCtx& fc, int
   const int64_t* itab = p.c.itab;
   const int32_t* off = p.off[fc.src];
   const int64_t* val = p.val[fc.src];
+  trace_clk(p.c, 8, 0);
   const Quad qd = load_quad(off, p.svalid[fc.src], r0, lane, B, (reinterpret_cast<uintptr_t>(off) & 15) == 0);
+  trace_clk(p.c, 9, qd.a[0] + qd.a[4] + qd.w);
   int32_t l[4], e[4];
   int tot = 0;
 #pragma unroll
@@ -565,19 +606,22 @@ __device__ __noinline__ void value_tile_canon(const P& p, const FeatCtx& fc, int
   const int incl = warp_incl_scan(tot, lane);
   const int L = incl - tot;  // lane exclusive prefix within the tile
   const int T = __shfl_sync(0xffffffffu, incl, 31);
-  publish_agg(tr, T, lane);
   const bool last = f == p.c.n_sparse_out - 1 && rt == p.c.tiles_per_feature - 1;
   int32_t* lp = p.c.lengths + (int64_t)f * B + row;
   int64_t* op = p.c.offsets + (int64_t)f * B + row;
   if (__all_sync(0xffffffffu, l[0] <= 1 && l[1] <= 1 && l[2] <= 1 && l[3] <= 1)) {
     // at most one id per row: the ids are computed before the base is known
     int64_t v[4];
+    unsigned act = 0, full = 0;
 #pragma unroll
-    for (int k = 0; k < 4; ++k) v[k] = (l[k] == 1 && quad_valid(qd, k, lane)) ? __ldg(val + qd.a[k]) : fc.fill;
-#pragma unroll
-    for (int k = 0; k < 4; ++k)
-      if (l[k] == 1) v[k] = canon_apply<MASK>(q, itab, v[k], quad_valid(qd, k, lane) ? 15 : q.null_mask);
-    const long long base = tile_lookback(tr, T, lane);
+    for (int k = 0; k < 4; ++k) {
+      act |= (l[k] == 1 ? 1u : 0u) << k;
+      full |= (quad_valid(qd, k, lane) ? 1u : 0u) << k;
+      v[k] = (l[k] == 1 && quad_valid(qd, k, lane)) ? __ldg(val + qd.a[k]) : fc.fill;
+    }
+    trace_clk(p.c, 10, v[0] + v[1] + v[2] + v[3]);
+    canon_apply_n<4>(q, itab, v, act, full);
+    trace_clk(p.c, 11, v[0] + v[1] + v[2] + v[3]);
     const long long lb = base + L;
     store_quad(lp, op, row, B, l, lb, e);
 #pragma unroll
@@ -585,51 +629,61 @@ __device__ __noinline__ void value_tile_canon(const P& p, const FeatCtx& fc, int
       const long long pos = lb + e[k];
       if (l[k] == 1 && pos < cap) values[pos] = v[k];
     }
+    trace_clk(p.c, 12, 0);
     if (last && lane == 31) {
       p.c.offsets[(int64_t)p.c.n_sparse_out * B] = base + T;  // total, R17
       if (base + T > cap) atomicExch(p.c.err, 1);
     }
-    return;
+    return T;
   }
-  const long long base = tile_lookback(tr, T, lane);
   store_quad(lp, op, row, B, l, base + L, e);
   if (last && lane == 31) {
     p.c.offsets[(int64_t)p.c.n_sparse_out * B] = base + T;
     if (base + T > cap) atomicExch(p.c.err, 1);
   }
-  // multi-id rows: elements in output order; owning lane by a 5-step shuffle
-  // search over the lane prefixes, then the row within the lane
+  // multi-id rows: elements in output order, 128 per round (4 per lane, all
+  // loads in flight together); owning lane by a 5-step shuffle search over
+  // the lane prefixes, then the row within the lane
   const int mylex = L;
-  for (int eb = 0; eb < T; eb += 32) {
-    const int ee = eb + lane;
-    int r = 0;
+  for (int eb = 0; eb < T; eb += 128) {
+    int64_t x[4];
+    unsigned act = 0, full = 0;
 #pragma unroll
-    for (int step = 16; step >= 1; step >>= 1) {
-      const int c = __shfl_sync(0xffffffffu, mylex, r + step);
-      if (c <= ee) r += step;
+    for (int u = 0; u < 4; ++u) {
+      const int ee = eb + 32 * u + lane;
+      int r = 0;
+#pragma unroll
+      for (int step = 16; step >= 1; step >>= 1) {
+        const int c = __shfl_sync(0xffffffffu, mylex, r + step);
+        if (c <= ee) r += step;
+      }
+      const int in_lane = ee - __shfl_sync(0xffffffffu, mylex, r);
+      const int e1 = __shfl_sync(0xffffffffu, e[1], r), e2 = __shfl_sync(0xffffffffu, e[2], r),
+                e3 = __shfl_sync(0xffffffffu, e[3], r);
+      const int k = in_lane >= e3 ? 3 : (in_lane >= e2 ? 2 : (in_lane >= e1 ? 1 : 0));
+      const int ek = k == 3 ? e3 : (k == 2 ? e2 : (k == 1 ? e1 : 0));
+      const int32_t a0 = __shfl_sync(0xffffffffu, qd.a[0], r), a1 = __shfl_sync(0xffffffffu, qd.a[1], r),
+                    a2 = __shfl_sync(0xffffffffu, qd.a[2], r), a3 = __shfl_sync(0xffffffffu, qd.a[3], r);
+      const uint32_t wr = __shfl_sync(0xffffffffu, qd.w, r);
+      const int32_t ak = k == 3 ? a3 : (k == 2 ? a2 : (k == 1 ? a1 : a0));
+      const bool au = ee < T, fu = (wr >> ((4 * r + k) & 31)) & 1u;
+      act |= (au ? 1u : 0u) << u;
+      full |= (fu ? 1u : 0u) << u;
+      x[u] = (au && fu) ? __ldg(val + ak + (in_lane - ek)) : fc.fill;
     }
-    const int in_lane = ee - __shfl_sync(0xffffffffu, mylex, r);
-    const int e1 = __shfl_sync(0xffffffffu, e[1], r), e2 = __shfl_sync(0xffffffffu, e[2], r),
-              e3 = __shfl_sync(0xffffffffu, e[3], r);
-    const int k = in_lane >= e3 ? 3 : (in_lane >= e2 ? 2 : (in_lane >= e1 ? 1 : 0));
-    const int ek = k == 3 ? e3 : (k == 2 ? e2 : (k == 1 ? e1 : 0));
-    const int32_t a0 = __shfl_sync(0xffffffffu, qd.a[0], r), a1 = __shfl_sync(0xffffffffu, qd.a[1], r),
-                  a2 = __shfl_sync(0xffffffffu, qd.a[2], r), a3 = __shfl_sync(0xffffffffu, qd.a[3], r);
-    const uint32_t wr = __shfl_sync(0xffffffffu, qd.w, r);
-    const int32_t ak = k == 3 ? a3 : (k == 2 ? a2 : (k == 1 ? a1 : a0));
-    const bool vk = (wr >> ((4 * r + k) & 31)) & 1u;
-    if (ee < T) {
-      const int64_t x = vk ? __ldg(val + ak + (in_lane - ek)) : fc.fill;
-      const int64_t v = canon_apply<MASK>(q, itab, x, vk ? 15 : q.null_mask);
-      const long long pos = base + ee;
-      if (pos < cap) values[pos] = v;
+    canon_apply_n<4>(q, itab, x, act, full);
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const long long pos = base + eb + 32 * u + lane;
+      if (((act >> u) & 1u) && pos < cap) values[pos] = x[u];
     }
   }
+  return T;
 }
 
 // Tile of any other SRC_SPARSE / SRC_DENSE_BUCKET chain (op interpreter).
 template <class P>
-__device__ __noinline__ void value_tile_generic(const P& p, int f, int64_t rt, int lane, const TileRef& tr) {
+__device__ __noinline__ long long value_tile_generic(const P& p, int f, int64_t rt, int lane, long long base) {
   const SProg& pg = p.c.sprogs[f];
   const DevOp* ops = prog_ops(pg, p.c.ops);
   const int64_t B = p.c.n_rows;
@@ -660,7 +714,6 @@ __device__ __noinline__ void value_tile_generic(const P& p, int f, int64_t rt, i
     gb[g] = run;
     run += __shfl_sync(0xffffffffu, incl, 31);
   }
-  publish_agg(tr, run, lane);
   const bool use_pipe = ch.src_kind == SRC_SPARSE && pipe_ok(ops, ch.op_begin, ch.op_end);
   Pipe pipe;
   if (use_pipe) load_pipe(pipe, ops, ch.op_begin, ch.op_end, pg.tab_off);
@@ -681,7 +734,6 @@ __device__ __noinline__ void value_tile_generic(const P& p, int f, int64_t rt, i
       }
     }
   }
-  const long long base = tile_lookback(tr, run, lane);
 #pragma unroll
   for (int g = 0; g < kGroups; ++g) {
     const int64_t row = r0 + 32 * g + lane;
@@ -700,26 +752,27 @@ __device__ __noinline__ void value_tile_generic(const P& p, int f, int64_t rt, i
       const long long pos = base + gb[g] + lex[g];
       if (len[g] == 1 && pos < cap) values[pos] = v1[g];
     }
-    return;
+    return run;
   }
   // general (multi-id rows): elements in output order, per row group
 #pragma unroll 1
   for (int g = 0; g < kGroups; ++g)
     value_group_general(p, f, r0 + 32 * g, lane, len[g], st[g], lex[g], base + gb[g]);
+  return run;
 }
 
+// Offsets and ids of sparse tile (f, rt) whose first id goes to
+// values[base]; returns the tile's output length total.
 template <class P>
-__device__ __forceinline__ void value_tile(const P& p, const FeatCtx& fc, int64_t rt, int lane, const TileRef& tr,
-                                           int32_t* scr) {
-  if (fc.canon) {
-#define RAP_VT_CALL(M) value_tile_canon<M>(p, fc, rt, lane, tr)
-    RAP_CANON_DISPATCH(fc.mask, RAP_VT_CALL)
-#undef RAP_VT_CALL
-  } else if (fc.kind == SRC_NGRAM) {
-    value_tile_ngram(p, fc.f, rt, lane, tr, scr);
-  } else {
-    value_tile_generic(p, fc.f, rt, lane, tr);
+__device__ __forceinline__ long long value_tile(const P& p, const FeatCtx& fc, int64_t rt, int lane, long long base,
+                                                int32_t* scr) {
+  if (fc.kind == TK_CANON) return value_tile_canon(p, fc, rt, lane, base);
+  if (fc.kind == TK_NGRAM_FAST) {
+    const long long T = ngram_tile_fast(p, fc.f, rt, lane, base, scr);
+    if (T >= 0) return T;
   }
+  if (fc.kind != TK_GENERIC) return value_tile_ngram(p, fc.f, rt, lane, base, scr);
+  return value_tile_generic(p, fc.f, rt, lane, base);
 }
 
 // Ids of one 32-row group with multi-id rows: elements in output order, the
@@ -762,11 +815,181 @@ __device__ __noinline__ void value_group_general(const P& p, int f, int64_t row0
   }
 }
 
+// Output length total of the NGram tile starting at row r0 (R7 count
+// max(0, sum of source lengths - n + 1), capped by FirstX): quad layout, 4
+// rows per lane, every source's offsets requested before any is used.
+template <class P>
+__device__ __noinline__ long long ngram_tile_len(const P& p, const SProg& pg, int64_t r0, int lane) {
+  const int64_t B = p.c.n_rows;
+  int32_t tot4[4] = {0, 0, 0, 0};
+#pragma unroll 1
+  for (int c0 = 0; c0 < pg.ng.k; c0 += 4) {  // 4 sources' offsets in flight at a time
+    Quad qs[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int c = c0 + j;
+      if (c < pg.ng.k && pg.src[c].src_kind == SRC_SPARSE) {
+        const int32_t* off = p.off[pg.src[c].src];
+        qs[j] = load_quad(off, p.svalid[pg.src[c].src], r0, lane, B, (reinterpret_cast<uintptr_t>(off) & 15) == 0);
+      }
+    }
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int c = c0 + j;
+      if (c < pg.ng.k) {
+        const Chain& sc = pg.src[c];
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          const int64_t row = r0 + 4 * lane + q;
+          if (sc.src_kind == SRC_SPARSE)
+            tot4[q] += quad_len(qs[j], q, lane, row, B, sc.xcap, sc.has_fill, sc.null_xcap);
+          else
+            tot4[q] += row < B ? (int32_t)min((int64_t)1, sc.xcap) : 0;
+        }
+      }
+    }
+  }
+  int sum = 0;
+#pragma unroll
+  for (int q = 0; q < 4; ++q)
+    if (r0 + 4 * lane + q < B) sum += (int32_t)min((int64_t)max(tot4[q] - pg.ng.n + 1, 0), pg.ch.xcap);
+  return warp_sum64(sum);
+}
+
+// Warp-cooperative copy of `bytes` (a multiple of 8) from global to shared.
+__device__ __forceinline__ void warp_copy8(void* dst, const void* src, int bytes, int lane) {
+  const long long* s8 = reinterpret_cast<const long long*>(src);
+  long long* d8 = reinterpret_cast<long long*>(dst);
+  for (int i = lane; i < (bytes >> 3); i += 32) d8[i] = __ldg(s8 + i);
+}
+
+struct NgParams {  // ngram_tile_fast parameters, staged in warp scratch
+  Chain src[4];
+  Canon scn[4];
+  Canon post;
+  NGramDesc ng;
+  int64_t xcap;
+};
+static_assert(sizeof(NgParams) <= 4 * kMaxNgramK * 32 * 4, "NgParams exceeds the warp scratch");
+
+// Fast NGram tile (R7) for k <= 4 canonical single-source chains when every
+// row of every source has at most one id and at most n ids in total: then a
+// row has one window (exactly n ids) or none, and its hash is the chain over
+// the present ids in source order.  Quad layout (4 rows per lane); all
+// sources' offsets, then all their ids, are in flight together.  Returns
+// the tile's output length total, or -1 with nothing written when the tile
+// is not eligible.
+template <class P>
+__device__ __noinline__ long long ngram_tile_fast(const P& p, int f, int64_t rt, int lane, long long base,
+                                                 int32_t* scr) {
+  const SProg& pg = p.c.sprogs[f];
+  trace_clk(p.c, 13, 0);
+  // the parameters go to warp-private shared memory in one burst (no lazy
+  // global reads on the dependent path)
+  NgParams& G = *reinterpret_cast<NgParams*>(scr);
+  warp_copy8(G.src, pg.src, sizeof(G.src), lane);
+  warp_copy8(G.scn, pg.src_cn, sizeof(G.scn), lane);
+  warp_copy8(&G.post, &pg.cn, sizeof(G.post), lane);
+  warp_copy8(&G.ng, &pg.ng, sizeof(G.ng), lane);
+  if (lane == 0) G.xcap = pg.ch.xcap;
+  __syncwarp();
+  const int k = G.ng.k, n = G.ng.n;
+  const int64_t B = p.c.n_rows;
+  const int64_t r0 = rt * kTileRows;
+  const int64_t row = r0 + 4 * lane;
+  Quad q[4];
+#pragma unroll
+  for (int j = 0; j < 4; ++j)
+    if (j < k) {
+      const int32_t* off = p.off[G.src[j].src];
+      q[j] = load_quad(off, p.svalid[G.src[j].src], r0, lane, B, (reinterpret_cast<uintptr_t>(off) & 15) == 0);
+    }
+  int pn[4] = {0, 0, 0, 0};
+  bool ok = true;
+#pragma unroll
+  for (int j = 0; j < 4; ++j)
+    if (j < k) {
+      const Chain& sc = G.src[j];
+#pragma unroll
+      for (int kk = 0; kk < 4; ++kk) {
+        const int l = quad_len(q[j], kk, lane, row + kk, B, sc.xcap, sc.has_fill, sc.null_xcap);
+        ok &= l <= 1;
+        pn[kk] += l;
+      }
+    }
+#pragma unroll
+  for (int kk = 0; kk < 4; ++kk) ok &= pn[kk] <= n;
+  if (!__all_sync(0xffffffffu, ok)) return -1;
+  // all ids of all sources in flight
+  int64_t v[4][4];
+  unsigned pres[4], full[4];
+  int32_t l[4], e[4];
+  int tot = 0;
+#pragma unroll
+  for (int kk = 0; kk < 4; ++kk) {
+    l[kk] = (row + kk < B && pn[kk] == n) ? (int32_t)min((int64_t)1, G.xcap) : 0;
+    e[kk] = tot;
+    tot += l[kk];
+  }
+#pragma unroll
+  for (int j = 0; j < 4; ++j)
+    if (j < k) {
+      const Chain& sc = G.src[j];
+      const int64_t* val = p.val[sc.src];
+      pres[j] = full[j] = 0;
+#pragma unroll
+      for (int kk = 0; kk < 4; ++kk) {
+        const bool pr = l[kk] == 1 && quad_len(q[j], kk, lane, row + kk, B, sc.xcap, sc.has_fill, sc.null_xcap) == 1;
+        const bool fu = quad_valid(q[j], kk, lane);
+        pres[j] |= (pr ? 1u : 0u) << kk;
+        full[j] |= (fu ? 1u : 0u) << kk;
+        v[j][kk] = (pr && fu) ? __ldg(val + q[j].a[kk]) : sc.fill;
+      }
+    }
+  trace_clk(p.c, 14, v[0][0] + v[1][0] + v[2][0] + v[0][3] + v[1][3] + v[2][3]);
+  const int incl = warp_incl_scan(tot, lane);
+  const int L = incl - tot;
+  const int T = __shfl_sync(0xffffffffu, incl, 31);
+  const long long lb = base + L;
+  store_quad(p.c.lengths + (int64_t)f * B + row, p.c.offsets + (int64_t)f * B + row, row, B, l, lb, e);
+  const int64_t* itab = p.c.itab;
+  uint64_t h[4];
+#pragma unroll
+  for (int kk = 0; kk < 4; ++kk) h[kk] = G.ng.hsalt;  // R7: h = H(salt); h = H(h ^ c[q])
+#pragma unroll
+  for (int j = 0; j < 4; ++j)
+    if (j < k) {
+      canon_apply_n<4>(G.scn[j], itab, v[j], pres[j], full[j]);
+#pragma unroll
+      for (int kk = 0; kk < 4; ++kk)
+        if ((pres[j] >> kk) & 1u) h[kk] = splitmix_H(h[kk] ^ (uint64_t)v[j][kk]);
+    }
+  int64_t o[4];
+  unsigned act = 0;
+#pragma unroll
+  for (int kk = 0; kk < 4; ++kk) {
+    o[kk] = (int64_t)reduce_M(h[kk], G.ng.M);
+    act |= (l[kk] == 1 ? 1u : 0u) << kk;
+  }
+  canon_apply_n<4>(G.post, itab, o, act, 15u);
+  const long long cap = p.c.values_cap;
+#pragma unroll
+  for (int kk = 0; kk < 4; ++kk)
+    if (((act >> kk) & 1u) && lb + e[kk] < cap) p.c.values[lb + e[kk]] = o[kk];
+  if (f == p.c.n_sparse_out - 1 && rt == p.c.tiles_per_feature - 1 && lane == 31) {
+    p.c.offsets[(int64_t)p.c.n_sparse_out * B] = base + T;  // total, R17
+    if (base + T > cap) atomicExch(p.c.err, 1);
+  }
+  trace_clk(p.c, 15, 0);
+  __syncwarp();
+  return T;
+}
+
 // NGram feature tile (R7): per row the k source lists, windows over their
 // concatenation.
 template <class P>
-__device__ __noinline__ void value_tile_ngram(const P& p, int f, int64_t rt, int lane, const TileRef& tr,
-                                              int32_t* scr) {
+__device__ __noinline__ long long value_tile_ngram(const P& p, int f, int64_t rt, int lane, long long base,
+                                                   int32_t* scr) {
   const SProg& pg = p.c.sprogs[f];
   const DevOp* ops = prog_ops(pg, p.c.ops);
   const int64_t B = p.c.n_rows;
@@ -775,46 +998,6 @@ __device__ __noinline__ void value_tile_ngram(const P& p, int f, int64_t rt, int
   int32_t* lengths = p.c.lengths + (int64_t)f * B;
   int64_t* values = p.c.values;
   const long long cap = p.c.values_cap;
-  // pass 1: the tile's output length total (quad layout: 4 rows per lane,
-  // every source's offsets requested before any is used), published at once
-  long long base;
-  {
-    int32_t tot4[4] = {0, 0, 0, 0};
-#pragma unroll 1
-    for (int c0 = 0; c0 < pg.ng.k; c0 += 4) {  // 4 sources' offsets in flight at a time
-      Quad qs[4];
-#pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        const int c = c0 + j;
-        if (c < pg.ng.k && pg.src[c].src_kind == SRC_SPARSE) {
-          const int32_t* off = p.off[pg.src[c].src];
-          qs[j] = load_quad(off, p.svalid[pg.src[c].src], r0, lane, B, (reinterpret_cast<uintptr_t>(off) & 15) == 0);
-        }
-      }
-#pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        const int c = c0 + j;
-        if (c < pg.ng.k) {
-          const Chain& sc = pg.src[c];
-#pragma unroll
-          for (int q = 0; q < 4; ++q) {
-            const int64_t row = r0 + 4 * lane + q;
-            if (sc.src_kind == SRC_SPARSE)
-              tot4[q] += quad_len(qs[j], q, lane, row, B, sc.xcap, sc.has_fill, sc.null_xcap);
-            else
-              tot4[q] += row < B ? (int32_t)min((int64_t)1, sc.xcap) : 0;
-          }
-        }
-      }
-    }
-    int sum = 0;
-#pragma unroll
-    for (int q = 0; q < 4; ++q)
-      if (r0 + 4 * lane + q < B) sum += (int32_t)min((int64_t)max(tot4[q] - pg.ng.n + 1, 0), pg.ch.xcap);
-    const long long T = warp_sum64(sum);
-    publish_agg(tr, T, lane);
-    base = tile_lookback(tr, T, lane);
-  }
 
   // NGram feature (R7): per row the k source lists, windows over their
   // concatenation.  Per-source (start, length) of the warp's 32 rows live in
@@ -868,12 +1051,7 @@ __device__ __noinline__ void value_tile_ngram(const P& p, int f, int64_t rt, int
         const int sl = sl_s[c * 32 + lane];
         if (sl == 1) {
           present |= 1u << c;
-          const int act = st_s[c * 32 + lane] >= 0 ? 15 : qc.null_mask;
-          int64_t x = ev_s[c * 32 + lane];
-#define RAP_NG_CALL(M) x = canon_apply<M>(qc, itab, x, act)
-          RAP_CANON_DISPATCH(qc.mask, RAP_NG_CALL)
-#undef RAP_NG_CALL
-          ev_s[c * 32 + lane] = x;
+          ev_s[c * 32 + lane] = canon1(qc, itab, ev_s[c * 32 + lane], st_s[c * 32 + lane] >= 0);
         }
       }
       const Canon qp = pg.cn;
@@ -889,10 +1067,7 @@ __device__ __noinline__ void value_tile_ngram(const P& p, int f, int64_t rt, int
             ++seen;
           }
         }
-        int64_t v = (int64_t)reduce_M(h, pg.ng.M);
-#define RAP_NP_CALL(M) v = canon_apply<M>(qp, itab, v, 15)
-        RAP_CANON_DISPATCH(qp.mask, RAP_NP_CALL)
-#undef RAP_NP_CALL
+        const int64_t v = canon1(qp, itab, (int64_t)reduce_M(h, pg.ng.M), true);
         const long long pos = run + lx + j;
         if (pos < cap) values[pos] = v;
       }
@@ -927,6 +1102,7 @@ __device__ __noinline__ void value_tile_ngram(const P& p, int f, int64_t rt, int
     p.c.offsets[(int64_t)p.c.n_sparse_out * B] = run;
     if (run > cap) atomicExch(p.c.err, 1);
   }
+  return run - base;
 }
 
 // ----------------------------------------------------------------------------
@@ -1076,6 +1252,29 @@ __device__ void dense_block(const P& p, int gi, int64_t rb, unsigned char* smem,
 }
 
 // ----------------------------------------------------------------------------
+// Phase L: output length total of sparse tile (f, rt) (closed forms R5, R7,
+// R10, R14 from the Arrow offsets and validity words only).
+template <class P>
+__device__ __noinline__ long long tile_total(const P& p, int f, int64_t rt, int lane) {
+  const int64_t B = p.c.n_rows;
+  const int64_t r0 = rt * kTileRows;
+  const SProg& pg = p.c.sprogs[f];
+  if (pg.ch.src_kind == SRC_NGRAM) return ngram_tile_len(p, pg, r0, lane);
+  return min((int64_t)kTileRows, B - r0) * min((int64_t)1, pg.ch.xcap);  // R4: dense bucket, 1 id per row
+}
+
+__device__ __forceinline__ long long block_sum(long long v, long long* red) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  v = warp_sum64(v);
+  __syncthreads();
+  if (lane == 0) red[warp] = v;
+  __syncthreads();
+  long long t = 0;
+#pragma unroll
+  for (int j = 0; j < kWarps; ++j) t += red[j];
+  return t;
+}
+
 #ifndef RAP_MIN_CTAS
 #define RAP_MIN_CTAS 4
 #endif
@@ -1083,57 +1282,140 @@ template <int MD, int MS>
 __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const __grid_constant__ KParams<MD, MS> p) {
   extern __shared__ __align__(128) unsigned char smem[];
   __shared__ CtaState cs;
-  __shared__ long long s_item;
+  __shared__ long long s_slots[kWarps];
+  __shared__ long long s_red[kWarps];
   __shared__ unsigned long long s_epoch;
-  __shared__ int s_last;
+  __shared__ int s_rank, s_last;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   if (tid == 0) {
     mbar_init(&cs.bar, 1);
     cs.phase = 0;
+    // partition rank = arrival order, so a CTA only ever waits on CTAs that
+    // are already resident (deadlock-free under any co-running load)
+    s_rank = (int)atomicAdd(p.c.sched + 2, 1ull);
     s_epoch = ld_relaxed(p.c.sched + 1);
   }
   __syncthreads();
   trace_stamp(p.c, 0);
+  if (p.c.trace != nullptr && tid == 0 && (int64_t)blockIdx.x < p.c.trace_cap) {
+    unsigned smid;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    p.c.trace[(int64_t)blockIdx.x * kTracePts + 6] = smid;
+    p.c.trace[(int64_t)blockIdx.x * kTracePts + 7] = (unsigned long long)s_rank;
+  }
   const unsigned long long epoch = s_epoch;
+  const int rank = s_rank;
+  const int64_t S = p.c.n_sparse_tiles, T = p.c.tiles_per_feature;
+  const int64_t s0 = __ldg(p.c.part + rank), s1 = __ldg(p.c.part + rank + 1);  // my sparse tiles
+  int32_t* scr = reinterpret_cast<int32_t*>(smem) + warp * (4 * kMaxNgramK * 32);
+  if (p.c.trace != nullptr && tid == 0 && (int64_t)blockIdx.x < p.c.trace_cap)
+    p.c.trace[(int64_t)blockIdx.x * kTracePts + 5] = (unsigned long long)(s0 | ((s1 - s0) << 32));
 
-  // (1) sparse tiles (warp units) from a global queue, in scan order
+  // (L) output length total of my warp's sub-range -> CTA aggregate
+  const int64_t ns = s1 - s0;
+  const int64_t w0 = s0 + ns * warp / kWarps, w1 = s0 + ns * (warp + 1) / kWarps;
+  long long mine = 0, part = 0;  // warp-uniform / per-lane partial totals
   {
     FeatCtx fc;
     fc.f = -1;
-    int32_t* scr = reinterpret_cast<int32_t*>(smem) + warp * (4 * kMaxNgramK * 32);
-    const int64_t S = p.c.n_sparse_tiles, T = p.c.tiles_per_feature;
-    TileRef tr;
-    tr.status = p.c.status;
-    tr.tag = epoch << kEpochShift;
-    while (true) {
-      long long t = 0;
-      if (lane == 0) t = (long long)atomicAdd(p.c.sched + 3, 1ull);
-      t = __shfl_sync(0xffffffffu, t, 0);
-      if (t >= S) break;
+    const int64_t B = p.c.n_rows;
+    for (int64_t t = w0; t < w1;) {
       const int f = (int)((uint64_t)t / (uint64_t)T);
       if (f != fc.f) load_ctx(p, f, fc);
-      tr.t = t;
-      value_tile(p, fc, (int64_t)t - (int64_t)f * T, lane, tr, scr);
+      const int64_t tend = min(w1, (int64_t)(f + 1) * T);
+      if (fc.sk == SRC_SPARSE) {
+        // 4 tiles' offsets in flight at a time
+        const int32_t* off = p.off[fc.src];
+        const uint32_t* bm = p.svalid[fc.src];
+        const bool al = (reinterpret_cast<uintptr_t>(off) & 15) == 0;
+        for (; t < tend; t += 4) {
+          Quad q[4];
+#pragma unroll
+          for (int j = 0; j < 4; ++j)
+            if (t + j < tend) q[j] = load_quad(off, bm, (t + j - (int64_t)f * T) * kTileRows, lane, B, al);
+#pragma unroll
+          for (int j = 0; j < 4; ++j)
+            if (t + j < tend) {
+              const int64_t row = (t + j - (int64_t)f * T) * kTileRows + 4 * lane;
+#pragma unroll
+              for (int k = 0; k < 4; ++k) part += quad_len(q[j], k, lane, row + k, B, fc.xcap, fc.has_fill, fc.null_xcap);
+            }
+        }
+        t = tend;
+      } else {
+        for (; t < tend; ++t) mine += tile_total(p, f, t - (int64_t)f * T, lane);  // warp-uniform
+      }
     }
   }
+  mine += warp_sum64(part);
+  if (lane == 0) s_slots[warp] = mine;
+  const long long agg = block_sum(lane == 0 ? mine : 0ll, s_red);
+  const unsigned long long tag = epoch + 1ull;
+  if (tid == 0) st_relaxed(p.c.agg + rank, (tag << kEpochShift) | (unsigned long long)agg);
   trace_stamp(p.c, 1);
-  __syncthreads();
 
-  // (2) dense blocks (CTA units) from a second global queue
-  while (true) {
-    if (tid == 0) s_item = (long long)atomicAdd(p.c.sched + 2, 1ull);
-    __syncthreads();
-    const long long d = s_item;
-    __syncthreads();
-    if (d >= p.c.n_dense_tiles) break;
+  // (D) my dense blocks, round robin over the ranks (independent of the
+  // scan: they hide the wait below)
+#ifdef RAP_DBG_SKIP_D
+  if (false)
+#endif
+  for (int64_t d = rank; d < p.c.n_dense_tiles; d += gridDim.x) {
     const uint32_t gi = (uint32_t)d % (uint32_t)p.c.n_groups;
     dense_block(p, (int)gi, (int64_t)((uint32_t)d / (uint32_t)p.c.n_groups), smem, cs);
     __syncthreads();
   }
   trace_stamp(p.c, 2);
 
-  // The last CTA out resets the queue heads and advances the epoch of the
-  // look-back words (clearing them when the 20-bit epoch wraps), so launch
+  if (s1 > s0) {
+    // (W) base of my range = sum of the aggregates of the CTAs ranked before
+    // me; all of them were resident before I started
+    // warp 0 polls (32 lanes, backoff), so waiting CTAs do not flood the
+    // L2 slices that hold the aggregate words
+    long long pre = 0;
+    if (warp == 0) {
+      for (int j0 = 0; j0 < rank; j0 += 32 * 8) {
+        unsigned long long w[8];
+        bool ready = false;
+        int ns = 128;
+        while (!ready) {
+          ready = true;
+#pragma unroll
+          for (int u = 0; u < 8; ++u) {
+            const int j = j0 + 32 * u + lane;
+            w[u] = j < rank ? ld_relaxed(p.c.agg + j) : (tag << kEpochShift);
+            ready &= (w[u] >> kEpochShift) == tag;
+          }
+          ready = __all_sync(0xffffffffu, ready);
+          if (!ready) {
+            __nanosleep(ns);
+            ns = min(ns * 2, 2048);
+          }
+        }
+#pragma unroll
+        for (int u = 0; u < 8; ++u) pre += (long long)(w[u] & kValueMask);
+      }
+    }
+    const long long base = block_sum(pre, s_red);
+    trace_stamp(p.c, 3);
+
+    // (V) offsets and ids of my warp's tiles, in scan order
+    FeatCtx fc;
+    fc.f = -1;
+    long long run = base;
+    for (int j = 0; j < warp; ++j) run += s_slots[j];
+#ifdef RAP_DBG_SKIP_V
+    if (false)
+#endif
+    for (int64_t t = w0; t < w1; ++t) {
+      const int f = (int)((uint64_t)t / (uint64_t)T);
+      if (f != fc.f) load_ctx(p, f, fc);
+      run += value_tile(p, fc, t - (int64_t)f * T, lane, run, scr);
+    }
+  }
+  trace_stamp(p.c, 4);
+
+  // The last CTA out resets the rank counter and advances the epoch of the
+  // aggregate words (clearing them when the 20-bit epoch wraps), so launch
   // parameters are identical from call to call (CUDA-graph replayable).
   __syncthreads();
   if (tid == 0) {
@@ -1146,13 +1428,12 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
   if (s_last) {
     const bool wrap = epoch >= kEpochMax;
     if (wrap)
-      for (int64_t i = tid; i < p.c.n_sparse_tiles; i += kThreads) p.c.status[i] = 0ull;
+      for (int64_t i = tid; i < kMaxCtas; i += kThreads) p.c.agg[i] = 0ull;
     __syncthreads();
     if (tid == 0) {
       p.c.sched[0] = 0ull;
       p.c.sched[2] = 0ull;
-      p.c.sched[3] = 0ull;
-      p.c.sched[1] = wrap ? 1ull : epoch + 1ull;
+      p.c.sched[1] = wrap ? 0ull : epoch + 1ull;
       __threadfence();
     }
   }

@@ -84,13 +84,13 @@ struct rap_plan {
   // device program blob
   unsigned char* blob = nullptr;
   size_t off_ops = 0, off_sprogs = 0, off_oprogs = 0, off_dprogs = 0, off_ftab = 0, off_itab = 0;
-  // per-n_rows descriptor table
-  // per-CTA partition (cost model), cached by its key
-  std::vector<double> sparse_row_cost, dense_row_cost;
+  // per-CTA partition of the unit sequence (cost model),
+  // re-uploaded only when its key (rows, grid, quantised list lengths) changes
+  std::vector<int64_t> part_key;
+  int64_t* d_part = nullptr;               // [kMaxCtas + 1]
   // scheduling state
-  unsigned long long* d_sched = nullptr;   // CTAs done, look-back epoch
-  unsigned long long* d_status = nullptr;  // look-back words, one per sparse tile (grows)
-  int64_t status_cap = 0;
+  unsigned long long* d_sched = nullptr;   // CTAs done, launch epoch, rank counter
+  unsigned long long* d_agg = nullptr;     // [kMaxCtas] per-rank aggregate words
   int32_t* d_err = nullptr;
   int64_t n_launches = 0;
   int64_t last_n_desc = 0;
@@ -509,7 +509,10 @@ int64_t chain_bound(const rap_plan* P, const Chain& ch, int64_t B, const int64_t
 double expected_len(const rap_plan* P, const Chain& ch, int64_t B, const int64_t* nnz) {
   double e;
   if (ch.src_kind == SRC_SPARSE) {
-    e = (nnz && B > 0 ? (double)std::max<int64_t>(nnz[ch.src], 0) / (double)B : 1.0) + (ch.has_fill ? 1.0 : 0.0);
+    // mean list length; a filled null row counts as one id (R10), so a
+    // filled feature averages at least one id per row
+    e = nnz && B > 0 ? (double)std::max<int64_t>(nnz[ch.src], 0) / (double)B : 1.0;
+    if (ch.has_fill) e = std::max(e, 1.0);
   } else if (ch.src_kind == SRC_DENSE_BUCKET) {
     e = 1.0;
   } else {
@@ -879,6 +882,9 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
     const unsigned long long init[8] = {0ull, 0ull, 0ull, 0ull, 0ull, 0ull, 0ull, 0ull};
     e = cudaMemcpy(P->d_sched, init, sizeof(init), cudaMemcpyHostToDevice);
   }
+  if (e == cudaSuccess) e = cudaMalloc(&P->d_agg, kMaxCtas * sizeof(unsigned long long));
+  if (e == cudaSuccess) e = cudaMemset(P->d_agg, 0, kMaxCtas * sizeof(unsigned long long));
+  if (e == cudaSuccess) e = cudaMalloc(&P->d_part, (kMaxCtas + 1) * sizeof(int64_t));
   if (e == cudaSuccess) e = cudaMalloc(&P->d_err, sizeof(int32_t));
   if (e == cudaSuccess) e = cudaMemset(P->d_err, 0, sizeof(int32_t));
   if (e != cudaSuccess) {
@@ -906,7 +912,8 @@ void rap_plan_destroy(rap_plan* P) {
   DeviceGuard dg(P->device);
   cudaFree(P->blob);
   cudaFree(P->d_sched);
-  cudaFree(P->d_status);
+  cudaFree(P->d_agg);
+  cudaFree(P->d_part);
   cudaFree(P->d_err);
   cudaFree(P->d_trace);
   for (void* s : P->stage) cudaFree(s);
@@ -1019,13 +1026,16 @@ static rap_status check_batch(const rap_plan* P, const rap_raw_batch* raw, const
 // It plays the role of the paper's preprocessing latency predictor
 // (L1037-1057) for the intra-kernel schedule: the partition gives every CTA
 // about the same predicted work.
+// Units: ~0.03 ns of one CTA slot per row; calibrated on B200 against the
+// per-feature phase times of scripts/trace.py (C2 graph: a Clamp+SigridHash
+// row ~2.8 ns, +MapId ~5.6 ns, +Bucketize(1024) ~5.3 ns, a trigram ~15.6 ns).
 static double op_cost(const DevOp& op) {
   switch (op.kind) {
     case OK_CLAMP: return 8;
     case OK_SIGRID: return 40;
-    case OK_MAPID: return 30;
+    case OK_MAPID: return 126;
     case OK_BUCKET_I:
-    case OK_BUCKET_S: return 4 + 6 * std::log2((double)op.m + 1);
+    case OK_BUCKET_S: return 4 + 8 * std::log2((double)op.m + 1);
     case OK_FILL_F: return 3;
     case OK_LOGIT: return 40;
     default: return 70;  // OK_BOXCOX
@@ -1054,7 +1064,7 @@ static double sparse_row_cost(const rap_plan* P, const Chain& ch, int64_t B, con
     c += 15;
   }
   const double windows = std::min((double)ch.xcap, std::max(0.0, lens - ng.n + 1));
-  return c + windows * (ng.n * (elem / std::max(lens, 1.0) + 35) + 10 + chain_ops_cost(P, ch));
+  return c + windows * (ng.n * (elem / std::max(lens, 1.0) + 90) + 10 + chain_ops_cost(P, ch));
 }
 
 static double dense_row_cost(const rap_plan* P, const DProg& dp) {
@@ -1076,6 +1086,48 @@ static double dense_row_cost(const rap_plan* P, const DProg& dp) {
   return c + 2.0 * dp.width;
 }
 
+// Split the sparse tile sequence (feature-major, the scan order) into `grid`
+// contiguous ranges of about equal predicted cost.  The key is
+// (rows, grid, each used source's mean list length quantised to 2^(1/4)
+// steps), so batches of the same shape reuse the uploaded table.
+static rap_status update_partition(rap_plan* P, int64_t B, const int64_t* nnz, int64_t S, int64_t D, int grid,
+                                   cudaStream_t stream) {
+  std::vector<int64_t> key = {B, grid};
+  for (int s : P->used_sparse) {
+    const double m = nnz && B > 0 ? (double)std::max<int64_t>(nnz[s], 0) / (double)B : 0.0;
+    key.push_back(m <= 1.0 / 64 ? -1000 : (int64_t)std::lround(4.0 * std::log2(m)));
+  }
+  if (key == P->part_key) return RAP_OK;
+  const int64_t F = (int64_t)P->souts.size();
+  const int64_t T = F ? S / F : 0;
+  const double kTileFixed = 400.0;  // per-unit overhead (lane-instructions)
+  std::vector<double> fcost(F);
+  for (int64_t f = 0; f < F; ++f) fcost[f] = sparse_row_cost(P, P->chains[P->souts[f].chain], B, nnz);
+  (void)D;
+  auto unit_cost = [&](int64_t u) -> double {
+    const int64_t f = u / T, rt = u - f * T;
+    const int64_t rows = std::min<int64_t>(kTileRows, B - rt * kTileRows);
+    return kTileFixed + (double)rows * fcost[f];
+  };
+  const int64_t U = S;  // dense blocks go round robin over the ranks
+  double W = 0;
+  for (int64_t u = 0; u < U; ++u) W += unit_cost(u);
+  std::vector<int64_t> part(grid + 1);
+  part[0] = 0;
+  double acc = 0;
+  int64_t u = 0;
+  for (int c = 1; c < grid; ++c) {
+    const double target = W * (double)c / (double)grid;
+    while (u < U && acc + 0.5 * unit_cost(u) < target) acc += unit_cost(u++);
+    part[c] = u;
+  }
+  part[grid] = U;
+  cudaError_t e = cudaMemcpyAsync(P->d_part, part.data(), sizeof(int64_t) * (grid + 1), cudaMemcpyHostToDevice, stream);
+  if (e != cudaSuccess) return cuda_fail(e, "partition upload");
+  P->part_key = key;
+  return RAP_OK;
+}
+
 static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output* out, cudaStream_t stream) {
   const int64_t B = raw->n_rows;
   cudaError_t e;
@@ -1086,29 +1138,17 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
     }
     return RAP_OK;
   }
-  // Work decomposition: 128-row sparse tiles per output,
-  // 128-row dense blocks per column group; one look-back word per sparse tile.
+  // Work decomposition: 128-row sparse tiles per output, then
+  // 128-row dense blocks per column group; one contiguous cost-balanced unit
+  // range per CTA.
   const int64_t F = (int64_t)P->souts.size();
   const int64_t T = (B + kTileRows - 1) / kTileRows;
   const int64_t n_sparse_tiles = F * T;
   const int64_t n_dense = P->dprogs.empty() ? 0 : (int64_t)P->dprogs.size() * ((B + kDenseBlockRows - 1) / kDenseBlockRows);
   if (n_sparse_tiles == 0 && n_dense == 0) return RAP_OK;
   const int64_t grid = std::min<int64_t>((int64_t)P->budget * P->ctas_per_sm, kMaxCtas);
-  if (n_sparse_tiles > P->status_cap) {  // look-back words (grow, never shrink; zero = no epoch)
-    if (P->d_status) {
-      e = cudaStreamSynchronize(stream);
-      if (e != cudaSuccess) return cuda_fail(e, "cudaStreamSynchronize");
-      cudaFree(P->d_status);
-      P->d_status = nullptr;
-      P->status_cap = 0;
-    }
-    const int64_t cap = std::max<int64_t>(n_sparse_tiles, 4096);
-    e = cudaMalloc(&P->d_status, sizeof(unsigned long long) * cap);
-    if (e != cudaSuccess) return fail(RAP_ERR_OUT_OF_MEMORY, "look-back word allocation");
-    e = cudaMemsetAsync(P->d_status, 0, sizeof(unsigned long long) * cap, stream);
-    if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync");
-    P->status_cap = cap;
-  }
+  rap_status pst = update_partition(P, B, raw->sp_nnz, n_sparse_tiles, n_dense, (int)grid, stream);
+  if (pst != RAP_OK) return pst;
   Common c{};
   c.ops = reinterpret_cast<const DevOp*>(P->blob + P->off_ops);
   c.sprogs = reinterpret_cast<const SProg*>(P->blob + P->off_sprogs);
@@ -1123,7 +1163,8 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
   c.n_sparse_tiles = n_sparse_tiles;
   c.n_dense_tiles = n_dense;
   c.sched = P->d_sched;
-  c.status = P->d_status;
+  c.part = P->d_part;
+  c.agg = P->d_agg;
   c.dense_out = out->dense_out;
   c.ld = out->dense_ld;
   c.lengths = out->lengths;
