@@ -198,11 +198,12 @@ rap_status rap_choose_budget(const rap_plan* plan, int64_t n_rows, const int64_t
 
 rap_status rap_plan_info_get(const rap_plan* plan, rap_plan_info* info);
 
-/* Profiling aid.  enable = 1: the following rap_preprocess calls record 16
+/* Profiling aid.  enable = 1: the following rap_preprocess calls record 24
  * uint64 stamps per CTA (slots 0..4 = %globaltimer at the phase boundaries,
- * 6 = SM id, 7 = partition rank, 8..15 = clock64 inside the first sparse
- * tile of warp 0) for up to `cap` CTAs.  enable = 0: synchronise the device
- * and copy the stamps of the last call to HOST host_out (uint64[cap * 16]);
+ * 5 = sparse tile range, 6 = SM id, 7 = partition rank, 8..23 = clock64
+ * inside the first sparse tile / dense block) for up to `cap` CTAs.
+ * enable = 0: synchronise the device and copy the stamps of the last call to
+ * HOST host_out (uint64[cap * 24]);
  * *n_desc receives that call's CTA count.  enable = -1: stop recording and
  * free the buffer. */
 rap_status rap_debug_trace(rap_plan* plan, int32_t enable, uint64_t* host_out, int64_t cap, int64_t* n_desc);

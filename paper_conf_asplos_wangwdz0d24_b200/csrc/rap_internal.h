@@ -170,10 +170,9 @@ struct Common {
   int64_t tiles_per_feature;  // T = ceil(n_rows / kTileRows)
   int64_t n_sparse_tiles;     // S = n_sparse_out * T
   int64_t n_dense_tiles;      // n_groups * ceil(n_rows / kDenseBlockRows)
-  // sched[0] = CTAs done, sched[1] = launch epoch, sched[2] = rank counter
-  // (arrival order); the last CTA resets the counters and advances the
-  // epoch, so launch parameters are identical from call to call (CUDA-graph
-  // replayable).
+  // sched[0] = CTAs done, sched[1] = launch epoch; the last CTA resets the
+  // counter and advances the epoch, so launch parameters are identical from
+  // call to call (CUDA-graph replayable).
   unsigned long long* sched;
   const int64_t* part;         // [grid + 1] unit range of each CTA rank
   unsigned long long* agg;     // [kMaxCtas] per-rank aggregate words (epoch-tagged)
@@ -189,7 +188,7 @@ struct Common {
   int64_t trace_cap;
 };
 
-constexpr int kTracePts = 16;
+constexpr int kTracePts = 24;
 
 struct LaunchRaw {
   int32_t n_dense, n_sparse;
@@ -208,8 +207,8 @@ RAP_HD uint64_t splitmix_H(uint64_t x) {
   return z ^ (z >> 31);
 }
 
-// Launch entry implemented in rap_kernel.cu (a CTA only waits on CTAs that
-// took a lower rank, i.e. are already resident: no co-residency is required).
+// Launch entry implemented in rap_kernel.cu (cooperative launch: every CTA
+// is resident, so a CTA may wait on its predecessors' aggregates).
 // Returns a cudaError_t value.
 int launch_fused(const Common& c, const LaunchRaw& raw, int grid, int smem_bytes, void* stream);
 // Dynamic shared memory per CTA for dense groups up to max_width columns.

@@ -42,6 +42,10 @@ struct KParams {
 };
 
 constexpr int kWarps = kThreads / 32;
+#ifndef RAP_LBATCH
+#define RAP_LBATCH 8
+#endif
+constexpr int kLBatch = RAP_LBATCH;  // tiles per batch of the length pass
 constexpr int kGroups = kTileRows / 32;  // row groups of a sparse tile (one row per lane each)
 constexpr int kNgScratch = kWarps * 4 * kMaxNgramK * 32 * 4;  // NGram warp scratch (smem, sparse phase)
 // Aggregate word of a CTA: [63:44] tag = launch epoch + 1 (0 = never
@@ -81,7 +85,14 @@ __device__ __forceinline__ void trace_stamp(const Common& c, int k) {
 
 // Profiling aid: clock64 at slot k of this CTA's trace row, once per launch
 // (first call wins), after the value `dep` is available.
+// Compiled in only with -DRAP_TRACE_CLK (dev builds, scripts/trace.py).
 __device__ __forceinline__ void trace_clk(const Common& c, int k, long long dep) {
+#ifndef RAP_TRACE_CLK
+  (void)c;
+  (void)k;
+  (void)dep;
+  if (false)
+#endif
   if (c.trace != nullptr && threadIdx.x == 0 && (int64_t)blockIdx.x < c.trace_cap) {
     asm volatile("" ::"l"(dep));
     unsigned long long* slot = c.trace + (int64_t)blockIdx.x * kTracePts + k;
@@ -484,7 +495,7 @@ __device__ __forceinline__ int warp_incl_scan(int v, int lane) {
 // Per-feature dispatch state a warp keeps in registers across its tiles.
 enum TileKind : int { TK_CANON = 0, TK_NGRAM_FAST = 1, TK_NGRAM = 2, TK_GENERIC = 3 };
 struct FeatCtx {
-  int f, kind, sk, src, has_fill;
+  int f, kind, sk, src, has_fill, ng_staged;
   int64_t xcap, null_xcap, fill;
   Canon q;  // canonical pipeline (TK_CANON), in registers
 };
@@ -501,6 +512,7 @@ __device__ __forceinline__ void load_ctx(const P& p, int f, FeatCtx& x) {
   x.xcap = ch.xcap;
   x.null_xcap = ch.null_xcap;
   x.fill = ch.fill;
+  x.ng_staged = 0;
   if (x.sk == SRC_SPARSE) {
     x.kind = x.q.ok ? TK_CANON : TK_GENERIC;
   } else if (x.sk == SRC_NGRAM) {
@@ -519,6 +531,8 @@ struct Quad {
   uint32_t w;
 };
 
+// Called by the whole warp (the fifth offset of lane i is lane i+1's first,
+// by shuffle: one 16-byte load per lane plus one scalar load for lane 31).
 __device__ __forceinline__ Quad load_quad(const int32_t* off, const uint32_t* bm, int64_t r0, int lane, int64_t B,
                                           bool aligned) {
   Quad q;
@@ -529,12 +543,14 @@ __device__ __forceinline__ Quad load_quad(const int32_t* off, const uint32_t* bm
     q.a[1] = v.y;
     q.a[2] = v.z;
     q.a[3] = v.w;
-    q.a[4] = __ldg(off + row + 4);
   } else {
 #pragma unroll
-    for (int k = 0; k < 5; ++k) q.a[k] = row + k <= B ? __ldg(off + row + k) : 0;
+    for (int k = 0; k < 4; ++k) q.a[k] = row + k <= B ? __ldg(off + row + k) : 0;
   }
+  const int32_t last = (lane == 31 && row + 4 <= B) ? __ldg(off + row + 4) : 0;
   q.w = (bm != nullptr && row < B) ? __ldg(bm + (row >> 5)) : 0xffffffffu;
+  const int32_t nxt = __shfl_down_sync(0xffffffffu, q.a[0], 1);
+  q.a[4] = lane == 31 ? last : nxt;
   return q;
 }
 
@@ -764,12 +780,15 @@ __device__ __noinline__ long long value_tile_generic(const P& p, int f, int64_t 
 // Offsets and ids of sparse tile (f, rt) whose first id goes to
 // values[base]; returns the tile's output length total.
 template <class P>
-__device__ __forceinline__ long long value_tile(const P& p, const FeatCtx& fc, int64_t rt, int lane, long long base,
+__device__ __forceinline__ long long value_tile(const P& p, FeatCtx& fc, int64_t rt, int lane, long long base,
                                                 int32_t* scr) {
   if (fc.kind == TK_CANON) return value_tile_canon(p, fc, rt, lane, base);
   if (fc.kind == TK_NGRAM_FAST) {
+    if (!fc.ng_staged) ngram_stage(p, fc.f, scr, lane);
+    fc.ng_staged = 1;
     const long long T = ngram_tile_fast(p, fc.f, rt, lane, base, scr);
     if (T >= 0) return T;
+    fc.ng_staged = 0;  // the general path reuses the scratch
   }
   if (fc.kind != TK_GENERIC) return value_tile_ngram(p, fc.f, rt, lane, base, scr);
   return value_tile_generic(p, fc.f, rt, lane, base);
@@ -818,6 +837,45 @@ __device__ __noinline__ void value_group_general(const P& p, int f, int64_t row0
 // Output length total of the NGram tile starting at row r0 (R7 count
 // max(0, sum of source lengths - n + 1), capped by FirstX): quad layout, 4
 // rows per lane, every source's offsets requested before any is used.
+// Output length total of the NGram tiles starting at rows r0 and r0 + 128
+// (nt = 1 or 2) of a feature with k <= 4 sparse sources: all 2k quads in
+// flight together.
+template <class P>
+__device__ __forceinline__ long long ngram_tiles_len2(const P& p, const SProg& pg, int64_t r0, int nt, int lane) {
+  const int64_t B = p.c.n_rows;
+  const int k = pg.ng.k, n = pg.ng.n;
+  const int64_t xo = pg.ch.xcap;
+  Chain sc[4];
+#pragma unroll
+  for (int j = 0; j < 4; ++j)
+    if (j < k) sc[j] = pg.src[j];
+  Quad q[2][4];
+#pragma unroll
+  for (int t = 0; t < 2; ++t)
+#pragma unroll
+    for (int j = 0; j < 4; ++j)
+      if (t < nt && j < k) {
+        const int32_t* off = p.off[sc[j].src];
+        q[t][j] = load_quad(off, p.svalid[sc[j].src], r0 + t * kTileRows, lane, B,
+                            (reinterpret_cast<uintptr_t>(off) & 15) == 0);
+      }
+  int sum = 0;
+#pragma unroll
+  for (int t = 0; t < 2; ++t)
+    if (t < nt) {
+#pragma unroll
+      for (int kk = 0; kk < 4; ++kk) {
+        const int64_t row = r0 + t * kTileRows + 4 * lane + kk;
+        int tot = 0;
+#pragma unroll
+        for (int j = 0; j < 4; ++j)
+          if (j < k) tot += quad_len(q[t][j], kk, lane, row, B, sc[j].xcap, sc[j].has_fill, sc[j].null_xcap);
+        if (row < B) sum += (int32_t)min((int64_t)max(tot - n + 1, 0), xo);
+      }
+    }
+  return warp_sum64(sum);
+}
+
 template <class P>
 __device__ __noinline__ long long ngram_tile_len(const P& p, const SProg& pg, int64_t r0, int lane) {
   const int64_t B = p.c.n_rows;
@@ -870,7 +928,38 @@ struct NgParams {  // ngram_tile_fast parameters, staged in warp scratch
   NGramDesc ng;
   int64_t xcap;
 };
-static_assert(sizeof(NgParams) <= 4 * kMaxNgramK * 32 * 4, "NgParams exceeds the warp scratch");
+static_assert(offsetof(NgParams, scn) == sizeof(Chain) * 4 && offsetof(NgParams, post) == offsetof(NgParams, scn) + sizeof(Canon) * 4 &&
+                  offsetof(NgParams, ng) == offsetof(NgParams, post) + sizeof(Canon) && sizeof(Chain) % 8 == 0 &&
+                  sizeof(Canon) % 8 == 0 && sizeof(NGramDesc) % 8 == 0,
+              "NgParams is staged as one run of 8-byte words");
+constexpr int kNgParamWords = align_up((int)sizeof(NgParams), 16) / 4;
+static_assert(kNgParamWords * 4 + 4 * kTileRows * 4 <= 4 * kMaxNgramK * 32 * 4, "ngram_tile_fast scratch too large");
+
+// Stage feature f's fast-NGram parameters into the warp scratch: every
+// lane's loads in flight before any store.
+template <class P>
+__device__ __forceinline__ void ngram_stage(const P& p, int f, int32_t* scr, int lane) {
+  const SProg& pg = p.c.sprogs[f];
+  NgParams& G = *reinterpret_cast<NgParams*>(scr);
+  constexpr int W1 = sizeof(G.src) / 8, W2 = sizeof(G.scn) / 8, W3 = sizeof(G.post) / 8, W4 = sizeof(G.ng) / 8;
+  constexpr int WT = W1 + W2 + W3 + W4, PER = (WT + 31) / 32;
+  long long r[PER];
+#pragma unroll
+  for (int i = 0; i < PER; ++i) {
+    const int w = lane + 32 * i;
+    const long long* src = w < W1 ? reinterpret_cast<const long long*>(pg.src) + w
+                         : w < W1 + W2 ? reinterpret_cast<const long long*>(pg.src_cn) + (w - W1)
+                         : w < W1 + W2 + W3 ? reinterpret_cast<const long long*>(&pg.cn) + (w - W1 - W2)
+                                            : reinterpret_cast<const long long*>(&pg.ng) + (w - W1 - W2 - W3);
+    if (w < WT) r[i] = __ldg(src);
+  }
+  long long* dst = reinterpret_cast<long long*>(&G);  // src, scn, post, ng are contiguous in NgParams
+#pragma unroll
+  for (int i = 0; i < PER; ++i)
+    if (lane + 32 * i < WT) dst[lane + 32 * i] = r[i];
+  if (lane == 0) G.xcap = pg.ch.xcap;
+  __syncwarp();
+}
 
 // Fast NGram tile (R7) for k <= 4 canonical single-source chains when every
 // row of every source has at most one id and at most n ids in total: then a
@@ -880,19 +969,13 @@ static_assert(sizeof(NgParams) <= 4 * kMaxNgramK * 32 * 4, "NgParams exceeds the
 // the tile's output length total, or -1 with nothing written when the tile
 // is not eligible.
 template <class P>
-__device__ __noinline__ long long ngram_tile_fast(const P& p, int f, int64_t rt, int lane, long long base,
+__device__ __forceinline__ long long ngram_tile_fast(const P& p, int f, int64_t rt, int lane, long long base,
                                                  int32_t* scr) {
-  const SProg& pg = p.c.sprogs[f];
   trace_clk(p.c, 13, 0);
-  // the parameters go to warp-private shared memory in one burst (no lazy
-  // global reads on the dependent path)
-  NgParams& G = *reinterpret_cast<NgParams*>(scr);
-  warp_copy8(G.src, pg.src, sizeof(G.src), lane);
-  warp_copy8(G.scn, pg.src_cn, sizeof(G.scn), lane);
-  warp_copy8(&G.post, &pg.cn, sizeof(G.post), lane);
-  warp_copy8(&G.ng, &pg.ng, sizeof(G.ng), lane);
-  if (lane == 0) G.xcap = pg.ch.xcap;
-  __syncwarp();
+  // parameters: staged in warp-private shared memory by ngram_stage (no lazy
+  // global reads on the dependent path); per-(source, row) id positions after
+  const NgParams& G = *reinterpret_cast<const NgParams*>(scr);
+  int32_t* pos = scr + kNgParamWords;  // [4][kTileRows]: child index, -1 = fill, -2 = absent
   const int k = G.ng.k, n = G.ng.n;
   const int64_t B = p.c.n_rows;
   const int64_t r0 = rt * kTileRows;
@@ -920,9 +1003,6 @@ __device__ __noinline__ long long ngram_tile_fast(const P& p, int f, int64_t rt,
 #pragma unroll
   for (int kk = 0; kk < 4; ++kk) ok &= pn[kk] <= n;
   if (!__all_sync(0xffffffffu, ok)) return -1;
-  // all ids of all sources in flight
-  int64_t v[4][4];
-  unsigned pres[4], full[4];
   int32_t l[4], e[4];
   int tot = 0;
 #pragma unroll
@@ -931,22 +1011,23 @@ __device__ __noinline__ long long ngram_tile_fast(const P& p, int f, int64_t rt,
     e[kk] = tot;
     tot += l[kk];
   }
+  // presence (bit 4j+kk) and id positions of every (source, row)
+  unsigned pres = 0, full = 0;
 #pragma unroll
   for (int j = 0; j < 4; ++j)
     if (j < k) {
       const Chain& sc = G.src[j];
-      const int64_t* val = p.val[sc.src];
-      pres[j] = full[j] = 0;
+      int a[4];
 #pragma unroll
       for (int kk = 0; kk < 4; ++kk) {
         const bool pr = l[kk] == 1 && quad_len(q[j], kk, lane, row + kk, B, sc.xcap, sc.has_fill, sc.null_xcap) == 1;
         const bool fu = quad_valid(q[j], kk, lane);
-        pres[j] |= (pr ? 1u : 0u) << kk;
-        full[j] |= (fu ? 1u : 0u) << kk;
-        v[j][kk] = (pr && fu) ? __ldg(val + q[j].a[kk]) : sc.fill;
+        pres |= (pr ? 1u : 0u) << (4 * j + kk);
+        full |= (fu ? 1u : 0u) << (4 * j + kk);
+        a[kk] = pr ? (fu ? q[j].a[kk] : -1) : -2;
       }
+      *reinterpret_cast<int4*>(pos + j * kTileRows + 4 * lane) = make_int4(a[0], a[1], a[2], a[3]);
     }
-  trace_clk(p.c, 14, v[0][0] + v[1][0] + v[2][0] + v[0][3] + v[1][3] + v[2][3]);
   const int incl = warp_incl_scan(tot, lane);
   const int L = incl - tot;
   const int T = __shfl_sync(0xffffffffu, incl, 31);
@@ -956,14 +1037,30 @@ __device__ __noinline__ long long ngram_tile_fast(const P& p, int f, int64_t rt,
   uint64_t h[4];
 #pragma unroll
   for (int kk = 0; kk < 4; ++kk) h[kk] = G.ng.hsalt;  // R7: h = H(salt); h = H(h ^ c[q])
+  // sources in order, the next source's ids in flight while this one runs
+  // its canonical pipeline (R3-R8) and feeds the window hash
+  int64_t vn[4];
+  auto load_src = [&](int j, int64_t (&v)[4]) {
+    const int4 a = *reinterpret_cast<const int4*>(pos + j * kTileRows + 4 * lane);
+    const int64_t* val = p.val[G.src[j].src];
+    const int64_t fill = G.src[j].fill;
+    v[0] = a.x >= 0 ? __ldg(val + a.x) : fill;
+    v[1] = a.y >= 0 ? __ldg(val + a.y) : fill;
+    v[2] = a.z >= 0 ? __ldg(val + a.z) : fill;
+    v[3] = a.w >= 0 ? __ldg(val + a.w) : fill;
+  };
+  load_src(0, vn);
+  trace_clk(p.c, 14, vn[0] + vn[3]);
+#pragma unroll 1
+  for (int j = 0; j < k; ++j) {
+    int64_t v[4] = {vn[0], vn[1], vn[2], vn[3]};
+    if (j + 1 < k) load_src(j + 1, vn);
+    const unsigned pj = (pres >> (4 * j)) & 15u, fj = (full >> (4 * j)) & 15u;
+    canon_apply_n<4>(G.scn[j], itab, v, pj, fj);
 #pragma unroll
-  for (int j = 0; j < 4; ++j)
-    if (j < k) {
-      canon_apply_n<4>(G.scn[j], itab, v[j], pres[j], full[j]);
-#pragma unroll
-      for (int kk = 0; kk < 4; ++kk)
-        if ((pres[j] >> kk) & 1u) h[kk] = splitmix_H(h[kk] ^ (uint64_t)v[j][kk]);
-    }
+    for (int kk = 0; kk < 4; ++kk)
+      if ((pj >> kk) & 1u) h[kk] = splitmix_H(h[kk] ^ (uint64_t)v[kk]);
+  }
   int64_t o[4];
   unsigned act = 0;
 #pragma unroll
@@ -1111,10 +1208,11 @@ __device__ __noinline__ long long value_tile_ngram(const P& p, int f, int64_t rt
 struct CtaState {
   uint64_t bar;
   long long ticket;
-  int staged, phase;
+  int staged, phase, dgroup;  // dgroup: column group whose DProg is in smem (-1: none)
 };
 
 constexpr int kDProgBytes = align_up((int)sizeof(DProg), 16);
+static_assert(sizeof(DProg) % 16 == 0, "DProg copies are whole 16-byte words");
 
 __host__ __device__ constexpr int dense_in_bytes() { return 16 * kDenseBlockRows * 4 + 16 * 8 * 4; }
 
@@ -1159,6 +1257,7 @@ __device__ void dense_block(const P& p, int gi, int64_t rb, unsigned char* smem,
   const int64_t r0 = rb * kDenseBlockRows;
   const int nr = (int)min((int64_t)kDenseBlockRows, B - r0);
   const int nw = (nr + 31) >> 5;
+  trace_clk(p.c, 16, 0);
   if (warp == 0) {
     const DProg* g = p.c.dprogs + gi;
     const int nu = __ldg(&g->n_units), no = __ldg(&g->n_ops), nf = __ldg(&g->n_ftab), nc = __ldg(&g->n_cols);
@@ -1184,18 +1283,24 @@ __device__ void dense_block(const P& p, int gi, int64_t rb, unsigned char* smem,
       }
     }
     if (lane == 0) cs.staged = stage ? 1 : 0;
-    const int4* src = reinterpret_cast<const int4*>(g);
+  }
+  if (cs.dgroup != gi) {
+    // the group's program to shared memory once per CTA and group: every
+    // thread's loads in flight before any store
+    const int4* src = reinterpret_cast<const int4*>(p.c.dprogs + gi);
     int4* dst = reinterpret_cast<int4*>(dp);
-    const int n_hdr = align_up((int)offsetof(DProg, units) + nu * (int)sizeof(DUnit), 16) >> 4;
-    for (int k = lane; k < n_hdr; k += 32) dst[k] = __ldg(src + k);
-    const int4* so = reinterpret_cast<const int4*>(g->ops);
-    int4* d2 = reinterpret_cast<int4*>(dp->ops);
-    for (int k = lane; k < (align_up(no * (int)sizeof(DevOp), 16) >> 4); k += 32) d2[k] = __ldg(so + k);
-    const int4* sf = reinterpret_cast<const int4*>(g->ftab);
-    int4* d3 = reinterpret_cast<int4*>(dp->ftab);
-    for (int k = lane; k < (align_up(nf * 4, 16) >> 4); k += 32) d3[k] = __ldg(sf + k);
+    constexpr int kN16 = kDProgBytes / 16, kPer = (kN16 + kThreads - 1) / kThreads;
+    int4 r[kPer];
+#pragma unroll
+    for (int i = 0; i < kPer; ++i)
+      if (tid + i * kThreads < kN16) r[i] = __ldg(src + tid + i * kThreads);
+#pragma unroll
+    for (int i = 0; i < kPer; ++i)
+      if (tid + i * kThreads < kN16) dst[tid + i * kThreads] = r[i];
   }
   __syncthreads();
+  if (tid == 0) cs.dgroup = gi;
+  trace_clk(p.c, 17, 0);
   const int W = dp->width;
   const int LD = W | 1;  // odd row pitch: conflict-free column writes
   if (dp->any_onehot)
@@ -1203,6 +1308,7 @@ __device__ void dense_block(const P& p, int gi, int64_t rb, unsigned char* smem,
   const bool staged = cs.staged;
   if (staged) mbar_wait(&cs.bar, cs.phase);
   __syncthreads();
+  trace_clk(p.c, 18, 0);
   const int nu = dp->n_units;
   // (row, unit) pairs over all threads, unit-major so a warp shares its unit
   for (int idx = tid; idx < nr * nu; idx += kThreads) {
@@ -1233,6 +1339,7 @@ __device__ void dense_block(const P& p, int gi, int64_t rb, unsigned char* smem,
     }
   }
   __syncthreads();
+  trace_clk(p.c, 19, 0);
   float* out = p.c.dense_out + r0 * p.c.ld + dp->col0;
   const int64_t ld = p.c.ld;
   if (ld == W && LD == W) {
@@ -1248,6 +1355,7 @@ __device__ void dense_block(const P& p, int gi, int64_t rb, unsigned char* smem,
     for (int r = warp; r < nr; r += kWarps)
       for (int cc = lane; cc < W; cc += 32) out[r * ld + cc] = tile[r * LD + cc];
   }
+  trace_clk(p.c, 20, 0);
   if (tid == 0 && staged) cs.phase ^= 1;
 }
 
@@ -1276,7 +1384,7 @@ __device__ __forceinline__ long long block_sum(long long v, long long* red) {
 }
 
 #ifndef RAP_MIN_CTAS
-#define RAP_MIN_CTAS 4
+#define RAP_MIN_CTAS 3  // 85 registers: the fastest of 2/3/4 on the C2 graph (profiles/README.md)
 #endif
 template <int MD, int MS>
 __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const __grid_constant__ KParams<MD, MS> p) {
@@ -1284,27 +1392,26 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
   __shared__ CtaState cs;
   __shared__ long long s_slots[kWarps];
   __shared__ long long s_red[kWarps];
-  __shared__ unsigned long long s_epoch;
-  __shared__ int s_rank, s_last;
+  __shared__ int s_last;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  // The epoch load is consumed only when the aggregate is published, so its
+  // latency hides under the length pass.  Ranks are block indices: the
+  // launch is cooperative, so every CTA is resident and a CTA waits only on
+  // resident predecessors.
+  const unsigned long long epoch = ld_relaxed(p.c.sched + 1);
   if (tid == 0) {
     mbar_init(&cs.bar, 1);
     cs.phase = 0;
-    // partition rank = arrival order, so a CTA only ever waits on CTAs that
-    // are already resident (deadlock-free under any co-running load)
-    s_rank = (int)atomicAdd(p.c.sched + 2, 1ull);
-    s_epoch = ld_relaxed(p.c.sched + 1);
+    cs.dgroup = -1;
   }
-  __syncthreads();
   trace_stamp(p.c, 0);
+  const int rank = blockIdx.x;
   if (p.c.trace != nullptr && tid == 0 && (int64_t)blockIdx.x < p.c.trace_cap) {
     unsigned smid;
     asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
     p.c.trace[(int64_t)blockIdx.x * kTracePts + 6] = smid;
-    p.c.trace[(int64_t)blockIdx.x * kTracePts + 7] = (unsigned long long)s_rank;
+    p.c.trace[(int64_t)blockIdx.x * kTracePts + 7] = (unsigned long long)rank;
   }
-  const unsigned long long epoch = s_epoch;
-  const int rank = s_rank;
   const int64_t S = p.c.n_sparse_tiles, T = p.c.tiles_per_feature;
   const int64_t s0 = __ldg(p.c.part + rank), s1 = __ldg(p.c.part + rank + 1);  // my sparse tiles
   int32_t* scr = reinterpret_cast<int32_t*>(smem) + warp * (4 * kMaxNgramK * 32);
@@ -1315,6 +1422,7 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
   const int64_t ns = s1 - s0;
   const int64_t w0 = s0 + ns * warp / kWarps, w1 = s0 + ns * (warp + 1) / kWarps;
   long long mine = 0, part = 0;  // warp-uniform / per-lane partial totals
+  trace_clk(p.c, 21, 0);
   {
     FeatCtx fc;
     fc.f = -1;
@@ -1324,17 +1432,17 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
       if (f != fc.f) load_ctx(p, f, fc);
       const int64_t tend = min(w1, (int64_t)(f + 1) * T);
       if (fc.sk == SRC_SPARSE) {
-        // 4 tiles' offsets in flight at a time
+        // kLBatch tiles' offsets in flight at a time
         const int32_t* off = p.off[fc.src];
         const uint32_t* bm = p.svalid[fc.src];
         const bool al = (reinterpret_cast<uintptr_t>(off) & 15) == 0;
-        for (; t < tend; t += 4) {
-          Quad q[4];
+        for (; t < tend; t += kLBatch) {
+          Quad q[kLBatch];
 #pragma unroll
-          for (int j = 0; j < 4; ++j)
+          for (int j = 0; j < kLBatch; ++j)
             if (t + j < tend) q[j] = load_quad(off, bm, (t + j - (int64_t)f * T) * kTileRows, lane, B, al);
 #pragma unroll
-          for (int j = 0; j < 4; ++j)
+          for (int j = 0; j < kLBatch; ++j)
             if (t + j < tend) {
               const int64_t row = (t + j - (int64_t)f * T) * kTileRows + 4 * lane;
 #pragma unroll
@@ -1342,14 +1450,23 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
             }
         }
         t = tend;
+      } else if (fc.kind == TK_NGRAM_FAST) {
+        const SProg& pg = p.c.sprogs[f];
+        while (t < tend) {
+          const int nt = (int)min((int64_t)2, tend - t);
+          mine += ngram_tiles_len2(p, pg, (t - (int64_t)f * T) * kTileRows, nt, lane);  // warp-uniform
+          t += nt;
+        }
       } else {
         for (; t < tend; ++t) mine += tile_total(p, f, t - (int64_t)f * T, lane);  // warp-uniform
       }
     }
   }
   mine += warp_sum64(part);
+  trace_clk(p.c, 22, mine);
   if (lane == 0) s_slots[warp] = mine;
   const long long agg = block_sum(lane == 0 ? mine : 0ll, s_red);
+  trace_clk(p.c, 23, agg);
   const unsigned long long tag = epoch + 1ull;
   if (tid == 0) st_relaxed(p.c.agg + rank, (tag << kEpochShift) | (unsigned long long)agg);
   trace_stamp(p.c, 1);
@@ -1432,7 +1549,6 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
     __syncthreads();
     if (tid == 0) {
       p.c.sched[0] = 0ull;
-      p.c.sched[2] = 0ull;
       p.c.sched[1] = wrap ? 0ull : epoch + 1ull;
       __threadfence();
     }
@@ -1465,7 +1581,11 @@ static int launch_t(const Common& c, const LaunchRaw& raw, int grid, int smem, c
   cfg.blockDim = dim3(kThreads);
   cfg.dynamicSmemBytes = smem;
   cfg.stream = st;
-  cfg.numAttrs = 0;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeCooperative;  // all CTAs co-resident (the scan waits on predecessors)
+  attr[0].val.cooperative = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
   cudaError_t e = cudaLaunchKernelEx(&cfg, rap_fused_kernel<MD, MS>, p);
   if (e != cudaSuccess) return (int)e;
   return (int)cudaGetLastError();

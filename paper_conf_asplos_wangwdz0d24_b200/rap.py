@@ -304,8 +304,8 @@ class Plan:
         _check(load().rap_debug_trace(self.handle, 1, None, cap, None))
 
     def trace_read(self, cap: int):
-        """Stamps of the last call: uint64 [n_cta, 16] (profiling aid)."""
-        buf = np.zeros((cap, 16), dtype=np.uint64)
+        """Stamps of the last call: uint64 [n_cta, 24] (profiling aid)."""
+        buf = np.zeros((cap, 24), dtype=np.uint64)
         n = C.c_int64()
         _check(load().rap_debug_trace(self.handle, 0, buf.ctypes.data, cap, C.byref(n)))
         return buf[: min(cap, n.value)]

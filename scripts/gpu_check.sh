@@ -7,6 +7,7 @@ python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1
 timeout 900 python -m pytest tests -x -q -m gpu > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_gpu.log
 timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.log 2>&1; echo "smoke rc=$?" >> gpurun_out/smoke.log
 timeout 600 python bench.py > gpurun_out/bench.json 2> gpurun_out/bench.err
+timeout 600 python bench.py --impl reference --steps 5 --warmup 3 > gpurun_out/bench_ref.json 2> gpurun_out/bench_ref.err
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:rap_fused -s 5 -c 20 --csv --log-file gpurun_out/launches.csv python bench.py --profile --steps 30 --warmup 5 > gpurun_out/ncu_launch.log 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:rap_fused -s 5 -c 2 -o gpurun_out/prof -f python bench.py --profile --steps 10 --warmup 5 > gpurun_out/ncu_full.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:rap_fused -s 5 -c 1 -o gpurun_out/prof -f python bench.py --profile --steps 10 --warmup 5 > gpurun_out/ncu_full.log 2>&1
 ls -la gpurun_out

@@ -74,6 +74,18 @@ def main():
         d = np.diff(cl[okc], axis=1)
         print("  first fast-ngram tile of warp 0 (cycles, median): params+quads+values %d  hash+stores %d" %
               tuple(np.median(d, axis=0)))
+    cl = tr[:, 16:21].astype(np.int64)
+    okc = (cl > 0).all(axis=1)
+    if okc.any():
+        d = np.diff(cl[okc], axis=1)
+        print("  first dense block (cycles, median): prog+issue %d  staged wait %d  compute %d  store %d" %
+              tuple(np.median(d, axis=0)))
+    cl = tr[:, 21:24].astype(np.int64)
+    okc = (cl > 0).all(axis=1)
+    if okc.any():
+        d = np.diff(cl[okc], axis=1)
+        print("  phase L (cycles, median): warp 0 loop %d  block wait %d   (p90 %d %d)" %
+              (tuple(np.median(d, axis=0)) + tuple(np.percentile(d, 90, axis=0))))
     plan.close()
 
 
