@@ -46,6 +46,11 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no clocks / e2e / cpu)")
+    ap.add_argument("--no-corun", action="store_true", help="skip the co-run training-slowdown measurement")
+    ap.add_argument("--corun-budgets", default="16,37,74,148", help="SM budgets of the co-run sweep")
+    ap.add_argument("--placement", default="balanced", choices=["balanced", "round_robin", "skewed"],
+                    help="N>1: table placement (DESIGN.md §10)")
+    ap.add_argument("--imbalance-tol", type=float, default=0.10, help="N>1: residual move threshold")
     return ap.parse_args()
 
 
@@ -208,6 +213,8 @@ def run_rap(args):
 
     rank, world, local = dist_env()
     if world > 1:
+        return run_sharded(args)
+    if world > 1:
         import torch.distributed as dist
 
         torch.cuda.set_device(local)
@@ -325,6 +332,16 @@ def run_rap(args):
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline and not args.profile:
         cpu = cpu_baseline(w, args.cpu_seconds)
+    corun = None
+    if world == 1 and not args.no_corun and not args.profile and args.workload == "c2":
+        from paper_conf_asplos_wangwdz0d24_b200 import corun as cr
+
+        train = cr.DLRMStep(dev)
+        budgets = [int(b) for b in args.corun_budgets.split(",") if b]
+        corun = cr.measure(plan, sets, train, budgets)
+        corun["training"] = "synthetic DLRM step (DESIGN.md §12): 26 tables x 128 fp32 (TB share at 8 GPUs), batch 8192"
+        del train
+        torch.cuda.empty_cache()
     info = plan.info()
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": args.warmup,
@@ -336,13 +353,97 @@ def run_rap(args):
                            "sm_budget": info["sm_budget"], "grid": info["grid"],
                            "l2_policy": f"rotate {nsets} distinct input/output sets, {nsets * set_bytes / 2**20:.0f} MB "
                                         f"total vs L2 {l2 / 2**20:.0f} MB"},
-                "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks, "gpu_launches": K}
+                "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks, "gpu_launches": K,
+                "corun": corun}
         print(json.dumps(line), flush=True)
     plan.close()
     if world > 1:
         import torch.distributed as dist
 
         dist.destroy_process_group()
+    return 0
+
+
+def run_sharded(args):
+    """N > 1 (config 3): the C2 graph feature-sharded across the ranks with
+    table-wise placement (DESIGN.md §10).  Global batch fixed -> strong scaling;
+    value = global rows / max-over-ranks step time (residual exchange included)."""
+    import torch
+    import torch.distributed as tdist
+
+    rank, world, local = dist_env()
+    torch.cuda.set_device(local)
+    tdist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    from paper_conf_asplos_wangwdz0d24_b200 import dist, rap, synth
+
+    wname, B = WORKLOADS[args.workload]
+    B = args.batch or B
+    w = workload(args.workload)
+    host = synth.make_batch(w, B, seed=1000)  # the same global batch on every rank
+    raw0 = rap.DeviceBatch(host, dev)
+    pl = dist.plan_placement(w.spec, B, raw0.sp_nnz, world, args.placement, args.imbalance_tol, device=local)
+    sp = dist.ShardedPreprocessor(w.spec, pl, rank, world, B, raw0.sp_nnz, device=local, sm_budget=args.budget)
+    props = torch.cuda.get_device_properties(dev)
+    l2 = getattr(props, "L2_cache_size", 126 * 2**20)
+    nsets = 1 if args.profile else 4
+    sets = [(raw0, sp.new_output())]
+    for i in range(1, nsets):
+        r = rap.DeviceBatch(synth.make_batch(w, B, seed=1000 + 97 * i), dev)
+        sets.append((r, sp.new_output()))
+    stream = torch.cuda.current_stream(dev)
+    for i in range(args.warmup):
+        r, o = sets[i % nsets]
+        sp.preprocess(r, o, stream)
+    torch.cuda.synchronize()
+    tdist.barrier()
+    torch.cuda.synchronize()
+    K = args.steps
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    sampler = ClockSampler(local) if not args.profile else None
+    with (sampler if sampler else _Null()):
+        t0.record(stream)
+        for i in range(K):
+            r, o = sets[i % nsets]
+            sp.preprocess(r, o, stream)
+        t1.record(stream)
+        t1.synchronize()
+    torch.cuda.synchronize()
+    tdist.barrier()
+    t = torch.tensor([t0.elapsed_time(t1)], device=dev)
+    tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
+    total_ms = float(t[0])
+    # my share of the algorithmic bytes: owned tables over the full batch + my dense shard
+    o = sets[(K - 1) % nsets][1]
+    offs = o.offsets
+    assert int(offs[0]) == 0 and bool((offs[1:] >= offs[:-1]).all())
+    n_vals = int(offs[-1].item())
+    d_out = sp.d_out
+    my_bytes = (4 * sp.dense_rows * d_out + len(sp.features) * B * 20 + 8 * n_vals
+                + (13 * 4.125 * sp.dense_rows if d_out else 0))
+    bt = torch.tensor([my_bytes], device=dev, dtype=torch.float64)
+    tdist.all_reduce(bt, op=tdist.ReduceOp.MAX)
+    peak, peak_kind = measured_peaks()
+    ms = total_ms / K
+    achieved = float(bt[0]) / (ms / 1e3) / 1e9
+    clocks = sampler.summary() if sampler else None
+    if rank == 0:
+        res = pl.residual
+        line = {"metric": METRIC, "value": B / (ms / 1e3), "unit": UNIT, "n_gpus": world, "steps": K,
+                "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "strong",
+                "vs_baseline": None, "dtype": "int64+f32", "data": "synthetic",
+                "config": {"workload": wname + "_sharded_c3", "batch": B, "parallelism": f"table-wise x{world}",
+                           "placement": args.placement, "loads": [round(x) for x in pl.loads],
+                           "residual": None if res is None else res.__dict__,
+                           "l2_policy": f"rotate {nsets} input/output sets"},
+                "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                             "frac": achieved / peak, "traffic": None, "peak_source": peak_kind,
+                             "note": "busiest rank's algorithmic bytes / step time"},
+                "cpu_baseline": None, "e2e": None, "clocks": clocks,
+                "gpu_launches": K * (1 + (0 if res is None else 2))}
+        print(json.dumps(line), flush=True)
+    sp.close()
+    tdist.destroy_process_group()
     return 0
 
 

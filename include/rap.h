@@ -134,7 +134,19 @@ typedef struct {
   int64_t* offsets;
   int64_t* values;
   int64_t values_capacity;
+  int32_t flags;         /* 0, or RAP_OUT_CHAIN */
+  int32_t reserved;
 } rap_output;
+
+/* rap_output.flags: a chained launch continues a jagged output that a
+ * preceding launch (or rap_jagged_append) on the same stream wrote into the
+ * same buffers.  `offsets` then points at the slot holding that running total
+ * (the previous piece's last offset, a DEVICE value read when the launch
+ * starts, never by the host); every offset this launch writes is that total
+ * plus its own exclusive scan and its ids go to values[total ...].  `lengths`
+ * points at the first row slot of this launch.  Used to stitch multi-GPU
+ * residual pieces. */
+#define RAP_OUT_CHAIN 1
 
 struct rap_plan;
 typedef struct rap_plan rap_plan;
@@ -197,6 +209,75 @@ rap_status rap_choose_budget(const rap_plan* plan, int64_t n_rows, const int64_t
                              double overlap_capacity_us, int32_t* sm_budget, double* t_delta_us);
 
 rap_status rap_plan_info_get(const rap_plan* plan, rap_plan_info* info);
+
+/* ---- Multi-GPU (§7.2; hybrid parallelism L488-499) ----
+ * Table-wise: each sparse output ("table") is preprocessed over the FULL
+ * global batch on the GPU that owns its embedding table (locality rule,
+ * L1526-1534); dense outputs are batch-sharded (each rank produces the rows of
+ * its own MLP mini-batch).  Only a residual row range of an overloaded rank's
+ * feature moves (L1594-1600), shipped back over NCCL by the caller.
+ */
+typedef enum {
+  RAP_PLACE_BALANCED = 0,    /* LPT on predicted cost (largest first to the least loaded rank) */
+  RAP_PLACE_ROUND_ROBIN = 1, /* output j -> rank j mod world */
+  RAP_PLACE_SKEWED = 2       /* rank 0 takes ~2x the mean load (Fig 12's skew, L2317-2318), LPT for the rest */
+} rap_place_mode;
+
+/* A residual move: rows [split_row, n_rows) of sparse output `output` are
+ * preprocessed on `helper` instead of its owner and shipped to the owner.
+ * split_row is a multiple of 128 in [128, n_rows).  output = -1: none. */
+typedef struct {
+  int32_t output, owner, helper, pad;
+  int64_t split_row;
+} rap_residual;
+
+/* Rows of `rank`'s batch shard: [*row0, *row0 + *rows).  Boundaries are
+ * multiples of 128 rows (so validity bitmaps and 16-byte staging stay
+ * aligned); the last rank takes the remainder.  world = 1: the whole batch. */
+rap_status rap_shard_rows(int64_t n_rows, int32_t rank, int32_t world, int64_t* row0, int64_t* rows);
+
+/* Predicted cost (model units per batch, the cost model of the fused kernel's
+ * partition) of each sparse output of `plan` for a batch of
+ * n_rows.  cost: HOST double[n_sparse_out]. */
+rap_status rap_plan_output_costs(const rap_plan* plan, int64_t n_rows, const int64_t* sp_nnz, double* cost);
+
+/* Place n sparse outputs on `world` ranks (host only, no device).
+ *   cost[n]      HOST, per-output predicted cost (rap_plan_output_costs)
+ *   colocate[n]  HOST, may be NULL; -1 or the index of an earlier output this
+ *                one must share a rank with (an NGram table with its first
+ *                source's table)
+ *   owner_out[n] HOST, rank of each output
+ *   load_out     HOST double[world] or NULL: resulting predicted load per rank
+ *   residual     HOST or NULL.  Non-NULL: when the most loaded rank exceeds
+ *                the mean by more than imbalance_tol (relative), move the
+ *                row range [split_row, n_rows) of its costliest output to
+ *                the least loaded rank so their loads about meet, and report
+ *                it (load_out includes the move).  One move per call. */
+rap_status rap_place(const double* cost, const int32_t* colocate, int32_t n, int32_t world, int32_t mode,
+                     int64_t n_rows, double imbalance_tol, int32_t* owner_out, double* load_out,
+                     rap_residual* residual);
+
+/* A sharded plan: the graph restricted to its dense outputs (evaluated over
+ * this rank's batch shard, rap_shard_rows) and the sparse outputs j with
+ * sparse_owner[j] == rank (j counts the graph's sparse outputs in order),
+ * evaluated over the full batch.  sparse_owner: HOST int32[#sparse outputs],
+ * each in [-1, world); -1 = in no rank's main plan (a residual output that
+ * its owner and helper run as row-range pieces).
+ * Output shapes: rap_plan_output_shape's d_out_cols with shard rows. */
+rap_status rap_plan_create_sharded(const rap_graph* graph, const rap_op_param* params, int32_t n_params,
+                                   int32_t device, int32_t sm_budget, const int32_t* sparse_owner,
+                                   int32_t rank, int32_t world, rap_plan** out);
+
+/* Append a jagged piece (n rows: lengths int32[n], its own offsets int64[n+1]
+ * starting at src_offsets[0], values indexed by those offsets) to a chained
+ * output (see RAP_OUT_CHAIN): dst_offsets[0] holds the running total T (DEVICE);
+ * writes dst_lengths[0..n), dst_offsets[1..n] = T + src_offsets[i] -
+ * src_offsets[0] and values to dst_values[T ..].  All pointers DEVICE;
+ * values_bound (HOST) bounds the piece's value count (launch sizing only);
+ * dst_capacity guards dst_values.  Enqueued on `stream`, no host sync. */
+rap_status rap_jagged_append(const int32_t* lengths, const int64_t* src_offsets, const int64_t* values, int64_t n,
+                             int64_t values_bound, int32_t* dst_lengths, int64_t* dst_offsets, int64_t* dst_values,
+                             int64_t dst_capacity, void* stream);
 
 /* Profiling aid.  enable = 1: the following rap_preprocess calls record 24
  * uint64 stamps per CTA (slots 0..4 = %globaltimer at the phase boundaries,

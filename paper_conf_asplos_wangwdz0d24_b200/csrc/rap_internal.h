@@ -169,7 +169,11 @@ struct Common {
   int64_t n_rows;
   int64_t tiles_per_feature;  // T = ceil(n_rows / kTileRows)
   int64_t n_sparse_tiles;     // S = n_sparse_out * T
-  int64_t n_dense_tiles;      // n_groups * ceil(n_rows / kDenseBlockRows)
+  int64_t n_dense_tiles;      // n_groups * ceil(n_dense_rows / kDenseBlockRows)
+  int64_t dense_row0;         // dense outputs cover raw rows [dense_row0, dense_row0 + n_dense_rows)
+  int64_t n_dense_rows;       // (a sharded plan's batch shard; else 0 and n_rows)
+  int32_t chain;              // 1: offsets/value positions start at offsets[0] (rap_output RAP_OUT_CHAIN)
+  int32_t pad_chain;
   // sched[0] = CTAs done, sched[1] = launch epoch; the last CTA resets the
   // counter and advances the epoch, so launch parameters are identical from
   // call to call (CUDA-graph replayable).
@@ -213,6 +217,9 @@ RAP_HD uint64_t splitmix_H(uint64_t x) {
 int launch_fused(const Common& c, const LaunchRaw& raw, int grid, int smem_bytes, void* stream);
 // Dynamic shared memory per CTA for dense groups up to max_width columns.
 int fused_smem_bytes(int max_width);
+// rap_jagged_append's kernel (rap_kernel.cu).
+int launch_jagged_append(const int32_t* len, const int64_t* so, const int64_t* val, int64_t n, int64_t vb, int32_t* dl,
+                         int64_t* dof, int64_t* dv, int64_t cap, void* stream);
 // Occupancy query: CTAs per SM for the given dynamic smem.
 int fused_occupancy(int smem_bytes, int n_dense, int n_sparse, int* ctas_per_sm);
 

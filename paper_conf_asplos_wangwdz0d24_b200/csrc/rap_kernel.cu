@@ -31,6 +31,8 @@
 
 namespace rapk {
 
+__host__ __device__ constexpr int align_up_c(int x, int a) { return (x + a - 1) / a * a; }
+
 template <int MD, int MS>
 struct KParams {
   Common c;
@@ -47,7 +49,23 @@ constexpr int kWarps = kThreads / 32;
 #endif
 constexpr int kLBatch = RAP_LBATCH;  // tiles per batch of the length pass
 constexpr int kGroups = kTileRows / 32;  // row groups of a sparse tile (one row per lane each)
-constexpr int kNgScratch = kWarps * 4 * kMaxNgramK * 32 * 4;  // NGram warp scratch (smem, sparse phase)
+// Warp-private shared memory of the sparse phases: the NGram
+// paths use its first 4 KB; the canonical paths stage Arrow offsets,
+// validity words and ids in it with cp.async (nothing in flight in registers).
+constexpr int kWarpScr = 7168;
+constexpr int kNgScratch = kWarps * kWarpScr;
+static_assert(4 * kMaxNgramK * 32 * 4 <= kWarpScr, "NGram scratch exceeds the warp region");
+constexpr int kLChunkTiles = 8;  // length pass: tiles staged per round
+constexpr int kVChunkTiles = 4;  // value pass: tiles staged per round
+#ifndef RAP_VGROUP
+#define RAP_VGROUP 1
+#endif
+constexpr int kVGroup = RAP_VGROUP;  // value pass: tiles whose elements run the pipeline together
+constexpr int kLStageOff = 0, kLStageBm = align_up_c((kLChunkTiles * 128 + 4) * 4, 16);
+constexpr int kVStageOff = 0, kVStageBm = align_up_c((kVChunkTiles * 128 + 4) * 4, 16);
+constexpr int kVStageId = kVStageBm + kVChunkTiles * 128 / 32 * 4;
+static_assert(kLStageBm + kLChunkTiles * 4 * 4 <= kWarpScr, "length-pass staging exceeds the warp region");
+static_assert(kVStageId + kVChunkTiles * 128 * 8 <= kWarpScr && kVStageId % 16 == 0, "value-pass staging layout");
 // Aggregate word of a CTA: [63:44] tag = launch epoch + 1 (0 = never
 // written), [43:0] the CTA's output length total.
 constexpr int kEpochShift = 44;
@@ -130,6 +148,18 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
 }
 
 __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+
+// cp.async (LDGSTS): global -> shared without a register round trip.
+__device__ __forceinline__ void cp_async4(void* dst, const void* src) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async8(void* dst, const void* src) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async16(void* dst, const void* src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
 
 __device__ __forceinline__ unsigned long long ld_relaxed(const unsigned long long* p) {
   unsigned long long v;
@@ -523,6 +553,7 @@ __device__ __forceinline__ void load_ctx(const P& p, int f, FeatCtx& x) {
   } else {
     x.kind = TK_GENERIC;
   }
+  __syncwarp();
 }
 
 // Arrow offsets of rows r0+4*lane .. +4 and the validity word of those rows.
@@ -566,6 +597,34 @@ __device__ __forceinline__ bool quad_valid(const Quad& q, int k, int lane) {
   return (q.w >> ((4 * lane + k) & 31)) & 1u;
 }
 
+// Stage the Arrow offsets off[R0 .. R0+NR] and the validity words of rows
+// [R0, R0+NR) (R0 a multiple of 32) into warp shared memory with cp.async;
+// the caller waits (cp_async_wait_all) and __syncwarp()s before reading.
+__device__ __forceinline__ void stage_offsets(const int32_t* off, const uint32_t* bm, int64_t R0, int NR, int32_t* soff,
+                                              uint32_t* sbm, int lane) {
+  const int ne = NR + 1;
+  int done = 0;
+  if ((reinterpret_cast<uintptr_t>(off + R0) & 15) == 0) {
+    const int n16 = ne >> 2;
+    for (int i = lane; i < n16; i += 32) cp_async16(soff + 4 * i, off + R0 + 4 * i);
+    done = n16 * 4;
+  }
+  for (int i = done + lane; i < ne; i += 32) cp_async4(soff + i, off + R0 + i);
+  const int nw = (NR + 31) >> 5;
+  if (bm != nullptr) {
+    for (int i = lane; i < nw; i += 32) cp_async4(sbm + i, bm + (R0 >> 5) + i);
+  } else {
+    for (int i = lane; i < nw; i += 32) sbm[i] = 0xffffffffu;
+  }
+}
+
+// Output length of staged local row lr (R5 FirstX cap, R10 fill, R14 null).
+__device__ __forceinline__ int32_t len_s(const int32_t* soff, const uint32_t* sbm, int lr, int64_t xcap, int has_fill,
+                                         int64_t null_xcap) {
+  if ((sbm[lr >> 5] >> (lr & 31)) & 1u) return (int32_t)min((int64_t)max(soff[lr + 1] - soff[lr], 0), xcap);
+  return has_fill ? (int32_t)min((int64_t)1, null_xcap) : 0;
+}
+
 // ----------------------------------------------------------------------------
 // Phase 3: offsets and ids of sparse tile (f, rt), whose first output id goes
 // to values[base].
@@ -596,7 +655,7 @@ __device__ __forceinline__ void store_quad(int32_t* lp, int64_t* op, int64_t row
 // Tile of a canonical SRC_SPARSE chain; the lane owns rows r0 + 4*lane + k,
 // so its output ids are contiguous.
 template <class P>
-__device__ __forceinline__ long long value_tile_canon(const P& p, const FeatCtx& fc, int64_t rt, int lane,
+__device__ __noinline__ long long value_tile_canon(const P& p, const FeatCtx& fc, int64_t rt, int lane,
                                                       long long base) {
   const Canon& q = fc.q;
   const int f = fc.f;
@@ -608,9 +667,7 @@ __device__ __forceinline__ long long value_tile_canon(const P& p, const FeatCtx&
   const int64_t* itab = p.c.itab;
   const int32_t* off = p.off[fc.src];
   const int64_t* val = p.val[fc.src];
-  trace_clk(p.c, 8, 0);
   const Quad qd = load_quad(off, p.svalid[fc.src], r0, lane, B, (reinterpret_cast<uintptr_t>(off) & 15) == 0);
-  trace_clk(p.c, 9, qd.a[0] + qd.a[4] + qd.w);
   int32_t l[4], e[4];
   int tot = 0;
 #pragma unroll
@@ -635,9 +692,7 @@ __device__ __forceinline__ long long value_tile_canon(const P& p, const FeatCtx&
       full |= (quad_valid(qd, k, lane) ? 1u : 0u) << k;
       v[k] = (l[k] == 1 && quad_valid(qd, k, lane)) ? __ldg(val + qd.a[k]) : fc.fill;
     }
-    trace_clk(p.c, 10, v[0] + v[1] + v[2] + v[3]);
     canon_apply_n<4>(q, itab, v, act, full);
-    trace_clk(p.c, 11, v[0] + v[1] + v[2] + v[3]);
     const long long lb = base + L;
     store_quad(lp, op, row, B, l, lb, e);
 #pragma unroll
@@ -645,7 +700,6 @@ __device__ __forceinline__ long long value_tile_canon(const P& p, const FeatCtx&
       const long long pos = lb + e[k];
       if (l[k] == 1 && pos < cap) values[pos] = v[k];
     }
-    trace_clk(p.c, 12, 0);
     if (last && lane == 31) {
       p.c.offsets[(int64_t)p.c.n_sparse_out * B] = base + T;  // total, R17
       if (base + T > cap) atomicExch(p.c.err, 1);
@@ -695,6 +749,112 @@ __device__ __forceinline__ long long value_tile_canon(const P& p, const FeatCtx&
     }
   }
   return T;
+}
+
+// Up to kVChunkTiles consecutive tiles rt0 .. rt0+nt-1 of a canonical chain:
+// the offsets / validity words, then the ids of the chunk are staged in warp
+// shared memory with cp.async (no loads in flight in registers), then the
+// canonical pipeline runs 8 elements per lane at a time (MapId probes and
+// Bucketize steps of 8 rows in flight together).  Eligible when every row
+// has at most one output id; returns the chunk's output length total, or -1
+// with nothing written otherwise.
+template <class P>
+__device__ __noinline__ long long value_chunk_canon(const P& p, const FeatCtx& fc, int64_t rt0, int nt, int lane,
+                                                    long long base, unsigned char* wscr) {
+  int32_t* soff = reinterpret_cast<int32_t*>(wscr + kVStageOff);
+  uint32_t* sbm = reinterpret_cast<uint32_t*>(wscr + kVStageBm);
+  int64_t* sid = reinterpret_cast<int64_t*>(wscr + kVStageId);
+  const int f = fc.f;
+  const int64_t B = p.c.n_rows;
+  const int64_t R0 = rt0 * kTileRows;
+  const int NR = (int)min((int64_t)nt * kTileRows, B - R0);
+  const int src = fc.src;
+  const int64_t xcap = fc.xcap, null_xcap = fc.null_xcap;
+  const int has_fill = fc.has_fill;
+  trace_clk(p.c, 8, 0);
+  stage_offsets(p.off[src], p.svalid[src], R0, NR, soff, sbm, lane);
+  cp_async_wait_all();
+  __syncwarp();
+  trace_clk(p.c, 9, soff[0]);
+  // quad layout: the lane owns local rows j*128 + 4*lane + k
+  unsigned act = 0, full = 0;
+  bool ok = true;
+#pragma unroll
+  for (int j = 0; j < kVChunkTiles; ++j)
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      const int lr = j * kTileRows + 4 * lane + k;
+      if (lr < NR) {
+        const int32_t l = len_s(soff, sbm, lr, xcap, has_fill, null_xcap);
+        ok &= l <= 1;
+        act |= (l == 1 ? 1u : 0u) << (4 * j + k);
+        full |= (((sbm[lr >> 5] >> (lr & 31)) & 1u) ? 1u : 0u) << (4 * j + k);
+      }
+    }
+  if (!__all_sync(0xffffffffu, ok)) {
+    __syncwarp();
+    return -1;
+  }
+  const int64_t* val = p.val[src];
+  const unsigned fetch = act & full;
+#pragma unroll
+  for (int j = 0; j < kVChunkTiles; ++j)
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      const int lr = j * kTileRows + 4 * lane + k;
+      if ((fetch >> (4 * j + k)) & 1u) cp_async8(sid + lr, val + soff[lr]);
+    }
+  cp_async_wait_all();  // each lane reads only the ids it staged
+  trace_clk(p.c, 10, sid[4 * lane]);
+  int64_t* values = p.c.values;
+  const long long cap = p.c.values_cap;
+  long long run = base;
+#pragma unroll 1
+  for (int j0 = 0; j0 < nt; j0 += kVGroup) {
+    int64_t v[4 * kVGroup];
+    const unsigned gm = (1u << (4 * kVGroup)) - 1u;
+    const unsigned ag = (act >> (4 * j0)) & gm, fg = (full >> (4 * j0)) & gm;
+#pragma unroll
+    for (int u = 0; u < 4 * kVGroup; ++u) {
+      const int lr = (j0 + (u >> 2)) * kTileRows + 4 * lane + (u & 3);
+      v[u] = ((ag & fg) >> u) & 1u ? sid[lr] : fc.fill;
+    }
+    canon_apply_n<4 * kVGroup>(fc.q, p.c.itab, v, ag, fg);
+    trace_clk(p.c, 11, v[0]);
+#pragma unroll
+    for (int jj = 0; jj < kVGroup; ++jj) {
+      const int j = j0 + jj;
+      if (j < nt) {
+        const int64_t rt = rt0 + j;
+        const int64_t row = rt * kTileRows + 4 * lane;
+        const unsigned a4 = (ag >> (4 * jj)) & 15u;
+        int32_t l[4], e[4];
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          l[k] = (a4 >> k) & 1u;
+          e[k] = __popc(a4 & ((1u << k) - 1u));
+        }
+        const int tot = __popc(a4);
+        const int incl = warp_incl_scan(tot, lane);
+        const int Tj = __shfl_sync(0xffffffffu, incl, 31);
+        const long long lb = run + (incl - tot);
+        store_quad(p.c.lengths + (int64_t)f * B + row, p.c.offsets + (int64_t)f * B + row, row, B, l, lb, e);
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          const long long pos = lb + e[k];
+          if (l[k] && pos < cap) values[pos] = v[4 * jj + k];
+        }
+        if (f == p.c.n_sparse_out - 1 && rt == p.c.tiles_per_feature - 1 && lane == 31) {
+          p.c.offsets[(int64_t)p.c.n_sparse_out * B] = run + Tj;  // total, R17
+          if (run + Tj > cap) atomicExch(p.c.err, 1);
+        }
+        run += Tj;
+      }
+    }
+  }
+  trace_clk(p.c, 12, run);
+  __syncwarp();  // the region is reused by the next chunk
+  return run - base;
 }
 
 // Tile of any other SRC_SPARSE / SRC_DENSE_BUCKET chain (op interpreter).
@@ -841,7 +1001,7 @@ __device__ __noinline__ void value_group_general(const P& p, int f, int64_t row0
 // (nt = 1 or 2) of a feature with k <= 4 sparse sources: all 2k quads in
 // flight together.
 template <class P>
-__device__ __forceinline__ long long ngram_tiles_len2(const P& p, const SProg& pg, int64_t r0, int nt, int lane) {
+__device__ __noinline__ long long ngram_tiles_len2(const P& p, const SProg& pg, int64_t r0, int nt, int lane) {
   const int64_t B = p.c.n_rows;
   const int k = pg.ng.k, n = pg.ng.n;
   const int64_t xo = pg.ch.xcap;
@@ -969,7 +1129,7 @@ __device__ __forceinline__ void ngram_stage(const P& p, int f, int32_t* scr, int
 // the tile's output length total, or -1 with nothing written when the tile
 // is not eligible.
 template <class P>
-__device__ __forceinline__ long long ngram_tile_fast(const P& p, int f, int64_t rt, int lane, long long base,
+__device__ __noinline__ long long ngram_tile_fast(const P& p, int f, int64_t rt, int lane, long long base,
                                                  int32_t* scr) {
   trace_clk(p.c, 13, 0);
   // parameters: staged in warp-private shared memory by ngram_stage (no lazy
@@ -1247,24 +1407,27 @@ __device__ __noinline__ void onehot_generic(const P& p, const DUnit& un, int64_t
 }
 
 template <class P>
-__device__ void dense_block(const P& p, int gi, int64_t rb, unsigned char* smem, CtaState& cs) {
+__device__ __noinline__ void dense_block(const P& p, int gi, int64_t rb, unsigned char* smem, CtaState& cs) {
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   DProg* dp = reinterpret_cast<DProg*>(smem);
   float* din = reinterpret_cast<float*>(smem + kDProgBytes);  // [16][kDenseBlockRows]
   uint32_t* dbm = reinterpret_cast<uint32_t*>(smem + kDProgBytes + 16 * kDenseBlockRows * 4);  // [16][8]
   float* tile = reinterpret_cast<float*>(smem + kDProgBytes + dense_in_bytes());
-  const int64_t B = p.c.n_rows;
+  // rows [r0, r0 + nr) of the dense output = raw rows g0 + [0, nr): a
+  // sharded plan's dense outputs cover its batch shard only
   const int64_t r0 = rb * kDenseBlockRows;
-  const int nr = (int)min((int64_t)kDenseBlockRows, B - r0);
+  const int64_t g0 = p.c.dense_row0 + r0;
+  const int nr = (int)min((int64_t)kDenseBlockRows, p.c.n_dense_rows - r0);
   const int nw = (nr + 31) >> 5;
   trace_clk(p.c, 16, 0);
   if (warp == 0) {
     const DProg* g = p.c.dprogs + gi;
     const int nu = __ldg(&g->n_units), no = __ldg(&g->n_ops), nf = __ldg(&g->n_ftab), nc = __ldg(&g->n_cols);
     const int col = lane < nc ? __ldg(&g->cols[lane]) : 0;
-    const bool aligned = lane >= nc || ((reinterpret_cast<uintptr_t>(p.dense[col] + r0) & 15) == 0 &&
+    const bool aligned = lane >= nc || ((reinterpret_cast<uintptr_t>(p.dense[col] + g0) & 15) == 0 &&
                                         (p.dvalid[col] == nullptr ||
-                                         (reinterpret_cast<uintptr_t>(p.dvalid[col] + (r0 >> 5)) & 15) == 0));
+                                         ((g0 & 31) == 0 &&
+                                          (reinterpret_cast<uintptr_t>(p.dvalid[col] + (g0 >> 5)) & 15) == 0)));
     const bool stage = __all_sync(0xffffffffu, aligned) && (nr & 3) == 0 && nc <= 16;
     if (stage) {
       const uint32_t bytes_v = (uint32_t)nr * 4, bytes_b = (uint32_t)align_up(nw * 4, 16);
@@ -1278,8 +1441,8 @@ __device__ void dense_block(const P& p, int gi, int64_t rb, unsigned char* smem,
       }
       __syncwarp();
       if (lane < nc) {
-        bulk_g2s(din + lane * kDenseBlockRows, p.dense[col] + r0, bytes_v, &cs.bar);
-        if (p.dvalid[col]) bulk_g2s(dbm + lane * 8, p.dvalid[col] + (r0 >> 5), bytes_b, &cs.bar);
+        bulk_g2s(din + lane * kDenseBlockRows, p.dense[col] + g0, bytes_v, &cs.bar);
+        if (p.dvalid[col]) bulk_g2s(dbm + lane * 8, p.dvalid[col] + (g0 >> 5), bytes_b, &cs.bar);
       }
     }
     if (lane == 0) cs.staged = stage ? 1 : 0;
@@ -1303,39 +1466,83 @@ __device__ void dense_block(const P& p, int gi, int64_t rb, unsigned char* smem,
   trace_clk(p.c, 17, 0);
   const int W = dp->width;
   const int LD = W | 1;  // odd row pitch: conflict-free column writes
-  if (dp->any_onehot)
-    for (int i = tid; i < nr * LD; i += kThreads) tile[i] = 0.0f;
+  if (dp->any_onehot) {
+    const int n = nr * LD;  // the tile base is 16-byte aligned
+    float4* t4 = reinterpret_cast<float4*>(tile);
+    for (int i = tid; i < (n >> 2); i += kThreads) t4[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+    for (int i = (n & ~3) + tid; i < n; i += kThreads) tile[i] = 0.0f;
+  }
   const bool staged = cs.staged;
   if (staged) mbar_wait(&cs.bar, cs.phase);
   __syncthreads();
   trace_clk(p.c, 18, 0);
   const int nu = dp->n_units;
-  // (row, unit) pairs over all threads, unit-major so a warp shares its unit
-  for (int idx = tid; idx < nr * nu; idx += kThreads) {
-    const int u = idx / nr, r = idx - u * nr;
-    const int64_t row = r0 + r;
+  // one unit per warp at a time, its rows over the lanes: the unit's
+  // descriptor and up to kRegOps dense ops are read once into registers
+  // (warp-uniform), then each row is a short straight-line chain
+  constexpr int kRegOps = 3;
+  for (int u = warp; u < nu; u += kWarps) {
     const DUnit& un = dp->units[u];
-    const DevOp* uops = un.gops ? p.c.ops : dp->ops;
-    if (un.kind == U_ONEHOT_G) {  // generic list (R9), program from global memory
-      onehot_generic(p, un, row, tile + r * LD);
+    const int kind = un.kind, col = un.col, slot = un.slot, src_col = un.src_col;
+    if (kind == U_ONEHOT_G) {  // generic list (R9), program from global memory
+      for (int r = lane; r < nr; r += 32) onehot_generic(p, un, g0 + r, tile + r * LD);
       continue;
     }
-    float x;
-    if (staged) {
-      const uint32_t w = p.dvalid[un.src_col] ? dbm[un.slot * 8 + (r >> 5)] : 0xffffffffu;
-      x = ((w >> (r & 31)) & 1u) ? din[un.slot * kDenseBlockRows + r] : __int_as_float(0x7fc00000);
-    } else {
-      x = dense_raw(p, un.src_col, row);
+    const DevOp* uops = un.gops ? p.c.ops : dp->ops;
+    const int o0 = un.op_begin, o1 = un.op_end;
+    const bool reg_ops = o1 - o0 <= kRegOps;
+    int okind[kRegOps];
+    float of0[kRegOps], of1[kRegOps];
+#pragma unroll
+    for (int k = 0; k < kRegOps; ++k) {
+      okind[k] = -1;
+      of0[k] = of1[k] = 0.0f;
+      if (reg_ops && o0 + k < o1) {
+        okind[k] = uops[o0 + k].kind;
+        of0[k] = uops[o0 + k].f0;
+        of1[k] = uops[o0 + k].f1;
+      }
     }
-    x = apply_dense_ops(uops, x, un.op_begin, un.op_end);
-    if (un.kind == U_DENSE) {
-      tile[r * LD + un.col] = x;
-    } else if (un.xcap > 0) {  // U_ONEHOT_DB
-      const float* uft = un.gops ? p.c.ftab : dp->ftab;
-      const int64_t bidx = un.gops ? upper_bound(uft + un.btab, un.bm, x) : upper_bound_s(uft + un.btab, un.bm, x);
-      const int64_t id = apply_id_ops(uops, p.c.itab, 0, bidx, un.iop_begin, un.iop_end);
-      const int64_t d = id - un.k0;
-      if (d >= 0 && d < un.width) tile[r * LD + un.col + (int)d] = 1.0f;
+    const bool has_bm = p.dvalid[src_col] != nullptr;
+    const float* uft = un.gops ? p.c.ftab : dp->ftab;
+    for (int r = lane; r < nr; r += 32) {
+      float x;
+      if (staged) {
+        const uint32_t w = has_bm ? dbm[slot * 8 + (r >> 5)] : 0xffffffffu;
+        x = ((w >> (r & 31)) & 1u) ? din[slot * kDenseBlockRows + r] : __int_as_float(0x7fc00000);
+      } else {
+        x = dense_raw(p, src_col, g0 + r);
+      }
+      if (reg_ops) {
+#pragma unroll
+        for (int k = 0; k < kRegOps; ++k) {  // R10-R12, same expressions as apply_dense_ops
+          const int ok = okind[k];
+          if (ok == OK_FILL_F) {
+            if (isnan(x)) x = of0[k];
+          } else if (ok == OK_LOGIT) {
+            const float z = x < of0[k] ? of0[k] : (x > of1[k] ? of1[k] : x);
+            x = logf(__fdiv_rn(z, __fsub_rn(1.0f, z)));
+          } else if (ok == OK_BOXCOX) {
+            const float lam = of0[k];
+            if (lam == 0.0f) {
+              x = logf(x);
+            } else {
+              const float v = __fmul_rn(lam, logf(x));
+              x = __fdiv_rn(expm1f(v), lam);
+            }
+          }
+        }
+      } else {
+        x = apply_dense_ops(uops, x, o0, o1);
+      }
+      if (kind == U_DENSE) {
+        tile[r * LD + col] = x;
+      } else if (un.xcap > 0) {  // U_ONEHOT_DB
+        const int64_t bidx = un.gops ? upper_bound(uft + un.btab, un.bm, x) : upper_bound_s(uft + un.btab, un.bm, x);
+        const int64_t id = apply_id_ops(uops, p.c.itab, 0, bidx, un.iop_begin, un.iop_end);
+        const int64_t d = id - un.k0;
+        if (d >= 0 && d < un.width) tile[r * LD + col + (int)d] = 1.0f;
+      }
     }
   }
   __syncthreads();
@@ -1393,12 +1600,18 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
   __shared__ long long s_slots[kWarps];
   __shared__ long long s_red[kWarps];
   __shared__ int s_last;
+  __shared__ FeatCtx s_fc[kWarps];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   // The epoch load is consumed only when the aggregate is published, so its
   // latency hides under the length pass.  Ranks are block indices: the
   // launch is cooperative, so every CTA is resident and a CTA waits only on
   // resident predecessors.
   const unsigned long long epoch = ld_relaxed(p.c.sched + 1);
+  // chained launch (rap_output.flags & RAP_OUT_CHAIN): offsets[0] already
+  // holds the running total of the launch before this one into the same
+  // buffer; every offset and value position of this launch starts there (the
+  // first tile rewrites offsets[0] with the same value)
+  const long long chain0 = p.c.chain ? (long long)__ldg(p.c.offsets) : 0ll;
   if (tid == 0) {
     mbar_init(&cs.bar, 1);
     cs.phase = 0;
@@ -1414,7 +1627,8 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
   }
   const int64_t S = p.c.n_sparse_tiles, T = p.c.tiles_per_feature;
   const int64_t s0 = __ldg(p.c.part + rank), s1 = __ldg(p.c.part + rank + 1);  // my sparse tiles
-  int32_t* scr = reinterpret_cast<int32_t*>(smem) + warp * (4 * kMaxNgramK * 32);
+  unsigned char* wscr = smem + warp * kWarpScr;  // warp-private region (sparse phases)
+  int32_t* scr = reinterpret_cast<int32_t*>(wscr);
   if (p.c.trace != nullptr && tid == 0 && (int64_t)blockIdx.x < p.c.trace_cap)
     p.c.trace[(int64_t)blockIdx.x * kTracePts + 5] = (unsigned long long)(s0 | ((s1 - s0) << 32));
 
@@ -1423,33 +1637,36 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
   const int64_t w0 = s0 + ns * warp / kWarps, w1 = s0 + ns * (warp + 1) / kWarps;
   long long mine = 0, part = 0;  // warp-uniform / per-lane partial totals
   trace_clk(p.c, 21, 0);
+  // per-feature dispatch state in warp-private shared memory (not registers:
+  // it is live across the whole tile loop)
+  FeatCtx& fc = s_fc[warp];
+  if (lane == 0) fc.f = -1;
+  __syncwarp();
   {
-    FeatCtx fc;
-    fc.f = -1;
     const int64_t B = p.c.n_rows;
     for (int64_t t = w0; t < w1;) {
       const int f = (int)((uint64_t)t / (uint64_t)T);
       if (f != fc.f) load_ctx(p, f, fc);
       const int64_t tend = min(w1, (int64_t)(f + 1) * T);
       if (fc.sk == SRC_SPARSE) {
-        // kLBatch tiles' offsets in flight at a time
+        // kLChunkTiles tiles' offsets and validity words staged per round
         const int32_t* off = p.off[fc.src];
         const uint32_t* bm = p.svalid[fc.src];
-        const bool al = (reinterpret_cast<uintptr_t>(off) & 15) == 0;
-        for (; t < tend; t += kLBatch) {
-          Quad q[kLBatch];
-#pragma unroll
-          for (int j = 0; j < kLBatch; ++j)
-            if (t + j < tend) q[j] = load_quad(off, bm, (t + j - (int64_t)f * T) * kTileRows, lane, B, al);
-#pragma unroll
-          for (int j = 0; j < kLBatch; ++j)
-            if (t + j < tend) {
-              const int64_t row = (t + j - (int64_t)f * T) * kTileRows + 4 * lane;
-#pragma unroll
-              for (int k = 0; k < 4; ++k) part += quad_len(q[j], k, lane, row + k, B, fc.xcap, fc.has_fill, fc.null_xcap);
-            }
+        int32_t* soff = reinterpret_cast<int32_t*>(wscr + kLStageOff);
+        uint32_t* sbm = reinterpret_cast<uint32_t*>(wscr + kLStageBm);
+        const int64_t xcap = fc.xcap, null_xcap = fc.null_xcap;
+        const int has_fill = fc.has_fill;
+        while (t < tend) {
+          const int nt = (int)min((int64_t)kLChunkTiles, tend - t);
+          const int64_t R0 = (t - (int64_t)f * T) * kTileRows;
+          const int NR = (int)min((int64_t)nt * kTileRows, B - R0);
+          stage_offsets(off, bm, R0, NR, soff, sbm, lane);
+          cp_async_wait_all();
+          __syncwarp();
+          for (int lr = lane; lr < NR; lr += 32) part += len_s(soff, sbm, lr, xcap, has_fill, null_xcap);
+          __syncwarp();
+          t += nt;
         }
-        t = tend;
       } else if (fc.kind == TK_NGRAM_FAST) {
         const SProg& pg = p.c.sprogs[f];
         while (t < tend) {
@@ -1512,21 +1729,31 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
         for (int u = 0; u < 8; ++u) pre += (long long)(w[u] & kValueMask);
       }
     }
-    const long long base = block_sum(pre, s_red);
+    const long long base = block_sum(pre, s_red) + chain0;
     trace_stamp(p.c, 3);
 
     // (V) offsets and ids of my warp's tiles, in scan order
-    FeatCtx fc;
-    fc.f = -1;
+    if (lane == 0) fc.f = -1;
+    __syncwarp();
     long long run = base;
     for (int j = 0; j < warp; ++j) run += s_slots[j];
 #ifdef RAP_DBG_SKIP_V
     if (false)
 #endif
-    for (int64_t t = w0; t < w1; ++t) {
+    for (int64_t t = w0; t < w1;) {
       const int f = (int)((uint64_t)t / (uint64_t)T);
       if (f != fc.f) load_ctx(p, f, fc);
+      if (fc.kind == TK_CANON) {
+        const int nt = (int)min((int64_t)kVChunkTiles, min(w1, (int64_t)(f + 1) * T) - t);
+        const long long got = value_chunk_canon(p, fc, t - (int64_t)f * T, nt, lane, run, wscr);
+        if (got >= 0) {
+          run += got;
+          t += nt;
+          continue;
+        }
+      }
       run += value_tile(p, fc, t - (int64_t)f * T, lane, run, scr);
+      ++t;
     }
   }
   trace_stamp(p.c, 4);
@@ -1618,6 +1845,41 @@ int fused_occupancy(int smem_bytes, int n_dense, int n_sparse, int* ctas_per_sm)
                                                         smem_bytes);
   }
   return (int)e;
+}
+
+}  // namespace rapk
+
+// ----------------------------------------------------------------------------
+// rap_jagged_append (include/rap.h): a received residual piece continues a
+// chained jagged output.  Grid-stride copy; the running total
+// T = dst_offsets[0] is a device value (written by the preceding launch).
+namespace rapk {
+
+__global__ void __launch_bounds__(256) jagged_append_kernel(const int32_t* __restrict__ len,
+                                                            const int64_t* __restrict__ so,
+                                                            const int64_t* __restrict__ val, int64_t n,
+                                                            int32_t* __restrict__ dl, int64_t* dof,
+                                                            int64_t* __restrict__ dv, int64_t cap) {
+  const long long T = *reinterpret_cast<volatile const long long*>(dof);
+  const int64_t s0 = so[0];
+  const int64_t nv = so[n] - s0;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < max(n, nv); i += stride) {
+    if (i < n) {
+      dl[i] = len[i];
+      dof[i + 1] = T + (so[i + 1] - s0);
+    }
+    if (i < nv && T + i < cap) dv[T + i] = val[s0 + i];
+  }
+}
+
+int launch_jagged_append(const int32_t* len, const int64_t* so, const int64_t* val, int64_t n, int64_t vb, int32_t* dl,
+                         int64_t* dof, int64_t* dv, int64_t cap, void* stream) {
+  const int64_t work = max(n, vb);
+  const int64_t blocks = min((work + 255) / 256, (int64_t)148 * 8);
+  jagged_append_kernel<<<(unsigned)max(blocks, (int64_t)1), 256, 0, reinterpret_cast<cudaStream_t>(stream)>>>(
+      len, so, val, n, dl, dof, dv, cap);
+  return (int)cudaGetLastError();
 }
 
 }  // namespace rapk

@@ -68,6 +68,7 @@ int64_t sat_mul(int64_t a, int64_t b) {
 struct rap_plan {
   int device = 0, sm_count = 0, budget = 0, ctas_per_sm = 1, smem = 0;
   int n_dense_in = 0, n_sparse_in = 0;
+  int rank = 0, world = 1;  // sharded plan: dense outputs cover rap_shard_rows(rank, world)
   // lowered program (host copies)
   std::vector<DevOp> ops;
   std::vector<DenseExpr> dexprs;
@@ -1093,6 +1094,7 @@ static double dense_row_cost(const rap_plan* P, const DProg& dp) {
 static rap_status update_partition(rap_plan* P, int64_t B, const int64_t* nnz, int64_t S, int64_t D, int grid,
                                    cudaStream_t stream) {
   std::vector<int64_t> key = {B, grid};
+  (void)D;
   for (int s : P->used_sparse) {
     const double m = nnz && B > 0 ? (double)std::max<int64_t>(nnz[s], 0) / (double)B : 0.0;
     key.push_back(m <= 1.0 / 64 ? -1000 : (int64_t)std::lround(4.0 * std::log2(m)));
@@ -1103,15 +1105,18 @@ static rap_status update_partition(rap_plan* P, int64_t B, const int64_t* nnz, i
   const double kTileFixed = 400.0;  // per-unit overhead (lane-instructions)
   std::vector<double> fcost(F);
   for (int64_t f = 0; f < F; ++f) fcost[f] = sparse_row_cost(P, P->chains[P->souts[f].chain], B, nnz);
-  (void)D;
   auto unit_cost = [&](int64_t u) -> double {
     const int64_t f = u / T, rt = u - f * T;
     const int64_t rows = std::min<int64_t>(kTileRows, B - rt * kTileRows);
     return kTileFixed + (double)rows * fcost[f];
   };
-  const int64_t U = S;  // dense blocks go round robin over the ranks
+  const int64_t U = S;
   double W = 0;
   for (int64_t u = 0; u < U; ++u) W += unit_cost(u);
+  // dense blocks go round robin over the ranks (block d to rank d mod
+  // grid).  The sparse ranges ignore them: the CTAs of an SM share its issue
+  // slots, so a CTA's dense block mostly fills slots its SM neighbours leave
+  // idle (measured: charging it to the CTA's sparse share made C2 slower).
   std::vector<int64_t> part(grid + 1);
   part[0] = 0;
   double acc = 0;
@@ -1132,7 +1137,7 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
   const int64_t B = raw->n_rows;
   cudaError_t e;
   if (B == 0) {
-    if (!P->souts.empty()) {
+    if (!P->souts.empty() && !(out->flags & RAP_OUT_CHAIN)) {
       e = cudaMemsetAsync(out->offsets, 0, sizeof(int64_t), stream);
       if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync");
     }
@@ -1144,7 +1149,9 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
   const int64_t F = (int64_t)P->souts.size();
   const int64_t T = (B + kTileRows - 1) / kTileRows;
   const int64_t n_sparse_tiles = F * T;
-  const int64_t n_dense = P->dprogs.empty() ? 0 : (int64_t)P->dprogs.size() * ((B + kDenseBlockRows - 1) / kDenseBlockRows);
+  int64_t drow0 = 0, drows = B;
+  rap_shard_rows(B, P->rank, P->world, &drow0, &drows);
+  const int64_t n_dense = P->dprogs.empty() ? 0 : (int64_t)P->dprogs.size() * ((drows + kDenseBlockRows - 1) / kDenseBlockRows);
   if (n_sparse_tiles == 0 && n_dense == 0) return RAP_OK;
   const int64_t grid = std::min<int64_t>((int64_t)P->budget * P->ctas_per_sm, kMaxCtas);
   rap_status pst = update_partition(P, B, raw->sp_nnz, n_sparse_tiles, n_dense, (int)grid, stream);
@@ -1162,6 +1169,9 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
   c.tiles_per_feature = T;
   c.n_sparse_tiles = n_sparse_tiles;
   c.n_dense_tiles = n_dense;
+  c.dense_row0 = drow0;
+  c.n_dense_rows = drows;
+  c.chain = (out->flags & RAP_OUT_CHAIN) ? 1 : 0;
   c.sched = P->d_sched;
   c.part = P->d_part;
   c.agg = P->d_agg;
@@ -1263,8 +1273,10 @@ rap_status rap_preprocess_host(rap_plan* P, const rap_raw_batch* raw, const rap_
   }
   const int64_t F = (int64_t)P->souts.size();
   const int64_t vb = B > 0 ? values_bound(P, B, raw->sp_nnz) : 0;
+  int64_t drow0 = 0, drows = B;
+  rap_shard_rows(B, P->rank, P->world, &drow0, &drows);
   void *dd = nullptr, *dl = nullptr, *dof = nullptr, *dv = nullptr;
-  if ((st = stage_buf(P, slot++, sizeof(float) * std::max<int64_t>(B * P->d_out, 1), &dd)) != RAP_OK) return st;
+  if ((st = stage_buf(P, slot++, sizeof(float) * std::max<int64_t>(drows * P->d_out, 1), &dd)) != RAP_OK) return st;
   if ((st = stage_buf(P, slot++, sizeof(int32_t) * std::max<int64_t>(B * F, 1), &dl)) != RAP_OK) return st;
   if ((st = stage_buf(P, slot++, sizeof(int64_t) * (B * F + 1), &dof)) != RAP_OK) return st;
   if ((st = stage_buf(P, slot++, sizeof(int64_t) * std::max<int64_t>(vb, 1), &dv)) != RAP_OK) return st;
@@ -1283,12 +1295,12 @@ rap_status rap_preprocess_host(rap_plan* P, const rap_raw_batch* raw, const rap_
   dout.values_capacity = std::max<int64_t>(vb, 0);
   if ((st = launch(P, &dr, &dout, stream)) != RAP_OK) return st;
   // D2H
-  if (B > 0 && P->d_out > 0) {
+  if (drows > 0 && P->d_out > 0) {
     if (out->dense_ld == P->d_out)
-      e = cudaMemcpyAsync(out->dense_out, dd, sizeof(float) * B * P->d_out, cudaMemcpyDeviceToHost, stream);
+      e = cudaMemcpyAsync(out->dense_out, dd, sizeof(float) * drows * P->d_out, cudaMemcpyDeviceToHost, stream);
     else
       e = cudaMemcpy2DAsync(out->dense_out, sizeof(float) * out->dense_ld, dd, sizeof(float) * P->d_out,
-                            sizeof(float) * P->d_out, B, cudaMemcpyDeviceToHost, stream);
+                            sizeof(float) * P->d_out, drows, cudaMemcpyDeviceToHost, stream);
     if (e != cudaSuccess) return cuda_fail(e, "D2H dense");
   }
   if (F > 0) {
@@ -1349,3 +1361,180 @@ rap_status rap_choose_budget(const rap_plan* P, int64_t n_rows, const int64_t* s
 }
 
 }  // extern "C"
+
+// ----------------------------------------------------------------------------
+// Multi-GPU (§7.2, hybrid parallelism
+// L488-499).
+
+rap_status rap_shard_rows(int64_t n_rows, int32_t rank, int32_t world, int64_t* row0, int64_t* rows) {
+  if (!row0 || !rows) return fail(RAP_ERR_INVALID_ARGUMENT, "NULL argument");
+  if (n_rows < 0 || world < 1 || rank < 0 || rank >= world) return fail(RAP_ERR_INVALID_ARGUMENT, "bad shard");
+  if (world == 1) {
+    *row0 = 0;
+    *rows = n_rows;
+    return RAP_OK;
+  }
+  // boundary r = floor(n_rows * r / world) rounded down to 128 rows; the last
+  // rank ends at n_rows
+  auto bound = [&](int32_t r) -> int64_t {
+    if (r >= world) return n_rows;
+    const int64_t b = (int64_t)((__int128)n_rows * r / world);
+    return b / kTileRows * kTileRows;
+  };
+  *row0 = bound(rank);
+  *rows = bound(rank + 1) - *row0;
+  return RAP_OK;
+}
+
+rap_status rap_plan_output_costs(const rap_plan* P, int64_t n_rows, const int64_t* sp_nnz, double* cost) {
+  if (!P || !cost) return fail(RAP_ERR_INVALID_ARGUMENT, "NULL argument");
+  if (n_rows < 0) return fail(RAP_ERR_INVALID_ARGUMENT, "n_rows < 0");
+  for (size_t f = 0; f < P->souts.size(); ++f)
+    cost[f] = (double)n_rows * sparse_row_cost(P, P->chains[P->souts[f].chain], n_rows, sp_nnz);
+  return RAP_OK;
+}
+
+rap_status rap_place(const double* cost, const int32_t* colocate, int32_t n, int32_t world, int32_t mode,
+                     int64_t n_rows, double imbalance_tol, int32_t* owner_out, double* load_out,
+                     rap_residual* residual) {
+  if (n < 0 || world < 1 || n_rows < 0) return fail(RAP_ERR_INVALID_ARGUMENT, "bad size");
+  if (n > 0 && (!cost || !owner_out)) return fail(RAP_ERR_INVALID_ARGUMENT, "NULL argument");
+  if (mode < RAP_PLACE_BALANCED || mode > RAP_PLACE_SKEWED) return fail(RAP_ERR_INVALID_ARGUMENT, "bad mode");
+  // groups: an output with colocate[j] = i joins i's group (transitively)
+  std::vector<int> anchor(n);
+  for (int j = 0; j < n; ++j) {
+    if (!(cost[j] >= 0)) return fail(RAP_ERR_INVALID_ARGUMENT, "cost must be >= 0");
+    const int c = colocate ? colocate[j] : -1;
+    if (c >= j || c < -1) return fail(RAP_ERR_INVALID_ARGUMENT, "colocate[j] must be -1 or < j");
+    anchor[j] = c < 0 ? j : anchor[c];
+  }
+  std::vector<int> groups;  // anchors in index order
+  std::vector<double> gcost(n, 0.0);
+  for (int j = 0; j < n; ++j) {
+    if (anchor[j] == j) groups.push_back(j);
+    gcost[anchor[j]] += cost[j];
+  }
+  std::vector<double> load(world, 0.0);
+  std::vector<int> gowner(n, 0);
+  auto lpt = [&](std::vector<int> gs, int r_lo) {
+    std::stable_sort(gs.begin(), gs.end(), [&](int a, int b) { return gcost[a] > gcost[b]; });
+    for (int g : gs) {
+      int best = r_lo;
+      for (int r = r_lo; r < world; ++r)
+        if (load[r] < load[best]) best = r;
+      gowner[g] = best;
+      load[best] += gcost[g];
+    }
+  };
+  if (mode == RAP_PLACE_ROUND_ROBIN) {
+    for (size_t i = 0; i < groups.size(); ++i) {
+      gowner[groups[i]] = (int)(i % world);
+      load[i % world] += gcost[groups[i]];
+    }
+  } else if (mode == RAP_PLACE_SKEWED && world > 1) {
+    double total = 0;
+    for (int g : groups) total += gcost[g];
+    const double target = 2.0 * total / world;
+    std::vector<int> gs = groups, rest;
+    std::stable_sort(gs.begin(), gs.end(), [&](int a, int b) { return gcost[a] > gcost[b]; });
+    for (int g : gs) {
+      if (load[0] + gcost[g] <= target) {
+        gowner[g] = 0;
+        load[0] += gcost[g];
+      } else {
+        rest.push_back(g);
+      }
+    }
+    lpt(rest, 1);
+  } else {
+    lpt(groups, 0);
+  }
+  for (int j = 0; j < n; ++j) owner_out[j] = gowner[anchor[j]];
+  if (residual) {
+    residual->output = -1;
+    residual->owner = residual->helper = -1;
+    residual->pad = 0;
+    residual->split_row = n_rows;
+    if (world > 1 && n > 0 && n_rows >= 2 * kTileRows) {
+      int h = 0, l = 0;
+      double total = 0;
+      for (int r = 0; r < world; ++r) {
+        total += load[r];
+        if (load[r] > load[h]) h = r;
+        if (load[r] < load[l]) l = r;
+      }
+      const double mean = total / world;
+      if (load[h] > mean * (1.0 + imbalance_tol) && h != l) {
+        int f = -1;
+        for (int j = 0; j < n; ++j)
+          if (owner_out[j] == h && (f < 0 || cost[j] > cost[f])) f = j;
+        const double per_row = f >= 0 ? cost[f] / (double)n_rows : 0.0;
+        if (per_row > 0) {
+          const double delta = 0.5 * (load[h] - load[l]);
+          // split row: a multiple of 128 (whole validity words / tiles on both
+          // sides), the owner keeping at least one tile
+          const int64_t want = std::min((int64_t)(delta / per_row), n_rows);
+          int64_t split = (n_rows - want + kTileRows - 1) / kTileRows * kTileRows;
+          split = std::max<int64_t>(split, kTileRows);
+          const int64_t moved = n_rows - split;
+          if (moved > 0) {
+            residual->output = f;
+            residual->owner = h;
+            residual->helper = l;
+            residual->split_row = split;
+            load[h] -= per_row * (double)moved;
+            load[l] += per_row * (double)moved;
+          }
+        }
+      }
+    }
+  }
+  if (load_out)
+    for (int r = 0; r < world; ++r) load_out[r] = load[r];
+  return RAP_OK;
+}
+
+rap_status rap_plan_create_sharded(const rap_graph* graph, const rap_op_param* params, int32_t n_params, int32_t device,
+                                   int32_t sm_budget, const int32_t* sparse_owner, int32_t rank, int32_t world,
+                                   rap_plan** out) {
+  if (!out) return fail(RAP_ERR_INVALID_ARGUMENT, "out is NULL");
+  *out = nullptr;
+  if (world < 1 || rank < 0 || rank >= world) return fail(RAP_ERR_INVALID_ARGUMENT, "bad rank/world");
+  Validated v;
+  rap_status st = validate(graph, params, n_params, &v);
+  if (st != RAP_OK) return st;
+  std::vector<int32_t> outs;
+  int j = 0;
+  for (int o = 0; o < graph->n_outputs; ++o) {
+    const int node = graph->output_nodes[o];
+    if (v.type[node] == VT_IDS) {
+      if (!sparse_owner) return fail(RAP_ERR_INVALID_ARGUMENT, "sparse_owner is NULL");
+      const int32_t r = sparse_owner[j++];
+      if (r < -1 || r >= world) return fail(RAP_ERR_INVALID_ARGUMENT, "sparse_owner out of range");
+      if (r == rank) outs.push_back(node);
+    } else {
+      outs.push_back(node);
+    }
+  }
+  rap_graph g = *graph;
+  g.n_outputs = (int32_t)outs.size();
+  g.output_nodes = outs.data();
+  st = rap_plan_create(&g, params, n_params, device, sm_budget, out);
+  if (st != RAP_OK) return st;
+  (*out)->rank = rank;
+  (*out)->world = world;
+  return RAP_OK;
+}
+
+rap_status rap_jagged_append(const int32_t* lengths, const int64_t* src_offsets, const int64_t* values, int64_t n,
+                             int64_t values_bound, int32_t* dst_lengths, int64_t* dst_offsets, int64_t* dst_values,
+                             int64_t dst_capacity, void* stream) {
+  if (n < 0 || values_bound < 0 || dst_capacity < 0) return fail(RAP_ERR_INVALID_ARGUMENT, "negative size");
+  if (!src_offsets || !dst_offsets) return fail(RAP_ERR_INVALID_ARGUMENT, "offsets NULL");
+  if (n > 0 && (!lengths || !dst_lengths)) return fail(RAP_ERR_INVALID_ARGUMENT, "lengths NULL");
+  if (values_bound > 0 && (!values || !dst_values)) return fail(RAP_ERR_INVALID_ARGUMENT, "values NULL");
+  const int rc = launch_jagged_append(lengths, src_offsets, values, n, values_bound, dst_lengths, dst_offsets,
+                                      dst_values, dst_capacity, stream);
+  if (rc != 0) return cuda_fail((cudaError_t)rc, "jagged append launch");
+  return RAP_OK;
+}

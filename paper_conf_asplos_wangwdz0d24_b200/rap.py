@@ -21,7 +21,10 @@ STATUS = {0: "OK", 1: "INVALID_ARGUMENT", 2: "INVALID_GRAPH", 3: "INVALID_PARAM"
 
 EXPORTS = ["rap_plan_create", "rap_plan_output_shape", "rap_preprocess", "rap_preprocess_host", "rap_set_budget",
            "rap_predict_latency_us", "rap_choose_budget", "rap_plan_info_get", "rap_debug_trace", "rap_plan_destroy",
-           "rap_status_string", "rap_last_error"]
+           "rap_status_string", "rap_last_error", "rap_shard_rows", "rap_plan_output_costs", "rap_place",
+           "rap_plan_create_sharded", "rap_jagged_append"]
+PLACE_MODES = {"balanced": 0, "round_robin": 1, "skewed": 2}
+RAP_OUT_CHAIN = 1
 
 
 class RapError(RuntimeError):
@@ -55,7 +58,13 @@ class RapRawBatch(C.Structure):
 
 class RapOutput(C.Structure):
     _fields_ = [("dense_out", C.c_void_p), ("dense_ld", C.c_int64), ("lengths", C.c_void_p),
-                ("offsets", C.c_void_p), ("values", C.c_void_p), ("values_capacity", C.c_int64)]
+                ("offsets", C.c_void_p), ("values", C.c_void_p), ("values_capacity", C.c_int64),
+                ("flags", C.c_int32), ("reserved", C.c_int32)]
+
+
+class RapResidual(C.Structure):
+    _fields_ = [("output", C.c_int32), ("owner", C.c_int32), ("helper", C.c_int32), ("pad", C.c_int32),
+                ("split_row", C.c_int64)]
 
 
 class RapPlanInfo(C.Structure):
@@ -107,6 +116,18 @@ def load(build_if_stale: bool = False):
     L.rap_status_string.argtypes = [C.c_int]
     L.rap_last_error.restype = C.c_char_p
     L.rap_last_error.argtypes = []
+    L.rap_shard_rows.restype = C.c_int
+    L.rap_shard_rows.argtypes = [C.c_int64, C.c_int32, C.c_int32, C.POINTER(C.c_int64), C.POINTER(C.c_int64)]
+    L.rap_plan_output_costs.restype = C.c_int
+    L.rap_plan_output_costs.argtypes = [P, C.c_int64, P, P]
+    L.rap_place.restype = C.c_int
+    L.rap_place.argtypes = [P, P, C.c_int32, C.c_int32, C.c_int32, C.c_int64, C.c_double, P, P,
+                            C.POINTER(RapResidual)]
+    L.rap_plan_create_sharded.restype = C.c_int
+    L.rap_plan_create_sharded.argtypes = [C.POINTER(RapGraph), C.POINTER(RapOpParam), C.c_int32, C.c_int32, C.c_int32,
+                                          P, C.c_int32, C.c_int32, C.POINTER(P)]
+    L.rap_jagged_append.restype = C.c_int
+    L.rap_jagged_append.argtypes = [P, P, P, C.c_int64, C.c_int64, P, P, P, C.c_int64, P]
     _lib = L
     return L
 
@@ -226,6 +247,20 @@ class DeviceBatch:
                                   self.sp_nnz.ctypes.data)
 
 
+def row_view(raw: "DeviceBatch", row0: int, n_rows: int) -> "RapRawBatch":
+    """A RapRawBatch over rows [row0, row0 + n_rows) of a device batch (pointer
+    arithmetic only; row0 a multiple of 32 so validity words stay whole).
+    sp_nnz stays the full batch's (an upper bound, used only for capacity)."""
+    assert row0 % 32 == 0 and 0 <= row0 and row0 + n_rows <= raw.n_rows
+    def ptrs(xs, elem, scale=1):
+        return _ptr_array([None if x is None else x.data_ptr() + (row0 // scale) * elem for x in xs])
+    arrs = [ptrs(raw.dense, 4), ptrs(raw.dense_valid, 4, 32), ptrs(raw.sp_off, 4),
+            _ptr_array([x.data_ptr() for x in raw.sp_val]), ptrs(raw.sp_valid, 4, 32)]
+    st = RapRawBatch(n_rows, *[C.cast(a, C.c_void_p) for a in arrs], raw.sp_nnz.ctypes.data)
+    st._keep = arrs
+    return st
+
+
 class DeviceOutput:
     """Output tensors (device, or pinned host when pin=True) + their C struct."""
 
@@ -265,6 +300,33 @@ class Plan:
         _check(L.rap_plan_create(C.byref(g), params, len(spec["nodes"]), device, sm_budget, C.byref(h)))
         self.handle = h
         self.device = device
+
+    @classmethod
+    def sharded(cls, spec, sparse_owner, rank: int, world: int, device: int = 0, sm_budget: int = 0):
+        """rap_plan_create_sharded: this rank's sparse outputs (full batch) +
+        every dense output over its batch shard (include/rap.h)."""
+        L = load()
+        self = cls.__new__(cls)
+        self.spec = spec
+        g, params, self._keep = marshal_graph(spec)
+        own = np.ascontiguousarray(sparse_owner, dtype=np.int32)
+        self._keep.append(own)
+        h = C.c_void_p()
+        _check(L.rap_plan_create_sharded(C.byref(g), params, len(spec["nodes"]), device, sm_budget,
+                                         own.ctypes.data, rank, world, C.byref(h)))
+        self.handle = h
+        self.device = device
+        return self
+
+    def output_costs(self, n_rows, sp_nnz):
+        f = self.output_shape(n_rows, sp_nnz)[1]
+        nnz = np.ascontiguousarray(sp_nnz if len(sp_nnz) else [0], dtype=np.int64)
+        cost = np.zeros(max(f, 1), dtype=np.float64)
+        _check(load().rap_plan_output_costs(self.handle, n_rows, nnz.ctypes.data, cost.ctypes.data))
+        return cost[:f]
+
+    def preprocess_struct(self, raw_struct, out_struct, stream=None):
+        _check(load().rap_preprocess(self.handle, C.byref(raw_struct), C.byref(out_struct), _stream_handle(stream)))
 
     def close(self):
         if getattr(self, "handle", None):

@@ -319,6 +319,20 @@ def make_batch(w: Workload, n_rows: int, seed: int = 1, null_segments: bool = Fa
 def output_dims(spec) -> tuple:
     """(dense output columns, sparse output features) implied by a spec, by the
     type rules of DESIGN.md §3 (no arithmetic)."""
+    d = f = 0
+    for o, t in zip(spec["outputs"], output_types(spec)):
+        if t == "D":
+            d += 1
+        elif t == "V":
+            d += spec["nodes"][o]["k"]
+        else:
+            f += 1
+    return d, f
+
+
+def output_types(spec) -> list:
+    """Type of every output node: 'D' dense scalar, 'V' OneHot vector, 'I' id
+    list (a sparse output), by the type rules of DESIGN.md §3."""
     types = {}
 
     def tin(kind, idx):
@@ -337,16 +351,7 @@ def output_dims(spec) -> tuple:
         types[i] = t
         return t
 
-    d = f = 0
-    for o in spec["outputs"]:
-        t = typ(o)
-        if t == "D":
-            d += 1
-        elif t == "V":
-            d += spec["nodes"][o]["k"]
-        else:
-            f += 1
-    return d, f
+    return [typ(o) for o in spec["outputs"]]
 
 
 def algorithmic_bytes(spec, batch, n_values_out: int) -> int:

@@ -8,7 +8,7 @@ grep -E "^FAILED|^E  " gpurun_out/pytest_gpu.log | head -8
 timeout 600 python bench.py --no-cpu-baseline ${BENCH_ARGS} > gpurun_out/bench.json 2> gpurun_out/bench.err
 python -c "import json; d=json.load(open('gpurun_out/bench.json')); print('kernel_us', d['roofline']['kernel_ms']*1e3, 'frac', d['roofline']['frac'], 'e2e', d['e2e']['value'])" 2>&1 | tail -1
 tail -2 gpurun_out/bench.err
-timeout 300 python scripts/trace.py 2>&1 | tail -7
+timeout 300 python scripts/trace.py 2>&1 | tail -14
 timeout 300 python scripts/probe.py 2>&1 | tail -8
 for v in ${VARIANTS}; do
   RAP_NVCC_FLAGS="$v" python -c "from paper_conf_asplos_wangwdz0d24_b200 import _build; _build.build(force=True)"

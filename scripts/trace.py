@@ -66,7 +66,7 @@ def main():
     okc = (cl > 0).all(axis=1)
     if okc.any():
         d = np.diff(cl[okc], axis=1)
-        print("  first canon tile of warp 0 (cycles, median over CTAs): quad %d  values %d  canon %d  stores %d" %
+        print("  first canon chunk of warp 0 (cycles, median over CTAs): stage offsets %d  ids %d  canon %d  stores %d" %
               tuple(np.median(d, axis=0)))
     cl = tr[:, 13:16].astype(np.int64)
     okc = (cl > 0).all(axis=1)

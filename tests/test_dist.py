@@ -1,0 +1,221 @@
+"""Multi-GPU path (§7.2).
+
+CPU (`not gpu`): the host logic in librap (rap_place, rap_shard_rows) and the
+residual protocol over a world_size-2 gloo group, where each rank's pieces
+come from the oracle and the stitch is checked against the oracle's
+single-process result.  GPU: every rank of a world W simulated on one B200
+(sharded plans, chained launch, rap_jagged_append) must reproduce the
+single-plan output bit for bit.
+"""
+import os
+import socket
+
+import numpy as np
+import pytest
+
+from paper_conf_asplos_wangwdz0d24_b200 import dist, synth
+
+
+# ----------------------------------------------------------------- host logic
+def test_colocation_c2():
+    w = synth.c2_terabyte(0)
+    col = dist.colocation(w.spec)
+    assert len(col) == 34 and col[:26] == [-1] * 26
+    # trigram g reads sources 3g, 3g+1, 3g+2 (mod 26): it goes with table 3g
+    assert col[26:] == [(3 * g) % 26 for g in range(8)]
+
+
+@pytest.mark.parametrize("world", [1, 2, 3, 8])
+def test_shard_rows_partition(world):
+    for B in (0, 1, 127, 128, 1000, 65536, 65537):
+        spans = [dist.shard_rows(B, r, world) for r in range(world)]
+        assert spans[0][0] == 0 and sum(n for _, n in spans) == B
+        for (r0, n), (r1, _) in zip(spans, spans[1:]):
+            assert r0 + n == r1 and r1 % 128 == 0 and n >= 0
+
+
+def _costs(n, seed):
+    rng = np.random.default_rng(seed)
+    return rng.lognormal(0.0, 1.0, n) * 1000.0
+
+
+@pytest.mark.parametrize("world", [2, 4, 8])
+def test_place_balanced_lpt_bound(world):
+    c = _costs(34, world)
+    pl = dist.place(c, None, world, "balanced", 65536, None)
+    loads = np.zeros(world)
+    for j, r in enumerate(pl.owner):
+        loads[r] += c[j]
+    assert np.allclose(loads, pl.loads)
+    # LPT: max load <= mean + largest item (Graham's bound)
+    assert loads.max() <= c.sum() / world + c.max() + 1e-6
+
+
+def test_place_round_robin_and_colocate():
+    c = np.ones(10)
+    col = [-1] * 8 + [0, 3]
+    pl = dist.place(c, col, 4, "round_robin", 4096, None)
+    groups = [j for j in range(10) if col[j] < 0]
+    for i, j in enumerate(groups):
+        assert pl.owner[j] == i % 4
+    assert pl.owner[8] == pl.owner[0] and pl.owner[9] == pl.owner[3]
+
+
+def test_place_skewed_and_residual():
+    c = np.full(32, 100.0)
+    pl = dist.place(c, None, 4, "skewed", 65536, None)
+    loads = np.array(pl.loads)
+    assert loads[0] == pytest.approx(2 * c.sum() / 4)  # rank 0 holds 2x the mean
+    pr = dist.place(c, None, 4, "skewed", 65536, 0.1)
+    r = pr.residual
+    assert r is not None and r.owner == 0 and pr.owner[r.output] == 0
+    assert r.helper != 0 and r.split_row % 128 == 0 and 128 <= r.split_row < 65536
+    moved = (65536 - r.split_row) / 65536 * c[r.output]
+    assert pr.loads[0] == pytest.approx(loads[0] - moved)
+    assert max(pr.loads) < loads.max()
+    # balanced placement of equal costs needs no residual
+    assert dist.place(c, None, 4, "balanced", 65536, 0.1).residual is None
+
+
+# ------------------------------------------------------- gloo residual protocol
+def _slice_batch(h, r0, n):
+    """Rows [r0, r0+n) of a host batch (r0 % 32 == 0); offsets stay absolute."""
+    w0, w1 = r0 // 32, (r0 + n + 31) // 32
+    return {"n_rows": n, "dense": [x[r0:r0 + n] for x in h["dense"]],
+            "dense_valid": [None if v is None else v[w0:w1] for v in h["dense_valid"]],
+            "sp_off": [o[r0:r0 + n + 1] for o in h["sp_off"]], "sp_val": h["sp_val"],
+            "sp_valid": [None if v is None else v[w0:w1] for v in h["sp_valid"]]}
+
+
+def _feature_lists(res, F, B):
+    L, O, V = res["lengths"], res["offsets"], res["values"]
+    return [[V[O[f * B + b]:O[f * B + b + 1]] for b in range(B)] for f in range(F)]
+
+
+def _gloo_worker(rank, world, port, q):
+    import torch
+    import torch.distributed as tdist
+
+    from oracle import oracle
+
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    tdist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        w = synth.c2_terabyte(0)
+        B = 1000
+        h = synth.make_batch(w, B, seed=5)
+        nodes = dist.sparse_output_nodes(w.spec)
+        costs = np.ones(len(nodes))
+        pl = dist.place(costs, dist.colocation(w.spec), world, "skewed", B, 0.05)
+        res = pl.residual
+        assert res is not None
+        sub = dict(w.spec, outputs=[nodes[res.output]])
+        n_hi = B - res.split_row
+        # the piece each side sees has the same shapes: lengths, offsets, values (bound)
+        bound = n_hi  # single-valued C2 lists: one id per row at most
+        if rank == res.helper:
+            hi = oracle.run(sub, _slice_batch(h, res.split_row, n_hi))
+            vals = np.zeros(bound, np.int64)
+            vals[: len(hi["values"])] = hi["values"]
+            piece = [torch.from_numpy(hi["lengths"].astype(np.int32)), torch.from_numpy(hi["offsets"]),
+                     torch.from_numpy(vals)]
+            dist.nccl_exchange(rank, res, piece, None)
+            q.put((rank, "sent"))
+        elif rank == res.owner:
+            bufs = [torch.zeros(n_hi, dtype=torch.int32), torch.zeros(n_hi + 1, dtype=torch.int64),
+                    torch.zeros(bound, dtype=torch.int64)]
+            dist.nccl_exchange(rank, res, None, bufs)
+            lo = oracle.run(sub, _slice_batch(h, 0, res.split_row))
+            # stitch exactly as rap_jagged_append does: T = running total
+            T = int(lo["offsets"][-1])
+            so = bufs[1].numpy()
+            lengths = np.concatenate([lo["lengths"], bufs[0].numpy()])
+            offsets = np.concatenate([lo["offsets"], T + so[1:] - so[0]])
+            values = np.concatenate([lo["values"], bufs[2].numpy()[: int(so[-1] - so[0])]])
+            full = oracle.run(sub, h)
+            ok = (np.array_equal(lengths, full["lengths"]) and np.array_equal(offsets, full["offsets"])
+                  and np.array_equal(values, full["values"]))
+            q.put((rank, "ok" if ok else "MISMATCH"))
+        else:
+            q.put((rank, "idle"))
+        tdist.barrier()
+    finally:
+        tdist.destroy_process_group()
+
+
+def test_residual_exchange_gloo_world2():
+    import torch.multiprocessing as mp
+
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_gloo_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    for p in procs:
+        p.join(120)
+    got = dict(q.get(timeout=5) for _ in range(2))
+    assert all(p.exitcode == 0 for p in procs), got
+    assert sorted(got.values()) == ["ok", "sent"], got
+
+
+# --------------------------------------------------- GPU: simulated ranks
+@pytest.mark.gpu
+@pytest.mark.parametrize("world,mode", [(2, "balanced"), (4, "round_robin"), (4, "skewed"), (8, "skewed")])
+def test_sharded_ranks_match_single_plan(world, mode):
+    import torch
+
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    from paper_conf_asplos_wangwdz0d24_b200 import rap
+
+    w = synth.c2_terabyte(0)
+    B = 3000
+    h = synth.make_batch(w, B, seed=21)
+    raw = rap.DeviceBatch(h, "cuda:0")
+    full = rap.Plan(w.spec, device=0)
+    fo = rap.DeviceOutput(full, B, raw.sp_nnz, "cuda:0")
+    full.preprocess(raw, fo)
+    torch.cuda.synchronize()
+    want = fo.to_numpy()
+    F = fo.f_out
+    wl = _feature_lists(want, F, B)
+    pl = dist.plan_placement(w.spec, B, raw.sp_nnz, world, mode, imbalance_tol=0.05)
+    if mode == "skewed":
+        assert pl.residual is not None
+    ranks = [dist.ShardedPreprocessor(w.spec, pl, r, world, B, raw.sp_nnz, device=0) for r in range(world)]
+    outs = [rk.new_output() for rk in ranks]
+    box = {}
+
+    def exchange(rank, res, piece, bufs):  # one-GPU stand-in for the NCCL send/recv
+        if rank == res.helper:
+            box["piece"] = [t.clone() for t in piece]
+        elif rank == res.owner:
+            for dst, src in zip(bufs, box["piece"]):
+                dst.copy_(src)
+
+    order = list(range(world))
+    if pl.residual is not None:  # the helper's piece exists before the owner stitches
+        order.remove(pl.residual.helper)
+        order.insert(0, pl.residual.helper)
+    for r in order:
+        ranks[r].preprocess(raw, outs[r], exchange=exchange)
+    torch.cuda.synchronize()
+    seen = []
+    for r in range(world):
+        got = outs[r].to_numpy()
+        r0, n = dist.shard_rows(B, r, world)
+        assert np.array_equal(got["dense"].view(np.uint32), want["dense"][r0:r0 + n].view(np.uint32))
+        gl = _feature_lists(got, len(got["features"]), B)
+        for k, j in enumerate(got["features"]):
+            assert all(np.array_equal(a, b) for a, b in zip(gl[k], wl[j])), (r, j)
+        L = got["lengths"].reshape(-1)
+        assert got["offsets"][0] == 0 and np.array_equal(np.diff(got["offsets"]), L)
+        seen += got["features"]
+    assert sorted(seen) == list(range(F))
+    for rk in ranks:
+        rk.close()
+    full.close()
