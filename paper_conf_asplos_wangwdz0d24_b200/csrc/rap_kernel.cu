@@ -52,7 +52,10 @@ constexpr int kGroups = kTileRows / 32;  // row groups of a sparse tile (one row
 // Warp-private shared memory of the sparse phases: the NGram
 // paths use its first 4 KB; the canonical paths stage Arrow offsets,
 // validity words and ids in it with cp.async (nothing in flight in registers).
-constexpr int kWarpScr = 7168;
+#ifndef RAP_WARP_SCR
+#define RAP_WARP_SCR 6656
+#endif
+constexpr int kWarpScr = RAP_WARP_SCR;  // 8 warps x 6.5 KB: 4 CTAs fit an SM's 228 KB
 constexpr int kNgScratch = kWarps * kWarpScr;
 static_assert(4 * kMaxNgramK * 32 * 4 <= kWarpScr, "NGram scratch exceeds the warp region");
 constexpr int kLChunkTiles = 8;  // length pass: tiles staged per round
@@ -776,21 +779,31 @@ __device__ __noinline__ long long value_chunk_canon(const P& p, const FeatCtx& f
   cp_async_wait_all();
   __syncwarp();
   trace_clk(p.c, 9, soff[0]);
-  // quad layout: the lane owns local rows j*128 + 4*lane + k
+  // quad layout: the lane owns local rows j*128 + 4*lane + k; one 16-byte
+  // and one 4-byte shared load give its 5 offsets, one word its 4 validity bits
   unsigned act = 0, full = 0;
   bool ok = true;
+  const int xc = (int)min(xcap, (int64_t)INT32_MAX);
+  const int nl = has_fill ? (int)min((int64_t)1, null_xcap) : 0;  // R10 / R14
 #pragma unroll
-  for (int j = 0; j < kVChunkTiles; ++j)
+  for (int j = 0; j < kVChunkTiles; ++j) {
+    const int lr0 = j * kTileRows + 4 * lane;
+    if (lr0 < NR) {
+      const int4 a = *reinterpret_cast<const int4*>(soff + lr0);
+      const int a4 = soff[lr0 + 4];
+      const unsigned vb = (sbm[lr0 >> 5] >> (lr0 & 31)) & 15u;
+      const int d[4] = {a.y - a.x, a.z - a.y, a.w - a.z, a4 - a.w};
 #pragma unroll
-    for (int k = 0; k < 4; ++k) {
-      const int lr = j * kTileRows + 4 * lane + k;
-      if (lr < NR) {
-        const int32_t l = len_s(soff, sbm, lr, xcap, has_fill, null_xcap);
+      for (int k = 0; k < 4; ++k) {
+        const bool in = lr0 + k < NR;
+        const bool va = in && ((vb >> k) & 1u);
+        const int l = !in ? 0 : (va ? min(max(d[k], 0), xc) : nl);  // R5 FirstX cap
         ok &= l <= 1;
         act |= (l == 1 ? 1u : 0u) << (4 * j + k);
-        full |= (((sbm[lr >> 5] >> (lr & 31)) & 1u) ? 1u : 0u) << (4 * j + k);
+        full |= (va ? 1u : 0u) << (4 * j + k);
       }
     }
+  }
   if (!__all_sync(0xffffffffu, ok)) {
     __syncwarp();
     return -1;
@@ -1093,7 +1106,8 @@ static_assert(offsetof(NgParams, scn) == sizeof(Chain) * 4 && offsetof(NgParams,
                   sizeof(Canon) % 8 == 0 && sizeof(NGramDesc) % 8 == 0,
               "NgParams is staged as one run of 8-byte words");
 constexpr int kNgParamWords = align_up((int)sizeof(NgParams), 16) / 4;
-static_assert(kNgParamWords * 4 + 4 * kTileRows * 4 <= 4 * kMaxNgramK * 32 * 4, "ngram_tile_fast scratch too large");
+constexpr int kNgStageOff = kTileRows + 4;  // staged offsets per source (129 used, 16-byte rows)
+static_assert((kNgParamWords + 4 * kTileRows + 4 * kNgStageOff + 16) * 4 <= kWarpScr, "ngram_tile_fast scratch too large");
 
 // Stage feature f's fast-NGram parameters into the warp scratch: every
 // lane's loads in flight before any store.
@@ -1136,18 +1150,23 @@ __device__ __noinline__ long long ngram_tile_fast(const P& p, int f, int64_t rt,
   // global reads on the dependent path); per-(source, row) id positions after
   const NgParams& G = *reinterpret_cast<const NgParams*>(scr);
   int32_t* pos = scr + kNgParamWords;  // [4][kTileRows]: child index, -1 = fill, -2 = absent
+  // every source's offsets / validity words staged with cp.async (no quads
+  // held in registers): [4][kNgStageOff] int32 then [4][4] u32 after pos
+  int32_t* soff = pos + 4 * kTileRows;
+  uint32_t* sbm = reinterpret_cast<uint32_t*>(soff + 4 * kNgStageOff);
   const int k = G.ng.k, n = G.ng.n;
   const int64_t B = p.c.n_rows;
   const int64_t r0 = rt * kTileRows;
   const int64_t row = r0 + 4 * lane;
-  Quad q[4];
+  const int NR = (int)min((int64_t)kTileRows, B - r0);
 #pragma unroll
   for (int j = 0; j < 4; ++j)
-    if (j < k) {
-      const int32_t* off = p.off[G.src[j].src];
-      q[j] = load_quad(off, p.svalid[G.src[j].src], r0, lane, B, (reinterpret_cast<uintptr_t>(off) & 15) == 0);
-    }
+    if (j < k) stage_offsets(p.off[G.src[j].src], p.svalid[G.src[j].src], r0, NR, soff + j * kNgStageOff, sbm + 4 * j, lane);
+  cp_async_wait_all();
+  __syncwarp();
+  // per (source, row) output lengths of the lane's 4 rows, 4 bits each
   int pn[4] = {0, 0, 0, 0};
+  unsigned l1 = 0, fullm = 0;  // bit 4j+kk: source j of row kk has one id / is valid
   bool ok = true;
 #pragma unroll
   for (int j = 0; j < 4; ++j)
@@ -1155,14 +1174,25 @@ __device__ __noinline__ long long ngram_tile_fast(const P& p, int f, int64_t rt,
       const Chain& sc = G.src[j];
 #pragma unroll
       for (int kk = 0; kk < 4; ++kk) {
-        const int l = quad_len(q[j], kk, lane, row + kk, B, sc.xcap, sc.has_fill, sc.null_xcap);
+        const int lr = 4 * lane + kk;
+        int l = 0;
+        bool fu = false;
+        if (lr < NR) {
+          l = len_s(soff + j * kNgStageOff, sbm + 4 * j, lr, sc.xcap, sc.has_fill, sc.null_xcap);
+          fu = (sbm[4 * j + (lr >> 5)] >> (lr & 31)) & 1u;
+        }
         ok &= l <= 1;
         pn[kk] += l;
+        l1 |= (l == 1 ? 1u : 0u) << (4 * j + kk);
+        fullm |= (fu ? 1u : 0u) << (4 * j + kk);
       }
     }
 #pragma unroll
   for (int kk = 0; kk < 4; ++kk) ok &= pn[kk] <= n;
-  if (!__all_sync(0xffffffffu, ok)) return -1;
+  if (!__all_sync(0xffffffffu, ok)) {
+    __syncwarp();
+    return -1;
+  }
   int32_t l[4], e[4];
   int tot = 0;
 #pragma unroll
@@ -1176,15 +1206,15 @@ __device__ __noinline__ long long ngram_tile_fast(const P& p, int f, int64_t rt,
 #pragma unroll
   for (int j = 0; j < 4; ++j)
     if (j < k) {
-      const Chain& sc = G.src[j];
       int a[4];
 #pragma unroll
       for (int kk = 0; kk < 4; ++kk) {
-        const bool pr = l[kk] == 1 && quad_len(q[j], kk, lane, row + kk, B, sc.xcap, sc.has_fill, sc.null_xcap) == 1;
-        const bool fu = quad_valid(q[j], kk, lane);
-        pres |= (pr ? 1u : 0u) << (4 * j + kk);
-        full |= (fu ? 1u : 0u) << (4 * j + kk);
-        a[kk] = pr ? (fu ? q[j].a[kk] : -1) : -2;
+        const unsigned bit = 1u << (4 * j + kk);
+        const bool pr = l[kk] == 1 && (l1 & bit);
+        const bool fu = fullm & bit;
+        pres |= pr ? bit : 0u;
+        full |= fu ? bit : 0u;
+        a[kk] = pr ? (fu ? soff[j * kNgStageOff + 4 * lane + kk] : -1) : -2;
       }
       *reinterpret_cast<int4*>(pos + j * kTileRows + 4 * lane) = make_int4(a[0], a[1], a[2], a[3]);
     }
@@ -1663,7 +1693,17 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
           stage_offsets(off, bm, R0, NR, soff, sbm, lane);
           cp_async_wait_all();
           __syncwarp();
-          for (int lr = lane; lr < NR; lr += 32) part += len_s(soff, sbm, lr, xcap, has_fill, null_xcap);
+          const int xc = (int)min(xcap, (int64_t)INT32_MAX);
+          const int nl = has_fill ? (int)min((int64_t)1, null_xcap) : 0;  // R10 / R14
+          for (int lr0 = 4 * lane; lr0 < NR; lr0 += 128) {  // 4 rows per lane per step
+            const int4 a = *reinterpret_cast<const int4*>(soff + lr0);
+            const int a4 = soff[lr0 + 4];
+            const unsigned vb = (sbm[lr0 >> 5] >> (lr0 & 31)) & 15u;
+            const int d[4] = {a.y - a.x, a.z - a.y, a.w - a.z, a4 - a.w};
+#pragma unroll
+            for (int k = 0; k < 4; ++k)
+              if (lr0 + k < NR) part += ((vb >> k) & 1u) ? min(max(d[k], 0), xc) : nl;  // R5 FirstX cap
+          }
           __syncwarp();
           t += nt;
         }
