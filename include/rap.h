@@ -176,10 +176,11 @@ rap_status rap_plan_output_shape(const rap_plan* plan, int64_t n_rows, const int
                                  int64_t* d_out_cols, int64_t* n_sparse_out, int64_t* values_upper_bound);
 
 /* Enqueue one fused preprocessing launch on `stream` (a cudaStream_t; NULL =
- * legacy default stream).  Device buffers.  No host synchronisation, no host
- * reads of device data; the only allocation is the one-time growth of the
- * plan's scan-state when n_rows exceeds every earlier call.  Outputs are valid
- * when the stream reaches this point. */
+ * legacy default stream).  Device buffers.  No allocation and no host reads
+ * of device data.  A batch whose shape (rows, grid, quantised mean list
+ * lengths) is new uploads its per-warp work partition (async, pinned); the
+ * plan caches 8 shapes and only evicting one synchronises `stream`.  Outputs
+ * are valid when the stream reaches this point. */
 rap_status rap_preprocess(rap_plan* plan, const rap_raw_batch* raw, const rap_output* out, void* stream);
 
 /* Same as rap_preprocess with HOST raw and output buffers (pinned memory makes

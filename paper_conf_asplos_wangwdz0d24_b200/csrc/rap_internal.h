@@ -154,6 +154,9 @@ struct DProg {
 // blocks, adds its predecessors' aggregates and then writes its tiles.  No
 // grid barrier, no per-tile look-back.
 constexpr int kMaxCtas = 2048;        // grid cap
+constexpr int kWarpsPerCta = kThreads / 32;
+constexpr int kPartLen = kMaxCtas * kWarpsPerCta + 1;  // per-warp partition boundaries
+constexpr int kPartSlots = 8;         // cached partitions per plan
 constexpr int kTileRows = 128;        // rows of a sparse tile (4 groups of 32)
 constexpr int kDenseBlockRows = 128;  // rows of a dense block (CTA unit)
 
@@ -178,7 +181,7 @@ struct Common {
   // counter and advances the epoch, so launch parameters are identical from
   // call to call (CUDA-graph replayable).
   unsigned long long* sched;
-  const int64_t* part;         // [grid + 1] unit range of each CTA rank
+  const int64_t* part;         // [grid * 8 + 1] unit range of each warp (CTA rank r: slots 8r .. 8r+8)
   unsigned long long* agg;     // [kMaxCtas] per-rank aggregate words (epoch-tagged)
   float* dense_out;
   int64_t ld;

@@ -80,7 +80,13 @@ __host__ __device__ constexpr int align_up(int x, int a) { return (x + a - 1) / 
 // ----------------------------------------------------------------------------
 // Scalar helpers.
 
-__device__ __forceinline__ uint64_t reduce_M(uint64_t h, int64_t M) {  // R2
+__device__ __forceinline__ uint64_t reduce_M(uint64_t h, int64_t M) {  // R2: floor(h * M / 2^64)
+  if (((uint64_t)M >> 32) == 0) {
+    // M < 2^32 (every table size here): floor((hi*M + floor(lo*M / 2^32)) / 2^32), exact
+    const uint64_t m = (uint64_t)M;
+    const uint64_t t = (uint64_t)(uint32_t)(h >> 32) * m + (((uint64_t)(uint32_t)h * m) >> 32);
+    return t >> 32;
+  }
   return __umul64hi(h, (uint64_t)M);
 }
 
@@ -870,6 +876,110 @@ __device__ __noinline__ long long value_chunk_canon(const P& p, const FeatCtx& f
   return run - base;
 }
 
+constexpr int kNullRow = INT_MIN;
+// Tile rt of a canonical chain whose rows may hold several ids (multi-hot,
+// FirstX caps): element-parallel.  Offsets / validity staged with cp.async;
+// per row its output start goes to shared memory; each 128-element window of
+// the tile's output marks the rows that start in it and a warp max-scan gives
+// every element its row (elements e = eb + 32u + lane, so id loads and value
+// stores are coalesced).  Element e of row r reads input soff[r] + (e -
+// out_start[r]) (FirstX keeps a prefix, R5) or the fill id of a null row (R10).
+template <class P>
+__device__ __noinline__ long long value_tile_multi(const P& p, const FeatCtx& fc, int64_t rt, int lane, long long base,
+                                                   unsigned char* wscr) {
+  int32_t* soff = reinterpret_cast<int32_t*>(wscr);             // [132]
+  uint32_t* sbm = reinterpret_cast<uint32_t*>(wscr + 528);       // [4]
+  int32_t* sdelta = reinterpret_cast<int32_t*>(wscr + 544);     // [128] input index - output index of a row
+  int32_t* mark = reinterpret_cast<int32_t*>(wscr + 1056);      // [128] row starting at window slot
+  const int f = fc.f;
+  const int64_t B = p.c.n_rows;
+  const int64_t R0 = rt * kTileRows;
+  const int NR = (int)min((int64_t)kTileRows, B - R0);
+  const int src = fc.src;
+  stage_offsets(p.off[src], p.svalid[src], R0, NR, soff, sbm, lane);
+  cp_async_wait_all();
+  __syncwarp();
+  const int xc = (int)min(fc.xcap, (int64_t)INT32_MAX);
+  const int nl = fc.has_fill ? (int)min((int64_t)1, fc.null_xcap) : 0;  // R10 / R14
+  const int lr0 = 4 * lane;
+  int l[4], e[4], tot = 0;
+  unsigned vbits = 0;
+  {
+    const int4 a = *reinterpret_cast<const int4*>(soff + lr0);
+    const int a4 = soff[lr0 + 4];
+    vbits = (sbm[lr0 >> 5] >> (lr0 & 31)) & 15u;
+    const int d[4] = {a.y - a.x, a.z - a.y, a.w - a.z, a4 - a.w};
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      const bool in = lr0 + k < NR;
+      l[k] = !in ? 0 : (((vbits >> k) & 1u) ? min(max(d[k], 0), xc) : nl);  // R5 FirstX cap
+      if (!in) vbits &= ~(1u << k);
+      e[k] = tot;
+      tot += l[k];
+    }
+  }
+  const int incl = warp_incl_scan(tot, lane);
+  const int L = incl - tot;
+  const int T = __shfl_sync(0xffffffffu, incl, 31);
+  {
+    // element ee of row r reads input ee + sdelta[r]; kNullRow: a filled null row
+    int dl[4];
+#pragma unroll
+    for (int k = 0; k < 4; ++k) dl[k] = ((vbits >> k) & 1u) ? soff[lr0 + k] - (L + e[k]) : kNullRow;
+    *reinterpret_cast<int4*>(sdelta + lr0) = make_int4(dl[0], dl[1], dl[2], dl[3]);
+  }
+  const long long lb = base + L;
+  store_quad(p.c.lengths + (int64_t)f * B + R0 + lr0, p.c.offsets + (int64_t)f * B + R0 + lr0, R0 + lr0, B, l, lb,
+             e);
+  if (f == p.c.n_sparse_out - 1 && rt == p.c.tiles_per_feature - 1 && lane == 31) {
+    p.c.offsets[(int64_t)p.c.n_sparse_out * B] = base + T;  // total, R17
+    if (base + T > p.c.values_cap) atomicExch(p.c.err, 1);
+  }
+  __syncwarp();
+  const int64_t* val = p.val[src];
+  int64_t* values = p.c.values;
+  const long long cap = p.c.values_cap;
+  int carry = 0;  // row of the last element of the previous window
+  for (int eb = 0; eb < T; eb += 128) {
+    *reinterpret_cast<int4*>(mark + lr0) = make_int4(-1, -1, -1, -1);
+    __syncwarp();
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      const int st = L + e[k] - eb;
+      if (l[k] > 0 && st >= 0 && st < 128) mark[st] = lr0 + k;
+    }
+    __syncwarp();
+    int64_t x[4];
+    unsigned act = 0, full = 0;
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      // row of element eb + 32u + lane: the last row starting at or before it
+      const int m = mark[32 * u + lane];
+      const unsigned starts = __ballot_sync(0xffffffffu, m >= 0);
+      const unsigned le = starts & (0xffffffffu >> (31 - lane));
+      const int from = le ? 31 - __clz(le) : 0;
+      const int got = __shfl_sync(0xffffffffu, m, from);
+      const int r = le ? got : carry;
+      carry = __shfl_sync(0xffffffffu, r, 31);
+      const int ee = eb + 32 * u + lane;
+      const bool in = ee < T;
+      const int dlt = sdelta[r];
+      const bool va = in && dlt != kNullRow;
+      act |= (in ? 1u : 0u) << u;
+      full |= (va ? 1u : 0u) << u;
+      x[u] = va ? __ldg(val + (ee + dlt)) : fc.fill;
+    }
+    canon_apply_n<4>(fc.q, p.c.itab, x, act, full);
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const long long pos = base + eb + 32 * u + lane;
+      if (((act >> u) & 1u) && pos < cap) values[pos] = x[u];
+    }
+    __syncwarp();
+  }
+  return T;
+}
+
 // Tile of any other SRC_SPARSE / SRC_DENSE_BUCKET chain (op interpreter).
 template <class P>
 __device__ __noinline__ long long value_tile_generic(const P& p, int f, int64_t rt, int lane, long long base) {
@@ -1656,15 +1766,15 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
     p.c.trace[(int64_t)blockIdx.x * kTracePts + 7] = (unsigned long long)rank;
   }
   const int64_t S = p.c.n_sparse_tiles, T = p.c.tiles_per_feature;
-  const int64_t s0 = __ldg(p.c.part + rank), s1 = __ldg(p.c.part + rank + 1);  // my sparse tiles
+  // my sparse tiles [s0, s1) and my warp's [w0, w1) (host per-warp partition)
+  const int64_t s0 = __ldg(p.c.part + rank * kWarps), s1 = __ldg(p.c.part + (rank + 1) * kWarps);
+  const int64_t w0 = __ldg(p.c.part + rank * kWarps + warp), w1 = __ldg(p.c.part + rank * kWarps + warp + 1);
   unsigned char* wscr = smem + warp * kWarpScr;  // warp-private region (sparse phases)
   int32_t* scr = reinterpret_cast<int32_t*>(wscr);
   if (p.c.trace != nullptr && tid == 0 && (int64_t)blockIdx.x < p.c.trace_cap)
     p.c.trace[(int64_t)blockIdx.x * kTracePts + 5] = (unsigned long long)(s0 | ((s1 - s0) << 32));
 
   // (L) output length total of my warp's sub-range -> CTA aggregate
-  const int64_t ns = s1 - s0;
-  const int64_t w0 = s0 + ns * warp / kWarps, w1 = s0 + ns * (warp + 1) / kWarps;
   long long mine = 0, part = 0;  // warp-uniform / per-lane partial totals
   trace_clk(p.c, 21, 0);
   // per-feature dispatch state in warp-private shared memory (not registers:
@@ -1674,8 +1784,14 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
   __syncwarp();
   {
     const int64_t B = p.c.n_rows;
+    int fcur = 0;
+    int64_t fend = -1;
     for (int64_t t = w0; t < w1;) {
-      const int f = (int)((uint64_t)t / (uint64_t)T);
+      if (t >= fend) {  // feature boundary: one 64-bit division per feature, not per tile
+        fcur = (int)((uint64_t)t / (uint64_t)T);
+        fend = (int64_t)(fcur + 1) * T;
+      }
+      const int f = fcur;
       if (f != fc.f) load_ctx(p, f, fc);
       const int64_t tend = min(w1, (int64_t)(f + 1) * T);
       if (fc.sk == SRC_SPARSE) {
@@ -1780,8 +1896,14 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
 #ifdef RAP_DBG_SKIP_V
     if (false)
 #endif
+    int fcur = 0;
+    int64_t fend = -1;
     for (int64_t t = w0; t < w1;) {
-      const int f = (int)((uint64_t)t / (uint64_t)T);
+      if (t >= fend) {  // feature boundary: one 64-bit division per feature, not per tile
+        fcur = (int)((uint64_t)t / (uint64_t)T);
+        fend = (int64_t)(fcur + 1) * T;
+      }
+      const int f = fcur;
       if (f != fc.f) load_ctx(p, f, fc);
       if (fc.kind == TK_CANON) {
         const int nt = (int)min((int64_t)kVChunkTiles, min(w1, (int64_t)(f + 1) * T) - t);
@@ -1791,6 +1913,10 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
           t += nt;
           continue;
         }
+        // multi-id rows: element-parallel tiles
+        for (int j = 0; j < nt; ++j) run += value_tile_multi(p, fc, t + j - (int64_t)f * T, lane, run, wscr);
+        t += nt;
+        continue;
       }
       run += value_tile(p, fc, t - (int64_t)f * T, lane, run, scr);
       ++t;

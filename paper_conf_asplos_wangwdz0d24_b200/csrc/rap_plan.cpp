@@ -87,8 +87,12 @@ struct rap_plan {
   size_t off_ops = 0, off_sprogs = 0, off_oprogs = 0, off_dprogs = 0, off_ftab = 0, off_itab = 0;
   // per-CTA partition of the unit sequence (cost model),
   // re-uploaded only when its key (rows, grid, quantised list lengths) changes
-  std::vector<int64_t> part_key;
-  int64_t* d_part = nullptr;               // [kMaxCtas + 1]
+  // kPartSlots cached partitions (batches of different shapes alternate
+  // without re-uploads); slot i: key part_keys[i], device d_part + i * kPartLen
+  std::vector<std::vector<int64_t>> part_keys;
+  int part_next = 0;
+  int64_t* d_part = nullptr;               // [kPartSlots * kPartLen]
+  int64_t* h_part = nullptr;               // pinned staging, same layout
   // scheduling state
   unsigned long long* d_sched = nullptr;   // CTAs done, launch epoch, rank counter
   unsigned long long* d_agg = nullptr;     // [kMaxCtas] per-rank aggregate words
@@ -885,7 +889,8 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
   }
   if (e == cudaSuccess) e = cudaMalloc(&P->d_agg, kMaxCtas * sizeof(unsigned long long));
   if (e == cudaSuccess) e = cudaMemset(P->d_agg, 0, kMaxCtas * sizeof(unsigned long long));
-  if (e == cudaSuccess) e = cudaMalloc(&P->d_part, (kMaxCtas + 1) * sizeof(int64_t));
+  if (e == cudaSuccess) e = cudaMalloc(&P->d_part, kPartSlots * kPartLen * sizeof(int64_t));
+  if (e == cudaSuccess) e = cudaMallocHost(&P->h_part, kPartSlots * kPartLen * sizeof(int64_t));
   if (e == cudaSuccess) e = cudaMalloc(&P->d_err, sizeof(int32_t));
   if (e == cudaSuccess) e = cudaMemset(P->d_err, 0, sizeof(int32_t));
   if (e != cudaSuccess) {
@@ -915,6 +920,7 @@ void rap_plan_destroy(rap_plan* P) {
   cudaFree(P->d_sched);
   cudaFree(P->d_agg);
   cudaFree(P->d_part);
+  cudaFreeHost(P->h_part);
   cudaFree(P->d_err);
   cudaFree(P->d_trace);
   for (void* s : P->stage) cudaFree(s);
@@ -1092,14 +1098,18 @@ static double dense_row_cost(const rap_plan* P, const DProg& dp) {
 // (rows, grid, each used source's mean list length quantised to 2^(1/4)
 // steps), so batches of the same shape reuse the uploaded table.
 static rap_status update_partition(rap_plan* P, int64_t B, const int64_t* nnz, int64_t S, int64_t D, int grid,
-                                   cudaStream_t stream) {
+                                   cudaStream_t stream, const int64_t** d_part_out) {
   std::vector<int64_t> key = {B, grid};
   (void)D;
   for (int s : P->used_sparse) {
     const double m = nnz && B > 0 ? (double)std::max<int64_t>(nnz[s], 0) / (double)B : 0.0;
     key.push_back(m <= 1.0 / 64 ? -1000 : (int64_t)std::lround(4.0 * std::log2(m)));
   }
-  if (key == P->part_key) return RAP_OK;
+  for (size_t i = 0; i < P->part_keys.size(); ++i)
+    if (P->part_keys[i] == key) {
+      *d_part_out = P->d_part + i * kPartLen;
+      return RAP_OK;
+    }
   const int64_t F = (int64_t)P->souts.size();
   const int64_t T = F ? S / F : 0;
   const double kTileFixed = 400.0;  // per-unit overhead (lane-instructions)
@@ -1113,23 +1123,38 @@ static rap_status update_partition(rap_plan* P, int64_t B, const int64_t* nnz, i
   const int64_t U = S;
   double W = 0;
   for (int64_t u = 0; u < U; ++u) W += unit_cost(u);
-  // dense blocks go round robin over the ranks (block d to rank d mod
-  // grid).  The sparse ranges ignore them: the CTAs of an SM share its issue
-  // slots, so a CTA's dense block mostly fills slots its SM neighbours leave
-  // idle (measured: charging it to the CTA's sparse share made C2 slower).
-  std::vector<int64_t> part(grid + 1);
+  // One contiguous cost-balanced range per WARP (grid x kWarps slots; a CTA
+  // owns the ranges of its 8 warps): warps of a CTA finish together, so no
+  // warp idles at the CTA's barriers.  Dense blocks go round robin over the
+  // ranks (block d to rank d mod grid) and are not charged here: the CTAs of
+  // an SM share its issue slots, so a dense block mostly fills slots its SM
+  // neighbours leave idle (measured: charging it made C2 slower).
+  const int slot = (int)P->part_keys.size() < kPartSlots ? (int)P->part_keys.size() : P->part_next;
+  P->part_next = (slot + 1) % kPartSlots;
+  int64_t* part = P->h_part + (size_t)slot * kPartLen;
+  const int n = grid * kWarpsPerCta;
+  // evicting: the pinned slot may still feed an in-flight upload (only
+  // after kPartSlots distinct batch shapes; never in steady state)
+  cudaError_t e = cudaSuccess;
+  if ((int)P->part_keys.size() == kPartSlots) e = cudaStreamSynchronize(stream);
+  if (e != cudaSuccess) return cuda_fail(e, "partition slot reuse");
   part[0] = 0;
   double acc = 0;
   int64_t u = 0;
-  for (int c = 1; c < grid; ++c) {
-    const double target = W * (double)c / (double)grid;
+  for (int c = 1; c < n; ++c) {
+    const double target = W * (double)c / (double)n;
     while (u < U && acc + 0.5 * unit_cost(u) < target) acc += unit_cost(u++);
     part[c] = u;
   }
-  part[grid] = U;
-  cudaError_t e = cudaMemcpyAsync(P->d_part, part.data(), sizeof(int64_t) * (grid + 1), cudaMemcpyHostToDevice, stream);
+  part[n] = U;
+  int64_t* d = P->d_part + (size_t)slot * kPartLen;
+  e = cudaMemcpyAsync(d, part, sizeof(int64_t) * (n + 1), cudaMemcpyHostToDevice, stream);
   if (e != cudaSuccess) return cuda_fail(e, "partition upload");
-  P->part_key = key;
+  if ((int)P->part_keys.size() < kPartSlots)
+    P->part_keys.push_back(key);
+  else
+    P->part_keys[slot] = key;
+  *d_part_out = d;
   return RAP_OK;
 }
 
@@ -1154,7 +1179,8 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
   const int64_t n_dense = P->dprogs.empty() ? 0 : (int64_t)P->dprogs.size() * ((drows + kDenseBlockRows - 1) / kDenseBlockRows);
   if (n_sparse_tiles == 0 && n_dense == 0) return RAP_OK;
   const int64_t grid = std::min<int64_t>((int64_t)P->budget * P->ctas_per_sm, kMaxCtas);
-  rap_status pst = update_partition(P, B, raw->sp_nnz, n_sparse_tiles, n_dense, (int)grid, stream);
+  const int64_t* d_part = nullptr;
+  rap_status pst = update_partition(P, B, raw->sp_nnz, n_sparse_tiles, n_dense, (int)grid, stream, &d_part);
   if (pst != RAP_OK) return pst;
   Common c{};
   c.ops = reinterpret_cast<const DevOp*>(P->blob + P->off_ops);
@@ -1173,7 +1199,7 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
   c.n_dense_rows = drows;
   c.chain = (out->flags & RAP_OUT_CHAIN) ? 1 : 0;
   c.sched = P->d_sched;
-  c.part = P->d_part;
+  c.part = d_part;
   c.agg = P->d_agg;
   c.dense_out = out->dense_out;
   c.ld = out->dense_ld;
