@@ -169,6 +169,9 @@ __device__ __forceinline__ void cp_async16(void* dst, const void* src) {
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
 }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait_group() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 
 __device__ __forceinline__ unsigned long long ld_relaxed(const unsigned long long* p) {
   unsigned long long v;
@@ -877,6 +880,12 @@ __device__ __noinline__ long long value_chunk_canon(const P& p, const FeatCtx& f
 }
 
 constexpr int kNullRow = INT_MIN;
+#ifndef RAP_MULTI_DEPTH
+#define RAP_MULTI_DEPTH 3
+#endif
+constexpr int kMultiDepth = RAP_MULTI_DEPTH;  // id windows in flight (ring of 4)
+static_assert(kMultiDepth >= 1 && kMultiDepth <= 3, "ring of 4 window slots");
+static_assert(1568 + 4 * 128 * 8 <= kWarpScr, "multi-id tile scratch");
 // Tile rt of a canonical chain whose rows may hold several ids (multi-hot,
 // FirstX caps): element-parallel.  Offsets / validity staged with cp.async;
 // per row its output start goes to shared memory; each 128-element window of
@@ -940,7 +949,15 @@ __device__ __noinline__ long long value_tile_multi(const P& p, const FeatCtx& fc
   int64_t* values = p.c.values;
   const long long cap = p.c.values_cap;
   int carry = 0;  // row of the last element of the previous window
-  for (int eb = 0; eb < T; eb += 128) {
+  // Window w (elements w*128 ..): mark the rows starting in it, give each of
+  // the lane's 4 elements its row and cp.async its id into ring slot w % 4
+  // (a filled null row stores the fill id); act/full masks kept in registers,
+  // 8 bits per slot.  kMultiDepth windows are in flight while one is computed.
+  int64_t* ring = reinterpret_cast<int64_t*>(wscr + 1568);  // [4][128]
+  uint32_t masks = 0;
+  const int nwin = (T + 127) >> 7;
+  auto issue = [&](int w) {
+    const int eb = w * 128;
     *reinterpret_cast<int4*>(mark + lr0) = make_int4(-1, -1, -1, -1);
     __syncwarp();
 #pragma unroll
@@ -949,8 +966,8 @@ __device__ __noinline__ long long value_tile_multi(const P& p, const FeatCtx& fc
       if (l[k] > 0 && st >= 0 && st < 128) mark[st] = lr0 + k;
     }
     __syncwarp();
-    int64_t x[4];
     unsigned act = 0, full = 0;
+    int64_t* slot = ring + (w & 3) * 128;
 #pragma unroll
     for (int u = 0; u < 4; ++u) {
       // row of element eb + 32u + lane: the last row starting at or before it
@@ -967,16 +984,38 @@ __device__ __noinline__ long long value_tile_multi(const P& p, const FeatCtx& fc
       const bool va = in && dlt != kNullRow;
       act |= (in ? 1u : 0u) << u;
       full |= (va ? 1u : 0u) << u;
-      x[u] = va ? __ldg(val + (ee + dlt)) : fc.fill;
+      if (va)
+        cp_async8(slot + 32 * u + lane, val + (ee + dlt));
+      else
+        slot[32 * u + lane] = fc.fill;
     }
+    masks = (masks & ~(0xffu << (8 * (w & 3)))) | ((act | (full << 4)) << (8 * (w & 3)));
+    __syncwarp();  // marks are rebuilt by the next window
+  };
+  for (int w = 0; w < kMultiDepth && w < nwin; ++w) {
+    issue(w);
+    cp_async_commit();
+  }
+  for (int w = 0; w < nwin; ++w) {
+    if (w + kMultiDepth < nwin) issue(w + kMultiDepth);
+    cp_async_commit();  // (possibly empty) keeps one group per window
+    cp_async_wait_group<kMultiDepth>();
+    const unsigned mk = (masks >> (8 * (w & 3))) & 0xffu;
+    const unsigned act = mk & 15u, full = mk >> 4;
+    const int64_t* slot = ring + (w & 3) * 128;
+    int64_t x[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) x[u] = slot[32 * u + lane];  // this lane's own copies
     canon_apply_n<4>(fc.q, p.c.itab, x, act, full);
+    const int eb = w * 128;
 #pragma unroll
     for (int u = 0; u < 4; ++u) {
       const long long pos = base + eb + 32 * u + lane;
       if (((act >> u) & 1u) && pos < cap) values[pos] = x[u];
     }
-    __syncwarp();
   }
+  cp_async_wait_all();
+  __syncwarp();
   return T;
 }
 
