@@ -992,9 +992,9 @@ __device__ __noinline__ long long value_tile_multi(const P& p, const FeatCtx& fc
     masks = (masks & ~(0xffu << (8 * (w & 3)))) | ((act | (full << 4)) << (8 * (w & 3)));
     __syncwarp();  // marks are rebuilt by the next window
   };
-  for (int w = 0; w < kMultiDepth && w < nwin; ++w) {
-    issue(w);
-    cp_async_commit();
+  for (int w = 0; w < kMultiDepth; ++w) {  // exactly kMultiDepth groups (some empty),
+    if (w < nwin) issue(w);                  // so wait_group<kMultiDepth> below
+    cp_async_commit();                       // always covers window w
   }
   for (int w = 0; w < nwin; ++w) {
     if (w + kMultiDepth < nwin) issue(w + kMultiDepth);
