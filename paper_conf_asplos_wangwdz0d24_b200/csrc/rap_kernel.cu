@@ -113,6 +113,7 @@ __device__ __forceinline__ void trace_stamp(const Common& c, int k) {
 // Profiling aid: clock64 at slot k of this CTA's trace row, once per launch
 // (first call wins), after the value `dep` is available.
 // Compiled in only with -DRAP_TRACE_CLK (dev builds, scripts/trace.py).
+__shared__ unsigned long long s_clk[24];  // trace_clk stamps of this CTA (flushed at kernel end)
 __device__ __forceinline__ void trace_clk(const Common& c, int k, long long dep) {
 #ifndef RAP_TRACE_CLK
   (void)c;
@@ -120,10 +121,9 @@ __device__ __forceinline__ void trace_clk(const Common& c, int k, long long dep)
   (void)dep;
   if (false)
 #endif
-  if (c.trace != nullptr && threadIdx.x == 0 && (int64_t)blockIdx.x < c.trace_cap) {
+  if (c.trace != nullptr && threadIdx.x == 0) {
     asm volatile("" ::"l"(dep));
-    unsigned long long* slot = c.trace + (int64_t)blockIdx.x * kTracePts + k;
-    if (*slot == 0) *slot = clock64();
+    if (s_clk[k] == 0) s_clk[k] = clock64();  // shared: no global round trip inside the timed span
   }
 }
 
@@ -1321,15 +1321,19 @@ __device__ __noinline__ long long ngram_tile_fast(const P& p, int f, int64_t rt,
   for (int j = 0; j < 4; ++j)
     if (j < k) {
       const Chain& sc = G.src[j];
+      const int xc = (int)min(sc.xcap, (int64_t)INT32_MAX);
+      const int nl = sc.has_fill ? (int)min((int64_t)1, sc.null_xcap) : 0;  // R10 / R14
+      const int32_t* so = soff + j * kNgStageOff;
+      const int lr0 = 4 * lane;
+      const int4 a = *reinterpret_cast<const int4*>(so + lr0);  // 16-byte aligned rows
+      const int a4 = so[lr0 + 4];
+      const unsigned vb = (sbm[4 * j + (lr0 >> 5)] >> (lr0 & 31)) & 15u;
+      const int d[4] = {a.y - a.x, a.z - a.y, a.w - a.z, a4 - a.w};
 #pragma unroll
       for (int kk = 0; kk < 4; ++kk) {
-        const int lr = 4 * lane + kk;
-        int l = 0;
-        bool fu = false;
-        if (lr < NR) {
-          l = len_s(soff + j * kNgStageOff, sbm + 4 * j, lr, sc.xcap, sc.has_fill, sc.null_xcap);
-          fu = (sbm[4 * j + (lr >> 5)] >> (lr & 31)) & 1u;
-        }
+        const bool in = lr0 + kk < NR;
+        const bool fu = in && ((vb >> kk) & 1u);
+        const int l = !in ? 0 : (fu ? min(max(d[kk], 0), xc) : nl);  // R5 FirstX cap
         ok &= l <= 1;
         pn[kk] += l;
         l1 |= (l == 1 ? 1u : 0u) << (4 * j + kk);
@@ -1683,6 +1687,40 @@ __device__ __noinline__ void dense_block(const P& p, int gi, int64_t rb, unsigne
       }
     }
     const bool has_bm = p.dvalid[src_col] != nullptr;
+    // specialised unit: a staged dense column through [FillNull] [Logit |
+    // BoxCox] (the Criteo chains): one uniform dispatch per unit, none per row
+    {
+      const bool f0 = okind[0] == OK_FILL_F;
+      const int t = f0 ? okind[1] : okind[0];
+      const int rest = f0 ? okind[2] : okind[1];
+      const int tp = f0 ? 1 : 0;
+      if (staged && kind == U_DENSE && reg_ops && rest < 0 && (t < 0 || t == OK_LOGIT || t == OK_BOXCOX)) {
+        const float fill = of0[0], a = of0[tp], b = of1[tp];
+        const float* xin = din + slot * kDenseBlockRows;
+        const uint32_t* bmp = dbm + slot * 8;
+        float* tc = tile + col;
+        auto in = [&](int r) -> float {  // R14 null -> NaN, then R10
+          const uint32_t w = has_bm ? bmp[r >> 5] : 0xffffffffu;
+          float x = ((w >> (r & 31)) & 1u) ? xin[r] : __int_as_float(0x7fc00000);
+          if (f0 && isnan(x)) x = fill;
+          return x;
+        };
+        if (t == OK_LOGIT) {  // R11
+          for (int r = lane; r < nr; r += 32) {
+            const float x = in(r);
+            const float z = x < a ? a : (x > b ? b : x);
+            tc[r * LD] = logf(__fdiv_rn(z, __fsub_rn(1.0f, z)));
+          }
+        } else if (t == OK_BOXCOX && a == 0.0f) {  // R12, lambda = 0
+          for (int r = lane; r < nr; r += 32) tc[r * LD] = logf(in(r));
+        } else if (t == OK_BOXCOX) {  // R12
+          for (int r = lane; r < nr; r += 32) tc[r * LD] = __fdiv_rn(expm1f(__fmul_rn(a, logf(in(r)))), a);
+        } else {
+          for (int r = lane; r < nr; r += 32) tc[r * LD] = in(r);
+        }
+        continue;
+      }
+    }
     const float* uft = un.gops ? p.c.ftab : dp->ftab;
     for (int r = lane; r < nr; r += 32) {
       float x;
@@ -1791,6 +1829,9 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
   // buffer; every offset and value position of this launch starts there (the
   // first tile rewrites offsets[0] with the same value)
   const long long chain0 = p.c.chain ? (long long)__ldg(p.c.offsets) : 0ll;
+#ifdef RAP_TRACE_CLK
+  if (tid < 24) s_clk[tid] = 0;
+#endif
   if (tid == 0) {
     mbar_init(&cs.bar, 1);
     cs.phase = 0;
@@ -1963,6 +2004,11 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
   }
   trace_stamp(p.c, 4);
 
+#ifdef RAP_TRACE_CLK
+  __syncthreads();
+  if (p.c.trace != nullptr && tid >= 8 && tid < 24 && (int64_t)blockIdx.x < p.c.trace_cap)
+    p.c.trace[(int64_t)blockIdx.x * kTracePts + tid] = s_clk[tid];
+#endif
   // The last CTA out resets the rank counter and advances the epoch of the
   // aggregate words (clearing them when the 20-bit epoch wraps), so launch
   // parameters are identical from call to call (CUDA-graph replayable).

@@ -1178,7 +1178,11 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
   rap_shard_rows(B, P->rank, P->world, &drow0, &drows);
   const int64_t n_dense = P->dprogs.empty() ? 0 : (int64_t)P->dprogs.size() * ((drows + kDenseBlockRows - 1) / kDenseBlockRows);
   if (n_sparse_tiles == 0 && n_dense == 0) return RAP_OK;
-  const int64_t grid = std::min<int64_t>((int64_t)P->budget * P->ctas_per_sm, kMaxCtas);
+  // grid: the budget's CTA slots, but no more CTAs than there is work for
+  // (a warp per sparse tile, a CTA per dense block): small batches then pay
+  // a shorter aggregate chain and fewer idle CTAs
+  const int64_t want = std::max<int64_t>(1, std::max<int64_t>(n_dense, (n_sparse_tiles + kWarpsPerCta - 1) / kWarpsPerCta));
+  const int64_t grid = std::min<int64_t>(std::min<int64_t>((int64_t)P->budget * P->ctas_per_sm, kMaxCtas), want);
   const int64_t* d_part = nullptr;
   rap_status pst = update_partition(P, B, raw->sp_nnz, n_sparse_tiles, n_dense, (int)grid, stream, &d_part);
   if (pst != RAP_OK) return pst;
