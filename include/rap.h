@@ -190,6 +190,15 @@ rap_status rap_preprocess(rap_plan* plan, const rap_raw_batch* raw, const rap_ou
  * offsets[end] are unspecified. */
 rap_status rap_preprocess_host(rap_plan* plan, const rap_raw_batch* raw, const rap_output* out, void* stream);
 
+/* rap_preprocess_host without the final synchronisation: H2D copies, the
+ * launch and the D2H copies are enqueued on `stream` and the call returns.
+ * The host buffers must stay alive and unmodified, and the outputs are valid,
+ * once the stream reaches this point.  The plan's device staging is reused by
+ * its next call, so use one plan per stream in flight: with two plans on two
+ * streams, batch i+1's H2D copies and kernel overlap batch i's D2H copies
+ * (inter-batch pipelining, §6.3). */
+rap_status rap_preprocess_host_async(rap_plan* plan, const rap_raw_batch* raw, const rap_output* out, void* stream);
+
 /* Change the SM budget for the next rap_preprocess (resource-aware sharding,
  * L1351-1366).  sm_budget in [1, #SMs]; 0 = all SMs. */
 rap_status rap_set_budget(rap_plan* plan, int32_t sm_budget);

@@ -392,9 +392,19 @@ __device__ __forceinline__ void canon_apply_n(const Canon& q, const int64_t* ita
     map_lookup_n<N>(itab, q.map_a, q.map_m, q.map_def, v, (q.null_mask & CB_MAPID) ? act : (act & full));
   if (q.mask & CB_SIGRID) {  // R3
     const unsigned on = (q.null_mask & CB_SIGRID) ? act : (act & full);
+    if (((uint64_t)q.M >> 32) == 0) {  // warp-uniform: the 64x32 multiply-high path for the whole batch
+      const uint64_t m = (uint64_t)q.M;
 #pragma unroll
-    for (int j = 0; j < N; ++j)
-      if ((on >> j) & 1u) v[j] = (int64_t)reduce_M(splitmix_H(q.hs ^ (uint64_t)v[j]), q.M);
+      for (int j = 0; j < N; ++j)
+        if ((on >> j) & 1u) {
+          const uint64_t h = splitmix_H(q.hs ^ (uint64_t)v[j]);
+          v[j] = (int64_t)(((uint64_t)(uint32_t)(h >> 32) * m + (((uint64_t)(uint32_t)h * m) >> 32)) >> 32);
+        }
+    } else {
+#pragma unroll
+      for (int j = 0; j < N; ++j)
+        if ((on >> j) & 1u) v[j] = (int64_t)__umul64hi(splitmix_H(q.hs ^ (uint64_t)v[j]), (uint64_t)q.M);
+    }
   }
   if (q.mask & CB_BUCKET)  // R4
     upper_bound_n<N>(itab + q.bk_a, q.bk_m, v, (q.null_mask & CB_BUCKET) ? act : (act & full));

@@ -1257,7 +1257,8 @@ static rap_status stage_buf(rap_plan* P, size_t slot, size_t bytes, void** ptr) 
   return RAP_OK;
 }
 
-rap_status rap_preprocess_host(rap_plan* P, const rap_raw_batch* raw, const rap_output* out, void* stream_v) {
+static rap_status preprocess_host_impl(rap_plan* P, const rap_raw_batch* raw, const rap_output* out, void* stream_v,
+                                       bool sync) {
   rap_status st = check_batch(P, raw, out);
   if (st != RAP_OK) return st;
   DeviceGuard dg(P->device);
@@ -1341,9 +1342,18 @@ rap_status rap_preprocess_host(rap_plan* P, const rap_raw_batch* raw, const rap_
       e = cudaMemcpyAsync(out->values, dv, sizeof(int64_t) * vb, cudaMemcpyDeviceToHost, stream);
     if (e != cudaSuccess) return cuda_fail(e, "D2H sparse");
   }
+  if (!sync) return RAP_OK;
   e = cudaStreamSynchronize(stream);
   if (e != cudaSuccess) return cuda_fail(e, "cudaStreamSynchronize");
   return RAP_OK;
+}
+
+rap_status rap_preprocess_host(rap_plan* P, const rap_raw_batch* raw, const rap_output* out, void* stream) {
+  return preprocess_host_impl(P, raw, out, stream, true);
+}
+
+rap_status rap_preprocess_host_async(rap_plan* P, const rap_raw_batch* raw, const rap_output* out, void* stream) {
+  return preprocess_host_impl(P, raw, out, stream, false);
 }
 
 rap_status rap_predict_latency_us(const rap_plan* P, int64_t n_rows, const int64_t* sp_nnz, int32_t sm_budget,

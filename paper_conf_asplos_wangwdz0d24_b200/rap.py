@@ -19,7 +19,7 @@ OPS = {"fillnull": 0, "logit": 1, "boxcox": 2, "onehot": 3, "sigridhash": 4,
 STATUS = {0: "OK", 1: "INVALID_ARGUMENT", 2: "INVALID_GRAPH", 3: "INVALID_PARAM", 4: "CAPACITY",
           5: "UNSUPPORTED", 6: "CUDA", 7: "OUT_OF_MEMORY"}
 
-EXPORTS = ["rap_plan_create", "rap_plan_output_shape", "rap_preprocess", "rap_preprocess_host", "rap_set_budget",
+EXPORTS = ["rap_plan_create", "rap_plan_output_shape", "rap_preprocess", "rap_preprocess_host", "rap_preprocess_host_async", "rap_set_budget",
            "rap_predict_latency_us", "rap_choose_budget", "rap_plan_info_get", "rap_debug_trace", "rap_plan_destroy",
            "rap_status_string", "rap_last_error", "rap_shard_rows", "rap_plan_output_costs", "rap_place",
            "rap_plan_create_sharded", "rap_jagged_append"]
@@ -100,6 +100,8 @@ def load(build_if_stale: bool = False):
     L.rap_preprocess.argtypes = [P, C.POINTER(RapRawBatch), C.POINTER(RapOutput), P]
     L.rap_preprocess_host.restype = C.c_int
     L.rap_preprocess_host.argtypes = [P, C.POINTER(RapRawBatch), C.POINTER(RapOutput), P]
+    L.rap_preprocess_host_async.restype = C.c_int
+    L.rap_preprocess_host_async.argtypes = [P, C.POINTER(RapRawBatch), C.POINTER(RapOutput), P]
     L.rap_set_budget.restype = C.c_int
     L.rap_set_budget.argtypes = [P, C.c_int32]
     L.rap_predict_latency_us.restype = C.c_int
@@ -353,6 +355,11 @@ class Plan:
         """raw / out built with pin=True (host buffers); synchronises the stream."""
         _check(load().rap_preprocess_host(self.handle, C.byref(raw.struct), C.byref(out.struct),
                                           _stream_handle(stream)))
+
+    def preprocess_host_async(self, raw: DeviceBatch, out: DeviceOutput, stream=None):
+        """Host buffers (pin=True); enqueue only — sync the stream before reading out."""
+        _check(load().rap_preprocess_host_async(self.handle, C.byref(raw.struct), C.byref(out.struct),
+                                                _stream_handle(stream)))
 
     def set_budget(self, sm_budget: int):
         _check(load().rap_set_budget(self.handle, sm_budget))

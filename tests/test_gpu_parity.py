@@ -226,6 +226,25 @@ def test_host_buffers_entry(env):
     plan.close()
 
 
+def test_host_async_two_plans_pipelined(env):
+    """rap_preprocess_host_async: two plans on two streams, batches alternating,
+    each result equal to the oracle once its stream is synchronised."""
+    rap, synth, oracle, torch = env
+    w = synth.c2_terabyte(0)
+    hosts = [synth.make_batch(w, 3000 + 100 * i, seed=40 + i) for i in range(4)]
+    plans = [rap.Plan(w.spec, device=0), rap.Plan(w.spec, device=0)]
+    streams = [torch.cuda.Stream(), torch.cuda.Stream()]
+    raws = [rap.DeviceBatch(h, None, pin=True) for h in hosts]
+    outs = [rap.DeviceOutput(plans[i % 2], h["n_rows"], raws[i].sp_nnz, None, pin=True) for i, h in enumerate(hosts)]
+    for i in range(4):
+        plans[i % 2].preprocess_host_async(raws[i], outs[i], streams[i % 2])
+    torch.cuda.synchronize()
+    for i in range(4):
+        assert_parity(outs[i].to_numpy(), oracle.run(w.spec, hosts[i]), ctx=f"batch {i}")
+    for p_ in plans:
+        p_.close()
+
+
 def test_capacity_error(env):
     rap, synth, oracle, torch = env
     w = synth.c1_kaggle(0)
