@@ -377,38 +377,58 @@ __device__ __forceinline__ void upper_bound_n(const int64_t* b, int m, int64_t (
 template <int N>
 __device__ __forceinline__ void canon_apply_n(const Canon& q, const int64_t* itab, int64_t (&v)[N], unsigned act,
                                               unsigned full) {
-  // element j runs stage X iff act bit j and (full bit j or X in null_mask)
-  const unsigned nul = act & ~full;
-  if (q.mask & CB_CLAMP) {  // R6
-    const unsigned on = (q.null_mask & CB_CLAMP) ? act : (act & full);
+  // element j runs stage X iff act bit j and (full bit j or X in null_mask).
+  // Stage parameters are read once into registers; when every element runs
+  // a stage (the steady state: full windows, FillNull first) the stage is
+  // straight-line code with no per-element predicate or branch.
+  constexpr unsigned kAll = N >= 32 ? 0xffffffffu : ((1u << N) - 1u);
+  const int mask = q.mask, nmask = q.null_mask;
+  if (mask & CB_CLAMP) {  // R6
+    const int64_t lo = q.lo, hi = q.hi;
+    const unsigned on = (nmask & CB_CLAMP) ? act : (act & full);
+    if (on == kAll) {
 #pragma unroll
-    for (int j = 0; j < N; ++j)
-      if ((on >> j) & 1u) {
-        v[j] = v[j] < q.lo ? q.lo : v[j];
-        v[j] = v[j] > q.hi ? q.hi : v[j];
+      for (int j = 0; j < N; ++j) {
+        v[j] = v[j] < lo ? lo : v[j];
+        v[j] = v[j] > hi ? hi : v[j];
       }
-  }
-  if (q.mask & CB_MAPID)  // R8
-    map_lookup_n<N>(itab, q.map_a, q.map_m, q.map_def, v, (q.null_mask & CB_MAPID) ? act : (act & full));
-  if (q.mask & CB_SIGRID) {  // R3
-    const unsigned on = (q.null_mask & CB_SIGRID) ? act : (act & full);
-    if (((uint64_t)q.M >> 32) == 0) {  // warp-uniform: the 64x32 multiply-high path for the whole batch
-      const uint64_t m = (uint64_t)q.M;
-#pragma unroll
-      for (int j = 0; j < N; ++j)
-        if ((on >> j) & 1u) {
-          const uint64_t h = splitmix_H(q.hs ^ (uint64_t)v[j]);
-          v[j] = (int64_t)(((uint64_t)(uint32_t)(h >> 32) * m + (((uint64_t)(uint32_t)h * m) >> 32)) >> 32);
-        }
     } else {
 #pragma unroll
       for (int j = 0; j < N; ++j)
-        if ((on >> j) & 1u) v[j] = (int64_t)__umul64hi(splitmix_H(q.hs ^ (uint64_t)v[j]), (uint64_t)q.M);
+        if ((on >> j) & 1u) {
+          v[j] = v[j] < lo ? lo : v[j];
+          v[j] = v[j] > hi ? hi : v[j];
+        }
     }
   }
-  if (q.mask & CB_BUCKET)  // R4
-    upper_bound_n<N>(itab + q.bk_a, q.bk_m, v, (q.null_mask & CB_BUCKET) ? act : (act & full));
-  (void)nul;
+  if (mask & CB_MAPID)  // R8
+    map_lookup_n<N>(itab, q.map_a, q.map_m, q.map_def, v, (nmask & CB_MAPID) ? act : (act & full));
+  if (mask & CB_SIGRID) {  // R3
+    const unsigned on = (nmask & CB_SIGRID) ? act : (act & full);
+    const uint64_t hs = q.hs, M = (uint64_t)q.M;
+    if ((M >> 32) == 0) {  // warp-uniform: the 64x32 multiply-high path for the whole batch
+      if (on == kAll) {
+#pragma unroll
+        for (int j = 0; j < N; ++j) {
+          const uint64_t h = splitmix_H(hs ^ (uint64_t)v[j]);
+          v[j] = (int64_t)(((uint64_t)(uint32_t)(h >> 32) * M + (((uint64_t)(uint32_t)h * M) >> 32)) >> 32);
+        }
+      } else {
+#pragma unroll
+        for (int j = 0; j < N; ++j)
+          if ((on >> j) & 1u) {
+            const uint64_t h = splitmix_H(hs ^ (uint64_t)v[j]);
+            v[j] = (int64_t)(((uint64_t)(uint32_t)(h >> 32) * M + (((uint64_t)(uint32_t)h * M) >> 32)) >> 32);
+          }
+      }
+    } else {
+#pragma unroll
+      for (int j = 0; j < N; ++j)
+        if ((on >> j) & 1u) v[j] = (int64_t)__umul64hi(splitmix_H(hs ^ (uint64_t)v[j]), M);
+    }
+  }
+  if (mask & CB_BUCKET)  // R4
+    upper_bound_n<N>(itab + q.bk_a, q.bk_m, v, (nmask & CB_BUCKET) ? act : (act & full));
 }
 
 // One element through the canonical pipeline (not inlined: cold paths).
@@ -895,21 +915,27 @@ constexpr int kNullRow = INT_MIN;
 #endif
 constexpr int kMultiDepth = RAP_MULTI_DEPTH;  // id windows in flight (ring of 4)
 static_assert(kMultiDepth >= 1 && kMultiDepth <= 3, "ring of 4 window slots");
-static_assert(1568 + 4 * 128 * 8 <= kWarpScr, "multi-id tile scratch");
+constexpr int kMultiRing = 1584;  // byte offset of the id ring in the warp scratch
+static_assert(kMultiRing + 4 * 128 * 8 <= kWarpScr, "multi-id tile scratch");
 // Tile rt of a canonical chain whose rows may hold several ids (multi-hot,
-// FirstX caps): element-parallel.  Offsets / validity staged with cp.async;
-// per row its output start goes to shared memory; each 128-element window of
-// the tile's output marks the rows that start in it and a warp max-scan gives
-// every element its row (elements e = eb + 32u + lane, so id loads and value
-// stores are coalesced).  Element e of row r reads input soff[r] + (e -
-// out_start[r]) (FirstX keeps a prefix, R5) or the fill id of a null row (R10).
+// FirstX caps): element-parallel.  Offsets / validity staged with cp.async.
+// Output element e of a valid row r reads input e + delta_r, delta_r =
+// soff[r] - out_start[r] (FirstX keeps a prefix, R5); a filled null row
+// (R10) emits the fill id.  delta is constant over runs of consecutive valid
+// rows that FirstX does not truncate, so the tile keeps only its *change
+// points* (output position where delta changes, or a filled null's element)
+// in shared memory: ~10 per 128 multi-hot rows instead of one per row.  Each
+// 128-element window of the output (e = window + 32u + lane: coalesced id
+// loads and value stores) takes the delta of the last change point at or
+// before its start, then applies the few change points inside the window;
+// ids are cp.async-staged into a 4-slot ring with kMultiDepth windows in
+// flight.
 template <class P>
 __device__ __noinline__ long long value_tile_multi(const P& p, const FeatCtx& fc, int64_t rt, int lane, long long base,
                                                    unsigned char* wscr) {
-  int32_t* soff = reinterpret_cast<int32_t*>(wscr);             // [132]
-  uint32_t* sbm = reinterpret_cast<uint32_t*>(wscr + 528);       // [4]
-  int32_t* sdelta = reinterpret_cast<int32_t*>(wscr + 544);     // [128] input index - output index of a row
-  int32_t* mark = reinterpret_cast<int32_t*>(wscr + 1056);      // [128] row starting at window slot
+  int32_t* soff = reinterpret_cast<int32_t*>(wscr);        // [132]
+  uint32_t* sbm = reinterpret_cast<uint32_t*>(wscr + 528);  // [4]
+  int2* cps = reinterpret_cast<int2*>(wscr + 544);          // [128] change points (position, delta)
   const int f = fc.f;
   const int64_t B = p.c.n_rows;
   const int64_t R0 = rt * kTileRows;
@@ -923,11 +949,13 @@ __device__ __noinline__ long long value_tile_multi(const P& p, const FeatCtx& fc
   const int lr0 = 4 * lane;
   int l[4], e[4], tot = 0;
   unsigned vbits = 0;
+  int a[4];
   {
-    const int4 a = *reinterpret_cast<const int4*>(soff + lr0);
+    const int4 q = *reinterpret_cast<const int4*>(soff + lr0);
     const int a4 = soff[lr0 + 4];
+    a[0] = q.x, a[1] = q.y, a[2] = q.z, a[3] = q.w;
     vbits = (sbm[lr0 >> 5] >> (lr0 & 31)) & 15u;
-    const int d[4] = {a.y - a.x, a.z - a.y, a.w - a.z, a4 - a.w};
+    const int d[4] = {q.y - q.x, q.z - q.y, q.w - q.z, a4 - q.w};
 #pragma unroll
     for (int k = 0; k < 4; ++k) {
       const bool in = lr0 + k < NR;
@@ -940,13 +968,6 @@ __device__ __noinline__ long long value_tile_multi(const P& p, const FeatCtx& fc
   const int incl = warp_incl_scan(tot, lane);
   const int L = incl - tot;
   const int T = __shfl_sync(0xffffffffu, incl, 31);
-  {
-    // element ee of row r reads input ee + sdelta[r]; kNullRow: a filled null row
-    int dl[4];
-#pragma unroll
-    for (int k = 0; k < 4; ++k) dl[k] = ((vbits >> k) & 1u) ? soff[lr0 + k] - (L + e[k]) : kNullRow;
-    *reinterpret_cast<int4*>(sdelta + lr0) = make_int4(dl[0], dl[1], dl[2], dl[3]);
-  }
   const long long lb = base + L;
   store_quad(p.c.lengths + (int64_t)f * B + R0 + lr0, p.c.offsets + (int64_t)f * B + R0 + lr0, R0 + lr0, B, l, lb,
              e);
@@ -954,53 +975,65 @@ __device__ __noinline__ long long value_tile_multi(const P& p, const FeatCtx& fc
     p.c.offsets[(int64_t)p.c.n_sparse_out * B] = base + T;  // total, R17
     if (base + T > p.c.values_cap) atomicExch(p.c.err, 1);
   }
+  // change points: a producing row whose delta differs from the previous
+  // row's, follows a row that emits nothing, or is a filled null
+  int nc = 0;
+  {
+    int eff[4];
+#pragma unroll
+    for (int k = 0; k < 4; ++k) eff[k] = ((vbits >> k) & 1u) ? a[k] - (L + e[k]) : kNullRow;
+    int pe = __shfl_up_sync(0xffffffffu, eff[3], 1), pl = __shfl_up_sync(0xffffffffu, l[3], 1);
+    if (lane == 0) pl = 0;
+    unsigned cpm = 0;
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      const bool c = l[k] > 0 && (pl == 0 || eff[k] != pe || eff[k] == kNullRow);
+      cpm |= (c ? 1u : 0u) << k;
+      pe = eff[k];
+      pl = l[k];
+    }
+    const int cnt = __popc(cpm);
+    const int ci = warp_incl_scan(cnt, lane);
+    nc = __shfl_sync(0xffffffffu, ci, 31);
+    int w = ci - cnt;
+#pragma unroll
+    for (int k = 0; k < 4; ++k)
+      if ((cpm >> k) & 1u) cps[w++] = make_int2(L + e[k], eff[k]);
+  }
   __syncwarp();
   const int64_t* val = p.val[src];
   int64_t* values = p.c.values;
   const long long cap = p.c.values_cap;
-  int carry = 0;  // row of the last element of the previous window
-  // Window w (elements w*128 ..): mark the rows starting in it, give each of
-  // the lane's 4 elements its row and cp.async its id into ring slot w % 4
-  // (a filled null row stores the fill id); act/full masks kept in registers,
-  // 8 bits per slot.  kMultiDepth windows are in flight while one is computed.
-  int64_t* ring = reinterpret_cast<int64_t*>(wscr + 1568);  // [4][128]
+  int64_t* ring = reinterpret_cast<int64_t*>(wscr + kMultiRing);  // [4][128]
   uint32_t masks = 0;
   const int nwin = (T + 127) >> 7;
+  int cur = 0;  // last change point at or before the window start (warp-uniform)
   auto issue = [&](int w) {
     const int eb = w * 128;
-    *reinterpret_cast<int4*>(mark + lr0) = make_int4(-1, -1, -1, -1);
-    __syncwarp();
+    while (cur + 1 < nc && cps[cur + 1].x <= eb) ++cur;
+    const int d0 = cps[cur].y;
+    int dd[4] = {d0, d0, d0, d0};
+    for (int j = cur + 1; j < nc; ++j) {  // change points inside the window (few)
+      const int2 c = cps[j];
+      if (c.x >= eb + 128) break;
 #pragma unroll
-    for (int k = 0; k < 4; ++k) {
-      const int st = L + e[k] - eb;
-      if (l[k] > 0 && st >= 0 && st < 128) mark[st] = lr0 + k;
+      for (int u = 0; u < 4; ++u) dd[u] = c.x <= eb + 32 * u + lane ? c.y : dd[u];
     }
-    __syncwarp();
     unsigned act = 0, full = 0;
     int64_t* slot = ring + (w & 3) * 128;
 #pragma unroll
     for (int u = 0; u < 4; ++u) {
-      // row of element eb + 32u + lane: the last row starting at or before it
-      const int m = mark[32 * u + lane];
-      const unsigned starts = __ballot_sync(0xffffffffu, m >= 0);
-      const unsigned le = starts & (0xffffffffu >> (31 - lane));
-      const int from = le ? 31 - __clz(le) : 0;
-      const int got = __shfl_sync(0xffffffffu, m, from);
-      const int r = le ? got : carry;
-      carry = __shfl_sync(0xffffffffu, r, 31);
       const int ee = eb + 32 * u + lane;
       const bool in = ee < T;
-      const int dlt = sdelta[r];
-      const bool va = in && dlt != kNullRow;
+      const bool va = in && dd[u] != kNullRow;
       act |= (in ? 1u : 0u) << u;
       full |= (va ? 1u : 0u) << u;
       if (va)
-        cp_async8(slot + 32 * u + lane, val + (ee + dlt));
+        cp_async8(slot + 32 * u + lane, val + (ee + dd[u]));
       else
         slot[32 * u + lane] = fc.fill;
     }
     masks = (masks & ~(0xffu << (8 * (w & 3)))) | ((act | (full << 4)) << (8 * (w & 3)));
-    __syncwarp();  // marks are rebuilt by the next window
   };
   for (int w = 0; w < kMultiDepth; ++w) {  // exactly kMultiDepth groups (some empty),
     if (w < nwin) issue(w);                  // so wait_group<kMultiDepth> below
@@ -1017,10 +1050,10 @@ __device__ __noinline__ long long value_tile_multi(const P& p, const FeatCtx& fc
 #pragma unroll
     for (int u = 0; u < 4; ++u) x[u] = slot[32 * u + lane];  // this lane's own copies
     canon_apply_n<4>(fc.q, p.c.itab, x, act, full);
-    const int eb = w * 128;
+    const long long pos0 = base + w * 128 + lane;
 #pragma unroll
     for (int u = 0; u < 4; ++u) {
-      const long long pos = base + eb + 32 * u + lane;
+      const long long pos = pos0 + 32 * u;
       if (((act >> u) & 1u) && pos < cap) values[pos] = x[u];
     }
   }
