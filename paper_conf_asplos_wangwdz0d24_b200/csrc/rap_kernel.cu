@@ -1007,31 +1007,46 @@ __device__ __noinline__ long long value_tile_multi(const P& p, const FeatCtx& fc
   int64_t* ring = reinterpret_cast<int64_t*>(wscr + kMultiRing);  // [4][128]
   uint32_t masks = 0;
   const int nwin = (T + 127) >> 7;
-  int cur = 0;  // last change point at or before the window start (warp-uniform)
+  // cur: last change point at or before the window start; nxp: position of
+  // the next one (INT_MAX: none) -- warp-uniform, kept in registers
+  int cur = 0, nxp = nc > 1 ? cps[1].x : INT_MAX;
   auto issue = [&](int w) {
     const int eb = w * 128;
-    while (cur + 1 < nc && cps[cur + 1].x <= eb) ++cur;
+    while (nxp <= eb) {
+      ++cur;
+      nxp = cur + 1 < nc ? cps[cur + 1].x : INT_MAX;
+    }
     const int d0 = cps[cur].y;
     int dd[4] = {d0, d0, d0, d0};
-    for (int j = cur + 1; j < nc; ++j) {  // change points inside the window (few)
-      const int2 c = cps[j];
-      if (c.x >= eb + 128) break;
+    const bool inner = nxp < eb + 128;  // a change point inside the window
+    if (inner)
+      for (int j = cur + 1; j < nc; ++j) {  // (few)
+        const int2 c = cps[j];
+        if (c.x >= eb + 128) break;
 #pragma unroll
-      for (int u = 0; u < 4; ++u) dd[u] = c.x <= eb + 32 * u + lane ? c.y : dd[u];
-    }
+        for (int u = 0; u < 4; ++u) dd[u] = c.x <= eb + 32 * u + lane ? c.y : dd[u];
+      }
     unsigned act = 0, full = 0;
     int64_t* slot = ring + (w & 3) * 128;
+    if (eb + 128 <= T && !inner && d0 != kNullRow) {
+      // one contiguous input run (the steady state): 4 copies off one address
+      const int64_t* src = val + (eb + lane + d0);
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      const int ee = eb + 32 * u + lane;
-      const bool in = ee < T;
-      const bool va = in && dd[u] != kNullRow;
-      act |= (in ? 1u : 0u) << u;
-      full |= (va ? 1u : 0u) << u;
-      if (va)
-        cp_async8(slot + 32 * u + lane, val + (ee + dd[u]));
-      else
-        slot[32 * u + lane] = fc.fill;
+      for (int u = 0; u < 4; ++u) cp_async8(slot + 32 * u + lane, src + 32 * u);
+      act = full = 15u;
+    } else {
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const int ee = eb + 32 * u + lane;
+        const bool in = ee < T;
+        const bool va = in && dd[u] != kNullRow;
+        act |= (in ? 1u : 0u) << u;
+        full |= (va ? 1u : 0u) << u;
+        if (va)
+          cp_async8(slot + 32 * u + lane, val + (ee + dd[u]));
+        else
+          slot[32 * u + lane] = fc.fill;
+      }
     }
     masks = (masks & ~(0xffu << (8 * (w & 3)))) | ((act | (full << 4)) << (8 * (w & 3)));
   };
@@ -1051,10 +1066,16 @@ __device__ __noinline__ long long value_tile_multi(const P& p, const FeatCtx& fc
     for (int u = 0; u < 4; ++u) x[u] = slot[32 * u + lane];  // this lane's own copies
     canon_apply_n<4>(fc.q, p.c.itab, x, act, full);
     const long long pos0 = base + w * 128 + lane;
+    if (act == 15u && pos0 + 96 < cap) {
+      int64_t* dst = values + pos0;
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      const long long pos = pos0 + 32 * u;
-      if (((act >> u) & 1u) && pos < cap) values[pos] = x[u];
+      for (int u = 0; u < 4; ++u) dst[32 * u] = x[u];
+    } else {
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const long long pos = pos0 + 32 * u;
+        if (((act >> u) & 1u) && pos < cap) values[pos] = x[u];
+      }
     }
   }
   cp_async_wait_all();
