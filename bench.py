@@ -47,6 +47,7 @@ def parse():
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no clocks / e2e / cpu)")
     ap.add_argument("--no-corun", action="store_true", help="skip the co-run training-slowdown measurement")
+    ap.add_argument("--no-fusion", action="store_true", help="skip the one-launch-per-feature fusion ablation")
     ap.add_argument("--corun-budgets", default="16,37,74,148", help="SM budgets of the co-run sweep")
     ap.add_argument("--placement", default="balanced", choices=["balanced", "round_robin", "skewed"],
                     help="N>1: table placement (DESIGN.md §10)")
@@ -352,6 +353,9 @@ def run_rap(args):
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline and not args.profile:
         cpu = cpu_baseline(w, args.cpu_seconds)
+    fusion = None
+    if world == 1 and not args.no_fusion and not args.profile and args.workload in ("c1", "c2"):
+        fusion = fusion_ablation(w, sets, B, dev, stream, kern_ms, steps=min(K, 200))
     corun = None
     if world == 1 and not args.no_corun and not args.profile and args.workload == "c2":
         from paper_conf_asplos_wangwdz0d24_b200 import corun as cr
@@ -374,7 +378,7 @@ def run_rap(args):
                            "l2_policy": f"rotate {nsets} distinct input/output sets, {nsets * set_bytes / 2**20:.0f} MB "
                                         f"total vs L2 {l2 / 2**20:.0f} MB"},
                 "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks, "gpu_launches": K,
-                "corun": corun}
+                "corun": corun, "fusion": fusion}
         print(json.dumps(line), flush=True)
     plan.close()
     if world > 1:
@@ -382,6 +386,50 @@ def run_rap(args):
 
         dist.destroy_process_group()
     return 0
+
+
+def fusion_ablation(w, sets, B, dev, stream, fused_ms, steps):
+    """"RAP w/o fusion" analog (Fig 10 ablation): the same graph
+    run as one launch per output feature (each its own single-output plan, the
+    features executed back to back on one stream) instead of one horizontally fused
+    launch.  Same kernel code and inputs; only the fusion differs.  Reported as
+    context next to the paper's 1.15x (w/o fusion vs full RAP is not printed as a
+    ratio there)."""
+    import torch
+
+    from paper_conf_asplos_wangwdz0d24_b200 import rap
+
+    plans = []
+    for o in w.spec["outputs"]:
+        s = dict(w.spec)
+        s["outputs"] = [o]
+        plans.append(rap.Plan(s, device=dev.index))
+    nsets = len(sets)
+    outs = [[rap.DeviceOutput(p, B, r.sp_nnz, dev) for p in plans] for r, _ in sets]
+
+    def one(i):
+        r = sets[i % nsets][0]
+        for p, o in zip(plans, outs[i % nsets]):
+            p.preprocess(r, o, stream)
+
+    for i in range(5):
+        one(i)
+    torch.cuda.synchronize()
+    t0 = torch.cuda.Event(enable_timing=True)
+    t1 = torch.cuda.Event(enable_timing=True)
+    t0.record(stream)
+    for i in range(steps):
+        one(i)
+    t1.record(stream)
+    t1.synchronize()
+    unfused_ms = t0.elapsed_time(t1) / steps
+    for p in plans:
+        p.close()
+    del outs
+    torch.cuda.empty_cache()
+    return {"fused_ms": fused_ms, "unfused_ms": unfused_ms, "launches_unfused": len(plans),
+            "fusion_speedup": unfused_ms / fused_ms, "steps": steps,
+            "what": "one fused launch vs one launch per output feature (same kernel, same inputs)"}
 
 
 def run_sharded(args):

@@ -71,6 +71,18 @@ def test_c2_terabyte_full_size(env):
     assert got["values"].shape[0] == 34 * 65536
 
 
+def test_single_output_plans(env):
+    """Every output of the C2 graph as its own plan (the unfused arm of bench.py's
+    fusion ablation): dense-only and sparse-only plans, each equal to the oracle."""
+    _, synth, _, _ = env
+    w = synth.c2_terabyte(0)
+    host = synth.make_batch(w, 1500, seed=5)
+    for o in w.spec["outputs"]:
+        s = dict(w.spec)
+        s["outputs"] = [o]
+        check(env, s, host)
+
+
 def test_multihot_small(env):
     _, synth, _, _ = env
     w = synth.c4_multihot(0, n_features=24)
