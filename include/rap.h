@@ -124,7 +124,8 @@ typedef struct {
  * rap_preprocess_host.
  *   dense_out  f32[n_rows * dense_ld], row-major, dense_ld >= d_out_cols
  *   lengths    int32[n_sparse_out * n_rows], feature-major
- *   offsets    int64[n_sparse_out * n_rows + 1]
+ *   offsets    int64[n_sparse_out * n_rows + 1] (may be NULL when
+ *              n_sparse_out == 0; if given, offsets[0] = 0 is written)
  *   values     int64[values_capacity]; values_capacity must be >= the bound
  *              returned by rap_plan_output_shape, else RAP_ERR_CAPACITY. */
 typedef struct {

@@ -1900,6 +1900,8 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
     mbar_init(&cs.bar, 1);
     cs.phase = 0;
     cs.dgroup = -1;
+    // no sparse outputs: the offsets array is the single total 0 (R17)
+    if (blockIdx.x == 0 && p.c.n_sparse_out == 0 && !p.c.chain && p.c.offsets) p.c.offsets[0] = 0;
   }
   trace_stamp(p.c, 0);
   const int rank = blockIdx.x;

@@ -1162,7 +1162,7 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
   const int64_t B = raw->n_rows;
   cudaError_t e;
   if (B == 0) {
-    if (!P->souts.empty() && !(out->flags & RAP_OUT_CHAIN)) {
+    if (out->offsets && !(out->flags & RAP_OUT_CHAIN)) {  // offsets[F * 0] = 0, also when F = 0
       e = cudaMemsetAsync(out->offsets, 0, sizeof(int64_t), stream);
       if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync");
     }
@@ -1341,6 +1341,8 @@ static rap_status preprocess_host_impl(rap_plan* P, const rap_raw_batch* raw, co
     if (e == cudaSuccess && vb > 0)
       e = cudaMemcpyAsync(out->values, dv, sizeof(int64_t) * vb, cudaMemcpyDeviceToHost, stream);
     if (e != cudaSuccess) return cuda_fail(e, "D2H sparse");
+  } else if (out->offsets) {
+    out->offsets[0] = 0;  // no sparse outputs: the single total (HOST buffer)
   }
   if (!sync) return RAP_OK;
   e = cudaStreamSynchronize(stream);

@@ -77,10 +77,21 @@ def test_single_output_plans(env):
     _, synth, _, _ = env
     w = synth.c2_terabyte(0)
     host = synth.make_batch(w, 1500, seed=5)
-    for o in w.spec["outputs"]:
+    rap, _, oracle, torch = env
+    for i, o in enumerate(w.spec["outputs"]):
         s = dict(w.spec)
         s["outputs"] = [o]
-        check(env, s, host)
+        assert_parity(run_gpu(rap, torch, s, host), oracle.run(s, host), ctx=f"output {i} (node {o})")
+    # dense-only plan through the host-buffer entry: offsets = [0]
+    s = dict(w.spec)
+    s["outputs"] = [w.spec["outputs"][0]]
+    plan = rap.Plan(s, device=0)
+    hraw = rap.DeviceBatch(host, None, pin=True)
+    hout = rap.DeviceOutput(plan, host["n_rows"], hraw.sp_nnz, None, pin=True)
+    hout.offsets.fill_(-7)
+    plan.preprocess_host(hraw, hout)
+    assert_parity(hout.to_numpy(), oracle.run(s, host), ctx="dense-only host entry")
+    plan.close()
 
 
 def test_multihot_small(env):
