@@ -1110,6 +1110,21 @@ static rap_status update_partition(rap_plan* P, int64_t B, const int64_t* nnz, i
       *d_part_out = P->d_part + i * kPartLen;
       return RAP_OK;
     }
+  // A partition only balances work: any cached one with the same rows and grid
+  // covers exactly the same tiles, so a batch whose quantised mean lengths are
+  // within one step of a cached shape reuses it (no re-plan, upload or slot
+  // eviction when a mean sits on a quantisation boundary and flips from batch
+  // to batch).
+  for (size_t i = 0; i < P->part_keys.size(); ++i) {
+    const std::vector<int64_t>& k = P->part_keys[i];
+    if (k.size() != key.size() || k[0] != key[0] || k[1] != key[1]) continue;
+    bool near = true;
+    for (size_t j = 2; j < k.size() && near; ++j) near = std::llabs(k[j] - key[j]) <= 1;
+    if (near) {
+      *d_part_out = P->d_part + i * kPartLen;
+      return RAP_OK;
+    }
+  }
   const int64_t F = (int64_t)P->souts.size();
   const int64_t T = F ? S / F : 0;
   const double kTileFixed = 400.0;  // per-unit overhead (lane-instructions)
