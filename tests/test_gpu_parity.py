@@ -212,6 +212,19 @@ def test_many_launches_same_plan(env):
     plan.close()
 
 
+def test_partition_cache_across_batch_shapes(env):
+    """One plan over 12 batches whose null rates / list lengths differ (cached,
+    near-shape-reused and evicted work partitions): every output exact."""
+    rap, synth, oracle, torch = env
+    w = synth.c4_multihot(0, n_features=16)
+    plan = rap.Plan(w.spec, device=0)
+    for i in range(12):
+        host = synth.make_batch(w, 1024 + 128 * (i % 10), seed=40 + i)
+        got = run_gpu(rap, torch, w.spec, host, plan=plan)
+        assert_parity(got, oracle.run(w.spec, host), ctx=f"batch {i}")
+    plan.close()
+
+
 def test_cuda_graph_replay(env):
     rap, synth, oracle, torch = env
     w = synth.c2_terabyte(0)
