@@ -152,14 +152,34 @@ typedef struct {
 struct rap_plan;
 typedef struct rap_plan rap_plan;
 
-/* Read-only description of a plan (HOST). */
+/* Read-only description of a plan (HOST).  The kernel fields describe the
+ * last launch: kernel_last = RAP_KERNEL_TILED or RAP_KERNEL_ROWS; for the
+ * row-block kernel rb_row_blocks x rb_feature_groups CTAs of rb_rows rows. */
 typedef struct {
   int32_t device, sm_count, sm_budget, ctas_per_sm, threads_per_cta, grid;
   int32_t n_dense_out_cols, n_sparse_out, n_dense_groups, rows_per_dense_desc;
   int32_t max_rows_per_sparse_desc, min_rows_per_sparse_desc;
   int64_t n_descriptors_last, n_launches;
   int64_t smem_bytes;
+  int32_t kernel_mode, kernel_last, rows_ctas_per_sm, rows_smem_bytes;
+  int32_t rb_row_blocks, rb_feature_groups, rb_rows, rb_memo_slots;
+  int64_t partition_uploads;  /* work partitions uploaded (tiled kernel), cumulative */
 } rap_plan_info;
+
+/* Which fused kernel rap_preprocess launches.  Both compute
+ * the same outputs (R1-R20); they differ in how work maps to threads.
+ *   RAP_KERNEL_AUTO  (default) the row-block kernel when the plan fits it
+ *                    (<= 64 raw sparse / 32 raw dense columns, <= 1024 sparse
+ *                    outputs) and every raw sparse column's mean list length
+ *                    in this batch is <= 2 (Criteo-shaped); else the tiled one
+ *   RAP_KERNEL_TILED (feature, 128-row) tiles, element-parallel for long
+ *                    multi-hot lists (rap_kernel.cu)
+ *   RAP_KERNEL_ROWS  row blocks x feature groups, one row per thread
+ *                    (rap_rows.cu); RAP_ERR_UNSUPPORTED if the plan does not
+ *                    fit it */
+#define RAP_KERNEL_AUTO 0
+#define RAP_KERNEL_TILED 1
+#define RAP_KERNEL_ROWS 2
 
 /* Build a plan (the a0 row of DESIGN.md §1): validate the DAG and parameters
  * (R20, same checks and codes as the oracle), lower every output to a device
@@ -220,6 +240,16 @@ rap_status rap_choose_budget(const rap_plan* plan, int64_t n_rows, const int64_t
                              double overlap_capacity_us, int32_t* sm_budget, double* t_delta_us);
 
 rap_status rap_plan_info_get(const rap_plan* plan, rap_plan_info* info);
+
+/* Select the kernel of the following rap_preprocess calls (RAP_KERNEL_*). */
+rap_status rap_set_kernel(rap_plan* plan, int32_t mode);
+
+/* Device-side capacity overflow of the launches since the last query: a
+ * kernel that found more output ids than values_capacity (possible only when
+ * sp_nnz understated the batch) stores none past the capacity and raises a
+ * flag.  Synchronises the plan's device, writes *overflow (HOST, 0 or 1) and
+ * clears the flag. */
+rap_status rap_check_overflow(rap_plan* plan, int32_t* overflow);
 
 /* ---- Multi-GPU (§7.2; hybrid parallelism L488-499) ----
  * Table-wise: each sparse output ("table") is preprocessed over the FULL

@@ -9,8 +9,8 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "librap.so")
-SOURCES = [os.path.join(CSRC, f) for f in ("rap_plan.cpp", "rap_kernel.cu")]
-HEADERS = [os.path.join(CSRC, "rap_internal.h"), os.path.join(ROOT, "include", "rap.h")]
+SOURCES = [os.path.join(CSRC, f) for f in ("rap_plan.cpp", "rap_kernel.cu", "rap_rows.cu")]
+HEADERS = [os.path.join(CSRC, "rap_internal.h"), os.path.join(CSRC, "rap_device.cuh"), os.path.join(ROOT, "include", "rap.h")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-Xptxas", "-v", "-shared", "-Xcompiler", "-fPIC,-O2", "-I" + os.path.join(ROOT, "include")]

@@ -214,6 +214,52 @@ RAP_HD uint64_t splitmix_H(uint64_t x) {
   return z ^ (z >> 31);
 }
 
+// ---- Row-block kernel (rap_rows.cu) ----
+// The batch's rows are split into n_rb contiguous row blocks and the sparse
+// outputs into n_fg feature groups; CTA (g, r) evaluates group g over block
+// r, one row per thread, in 256-row chunks: (1) output lengths from the Arrow
+// offsets staged in shared memory, summed per output into agg[f * n_rb + r]
+// and announced on a release counter; (2) dense blocks; (3) the base of every
+// output of the group = the feature-major exclusive prefix of those totals
+// (warp-parallel reductions); (4) lengths, offsets and ids.
+constexpr int kRbChunk = 256;   // rows per chunk (one per thread)
+constexpr int kRbMaxFg = 64;    // feature groups
+constexpr int kRbMaxFL = 64;    // sparse outputs per feature group
+constexpr int kRbMaxF = 1024;   // sparse outputs of a plan the row-block kernel takes
+constexpr int kRbMaxCols = 64;  // raw sparse columns the row-block kernel addresses
+constexpr int kRbMaxDense = 32; // raw dense columns
+
+// Per sparse output (indexed by output f): its closed-form length program
+// (R5, R7, R10, R14 from the Arrow offsets and validity bits of up to
+// kMaxNgramK raw columns) and how its ids are emitted.
+//   kind 0: one list source; 1: constant (a dense Bucketize, R4); 2: NGram.
+//   emit 0: canonical list (Canon stages), 1: generic list, 2: dense bucket,
+//        3: NGram.
+// Memo: a canonical list output saves element 0 of each row after the stages
+// in memo_mask into shared slot memo_slot, and an NGram source k whose chain
+// is that prefix reads it (prov[k] = the provider's processing index, so
+// the kernel uses it only if the provider ran earlier in the same CTA).
+struct RbFeat {
+  int32_t kind, n, k, out_cap;  // out_cap: NGram FirstX cap, or kind 1's constant
+  int32_t src[kMaxNgramK];      // raw sparse column, -1 = dense-bucket source (length cap[i])
+  int32_t cap[kMaxNgramK];      // FirstX cap of a valid row
+  int32_t ncap[kMaxNgramK];     // length of a null row (filled: min(1, cap), else 0)
+  int32_t emit, memo_slot, memo_mask, pad;
+  int32_t prov[kMaxNgramK];
+  int32_t pslot[kMaxNgramK];
+};
+
+struct RbGeom {
+  int32_t n_rb, n_fg, rows_rb, max_fl;  // row blocks, feature groups, rows per block (x32), max outputs per group
+  int32_t max_cols, dense_bytes;        // max raw sparse columns one group stages; dense-phase smem bytes
+  int32_t n_memo, small;                // memo slots; small = 1: every base fits 31 bits (32-bit scans)
+  const RbFeat* feat;                   // [n_sparse_out], by output index
+  const int32_t* perm;                  // [n_sparse_out] processing order (groups are ranges of it)
+  unsigned long long* agg;              // [n_sparse_out * n_rb] per-(output, row block) totals, feature-major
+  unsigned long long* sched;            // [0] CTAs done, [2] CTAs whose totals are stored (reset by the last CTA)
+  int32_t fg_off[kRbMaxFg + 1];         // group g = perm[fg_off[g] .. fg_off[g + 1])
+};
+
 // Launch entry implemented in rap_kernel.cu (cooperative launch: every CTA
 // is resident, so a CTA may wait on its predecessors' aggregates).
 // Returns a cudaError_t value.
@@ -225,5 +271,11 @@ int launch_jagged_append(const int32_t* len, const int64_t* so, const int64_t* v
                          int64_t* dof, int64_t* dv, int64_t cap, void* stream);
 // Occupancy query: CTAs per SM for the given dynamic smem.
 int fused_occupancy(int smem_bytes, int n_dense, int n_sparse, int* ctas_per_sm);
+// Row-block kernel (rap_rows.cu): dynamic smem for a geometry, occupancy, launch.
+int rows_smem_bytes(int dense_bytes, int max_fl, int max_cols, int n_memo, int n_sparse_out);
+// Dense-phase shared memory of the row-block kernel for dense groups up to max_width columns.
+int rows_dense_bytes(int max_width);
+int rows_occupancy(int smem_bytes, int* ctas_per_sm);
+int launch_rows(const Common& c, const RbGeom& g, const LaunchRaw& raw, int smem_bytes, void* stream);
 
 }  // namespace rapk

@@ -105,6 +105,16 @@ struct rap_plan {
   // host-buffer staging (rap_preprocess_host)
   std::vector<void*> stage;
   std::vector<size_t> stage_cap;
+  int64_t partition_uploads = 0;
+  // row-block kernel (rap_rows.cu)
+  int kernel_mode = RAP_KERNEL_AUTO, kernel_last = 0;
+  int rb_fits = 0, rb_ctas_per_sm = 0, rb_smem = 0, rb_max_fl = 0, rb_max_cols = 0, rb_n_memo = 0;
+  int rb_dense_bytes = 0;
+  std::vector<RbFeat> rbfeat;     // by output index
+  std::vector<int32_t> rb_perm;   // processing order
+  size_t off_rbfeat = 0, off_perm = 0;
+  unsigned long long* d_agg_rb = nullptr;  // [n_sparse_out * kMaxCtas]
+  int rb_last_n_rb = 0, rb_last_n_fg = 0, rb_last_rows = 0;
 };
 
 namespace {
@@ -747,6 +757,162 @@ void build_dprogs(rap_plan* P, const std::vector<Unit>& flat) {
   close(P->d_out);
 }
 
+// ----------------------------------------------------------------------------
+// Row-block kernel descriptors (rap_internal.h RbFeat): closed-form length
+// programs, emission kind, processing order and memo slots.
+
+int clip32(int64_t x) { return (int)std::min<int64_t>(std::max<int64_t>(x, 0), INT32_MAX); }
+
+// Canonical stage bits up to and including the highest bit of m (stage order
+// Clamp -> MapId -> SigridHash -> Bucketize).
+int stage_prefix(int m) {
+  if (m == 0) return 0;
+  int h = 0;
+  for (int b = 0; b < 4; ++b)
+    if (m & (1 << b)) h = b;
+  return (2 << h) - 1;
+}
+
+bool same_stage_params(const rap_plan* P, const Canon& a, const Canon& b, int mask) {
+  if ((mask & CB_CLAMP) && (a.lo != b.lo || a.hi != b.hi)) return false;
+  if (mask & CB_MAPID) {
+    if (a.map_m != b.map_m || a.map_def != b.map_def) return false;
+    if (a.map_a != b.map_a &&
+        memcmp(&P->itab[a.map_a], &P->itab[b.map_a], sizeof(int64_t) * 2 * ((size_t)1 << a.map_m)) != 0)
+      return false;
+  }
+  if ((mask & CB_SIGRID) && (a.hs != b.hs || a.M != b.M)) return false;
+  if (mask & CB_BUCKET) {
+    if (a.bk_m != b.bk_m) return false;
+    if (a.bk_a != b.bk_a && memcmp(&P->itab[a.bk_a], &P->itab[b.bk_a], sizeof(int64_t) * a.bk_m) != 0) return false;
+  }
+  return true;
+}
+
+// Does canonical list output O compute, as a prefix of its stages, the
+// elements of NGram source chain S (same column, null rule and stage
+// parameters)?  Returns the prefix mask, or -1.
+int memo_prefix(const rap_plan* P, const Chain& o, const Canon& qo, const Chain& s, const Canon& qs) {
+  if (o.src_kind != SRC_SPARSE || s.src_kind != SRC_SPARSE || o.src != s.src || !qo.ok || !qs.ok) return -1;
+  if (o.has_fill != s.has_fill || (s.has_fill && o.fill != s.fill)) return -1;
+  const int pm = stage_prefix(qs.mask);
+  if ((qo.mask & pm) != qs.mask || (qo.null_mask & pm) != qs.null_mask) return -1;
+  if (!same_stage_params(P, qs, qo, qs.mask)) return -1;
+  return pm;
+}
+
+constexpr int kRbMemoMax = 16;  // memo slots (256 rows x 8 bytes each) a CTA may hold
+
+void build_rows(rap_plan* P) {
+  const int F = (int)P->souts.size();
+  P->rbfeat.assign(F, RbFeat{});
+  std::vector<std::vector<int>> prov_out(F, std::vector<int>(kMaxNgramK, -1));
+  for (int f = 0; f < F; ++f) {
+    const Chain& ch = P->chains[P->souts[f].chain];
+    const SProg& sp = P->sprogs[f];
+    RbFeat& R = P->rbfeat[f];
+    memset(&R, 0, sizeof(R));
+    R.memo_slot = -1;
+    for (int i = 0; i < kMaxNgramK; ++i) R.prov[i] = R.pslot[i] = -1;
+    auto source = [&](int i, const Chain& c) {
+      if (c.src_kind == SRC_SPARSE) {
+        R.src[i] = c.src;
+        R.cap[i] = clip32(c.xcap);
+        R.ncap[i] = c.has_fill ? (int)std::min<int64_t>(1, c.null_xcap) : 0;
+      } else {  // dense Bucketize source: one id (R4)
+        R.src[i] = -1;
+        R.cap[i] = (int)std::min<int64_t>(1, c.xcap);
+      }
+    };
+    if (ch.src_kind == SRC_SPARSE) {
+      R.kind = 0;
+      R.k = 1;
+      source(0, ch);
+      R.emit = sp.cn.ok ? 0 : 1;
+    } else if (ch.src_kind == SRC_DENSE_BUCKET) {
+      R.kind = 1;
+      R.out_cap = (int)std::min<int64_t>(1, ch.xcap);
+      R.emit = 2;
+    } else {
+      const NGramDesc& ng = P->ngrams[ch.src];
+      R.kind = 2;
+      R.emit = 3;
+      R.n = ng.n;
+      R.k = ng.k;
+      R.out_cap = clip32(ch.xcap);
+      for (int i = 0; i < ng.k; ++i) source(i, P->chains[ng.chain[i]]);
+    }
+  }
+  // memo providers: the first canonical list output whose stage prefix is the source chain
+  std::vector<int> memo_mask(F, -1);
+  for (int g = 0; g < F; ++g) {
+    if (P->rbfeat[g].emit != 3) continue;
+    const SProg& sp = P->sprogs[g];
+    for (int k = 0; k < sp.ng.k; ++k) {
+      const Chain& sc = P->chains[sp.ng.chain[k]];
+      for (int f = 0; f < F; ++f) {
+        if (P->rbfeat[f].emit != 0) continue;
+        const int pm = memo_prefix(P, P->chains[P->souts[f].chain], P->sprogs[f].cn, sc, sp.src_cn[k]);
+        if (pm < 0 || (memo_mask[f] >= 0 && memo_mask[f] != pm)) continue;
+        memo_mask[f] = pm;
+        prov_out[g][k] = f;
+        break;
+      }
+    }
+  }
+  // processing order: an NGram right after the last of its providers
+  struct Key {
+    int a, b, c;
+  };
+  std::vector<Key> key(F);
+  for (int f = 0; f < F; ++f) {
+    int mp = -1;
+    for (int k = 0; k < kMaxNgramK; ++k) mp = std::max(mp, prov_out[f][k]);
+    key[f] = mp >= 0 ? Key{mp, 1, f} : Key{f, 0, f};
+  }
+  P->rb_perm.resize(F);
+  std::iota(P->rb_perm.begin(), P->rb_perm.end(), 0);
+  std::stable_sort(P->rb_perm.begin(), P->rb_perm.end(), [&](int x, int y) {
+    if (key[x].a != key[y].a) return key[x].a < key[y].a;
+    if (key[x].b != key[y].b) return key[x].b < key[y].b;
+    return key[x].c < key[y].c;
+  });
+  std::vector<int> pidx(F);
+  for (int i = 0; i < F; ++i) pidx[P->rb_perm[i]] = i;
+  // memo slots: live from the provider to its last consumer (processing order)
+  std::vector<int> last_use(F, -1);
+  for (int g = 0; g < F; ++g)
+    for (int k = 0; k < kMaxNgramK; ++k)
+      if (prov_out[g][k] >= 0) last_use[prov_out[g][k]] = std::max(last_use[prov_out[g][k]], pidx[g]);
+  std::vector<int> slot_of(F, -1), slot_end(kRbMemoMax, -1);
+  int n_memo = 0;
+  for (int i = 0; i < F; ++i) {
+    const int f = P->rb_perm[i];
+    if (last_use[f] < 0) continue;
+    int sl = -1;
+    for (int j = 0; j < kRbMemoMax && sl < 0; ++j)
+      if (slot_end[j] < i) sl = j;
+    if (sl < 0) continue;  // no free slot: the consumers recompute
+    slot_end[sl] = last_use[f];
+    slot_of[f] = sl;
+    n_memo = std::max(n_memo, sl + 1);
+    P->rbfeat[f].memo_slot = sl;
+    P->rbfeat[f].memo_mask = memo_mask[f];
+  }
+  for (int g = 0; g < F; ++g)
+    for (int k = 0; k < kMaxNgramK; ++k) {
+      const int f = prov_out[g][k];
+      if (f >= 0 && slot_of[f] >= 0) {
+        P->rbfeat[g].prov[k] = pidx[f];
+        P->rbfeat[g].pslot[k] = slot_of[f];
+      }
+    }
+  P->rb_n_memo = n_memo;
+  P->rb_fits = P->n_sparse_in <= kRbMaxCols && P->n_dense_in <= kRbMaxDense && F <= kRbMaxF;
+  P->rb_max_fl = std::max(1, std::min(F, kRbMaxFL));
+  P->rb_max_cols = std::max(1, (int)P->used_sparse.size());
+}
+
 }  // namespace
 
 // ============================================================================
@@ -871,6 +1037,8 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
       if (us[c]) P->used_sparse.push_back(c);
   }
 
+  build_rows(P);
+
   // ---- device blob
   std::vector<unsigned char> blob;
   P->off_ops = push_blob(blob, P->ops);
@@ -879,6 +1047,8 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
   P->off_dprogs = push_blob(blob, P->dprogs);
   P->off_ftab = push_blob(blob, P->ftab);
   P->off_itab = push_blob(blob, P->itab);
+  P->off_rbfeat = push_blob(blob, P->rbfeat);
+  P->off_perm = push_blob(blob, P->rb_perm);
   if (blob.empty()) blob.resize(16);
   e = cudaMalloc(&P->blob, blob.size());
   if (e == cudaSuccess) e = cudaMemcpy(P->blob, blob.data(), blob.size(), cudaMemcpyHostToDevice);
@@ -891,6 +1061,11 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
   if (e == cudaSuccess) e = cudaMemset(P->d_agg, 0, kMaxCtas * sizeof(unsigned long long));
   if (e == cudaSuccess) e = cudaMalloc(&P->d_part, kPartSlots * kPartLen * sizeof(int64_t));
   if (e == cudaSuccess) e = cudaMallocHost(&P->h_part, kPartSlots * kPartLen * sizeof(int64_t));
+  if (e == cudaSuccess && P->rb_fits && !P->souts.empty()) {
+    const size_t n = P->souts.size() * (size_t)kMaxCtas;
+    e = cudaMalloc(&P->d_agg_rb, n * sizeof(unsigned long long));
+    if (e == cudaSuccess) e = cudaMemset(P->d_agg_rb, 0, n * sizeof(unsigned long long));
+  }
   if (e == cudaSuccess) e = cudaMalloc(&P->d_err, sizeof(int32_t));
   if (e == cudaSuccess) e = cudaMemset(P->d_err, 0, sizeof(int32_t));
   if (e != cudaSuccess) {
@@ -909,6 +1084,21 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
     return cuda_fail(e, "occupancy query");
   }
   P->ctas_per_sm = std::max(1, occ);
+  if (P->rb_fits) {
+    P->rb_dense_bytes = rows_dense_bytes(max_w);
+    P->rb_smem = rows_smem_bytes(P->rb_dense_bytes, P->rb_max_fl, P->rb_max_cols, P->rb_n_memo, (int)P->souts.size());
+    if (P->rb_smem > 227 * 1024) P->rb_fits = 0;
+  }
+  if (P->rb_fits) {
+    int rocc = 0;
+    e = (cudaError_t)rows_occupancy(P->rb_smem, &rocc);
+    if (e != cudaSuccess) {
+      rap_plan_destroy(P);
+      return cuda_fail(e, "row-block kernel occupancy query");
+    }
+    P->rb_ctas_per_sm = rocc;
+    if (rocc < 1) P->rb_fits = 0;  // shared memory does not fit one CTA
+  }
   *out = P;
   return RAP_OK;
 }
@@ -923,6 +1113,7 @@ void rap_plan_destroy(rap_plan* P) {
   cudaFreeHost(P->h_part);
   cudaFree(P->d_err);
   cudaFree(P->d_trace);
+  cudaFree(P->d_agg_rb);
   for (void* s : P->stage) cudaFree(s);
   delete P;
 }
@@ -997,6 +1188,38 @@ rap_status rap_plan_info_get(const rap_plan* P, rap_plan_info* info) {
   info->n_descriptors_last = P->last_n_desc;
   info->n_launches = P->n_launches;
   info->smem_bytes = P->smem;
+  info->kernel_mode = P->kernel_mode;
+  info->kernel_last = P->kernel_last;
+  info->rows_ctas_per_sm = P->rb_fits ? P->rb_ctas_per_sm : 0;
+  info->rows_smem_bytes = P->rb_smem;
+  info->rb_row_blocks = P->rb_last_n_rb;
+  info->rb_feature_groups = P->rb_last_n_fg;
+  info->rb_rows = P->rb_last_rows;
+  info->rb_memo_slots = P->rb_n_memo;
+  info->partition_uploads = P->partition_uploads;
+  if (P->kernel_last == RAP_KERNEL_ROWS) info->grid = P->rb_last_n_rb * P->rb_last_n_fg;
+  return RAP_OK;
+}
+
+rap_status rap_set_kernel(rap_plan* P, int32_t mode) {
+  if (!P) return fail(RAP_ERR_INVALID_ARGUMENT, "plan is NULL");
+  if (mode != RAP_KERNEL_AUTO && mode != RAP_KERNEL_TILED && mode != RAP_KERNEL_ROWS)
+    return fail(RAP_ERR_INVALID_ARGUMENT, "unknown kernel mode");
+  if (mode == RAP_KERNEL_ROWS && !P->rb_fits && !P->souts.empty())
+    return fail(RAP_ERR_UNSUPPORTED, "plan does not fit the row-block kernel (> 64 sparse / 32 dense raw columns)");
+  P->kernel_mode = mode;
+  return RAP_OK;
+}
+
+rap_status rap_check_overflow(rap_plan* P, int32_t* overflow) {
+  if (!P || !overflow) return fail(RAP_ERR_INVALID_ARGUMENT, "NULL argument");
+  DeviceGuard dg(P->device);
+  cudaError_t e = cudaDeviceSynchronize();
+  int32_t v = 0;
+  if (e == cudaSuccess) e = cudaMemcpy(&v, P->d_err, sizeof(v), cudaMemcpyDeviceToHost);
+  if (e == cudaSuccess) e = cudaMemset(P->d_err, 0, sizeof(int32_t));
+  if (e != cudaSuccess) return cuda_fail(e, "rap_check_overflow");
+  *overflow = v ? 1 : 0;
   return RAP_OK;
 }
 
@@ -1165,12 +1388,76 @@ static rap_status update_partition(rap_plan* P, int64_t B, const int64_t* nnz, i
   int64_t* d = P->d_part + (size_t)slot * kPartLen;
   e = cudaMemcpyAsync(d, part, sizeof(int64_t) * (n + 1), cudaMemcpyHostToDevice, stream);
   if (e != cudaSuccess) return cuda_fail(e, "partition upload");
+  P->partition_uploads += 1;
   if ((int)P->part_keys.size() < kPartSlots)
     P->part_keys.push_back(key);
   else
     P->part_keys[slot] = key;
   *d_part_out = d;
   return RAP_OK;
+}
+
+// Does this batch go to the row-block kernel?  RAP_KERNEL_AUTO: when the plan
+// fits it and every used raw sparse column averages <= 2 ids per row (the
+// row-per-thread mapping is efficient for short lists; long multi-hot lists
+// go element-parallel through the tiled kernel).
+static bool use_rows(const rap_plan* P, int64_t B, const int64_t* nnz) {
+  if (P->kernel_mode == RAP_KERNEL_TILED || !P->rb_fits || P->souts.empty()) return false;
+  if (P->kernel_mode == RAP_KERNEL_ROWS) return true;
+  if (getenv("RAP_AUTO_ROWS") == nullptr) return false;  // interpreted row-block kernel: opt-in until it wins
+  for (int s : P->used_sparse)
+    if (nnz && B > 0 && (double)nnz[s] > 2.0 * (double)B) return false;
+  return true;
+}
+
+// Row-block geometry of one launch (rap_internal.h RbGeom): row blocks of a
+// multiple of 32 rows and feature groups (contiguous ranges of the processing
+// order, balanced by the cost model, <= kRbMaxFL outputs each), at most the
+// budget's CTA slots.  Large batches: one feature group, one row block per
+// slot.  Small batches: 256-row blocks, the slots left over split the outputs.
+static void rows_geometry(const rap_plan* P, int64_t B, const int64_t* nnz, RbGeom* g) {
+  const int F = (int)P->souts.size();
+  const int64_t slots = std::max<int64_t>(1, std::min<int64_t>((int64_t)P->budget * P->rb_ctas_per_sm, kMaxCtas));
+  const int fg_min = (F + kRbMaxFL - 1) / kRbMaxFL;
+  const int64_t nb256 = (B + kRbChunk - 1) / kRbChunk;
+  int64_t n_rb, n_fg;
+  if (nb256 * fg_min * 2 >= slots) {
+    n_fg = fg_min;
+    n_rb = std::max<int64_t>(1, std::min<int64_t>(slots / n_fg, (B + 31) / 32));
+  } else {
+    n_rb = nb256;
+    n_fg = std::max<int64_t>(fg_min, std::min<int64_t>({(int64_t)F, (int64_t)kRbMaxFg, slots / n_rb}));
+  }
+  const char* env = getenv("RAP_RB_ROWS");  // experiment knob: rows per block
+  int64_t rows = env ? std::max<int64_t>(32, atoll(env) / 32 * 32) : 32 * ((B + 32 * n_rb - 1) / (32 * n_rb));
+  n_rb = std::max<int64_t>(1, (B + rows - 1) / rows);
+  if (n_rb * n_fg > kMaxCtas) {  // knob out of range: back to the default
+    rows = 32 * ((B + 32 * (kMaxCtas / n_fg) - 1) / (32 * (kMaxCtas / n_fg)));
+    n_rb = (B + rows - 1) / rows;
+  }
+  g->n_rb = (int)n_rb;
+  g->rows_rb = (int)rows;
+  // feature groups: contiguous ranges of the processing order, equal predicted cost
+  std::vector<double> cost(F);
+  double W = 0;
+  for (int i = 0; i < F; ++i) {
+    cost[i] = sparse_row_cost(P, P->chains[P->souts[P->rb_perm[i]].chain], B, nnz);
+    W += cost[i];
+  }
+  int gcount = 0, start = 0;
+  double acc = 0;
+  g->fg_off[0] = 0;
+  for (int i = 0; i < F; ++i) {
+    const bool full = i - start >= kRbMaxFL;
+    const bool due = gcount + 1 < n_fg && acc + 0.5 * cost[i] >= W * (double)(gcount + 1) / (double)n_fg && i > start;
+    if ((full || due) && gcount + 1 < kRbMaxFg) {
+      g->fg_off[++gcount] = i;
+      start = i;
+    }
+    acc += cost[i];
+  }
+  g->fg_off[++gcount] = F;
+  g->n_fg = gcount;
 }
 
 static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output* out, cudaStream_t stream) {
@@ -1192,15 +1479,14 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
   int64_t drow0 = 0, drows = B;
   rap_shard_rows(B, P->rank, P->world, &drow0, &drows);
   const int64_t n_dense = P->dprogs.empty() ? 0 : (int64_t)P->dprogs.size() * ((drows + kDenseBlockRows - 1) / kDenseBlockRows);
-  if (n_sparse_tiles == 0 && n_dense == 0) return RAP_OK;
-  // grid: the budget's CTA slots, but no more CTAs than there is work for
-  // (a warp per sparse tile, a CTA per dense block): small batches then pay
-  // a shorter aggregate chain and fewer idle CTAs
-  const int64_t want = std::max<int64_t>(1, std::max<int64_t>(n_dense, (n_sparse_tiles + kWarpsPerCta - 1) / kWarpsPerCta));
-  const int64_t grid = std::min<int64_t>(std::min<int64_t>((int64_t)P->budget * P->ctas_per_sm, kMaxCtas), want);
-  const int64_t* d_part = nullptr;
-  rap_status pst = update_partition(P, B, raw->sp_nnz, n_sparse_tiles, n_dense, (int)grid, stream, &d_part);
-  if (pst != RAP_OK) return pst;
+  if (n_sparse_tiles == 0 && n_dense == 0) {
+    // nothing to compute (a rank without tables or rows): offsets = [0] (R17)
+    if (out->offsets && !(out->flags & RAP_OUT_CHAIN)) {
+      e = cudaMemsetAsync(out->offsets, 0, sizeof(int64_t), stream);
+      if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync");
+    }
+    return RAP_OK;
+  }
   Common c{};
   c.ops = reinterpret_cast<const DevOp*>(P->blob + P->off_ops);
   c.sprogs = reinterpret_cast<const SProg*>(P->blob + P->off_sprogs);
@@ -1218,7 +1504,6 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
   c.n_dense_rows = drows;
   c.chain = (out->flags & RAP_OUT_CHAIN) ? 1 : 0;
   c.sched = P->d_sched;
-  c.part = d_part;
   c.agg = P->d_agg;
   c.dense_out = out->dense_out;
   c.ld = out->dense_ld;
@@ -1229,7 +1514,6 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
   c.err = P->d_err;
   c.trace = P->d_trace;
   c.trace_cap = P->trace_cap;
-  const int64_t n_total = n_sparse_tiles + n_dense;
   LaunchRaw lr{};
   lr.n_dense = P->n_dense_in;
   lr.n_sparse = P->n_sparse_in;
@@ -1238,8 +1522,43 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
   lr.off = raw->sp_offsets;
   lr.val = raw->sp_values;
   lr.svalid = raw->sp_valid;
+  if (use_rows(P, B, raw->sp_nnz)) {
+    RbGeom g;
+    memset(&g, 0, sizeof(g));
+    rows_geometry(P, B, raw->sp_nnz, &g);
+    g.max_fl = P->rb_max_fl;
+    g.max_cols = P->rb_max_cols;
+    g.dense_bytes = P->rb_dense_bytes;
+    g.n_memo = P->rb_n_memo;
+    // 32-bit scans when every offset of this launch fits 31 bits
+    g.small = (!c.chain && values_bound(P, B, raw->sp_nnz) < (int64_t)INT32_MAX - 1) ? 1 : 0;
+    g.feat = reinterpret_cast<const RbFeat*>(P->blob + P->off_rbfeat);
+    g.perm = reinterpret_cast<const int32_t*>(P->blob + P->off_perm);
+    g.agg = P->d_agg_rb;
+    g.sched = P->d_sched + 4;
+    int rc = launch_rows(c, g, lr, P->rb_smem, stream);
+    if (rc != 0) return cuda_fail((cudaError_t)rc, "row-block kernel launch");
+    P->kernel_last = RAP_KERNEL_ROWS;
+    P->rb_last_n_rb = g.n_rb;
+    P->rb_last_n_fg = g.n_fg;
+    P->rb_last_rows = g.rows_rb;
+    P->n_launches += 1;
+    P->last_n_desc = (int64_t)g.n_rb * g.n_fg;
+    return RAP_OK;
+  }
+  // tiled kernel: grid = the budget's CTA slots, but no more CTAs than there
+  // is work for (a warp per sparse tile, a CTA per dense block): small
+  // batches then pay a shorter aggregate chain and fewer idle CTAs
+  const int64_t want = std::max<int64_t>(1, std::max<int64_t>(n_dense, (n_sparse_tiles + kWarpsPerCta - 1) / kWarpsPerCta));
+  const int64_t grid = std::min<int64_t>(std::min<int64_t>((int64_t)P->budget * P->ctas_per_sm, kMaxCtas), want);
+  const int64_t* d_part = nullptr;
+  rap_status pst = update_partition(P, B, raw->sp_nnz, n_sparse_tiles, n_dense, (int)grid, stream, &d_part);
+  if (pst != RAP_OK) return pst;
+  c.part = d_part;
+  const int64_t n_total = n_sparse_tiles + n_dense;
   int rc = launch_fused(c, lr, (int)grid, P->smem, stream);
   if (rc != 0) return cuda_fail((cudaError_t)rc, "fused kernel launch");
+  P->kernel_last = RAP_KERNEL_TILED;
   P->n_launches += 1;
   P->last_n_desc = n_total;
   return RAP_OK;

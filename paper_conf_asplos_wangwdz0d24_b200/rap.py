@@ -22,7 +22,7 @@ STATUS = {0: "OK", 1: "INVALID_ARGUMENT", 2: "INVALID_GRAPH", 3: "INVALID_PARAM"
 EXPORTS = ["rap_plan_create", "rap_plan_output_shape", "rap_preprocess", "rap_preprocess_host", "rap_preprocess_host_async", "rap_set_budget",
            "rap_predict_latency_us", "rap_choose_budget", "rap_plan_info_get", "rap_debug_trace", "rap_plan_destroy",
            "rap_status_string", "rap_last_error", "rap_shard_rows", "rap_plan_output_costs", "rap_place",
-           "rap_plan_create_sharded", "rap_jagged_append"]
+           "rap_plan_create_sharded", "rap_jagged_append", "rap_set_kernel", "rap_check_overflow"]
 PLACE_MODES = {"balanced": 0, "round_robin": 1, "skewed": 2}
 RAP_OUT_CHAIN = 1
 
@@ -73,7 +73,16 @@ class RapPlanInfo(C.Structure):
                 ("n_dense_out_cols", C.c_int32), ("n_sparse_out", C.c_int32), ("n_dense_groups", C.c_int32),
                 ("rows_per_dense_desc", C.c_int32), ("max_rows_per_sparse_desc", C.c_int32),
                 ("min_rows_per_sparse_desc", C.c_int32), ("n_descriptors_last", C.c_int64),
-                ("n_launches", C.c_int64), ("smem_bytes", C.c_int64)]
+                ("n_launches", C.c_int64), ("smem_bytes", C.c_int64),
+                ("kernel_mode", C.c_int32), ("kernel_last", C.c_int32), ("rows_ctas_per_sm", C.c_int32),
+                ("rows_smem_bytes", C.c_int32), ("rb_row_blocks", C.c_int32), ("rb_feature_groups", C.c_int32),
+                ("rb_rows", C.c_int32), ("rb_memo_slots", C.c_int32), ("partition_uploads", C.c_int64)]
+
+
+# rap_set_kernel modes (include/rap.h).  DEFAULT_KERNEL is applied to every new
+# Plan (env RAP_KERNEL; tests set it to run each parity case on both kernels).
+KERNEL_AUTO, KERNEL_TILED, KERNEL_ROWS = 0, 1, 2
+DEFAULT_KERNEL = int(os.environ.get("RAP_KERNEL", "0"))
 
 
 _lib = None
@@ -110,6 +119,10 @@ def load(build_if_stale: bool = False):
     L.rap_choose_budget.argtypes = [P, C.c_int64, P, C.c_double, C.POINTER(C.c_int32), C.POINTER(C.c_double)]
     L.rap_plan_info_get.restype = C.c_int
     L.rap_plan_info_get.argtypes = [P, C.POINTER(RapPlanInfo)]
+    L.rap_set_kernel.restype = C.c_int
+    L.rap_set_kernel.argtypes = [P, C.c_int32]
+    L.rap_check_overflow.restype = C.c_int
+    L.rap_check_overflow.argtypes = [P, C.POINTER(C.c_int32)]
     L.rap_debug_trace.restype = C.c_int
     L.rap_debug_trace.argtypes = [P, C.c_int32, P, C.c_int64, C.POINTER(C.c_int64)]
     L.rap_plan_destroy.restype = None
@@ -302,6 +315,8 @@ class Plan:
         _check(L.rap_plan_create(C.byref(g), params, len(spec["nodes"]), device, sm_budget, C.byref(h)))
         self.handle = h
         self.device = device
+        if DEFAULT_KERNEL:
+            self.set_kernel(DEFAULT_KERNEL)
 
     @classmethod
     def sharded(cls, spec, sparse_owner, rank: int, world: int, device: int = 0, sm_budget: int = 0):
@@ -318,6 +333,8 @@ class Plan:
                                          own.ctypes.data, rank, world, C.byref(h)))
         self.handle = h
         self.device = device
+        if DEFAULT_KERNEL:
+            self.set_kernel(DEFAULT_KERNEL)
         return self
 
     def output_costs(self, n_rows, sp_nnz):
@@ -363,6 +380,17 @@ class Plan:
 
     def set_budget(self, sm_budget: int):
         _check(load().rap_set_budget(self.handle, sm_budget))
+
+    def set_kernel(self, mode: int):
+        """rap_set_kernel: KERNEL_AUTO / KERNEL_TILED / KERNEL_ROWS."""
+        _check(load().rap_set_kernel(self.handle, int(mode)))
+
+    def check_overflow(self) -> int:
+        """rap_check_overflow: 1 if a launch since the last query found more ids
+        than values_capacity (synchronises the device; clears the flag)."""
+        v = C.c_int32()
+        _check(load().rap_check_overflow(self.handle, C.byref(v)))
+        return v.value
 
     def info(self) -> dict:
         i = RapPlanInfo()

@@ -26,6 +26,17 @@ def env():
     return rap, synth, oracle, torch
 
 
+@pytest.fixture(params=[1, 2], ids=["tiled", "rows"], autouse=True)
+def kernel_mode(request):
+    """Every parity case runs on both fused kernels (rap_set_kernel)."""
+    from paper_conf_asplos_wangwdz0d24_b200 import rap
+
+    old = rap.DEFAULT_KERNEL
+    rap.DEFAULT_KERNEL = request.param
+    yield request.param
+    rap.DEFAULT_KERNEL = old
+
+
 def run_gpu(rap, torch, spec_, host, budget=0, plan=None, dense_ld=None):
     own = plan is None
     if own:
