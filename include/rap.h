@@ -164,6 +164,9 @@ typedef struct {
   int32_t kernel_mode, kernel_last, rows_ctas_per_sm, rows_smem_bytes;
   int32_t rb_row_blocks, rb_feature_groups, rb_rows, rb_memo_slots;
   int64_t partition_uploads;  /* work partitions uploaded (tiled kernel), cumulative */
+  int32_t jit_state;          /* generated kernel: 0 not built yet, 1 built, -1 failed (see rap_last_error) */
+  int32_t jit_ctas_per_sm;
+  double jit_compile_seconds; /* NVRTC compile + load time of the generated kernel */
 } rap_plan_info;
 
 /* Which fused kernel rap_preprocess launches.  Both compute
@@ -171,15 +174,25 @@ typedef struct {
  *   RAP_KERNEL_AUTO  (default) the row-block kernel when the plan fits it
  *                    (<= 64 raw sparse / 32 raw dense columns, <= 1024 sparse
  *                    outputs) and every raw sparse column's mean list length
- *                    in this batch is <= 2 (Criteo-shaped); else the tiled one
+ *                    in this batch is <= 2 (Criteo-shaped) -- its generated
+ *                    form when the batch runs as one feature group -- else
+ *                    the tiled kernel
  *   RAP_KERNEL_TILED (feature, 128-row) tiles, element-parallel for long
  *                    multi-hot lists (rap_kernel.cu)
- *   RAP_KERNEL_ROWS  row blocks x feature groups, one row per thread
- *                    (rap_rows.cu); RAP_ERR_UNSUPPORTED if the plan does not
- *                    fit it */
+ *   RAP_KERNEL_ROWS  row blocks x feature groups, one row per thread, each
+ *                    output interpreted from its record (rap_rows.cu);
+ *                    RAP_ERR_UNSUPPORTED if the plan does not fit it
+ *   RAP_KERNEL_JIT   the row-block kernel with every output's chain generated
+ *                    as straight-line CUDA for this plan and compiled by NVRTC
+ *                    for sm_100a on the first launch that uses it (seconds of
+ *                    host time, cached per process); batches
+ *                    that split the outputs into several feature groups run
+ *                    the interpreted form.  If NVRTC fails the plan keeps the
+ *                    interpreted form (rap_plan_info.jit_state = -1). */
 #define RAP_KERNEL_AUTO 0
 #define RAP_KERNEL_TILED 1
 #define RAP_KERNEL_ROWS 2
+#define RAP_KERNEL_JIT 3
 
 /* Build a plan (the a0 row of DESIGN.md §1): validate the DAG and parameters
  * (R20, same checks and codes as the oracle), lower every output to a device
@@ -243,6 +256,15 @@ rap_status rap_plan_info_get(const rap_plan* plan, rap_plan_info* info);
 
 /* Select the kernel of the following rap_preprocess calls (RAP_KERNEL_*). */
 rap_status rap_set_kernel(rap_plan* plan, int32_t mode);
+
+/* Development aid (no device needed): validate and lower the graph, write the
+ * CUDA source the code generator emits for it into HOST buf[cap] (NUL
+ * terminated, truncated to fit) and, if compile != 0, compile it with NVRTC for
+ * sm_100a (no load); *ok = 1 if it compiled.  NVRTC's log goes to
+ * rap_last_error().  RAP_ERR_UNSUPPORTED if the plan does not fit the
+ * row-block kernel. */
+rap_status rap_debug_jit_source(const rap_graph* graph, const rap_op_param* params, int32_t n_params, char* buf,
+                                int64_t cap, int32_t compile, int32_t* ok);
 
 /* Device-side capacity overflow of the launches since the last query: a
  * kernel that found more output ids than values_capacity (possible only when

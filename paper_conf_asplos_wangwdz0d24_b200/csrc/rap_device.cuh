@@ -3,9 +3,11 @@
 // code only; nothing here is shared with oracle/.  Operator semantics:
 // DESIGN.md §3 readings R1-R20.
 #pragma once
+#ifndef __CUDACC_RTC__
 #include <cuda_runtime.h>
 #include <math.h>
 #include <stdint.h>
+#endif
 
 #include "rap_internal.h"
 
@@ -117,6 +119,74 @@ __device__ __forceinline__ int64_t upper_bound(const T* b, int m, T x) {
     }
   }
   return lo;
+}
+
+// #{i : b[i] <= x} over sorted int64 b[0..m) with a sample table
+// smp[i] = b[8i + 7] (i < m / 8): a binary search over the samples (a small
+// table, L1-resident) finds the first block whose last border exceeds x, then
+// the block's <= 8 borders are read in one burst (R4; same result as
+// upper_bound).
+__device__ __forceinline__ int64_t upper_bound_s8(const int64_t* b, int m, const int64_t* smp, int ns, int64_t x) {
+  int lo = 0, n = ns;
+  while (n > 0) {
+    const int half = n >> 1;
+    if (__ldg(smp + lo + half) <= x) {
+      lo += half + 1;
+      n -= half + 1;
+    } else {
+      n = half;
+    }
+  }
+  const int base = lo * 8;
+  const int rem = min(8, m - base);
+  int cnt = 0;
+  if (rem == 8 && (reinterpret_cast<uintptr_t>(b + base) & 15) == 0) {
+    const longlong2* q = reinterpret_cast<const longlong2*>(b + base);
+    const longlong2 a0 = __ldg(q), a1 = __ldg(q + 1), a2 = __ldg(q + 2), a3 = __ldg(q + 3);
+    cnt = (a0.x <= x) + (a0.y <= x) + (a1.x <= x) + (a1.y <= x) + (a2.x <= x) + (a2.y <= x) + (a3.x <= x) + (a3.y <= x);
+  } else {
+    for (int i = 0; i < rem; ++i) cnt += __ldg(b + base + i) <= x;
+  }
+  return base + cnt;
+}
+
+// Count of values <= x among 8 int64 at p (16-byte aligned), one burst.
+__device__ __forceinline__ int count_le8(const int64_t* p, int64_t x) {
+  const longlong2* q = reinterpret_cast<const longlong2*>(p);
+  const longlong2 a0 = __ldg(q), a1 = __ldg(q + 1), a2 = __ldg(q + 2), a3 = __ldg(q + 3);
+  return (a0.x <= x) + (a0.y <= x) + (a1.x <= x) + (a1.y <= x) + (a2.x <= x) + (a2.y <= x) + (a3.x <= x) + (a3.y <= x);
+}
+
+// #{i : b[i] <= x} over sorted int64 b[0..m), m a multiple of 64, given
+// level-0 index j0 = #{blocks of 64 whose last border <= x} (the generated
+// code computes it from immediates): then the 8 sub-block maxima of block j0
+// (smp8[8 j0 .. 8 j0 + 8), smp8[i] = b[8 i + 7]) and the 8 borders of the
+// chosen sub-block, two bursts (R4; same result as upper_bound).
+__device__ __forceinline__ int64_t upper_bound_64(const int64_t* b, int m, const int64_t* smp8, int j0, int64_t x) {
+  if (j0 * 64 >= m) return m;
+  const int j1 = 8 * j0 + count_le8(smp8 + 8 * j0, x);
+  if (j1 * 8 >= m) return m;
+  return (int64_t)j1 * 8 + count_le8(b + 8 * j1, x);
+}
+
+// MapId (R8) whose first probe kv0 = table slot of x was loaded ahead (no
+// INT64_MIN key; x may be INT64_MIN only if the table misses it).
+__device__ __forceinline__ int64_t map_lookup_from(const int64_t* itab, int64_t a, int m, int64_t dflt, int64_t x,
+                                                   longlong2 kv) {
+  if (x == INT64_MIN) return dflt;
+  const longlong2* t = reinterpret_cast<const longlong2*>(itab + a);
+  const uint32_t mask = (1u << m) - 1u;
+  uint32_t i = (uint32_t)(((uint64_t)x * 0x9E3779B97F4A7C15ull) >> (64 - m));
+  while (true) {
+    if (kv.x == x) return kv.y;
+    if (kv.x == INT64_MIN) return dflt;
+    i = (i + 1) & mask;
+    kv = __ldg(t + i);
+  }
+}
+__device__ __forceinline__ longlong2 map_first_probe(const int64_t* itab, int64_t a, int m, int64_t x) {
+  const longlong2* t = reinterpret_cast<const longlong2*>(itab + a);
+  return __ldg(t + (uint32_t)(((uint64_t)x * 0x9E3779B97F4A7C15ull) >> (64 - m)));
 }
 
 __device__ __forceinline__ int64_t upper_bound_s(const float* b, int m, float x) {  // shared-memory borders

@@ -13,7 +13,23 @@
 //    units that produce up to kGroupCols adjacent output columns.
 // DESIGN.md §7 describes the layout.
 #pragma once
+#ifdef __CUDACC_RTC__
+// NVRTC (the plan-specialised kernel, rap_jit.cpp): no system headers
+typedef signed char int8_t;
+typedef short int16_t;
+typedef int int32_t;
+typedef long long int64_t;
+typedef unsigned char uint8_t;
+typedef unsigned short uint16_t;
+typedef unsigned int uint32_t;
+typedef unsigned long long uint64_t;
+typedef unsigned long long uintptr_t;
+#define INT32_MAX 2147483647
+#define INT64_MAX 9223372036854775807LL
+#define INT64_MIN (-INT64_MAX - 1LL)
+#else
 #include <stdint.h>
+#endif
 
 #ifdef __CUDACC__
 #define RAP_HD __host__ __device__ __forceinline__
@@ -253,10 +269,13 @@ struct RbGeom {
   int32_t n_rb, n_fg, rows_rb, max_fl;  // row blocks, feature groups, rows per block (x32), max outputs per group
   int32_t max_cols, dense_bytes;        // max raw sparse columns one group stages; dense-phase smem bytes
   int32_t n_memo, small;                // memo slots; small = 1: every base fits 31 bits (32-bit scans)
+  int32_t len_cache, pad2;              // 1: the kernel keeps a uint16 length cache per (output, row) in smem
+  unsigned long long all_cols;          // raw sparse columns the outputs read (bit c: column c < 64)
   const RbFeat* feat;                   // [n_sparse_out], by output index
   const int32_t* perm;                  // [n_sparse_out] processing order (groups are ranges of it)
-  unsigned long long* agg;              // [n_sparse_out * n_rb] per-(output, row block) totals, feature-major
+  unsigned long long* agg;              // [n_sparse_out][n_rb] per-(output, row block) totals
   unsigned long long* sched;            // [0] CTAs done, [2] CTAs whose totals are stored (reset by the last CTA)
+  unsigned long long* tot;              // [n_sparse_out] per-output totals (red.add; zeroed by the last CTA)
   int32_t fg_off[kRbMaxFg + 1];         // group g = perm[fg_off[g] .. fg_off[g + 1])
 };
 
@@ -272,10 +291,44 @@ int launch_jagged_append(const int32_t* len, const int64_t* so, const int64_t* v
 // Occupancy query: CTAs per SM for the given dynamic smem.
 int fused_occupancy(int smem_bytes, int n_dense, int n_sparse, int* ctas_per_sm);
 // Row-block kernel (rap_rows.cu): dynamic smem for a geometry, occupancy, launch.
-int rows_smem_bytes(int dense_bytes, int max_fl, int max_cols, int n_memo, int n_sparse_out);
+int rows_smem_bytes(int dense_bytes, int max_fl, int max_cols, int n_memo, int n_sparse_out, int len_cache);
 // Dense-phase shared memory of the row-block kernel for dense groups up to max_width columns.
 int rows_dense_bytes(int max_width);
 int rows_occupancy(int smem_bytes, int* ctas_per_sm);
 int launch_rows(const Common& c, const RbGeom& g, const LaunchRaw& raw, int smem_bytes, void* stream);
+
+#ifndef __CUDACC_RTC__
+// ---- Plan-specialised row-block kernel (rap_jit.cpp) ----
+// The planner's view of a plan that the code generator reads.
+struct JitPlanView {
+  int n_sparse_out, n_sparse_in;
+  const RbFeat* feat;    // [n_sparse_out]
+  const SProg* sprogs;   // [n_sparse_out]
+  const int32_t* perm;   // [n_sparse_out] processing order
+  const int* used_sparse;
+  int n_used_sparse;
+  // dense outputs (DProg column groups, rap_internal.h)
+  const DProg* dprogs;
+  int n_dprogs, d_out, dense_bytes;  // dense_bytes: the kernel's dense-phase shared memory
+  const int64_t* itab;               // the plan's int64 table pool (Bucketize borders, MapId tables)
+};
+struct JitModule;  // compiled kernels (opaque)
+// Generate the CUDA source of the plan's policy (small: 32-bit scans, every
+// offset < 2^31; else 64-bit) and compile it with NVRTC for sm_100a (cached
+// per source text in the process).  Returns nullptr and fills *log on failure.
+JitModule* jit_build(const JitPlanView& v, bool small, char* log, int log_cap);
+int jit_occupancy(JitModule* m, int smem_bytes, int* ctas_per_sm);
+int launch_jit(JitModule* m, const Common& c, const RbGeom& g, const LaunchRaw& raw, int smem_bytes, void* stream);
+double jit_compile_seconds(const JitModule* m);
+#endif
+}  // namespace rapk
+#if !defined(__CUDACC_RTC__) && defined(__cplusplus)
+#include <string>
+namespace rapk {
+std::string jit_generate(const JitPlanView& v);
+bool jit_compile_only(const std::string& src, std::string* log);
+}  // namespace rapk
+#endif
+namespace rapk {
 
 }  // namespace rapk

@@ -1,0 +1,671 @@
+// rap_jit.cpp — plan-specialised row-block kernel: a code generator plus
+// NVRTC (the B200-native form of RAP's code generator, §4
+// L854-857: the optimizer's plan becomes "optimized CUDA kernels").
+//
+// For a plan, the generator writes one policy for the row-block kernel
+// skeleton (rap_rows_skel.cuh): every sparse output's closed-form length and
+// its chain as straight-line code, in the planner's processing order, with
+// every parameter (caps, fills, Clamp bounds, H(salt), M, MapId / Bucketize
+// table offsets) an immediate and the staged column slots constants.  An
+// NGram output over sources another output already hashed reads them from
+// registers (the provider's element 0, rows with at most one id).  Anything
+// else (non-canonical chains, dense-bucket sources, rows with longer lists)
+// calls the interpreter's generic functions (rap_rows_interp.cuh), so the
+// generated kernel computes exactly what the interpreter computes (R1-R20).
+// The source is compiled with NVRTC for sm_100a once per distinct plan source
+// in the process and loaded as a cudaLibrary; the launch path is the same
+// cooperative launch as rap_rows.cu.
+#include <cuda_runtime.h>
+#include <nvrtc.h>
+#include <math.h>
+#include <stdio.h>
+#include <string.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cstdlib>
+#include <cinttypes>
+#include <map>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "rap_internal.h"
+
+namespace rapk {
+
+// Header texts (generated from the csrc/ headers at build time by _build.py).
+#include "rap_jit_embed.inc"
+
+struct JitModule {
+  cudaLibrary_t lib = nullptr;
+  cudaKernel_t k = nullptr;
+  int smem_set = -1;
+  double compile_s = 0;
+  std::mutex mu;
+};
+
+namespace {
+
+std::string lit64(int64_t v) {
+  if (v == INT64_MIN) return "(-9223372036854775807LL - 1LL)";
+  return std::to_string(v) + "LL";
+}
+std::string litu64(uint64_t v) { return std::to_string(v) + "ULL"; }
+std::string i2s(long long v) { return std::to_string(v); }
+std::string f2lit(float f) {  // exact (hex float)
+  if (f != f) return "__int_as_float(0x7fc00000)";
+  if (f == INFINITY) return "__int_as_float(0x7f800000)";
+  if (f == -INFINITY) return "__int_as_float(0xff800000)";
+  char buf[64];
+  snprintf(buf, sizeof(buf), "%af", (double)f);
+  return buf;
+}
+
+struct Gen {
+  const JitPlanView& v;
+  int F;
+  std::vector<int> slot;     // raw column -> staged slot (rank among the columns the outputs read)
+  std::vector<int> provider; // per output f: a memo provider for NGram source i? see prov_out
+  std::string out;
+
+  explicit Gen(const JitPlanView& view) : v(view), F(view.n_sparse_out) {
+    std::vector<char> used(std::max(1, view.n_sparse_in), 0);
+    for (int f = 0; f < F; ++f) {
+      const RbFeat& R = v.feat[f];
+      const int kk = R.kind == 1 ? 0 : R.k;
+      for (int i = 0; i < kk; ++i)
+        if (R.src[i] >= 0) used[R.src[i]] = 1;
+    }
+    slot.assign(used.size(), -1);
+    int n = 0;
+    for (size_t c = 0; c < used.size(); ++c)
+      if (used[c]) slot[c] = n++;
+  }
+
+  static std::string cap_expr(const std::string& X, int cap) {
+    if (cap >= INT32_MAX) return "max(" + X + ".b - " + X + ".a, 0)";
+    return "min(max(" + X + ".b - " + X + ".a, 0), " + i2s(cap) + ")";
+  }
+
+  // int32_t L<q> (and RbRow X<q>_<i>, int32_t l<q>_<i> for NGram sources)
+  std::string len_code(int q) {
+    const int f = v.perm[q];
+    const RbFeat& R = v.feat[f];
+    const std::string Q = i2s(q);
+    std::string s;
+    if (R.kind == 1) return "    const int32_t L" + Q + " = in ? " + i2s(R.out_cap) + " : 0;\n";
+    if (R.kind == 0) {
+      const std::string X = "X" + Q + "_0";
+      s += "    const RbRow " + X + " = rb_row(s, " + i2s(slot[R.src[0]]) + ", r);\n";
+      s += "    const int32_t L" + Q + " = !in ? 0 : (" + X + ".valid ? " + cap_expr(X, R.cap[0]) + " : " +
+           i2s(R.ncap[0]) + ");\n";
+      return s;
+    }
+    std::string sum = "0LL";
+    for (int i = 0; i < R.k; ++i) {
+      const std::string l = "l" + Q + "_" + i2s(i);
+      if (R.src[i] < 0) {
+        s += "    const int32_t " + l + " = " + i2s(R.cap[i]) + ";\n";
+      } else {
+        const std::string X = "X" + Q + "_" + i2s(i);
+        s += "    const RbRow " + X + " = rb_row(s, " + i2s(slot[R.src[i]]) + ", r);\n";
+        s += "    const int32_t " + l + " = " + X + ".valid ? " + cap_expr(X, R.cap[i]) + " : " + i2s(R.ncap[i]) +
+             ";\n";
+      }
+      sum += " + " + l;
+    }
+    s += "    const int32_t L" + Q + " = !in ? 0 : (int32_t)min(max((long long)(" + sum + ") - " + i2s(R.n) +
+         "LL + 1LL, 0LL), " + i2s(R.out_cap) + "LL);\n";
+    return s;
+  }
+
+  // Canonical stages (R6, R8, R1-R3, R4) on variable x; memo: store after
+  // stage bit memo_after into variable mvar (16: before the first stage).
+  std::string stages(const Canon& q, int mask, const std::string& x, const std::string& full, int memo_after,
+                     const std::string& mvar, const std::string& probe = "") {
+    std::string s;
+    auto cond = [&](int bit) { return (q.null_mask & bit) ? std::string() : "if (" + full + ") "; };
+    if (memo_after == 16) s += "        " + mvar + " = " + x + ";\n";
+    if (mask & CB_CLAMP) {
+      s += "        " + cond(CB_CLAMP) + "{ " + x + " = " + x + " < " + lit64(q.lo) + " ? " + lit64(q.lo) + " : " + x +
+           "; " + x + " = " + x + " > " + lit64(q.hi) + " ? " + lit64(q.hi) + " : " + x + "; }\n";
+      if (memo_after == CB_CLAMP) s += "        " + mvar + " = " + x + ";\n";
+    }
+    if (mask & CB_MAPID) {
+      if (!probe.empty())  // first probe loaded ahead
+        s += "        " + cond(CB_MAPID) + x + " = map_lookup_from(c.itab, " + lit64(q.map_a) + ", " + i2s(q.map_m) + ", " +
+             lit64(q.map_def) + ", " + x + ", " + probe + ");\n";
+      else
+        s += "        " + cond(CB_MAPID) + x + " = map_lookup(c.itab, " + lit64(q.map_a) + ", " + i2s(q.map_m) + ", " +
+             lit64(q.map_def) + ", 0, 0, " + x + ");\n";
+      if (memo_after == CB_MAPID) s += "        " + mvar + " = " + x + ";\n";
+    }
+    if (mask & CB_SIGRID) {
+      s += "        " + cond(CB_SIGRID) + x + " = (int64_t)reduce_M(splitmix_H(" + litu64(q.hs) + " ^ (uint64_t)" + x +
+           "), " + lit64(q.M) + ");\n";
+      if (memo_after == CB_SIGRID) s += "        " + mvar + " = " + x + ";\n";
+    }
+    if (mask & CB_BUCKET) {
+      if (q.bk_m >= 64 && q.bk_m % 64 == 0 && q.bk_a % 2 == 0) {
+        // three levels: the maxima of the 64-border blocks as immediates, then
+        // one burst of 8 sub-block maxima and one of 8 borders (R4)
+        const std::string nm = sample_table(q.bk_a, q.bk_m);
+        s += "        " + cond(CB_BUCKET) + "{ const int j0 = 0";
+        for (int k = 0; k < q.bk_m / 64; ++k) s += " + (" + x + " >= " + lit64(v.itab[q.bk_a + 64 * k + 63]) + ")";
+        s += "; " + x + " = upper_bound_64(c.itab + " + lit64(q.bk_a) + ", " + i2s(q.bk_m) + ", " + nm + ", j0, " + x +
+             "); }\n";
+      } else if (q.bk_m >= 64) {  // two-level search over a sample table in the module
+        const std::string nm = sample_table(q.bk_a, q.bk_m);
+        s += "        " + cond(CB_BUCKET) + x + " = upper_bound_s8(c.itab + " + lit64(q.bk_a) + ", " + i2s(q.bk_m) +
+             ", " + nm + ", " + i2s(q.bk_m / 8) + ", " + x + ");\n";
+      } else {
+        s += "        " + cond(CB_BUCKET) + x + " = upper_bound(c.itab + " + lit64(q.bk_a) + ", " + i2s(q.bk_m) + ", " +
+             x + ");\n";
+      }
+      if (memo_after == CB_BUCKET) s += "        " + mvar + " = " + x + ";\n";
+    }
+    return s;
+  }
+
+  // __device__ table of every 8th border of itab[a .. a+m) (upper_bound_s8)
+  std::map<int64_t, std::string> samples;
+  std::string sample_globals;
+  std::string sample_table(int64_t a, int m) {
+    auto it = samples.find(a);
+    if (it != samples.end()) return it->second;
+    const std::string nm = "kS" + i2s((long long)samples.size());
+    sample_globals += "__device__ __align__(16) const int64_t " + nm + "[" + i2s(std::max(1, m / 8)) + "] = {";
+    for (int i = 0; i < m / 8; ++i) sample_globals += (i ? ", " : "") + lit64(v.itab[a + 8 * i + 7]);
+    if (m / 8 == 0) sample_globals += "0";
+    sample_globals += "};\n";
+    samples[a] = nm;
+    return nm;
+  }
+
+  static int memo_point(const RbFeat& R, const Canon& cn) {
+    if (R.memo_slot < 0) return -1;
+    const int pm = R.memo_mask & cn.mask;
+    if (pm == 0) return 16;
+    int ma = 1;
+    while ((pm >> 1) >= ma) ma <<= 1;
+    return ma;
+  }
+
+  // ---- dense outputs (a2): thread per row, units split over two halves ----
+  int pitch() const { return v.d_out | 1; }
+  bool gen_dense_ok() const {
+    if (v.n_dprogs == 0 || v.d_out <= 0) return false;
+    return 128 * pitch() * 4 <= v.dense_bytes;
+  }
+  static double unit_cost(const DProg& dp, const DUnit& un) {
+    const DevOp* ops = dp.ops;
+    double c = 8;
+    if (un.kind == U_ONEHOT_G) return 200;
+    if (!un.gops)
+      for (int o = un.op_begin; o < un.op_end; ++o)
+        c += ops[o].kind == OK_LOGIT ? 40 : ops[o].kind == OK_BOXCOX ? 70 : 3;
+    if (un.kind == U_ONEHOT_DB) c += 10 + un.width + un.bm / 2;
+    return c;
+  }
+  std::string dense_ops(const DevOp* ops, int o0, int o1, const std::string& x) {
+    std::string s;
+    for (int o = o0; o < o1; ++o) {
+      const DevOp& op = ops[o];
+      if (op.kind == OK_FILL_F) {
+        s += "        if (isnan(" + x + ")) " + x + " = " + f2lit(op.f0) + ";\n";  // R10
+      } else if (op.kind == OK_LOGIT) {                                          // R11
+        s += "        { const float z = " + x + " < " + f2lit(op.f0) + " ? " + f2lit(op.f0) + " : (" + x + " > " +
+             f2lit(op.f1) + " ? " + f2lit(op.f1) + " : " + x + "); " + x + " = logf(__fdiv_rn(z, __fsub_rn(1.0f, z))); }\n";
+      } else if (op.f0 == 0.0f) {  // R12, lambda = 0
+        s += "        " + x + " = logf(" + x + ");\n";
+      } else {  // R12
+        s += "        " + x + " = __fdiv_rn(expm1f(__fmul_rn(" + f2lit(op.f0) + ", logf(" + x + "))), " + f2lit(op.f0) +
+             ");\n";
+      }
+    }
+    return s;
+  }
+  std::string id_ops(const DevOp* ops, int o0, int o1, const std::string& b) {
+    std::string s;
+    for (int o = o0; o < o1; ++o) {
+      const DevOp& op = ops[o];
+      if (op.kind == OK_CLAMP) {
+        s += "        " + b + " = " + b + " < " + lit64(op.a) + " ? " + lit64(op.a) + " : " + b + "; " + b + " = " + b +
+             " > " + lit64(op.b) + " ? " + lit64(op.b) + " : " + b + ";\n";
+      } else if (op.kind == OK_SIGRID) {
+        s += "        " + b + " = (int64_t)reduce_M(splitmix_H(" + litu64(op.hsalt) + " ^ (uint64_t)" + b + "), " +
+             lit64(op.M) + ");\n";
+      } else if (op.kind == OK_BUCKET_I) {
+        s += "        " + b + " = upper_bound(c.itab + " + lit64(op.a) + ", " + i2s(op.m) + ", " + b + ");\n";
+      } else {  // OK_MAPID
+        s += "        " + b + " = map_lookup(c.itab, " + lit64(op.a) + ", " + i2s(op.m) + ", " + lit64(op.b) + ", " +
+             i2s((int)op.M) + ", " + lit64((int64_t)op.hsalt) + ", " + b + ");\n";
+      }
+    }
+    return s;
+  }
+  std::string dense_unit(int gi, int ui, std::string* globals) {
+    const DProg& dp = v.dprogs[gi];
+    const DUnit& un = dp.units[ui];
+    const int col = dp.col0 + un.col;  // absolute output column
+    std::string s = "      {  // dense unit " + i2s(gi) + "." + i2s(ui) + "\n";
+    if (un.kind == U_ONEHOT_G) {  // generic list (R9): the interpreter's code
+      s += "        for (int k = 0; k < " + i2s(un.width) + "; ++k) trow[" + i2s(col) + " + k] = 0.0f;\n";
+      s += "        onehot_generic(p, p.c.dprogs[" + i2s(gi) + "].units[" + i2s(ui) + "], row, trow + " + i2s(dp.col0) +
+           ");\n      }\n";
+      return s;
+    }
+    s += "        float v = in" + i2s(un.src_col) + ";\n";
+    s += dense_ops(dp.ops, un.op_begin, un.op_end, "v");
+    if (un.kind == U_DENSE) {
+      s += "        trow[" + i2s(col) + "] = v;\n      }\n";
+      return s;
+    }
+    // U_ONEHOT_DB: Bucketize (f32 borders, R4) -> id ops -> OneHot (R9)
+    if (un.xcap <= 0) {
+      s += "        for (int k = 0; k < " + i2s(un.width) + "; ++k) trow[" + i2s(col) + " + k] = 0.0f;\n      }\n";
+      return s;
+    }
+    const float* bt = dp.ftab + un.btab;
+    if (un.bm <= 32) {
+      s += "        int64_t b = 0";
+      for (int i = 0; i < un.bm; ++i) s += " + (v >= " + f2lit(bt[i]) + ")";
+      s += ";\n";
+    } else {
+      const std::string nm = "kB" + i2s(gi) + "_" + i2s(ui);
+      *globals += "__device__ const float " + nm + "[" + i2s(un.bm) + "] = {";
+      for (int i = 0; i < un.bm; ++i) *globals += (i ? ", " : "") + f2lit(bt[i]);
+      *globals += "};\n";
+      s += "        int64_t b = upper_bound(" + nm + ", " + i2s(un.bm) + ", v);\n";
+    }
+    s += id_ops(dp.ops, un.iop_begin, un.iop_end, "b");
+    s += "        const int64_t d = b - " + lit64(un.k0) + ";\n";
+    s += "#pragma unroll\n        for (int k = 0; k < " + i2s(un.width) + "; ++k) trow[" + i2s(col) +
+         " + k] = d == k ? 1.0f : 0.0f;\n      }\n";
+    return s;
+  }
+  std::string dense_fn(std::string* globals) {
+    std::string s;
+    const bool ok = gen_dense_ok();
+    s += "  static constexpr bool kGenDense = " + std::string(ok ? "true" : "false") + ";\n";
+    s += "  template <class P>\n  static __device__ __forceinline__ void dense(const P& p, const RbSmem& s, const RbCtx& x) {\n";
+    if (!ok) return s + "  }\n";
+    // split the units over the two halves of the CTA by predicted cost
+    std::vector<std::pair<int, int>> half[2];
+    double load[2] = {0, 0};
+    std::vector<std::pair<double, std::pair<int, int>>> units;
+    for (int gi = 0; gi < v.n_dprogs; ++gi)
+      for (int ui = 0; ui < v.dprogs[gi].n_units; ++ui)
+        units.push_back({unit_cost(v.dprogs[gi], v.dprogs[gi].units[ui]), {gi, ui}});
+    std::stable_sort(units.begin(), units.end(), [](const auto& a, const auto& b) { return a.first > b.first; });
+    for (const auto& u : units) {
+      const int h = load[0] <= load[1] ? 0 : 1;
+      load[h] += u.first;
+      half[h].push_back(u.second);
+    }
+    s += "    const Common& c = p.c;\n";
+    s += "    const int tid = threadIdx.x, r = tid & 127, half = tid >> 7;\n";
+    s += "    float* tile = reinterpret_cast<float*>(s.dense);  // [128][" + i2s(pitch()) + "]\n";
+    s += "    for (int64_t d0 = x.R0; d0 < x.R1; d0 += 128) {\n";
+    s += "      const int nr = (int)min((int64_t)128, x.R1 - d0);\n";
+    s += "      if (r < nr) {\n        const int64_t row = d0 + r;\n";
+    s += "        float* trow = tile + r * " + i2s(pitch()) + ";\n";
+    for (int h = 0; h < 2; ++h) {
+      s += std::string(h == 0 ? "        if (half == 0) {\n" : "        } else {\n");
+      // every raw value of the half first (independent loads in flight), then the chains
+      std::vector<int> cols;
+      for (const auto& u : half[h]) {
+        const DUnit& un = v.dprogs[u.first].units[u.second];
+        if (un.kind != U_ONEHOT_G && std::find(cols.begin(), cols.end(), un.src_col) == cols.end())
+          cols.push_back(un.src_col);
+      }
+      for (int cc : cols) s += "        const float in" + i2s(cc) + " = rb_dense_in(p, " + i2s(cc) + ", row);\n";
+      for (const auto& u : half[h]) s += dense_unit(u.first, u.second, globals);
+    }
+    s += "        }\n      }\n      __syncthreads();\n";
+    s += "      rb_tile_store(c, tile, " + i2s(pitch()) + ", " + i2s(v.d_out) + ", d0, nr);\n      __syncthreads();\n    }\n  }\n";
+    return s;
+  }
+
+  std::string lengths_fn() {
+    std::string s;
+    s += "  template <bool kSmall, class P>\n"
+         "  static __device__ __forceinline__ void lengths(const P& p, const RbSmem& s, const RbCtx& x, int nr, "
+         "bool acc) {\n"
+         "    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, r = tid;\n"
+         "    const bool in = tid < nr;\n";
+    // batches of 8 outputs: every staged load of a batch before its warp sums
+    // are stored (a shared store would otherwise order the next loads)
+    for (int q0 = 0; q0 < F; q0 += 8) {
+      const int q1 = std::min(F, q0 + 8);
+      s += "  {\n";
+      for (int q = q0; q < q1; ++q) s += len_code(q);
+      for (int q = q0; q < q1; ++q) s += "    const long long w" + i2s(q) + " = rb_warp_sum<kSmall>(L" + i2s(q) + ");\n";
+      s += "    if (lane == 0) {\n";
+      for (int q = q0; q < q1; ++q)
+        s += "      s.ws[" + i2s(q * 8) + " + warp] = acc ? s.ws[" + i2s(q * 8) + " + warp] + w" + i2s(q) + " : w" + i2s(q) +
+             ";\n";
+      s += "    }\n  }\n";
+    }
+    s += "  }\n";
+    return s;
+  }
+
+  std::string emit_fn() {
+    std::string s;
+    s += "  template <bool kSmall, class P>\n"
+         "  static __device__ __forceinline__ void emit(const P& p, const RbSmem& s, const RbCtx& x, int64_t c0, "
+         "int nr) {\n"
+         "    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, r = tid;\n"
+         "    const Common& c = p.c;\n"
+         "    const int64_t B = x.B;\n"
+         "    const bool in = tid < nr;\n"
+         "    const int64_t row = c0 + tid;\n";
+    // memo registers of the providers
+    std::vector<char> is_prov(F, 0);
+    for (int f = 0; f < F; ++f)
+      if (v.feat[f].emit == 0 && v.feat[f].memo_slot >= 0) is_prov[f] = 1;
+    for (int f = 0; f < F; ++f)
+      if (is_prov[f]) s += "    int64_t m" + i2s(f) + " = 0;\n    int32_t ml" + i2s(f) + " = 0;\n";
+    // first ids of the canonical list outputs, loaded kAhead outputs before
+    // their use (the load latency hides under the outputs in between)
+    const int kAhead = 4;
+    std::vector<int> canon_q;
+    for (int q = 0; q < F; ++q)
+      if (v.feat[v.perm[q]].emit == 0) canon_q.push_back(q);
+    auto prefetch = [&](int q) {
+      const RbFeat& R = v.feat[v.perm[q]];
+      const std::string Y = "Y" + i2s(q);
+      return "    int64_t pf" + i2s(q) + " = 0;\n    { const RbRow " + Y + " = rb_row(s, " + i2s(slot[R.src[0]]) +
+             ", r);\n      if (in && " + Y + ".valid && " + Y + ".b > " + Y + ".a) pf" + i2s(q) + " = __ldg(p.val[" +
+             i2s(R.src[0]) + "] + " + Y + ".a); }\n";
+    };
+    // MapId outputs: their first table probe is loaded kProbe outputs ahead,
+    // from the prefetched id run through the stages before MapId
+    const int kProbe = 2;
+    auto has_map = [&](int q) { return (v.sprogs[v.perm[q]].cn.mask & CB_MAPID) != 0; };
+    auto probe = [&](int q) {
+      const int f = v.perm[q];
+      const RbFeat& R = v.feat[f];
+      const SProg& pg = v.sprogs[f];
+      const Canon& cn = pg.cn;
+      const std::string Q = i2s(q), Z = "Z" + Q;
+      std::string t = "    longlong2 pk" + Q + ";\n    { const RbRow " + Z + " = rb_row(s, " + i2s(slot[R.src[0]]) +
+                      ", r);\n      int64_t u = " + Z + ".valid ? pf" + Q + " : " + lit64(pg.ch.fill) + ";\n";
+      t += stages(cn, cn.mask & CB_CLAMP, "u", Z + ".valid", -1, "");
+      t += "      pk" + Q + " = map_first_probe(c.itab, " + lit64(cn.map_a) + ", " + i2s(cn.map_m) + ", u); }\n";
+      return t;
+    };
+    for (int i = 0; i < (int)canon_q.size() && i < kAhead; ++i) s += prefetch(canon_q[i]);
+    for (int i = 0; i < (int)canon_q.size() && i < kProbe; ++i)
+      if (has_map(canon_q[i])) s += probe(canon_q[i]);
+    int canon_i = 0;
+    for (int q = 0; q < F; ++q) {
+      const int f = v.perm[q];
+      const RbFeat& R = v.feat[f];
+      const SProg& pg = v.sprogs[f];
+      const std::string Q = i2s(q), Fs = i2s(f);
+      if (R.emit == 0) {
+        if (canon_i + kAhead < (int)canon_q.size()) s += prefetch(canon_q[canon_i + kAhead]);
+        if (canon_i + kProbe < (int)canon_q.size() && has_map(canon_q[canon_i + kProbe]))
+          s += probe(canon_q[canon_i + kProbe]);
+        ++canon_i;
+      }
+      s += "  {  // output " + Fs + "\n" + len_code(q);
+      s += "    const long long P" + Q + " = s.wb[" + i2s(q * 8) + " + warp] + rb_warp_excl<kSmall>(L" + Q +
+           ", lane);\n";
+      if (is_prov[f]) s += "    ml" + Fs + " = L" + Q + ";\n";
+      s += "    if (in) {\n";
+      s += "      const int64_t oi = (int64_t)" + Fs + " * B + row;\n";
+      s += "      rb_store_lo(c, oi, L" + Q + ", P" + Q + ");\n";
+      if (f == F - 1) s += "      if (row == B - 1) stg_s64(c.offsets + (int64_t)" + i2s(F) + " * B, P" + Q + " + L" + Q + ");\n";
+      s += "      if (L" + Q + " > 0) {\n";
+      if (R.emit == 0) {
+        const Canon& cn = pg.cn;
+        const std::string X = "X" + Q + "_0";
+        const int col = R.src[0];
+        s += "        int64_t v = " + X + ".valid ? pf" + Q + " : " + lit64(pg.ch.fill) + ";\n";
+        s += stages(cn, cn.mask, "v", X + ".valid", is_prov[f] ? memo_point(R, cn) : -1, "m" + Fs,
+                    (cn.mask & CB_MAPID) ? "pk" + Q : "");
+        s += "        rb_store(c, P" + Q + ", v);\n";
+        if (R.cap[0] > 1) {
+          s += "        for (int32_t j = 1; j < L" + Q + "; ++j) {\n";
+          s += "          int64_t w = __ldg(p.val[" + i2s(col) + "] + " + X + ".a + j);\n";
+          s += stages(cn, cn.mask, "w", "true", -1, "");
+          s += "          rb_store(c, P" + Q + " + j, w);\n        }\n";
+        }
+      } else if (R.emit == 3 && ngram_fast_ok(q)) {
+        // every source memoised by an earlier provider: push the present
+        // elements through an n-register window (R7)
+        const int n = R.n, K = R.k;
+        std::string cond;
+        for (int i = 0; i < K; ++i) {
+          const int fp = v.perm[R.prov[i]];
+          const std::string l = "l" + Q + "_" + i2s(i);
+          if (i) cond += " && ";
+          cond += "(" + l + " <= 1 && (" + l + " == 0 || ml" + i2s(fp) + " >= 1))";
+        }
+        s += "        if (" + cond + ") {\n";
+        s += "          int32_t cnt = 0;\n";
+        for (int j = 0; j < n; ++j) s += "          uint64_t w" + i2s(j) + " = 0;\n";
+        for (int i = 0; i < K; ++i) {
+          const int fp = v.perm[R.prov[i]];
+          s += "          if (l" + Q + "_" + i2s(i) + ") {\n";
+          for (int j = 0; j + 1 < n; ++j) s += "            w" + i2s(j) + " = w" + i2s(j + 1) + ";\n";
+          s += "            w" + i2s(n - 1) + " = (uint64_t)m" + i2s(fp) + ";\n            ++cnt;\n";
+          if (i + 1 >= n) {
+            s += "            if (cnt >= " + i2s(n) + " && cnt - " + i2s(n) + " < L" + Q + ") {\n";
+            s += "              uint64_t h = " + litu64(pg.ng.hsalt) + ";\n";
+            for (int j = 0; j < n; ++j) s += "              h = splitmix_H(h ^ w" + i2s(j) + ");\n";
+            s += "              int64_t v = (int64_t)reduce_M(h, " + lit64(pg.ng.M) + ");\n";
+            s += stages(pg.cn, pg.cn.mask, "v", "true", -1, "");
+            s += "              rb_store(c, P" + Q + " + (cnt - " + i2s(n) + "), v);\n            }\n";
+          }
+          s += "          }\n";
+        }
+        s += "        } else {\n";
+        s += "          rb_emit_ngram(p, s, s.feat[" + Q + "], -1, r, row, L" + Q + ", P" + Q + ", 0);\n";
+        s += "        }\n";
+      } else if (R.emit == 3) {
+        s += "        rb_emit_ngram(p, s, s.feat[" + Q + "], -1, r, row, L" + Q + ", P" + Q + ", 0);\n";
+      } else {
+        s += "        rb_emit_generic(p, s, s.feat[" + Q + "], r, row, L" + Q + ", P" + Q + ");\n";
+      }
+      s += "      }\n    }\n  }\n";
+    }
+    s += "  }\n";
+    return s;
+  }
+
+  // NGram q can take the register path: canonical post stages, every source
+  // a raw list with a provider processed before it.
+  bool ngram_fast_ok(int q) {
+    const int f = v.perm[q];
+    const RbFeat& R = v.feat[f];
+    const SProg& pg = v.sprogs[f];
+    if (!pg.cn.ok || R.n < 1 || R.n > kMaxNgramK) return false;
+    for (int i = 0; i < R.k; ++i) {
+      if (R.src[i] < 0 || R.prov[i] < 0 || R.prov[i] >= q) return false;
+      const int fp = v.perm[R.prov[i]];
+      if (v.feat[fp].emit != 0 || v.feat[fp].memo_slot < 0) return false;
+    }
+    return true;
+  }
+
+  std::string source(bool small) {
+    std::string s;
+    s += "// generated by rap_jit.cpp for one plan (" + i2s(F) + " sparse outputs)\n";
+    s += "#include \"rap_rows_interp.cuh\"\n\nnamespace rapk {\n\n";
+    bool records = false;  // does any output fall back to the interpreter's functions?
+    for (int f = 0; f < F; ++f) records |= v.feat[f].emit != 0;
+    std::string globals;
+    const std::string dense = dense_fn(&globals);
+    std::string body;
+    body += "struct JitPolicy {\n";
+    body += "  static constexpr bool kSetupEarly = false;  // records only feed the fallbacks of (4)\n";
+    body += "  template <class P>\n"
+            "  static __device__ __forceinline__ void setup(const P& p, const RbSmem& s, const RbCtx& x) {\n";
+    if (records) body += "    InterpPolicy::setup(p, s, x);  // records for the generic fallbacks\n";
+    body += "  }\n";
+    body += dense;
+    body += lengths_fn();
+    body += emit_fn();
+    body += "};\n\n}  // namespace rapk\n\n";
+    s += globals + sample_globals + "\n" + body;
+    // one variant per module: 32-bit scans (every offset < 2^31) or 64-bit
+    const char* mb = getenv("RAP_JIT_MINB");  // CTAs per SM the register budget targets (default 2)
+    s += "extern \"C\" __global__ void __launch_bounds__(rapk::kRbChunk, " + std::string(mb ? mb : "2") +
+         ") rap_jit_kernel(const __grid_constant__ "
+         "rapk::RbParams<rapk::kRbMaxDense, rapk::kRbMaxCols> p) {\n"
+         "  rapk::rows_body<rapk::JitPolicy, rapk::kRbMaxDense, rapk::kRbMaxCols, " +
+         std::string(small ? "true" : "false") + ">(p);\n}\n";
+    return s;
+  }
+};
+
+std::mutex g_cache_mu;
+std::map<std::string, JitModule*>* g_cache = nullptr;  // per process, never freed (kernels stay loaded)
+
+void put_log(char* log, int cap, const std::string& msg) {
+  if (!log || cap <= 0) return;
+  snprintf(log, (size_t)cap, "%s", msg.c_str());
+}
+
+}  // namespace
+
+namespace {
+
+// NVRTC: the plan source -> sm_100a CUBIN.  false + log on failure.
+bool nvrtc_cubin(const std::string& src, std::vector<char>* cubin, std::string* log) {
+  nvrtcProgram prog;
+  const char* hdrs[] = {kJitHdrInternal, kJitHdrDevice, kJitHdrSkel, kJitHdrInterp};
+  const char* names[] = {"rap_internal.h", "rap_device.cuh", "rap_rows_skel.cuh", "rap_rows_interp.cuh"};
+  nvrtcResult r = nvrtcCreateProgram(&prog, src.c_str(), "rap_jit_plan.cu", 4, hdrs, names);
+  if (r != NVRTC_SUCCESS) {
+    *log = std::string("nvrtcCreateProgram: ") + nvrtcGetErrorString(r);
+    return false;
+  }
+  const char* opts[] = {"--gpu-architecture=sm_100a", "-std=c++17", "-lineinfo", "-ftz=false", "-prec-div=true",
+                        "-prec-sqrt=true", "-fmad=true", "-default-device"};
+  r = nvrtcCompileProgram(prog, (int)(sizeof(opts) / sizeof(opts[0])), opts);
+  size_t n = 0;
+  nvrtcGetProgramLogSize(prog, &n);
+  std::string lg(n, '\0');
+  if (n) nvrtcGetProgramLog(prog, &lg[0]);
+  if (r != NVRTC_SUCCESS) {
+    nvrtcDestroyProgram(&prog);
+    *log = "NVRTC compile failed: " + lg.substr(0, 3000);
+    return false;
+  }
+  size_t cn = 0;
+  nvrtcGetCUBINSize(prog, &cn);
+  cubin->resize(cn);
+  nvrtcGetCUBIN(prog, cubin->data());
+  nvrtcDestroyProgram(&prog);
+  *log = lg;
+  return true;
+}
+
+}  // namespace
+
+std::string jit_generate(const JitPlanView& v) { return Gen(v).source(true); }
+
+bool jit_compile_only(const std::string& src, std::string* log) {
+  std::vector<char> cubin;
+  return nvrtc_cubin(src, &cubin, log);
+}
+
+JitModule* jit_build(const JitPlanView& v, bool small, char* log, int log_cap) {
+  Gen gen(v);
+  const std::string src = gen.source(small);
+  {
+    std::lock_guard<std::mutex> lk(g_cache_mu);
+    if (!g_cache) g_cache = new std::map<std::string, JitModule*>();
+    auto it = g_cache->find(src);
+    if (it != g_cache->end()) return it->second;
+  }
+  const auto t0 = std::chrono::steady_clock::now();
+  std::vector<char> cubin;
+  std::string lg;
+  if (!nvrtc_cubin(src, &cubin, &lg)) {
+    put_log(log, log_cap, lg);
+    return nullptr;
+  }
+  JitModule* m = new JitModule();
+  cudaError_t e = cudaLibraryLoadData(&m->lib, cubin.data(), nullptr, nullptr, 0, nullptr, nullptr, 0);
+  if (e == cudaSuccess) e = cudaLibraryGetKernel(&m->k, m->lib, "rap_jit_kernel");
+  if (e != cudaSuccess) {
+    put_log(log, log_cap, std::string("cudaLibrary: ") + cudaGetErrorString(e));
+    delete m;
+    return nullptr;
+  }
+  m->compile_s = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+  std::lock_guard<std::mutex> lk(g_cache_mu);
+  auto it = g_cache->find(src);
+  if (it != g_cache->end()) return it->second;  // another thread won the race (the loser's module stays loaded)
+  (*g_cache)[src] = m;
+  return m;
+}
+
+double jit_compile_seconds(const JitModule* m) { return m ? m->compile_s : 0.0; }
+
+int jit_occupancy(JitModule* m, int smem_bytes, int* ctas_per_sm) {
+  const void* k = reinterpret_cast<const void*>(m->k);
+  cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
+  if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(ctas_per_sm, k, kRbChunk, smem_bytes);
+  return (int)e;
+}
+
+// Same parameter block as rap_rows.cu's kernel (RbParams<kRbMaxDense, kRbMaxCols>).
+struct JitParams {
+  Common c;
+  RbGeom g;
+  const float* dense[kRbMaxDense];
+  const uint32_t* dvalid[kRbMaxDense];
+  const int32_t* off[kRbMaxCols];
+  const int64_t* val[kRbMaxCols];
+  const uint32_t* svalid[kRbMaxCols];
+};
+
+int launch_jit(JitModule* m, const Common& c, const RbGeom& g, const LaunchRaw& raw, int smem_bytes, void* stream) {
+  if (raw.n_dense > kRbMaxDense || raw.n_sparse > kRbMaxCols) return (int)cudaErrorInvalidValue;
+  const void* k = reinterpret_cast<const void*>(m->k);
+  {
+    std::lock_guard<std::mutex> lk(m->mu);
+    if (m->smem_set != smem_bytes) {
+      cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
+      if (e != cudaSuccess) return (int)e;
+      m->smem_set = smem_bytes;
+    }
+  }
+  JitParams p;
+  memset(&p, 0, sizeof(p));
+  p.c = c;
+  p.g = g;
+  for (int i = 0; i < raw.n_dense; ++i) {
+    p.dense[i] = raw.dense[i];
+    p.dvalid[i] = raw.dvalid ? raw.dvalid[i] : nullptr;
+  }
+  for (int i = 0; i < raw.n_sparse; ++i) {
+    p.off[i] = raw.off[i];
+    p.val[i] = raw.val[i];
+    p.svalid[i] = raw.svalid ? raw.svalid[i] : nullptr;
+  }
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)(g.n_rb * g.n_fg));
+  cfg.blockDim = dim3(kRbChunk);
+  cfg.dynamicSmemBytes = smem_bytes;
+  cfg.stream = reinterpret_cast<cudaStream_t>(stream);
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeCooperative;
+  attr[0].val.cooperative = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  void* args[1] = {&p};
+  cudaError_t e = cudaLaunchKernelExC(&cfg, k, args);
+  if (e != cudaSuccess) return (int)e;
+  return (int)cudaGetLastError();
+}
+
+}  // namespace rapk

@@ -110,11 +110,18 @@ struct rap_plan {
   int kernel_mode = RAP_KERNEL_AUTO, kernel_last = 0;
   int rb_fits = 0, rb_ctas_per_sm = 0, rb_smem = 0, rb_max_fl = 0, rb_max_cols = 0, rb_n_memo = 0;
   int rb_dense_bytes = 0;
+  unsigned long long rb_all_cols = 0;  // raw sparse columns the sparse outputs read
   std::vector<RbFeat> rbfeat;     // by output index
   std::vector<int32_t> rb_perm;   // processing order
   size_t off_rbfeat = 0, off_perm = 0;
-  unsigned long long* d_agg_rb = nullptr;  // [n_sparse_out * kMaxCtas]
+  unsigned long long* d_agg_rb = nullptr;  // [n_sparse_out][n_rb] row-block totals, then [n_sparse_out] totals
   int rb_last_n_rb = 0, rb_last_n_fg = 0, rb_last_rows = 0;
+  // plan-specialised row-block kernel (rap_jit.cpp), built on first use
+  JitModule* jit[2] = {nullptr, nullptr};  // [small] variants
+  int jit_state = 0, jit_ctas_per_sm = 0;  // state of the last variant asked for
+  int jit_st[2] = {0, 0}, jit_occ[2] = {0, 0};
+  int jit_smem = 0, jit_dense_bytes = 0;
+  double jit_s = 0;
 };
 
 namespace {
@@ -801,6 +808,23 @@ int memo_prefix(const rap_plan* P, const Chain& o, const Canon& qo, const Chain&
   return pm;
 }
 
+JitPlanView jit_view(const rap_plan* P) {
+  JitPlanView v;
+  v.n_sparse_out = (int)P->souts.size();
+  v.n_sparse_in = P->n_sparse_in;
+  v.feat = P->rbfeat.data();
+  v.sprogs = P->sprogs.data();
+  v.perm = P->rb_perm.data();
+  v.used_sparse = P->used_sparse.data();
+  v.n_used_sparse = (int)P->used_sparse.size();
+  v.dprogs = P->dprogs.data();
+  v.n_dprogs = (int)P->dprogs.size();
+  v.d_out = P->d_out;
+  v.dense_bytes = P->rb_dense_bytes;
+  v.itab = P->itab.data();
+  return v;
+}
+
 constexpr int kRbMemoMax = 16;  // memo slots (256 rows x 8 bytes each) a CTA may hold
 
 void build_rows(rap_plan* P) {
@@ -908,6 +932,13 @@ void build_rows(rap_plan* P) {
       }
     }
   P->rb_n_memo = n_memo;
+  P->rb_all_cols = 0;
+  for (int f = 0; f < F; ++f) {
+    const RbFeat& R = P->rbfeat[f];
+    const int kk = R.kind == 1 ? 0 : R.k;
+    for (int i = 0; i < kk; ++i)
+      if (R.src[i] >= 0 && R.src[i] < 64) P->rb_all_cols |= 1ull << R.src[i];
+  }
   P->rb_fits = P->n_sparse_in <= kRbMaxCols && P->n_dense_in <= kRbMaxDense && F <= kRbMaxF;
   P->rb_max_fl = std::max(1, std::min(F, kRbMaxFL));
   P->rb_max_cols = std::max(1, (int)P->used_sparse.size());
@@ -934,37 +965,10 @@ const char* rap_status_string(rap_status s) {
 
 const char* rap_last_error(void) { return g_last_error.c_str(); }
 
-rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, int32_t n_params, int32_t device,
-                           int32_t sm_budget, rap_plan** out) {
-  if (!out) return fail(RAP_ERR_INVALID_ARGUMENT, "out is NULL");
-  *out = nullptr;
-  Validated v;
-  rap_status st = validate(graph, params, n_params, &v);
-  if (st != RAP_OK) return st;
-  if (graph->n_dense_in > 128 || graph->n_sparse_in > 1024)
-    return fail(RAP_ERR_UNSUPPORTED, "more than 128 dense or 1024 sparse raw columns");
-
-  int n_dev = 0;
-  cudaError_t e = cudaGetDeviceCount(&n_dev);
-  if (e != cudaSuccess) return cuda_fail(e, "cudaGetDeviceCount");
-  if (device < 0 || device >= n_dev) return fail(RAP_ERR_INVALID_ARGUMENT, "bad device ordinal");
-  DeviceGuard dg(device);
-
-  rap_plan* P = new rap_plan();
-  P->device = device;
-  P->n_dense_in = graph->n_dense_in;
-  P->n_sparse_in = graph->n_sparse_in;
-  e = cudaDeviceGetAttribute(&P->sm_count, cudaDevAttrMultiProcessorCount, device);
-  if (e != cudaSuccess) {
-    delete P;
-    return cuda_fail(e, "cudaDeviceGetAttribute");
-  }
-  st = set_grid_budget(P, sm_budget);
-  if (st != RAP_OK) {
-    delete P;
-    return st;
-  }
-
+// Host half of rap_plan_create (no device calls): lower every output of a
+// validated graph to its device programs and row-block descriptors.
+static rap_status plan_lower(const rap_graph* graph, const rap_op_param* params, const Validated& v, rap_plan* P) {
+  rap_status st = RAP_OK;
   // ---- lower outputs
   Lowerer L{graph, params, P};
   L.dense_memo.assign(graph->n_nodes, -1);
@@ -987,7 +991,6 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
       const rap_node& nd = graph->nodes[node];
       int c = L.lower_ids(nd.inputs[0], true, &st);
       if (c < 0) {
-        delete P;
         return st;
       }
       Unit u{};
@@ -1000,7 +1003,6 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
     } else {
       int c = L.lower_ids(node, true, &st);
       if (c < 0) {
-        delete P;
         return st;
       }
       SparseOut so{};
@@ -1038,6 +1040,45 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
   }
 
   build_rows(P);
+  return RAP_OK;
+}
+
+rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, int32_t n_params, int32_t device,
+                           int32_t sm_budget, rap_plan** out) {
+  if (!out) return fail(RAP_ERR_INVALID_ARGUMENT, "out is NULL");
+  *out = nullptr;
+  Validated v;
+  rap_status st = validate(graph, params, n_params, &v);
+  if (st != RAP_OK) return st;
+  if (graph->n_dense_in > 128 || graph->n_sparse_in > 1024)
+    return fail(RAP_ERR_UNSUPPORTED, "more than 128 dense or 1024 sparse raw columns");
+
+  int n_dev = 0;
+  cudaError_t e = cudaGetDeviceCount(&n_dev);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaGetDeviceCount");
+  if (device < 0 || device >= n_dev) return fail(RAP_ERR_INVALID_ARGUMENT, "bad device ordinal");
+  DeviceGuard dg(device);
+
+  rap_plan* P = new rap_plan();
+  P->device = device;
+  P->n_dense_in = graph->n_dense_in;
+  P->n_sparse_in = graph->n_sparse_in;
+  e = cudaDeviceGetAttribute(&P->sm_count, cudaDevAttrMultiProcessorCount, device);
+  if (e != cudaSuccess) {
+    delete P;
+    return cuda_fail(e, "cudaDeviceGetAttribute");
+  }
+  st = set_grid_budget(P, sm_budget);
+  if (st != RAP_OK) {
+    delete P;
+    return st;
+  }
+
+  st = plan_lower(graph, params, v, P);
+  if (st != RAP_OK) {
+    delete P;
+    return st;
+  }
 
   // ---- device blob
   std::vector<unsigned char> blob;
@@ -1062,7 +1103,7 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
   if (e == cudaSuccess) e = cudaMalloc(&P->d_part, kPartSlots * kPartLen * sizeof(int64_t));
   if (e == cudaSuccess) e = cudaMallocHost(&P->h_part, kPartSlots * kPartLen * sizeof(int64_t));
   if (e == cudaSuccess && P->rb_fits && !P->souts.empty()) {
-    const size_t n = P->souts.size() * (size_t)kMaxCtas;
+    const size_t n = (P->souts.size() + 1) * (size_t)kMaxCtas + P->souts.size();  // agg [F][n_rb] + tot [F]
     e = cudaMalloc(&P->d_agg_rb, n * sizeof(unsigned long long));
     if (e == cudaSuccess) e = cudaMemset(P->d_agg_rb, 0, n * sizeof(unsigned long long));
   }
@@ -1086,7 +1127,12 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
   P->ctas_per_sm = std::max(1, occ);
   if (P->rb_fits) {
     P->rb_dense_bytes = rows_dense_bytes(max_w);
-    P->rb_smem = rows_smem_bytes(P->rb_dense_bytes, P->rb_max_fl, P->rb_max_cols, P->rb_n_memo, (int)P->souts.size());
+    P->rb_smem = rows_smem_bytes(P->rb_dense_bytes, P->rb_max_fl, P->rb_max_cols, P->rb_n_memo, (int)P->souts.size(), 1);
+    // the generated kernel: no length cache, no shared memo (registers), and
+    // only the dense tile when it generates the dense outputs (rap_jit.cpp)
+    const int tile = 128 * (P->d_out | 1) * 4;
+    P->jit_dense_bytes = (P->d_out > 0 && tile <= P->rb_dense_bytes) ? tile : P->rb_dense_bytes;
+    P->jit_smem = rows_smem_bytes(P->jit_dense_bytes, P->rb_max_fl, P->rb_max_cols, 0, (int)P->souts.size(), 0);
     if (P->rb_smem > 227 * 1024) P->rb_fits = 0;
   }
   if (P->rb_fits) {
@@ -1197,18 +1243,56 @@ rap_status rap_plan_info_get(const rap_plan* P, rap_plan_info* info) {
   info->rb_rows = P->rb_last_rows;
   info->rb_memo_slots = P->rb_n_memo;
   info->partition_uploads = P->partition_uploads;
+  info->jit_state = P->jit_state;
+  info->jit_ctas_per_sm = P->jit_ctas_per_sm;
+  info->jit_compile_seconds = P->jit_s;
   if (P->kernel_last == RAP_KERNEL_ROWS) info->grid = P->rb_last_n_rb * P->rb_last_n_fg;
   return RAP_OK;
 }
 
 rap_status rap_set_kernel(rap_plan* P, int32_t mode) {
   if (!P) return fail(RAP_ERR_INVALID_ARGUMENT, "plan is NULL");
-  if (mode != RAP_KERNEL_AUTO && mode != RAP_KERNEL_TILED && mode != RAP_KERNEL_ROWS)
+  if (mode != RAP_KERNEL_AUTO && mode != RAP_KERNEL_TILED && mode != RAP_KERNEL_ROWS && mode != RAP_KERNEL_JIT)
     return fail(RAP_ERR_INVALID_ARGUMENT, "unknown kernel mode");
-  if (mode == RAP_KERNEL_ROWS && !P->rb_fits && !P->souts.empty())
+  if ((mode == RAP_KERNEL_ROWS || mode == RAP_KERNEL_JIT) && !P->rb_fits && !P->souts.empty())
     return fail(RAP_ERR_UNSUPPORTED, "plan does not fit the row-block kernel (> 64 sparse / 32 dense raw columns)");
   P->kernel_mode = mode;
   return RAP_OK;
+}
+
+rap_status rap_debug_jit_source(const rap_graph* graph, const rap_op_param* params, int32_t n_params, char* buf,
+                                int64_t cap, int32_t compile, int32_t* ok) {
+  if (ok) *ok = 0;
+  Validated v;
+  rap_status st = validate(graph, params, n_params, &v);
+  if (st != RAP_OK) return st;
+  rap_plan* P = new rap_plan();
+  P->n_dense_in = graph->n_dense_in;
+  P->n_sparse_in = graph->n_sparse_in;
+  st = plan_lower(graph, params, v, P);
+  if (st == RAP_OK) {
+    int max_w = 1;
+    for (const DProg& dp : P->dprogs) max_w = std::max(max_w, dp.width);
+    P->rb_dense_bytes = rows_dense_bytes(max_w);
+  }
+  if (st == RAP_OK && (!P->rb_fits || P->souts.empty()))
+    st = fail(RAP_ERR_UNSUPPORTED, "plan does not fit the row-block kernel");
+  if (st == RAP_OK) {
+    const std::string src = jit_generate(jit_view(P));
+    if (buf && cap > 0) {
+      const size_t n = std::min<size_t>(src.size(), (size_t)cap - 1);
+      memcpy(buf, src.data(), n);
+      buf[n] = 0;
+    }
+    if (compile) {
+      std::string log;
+      const bool good = jit_compile_only(src, &log);
+      if (ok) *ok = good ? 1 : 0;
+      g_last_error = log;
+    }
+  }
+  delete P;
+  return st;
 }
 
 rap_status rap_check_overflow(rap_plan* P, int32_t* overflow) {
@@ -1397,14 +1481,41 @@ static rap_status update_partition(rap_plan* P, int64_t B, const int64_t* nnz, i
   return RAP_OK;
 }
 
+// The generated kernel of this plan (rap_jit.cpp), variant `small`: built on
+// first use; on failure the plan keeps the interpreted row-block kernel.
+static bool jit_ready(rap_plan* P, bool small) {
+  const int i = small ? 1 : 0;
+  if (P->jit_st[i] == 0) {
+    const char* env = getenv("RAP_JIT");
+    if (env && env[0] == '0') {
+      P->jit_st[i] = -1;
+    } else {
+      char log[2048] = {0};
+      JitModule* m = jit_build(jit_view(P), small, log, (int)sizeof(log));
+      int occ = 0;
+      if (m && jit_occupancy(m, P->jit_smem, &occ) == 0 && occ >= 1) {
+        P->jit[i] = m;
+        P->jit_occ[i] = occ;
+        P->jit_s += jit_compile_seconds(m);
+        P->jit_st[i] = 1;
+      } else {
+        P->jit_st[i] = -1;
+        g_last_error = std::string("generated kernel unavailable: ") + log;
+      }
+    }
+  }
+  P->jit_state = P->jit_st[i];
+  P->jit_ctas_per_sm = P->jit_occ[i];
+  return P->jit_st[i] == 1;
+}
+
 // Does this batch go to the row-block kernel?  RAP_KERNEL_AUTO: when the plan
 // fits it and every used raw sparse column averages <= 2 ids per row (the
 // row-per-thread mapping is efficient for short lists; long multi-hot lists
 // go element-parallel through the tiled kernel).
 static bool use_rows(const rap_plan* P, int64_t B, const int64_t* nnz) {
   if (P->kernel_mode == RAP_KERNEL_TILED || !P->rb_fits || P->souts.empty()) return false;
-  if (P->kernel_mode == RAP_KERNEL_ROWS) return true;
-  if (getenv("RAP_AUTO_ROWS") == nullptr) return false;  // interpreted row-block kernel: opt-in until it wins
+  if (P->kernel_mode == RAP_KERNEL_ROWS || P->kernel_mode == RAP_KERNEL_JIT) return true;
   for (int s : P->used_sparse)
     if (nnz && B > 0 && (double)nnz[s] > 2.0 * (double)B) return false;
   return true;
@@ -1415,9 +1526,9 @@ static bool use_rows(const rap_plan* P, int64_t B, const int64_t* nnz) {
 // order, balanced by the cost model, <= kRbMaxFL outputs each), at most the
 // budget's CTA slots.  Large batches: one feature group, one row block per
 // slot.  Small batches: 256-row blocks, the slots left over split the outputs.
-static void rows_geometry(const rap_plan* P, int64_t B, const int64_t* nnz, RbGeom* g) {
+static void rows_geometry(const rap_plan* P, int64_t B, const int64_t* nnz, int ctas_per_sm, RbGeom* g) {
   const int F = (int)P->souts.size();
-  const int64_t slots = std::max<int64_t>(1, std::min<int64_t>((int64_t)P->budget * P->rb_ctas_per_sm, kMaxCtas));
+  const int64_t slots = std::max<int64_t>(1, std::min<int64_t>((int64_t)P->budget * ctas_per_sm, kMaxCtas));
   const int fg_min = (F + kRbMaxFL - 1) / kRbMaxFL;
   const int64_t nb256 = (B + kRbChunk - 1) / kRbChunk;
   int64_t n_rb, n_fg;
@@ -1525,20 +1636,38 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
   if (use_rows(P, B, raw->sp_nnz)) {
     RbGeom g;
     memset(&g, 0, sizeof(g));
-    rows_geometry(P, B, raw->sp_nnz, &g);
+    // 32-bit scans when every offset of this launch fits 31 bits
+    const bool small = !c.chain && values_bound(P, B, raw->sp_nnz) < (int64_t)INT32_MAX - 1;
+    const bool want_jit = P->kernel_mode == RAP_KERNEL_JIT || P->kernel_mode == RAP_KERNEL_AUTO;
+    const bool jit = want_jit && jit_ready(P, small);
+    const int iv = small ? 1 : 0;
+    rows_geometry(P, B, raw->sp_nnz, jit ? P->jit_occ[iv] : P->rb_ctas_per_sm, &g);
+    if (jit && !(g.n_fg == 1 && drow0 == 0 && drows == B))  // the generated form does not apply: interpreted geometry
+      rows_geometry(P, B, raw->sp_nnz, P->rb_ctas_per_sm, &g);
     g.max_fl = P->rb_max_fl;
     g.max_cols = P->rb_max_cols;
     g.dense_bytes = P->rb_dense_bytes;
     g.n_memo = P->rb_n_memo;
-    // 32-bit scans when every offset of this launch fits 31 bits
-    g.small = (!c.chain && values_bound(P, B, raw->sp_nnz) < (int64_t)INT32_MAX - 1) ? 1 : 0;
+    g.small = small ? 1 : 0;
+    g.all_cols = P->rb_all_cols;
     g.feat = reinterpret_cast<const RbFeat*>(P->blob + P->off_rbfeat);
     g.perm = reinterpret_cast<const int32_t*>(P->blob + P->off_perm);
     g.agg = P->d_agg_rb;
+    g.tot = P->d_agg_rb + (P->souts.size() + 1) * (size_t)kMaxCtas;
     g.sched = P->d_sched + 4;
-    int rc = launch_rows(c, g, lr, P->rb_smem, stream);
-    if (rc != 0) return cuda_fail((cudaError_t)rc, "row-block kernel launch");
-    P->kernel_last = RAP_KERNEL_ROWS;
+    // the generated policy covers one group of every output, over the batch's
+    // own rows (a sharded plan's dense shard runs the interpreted form)
+    const bool gen = jit && g.n_fg == 1 && drow0 == 0 && drows == B;
+    if (gen) {
+      g.len_cache = 0;
+      g.n_memo = 0;
+      g.dense_bytes = P->jit_dense_bytes;
+    } else {
+      g.len_cache = 1;
+    }
+    int rc = gen ? launch_jit(P->jit[iv], c, g, lr, P->jit_smem, stream) : launch_rows(c, g, lr, P->rb_smem, stream);
+    if (rc != 0) return cuda_fail((cudaError_t)rc, gen ? "generated kernel launch" : "row-block kernel launch");
+    P->kernel_last = gen ? RAP_KERNEL_JIT : RAP_KERNEL_ROWS;
     P->rb_last_n_rb = g.n_rb;
     P->rb_last_n_fg = g.n_fg;
     P->rb_last_rows = g.rows_rb;

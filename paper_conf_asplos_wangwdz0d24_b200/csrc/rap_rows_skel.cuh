@@ -1,0 +1,521 @@
+// rap_rows_skel.cuh — skeleton of the row-block fused kernel (sm_100a),
+// shared by the built-in interpreter (rap_rows.cu) and the plan-specialised
+// kernel generated at plan time (rap_jit.cpp).
+//
+//
+// One cooperative launch turns a raw columnar batch into the "input
+// tensors" by evaluating every output's operator chain
+// (Table 1; DAG per feature, L718-720): horizontal fusion across
+// features and vertical fusion along each chain in one kernel (§6.1
+// L1161-1174), intermediates never leave the SM.  It is the kernel the planner
+// picks for Criteo-shaped batches (short id lists); rap_kernel.cu's tiled
+// kernel handles long multi-hot lists element-parallel.
+//
+// Work: the rows are split into n_rb contiguous row blocks and the sparse
+// outputs into n_fg feature groups (contiguous ranges of a processing order);
+// CTA (g, r) evaluates group g over row block r, one row per thread, in
+// 256-row chunks:
+//   (1) lengths: the Arrow offsets and validity words of every raw column the
+//       group reads are staged in shared memory with cp.async; each output's
+//       row length is a closed form of them (R5, R7, R10, R14), cached in
+//       shared memory; the per-output totals over the block are stored to
+//       agg[f * n_rb + r] and a release counter announces the CTA;
+//   (2) dense: the launch's dense blocks (FillNull / Logit / BoxCox /
+//       Bucketize -> OneHot, row-major through a shared-memory tile), round
+//       robin over the CTAs; they hide the wait of (3);
+//   (3) base: once every CTA is announced, each warp reduces the totals of a
+//       few outputs (all row blocks in parallel); every output's first offset
+//       for this block is the feature-major exclusive prefix (R17);
+//   (4) ids: per output, a warp scan gives each row its position; each
+//       thread runs its row's list through the output's chain (Canon stages,
+//       parameters in shared memory) and stores ids, lengths and offsets; the
+//       next output's first id is loaded while the current one hashes.  A
+//       canonical output memoises element 0 after a prefix of its stages, so
+//       NGram windows over that prefix (C2's trigrams over post-SigridHash
+//       sources) reuse it instead of re-hashing.
+// The last CTA out resets the counters, so launch parameters are the same
+// from call to call (CUDA-graph replayable).  The grid is capped by the SM
+// budget (§6.2).
+#pragma once
+#ifndef __CUDACC_RTC__
+#include <cuda_runtime.h>
+#include <stdint.h>
+#endif
+
+#include "rap_internal.h"
+#include "rap_device.cuh"
+
+namespace rapk {
+
+template <int MD, int MS>
+struct RbParams {
+  Common c;
+  RbGeom g;
+  const float* dense[MD];
+  const uint32_t* dvalid[MD];
+  const int32_t* off[MS];
+  const int64_t* val[MS];
+  const uint32_t* svalid[MS];
+};
+
+constexpr int kRbPitch = kRbChunk + 4;  // staged offsets of one column (257 used), 16-byte rows
+constexpr uint32_t kLenBig = 0xffffu;   // cached length >= this: recompute
+
+// Shared-memory record of one output of the CTA's group (built at CTA start
+// from RbFeat and the output's SProg).
+struct RbF {
+  int32_t kind, emit, n, k;
+  int32_t out_cap, memo_slot, memo_mask, f;
+  int32_t cap[kMaxNgramK];
+  int32_t ncap[kMaxNgramK];
+  int16_t slot[kMaxNgramK];  // staged slot of source i (-1: dense-bucket source)
+  int16_t prov[kMaxNgramK];  // NGram source i: processing index of its memo provider (-1: none)
+  int16_t pslot[kMaxNgramK]; // ... and the provider's memo slot
+  int64_t fill;              // emit 0: a filled null row's id (R10)
+  int32_t src0;              // emit 0: raw column of the list
+  int32_t memo_after;        // emit 0: memoise after this stage bit (16: before any stage, -1: no memo)
+  Canon cn;                  // emit 0: the chain's stages (NGram: post-hash stages)
+};
+
+// Dynamic shared memory layout (rows_smem_bytes computes the same sizes).
+struct RbSmem {
+  unsigned char* dense;  // dense_block's region; phase (3) reductions and phase (4) memo reuse it
+  RbF* feat;             // [max_fl]
+  int32_t* off;          // [max_cols][kRbPitch] staged offsets of the chunk
+  uint32_t* bm;          // [max_cols][8] staged validity words
+  uint16_t* len;         // [max_fl][kRbChunk] lengths of the chunk (kLenBig: recompute)
+  long long* ws;         // [max_fl][8] warp sums of the chunk
+  long long* wb;         // [max_fl][8] warp bases of the chunk
+  long long* base;       // [max_fl] running base (first offset of the next chunk)
+  long long* memo;       // [n_memo][kRbChunk] memoised element 0 (phase 4)
+};
+
+__host__ __device__ inline int rb_align(int x) { return (x + 15) & ~15; }
+
+__host__ __device__ inline int rb_region0(int dense_bytes, int n_memo, int max_f) {
+  const int m = n_memo * kRbChunk * 8, r = 2 * (max_f + 1) * 8;  // phase (3): T[f], L[f]
+  return rb_align(dense_bytes > m ? (dense_bytes > r ? dense_bytes : r) : (m > r ? m : r));
+}
+
+__device__ __forceinline__ RbSmem rb_carve(unsigned char* smem, const RbGeom& g, int n_sparse_out) {
+  RbSmem s;
+  int o = rb_region0(g.dense_bytes, g.n_memo, n_sparse_out);
+  s.dense = smem;
+  s.memo = reinterpret_cast<long long*>(smem);
+  s.ws = reinterpret_cast<long long*>(smem + o);
+  o += rb_align(g.max_fl * 8 * 8);
+  s.wb = reinterpret_cast<long long*>(smem + o);
+  o += rb_align(g.max_fl * 8 * 8);
+  s.base = reinterpret_cast<long long*>(smem + o);
+  o += rb_align(g.max_fl * 8);
+  s.feat = reinterpret_cast<RbF*>(smem + o);
+  o += rb_align(g.max_fl * (int)sizeof(RbF));
+  s.off = reinterpret_cast<int32_t*>(smem + o);
+  o += rb_align(g.max_cols * kRbPitch * 4);
+  s.bm = reinterpret_cast<uint32_t*>(smem + o);
+  o += rb_align(g.max_cols * 8 * 4);
+  s.len = g.len_cache ? reinterpret_cast<uint16_t*>(smem + o) : nullptr;
+  return s;
+}
+
+__device__ __forceinline__ ulonglong2 ld_cg128(const ulonglong2* p) {
+  ulonglong2 v;
+  asm volatile("ld.global.cg.v2.u64 {%0, %1}, [%2];" : "=l"(v.x), "=l"(v.y) : "l"(p));
+  return v;
+}
+
+__device__ __forceinline__ long long ld_cg64(const unsigned long long* p) {
+  long long v;
+  asm volatile("ld.global.cg.s64 %0, [%1];" : "=l"(v) : "l"(p));
+  return v;
+}
+
+// ---- warp-level sums and scans (32-bit when every offset fits, R17) ----
+template <bool kSmall>
+__device__ __forceinline__ long long rb_warp_sum(long long v) {
+  if (kSmall) return (long long)__reduce_add_sync(0xffffffffu, (unsigned)v);
+  return warp_sum64(v);
+}
+
+template <bool kSmall>
+__device__ __forceinline__ long long rb_warp_excl(int32_t v, int lane) {
+  if (kSmall) {
+    int x = v;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const int y = __shfl_up_sync(0xffffffffu, x, d);
+      if (lane >= d) x += y;
+    }
+    return (long long)(x - v);
+  }
+  long long x = v;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const long long y = __shfl_up_sync(0xffffffffu, x, d);
+    if (lane >= d) x += y;
+  }
+  return x - v;
+}
+
+// ---- staged raw rows ----
+struct RbRow {
+  int32_t a, b;
+  bool valid;
+};
+
+__device__ __forceinline__ RbRow rb_row(const RbSmem& s, int slot, int r) {
+  RbRow x;
+  x.a = s.off[slot * kRbPitch + r];
+  x.b = s.off[slot * kRbPitch + r + 1];
+  x.valid = (s.bm[slot * 8 + (r >> 5)] >> (r & 31)) & 1u;
+  return x;
+}
+
+// Stage the offsets [c0, c0 + nr] and validity words of the group's raw
+// columns: thread 0 issues one bulk copy (TMA engine, cp.async.bulk) per
+// column body onto the CTA's staging mbarrier; warp 0 loads the <= 3
+// unaligned tail words (and whole columns whose base is not 16-byte aligned).
+template <class P>
+__device__ __forceinline__ void rb_stage(const P& p, const RbSmem& s, const int16_t* cols, int n_cols, int64_t c0,
+                                         int nr, uint64_t* bar, int* phase) {
+  // thread k < n_cols stages column k: one bulk copy (TMA engine) each for the
+  // 16-byte-aligned body of its offsets and validity words, arriving on the
+  // staging mbarrier (expected arrivals = n_cols) with those bytes; the <= 3
+  // unaligned tail words (or a whole misaligned column) by plain loads
+  const int tid = threadIdx.x;
+  const int no = nr + 1, nw = (nr + 31) >> 5;
+  if (n_cols == 0) return;  // the group reads no list column
+  if (tid == 0) fence_proxy_async();  // the previous chunk's generic reads of the staging area come first
+  __syncthreads();
+  if (tid < n_cols) {
+    const int k = tid, col = cols[k];
+    const int32_t* src = p.off[col] + c0;
+    const bool oa = (reinterpret_cast<uintptr_t>(src) & 15) == 0;
+    const uint32_t ob = oa ? ((uint32_t)(no * 4) & ~15u) : 0u;
+    const uint32_t* bm = p.svalid[col];
+    const uint32_t* bs = bm ? bm + (c0 >> 5) : nullptr;
+    const bool wa = bs != nullptr && (reinterpret_cast<uintptr_t>(bs) & 15) == 0;
+    const uint32_t wb = wa ? ((uint32_t)(nw * 4) & ~15u) : 0u;
+    mbar_arrive_expect(bar, ob + wb);
+    if (ob) bulk_g2s(s.off + k * kRbPitch, src, ob, bar);
+    if (wb) bulk_g2s(s.bm + k * 8, bs, wb, bar);
+    for (int i = (int)(ob / 4); i < no; ++i) s.off[k * kRbPitch + i] = __ldg(src + i);
+    if (bs == nullptr) {
+      for (int i = 0; i < nw; ++i) s.bm[k * 8 + i] = 0xffffffffu;
+    } else {
+      for (int i = (int)(wb / 4); i < nw; ++i) s.bm[k * 8 + i] = __ldg(bs + i);
+    }
+  }
+  mbar_wait(bar, (uint32_t)*phase);
+  __syncthreads();
+  if (tid == 0) *phase ^= 1;
+}
+
+// ---- id emission ----
+// Output stores.  The outputs are write-only in the kernel, so the stores are
+// emitted as st.global without a memory clobber: the compiler may move shared
+// loads of later outputs above them (a store through a plain generic pointer
+// could alias shared memory and would pin every later LDS behind it).
+__device__ __forceinline__ void stg_s32(int32_t* p, int32_t v) {
+  asm volatile("st.global.s32 [%0], %1;" ::"l"(p), "r"(v));
+}
+__device__ __forceinline__ void stg_s64(int64_t* p, int64_t v) {
+  asm volatile("st.global.s64 [%0], %1;" ::"l"(p), "l"(v));
+}
+__device__ __forceinline__ void rb_store(const Common& c, long long pos, int64_t v) {
+  if (pos < c.values_cap)
+    stg_s64(c.values + pos, v);
+  else
+    atomicExch(c.err, 1);
+}
+// lengths[oi] and offsets[oi] of one (output, row)
+__device__ __forceinline__ void rb_store_lo(const Common& c, int64_t oi, int32_t len, long long pos) {
+  stg_s32(c.lengths + oi, len);
+  stg_s64(c.offsets + oi, pos);
+}
+
+// Canonical stages of q restricted to the bits in `keep` (Clamp -> MapId ->
+// SigridHash -> Bucketize order is fixed, so a prefix / suffix split of the
+// mask splits the pipeline).
+__device__ __forceinline__ void canon_part(const Canon& q, int keep, const int64_t* itab, int64_t& v, bool full) {
+  int64_t x[1] = {v};
+  canon_apply_nm<1>(q, q.mask & keep, itab, x, 1u, full ? 1u : 0u);
+  v = x[0];
+}
+
+
+// Raw dense value of a row with the R14 null rule (cleared validity bit ->
+// NaN), for generated dense code.
+template <class P>
+__device__ __forceinline__ float rb_dense_in(const P& p, int col, int64_t row) {
+  const uint32_t* bm = p.dvalid[col];
+  const float v = __ldg(p.dense[col] + row);
+  if (bm == nullptr) return v;
+  return ((__ldg(bm + (row >> 5)) >> (row & 31)) & 1u) ? v : __int_as_float(0x7fc00000);
+}
+
+// Store rows [0, nr) of a row-major tile (pitch floats per row, the first
+// width = d_out columns) to dense_out rows [d0, d0 + nr).
+__device__ __forceinline__ void rb_tile_store(const Common& c, const float* tile, int pitch, int width, int64_t d0,
+                                              int nr) {
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  float* out = c.dense_out + d0 * c.ld;
+  if (c.ld == width && pitch == width) {
+    const int n = nr * width;  // one contiguous run
+    if ((reinterpret_cast<uintptr_t>(out) & 15) == 0 && (n & 3) == 0) {
+      float4* o4 = reinterpret_cast<float4*>(out);
+      const float4* t4 = reinterpret_cast<const float4*>(tile);
+      for (int i = tid; i < (n >> 2); i += kRbChunk) o4[i] = t4[i];
+    } else {
+      for (int i = tid; i < n; i += kRbChunk) out[i] = tile[i];
+    }
+  } else {
+    for (int r = warp; r < nr; r += kWarps)
+      for (int cc = lane; cc < width; cc += 32) out[r * c.ld + cc] = tile[r * pitch + cc];
+  }
+}
+
+// Context of one CTA: its feature group (processing indices [pb, pe)) and
+// row block [R0, R1).
+struct RbCtx {
+  int pb, pe, FL, grp, rb, F, n_cols;
+  int64_t B, R0, R1;
+  const int16_t* slot;  // raw sparse column -> staged slot
+  const int16_t* fidx;  // [FL] output index of processing index pb + fl
+};
+
+// The row-block kernel, parameterised by how an output's lengths and ids are
+// evaluated (Pol): the built-in interpreter (rap_rows_interp.cuh) or the code
+// generated for the plan (rap_jit.cpp).  Pol provides
+//   setup(p, s, x)                   per-CTA records (threads < FL)
+//   lengths<kSmall>(p, s, x, nr, acc) -> s.ws warp sums of every output
+//   emit<kSmall>(p, s, x, c0, nr)     lengths, offsets, ids of the chunk
+template <class Pol, int MD, int MS, bool kSmall>
+__device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
+  unsigned char* const smem = rap_dyn_smem;
+  __shared__ CtaState cs;
+  __shared__ int16_t s_slot[MS];  // raw sparse column -> staged slot (-1: not staged)
+  __shared__ int16_t s_cols[MS];  // staged slot -> raw sparse column
+  __shared__ unsigned long long s_mask[(MS + 63) / 64];
+  __shared__ int16_t s_fidx[kRbMaxFL];
+  __shared__ int s_last, s_fmax;
+  __shared__ uint64_t s_sbar;  // staging mbarrier (bulk copies)
+  __shared__ int s_sphase;
+  const RbGeom& g = p.g;
+  const Common& c = p.c;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  RbCtx x;
+  x.F = c.n_sparse_out;
+  const RbSmem s = rb_carve(smem, g, x.F);
+  const int n_rb = g.n_rb;
+  x.grp = (int)blockIdx.x / n_rb;
+  x.rb = (int)blockIdx.x - x.grp * n_rb;
+  x.pb = g.fg_off[x.grp];
+  x.pe = g.fg_off[x.grp + 1];
+  x.FL = x.pe - x.pb;
+  x.B = c.n_rows;
+  x.R0 = (int64_t)x.rb * g.rows_rb;
+  x.R1 = min(x.B, x.R0 + (int64_t)g.rows_rb);
+  x.slot = s_slot;
+  x.fidx = s_fidx;
+  const int FL = x.FL, rb = x.rb;
+  const int nrows = (int)max((int64_t)0, x.R1 - x.R0);
+  const int nch = (nrows + kRbChunk - 1) / kRbChunk;
+  const long long chain0 = c.chain ? (long long)__ldg(c.offsets) : 0ll;
+  unsigned long long* const pub = g.sched + 2;  // CTAs whose totals are stored
+  trace_stamp(c, 0);
+
+  if (tid == 0) {
+    mbar_init(&cs.bar, 1);
+    s_sphase = 0;
+    cs.phase = 0;
+    cs.dgroup = -1;
+    s_fmax = 0;
+    if (blockIdx.x == 0 && x.F == 0 && !c.chain && c.offsets) c.offsets[0] = 0;  // no sparse outputs (R17)
+  }
+  for (int i = tid; i < (MS + 63) / 64; i += kRbChunk) s_mask[i] = 0ull;
+  __syncthreads();
+  // the raw columns the group reads -> staged slots (one group of every
+  // output: the plan's column mask, no per-output loads)
+  const bool all = x.pb == 0 && x.pe == x.F;
+  if (tid < FL) {
+    const int f = __ldg(g.perm + x.pb + tid);
+    s_fidx[tid] = (int16_t)f;
+    if (!all) {
+      atomicMax(&s_fmax, f);
+      const RbFeat& G = g.feat[f];
+      const int kk = __ldg(&G.kind) == 1 ? 0 : __ldg(&G.k);
+      for (int i = 0; i < kk; ++i) {
+        const int src = __ldg(&G.src[i]);
+        if (src >= 0) atomicOr(&s_mask[src >> 6], 1ull << (src & 63));
+      }
+    }
+  }
+  if (all && tid == 0) {
+    s_fmax = x.F - 1;
+    s_mask[0] = g.all_cols;
+  }
+  __syncthreads();
+  int n_cols = 0;
+  for (int i = 0; i < (MS + 63) / 64; ++i) n_cols += __popcll(s_mask[i]);
+  x.n_cols = n_cols;
+  if (tid == 0) mbar_init(&s_sbar, (uint32_t)max(n_cols, 1));  // staging: one arrival per column
+  for (int col = tid; col < MS; col += kRbChunk) {
+    const unsigned long long m = s_mask[col >> 6];
+    int before = __popcll(m & ((1ull << (col & 63)) - 1ull));
+    for (int i = 0; i < (col >> 6); ++i) before += __popcll(s_mask[i]);
+    const bool on = (m >> (col & 63)) & 1ull;
+    s_slot[col] = on ? (int16_t)before : (int16_t)-1;
+    if (on) s_cols[before] = (int16_t)col;
+  }
+  __syncthreads();
+  trace_stamp(c, 6);
+  if (Pol::kSetupEarly) {
+    Pol::setup(p, s, x);
+    __syncthreads();
+  }
+  trace_stamp(c, 7);
+
+  // (1) per-output totals of my rows -> agg, then announce the CTA
+  for (int ch = 0; ch < nch; ++ch) {
+    const int64_t c0 = x.R0 + (int64_t)ch * kRbChunk;
+    const int nr = (int)min((int64_t)kRbChunk, x.R1 - c0);
+    rb_stage(p, s, s_cols, n_cols, c0, nr, &s_sbar, &s_sphase);
+    if (ch == 0) trace_stamp(c, 8);
+    Pol::template lengths<kSmall>(p, s, x, nr, ch > 0);
+    __syncthreads();
+  }
+  if (tid < FL) {
+    long long tot = 0;
+    if (nch > 0)
+#pragma unroll
+      for (int w = 0; w < 8; ++w) tot += s.ws[tid * 8 + w];
+    const int f = s_fidx[tid];
+    g.agg[(int64_t)f * n_rb + rb] = (unsigned long long)tot;  // feature-major: row blocks of f contiguous
+    atomicAdd(g.tot + f, (unsigned long long)tot);           // red.add: the output's total over all blocks
+  }
+  __syncthreads();
+  if (tid == 0) {
+    __threadfence();  // release: the block's totals before the announcement
+    atomicAdd(pub, 1ull);
+  }
+  trace_stamp(c, 1);
+
+  if (!Pol::kSetupEarly) Pol::setup(p, s, x);  // records used only in (4)
+
+  // (2) dense outputs (independent of the scan): the policy's own rows-of-this-
+  // block code when it has one and the dense rows are the batch rows, else the
+  // launch's dense blocks round robin over the CTAs
+  if (Pol::kGenDense && all && c.dense_row0 == 0 && c.n_dense_rows == c.n_rows && c.n_groups > 0) {
+    Pol::dense(p, s, x);
+  } else {
+    for (int64_t d = blockIdx.x; d < c.n_dense_tiles; d += gridDim.x) {
+      const uint32_t gi = (uint32_t)d % (uint32_t)c.n_groups;
+      dense_block(p, (int)gi, (int64_t)((uint32_t)d / (uint32_t)c.n_groups), 0, cs);
+      __syncthreads();
+      if (d == (int64_t)blockIdx.x) trace_stamp(c, 9);
+    }
+  }
+  __syncthreads();
+  trace_stamp(c, 2);
+
+  if (FL > 0 && nrows > 0) {
+    // (3) wait until every CTA announced its totals (all resident: cooperative launch)
+    if (tid == 0) {
+      int ns = 32;
+      while (ld_acquire(pub) < (unsigned long long)gridDim.x) {
+        __nanosleep(ns);
+        ns = min(ns * 2, 256);
+      }
+    }
+    __syncthreads();
+    trace_stamp(c, 3);
+    // T[f] = the output's total (red.add into g.tot), L[f] = its words of the
+    // row blocks below mine (coalesced; warp w reduces outputs w, w + 8, ...,
+    // two at a time so their loads are in flight together)
+    const int fmax = s_fmax;
+    long long* sT = reinterpret_cast<long long*>(s.dense);  // [fmax + 1]
+    long long* sL = sT + (fmax + 1);                          // [fmax + 1]
+    for (int f = tid; f <= fmax; f += kRbChunk) sT[f] = (long long)__ldcg(g.tot + f);
+    for (int f = warp; f <= fmax; f += 2 * kWarps) {
+      const int f2 = f + kWarps;
+      const unsigned long long* ra = g.agg + (int64_t)f * n_rb;
+      const unsigned long long* rb2 = g.agg + (int64_t)min(f2, fmax) * n_rb;
+      long long la = 0, lb = 0;
+#pragma unroll 4
+      for (int j = lane; j < rb; j += 32) {
+        la += (long long)__ldcg(ra + j);
+        lb += (long long)__ldcg(rb2 + j);
+      }
+      la = rb_warp_sum<kSmall>(la);
+      lb = rb_warp_sum<kSmall>(lb);
+      if (lane == 0) {
+        sL[f] = la;
+        if (f2 <= fmax) sL[f2] = lb;
+      }
+    }
+    trace_stamp(c, 10);
+    __syncthreads();
+    trace_stamp(c, 11);
+    trace_stamp(c, 12);
+    if (tid == 0) {  // exclusive prefix over outputs in feature-major order
+      long long P = chain0;
+      for (int f = 0; f <= fmax; ++f) {
+        const long long t = sT[f];
+        sT[f] = P;
+        P += t;
+      }
+    }
+    __syncthreads();
+    if (tid < FL) {
+      const int f = s_fidx[tid];
+      s.base[tid] = sT[f] + sL[f];
+    }
+    __syncthreads();
+    trace_stamp(c, 4);
+
+    // (4) lengths, offsets and ids, chunk by chunk
+    for (int ch = 0; ch < nch; ++ch) {
+      const int64_t c0 = x.R0 + (int64_t)ch * kRbChunk;
+      const int nr = (int)min((int64_t)kRbChunk, x.R1 - c0);
+      if (nch > 1) {
+        rb_stage(p, s, s_cols, n_cols, c0, nr, &s_sbar, &s_sphase);
+        Pol::template lengths<kSmall>(p, s, x, nr, false);
+        __syncthreads();
+      }
+      if (tid < FL) {  // warp bases of this chunk; the running base advances
+        long long b = s.base[tid];
+#pragma unroll
+        for (int w = 0; w < 8; ++w) {
+          s.wb[tid * 8 + w] = b;
+          b += s.ws[tid * 8 + w];
+        }
+        s.base[tid] = b;
+      }
+      __syncthreads();
+      Pol::template emit<kSmall>(p, s, x, c0, nr);
+      __syncthreads();
+    }
+  }
+  trace_stamp(c, 5);
+
+  // last CTA out: reset the counters (launch parameters stay the same)
+  __syncthreads();
+  if (tid == 0) {
+    __threadfence();
+    const unsigned long long prev = atomicAdd(g.sched, 1ull);
+    s_last = (prev == (unsigned long long)gridDim.x - 1) ? 1 : 0;
+  }
+  __syncthreads();
+  if (s_last) {
+    __threadfence();
+    for (int f = tid; f < x.F; f += kRbChunk) g.tot[f] = 0ull;
+    if (tid == 0) {
+      g.sched[0] = 0ull;
+      g.sched[2] = 0ull;
+    }
+    __threadfence();
+  }
+}
+
+}  // namespace rapk

@@ -22,7 +22,8 @@ STATUS = {0: "OK", 1: "INVALID_ARGUMENT", 2: "INVALID_GRAPH", 3: "INVALID_PARAM"
 EXPORTS = ["rap_plan_create", "rap_plan_output_shape", "rap_preprocess", "rap_preprocess_host", "rap_preprocess_host_async", "rap_set_budget",
            "rap_predict_latency_us", "rap_choose_budget", "rap_plan_info_get", "rap_debug_trace", "rap_plan_destroy",
            "rap_status_string", "rap_last_error", "rap_shard_rows", "rap_plan_output_costs", "rap_place",
-           "rap_plan_create_sharded", "rap_jagged_append", "rap_set_kernel", "rap_check_overflow"]
+           "rap_plan_create_sharded", "rap_jagged_append", "rap_set_kernel", "rap_check_overflow",
+           "rap_debug_jit_source"]
 PLACE_MODES = {"balanced": 0, "round_robin": 1, "skewed": 2}
 RAP_OUT_CHAIN = 1
 
@@ -76,12 +77,13 @@ class RapPlanInfo(C.Structure):
                 ("n_launches", C.c_int64), ("smem_bytes", C.c_int64),
                 ("kernel_mode", C.c_int32), ("kernel_last", C.c_int32), ("rows_ctas_per_sm", C.c_int32),
                 ("rows_smem_bytes", C.c_int32), ("rb_row_blocks", C.c_int32), ("rb_feature_groups", C.c_int32),
-                ("rb_rows", C.c_int32), ("rb_memo_slots", C.c_int32), ("partition_uploads", C.c_int64)]
+                ("rb_rows", C.c_int32), ("rb_memo_slots", C.c_int32), ("partition_uploads", C.c_int64),
+                ("jit_state", C.c_int32), ("jit_ctas_per_sm", C.c_int32), ("jit_compile_seconds", C.c_double)]
 
 
 # rap_set_kernel modes (include/rap.h).  DEFAULT_KERNEL is applied to every new
 # Plan (env RAP_KERNEL; tests set it to run each parity case on both kernels).
-KERNEL_AUTO, KERNEL_TILED, KERNEL_ROWS = 0, 1, 2
+KERNEL_AUTO, KERNEL_TILED, KERNEL_ROWS, KERNEL_JIT = 0, 1, 2, 3
 DEFAULT_KERNEL = int(os.environ.get("RAP_KERNEL", "0"))
 
 
@@ -123,6 +125,9 @@ def load(build_if_stale: bool = False):
     L.rap_set_kernel.argtypes = [P, C.c_int32]
     L.rap_check_overflow.restype = C.c_int
     L.rap_check_overflow.argtypes = [P, C.POINTER(C.c_int32)]
+    L.rap_debug_jit_source.restype = C.c_int
+    L.rap_debug_jit_source.argtypes = [C.POINTER(RapGraph), C.POINTER(RapOpParam), C.c_int32, C.c_char_p, C.c_int64,
+                                       C.c_int32, C.POINTER(C.c_int32)]
     L.rap_debug_trace.restype = C.c_int
     L.rap_debug_trace.argtypes = [P, C.c_int32, P, C.c_int64, C.POINTER(C.c_int64)]
     L.rap_plan_destroy.restype = None
@@ -422,6 +427,19 @@ class Plan:
         _check(load().rap_choose_budget(self.handle, n_rows, nnz.ctypes.data, overlap_capacity_us, C.byref(b),
                                         C.byref(td)))
         return b.value, td.value
+
+
+def jit_source(spec, compile: bool = False):
+    """rap_debug_jit_source: the CUDA source the code generator emits for a
+    spec (no device needed) and, with compile=True, whether NVRTC compiles it
+    for sm_100a.  Returns (status name, source, compiled, nvrtc log)."""
+    L = load()
+    g, params, keep = marshal_graph(spec)
+    cap = 1 << 22
+    buf = C.create_string_buffer(cap)
+    ok = C.c_int32(0)
+    st = L.rap_debug_jit_source(C.byref(g), params, len(spec["nodes"]), buf, cap, 1 if compile else 0, C.byref(ok))
+    return STATUS.get(st, str(st)), buf.value.decode(), bool(ok.value), L.rap_last_error().decode()
 
 
 def validate_only(spec):

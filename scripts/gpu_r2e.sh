@@ -1,0 +1,10 @@
+#!/bin/bash
+# round 2, call E: generated (JIT) row-block kernel — parity, trace, fixed cost, ncu
+mkdir -p gpurun_out
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1
+timeout 900 python -m pytest tests/test_gpu_parity.py -q -m gpu -k "jit" -x > gpurun_out/r02e_pytest_jit.log 2>&1; echo "rc=$?" >> gpurun_out/r02e_pytest_jit.log
+tail -4 gpurun_out/r02e_pytest_jit.log; grep -E "^E  |FAILED" gpurun_out/r02e_pytest_jit.log | head -10
+KMODE=3 WL=c2 B=65536 timeout 120 python scripts/trace_rows.py 2>&1 | tail -8
+RAP_KERNEL=3 WL=c2 SIZES=65536 timeout 300 python scripts/fixed_cost.py 2>&1 | grep -v "^{"
+RAP_KERNEL=3 timeout 600 ncu --set full --clock-control none --import-source on -k regex:rap_jit -s 5 -c 1 -o gpurun_out/r02e_jit_c2 -f python bench.py --profile --steps 8 --warmup 5 > gpurun_out/r02e_ncu.log 2>&1
+tail -1 gpurun_out/r02e_ncu.log

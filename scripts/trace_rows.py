@@ -21,7 +21,7 @@ def main():
     B = int(os.environ.get("B", "65536"))
     host = synth.make_batch(w, B, seed=1)
     plan = rap.Plan(w.spec, device=0)
-    plan.set_kernel(rap.KERNEL_ROWS)
+    plan.set_kernel(int(os.environ.get("KMODE", rap.KERNEL_ROWS)))
     raw = rap.DeviceBatch(host, "cuda:0")
     out = rap.DeviceOutput(plan, B, raw.sp_nnz, "cuda:0")
     for _ in range(5):
@@ -45,6 +45,13 @@ def main():
               f"(abs end median {np.median(rel[:, k]):7.2f} max {rel[:, k].max():7.2f})")
     print(f"  CTA start: p50 {np.percentile(rel[:, 0], 50):.2f} p90 {np.percentile(rel[:, 0], 90):.2f} "
           f"max {rel[:, 0].max():.2f} us")
+    ex = (tr[:, 6:13] - t0) / 1e3
+    for k, nm in enumerate(["slots ready", "setup done", "chunk0 staged", "first dense block", "base loads+redux",
+                            "base sync", "base sums"]):
+        v = ex[:, k]
+        v = v[v > -1e6]
+        if len(v):
+            print(f"  {nm:>18s}: median abs {np.median(v):7.2f} us  max {v.max():7.2f}")
     plan.close()
 
 

@@ -26,9 +26,10 @@ def env():
     return rap, synth, oracle, torch
 
 
-@pytest.fixture(params=[1, 2], ids=["tiled", "rows"], autouse=True)
+@pytest.fixture(params=[1, 2, 3], ids=["tiled", "rows", "jit"], autouse=True)
 def kernel_mode(request):
-    """Every parity case runs on both fused kernels (rap_set_kernel)."""
+    """Every parity case runs on every fused kernel (rap_set_kernel): tiled,
+    interpreted row-block and the plan-specialised (generated) row-block kernel."""
     from paper_conf_asplos_wangwdz0d24_b200 import rap
 
     old = rap.DEFAULT_KERNEL
