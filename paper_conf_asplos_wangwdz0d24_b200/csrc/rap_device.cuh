@@ -163,10 +163,12 @@ __device__ __forceinline__ int count_le8(const int64_t* p, int64_t x) {
 // (smp8[8 j0 .. 8 j0 + 8), smp8[i] = b[8 i + 7]) and the 8 borders of the
 // chosen sub-block, two bursts (R4; same result as upper_bound).
 __device__ __forceinline__ int64_t upper_bound_64(const int64_t* b, int m, const int64_t* smp8, int j0, int64_t x) {
-  if (j0 * 64 >= m) return m;
-  const int j1 = 8 * j0 + count_le8(smp8 + 8 * j0, x);
-  if (j1 * 8 >= m) return m;
-  return (int64_t)j1 * 8 + count_le8(b + 8 * j1, x);
+  // branch-free: the loads stay in range, the selects pick the answer
+  const int nb = m >> 6;
+  const int jc = min(j0, nb - 1);
+  const int j1 = 8 * jc + min(count_le8(smp8 + 8 * jc, x), 7);
+  const int64_t r = (int64_t)j1 * 8 + count_le8(b + 8 * j1, x);
+  return j0 >= nb ? (int64_t)m : r;
 }
 
 // MapId (R8) whose first probe kv0 = table slot of x was loaded ahead (no

@@ -98,8 +98,8 @@ struct Gen {
     if (R.kind == 0) {
       const std::string X = "X" + Q + "_0";
       s += "    const RbRow " + X + " = rb_row(s, " + i2s(slot[R.src[0]]) + ", r);\n";
-      s += "    const int32_t L" + Q + " = !in ? 0 : (" + X + ".valid ? " + cap_expr(X, R.cap[0]) + " : " +
-           i2s(R.ncap[0]) + ");\n";
+      s += "    const int32_t L" + Q + " = in ? (" + X + ".valid ? " + cap_expr(X, R.cap[0]) + " : " + i2s(R.ncap[0]) +
+           ") : 0;\n";
       return s;
     }
     std::string sum = "0LL";
@@ -115,8 +115,8 @@ struct Gen {
       }
       sum += " + " + l;
     }
-    s += "    const int32_t L" + Q + " = !in ? 0 : (int32_t)min(max((long long)(" + sum + ") - " + i2s(R.n) +
-         "LL + 1LL, 0LL), " + i2s(R.out_cap) + "LL);\n";
+    s += "    const int32_t L" + Q + " = in ? (int32_t)min(max((long long)(" + sum + ") - " + i2s(R.n) +
+         "LL + 1LL, 0LL), " + i2s(R.out_cap) + "LL) : 0;\n";
     return s;
   }
 
@@ -183,6 +183,16 @@ struct Gen {
     return nm;
   }
 
+  // upper bound of an output's row length (its FirstX caps), for the scans
+  int max_len(int f) const {
+    const RbFeat& R = v.feat[f];
+    if (R.kind == 1) return R.out_cap;
+    if (R.kind == 0) return std::max(R.cap[0], R.ncap[0]);
+    long long t = 0;
+    for (int i = 0; i < R.k; ++i) t += std::max(R.cap[i], R.ncap[i]);
+    return (int)std::min<long long>(std::max(0LL, t - R.n + 1), R.out_cap);
+  }
+
   static int memo_point(const RbFeat& R, const Canon& cn) {
     if (R.memo_slot < 0) return -1;
     const int pm = R.memo_mask & cn.mask;
@@ -194,9 +204,11 @@ struct Gen {
 
   // ---- dense outputs (a2): thread per row, units split over two halves ----
   int pitch() const { return v.d_out | 1; }
+  // the dense warp's tile sits after the base-phase totals T[f], L[f]
+  int tile_offset() const { return ((2 * (F + 1) * 8) + 15) & ~15; }
   bool gen_dense_ok() const {
     if (v.n_dprogs == 0 || v.d_out <= 0) return false;
-    return 128 * pitch() * 4 <= v.dense_bytes;
+    return tile_offset() + 32 * pitch() * 4 <= v.dense_bytes;
   }
   static double unit_cost(const DProg& dp, const DUnit& un) {
     const DevOp* ops = dp.ops;
@@ -286,45 +298,35 @@ struct Gen {
     return s;
   }
   std::string dense_fn(std::string* globals) {
+    // the dense warp (warp 7): its lane = a row of the block, every unit of
+    // the row (independent loads first), a 32-row tile in shared memory after
+    // the base-phase totals, then stored by the warp
     std::string s;
     const bool ok = gen_dense_ok();
-    s += "  static constexpr bool kGenDense = " + std::string(ok ? "true" : "false") + ";\n";
-    s += "  template <class P>\n  static __device__ __forceinline__ void dense(const P& p, const RbSmem& s, const RbCtx& x) {\n";
+    s += "  static constexpr bool kGenDense = false;\n";
+    s += "  static constexpr bool kDenseWarp = " + std::string(ok ? "true" : "false") + ";\n";
+    s += "  template <class P>\n  static __device__ __forceinline__ void dense(const P&, const RbSmem&, const RbCtx&) {}\n";
+    s += "  template <class P>\n  static __device__ __forceinline__ void dense_warp(const P& p, const RbSmem& s, const RbCtx& x) {\n";
     if (!ok) return s + "  }\n";
-    // split the units over the two halves of the CTA by predicted cost
-    std::vector<std::pair<int, int>> half[2];
-    double load[2] = {0, 0};
-    std::vector<std::pair<double, std::pair<int, int>>> units;
+    std::vector<std::pair<int, int>> units;
+    std::vector<int> cols;
     for (int gi = 0; gi < v.n_dprogs; ++gi)
-      for (int ui = 0; ui < v.dprogs[gi].n_units; ++ui)
-        units.push_back({unit_cost(v.dprogs[gi], v.dprogs[gi].units[ui]), {gi, ui}});
-    std::stable_sort(units.begin(), units.end(), [](const auto& a, const auto& b) { return a.first > b.first; });
-    for (const auto& u : units) {
-      const int h = load[0] <= load[1] ? 0 : 1;
-      load[h] += u.first;
-      half[h].push_back(u.second);
-    }
-    s += "    const Common& c = p.c;\n";
-    s += "    const int tid = threadIdx.x, r = tid & 127, half = tid >> 7;\n";
-    s += "    float* tile = reinterpret_cast<float*>(s.dense);  // [128][" + i2s(pitch()) + "]\n";
-    s += "    for (int64_t d0 = x.R0; d0 < x.R1; d0 += 128) {\n";
-    s += "      const int nr = (int)min((int64_t)128, x.R1 - d0);\n";
-    s += "      if (r < nr) {\n        const int64_t row = d0 + r;\n";
-    s += "        float* trow = tile + r * " + i2s(pitch()) + ";\n";
-    for (int h = 0; h < 2; ++h) {
-      s += std::string(h == 0 ? "        if (half == 0) {\n" : "        } else {\n");
-      // every raw value of the half first (independent loads in flight), then the chains
-      std::vector<int> cols;
-      for (const auto& u : half[h]) {
-        const DUnit& un = v.dprogs[u.first].units[u.second];
+      for (int ui = 0; ui < v.dprogs[gi].n_units; ++ui) {
+        units.push_back({gi, ui});
+        const DUnit& un = v.dprogs[gi].units[ui];
         if (un.kind != U_ONEHOT_G && std::find(cols.begin(), cols.end(), un.src_col) == cols.end())
           cols.push_back(un.src_col);
       }
-      for (int cc : cols) s += "        const float in" + i2s(cc) + " = rb_dense_in(p, " + i2s(cc) + ", row);\n";
-      for (const auto& u : half[h]) s += dense_unit(u.first, u.second, globals);
-    }
-    s += "        }\n      }\n      __syncthreads();\n";
-    s += "      rb_tile_store(c, tile, " + i2s(pitch()) + ", " + i2s(v.d_out) + ", d0, nr);\n      __syncthreads();\n    }\n  }\n";
+    s += "    const Common& c = p.c;\n    const int lane = threadIdx.x & 31;\n";
+    s += "    float* tile = reinterpret_cast<float*>(s.dense + " + i2s(tile_offset()) + ");  // [32][" + i2s(pitch()) + "]\n";
+    s += "    for (int64_t d0 = x.R0; d0 < x.R1; d0 += 32) {\n";
+    s += "      const int nr = (int)min((int64_t)32, x.R1 - d0);\n";
+    s += "      if (lane < nr) {\n        const int64_t row = d0 + lane;\n";
+    s += "        float* trow = tile + lane * " + i2s(pitch()) + ";\n";
+    for (int cc : cols) s += "        const float in" + i2s(cc) + " = rb_dense_in(p, " + i2s(cc) + ", row);\n";
+    for (const auto& u : units) s += dense_unit(u.first, u.second, globals);
+    s += "      }\n      __syncwarp();\n";
+    s += "      rb_tile_store_warp(c, tile, " + i2s(pitch()) + ", " + i2s(v.d_out) + ", d0, nr);\n      __syncwarp();\n    }\n  }\n";
     return s;
   }
 
@@ -361,7 +363,11 @@ struct Gen {
          "    const Common& c = p.c;\n"
          "    const int64_t B = x.B;\n"
          "    const bool in = tid < nr;\n"
-         "    const int64_t row = c0 + tid;\n";
+         "    const int64_t row = c0 + tid;\n"
+         "    bool ovf = false;\n"
+         "    unsigned late = 0;\n";
+    std::vector<int> late_q;
+    int n_late = 0;
     // memo registers of the providers
     std::vector<char> is_prov(F, 0);
     for (int f = 0; f < F; ++f)
@@ -371,15 +377,17 @@ struct Gen {
     // first ids of the canonical list outputs, loaded kAhead outputs before
     // their use (the load latency hides under the outputs in between)
     const int kAhead = 4;
+    const int kSegment = 1 << 30;  // (barriers every few outputs to keep warps together: measured, no gain)
     std::vector<int> canon_q;
     for (int q = 0; q < F; ++q)
       if (v.feat[v.perm[q]].emit == 0) canon_q.push_back(q);
     auto prefetch = [&](int q) {
       const RbFeat& R = v.feat[v.perm[q]];
       const std::string Y = "Y" + i2s(q);
-      return "    int64_t pf" + i2s(q) + " = 0;\n    { const RbRow " + Y + " = rb_row(s, " + i2s(slot[R.src[0]]) +
-             ", r);\n      if (in && " + Y + ".valid && " + Y + ".b > " + Y + ".a) pf" + i2s(q) + " = __ldg(p.val[" +
-             i2s(R.src[0]) + "] + " + Y + ".a); }\n";
+      // unconditional load (no branch): rows without a first id read a word of the plan blob instead
+      return "    int64_t pf" + i2s(q) + ";\n    { const RbRow " + Y + " = rb_row(s, " + i2s(slot[R.src[0]]) +
+             ", r);\n      const bool ok = in && " + Y + ".valid && " + Y + ".b > " + Y + ".a;\n      pf" + i2s(q) +
+             " = __ldg(ok ? p.val[" + i2s(R.src[0]) + "] + " + Y + ".a : c.itab); }\n";
     };
     // MapId outputs: their first table probe is loaded kProbe outputs ahead,
     // from the prefetched id run through the stages before MapId
@@ -412,32 +420,41 @@ struct Gen {
           s += probe(canon_q[canon_i + kProbe]);
         ++canon_i;
       }
+      // branch-free block: every value is computed for every lane, the
+      // stores are predicated (lanes past the chunk, empty rows), so the
+      // scheduler interleaves neighbouring outputs
+      const bool le1 = max_len(f) <= 1;  // every row holds at most one id: ballot scan
+      // every kSegment outputs the sparse warps meet, so they run through the
+      // straight-line code together (the active window stays in the I-cache)
+      if (q > 0 && q % kSegment == 0)
+        s += std::string("    ") + (gen_dense_ok() ? "rb_sync<true>();" : "rb_sync<false>();") + "\n";
       s += "  {  // output " + Fs + "\n" + len_code(q);
-      s += "    const long long P" + Q + " = s.wb[" + i2s(q * 8) + " + warp] + rb_warp_excl<kSmall>(L" + Q +
-           ", lane);\n";
+      s += "    const long long P" + Q + " = s.wb[" + i2s(q * 8) + " + warp] + " +
+           (le1 ? "rb_ballot_excl(L" + Q + " != 0, lane)" : "rb_warp_excl<kSmall>(L" + Q + ", lane)") + ";\n";
       if (is_prov[f]) s += "    ml" + Fs + " = L" + Q + ";\n";
-      s += "    if (in) {\n";
-      s += "      const int64_t oi = (int64_t)" + Fs + " * B + row;\n";
-      s += "      rb_store_lo(c, oi, L" + Q + ", P" + Q + ");\n";
-      if (f == F - 1) s += "      if (row == B - 1) stg_s64(c.offsets + (int64_t)" + i2s(F) + " * B, P" + Q + " + L" + Q + ");\n";
-      s += "      if (L" + Q + " > 0) {\n";
+      s += "    stg_s32_if(in, c.lengths + ((int64_t)" + Fs + " * B + row), L" + Q + ");\n";
+      s += "    stg_s64_if(in, c.offsets + ((int64_t)" + Fs + " * B + row), P" + Q + ");\n";
+      if (f == F - 1) s += "    stg_s64_if(in && row == B - 1, c.offsets + (int64_t)" + i2s(F) + " * B, P" + Q + " + L" + Q + ");\n";
+      s += "    ovf |= P" + Q + " + L" + Q + " > c.values_cap;\n";
       if (R.emit == 0) {
         const Canon& cn = pg.cn;
         const std::string X = "X" + Q + "_0";
         const int col = R.src[0];
-        s += "        int64_t v = " + X + ".valid ? pf" + Q + " : " + lit64(pg.ch.fill) + ";\n";
+        s += "    {\n        int64_t v = " + X + ".valid ? pf" + Q + " : " + lit64(pg.ch.fill) + ";\n";
         s += stages(cn, cn.mask, "v", X + ".valid", is_prov[f] ? memo_point(R, cn) : -1, "m" + Fs,
                     (cn.mask & CB_MAPID) ? "pk" + Q : "");
-        s += "        rb_store(c, P" + Q + ", v);\n";
+        s += "        stg_s64_if(L" + Q + " > 0 && P" + Q + " < c.values_cap, c.values + P" + Q + ", v);\n";
         if (R.cap[0] > 1) {
           s += "        for (int32_t j = 1; j < L" + Q + "; ++j) {\n";
           s += "          int64_t w = __ldg(p.val[" + i2s(col) + "] + " + X + ".a + j);\n";
           s += stages(cn, cn.mask, "w", "true", -1, "");
           s += "          rb_store(c, P" + Q + " + j, w);\n        }\n";
         }
+        s += "    }\n";
       } else if (R.emit == 3 && ngram_fast_ok(q)) {
-        // every source memoised by an earlier provider: push the present
-        // elements through an n-register window (R7)
+        // every source memoised by an earlier provider: the present elements
+        // shift through an n-register window (selects, R7); rows whose sources
+        // hold more than one id run the generic path
         const int n = R.n, K = R.k;
         std::string cond;
         for (int i = 0; i < K; ++i) {
@@ -446,34 +463,50 @@ struct Gen {
           if (i) cond += " && ";
           cond += "(" + l + " <= 1 && (" + l + " == 0 || ml" + i2s(fp) + " >= 1))";
         }
-        s += "        if (" + cond + ") {\n";
-        s += "          int32_t cnt = 0;\n";
-        for (int j = 0; j < n; ++j) s += "          uint64_t w" + i2s(j) + " = 0;\n";
+        s += "    {\n      const bool fast = " + cond + ";\n      int32_t cnt = 0;\n";
+        for (int j = 0; j < n; ++j) s += "      uint64_t w" + i2s(j) + " = 0;\n";
         for (int i = 0; i < K; ++i) {
           const int fp = v.perm[R.prov[i]];
-          s += "          if (l" + Q + "_" + i2s(i) + ") {\n";
-          for (int j = 0; j + 1 < n; ++j) s += "            w" + i2s(j) + " = w" + i2s(j + 1) + ";\n";
-          s += "            w" + i2s(n - 1) + " = (uint64_t)m" + i2s(fp) + ";\n            ++cnt;\n";
+          const std::string pr = "pr" + i2s(i);
+          s += "      const bool " + pr + " = l" + Q + "_" + i2s(i) + " != 0;\n";
+          for (int j = 0; j + 1 < n; ++j)
+            s += "      w" + i2s(j) + " = " + pr + " ? w" + i2s(j + 1) + " : w" + i2s(j) + ";\n";
+          s += "      w" + i2s(n - 1) + " = " + pr + " ? (uint64_t)m" + i2s(fp) + " : w" + i2s(n - 1) + ";\n";
+          s += "      cnt += " + pr + ";\n";
           if (i + 1 >= n) {
-            s += "            if (cnt >= " + i2s(n) + " && cnt - " + i2s(n) + " < L" + Q + ") {\n";
-            s += "              uint64_t h = " + litu64(pg.ng.hsalt) + ";\n";
-            for (int j = 0; j < n; ++j) s += "              h = splitmix_H(h ^ w" + i2s(j) + ");\n";
-            s += "              int64_t v = (int64_t)reduce_M(h, " + lit64(pg.ng.M) + ");\n";
+            s += "      {\n        uint64_t h = " + litu64(pg.ng.hsalt) + ";\n";
+            for (int j = 0; j < n; ++j) s += "        h = splitmix_H(h ^ w" + i2s(j) + ");\n";
+            s += "        int64_t v = (int64_t)reduce_M(h, " + lit64(pg.ng.M) + ");\n";
             s += stages(pg.cn, pg.cn.mask, "v", "true", -1, "");
-            s += "              rb_store(c, P" + Q + " + (cnt - " + i2s(n) + "), v);\n            }\n";
+            s += "        const long long at = P" + Q + " + (cnt - " + i2s(n) + ");\n";
+            s += "        stg_s64_if(fast && " + pr + " && cnt >= " + i2s(n) + " && cnt - " + i2s(n) + " < L" + Q +
+                 " && at < c.values_cap, c.values + at, v);\n      }\n";
           }
-          s += "          }\n";
         }
-        s += "        } else {\n";
-        s += "          rb_emit_ngram(p, s, s.feat[" + Q + "], -1, r, row, L" + Q + ", P" + Q + ", 0);\n";
-        s += "        }\n";
+        if (n_late < 32) {  // rows the register path cannot take: after the straight-line code
+          s += "      if (!fast && L" + Q + " > 0) late |= 1u << " + i2s(n_late) + ";\n    }\n";
+          late_q.push_back(q);
+          ++n_late;
+        } else {
+          s += "      if (!fast && L" + Q + " > 0) rb_emit_ngram(p, s, s.feat[" + Q + "], -1, r, row, L" + Q + ", P" + Q +
+               ", 0);\n    }\n";
+        }
       } else if (R.emit == 3) {
-        s += "        rb_emit_ngram(p, s, s.feat[" + Q + "], -1, r, row, L" + Q + ", P" + Q + ", 0);\n";
+        s += "    if (L" + Q + " > 0) rb_fallback(p, s, x.slot, " + Fs + ", r, row, L" + Q + ", P" + Q + ");\n";
       } else {
-        s += "        rb_emit_generic(p, s, s.feat[" + Q + "], r, row, L" + Q + ", P" + Q + ");\n";
+        s += "    if (L" + Q + " > 0) rb_fallback(p, s, x.slot, " + Fs + ", r, row, L" + Q + ", P" + Q + ");\n";
       }
-      s += "      }\n    }\n  }\n";
+      s += "  }\n";
     }
+    for (int k = 0; k < (int)late_q.size(); ++k) {  // NGram rows off the register path (warp-uniform test)
+      const int q = late_q[k];
+      const std::string Q = i2s(q), Fs = i2s(v.perm[q]);
+      s += "  if (__any_sync(0xffffffffu, (late >> " + i2s(k) + ") & 1u)) {\n" + len_code(q);
+      s += "    const long long P" + Q + " = s.wb[" + i2s(q * 8) + " + warp] + rb_warp_excl<kSmall>(L" + Q + ", lane);\n";
+      s += "    if ((late >> " + i2s(k) + ") & 1u) rb_emit_ngram(p, s, s.feat[" + Q + "], -1, r, row, L" + Q + ", P" + Q +
+           ", 0);\n  }\n";
+    }
+    s += "    if (ovf) atomicExch(c.err, 1);  // values_capacity understated (sp_nnz): nothing stored past it\n";
     s += "  }\n";
     return s;
   }
@@ -506,7 +539,7 @@ struct Gen {
     body += "  static constexpr bool kSetupEarly = false;  // records only feed the fallbacks of (4)\n";
     body += "  template <class P>\n"
             "  static __device__ __forceinline__ void setup(const P& p, const RbSmem& s, const RbCtx& x) {\n";
-    if (records) body += "    InterpPolicy::setup(p, s, x);  // records for the generic fallbacks\n";
+    (void)records;  // the fallbacks rebuild their record from the plan blob (rb_fallback)
     body += "  }\n";
     body += dense;
     body += lengths_fn();

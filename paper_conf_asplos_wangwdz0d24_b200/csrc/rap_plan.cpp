@@ -1130,7 +1130,8 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
     P->rb_smem = rows_smem_bytes(P->rb_dense_bytes, P->rb_max_fl, P->rb_max_cols, P->rb_n_memo, (int)P->souts.size(), 1);
     // the generated kernel: no length cache, no shared memo (registers), and
     // only the dense tile when it generates the dense outputs (rap_jit.cpp)
-    const int tile = 128 * (P->d_out | 1) * 4;
+    // the dense warp's 32-row tile after the base-phase totals (rap_jit.cpp tile_offset)
+    const int tile = ((2 * ((int)P->souts.size() + 1) * 8 + 15) & ~15) + 32 * (P->d_out | 1) * 4;
     P->jit_dense_bytes = (P->d_out > 0 && tile <= P->rb_dense_bytes) ? tile : P->rb_dense_bytes;
     P->jit_smem = rows_smem_bytes(P->jit_dense_bytes, P->rb_max_fl, P->rb_max_cols, 0, (int)P->souts.size(), 0);
     if (P->rb_smem > 227 * 1024) P->rb_fits = 0;

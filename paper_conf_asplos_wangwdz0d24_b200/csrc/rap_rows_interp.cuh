@@ -266,13 +266,50 @@ __device__ __noinline__ void rb_emit_ngram(const P& p, const RbSmem s, const RbF
 }
 
 
+// Rare rows of the generated kernel (an NGram row whose sources hold more
+// than one id, a non-canonical chain): the output's record is rebuilt from the
+// plan blob (RbFeat, SProg) and the interpreter's functions run (no memo).
+template <class P>
+__device__ __noinline__ void rb_fallback(const P& p, const RbSmem s, const int16_t* slot_map, int f, int r,
+                                         int64_t row, int32_t len, long long pos) {
+  const RbFeat& G = p.g.feat[f];
+  const SProg& pg = p.c.sprogs[f];
+  RbF F;
+  F.kind = G.kind;
+  F.emit = G.emit;
+  F.n = G.n;
+  F.k = G.k;
+  F.out_cap = G.out_cap;
+  F.memo_slot = -1;
+  F.memo_mask = 0;
+  F.f = f;
+  const int kk = F.kind == 1 ? 0 : F.k;
+  for (int i = 0; i < kMaxNgramK; ++i) {
+    F.cap[i] = G.cap[i];
+    F.ncap[i] = G.ncap[i];
+    F.slot[i] = (i < kk && G.src[i] >= 0) ? slot_map[G.src[i]] : (int16_t)-1;
+    F.prov[i] = F.pslot[i] = -1;
+  }
+  F.fill = pg.ch.fill;
+  F.src0 = G.src[0];
+  F.memo_after = -1;
+  F.cn = pg.cn;
+  if (F.emit == 3)
+    rb_emit_ngram(p, s, F, -1, r, row, len, pos, 0);
+  else
+    rb_emit_generic(p, s, F, r, row, len, pos);
+}
+
 // The built-in policy: each output's record (RbF) in shared memory, read per
 // warp and output.
 struct InterpPolicy {
   static constexpr bool kSetupEarly = true;  // the records drive (1) as well
   static constexpr bool kGenDense = false;
+  static constexpr bool kDenseWarp = false;
   template <class P>
   static __device__ __forceinline__ void dense(const P&, const RbSmem&, const RbCtx&) {}
+  template <class P>
+  static __device__ __forceinline__ void dense_warp(const P&, const RbSmem&, const RbCtx&) {}
 
   template <class P>
   static __device__ __forceinline__ void setup(const P& p, const RbSmem& s, const RbCtx& x) {

@@ -157,6 +157,11 @@ __device__ __forceinline__ long long rb_warp_excl(int32_t v, int lane) {
   return x - v;
 }
 
+// Exclusive warp scan of 0/1 flags (rows holding at most one id).
+__device__ __forceinline__ long long rb_ballot_excl(bool f, int lane) {
+  return (long long)__popc(__ballot_sync(0xffffffffu, f) & ((1u << lane) - 1u));
+}
+
 // ---- staged raw rows ----
 struct RbRow {
   int32_t a, b;
@@ -171,11 +176,21 @@ __device__ __forceinline__ RbRow rb_row(const RbSmem& s, int slot, int r) {
   return x;
 }
 
+// Barrier of the threads that run the sparse phases: every thread, or (the
+// generated kernel with a dense warp) warps 0-6 on named barrier 1.
+template <bool kDW>
+__device__ __forceinline__ void rb_sync() {
+  if (kDW)
+    asm volatile("bar.sync 1, 224;" ::: "memory");
+  else
+    __syncthreads();
+}
+
 // Stage the offsets [c0, c0 + nr] and validity words of the group's raw
 // columns: thread 0 issues one bulk copy (TMA engine, cp.async.bulk) per
 // column body onto the CTA's staging mbarrier; warp 0 loads the <= 3
 // unaligned tail words (and whole columns whose base is not 16-byte aligned).
-template <class P>
+template <bool kDW, class P>
 __device__ __forceinline__ void rb_stage(const P& p, const RbSmem& s, const int16_t* cols, int n_cols, int64_t c0,
                                          int nr, uint64_t* bar, int* phase) {
   // thread k < n_cols stages column k: one bulk copy (TMA engine) each for the
@@ -186,7 +201,7 @@ __device__ __forceinline__ void rb_stage(const P& p, const RbSmem& s, const int1
   const int no = nr + 1, nw = (nr + 31) >> 5;
   if (n_cols == 0) return;  // the group reads no list column
   if (tid == 0) fence_proxy_async();  // the previous chunk's generic reads of the staging area come first
-  __syncthreads();
+  rb_sync<kDW>();
   if (tid < n_cols) {
     const int k = tid, col = cols[k];
     const int32_t* src = p.off[col] + c0;
@@ -207,7 +222,7 @@ __device__ __forceinline__ void rb_stage(const P& p, const RbSmem& s, const int1
     }
   }
   mbar_wait(bar, (uint32_t)*phase);
-  __syncthreads();
+  rb_sync<kDW>();
   if (tid == 0) *phase ^= 1;
 }
 
@@ -221,6 +236,15 @@ __device__ __forceinline__ void stg_s32(int32_t* p, int32_t v) {
 }
 __device__ __forceinline__ void stg_s64(int64_t* p, int64_t v) {
   asm volatile("st.global.s64 [%0], %1;" ::"l"(p), "l"(v));
+}
+// Predicated forms (one instruction, no branch around it).
+__device__ __forceinline__ void stg_s32_if(bool q, int32_t* p, int32_t v) {
+  asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q st.global.s32 [%0], %1;\n\t}" ::"l"(p), "r"(v),
+               "r"((unsigned)q));
+}
+__device__ __forceinline__ void stg_s64_if(bool q, int64_t* p, int64_t v) {
+  asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q st.global.s64 [%0], %1;\n\t}" ::"l"(p), "l"(v),
+               "r"((unsigned)q));
 }
 __device__ __forceinline__ void rb_store(const Common& c, long long pos, int64_t v) {
   if (pos < c.values_cap)
@@ -275,6 +299,27 @@ __device__ __forceinline__ void rb_tile_store(const Common& c, const float* tile
   }
 }
 
+// One warp stores rows [0, nr) of a row-major tile (pitch floats per row,
+// the first width = d_out columns) to dense_out rows [d0, d0 + nr).
+__device__ __forceinline__ void rb_tile_store_warp(const Common& c, const float* tile, int pitch, int width,
+                                                   int64_t d0, int nr) {
+  const int lane = threadIdx.x & 31;
+  float* out = c.dense_out + d0 * c.ld;
+  if (c.ld == width && pitch == width) {
+    const int n = nr * width;
+    if ((reinterpret_cast<uintptr_t>(out) & 15) == 0 && (n & 3) == 0) {
+      float4* o4 = reinterpret_cast<float4*>(out);
+      const float4* t4 = reinterpret_cast<const float4*>(tile);
+      for (int i = lane; i < (n >> 2); i += 32) o4[i] = t4[i];
+    } else {
+      for (int i = lane; i < n; i += 32) out[i] = tile[i];
+    }
+  } else {
+    for (int r = 0; r < nr; ++r)
+      for (int cc = lane; cc < width; cc += 32) out[r * c.ld + cc] = tile[r * pitch + cc];
+  }
+}
+
 // Context of one CTA: its feature group (processing indices [pb, pe)) and
 // row block [R0, R1).
 struct RbCtx {
@@ -304,6 +349,11 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
   const RbGeom& g = p.g;
   const Common& c = p.c;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  // generated kernel with a dense warp: warps 0-6 run the sparse phases over
+  // 224-row chunks while warp 7 evaluates the dense outputs of the block
+  constexpr bool kDW = Pol::kDenseWarp;
+  constexpr int kTS = kDW ? 224 : kRbChunk;  // sparse threads = rows per chunk
+  constexpr int kWS = kTS / 32;               // sparse warps
   RbCtx x;
   x.F = c.n_sparse_out;
   const RbSmem s = rb_carve(smem, g, x.F);
@@ -320,7 +370,7 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
   x.fidx = s_fidx;
   const int FL = x.FL, rb = x.rb;
   const int nrows = (int)max((int64_t)0, x.R1 - x.R0);
-  const int nch = (nrows + kRbChunk - 1) / kRbChunk;
+  const int nch = (nrows + kTS - 1) / kTS;
   const long long chain0 = c.chain ? (long long)__ldg(c.offsets) : 0ll;
   unsigned long long* const pub = g.sched + 2;  // CTAs whose totals are stored
   trace_stamp(c, 0);
@@ -375,26 +425,29 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
     __syncthreads();
   }
   trace_stamp(c, 7);
+  if (kDW && warp == kWS) {
+    Pol::dense_warp(p, s, x);  // the dense outputs of rows [R0, R1), concurrent with the sparse phases
+  } else {
 
   // (1) per-output totals of my rows -> agg, then announce the CTA
   for (int ch = 0; ch < nch; ++ch) {
-    const int64_t c0 = x.R0 + (int64_t)ch * kRbChunk;
-    const int nr = (int)min((int64_t)kRbChunk, x.R1 - c0);
-    rb_stage(p, s, s_cols, n_cols, c0, nr, &s_sbar, &s_sphase);
+    const int64_t c0 = x.R0 + (int64_t)ch * kTS;
+    const int nr = (int)min((int64_t)kTS, x.R1 - c0);
+    rb_stage<kDW>(p, s, s_cols, n_cols, c0, nr, &s_sbar, &s_sphase);
     if (ch == 0) trace_stamp(c, 8);
     Pol::template lengths<kSmall>(p, s, x, nr, ch > 0);
-    __syncthreads();
+    rb_sync<kDW>();
   }
   if (tid < FL) {
     long long tot = 0;
     if (nch > 0)
 #pragma unroll
-      for (int w = 0; w < 8; ++w) tot += s.ws[tid * 8 + w];
+      for (int w = 0; w < kWS; ++w) tot += s.ws[tid * 8 + w];
     const int f = s_fidx[tid];
     g.agg[(int64_t)f * n_rb + rb] = (unsigned long long)tot;  // feature-major: row blocks of f contiguous
     atomicAdd(g.tot + f, (unsigned long long)tot);           // red.add: the output's total over all blocks
   }
-  __syncthreads();
+  rb_sync<kDW>();
   if (tid == 0) {
     __threadfence();  // release: the block's totals before the announcement
     atomicAdd(pub, 1ull);
@@ -405,18 +458,20 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
 
   // (2) dense outputs (independent of the scan): the policy's own rows-of-this-
   // block code when it has one and the dense rows are the batch rows, else the
-  // launch's dense blocks round robin over the CTAs
-  if (Pol::kGenDense && all && c.dense_row0 == 0 && c.n_dense_rows == c.n_rows && c.n_groups > 0) {
-    Pol::dense(p, s, x);
-  } else {
-    for (int64_t d = blockIdx.x; d < c.n_dense_tiles; d += gridDim.x) {
-      const uint32_t gi = (uint32_t)d % (uint32_t)c.n_groups;
-      dense_block(p, (int)gi, (int64_t)((uint32_t)d / (uint32_t)c.n_groups), 0, cs);
-      __syncthreads();
-      if (d == (int64_t)blockIdx.x) trace_stamp(c, 9);
+  // launch's dense blocks round robin over the CTAs (the dense warp took them)
+  if (!kDW) {
+    if (Pol::kGenDense && all && c.dense_row0 == 0 && c.n_dense_rows == c.n_rows && c.n_groups > 0) {
+      Pol::dense(p, s, x);
+    } else {
+      for (int64_t d = blockIdx.x; d < c.n_dense_tiles; d += gridDim.x) {
+        const uint32_t gi = (uint32_t)d % (uint32_t)c.n_groups;
+        dense_block(p, (int)gi, (int64_t)((uint32_t)d / (uint32_t)c.n_groups), 0, cs);
+        __syncthreads();
+        if (d == (int64_t)blockIdx.x) trace_stamp(c, 9);
+      }
     }
   }
-  __syncthreads();
+  rb_sync<kDW>();
   trace_stamp(c, 2);
 
   if (FL > 0 && nrows > 0) {
@@ -428,7 +483,7 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
         ns = min(ns * 2, 256);
       }
     }
-    __syncthreads();
+    rb_sync<kDW>();
     trace_stamp(c, 3);
     // T[f] = the output's total (red.add into g.tot), L[f] = its words of the
     // row blocks below mine (coalesced; warp w reduces outputs w, w + 8, ...,
@@ -436,9 +491,9 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
     const int fmax = s_fmax;
     long long* sT = reinterpret_cast<long long*>(s.dense);  // [fmax + 1]
     long long* sL = sT + (fmax + 1);                          // [fmax + 1]
-    for (int f = tid; f <= fmax; f += kRbChunk) sT[f] = (long long)__ldcg(g.tot + f);
-    for (int f = warp; f <= fmax; f += 2 * kWarps) {
-      const int f2 = f + kWarps;
+    for (int f = tid; f <= fmax; f += kTS) sT[f] = (long long)__ldcg(g.tot + f);
+    for (int f = warp; f <= fmax; f += 2 * kWS) {
+      const int f2 = f + kWS;
       const unsigned long long* ra = g.agg + (int64_t)f * n_rb;
       const unsigned long long* rb2 = g.agg + (int64_t)min(f2, fmax) * n_rb;
       long long la = 0, lb = 0;
@@ -455,7 +510,7 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
       }
     }
     trace_stamp(c, 10);
-    __syncthreads();
+    rb_sync<kDW>();
     trace_stamp(c, 11);
     trace_stamp(c, 12);
     if (tid == 0) {  // exclusive prefix over outputs in feature-major order
@@ -466,37 +521,38 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
         P += t;
       }
     }
-    __syncthreads();
+    rb_sync<kDW>();
     if (tid < FL) {
       const int f = s_fidx[tid];
       s.base[tid] = sT[f] + sL[f];
     }
-    __syncthreads();
+    rb_sync<kDW>();
     trace_stamp(c, 4);
 
     // (4) lengths, offsets and ids, chunk by chunk
     for (int ch = 0; ch < nch; ++ch) {
-      const int64_t c0 = x.R0 + (int64_t)ch * kRbChunk;
-      const int nr = (int)min((int64_t)kRbChunk, x.R1 - c0);
+      const int64_t c0 = x.R0 + (int64_t)ch * kTS;
+      const int nr = (int)min((int64_t)kTS, x.R1 - c0);
       if (nch > 1) {
-        rb_stage(p, s, s_cols, n_cols, c0, nr, &s_sbar, &s_sphase);
+        rb_stage<kDW>(p, s, s_cols, n_cols, c0, nr, &s_sbar, &s_sphase);
         Pol::template lengths<kSmall>(p, s, x, nr, false);
-        __syncthreads();
+        rb_sync<kDW>();
       }
       if (tid < FL) {  // warp bases of this chunk; the running base advances
         long long b = s.base[tid];
 #pragma unroll
-        for (int w = 0; w < 8; ++w) {
+        for (int w = 0; w < kWS; ++w) {
           s.wb[tid * 8 + w] = b;
           b += s.ws[tid * 8 + w];
         }
         s.base[tid] = b;
       }
-      __syncthreads();
+      rb_sync<kDW>();
       Pol::template emit<kSmall>(p, s, x, c0, nr);
-      __syncthreads();
+      rb_sync<kDW>();
     }
   }
+  }  // sparse warps
   trace_stamp(c, 5);
 
   // last CTA out: reset the counters (launch parameters stay the same)
