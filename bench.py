@@ -52,6 +52,8 @@ def parse():
     ap.add_argument("--placement", default="balanced", choices=["balanced", "round_robin", "skewed"],
                     help="N>1: table placement (DESIGN.md §10)")
     ap.add_argument("--imbalance-tol", type=float, default=0.10, help="N>1: residual move threshold")
+    ap.add_argument("--no-c4", action="store_true", help="skip the config-4 (multi-hot) sub-measurement")
+    ap.add_argument("--c4-batch", type=int, default=16384, help="rows of the config-4 sub-measurement")
     return ap.parse_args()
 
 
@@ -144,8 +146,23 @@ def traffic_from_profile(workload_name):
         return None
 
 
+def cpu_model():
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
+
+
 def cpu_baseline(w, seconds, rows=8192):
-    """The oracle, as it stands, on a bounded sample of the same workload."""
+    """The oracle, as it stands, on a bounded sample of the same workload:
+    single-threaded, and on every core the process may use (one row slice per
+    thread; ctypes releases the GIL inside the C oracle)."""
+    from concurrent.futures import ThreadPoolExecutor
+
     from oracle import oracle
     from paper_conf_asplos_wangwdz0d24_b200 import synth
 
@@ -157,11 +174,30 @@ def cpu_baseline(w, seconds, rows=8192):
         r = oracle.run(w.spec, host)
         assert r["status"] == "OK"
         n += 1
-        if time.perf_counter() - t0 >= seconds:
+        if time.perf_counter() - t0 >= seconds / 2:
             break
-    dt = time.perf_counter() - t0
-    return {"value": n * rows / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
-            "sample": f"{n} x {rows}-row batches of {w.name} (seed 101), single-threaded C oracle, {dt:.1f} s"}
+    dt1 = time.perf_counter() - t0
+    one = n * rows / dt1
+    cores = len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else (os.cpu_count() or 1)
+    per = max(256, rows // 4)
+    slices = [synth.make_batch(w, per, seed=300 + i) for i in range(cores)]
+    done = [0] * cores
+
+    def work(i):
+        t = time.perf_counter()
+        while time.perf_counter() - t < seconds / 2:
+            assert oracle.run(w.spec, slices[i])["status"] == "OK"
+            done[i] += 1
+
+    t0 = time.perf_counter()
+    with ThreadPoolExecutor(cores) as ex:
+        list(ex.map(work, range(cores)))
+    dtm = time.perf_counter() - t0
+    allc = sum(done) * per / dtm
+    return {"value": allc, "unit": UNIT, "cores": cores, "kind": "oracle", "cpu_model": cpu_model(),
+            "value_1thread": one,
+            "sample": f"{w.name}: {n} x {rows}-row batches on 1 thread ({dt1:.1f} s), then {sum(done)} x {per}-row "
+                      f"slices over {cores} threads ({dtm:.1f} s); plain C oracle, untuned"}
 
 
 def dist_env():
@@ -198,7 +234,7 @@ def run_reference(args):
     value = args.steps * rows / dt
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": 0,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64+f32",
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "int64+f32",
             "data": "synthetic",
             "config": {"workload": wname, "batch": B, "sample_rows_per_step": rows, "parallelism": "cpu-1thread"},
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
@@ -215,13 +251,7 @@ def run_rap(args):
     rank, world, local = dist_env()
     if world > 1:
         return run_sharded(args)
-    if world > 1:
-        import torch.distributed as dist
-
-        torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    else:
-        torch.cuda.set_device(0)
+    torch.cuda.set_device(0)
     dev = torch.device("cuda", torch.cuda.current_device())
     from paper_conf_asplos_wangwdz0d24_b200 import rap, synth
 
@@ -277,6 +307,7 @@ def run_rap(args):
         t_end.record(stream)
         t_end.synchronize()
     torch.cuda.synchronize()
+    info = plan.info()  # the launches just timed (kernel, grid)
     total_ms = t_start.elapsed_time(t_end)
     kern_ms = float(np.mean([ev_s[i].elapsed_time(ev_e[i]) for i in range(K)]))
     if world > 1:
@@ -304,7 +335,8 @@ def run_rap(args):
         h2d += sum(x.numel() * x.element_size() for x in hraw.sp_off)
         h2d += sum(int(n) * 8 for n in hraw.sp_nnz)
         h2d += sum(x.numel() * x.element_size() for x in hraw.sp_valid if x is not None)
-        d2h = (B * d_out * 4) + (B * f_out * 4) + (B * f_out + 1) * 8 + vb * 8
+        # values: exactly offsets[end] ids (the pinned-output copy kernel, include/rap.h)
+        d2h = (B * d_out * 4) + (B * f_out * 4) + (B * f_out + 1) * 8 + n_vals * 8
         for _ in range(3):
             plan.preprocess_host(hraw, hout, stream)
         if world > 1:
@@ -373,19 +405,23 @@ def run_rap(args):
         corun["training"] = "synthetic DLRM step (DESIGN.md §12): 26 tables x 128 fp32 (TB share at 8 GPUs), batch 8192"
         del train
         torch.cuda.empty_cache()
-    info = plan.info()
+    c4 = None
+    if world == 1 and not args.profile and not args.no_c4 and args.workload != "c4":
+        c4 = c4_point(dev, args.c4_batch, steps=20)
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": args.warmup,
-                "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+                "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
                 "dtype": "int64+f32", "data": "synthetic",
                 "config": {"workload": wname, "batch": B, "graph_ops": len(w.spec["nodes"]),
                            "dense_out_cols": d_out, "sparse_out_features": f_out,
                            "parallelism": "replicas" if world > 1 else "single-gpu",
                            "sm_budget": info["sm_budget"], "grid": info["grid"],
+                           "kernel": KERNEL_NAMES.get(info["kernel_last"], str(info["kernel_last"])),
+                           "jit_compile_s": round(info["jit_compile_seconds"], 2),
                            "l2_policy": f"rotate {nsets} distinct input/output sets, {nsets * set_bytes / 2**20:.0f} MB "
                                         f"total vs L2 {l2 / 2**20:.0f} MB"},
                 "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks, "gpu_launches": K,
-                "corun": corun, "fusion": fusion, "graph": graph}
+                "corun": corun, "fusion": fusion, "graph": graph, "c4": c4}
         print(json.dumps(line), flush=True)
     plan.close()
     if world > 1:
@@ -393,6 +429,49 @@ def run_rap(args):
 
         dist.destroy_process_group()
     return 0
+
+
+KERNEL_NAMES = {1: "tiled", 2: "rows (interpreted)", 3: "rows (generated, NVRTC sm_100a)"}
+
+
+def c4_point(dev, B, steps=20):
+    """Config 4 (512 multi-hot features, mean 20 ids, FirstX(32)) at B rows on
+    this GPU: kernel time and HBM fraction of the launch (the tiled kernel's
+    element-parallel multi-id tiles).  Rotating 2 batches (each > the L2)."""
+    import torch
+
+    from paper_conf_asplos_wangwdz0d24_b200 import rap, synth
+
+    w = synth.c4_multihot(0)
+    plan = rap.Plan(w.spec, device=dev.index)
+    sets = []
+    for i in range(2):
+        h = synth.make_batch(w, B, seed=700 + i)
+        r = rap.DeviceBatch(h, dev)
+        sets.append((h, r, rap.DeviceOutput(plan, B, r.sp_nnz, dev)))
+    stream = torch.cuda.current_stream(dev)
+    for i in range(4):
+        plan.preprocess(sets[i % 2][1], sets[i % 2][2], stream)
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for i in range(steps):
+        plan.preprocess(sets[i % 2][1], sets[i % 2][2], stream)
+    e1.record(stream)
+    e1.synchronize()
+    ms = e0.elapsed_time(e1) / steps
+    n_vals = int(sets[(steps - 1) % 2][2].offsets[-1].item())
+    alg = synth.algorithmic_bytes(w.spec, sets[(steps - 1) % 2][0], n_vals)
+    peak, _ = measured_peaks()
+    info = plan.info()
+    plan.close()
+    del sets
+    torch.cuda.empty_cache()
+    gbs = alg / (ms / 1e3) / 1e9
+    return {"workload": "multihot_c4", "batch": B, "kernel_ms": ms, "value": B / (ms / 1e3), "unit": UNIT,
+            "alg_bytes_per_launch": int(alg), "achieved_gbs": gbs, "frac": gbs / peak,
+            "kernel": KERNEL_NAMES.get(info["kernel_last"], str(info["kernel_last"])),
+            "note": f"config 4 at {B} of its 131072 rows (host generation of the full batch is ~20 GB)"}
 
 
 def graph_replay(plan, sets, B, dev, steps, alg_bytes):
@@ -449,7 +528,9 @@ def fusion_ablation(w, sets, B, dev, stream, fused_ms, steps):
     for o in w.spec["outputs"]:
         s = dict(w.spec)
         s["outputs"] = [o]
-        plans.append(rap.Plan(s, device=dev.index))
+        p = rap.Plan(s, device=dev.index)
+        p.set_kernel(rap.KERNEL_ROWS)  # one-output launches: the interpreted row-block kernel (no NVRTC per plan)
+        plans.append(p)
     nsets = len(sets)
     outs = [[rap.DeviceOutput(p, B, r.sp_nnz, dev) for p in plans] for r, _ in sets]
 
@@ -475,7 +556,8 @@ def fusion_ablation(w, sets, B, dev, stream, fused_ms, steps):
     torch.cuda.empty_cache()
     return {"fused_ms": fused_ms, "unfused_ms": unfused_ms, "launches_unfused": len(plans),
             "fusion_speedup": unfused_ms / fused_ms, "steps": steps,
-            "what": "one fused launch vs one launch per output feature (same kernel, same inputs)"}
+            "what": "one fused launch (the timed kernel) vs one launch per output feature (interpreted row-block "
+                    "kernel, same inputs)"}
 
 
 def run_sharded(args):

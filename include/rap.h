@@ -219,9 +219,11 @@ rap_status rap_preprocess(rap_plan* plan, const rap_raw_batch* raw, const rap_ou
 
 /* Same as rap_preprocess with HOST raw and output buffers (pinned memory makes
  * the copies asynchronous): copies the batch into plan-owned device staging,
- * launches, copies dense/lengths/offsets and the first values_upper_bound
- * values back, and synchronises `stream` before returning.  Host values beyond
- * offsets[end] are unspecified. */
+ * launches, copies dense/lengths/offsets and the values back, and
+ * synchronises `stream` before returning.  When `values` is pinned host
+ * memory, a copy kernel moves exactly offsets[end] ids into it (no host sync,
+ * no padding over PCIe); pageable memory receives the first
+ * values_upper_bound ids.  Host values beyond offsets[end] are unspecified. */
 rap_status rap_preprocess_host(rap_plan* plan, const rap_raw_batch* raw, const rap_output* out, void* stream);
 
 /* rap_preprocess_host without the final synchronisation: H2D copies, the

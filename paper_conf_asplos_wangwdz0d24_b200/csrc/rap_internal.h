@@ -288,6 +288,8 @@ int fused_smem_bytes(int max_width);
 // rap_jagged_append's kernel (rap_kernel.cu).
 int launch_jagged_append(const int32_t* len, const int64_t* so, const int64_t* val, int64_t n, int64_t vb, int32_t* dl,
                          int64_t* dof, int64_t* dv, int64_t cap, void* stream);
+// Exact-size copy of values[0, *total) into device-mapped pinned host memory (rap_kernel.cu).
+int launch_values_to_host(const int64_t* src, const int64_t* total, int64_t cap, int64_t* dst, void* stream);
 // Occupancy query: CTAs per SM for the given dynamic smem.
 int fused_occupancy(int smem_bytes, int n_dense, int n_sparse, int* ctas_per_sm);
 // Row-block kernel (rap_rows.cu): dynamic smem for a geometry, occupancy, launch.
@@ -311,6 +313,8 @@ struct JitPlanView {
   const DProg* dprogs;
   int n_dprogs, d_out, dense_bytes;  // dense_bytes: the kernel's dense-phase shared memory
   const int64_t* itab;               // the plan's int64 table pool (Bucketize borders, MapId tables)
+  const DevOp* ops;                  // global op pool (DUnit::gops = 1: units too large to stage)
+  const float* ftab;                 // global f32 border pool (DUnit::gops = 1)
 };
 struct JitModule;  // compiled kernels (opaque)
 // Generate the CUDA source of the plan's policy (small: 32-bit scans, every

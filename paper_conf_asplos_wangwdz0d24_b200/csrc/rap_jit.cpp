@@ -210,12 +210,11 @@ struct Gen {
     if (v.n_dprogs == 0 || v.d_out <= 0) return false;
     return tile_offset() + 32 * pitch() * 4 <= v.dense_bytes;
   }
-  static double unit_cost(const DProg& dp, const DUnit& un) {
-    const DevOp* ops = dp.ops;
+  double unit_cost(const DProg& dp, const DUnit& un) const {
+    const DevOp* ops = un.gops ? v.ops : dp.ops;
     double c = 8;
     if (un.kind == U_ONEHOT_G) return 200;
-    if (!un.gops)
-      for (int o = un.op_begin; o < un.op_end; ++o)
+    for (int o = un.op_begin; o < un.op_end; ++o)
         c += ops[o].kind == OK_LOGIT ? 40 : ops[o].kind == OK_BOXCOX ? 70 : 3;
     if (un.kind == U_ONEHOT_DB) c += 10 + un.width + un.bm / 2;
     return c;
@@ -269,7 +268,8 @@ struct Gen {
       return s;
     }
     s += "        float v = in" + i2s(un.src_col) + ";\n";
-    s += dense_ops(dp.ops, un.op_begin, un.op_end, "v");
+    const DevOp* uops = un.gops ? v.ops : dp.ops;  // gops: indices into the global pools
+    s += dense_ops(uops, un.op_begin, un.op_end, "v");
     if (un.kind == U_DENSE) {
       s += "        trow[" + i2s(col) + "] = v;\n      }\n";
       return s;
@@ -279,7 +279,7 @@ struct Gen {
       s += "        for (int k = 0; k < " + i2s(un.width) + "; ++k) trow[" + i2s(col) + " + k] = 0.0f;\n      }\n";
       return s;
     }
-    const float* bt = dp.ftab + un.btab;
+    const float* bt = (un.gops ? v.ftab : dp.ftab) + un.btab;
     if (un.bm <= 32) {
       s += "        int64_t b = 0";
       for (int i = 0; i < un.bm; ++i) s += " + (v >= " + f2lit(bt[i]) + ")";
@@ -291,7 +291,7 @@ struct Gen {
       *globals += "};\n";
       s += "        int64_t b = upper_bound(" + nm + ", " + i2s(un.bm) + ", v);\n";
     }
-    s += id_ops(dp.ops, un.iop_begin, un.iop_end, "b");
+    s += id_ops(uops, un.iop_begin, un.iop_end, "b");
     s += "        const int64_t d = b - " + lit64(un.k0) + ";\n";
     s += "#pragma unroll\n        for (int k = 0; k < " + i2s(un.width) + "; ++k) trow[" + i2s(col) +
          " + k] = d == k ? 1.0f : 0.0f;\n      }\n";
@@ -365,7 +365,7 @@ struct Gen {
          "    const bool in = tid < nr;\n"
          "    const int64_t row = c0 + tid;\n"
          "    bool ovf = false;\n"
-         "    unsigned late = 0;\n";
+         "    unsigned late = 0;\n    (void)late;\n";
     std::vector<int> late_q;
     int n_late = 0;
     // memo registers of the providers

@@ -1474,6 +1474,30 @@ __global__ void __launch_bounds__(256) jagged_append_kernel(const int32_t* __res
   }
 }
 
+// Exact-size D2H of a jagged output's values (rap_preprocess_host*): the
+// total is the device value *total (offsets[F * B]); the kernel writes
+// values[0, total) straight into pinned (device-mapped) host memory, so no
+// host sync is needed to learn the count and no padding crosses PCIe.
+__global__ void __launch_bounds__(256) values_to_host_kernel(const int64_t* __restrict__ src,
+                                                             const int64_t* __restrict__ total, int64_t cap,
+                                                             int64_t* __restrict__ dst) {
+  const int64_t n = min(*total, cap);
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  // 16-byte moves (both buffers come from 256-byte aligned allocations)
+  const int64_t n2 = n >> 1;
+  const longlong2* s2 = reinterpret_cast<const longlong2*>(src);
+  longlong2* d2 = reinterpret_cast<longlong2*>(dst);
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n2; i += stride) d2[i] = s2[i];
+  if ((n & 1) && blockIdx.x == 0 && threadIdx.x == 0) dst[n - 1] = src[n - 1];
+}
+
+int launch_values_to_host(const int64_t* src, const int64_t* total, int64_t cap, int64_t* dst, void* stream) {
+  const int64_t blocks = min((cap / 2 + 255) / 256, (int64_t)148 * 4);
+  values_to_host_kernel<<<(unsigned)max(blocks, (int64_t)1), 256, 0, reinterpret_cast<cudaStream_t>(stream)>>>(
+      src, total, cap, dst);
+  return (int)cudaGetLastError();
+}
+
 int launch_jagged_append(const int32_t* len, const int64_t* so, const int64_t* val, int64_t n, int64_t vb, int32_t* dl,
                          int64_t* dof, int64_t* dv, int64_t cap, void* stream) {
   const int64_t work = max(n, vb);

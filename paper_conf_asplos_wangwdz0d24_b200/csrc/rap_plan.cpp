@@ -822,6 +822,8 @@ JitPlanView jit_view(const rap_plan* P) {
   v.d_out = P->d_out;
   v.dense_bytes = P->rb_dense_bytes;
   v.itab = P->itab.data();
+  v.ops = P->ops.data();
+  v.ftab = P->ftab.data();
   return v;
 }
 
@@ -1802,8 +1804,23 @@ static rap_status preprocess_host_impl(rap_plan* P, const rap_raw_batch* raw, co
     if (B > 0) e = cudaMemcpyAsync(out->lengths, dl, sizeof(int32_t) * B * F, cudaMemcpyDeviceToHost, stream);
     if (e == cudaSuccess)
       e = cudaMemcpyAsync(out->offsets, dof, sizeof(int64_t) * (B * F + 1), cudaMemcpyDeviceToHost, stream);
-    if (e == cudaSuccess && vb > 0)
-      e = cudaMemcpyAsync(out->values, dv, sizeof(int64_t) * vb, cudaMemcpyDeviceToHost, stream);
+    if (e == cudaSuccess && vb > 0) {
+      // exact count: pinned host memory is device-mapped (UVA), so a copy
+      // kernel reads the total on the device and moves only the written ids;
+      // pageable memory gets the bounded copy
+      cudaPointerAttributes pa;
+      const bool pinned = cudaPointerGetAttributes(&pa, out->values) == cudaSuccess && pa.type == cudaMemoryTypeHost &&
+                          pa.devicePointer != nullptr && (reinterpret_cast<uintptr_t>(out->values) & 15) == 0;
+      cudaGetLastError();
+      if (pinned && !(out->flags & RAP_OUT_CHAIN)) {
+        const int rc = launch_values_to_host(static_cast<const int64_t*>(dv), static_cast<const int64_t*>(dof) + B * F,
+                                             std::min<int64_t>(vb, out->values_capacity),
+                                             static_cast<int64_t*>(pa.devicePointer), stream);
+        e = (cudaError_t)rc;
+      } else {
+        e = cudaMemcpyAsync(out->values, dv, sizeof(int64_t) * vb, cudaMemcpyDeviceToHost, stream);
+      }
+    }
     if (e != cudaSuccess) return cuda_fail(e, "D2H sparse");
   } else if (out->offsets) {
     out->offsets[0] = 0;  // no sparse outputs: the single total (HOST buffer)

@@ -1,0 +1,171 @@
+"""Edge-case parity of every fused kernel against the CPU oracle (VERDICT r01
+"parity holes"): table sizes M >= 2^32 (the 64x64 multiply-high reduction),
+a MapId table holding INT64_MIN, NGram over k = 5..8 sources, programs longer
+than the 32 ops an SProg stages and dense groups beyond 96 ops, Clamp and ids
+at INT64_MIN / INT64_MAX, and the device-side capacity-overflow flag
+(rap_check_overflow).  Integer outputs bit-exact, dense within R16
+(tests/parity.py).  PAPER.md Table 1 (L440-463); readings DESIGN.md §3.
+"""
+import numpy as np
+import pytest
+
+from tests.helpers import batch, dense_from_values, node, sparse_from_lists, spec
+from tests.parity import assert_parity
+
+pytestmark = pytest.mark.gpu
+
+I64_MIN, I64_MAX = -(2**63), 2**63 - 1
+
+
+@pytest.fixture(scope="module")
+def env():
+    import torch
+
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    from paper_conf_asplos_wangwdz0d24_b200 import rap, synth
+    from oracle import oracle
+
+    rap.load()
+    return rap, synth, oracle, torch
+
+
+@pytest.fixture(params=[1, 2, 3], ids=["tiled", "rows", "jit"])
+def kmode(request):
+    return request.param
+
+
+def run_check(env, kmode, s, host, ctx=""):
+    rap, synth, oracle, torch = env
+    want = oracle.run(s, host)
+    plan = rap.Plan(s, device=0)
+    plan.set_kernel(kmode)
+    raw = rap.DeviceBatch(host, "cuda:0")
+    out = rap.DeviceOutput(plan, host["n_rows"], raw.sp_nnz, "cuda:0")
+    plan.preprocess(raw, out)
+    torch.cuda.synchronize()
+    got = out.to_numpy()
+    assert plan.check_overflow() == 0
+    plan.close()
+    assert_parity(got, want, ctx)
+    return got
+
+
+def _lists(rng, n, lo, hi, max_len=3, p_null=0.1, extremes=()):
+    rows = []
+    for _ in range(n):
+        if rng.random() < p_null:
+            rows.append(None)
+            continue
+        k = int(rng.integers(0, max_len + 1))
+        rows.append([int(v) for v in rng.integers(lo, hi, k)])
+    for i, e in enumerate(extremes):  # pin a few rows to the extremes
+        rows[(7 * i + 3) % n] = [e]
+    return rows
+
+
+def test_large_M_sigrid_and_ngram(env, kmode):
+    """M = 2^32, 2^40, 2^63 - 1: the reduction floor(h * M / 2^64) on the
+    __umul64hi path (R2), for SigridHash and for NGram windows (R3, R7)."""
+    rng = np.random.default_rng(1)
+    B = 1500
+    sp = [sparse_from_lists(_lists(rng, B, -(2**40), 2**40, extremes=(I64_MIN, I64_MAX, 0, -1)))
+          for _ in range(2)]
+    nodes, outs = [], []
+    for k, M in enumerate((2**32, 2**40, 2**63 - 1)):
+        nodes.append(node("sigridhash", [("s", 0)], salt=11 + k, max_value=M))
+        outs.append(len(nodes) - 1)
+        nodes.append(node("ngram", [("s", 0), ("s", 1)], n=2, salt=5 + k, max_value=M))
+        outs.append(len(nodes) - 1)
+    nodes.append(node("fillnull", [("s", 1)], i_fill=I64_MIN))
+    nodes.append(node("sigridhash", [("n", len(nodes) - 1)], salt=3, max_value=2**63 - 1))
+    outs.append(len(nodes) - 1)
+    run_check(env, kmode, spec(0, 2, nodes, outs), batch(B, sparse=sp))
+
+
+def test_mapid_int64_min_key_and_clamp_extremes(env, kmode):
+    """A MapId table holding INT64_MIN (the interpreter's has_min path, R8) and
+    Clamp at the int64 extremes (identity bounds and pinned bounds, R6)."""
+    rng = np.random.default_rng(2)
+    B = 1300
+    rows = _lists(rng, B, -50, 50, extremes=(I64_MIN, I64_MAX, I64_MIN, 0))
+    sp = sparse_from_lists(rows)
+    keys = np.array([I64_MIN, 0, 5, -7, I64_MAX, 42], dtype=np.int64)
+    vals = np.array([111, 222, 333, 444, 555, I64_MIN], dtype=np.int64)
+    nodes = [node("mapid", [("s", 0)], keys=keys, vals=vals, map_default=-9),
+             node("clamp", [("s", 0)], lo=I64_MIN, hi=I64_MAX),
+             node("clamp", [("s", 0)], lo=I64_MIN, hi=I64_MIN),
+             node("clamp", [("s", 0)], lo=I64_MAX, hi=I64_MAX),
+             node("clamp", [("s", 0)], lo=-3, hi=I64_MAX),
+             node("fillnull", [("s", 0)], i_fill=I64_MAX),
+             node("mapid", [("n", 5)], keys=keys, vals=vals, map_default=I64_MIN),
+             node("sigridhash", [("n", 6)], salt=I64_MAX, max_value=2**40)]
+    run_check(env, kmode, spec(0, 1, nodes, [0, 1, 2, 3, 4, 6, 7]), batch(B, sparse=[sp]))
+
+
+@pytest.mark.parametrize("k", [5, 6, 7, 8])
+def test_ngram_many_sources(env, kmode, k):
+    """NGram over k = 5..8 source lists (R7: concatenation in source order),
+    windows n in {2, k} so rows with several windows and exactly one occur."""
+    rng = np.random.default_rng(10 + k)
+    B = 900
+    sp = [sparse_from_lists(_lists(rng, B, 0, 10**6, max_len=2, p_null=0.2)) for _ in range(k)]
+    nodes = [node("fillnull", [("s", i)], i_fill=i) for i in range(k)]
+    nodes.append(node("ngram", [("n", i) for i in range(k)], n=2, salt=9, max_value=10**7))
+    nodes.append(node("ngram", [("s", i) for i in range(k)], n=k, salt=8, max_value=2**35))
+    nodes.append(node("firstx", [("n", k)], x=3))
+    run_check(env, kmode, spec(0, k, nodes, [k, k + 1, k + 2]), batch(B, sparse=sp))
+
+
+def test_long_programs(env, kmode):
+    """An id chain of 40 ops (beyond the 32 an SProg stages: global op indices)
+    and a dense group of 120 ops (beyond the 96 a DProg stages)."""
+    rng = np.random.default_rng(3)
+    B = 1100
+    sp = sparse_from_lists(_lists(rng, B, -(2**33), 2**33, max_len=4))
+    nodes, cur = [], ("s", 0)
+    for i in range(40):
+        if i % 3 == 0:
+            nodes.append(node("clamp", [cur], lo=-(2**34) + i, hi=2**34 - i))
+        elif i % 3 == 1:
+            nodes.append(node("sigridhash", [cur], salt=i, max_value=2**31 + i))
+        else:
+            nodes.append(node("mapid", [cur], keys=np.arange(i, i + 40, dtype=np.int64),
+                              vals=np.arange(40, dtype=np.int64) * 3, map_default=-i))
+        cur = ("n", len(nodes) - 1)
+    outs = [len(nodes) - 1]
+    vals = [0.1, 0.5, 0.9, None, float("nan"), 2.0, 0.0, 1.0] * (B // 8 + 1)
+    d = dense_from_values(vals[:B])
+    for c in range(30):  # 30 dense outputs x (FillNull, Logit, BoxCox, FillNull) = 120 ops over the groups
+        nodes.append(node("fillnull", [("d", 0)], f_fill=0.25 + 0.01 * c))
+        nodes.append(node("logit", [("n", len(nodes) - 1)], eps=1e-6 * (c + 1)))
+        nodes.append(node("boxcox", [("n", len(nodes) - 1)], **{"lambda": 0.5}))
+        nodes.append(node("fillnull", [("n", len(nodes) - 1)], f_fill=-1.0))
+        outs.append(len(nodes) - 1)
+    # one dense chain of 101 ops (more than a DProg carries: global op indices)
+    cur = ("d", 0)
+    for i in range(100):
+        nodes.append(node("fillnull", [cur], f_fill=0.125 * (i % 5)))
+        cur = ("n", len(nodes) - 1)
+    nodes.append(node("logit", [cur], eps=1e-3))
+    outs.append(len(nodes) - 1)
+    run_check(env, kmode, spec(1, 1, nodes, outs), batch(B, dense=[d], sparse=[sp]))
+
+
+def test_capacity_overflow_flag(env, kmode):
+    """sp_nnz understating the batch: values past values_capacity are not
+    written and rap_check_overflow reports it (then clears it)."""
+    rap, synth, oracle, torch = env
+    w = synth.c1_kaggle(0)
+    host = synth.make_batch(w, 3000, seed=2)
+    plan = rap.Plan(w.spec, device=0)
+    plan.set_kernel(kmode)
+    raw = rap.DeviceBatch(host, "cuda:0")
+    small = np.zeros_like(raw.sp_nnz)  # claims empty columns: bound = 0 ids
+    raw.sp_nnz[:] = small
+    out = rap.DeviceOutput(plan, 3000, raw.sp_nnz, "cuda:0", capacity=100)
+    plan.preprocess(raw, out)
+    torch.cuda.synchronize()
+    assert plan.check_overflow() == 1
+    assert plan.check_overflow() == 0  # cleared
+    plan.close()

@@ -54,3 +54,20 @@ def test_unsupported_plan(rap):
     nodes = [node("sigridhash", [("s", c)], salt=c, max_value=100) for c in range(70)]
     st, src, ok, log = rap.jit_source(spec(0, 70, nodes, list(range(70))), compile=False)
     assert st == "UNSUPPORTED"
+
+
+def test_dense_chain_beyond_staged_ops(rap):
+    """A dense chain of 101 ops exceeds what a DProg stages (kMaxDenseOps):
+    its unit refers to the plan's global op pool (DUnit::gops), and the
+    generated code must take those ops, not the DProg's staged array."""
+    nodes, cur = [], ("d", 0)
+    for i in range(100):
+        nodes.append(node("fillnull", [cur], f_fill=0.125 * (i % 5)))
+        cur = ("n", len(nodes) - 1)
+    nodes.append(node("logit", [cur], eps=1e-3))
+    nodes.append(node("sigridhash", [("s", 0)], salt=1, max_value=100))
+    st, src, ok, log = rap.jit_source(spec(1, 1, nodes, [100, 101]), compile=False)
+    assert st == "OK", log
+    assert src.count("if (isnan(v)) v = ") == 100
+    assert src.count("v = logf(__fdiv_rn(z, __fsub_rn(1.0f, z)))") == 1
+    assert "expm1f" not in src  # no BoxCox in the graph
