@@ -214,7 +214,14 @@ rap_status rap_plan_output_shape(const rap_plan* plan, int64_t n_rows, const int
  * of device data.  A batch whose shape (rows, grid, quantised mean list
  * lengths) is new uploads its per-warp work partition (async, pinned); the
  * plan caches 8 shapes and only evicting one synchronises `stream`.  Outputs
- * are valid when the stream reaches this point. */
+ * are valid when the stream reaches this point.
+ * CUDA-graph capture: a captured call bakes in its shape's cached partition
+ * slot, which is then pinned for the plan's lifetime (later eager calls never
+ * overwrite what a replay reads).  A replay must see the same batch shape it
+ * was captured with (rows; sp_nnz may vary within the cached shape).  A shape
+ * first seen during capture takes a free slot; when none is left (8 shapes
+ * cached) the call returns RAP_ERR_UNSUPPORTED instead of evicting -- launch
+ * each shape once before capturing. */
 rap_status rap_preprocess(rap_plan* plan, const rap_raw_batch* raw, const rap_output* out, void* stream);
 
 /* Same as rap_preprocess with HOST raw and output buffers (pinned memory makes

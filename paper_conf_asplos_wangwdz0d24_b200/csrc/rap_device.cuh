@@ -649,7 +649,9 @@ __device__ __noinline__ void dense_block(const P& p, int gi, int64_t rb, int sme
                                           (reinterpret_cast<uintptr_t>(p.dvalid[col] + (g0 >> 5)) & 15) == 0)));
     const bool stage = __all_sync(0xffffffffu, aligned) && (nr & 3) == 0 && nc <= 16;
     if (stage) {
-      const uint32_t bytes_v = (uint32_t)nr * 4, bytes_b = (uint32_t)align_up(nw * 4, 16);
+      // validity: the 16-byte body by the bulk copy, the <= 3 tail words by
+      // plain loads (a bitmap holds exactly ceil(B/32) words: never read past)
+      const uint32_t bytes_v = (uint32_t)nr * 4, bytes_b = (uint32_t)(nw * 4) & ~15u;
       uint32_t total = 0;
       if (lane < nc) total = bytes_v + (p.dvalid[col] ? bytes_b : 0);
 #pragma unroll
@@ -661,7 +663,10 @@ __device__ __noinline__ void dense_block(const P& p, int gi, int64_t rb, int sme
       __syncwarp();
       if (lane < nc) {
         bulk_g2s(din + lane * kDenseBlockRows, p.dense[col] + g0, bytes_v, &cs.bar);
-        if (p.dvalid[col]) bulk_g2s(dbm + lane * 8, p.dvalid[col] + (g0 >> 5), bytes_b, &cs.bar);
+        if (p.dvalid[col]) {
+          if (bytes_b) bulk_g2s(dbm + lane * 8, p.dvalid[col] + (g0 >> 5), bytes_b, &cs.bar);
+          for (int i = (int)(bytes_b / 4); i < nw; ++i) dbm[lane * 8 + i] = __ldg(p.dvalid[col] + (g0 >> 5) + i);
+        }
       }
     }
     if (lane == 0) cs.staged = stage ? 1 : 0;

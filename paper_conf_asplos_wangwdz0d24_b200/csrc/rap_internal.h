@@ -290,6 +290,11 @@ int launch_jagged_append(const int32_t* len, const int64_t* so, const int64_t* v
                          int64_t* dof, int64_t* dv, int64_t cap, void* stream);
 // Exact-size copy of values[0, *total) into device-mapped pinned host memory (rap_kernel.cu).
 int launch_values_to_host(const int64_t* src, const int64_t* total, int64_t cap, int64_t* dst, void* stream);
+// Raise a kernel's MaxDynamicSharedMemorySize on the current device to at
+// least smem (never lowers it: plans of different geometries share the kernel,
+// so an attribute set for one plan must stay valid for every other).  One
+// process-wide record per (kernel, device), mutex-guarded.  rap_kernel.cu.
+int ensure_dyn_smem(const void* kernel, int smem);
 // Occupancy query: CTAs per SM for the given dynamic smem.
 int fused_occupancy(int smem_bytes, int n_dense, int n_sparse, int* ctas_per_sm);
 // Row-block kernel (rap_rows.cu): dynamic smem for a geometry, occupancy, launch.

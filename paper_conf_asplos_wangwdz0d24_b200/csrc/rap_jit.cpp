@@ -40,9 +40,7 @@ namespace rapk {
 struct JitModule {
   cudaLibrary_t lib = nullptr;
   cudaKernel_t k = nullptr;
-  int smem_set = -1;
   double compile_s = 0;
-  std::mutex mu;
 };
 
 namespace {
@@ -645,9 +643,9 @@ double jit_compile_seconds(const JitModule* m) { return m ? m->compile_s : 0.0; 
 
 int jit_occupancy(JitModule* m, int smem_bytes, int* ctas_per_sm) {
   const void* k = reinterpret_cast<const void*>(m->k);
-  cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
-  if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(ctas_per_sm, k, kRbChunk, smem_bytes);
-  return (int)e;
+  const int rc = ensure_dyn_smem(k, smem_bytes);
+  if (rc != 0) return rc;
+  return (int)cudaOccupancyMaxActiveBlocksPerMultiprocessor(ctas_per_sm, k, kRbChunk, smem_bytes);
 }
 
 // Same parameter block as rap_rows.cu's kernel (RbParams<kRbMaxDense, kRbMaxCols>).
@@ -664,14 +662,8 @@ struct JitParams {
 int launch_jit(JitModule* m, const Common& c, const RbGeom& g, const LaunchRaw& raw, int smem_bytes, void* stream) {
   if (raw.n_dense > kRbMaxDense || raw.n_sparse > kRbMaxCols) return (int)cudaErrorInvalidValue;
   const void* k = reinterpret_cast<const void*>(m->k);
-  {
-    std::lock_guard<std::mutex> lk(m->mu);
-    if (m->smem_set != smem_bytes) {
-      cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
-      if (e != cudaSuccess) return (int)e;
-      m->smem_set = smem_bytes;
-    }
-  }
+  const int rc = ensure_dyn_smem(k, smem_bytes);
+  if (rc != 0) return rc;
   JitParams p;
   memset(&p, 0, sizeof(p));
   p.c = c;

@@ -27,6 +27,10 @@
 #include <stdint.h>
 #include <string.h>
 
+#include <map>
+#include <mutex>
+#include <utility>
+
 #include "rap_internal.h"
 #include "rap_device.cuh"
 
@@ -93,6 +97,8 @@ struct FeatCtx {
   int64_t xcap, null_xcap, fill;
   Canon q;  // canonical pipeline (TK_CANON), in registers
 };
+
+__device__ __forceinline__ int64_t clamp_tile(int64_t t, int64_t lo, int64_t hi) { return t < lo ? lo : (t > hi ? hi : t); }
 
 template <class P>
 __device__ __forceinline__ void load_ctx(const P& p, int f, FeatCtx& x) {
@@ -1197,8 +1203,12 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
   }
   const int64_t S = p.c.n_sparse_tiles, T = p.c.tiles_per_feature;
   // my sparse tiles [s0, s1) and my warp's [w0, w1) (host per-warp partition)
-  const int64_t s0 = __ldg(p.c.part + rank * kWarps), s1 = __ldg(p.c.part + (rank + 1) * kWarps);
-  const int64_t w0 = __ldg(p.c.part + rank * kWarps + warp), w1 = __ldg(p.c.part + rank * kWarps + warp + 1);
+  // (clamped to [0, S]: a partition of another batch shape -- a misuse of a
+  // captured graph, rap.h -- can leave tiles unwritten but never leave S)
+  const int64_t s0 = clamp_tile(__ldg(p.c.part + rank * kWarps), 0, S);
+  const int64_t s1 = clamp_tile(__ldg(p.c.part + (rank + 1) * kWarps), s0, S);
+  const int64_t w0 = clamp_tile(__ldg(p.c.part + rank * kWarps + warp), 0, S);
+  const int64_t w1 = clamp_tile(__ldg(p.c.part + rank * kWarps + warp + 1), w0, S);
   unsigned char* wscr = smem + warp * kWarpScr;  // warp-private region (sparse phases)
   int32_t* scr = reinterpret_cast<int32_t*>(wscr);
   if (p.c.trace != nullptr && tid == 0 && (int64_t)blockIdx.x < p.c.trace_cap)
@@ -1222,7 +1232,11 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
         fend = (int64_t)(fcur + 1) * T;
       }
       const int f = fcur;
-      if (f != fc.f) load_ctx(p, f, fc);
+      // every lane reads the cached feature before any lane rewrites it
+      // (independent thread scheduling: racecheck WAR otherwise)
+      const bool reload = f != fc.f;
+      __syncwarp();
+      if (reload) load_ctx(p, f, fc);  // ends with __syncwarp
       const int64_t tend = min(w1, (int64_t)(f + 1) * T);
       if (fc.sk == SRC_SPARSE) {
         // kLChunkTiles tiles' offsets and validity words staged per round
@@ -1334,7 +1348,9 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
         fend = (int64_t)(fcur + 1) * T;
       }
       const int f = fcur;
-      if (f != fc.f) load_ctx(p, f, fc);
+      const bool reload = f != fc.f;
+      __syncwarp();
+      if (reload) load_ctx(p, f, fc);  // ends with __syncwarp
       if (fc.kind == TK_CANON) {
         const int nt = (int)min((int64_t)kVChunkTiles, min(w1, (int64_t)(f + 1) * T) - t);
         const long long got = value_chunk_canon(p, fc, t - (int64_t)f * T, nt, lane, run, wscr);
@@ -1386,12 +1402,8 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
 template <int MD, int MS>
 static int launch_t(const Common& c, const LaunchRaw& raw, int grid, int smem, cudaStream_t st) {
   static_assert(sizeof(KParams<MD, MS>) <= 32000, "kernel parameter block too large");
-  static int configured_smem = -1;
-  if (configured_smem < smem) {
-    cudaError_t e = cudaFuncSetAttribute(rap_fused_kernel<MD, MS>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    if (e != cudaSuccess) return (int)e;
-    configured_smem = smem;
-  }
+  const int rc = ensure_dyn_smem(reinterpret_cast<const void*>(rap_fused_kernel<MD, MS>), smem);
+  if (rc != 0) return rc;
   KParams<MD, MS> p;
   memset(&p, 0, sizeof(p));
   p.c = c;
@@ -1433,19 +1445,27 @@ int fused_smem_bytes(int max_width) {
   return dense > kNgScratch ? dense : kNgScratch;
 }
 
+int ensure_dyn_smem(const void* kernel, int smem) {
+  static std::mutex mu;
+  static std::map<std::pair<const void*, int>, int> set;  // (kernel, device) -> attribute value
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return (int)e;
+  std::lock_guard<std::mutex> lk(mu);
+  int& cur = set[std::make_pair(kernel, dev)];
+  if (cur >= smem) return 0;
+  e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e != cudaSuccess) return (int)e;
+  cur = smem;
+  return 0;
+}
+
 int fused_occupancy(int smem_bytes, int n_dense, int n_sparse, int* ctas_per_sm) {
-  cudaError_t e;
-  if (n_dense <= 32 && n_sparse <= 64) {
-    e = cudaFuncSetAttribute(rap_fused_kernel<32, 64>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
-    if (e == cudaSuccess)
-      e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(ctas_per_sm, rap_fused_kernel<32, 64>, kThreads, smem_bytes);
-  } else {
-    e = cudaFuncSetAttribute(rap_fused_kernel<128, 1024>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
-    if (e == cudaSuccess)
-      e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(ctas_per_sm, rap_fused_kernel<128, 1024>, kThreads,
-                                                        smem_bytes);
-  }
-  return (int)e;
+  const void* k = n_dense <= 32 && n_sparse <= 64 ? reinterpret_cast<const void*>(rap_fused_kernel<32, 64>)
+                                                  : reinterpret_cast<const void*>(rap_fused_kernel<128, 1024>);
+  const int rc = ensure_dyn_smem(k, smem_bytes);
+  if (rc != 0) return rc;
+  return (int)cudaOccupancyMaxActiveBlocksPerMultiprocessor(ctas_per_sm, k, kThreads, smem_bytes);
 }
 
 }  // namespace rapk

@@ -90,6 +90,7 @@ struct rap_plan {
   // kPartSlots cached partitions (batches of different shapes alternate
   // without re-uploads); slot i: key part_keys[i], device d_part + i * kPartLen
   std::vector<std::vector<int64_t>> part_keys;
+  std::vector<char> part_pin;  // slot used by a launch captured into a CUDA graph: never evicted
   int part_next = 0;
   int64_t* d_part = nullptr;               // [kPartSlots * kPartLen]
   int64_t* h_part = nullptr;               // pinned staging, same layout
@@ -1411,15 +1412,26 @@ static rap_status update_partition(rap_plan* P, int64_t B, const int64_t* nnz, i
                                    cudaStream_t stream, const int64_t** d_part_out) {
   std::vector<int64_t> key = {B, grid};
   (void)D;
+  // a launch captured into a CUDA graph bakes in its slot (and, on a miss, the
+  // upload from the pinned staging slot): such slots are pinned for the plan's
+  // lifetime, so later eager calls never overwrite what a replay reads
+  cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
+  if (cudaStreamIsCapturing(stream, &cap) != cudaSuccess) {
+    cudaGetLastError();
+    cap = cudaStreamCaptureStatusNone;
+  }
+  const bool capturing = cap != cudaStreamCaptureStatusNone;
+  auto use = [&](size_t i) {
+    if (capturing) P->part_pin[i] = 1;
+    *d_part_out = P->d_part + i * kPartLen;
+    return RAP_OK;
+  };
   for (int s : P->used_sparse) {
     const double m = nnz && B > 0 ? (double)std::max<int64_t>(nnz[s], 0) / (double)B : 0.0;
     key.push_back(m <= 1.0 / 64 ? -1000 : (int64_t)std::lround(4.0 * std::log2(m)));
   }
   for (size_t i = 0; i < P->part_keys.size(); ++i)
-    if (P->part_keys[i] == key) {
-      *d_part_out = P->d_part + i * kPartLen;
-      return RAP_OK;
-    }
+    if (P->part_keys[i] == key) return use(i);
   // A partition only balances work: any cached one with the same rows and grid
   // covers exactly the same tiles, so a batch whose quantised mean lengths are
   // within one step of a cached shape reuses it (no re-plan, upload or slot
@@ -1430,10 +1442,7 @@ static rap_status update_partition(rap_plan* P, int64_t B, const int64_t* nnz, i
     if (k.size() != key.size() || k[0] != key[0] || k[1] != key[1]) continue;
     bool near = true;
     for (size_t j = 2; j < k.size() && near; ++j) near = std::llabs(k[j] - key[j]) <= 1;
-    if (near) {
-      *d_part_out = P->d_part + i * kPartLen;
-      return RAP_OK;
-    }
+    if (near) return use(i);
   }
   const int64_t F = (int64_t)P->souts.size();
   const int64_t T = F ? S / F : 0;
@@ -1454,14 +1463,28 @@ static rap_status update_partition(rap_plan* P, int64_t B, const int64_t* nnz, i
   // ranks (block d to rank d mod grid) and are not charged here: the CTAs of
   // an SM share its issue slots, so a dense block mostly fills slots its SM
   // neighbours leave idle (measured: charging it made C2 slower).
-  const int slot = (int)P->part_keys.size() < kPartSlots ? (int)P->part_keys.size() : P->part_next;
+  int slot = -1;
+  const bool evict = (int)P->part_keys.size() == kPartSlots;
+  if (!evict) {
+    slot = (int)P->part_keys.size();
+  } else {
+    for (int k = 0; k < kPartSlots && slot < 0; ++k) {
+      const int c = (P->part_next + k) % kPartSlots;
+      if (!P->part_pin[c]) slot = c;
+    }
+    if (slot < 0) return fail(RAP_ERR_UNSUPPORTED, "every partition slot is pinned by a captured CUDA graph");
+    // an eviction syncs the stream (the staging slot may feed an in-flight
+    // upload), which a capture cannot do
+    if (capturing) return fail(RAP_ERR_UNSUPPORTED, "a new batch shape during CUDA-graph capture needs a free "
+                                                   "partition slot: launch each shape once before capturing");
+  }
   P->part_next = (slot + 1) % kPartSlots;
   int64_t* part = P->h_part + (size_t)slot * kPartLen;
   const int n = grid * kWarpsPerCta;
   // evicting: the pinned slot may still feed an in-flight upload (only
   // after kPartSlots distinct batch shapes; never in steady state)
   cudaError_t e = cudaSuccess;
-  if ((int)P->part_keys.size() == kPartSlots) e = cudaStreamSynchronize(stream);
+  if (evict) e = cudaStreamSynchronize(stream);
   if (e != cudaSuccess) return cuda_fail(e, "partition slot reuse");
   part[0] = 0;
   double acc = 0;
@@ -1476,10 +1499,13 @@ static rap_status update_partition(rap_plan* P, int64_t B, const int64_t* nnz, i
   e = cudaMemcpyAsync(d, part, sizeof(int64_t) * (n + 1), cudaMemcpyHostToDevice, stream);
   if (e != cudaSuccess) return cuda_fail(e, "partition upload");
   P->partition_uploads += 1;
-  if ((int)P->part_keys.size() < kPartSlots)
+  if ((int)P->part_keys.size() < kPartSlots) {
     P->part_keys.push_back(key);
-  else
+    P->part_pin.push_back(0);
+  } else {
     P->part_keys[slot] = key;
+  }
+  if (capturing) P->part_pin[slot] = 1;
   *d_part_out = d;
   return RAP_OK;
 }

@@ -51,18 +51,8 @@ __global__ void __launch_bounds__(kRbChunk, RAP_RB_MIN_CTAS) rap_rows_kernel(con
 template <int MD, int MS, bool kSmall>
 static int launch_rows_t(const Common& c, const RbGeom& g, const LaunchRaw& raw, int smem, cudaStream_t st) {
   static_assert(sizeof(RbParams<MD, MS>) <= 32000, "kernel parameter block too large");
-  // the attribute is set on every launch whose smem differs from the value
-  // last set on this device (plans with different geometries alternate)
-  static thread_local int last_dev = -1, last_smem = -1;
-  int dev = 0;
-  cudaGetDevice(&dev);
-  if (dev != last_dev || smem != last_smem) {
-    cudaError_t e = cudaFuncSetAttribute(rap_rows_kernel<MD, MS, kSmall>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         smem);
-    if (e != cudaSuccess) return (int)e;
-    last_dev = dev;
-    last_smem = smem;
-  }
+  const int rc = ensure_dyn_smem(reinterpret_cast<const void*>(rap_rows_kernel<MD, MS, kSmall>), smem);
+  if (rc != 0) return rc;
   RbParams<MD, MS> p;
   memset(&p, 0, sizeof(p));
   p.c = c;
@@ -115,15 +105,12 @@ int rows_smem_bytes(int dense_bytes, int max_fl, int max_cols, int n_memo, int n
 }
 
 int rows_occupancy(int smem_bytes, int* ctas_per_sm) {
-  cudaError_t e = cudaFuncSetAttribute(rap_rows_kernel<kRbMaxDense, kRbMaxCols, true>,
-                                       cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
-  if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(rap_rows_kernel<kRbMaxDense, kRbMaxCols, false>,
-                             cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
-  if (e == cudaSuccess)
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(ctas_per_sm, rap_rows_kernel<kRbMaxDense, kRbMaxCols, true>,
-                                                      kRbChunk, smem_bytes);
-  return (int)e;
+  const void* k32 = reinterpret_cast<const void*>(rap_rows_kernel<kRbMaxDense, kRbMaxCols, true>);
+  const void* k64 = reinterpret_cast<const void*>(rap_rows_kernel<kRbMaxDense, kRbMaxCols, false>);
+  int rc = ensure_dyn_smem(k32, smem_bytes);
+  if (rc == 0) rc = ensure_dyn_smem(k64, smem_bytes);
+  if (rc != 0) return rc;
+  return (int)cudaOccupancyMaxActiveBlocksPerMultiprocessor(ctas_per_sm, k32, kRbChunk, smem_bytes);
 }
 
 }  // namespace rapk

@@ -304,9 +304,12 @@ class DeviceOutput:
         B, d, f = self.n_rows, self.d_out, self.f_out
         off = self.offsets.cpu().numpy()
         n = int(off[-1]) if len(off) else 0
-        return {"dense": self.dense.cpu().numpy()[: B * self.ld].reshape(B, self.ld)[:, :d],
-                "lengths": self.lengths.cpu().numpy()[: B * f], "offsets": off,
-                "values": self.values.cpu().numpy()[:n]}
+        # only the written elements are read (never the capacity tail or the
+        # ld padding columns: initcheck-clean)
+        dense = self.dense[: B * self.ld].view(B, self.ld)[:, :d] if B * self.ld else self.dense[:0].view(B, d)
+        return {"dense": dense.contiguous().cpu().numpy(),
+                "lengths": self.lengths[: B * f].cpu().numpy(), "offsets": off,
+                "values": self.values[:n].cpu().numpy()}
 
 
 class Plan:

@@ -169,3 +169,109 @@ def test_capacity_overflow_flag(env, kmode):
     assert plan.check_overflow() == 1
     assert plan.check_overflow() == 0  # cleared
     plan.close()
+
+
+def test_plans_with_different_smem_interleave(env, kmode):
+    """plan A (a 300-wide OneHot group: large dynamic smem) is
+    launched, plan B (small smem) is created and launched, then A launches
+    again -- the kernels' MaxDynamicSharedMemorySize must still admit A."""
+    rap, synth, oracle, torch = env
+    rng = np.random.default_rng(4)
+    B = 700
+    sp = sparse_from_lists(_lists(rng, B, 0, 300, max_len=2))
+    wide = spec(0, 1, [node("onehot", [("s", 0)], k=300), node("sigridhash", [("s", 0)], salt=1, max_value=1000)],
+                [0, 1])
+    host = batch(B, sparse=[sp])
+    want_a = oracle.run(wide, host)
+    w = synth.c1_kaggle(0)
+    hb = synth.make_batch(w, 500, seed=9)
+    want_b = oracle.run(w.spec, hb)
+
+    def launch(plan, h):
+        raw = rap.DeviceBatch(h, "cuda:0")
+        out = rap.DeviceOutput(plan, h["n_rows"], raw.sp_nnz, "cuda:0")
+        plan.preprocess(raw, out)
+        torch.cuda.synchronize()
+        return out.to_numpy()
+
+    a = rap.Plan(wide, device=0)
+    a.set_kernel(kmode)
+    assert_parity(launch(a, host), want_a, "A first")
+    b = rap.Plan(w.spec, device=0)
+    b.set_kernel(kmode)
+    assert_parity(launch(b, hb), want_b, "B")
+    assert_parity(launch(a, host), want_a, "A after B")
+    c = rap.Plan(w.spec, device=0)  # another small plan created between launches
+    assert_parity(launch(a, host), want_a, "A after C created")
+    for p in (a, b, c):
+        p.close()
+
+
+def _exact_nnz_lists(B, nnz, seed):
+    """B lists with exactly nnz ids (lengths 0..2*nnz/B), no nulls."""
+    rng = np.random.default_rng(seed)
+    lens = np.full(B, nnz // B)
+    lens[: nnz - lens.sum()] += 1
+    rng.shuffle(lens)
+    return [[int(v) for v in rng.integers(0, 10**6, n)] for n in lens]
+
+
+def test_partition_cache_near_shape_reuse(env):
+    """a batch whose mean list length sits one 2^(1/4) step from a
+    cached shape reuses that partition (no upload); a farther one uploads.
+    Tiled kernel (the only one with a per-warp partition)."""
+    rap, synth, oracle, torch = env
+    B = 1000
+    s = spec(0, 1, [node("sigridhash", [("s", 0)], salt=3, max_value=10**5)], [0])
+    plan = rap.Plan(s, device=0)
+    plan.set_kernel(rap.KERNEL_TILED)
+    # 4*log2(mean): 6.16 -> 10.49 (key 10), 6.19 -> 10.52 (key 11), 9.0 -> 12.68 (key 13)
+    ups = []
+    for nnz in (6160, 6190, 6160, 9000):
+        host = batch(B, sparse=[sparse_from_lists(_exact_nnz_lists(B, nnz, nnz))])
+        raw = rap.DeviceBatch(host, "cuda:0")
+        out = rap.DeviceOutput(plan, B, raw.sp_nnz, "cuda:0")
+        plan.preprocess(raw, out)
+        torch.cuda.synchronize()
+        assert_parity(out.to_numpy(), oracle.run(s, host), f"nnz {nnz}")
+        ups.append(plan.info()["partition_uploads"])
+    plan.close()
+    assert ups == [1, 1, 1, 2], ups
+
+
+def test_graph_replay_after_partition_evictions(env, kmode):
+    """a captured launch pins its partition slot, so eager calls
+    over more than 8 other batch shapes (evicting every unpinned slot) do not
+    change what the replay reads."""
+    rap, synth, oracle, torch = env
+    w = synth.c2_terabyte(0)
+    plan = rap.Plan(w.spec, device=0)
+    plan.set_kernel(kmode)
+    host = synth.make_batch(w, 2500, seed=31)
+    want = oracle.run(w.spec, host)
+    raw = rap.DeviceBatch(host, "cuda:0")
+    out = rap.DeviceOutput(plan, 2500, raw.sp_nnz, "cuda:0")
+    st = torch.cuda.Stream()
+    with torch.cuda.stream(st):
+        plan.preprocess(raw, out, stream=st)
+    st.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=st):
+        plan.preprocess(raw, out, stream=st)
+    others = []
+    for i in range(10):  # 10 other shapes: every unpinned slot is evicted
+        B = 1000 + 128 * i
+        h = synth.make_batch(w, B, seed=40 + i)
+        r = rap.DeviceBatch(h, "cuda:0")
+        o = rap.DeviceOutput(plan, B, r.sp_nnz, "cuda:0")
+        plan.preprocess(r, o)
+        others.append((h, o))
+    torch.cuda.synchronize()
+    h, o = others[-1]
+    assert_parity(o.to_numpy(), oracle.run(w.spec, h), "eager after evictions")
+    out.values.fill_(-1)
+    out.lengths.fill_(-1)
+    g.replay()
+    torch.cuda.synchronize()
+    assert_parity(out.to_numpy(), want, "replay")
+    plan.close()

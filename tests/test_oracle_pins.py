@@ -395,3 +395,20 @@ def test_c2_workload_invariants(orc):
     assert not np.isnan(r["dense"][:, :6]).any()
     onehot = r["dense"][:, 13:]
     assert np.all(onehot.reshape(B, 2, 16).sum(-1) == 1)
+
+
+def test_spec_goldens_regenerate():
+    """spec_goldens.json is what the committed big-int generator writes, and the
+    generator's H is itself pinned to the published SplitMix64 vectors."""
+    import importlib.util
+    import os
+
+    p = os.path.join(os.path.dirname(__file__), "golden", "make_spec_goldens.py")
+    sp = importlib.util.spec_from_file_location("make_spec_goldens", p)
+    m = importlib.util.module_from_spec(sp)
+    sp.loader.exec_module(m)
+    g = _load("splitmix64_vectors.json")
+    assert m.H(0) == int(g["seed_0_first"], 16)
+    have = _load("spec_goldens.json")
+    want = m.goldens()
+    assert have["sigridhash"] == want["sigridhash"] and have["ngram"] == want["ngram"]
