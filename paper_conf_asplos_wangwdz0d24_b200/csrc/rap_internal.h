@@ -265,17 +265,22 @@ struct RbFeat {
   int32_t pslot[kMaxNgramK];
 };
 
+constexpr int kRbSup = 32;                  // row blocks per super block (two-level lower-block sums)
+constexpr int kRbSupMax = kMaxCtas / kRbSup;  // super blocks per output
 struct RbGeom {
   int32_t n_rb, n_fg, rows_rb, max_fl;  // row blocks, feature groups, rows per block (x32), max outputs per group
   int32_t max_cols, dense_bytes;        // max raw sparse columns one group stages; dense-phase smem bytes
   int32_t n_memo, small;                // memo slots; small = 1: every base fits 31 bits (32-bit scans)
-  int32_t len_cache, pad2;              // 1: the kernel keeps a uint16 length cache per (output, row) in smem
+  int32_t len_cache;                    // 1: the kernel keeps a uint16 length cache per (output, row) in smem
+  int32_t n_dcta;                       // dedicated dense CTAs after the n_rb x n_fg sparse ones (0: dense
+                                        // blocks round robin over every CTA)
   unsigned long long all_cols;          // raw sparse columns the outputs read (bit c: column c < 64)
   const RbFeat* feat;                   // [n_sparse_out], by output index
   const int32_t* perm;                  // [n_sparse_out] processing order (groups are ranges of it)
   unsigned long long* agg;              // [n_sparse_out][n_rb] per-(output, row block) totals
   unsigned long long* sched;            // [0] CTAs done, [2] CTAs whose totals are stored (reset by the last CTA)
   unsigned long long* tot;              // [n_sparse_out] per-output totals (red.add; zeroed by the last CTA)
+  unsigned long long* sup;              // [n_sparse_out][kRbSupMax] totals of 32-row-block super blocks (red.add)
   int32_t fg_off[kRbMaxFg + 1];         // group g = perm[fg_off[g] .. fg_off[g + 1])
 };
 
@@ -327,6 +332,9 @@ struct JitModule;  // compiled kernels (opaque)
 // per source text in the process).  Returns nullptr and fills *log on failure.
 JitModule* jit_build(const JitPlanView& v, bool small, char* log, int log_cap);
 int jit_occupancy(JitModule* m, int smem_bytes, int* ctas_per_sm);
+// Region-0 shared-memory bytes the generated kernel needs beyond the dense
+// tile (the column emitter's memo rows; 0 if none).
+int jit_dense_need(const JitPlanView& v);
 int launch_jit(JitModule* m, const Common& c, const RbGeom& g, const LaunchRaw& raw, int smem_bytes, void* stream);
 double jit_compile_seconds(const JitModule* m);
 #endif

@@ -37,6 +37,11 @@ namespace rapk {
 // Header texts (generated from the csrc/ headers at build time by _build.py).
 #include "rap_jit_embed.inc"
 
+static int env_int(const char* name, int dflt) {
+  const char* e = getenv(name);
+  return (e && *e) ? atoi(e) : dflt;
+}
+
 struct JitModule {
   cudaLibrary_t lib = nullptr;
   cudaKernel_t k = nullptr;
@@ -374,7 +379,7 @@ struct Gen {
       if (is_prov[f]) s += "    int64_t m" + i2s(f) + " = 0;\n    int32_t ml" + i2s(f) + " = 0;\n";
     // first ids of the canonical list outputs, loaded kAhead outputs before
     // their use (the load latency hides under the outputs in between)
-    const int kAhead = 4;
+    const int kAhead = env_int("RAP_JIT_AHEAD", 4);  // (experiment knob)
     const int kSegment = 1 << 30;  // (barriers every few outputs to keep warps together: measured, no gain)
     std::vector<int> canon_q;
     for (int q = 0; q < F; ++q)
@@ -389,7 +394,7 @@ struct Gen {
     };
     // MapId outputs: their first table probe is loaded kProbe outputs ahead,
     // from the prefetched id run through the stages before MapId
-    const int kProbe = 2;
+    const int kProbe = env_int("RAP_JIT_PROBE", 2);  // (experiment knob)
     auto has_map = [&](int q) { return (v.sprogs[v.perm[q]].cn.mask & CB_MAPID) != 0; };
     auto probe = [&](int q) {
       const int f = v.perm[q];
@@ -486,8 +491,8 @@ struct Gen {
           late_q.push_back(q);
           ++n_late;
         } else {
-          s += "      if (!fast && L" + Q + " > 0) rb_emit_ngram(p, s, s.feat[" + Q + "], -1, r, row, L" + Q + ", P" + Q +
-               ", 0);\n    }\n";
+          s += "      if (!fast && L" + Q + " > 0) rb_fallback(p, s, x.slot, " + Fs + ", r, row, L" + Q + ", P" + Q +
+               ");\n    }\n";
         }
       } else if (R.emit == 3) {
         s += "    if (L" + Q + " > 0) rb_fallback(p, s, x.slot, " + Fs + ", r, row, L" + Q + ", P" + Q + ");\n";
@@ -501,8 +506,257 @@ struct Gen {
       const std::string Q = i2s(q), Fs = i2s(v.perm[q]);
       s += "  if (__any_sync(0xffffffffu, (late >> " + i2s(k) + ") & 1u)) {\n" + len_code(q);
       s += "    const long long P" + Q + " = s.wb[" + i2s(q * 8) + " + warp] + rb_warp_excl<kSmall>(L" + Q + ", lane);\n";
-      s += "    if ((late >> " + i2s(k) + ") & 1u) rb_emit_ngram(p, s, s.feat[" + Q + "], -1, r, row, L" + Q + ", P" + Q +
-           ", 0);\n  }\n";
+      s += "    if ((late >> " + i2s(k) + ") & 1u) rb_fallback(p, s, x.slot, " + Fs + ", r, row, L" + Q + ", P" + Q +
+           ");\n  }\n";
+    }
+    s += "    if (ovf) atomicExch(c.err, 1);  // values_capacity understated (sp_nnz): nothing stored past it\n";
+    s += "  }\n";
+    return s;
+  }
+
+  // ---- column emitter (RAP_JIT_EMIT=col; measured slower, kept for the record) ----
+  // Each sparse warp runs a static, cost-balanced list of outputs; for one
+  // output it loops over the chunk's row groups (32 rows each), so a warp
+  // re-executes one short output body (its immediates included) instead of
+  // streaming every output's code once -- the straight-line row emitter's
+  // code (~200 KB for C2) missed the instruction caches (ncu: no_instruction
+  // was the top stall of phase 4).  NGram sources memoised by their provider
+  // outputs go through shared memory: providers run first, one named barrier,
+  // then the NGram outputs.  Ids are loaded two row groups ahead and MapId's
+  // first probe one ahead.  Measured on C2 (B200, 65536 rows): phase 4 took
+  // 49.7 us against the row emitter's 21.3 us -- the row emitter's cross-output
+  // instruction-level parallelism outweighs its instruction-cache misses
+  // (a unit's row groups form one dependent chain per warp).
+  static bool column_mode() {
+    const char* e = getenv("RAP_JIT_EMIT");  // "col": this emitter (experiment knob)
+    return e && strcmp(e, "col") == 0;
+  }
+  int sparse_warps() const { return gen_dense_ok() ? 7 : 8; }
+  int memo_off() const { return gen_dense_ok() ? ((tile_offset() + 32 * pitch() * 4 + 15) & ~15) : 0; }
+  std::vector<int> col_memo;  // output f -> its memo row in column mode (-1: none)
+  int col_memo_slots() {
+    col_memo.assign(F, -1);
+    int n = 0;
+    for (int f = 0; f < F; ++f)
+      if (v.feat[f].emit == 0 && v.feat[f].memo_slot >= 0) col_memo[f] = n++;
+    return n;
+  }
+  // shared-memory bytes of region 0 the column emitter needs (0: no memo)
+  int dense_need() {
+    if (!column_mode()) return 0;
+    const int n = col_memo_slots();
+    return n ? memo_off() + n * kRbChunk * 8 : 0;
+  }
+  double out_cost(int q) const {
+    const int f = v.perm[q];
+    const RbFeat& R = v.feat[f];
+    const Canon& cn = v.sprogs[f].cn;
+    if (R.emit == 0) {
+      double c = 1.0;
+      if (cn.mask & CB_MAPID) c += 0.7;
+      if (cn.mask & CB_BUCKET) c += 0.5;
+      if (R.cap[0] > 1) c += 1.0;
+      return c;
+    }
+    if (R.emit == 3) return 0.6 + 0.5 * R.k + 0.6 * std::max(1, R.k - R.n + 1) * R.n;
+    return 4.0;
+  }
+  // Work units (output q, row groups [g0, g1)) of one phase over nw warps:
+  // each output split into k row-group ranges, k the smallest in {1, 2, 3, 4,
+  // 7} whose longest-processing-time assignment is within 8% of the mean load
+  // (a few NGram outputs over 7 warps need splitting; many outputs do not).
+  struct Unit {
+    int q, g0, g1;
+  };
+  std::vector<std::vector<Unit>> assign(const std::vector<int>& qs, int nw) const {
+    const int nrg = sparse_warps();
+    std::vector<std::vector<Unit>> best;
+    double best_ratio = 1e30;
+    for (int k : {1, 2, 3, 4, 7}) {
+      if (k > nrg) break;
+      std::vector<std::pair<double, Unit>> units;
+      double total = 0;
+      for (int q : qs)
+        for (int i = 0; i < k; ++i) {
+          const int g0 = nrg * i / k, g1 = nrg * (i + 1) / k;
+          const double c = out_cost(q) * (g1 - g0) / nrg + 0.15;  // + the pipeline warm-up of a unit
+          units.push_back({c, Unit{q, g0, g1}});
+          total += c;
+        }
+      std::stable_sort(units.begin(), units.end(), [](const auto& a, const auto& b) { return a.first > b.first; });
+      std::vector<std::vector<Unit>> w(nw);
+      std::vector<double> load(nw, 0.0);
+      for (const auto& u : units) {
+        const int j = (int)(std::min_element(load.begin(), load.end()) - load.begin());
+        w[j].push_back(u.second);
+        load[j] += u.first;
+      }
+      const double ratio = *std::max_element(load.begin(), load.end()) / (total / nw);
+      if (ratio < best_ratio) {
+        best_ratio = ratio;
+        best = w;
+      }
+      if (ratio <= 1.08) break;
+    }
+    for (auto& l : best)  // processing order inside a warp
+      std::sort(l.begin(), l.end(), [](const Unit& a, const Unit& b) { return a.q != b.q ? a.q < b.q : a.g0 < b.g0; });
+    return best;
+  }
+  // the row-group loop of one output over row groups [g0, g1)
+  std::string col_output(int q, int g0, int g1) {
+    const int f = v.perm[q];
+    const RbFeat& R = v.feat[f];
+    const SProg& pg = v.sprogs[f];
+    const std::string Q = i2s(q), Fs = i2s(f);
+    const int nrg = sparse_warps();
+    const bool le1 = max_len(f) <= 1;
+    std::string s = "  {  // output " + Fs + ", row groups " + i2s(g0) + ".." + i2s(g1 - 1) + "\n";
+    const bool canon = R.emit == 0;
+    const bool map = canon && (pg.cn.mask & CB_MAPID);
+    if (canon) {
+      const std::string sl = i2s(slot[R.src[0]]), col = i2s(R.src[0]);
+      s += "    auto ld = [&](int g2) -> int64_t {\n"
+           "      const int r2 = min(g2 * 32 + lane, " + i2s(kRbChunk - 1) + ");\n"
+           "      const RbRow Y = rb_row(s, " + sl + ", r2);\n"
+           "      return __ldg(r2 < nr && Y.valid && Y.b > Y.a ? p.val[" + col + "] + Y.a : c.itab);\n    };\n";
+      s += "    int64_t pfA = ld(" + i2s(g0) + "), pfB = ld(" + i2s(g0 + 1) + ");\n";
+      if (map) {
+        s += "    auto pr = [&](int g2, int64_t id) -> longlong2 {\n"
+             "      const int r2 = min(g2 * 32 + lane, " + i2s(kRbChunk - 1) + ");\n"
+             "      const RbRow Z = rb_row(s, " + sl + ", r2);\n"
+             "      int64_t u = Z.valid ? id : " + lit64(pg.ch.fill) + ";\n";
+        s += stages(pg.cn, pg.cn.mask & CB_CLAMP, "u", "Z.valid", -1, "");
+        s += "      return map_first_probe(c.itab, " + lit64(pg.cn.map_a) + ", " + i2s(pg.cn.map_m) + ", u);\n    };\n";
+        s += "    longlong2 pkA = pr(" + i2s(g0) + ", pfA);\n";
+      }
+    }
+    (void)nrg;
+    s += "#pragma unroll 1\n    for (int rg = " + i2s(g0) + "; rg < " + i2s(g1) + " && rg * 32 < nr; ++rg) {\n"
+         "    const int r = rg * 32 + lane;\n    const bool in = r < nr;\n    const int64_t row = c0 + r;\n";
+    if (canon) {
+      s += "    const int64_t pf" + Q + " = pfA;\n    pfA = pfB;\n    pfB = ld(rg + 2);\n";
+      if (map) s += "    const longlong2 pk" + Q + " = pkA;\n    pkA = pr(rg + 1, pfA);\n";
+    }
+    s += len_code(q);
+    s += "    const long long P" + Q + " = s.wb[" + i2s(q * 8) + " + rg] + " +
+         (le1 ? "rb_ballot_excl(L" + Q + " != 0, lane)" : "rb_warp_excl<kSmall>(L" + Q + ", lane)") + ";\n";
+    s += "    stg_s32_if(in, c.lengths + ((int64_t)" + Fs + " * B + row), L" + Q + ");\n";
+    s += "    stg_s64_if(in, c.offsets + ((int64_t)" + Fs + " * B + row), P" + Q + ");\n";
+    if (f == F - 1) s += "    stg_s64_if(in && row == B - 1, c.offsets + (int64_t)" + i2s(F) + " * B, P" + Q + " + L" + Q + ");\n";
+    s += "    ovf |= P" + Q + " + L" + Q + " > c.values_cap;\n";
+    if (canon) {
+      const Canon& cn = pg.cn;
+      const std::string X = "X" + Q + "_0";
+      const int col = R.src[0];
+      const bool prov = col_memo[f] >= 0;
+      s += "    {\n        int64_t v = " + X + ".valid ? pf" + Q + " : " + lit64(pg.ch.fill) + ";\n";
+      if (prov) s += "        int64_t mv = 0;\n";
+      s += stages(cn, cn.mask, "v", X + ".valid", prov ? memo_point(R, cn) : -1, "mv", map ? "pk" + Q : "");
+      if (prov) s += "        memo[" + i2s(col_memo[f] * kRbChunk) + " + r] = mv;\n";
+      s += "        stg_s64_if(L" + Q + " > 0 && P" + Q + " < c.values_cap, c.values + P" + Q + ", v);\n";
+      if (R.cap[0] > 1) {
+        s += "        for (int32_t j = 1; j < L" + Q + "; ++j) {\n";
+        s += "          int64_t w = __ldg(p.val[" + i2s(col) + "] + " + X + ".a + j);\n";
+        s += stages(cn, cn.mask, "w", "true", -1, "");
+        s += "          rb_store(c, P" + Q + " + j, w);\n        }\n";
+      }
+      s += "    }\n";
+    } else if (R.emit == 3 && col_fast_ok(q)) {
+      const int n = R.n, K = R.k;
+      // the providers' lengths (whether their memo holds an id) and memo words
+      std::vector<int> seen;
+      for (int i = 0; i < K; ++i) {
+        const int qp = R.prov[i];
+        if (std::find(seen.begin(), seen.end(), qp) != seen.end()) continue;
+        seen.push_back(qp);
+        s += len_code(qp);
+        s += "    const int64_t mm" + i2s(qp) + " = memo[" + i2s(col_memo[v.perm[qp]] * kRbChunk) + " + r];\n";
+      }
+      std::string cond;
+      for (int i = 0; i < K; ++i) {
+        const std::string l = "l" + Q + "_" + i2s(i);
+        if (i) cond += " && ";
+        cond += "(" + l + " <= 1 && (" + l + " == 0 || L" + i2s(R.prov[i]) + " >= 1))";
+      }
+      s += "    {\n      const bool fast = " + cond + ";\n      int32_t cnt = 0;\n";
+      for (int j = 0; j < n; ++j) s += "      uint64_t w" + i2s(j) + " = 0;\n";
+      for (int i = 0; i < K; ++i) {
+        const std::string pr = "pr" + i2s(i);
+        s += "      const bool " + pr + " = l" + Q + "_" + i2s(i) + " != 0;\n";
+        for (int j = 0; j + 1 < n; ++j)
+          s += "      w" + i2s(j) + " = " + pr + " ? w" + i2s(j + 1) + " : w" + i2s(j) + ";\n";
+        s += "      w" + i2s(n - 1) + " = " + pr + " ? (uint64_t)mm" + i2s(R.prov[i]) + " : w" + i2s(n - 1) + ";\n";
+        s += "      cnt += " + pr + ";\n";
+        if (i + 1 >= n) {
+          s += "      {\n        uint64_t h = " + litu64(pg.ng.hsalt) + ";\n";
+          for (int j = 0; j < n; ++j) s += "        h = splitmix_H(h ^ w" + i2s(j) + ");\n";
+          s += "        int64_t v = (int64_t)reduce_M(h, " + lit64(pg.ng.M) + ");\n";
+          s += stages(pg.cn, pg.cn.mask, "v", "true", -1, "");
+          s += "        const long long at = P" + Q + " + (cnt - " + i2s(n) + ");\n";
+          s += "        stg_s64_if(fast && " + pr + " && cnt >= " + i2s(n) + " && cnt - " + i2s(n) + " < L" + Q +
+               " && at < c.values_cap, c.values + at, v);\n      }\n";
+        }
+      }
+      s += "      const bool late = !fast && L" + Q + " > 0;\n"
+           "      if (__any_sync(0xffffffffu, late) && late) rb_fallback(p, s, x.slot, " + Fs + ", r, row, L" + Q +
+           ", P" + Q + ");\n    }\n";
+    } else {
+      s += "    if (L" + Q + " > 0) rb_fallback(p, s, x.slot, " + Fs + ", r, row, L" + Q + ", P" + Q + ");\n";
+    }
+    s += "    }\n  }\n";
+    return s;
+  }
+  // NGram q on the memo path: canonical post stages, every source a raw list
+  // whose provider memoises it (column mode: the provider runs in phase A)
+  bool col_fast_ok(int q) {
+    const int f = v.perm[q];
+    const RbFeat& R = v.feat[f];
+    const SProg& pg = v.sprogs[f];
+    if (!pg.cn.ok || R.n < 1 || R.n > kMaxNgramK) return false;
+    for (int i = 0; i < R.k; ++i) {
+      if (R.src[i] < 0 || R.prov[i] < 0) return false;
+      if (col_memo[v.perm[R.prov[i]]] < 0) return false;
+    }
+    return true;
+  }
+  std::string col_emit_fn() {
+    col_memo_slots();
+    const int nw = sparse_warps();
+    std::vector<int> phase_a, phase_b;
+    for (int q = 0; q < F; ++q) {
+      const int f = v.perm[q];
+      (col_memo[f] >= 0 ? phase_a : phase_b).push_back(q);
+    }
+    bool any_consumer = false;
+    for (int q : phase_b) any_consumer |= v.feat[v.perm[q]].emit == 3 && col_fast_ok(q);
+    if (!any_consumer) {  // no memo reads: one phase
+      phase_a.insert(phase_a.end(), phase_b.begin(), phase_b.end());
+      phase_b.clear();
+    }
+    std::string s;
+    s += "  template <bool kSmall, class P>\n"
+         "  static __device__ __forceinline__ void emit(const P& p, const RbSmem& s, const RbCtx& x, int64_t c0, "
+         "int nr) {\n"
+         "    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;\n"
+         "    const Common& c = p.c;\n"
+         "    const int64_t B = x.B;\n"
+         "    long long* memo = reinterpret_cast<long long*>(s.dense + " + i2s(memo_off()) + ");\n"
+         "    (void)memo;\n"
+         "    bool ovf = false;\n";
+    for (int ph = 0; ph < 2; ++ph) {
+      const std::vector<int>& qs = ph == 0 ? phase_a : phase_b;
+      if (qs.empty()) continue;
+      if (ph == 1) s += std::string("    ") + (gen_dense_ok() ? "rb_sync<true>();" : "rb_sync<false>();") +
+                        "  // providers' memo words visible\n";
+      const auto asg = assign(qs, nw);
+      s += "    switch (warp) {\n";
+      for (int w = 0; w < nw; ++w) {
+        if (asg[w].empty()) continue;
+        s += "    case " + i2s(w) + ":\n";
+        for (const Unit& u : asg[w]) s += col_output(u.q, u.g0, u.g1);
+        s += "    break;\n";
+      }
+      s += "    default: break;\n    }\n";
     }
     s += "    if (ovf) atomicExch(c.err, 1);  // values_capacity understated (sp_nnz): nothing stored past it\n";
     s += "  }\n";
@@ -541,7 +795,7 @@ struct Gen {
     body += "  }\n";
     body += dense;
     body += lengths_fn();
-    body += emit_fn();
+    body += column_mode() ? col_emit_fn() : emit_fn();
     body += "};\n\n}  // namespace rapk\n\n";
     s += globals + sample_globals + "\n" + body;
     // one variant per module: 32-bit scans (every offset < 2^31) or 64-bit
@@ -601,6 +855,8 @@ bool nvrtc_cubin(const std::string& src, std::vector<char>* cubin, std::string* 
 }  // namespace
 
 std::string jit_generate(const JitPlanView& v) { return Gen(v).source(true); }
+
+int jit_dense_need(const JitPlanView& v) { return Gen(v).dense_need(); }
 
 bool jit_compile_only(const std::string& src, std::string* log) {
   std::vector<char> cubin;
@@ -678,7 +934,7 @@ int launch_jit(JitModule* m, const Common& c, const RbGeom& g, const LaunchRaw& 
     p.svalid[i] = raw.svalid ? raw.svalid[i] : nullptr;
   }
   cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3((unsigned)(g.n_rb * g.n_fg));
+  cfg.gridDim = dim3((unsigned)(g.n_rb * g.n_fg + g.n_dcta));
   cfg.blockDim = dim3(kRbChunk);
   cfg.dynamicSmemBytes = smem_bytes;
   cfg.stream = reinterpret_cast<cudaStream_t>(stream);

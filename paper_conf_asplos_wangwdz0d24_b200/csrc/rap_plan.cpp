@@ -110,6 +110,7 @@ struct rap_plan {
   // row-block kernel (rap_rows.cu)
   int kernel_mode = RAP_KERNEL_AUTO, kernel_last = 0;
   int rb_fits = 0, rb_ctas_per_sm = 0, rb_smem = 0, rb_max_fl = 0, rb_max_cols = 0, rb_n_memo = 0;
+  int rb_last_grid = 0;  // CTAs of the last row-block / generated launch
   int rb_dense_bytes = 0;
   unsigned long long rb_all_cols = 0;  // raw sparse columns the sparse outputs read
   std::vector<RbFeat> rbfeat;     // by output index
@@ -1106,7 +1107,8 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
   if (e == cudaSuccess) e = cudaMalloc(&P->d_part, kPartSlots * kPartLen * sizeof(int64_t));
   if (e == cudaSuccess) e = cudaMallocHost(&P->h_part, kPartSlots * kPartLen * sizeof(int64_t));
   if (e == cudaSuccess && P->rb_fits && !P->souts.empty()) {
-    const size_t n = (P->souts.size() + 1) * (size_t)kMaxCtas + P->souts.size();  // agg [F][n_rb] + tot [F]
+    // agg [F][n_rb] + tot [F] + sup [F][kRbSupMax]
+    const size_t n = (P->souts.size() + 1) * (size_t)kMaxCtas + P->souts.size() * (size_t)(1 + kRbSupMax);
     e = cudaMalloc(&P->d_agg_rb, n * sizeof(unsigned long long));
     if (e == cudaSuccess) e = cudaMemset(P->d_agg_rb, 0, n * sizeof(unsigned long long));
   }
@@ -1136,6 +1138,7 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
     // the dense warp's 32-row tile after the base-phase totals (rap_jit.cpp tile_offset)
     const int tile = ((2 * ((int)P->souts.size() + 1) * 8 + 15) & ~15) + 32 * (P->d_out | 1) * 4;
     P->jit_dense_bytes = (P->d_out > 0 && tile <= P->rb_dense_bytes) ? tile : P->rb_dense_bytes;
+    P->jit_dense_bytes = std::max(P->jit_dense_bytes, jit_dense_need(jit_view(P)));  // + the emitter's memo rows
     P->jit_smem = rows_smem_bytes(P->jit_dense_bytes, P->rb_max_fl, P->rb_max_cols, 0, (int)P->souts.size(), 0);
     if (P->rb_smem > 227 * 1024) P->rb_fits = 0;
   }
@@ -1250,7 +1253,7 @@ rap_status rap_plan_info_get(const rap_plan* P, rap_plan_info* info) {
   info->jit_state = P->jit_state;
   info->jit_ctas_per_sm = P->jit_ctas_per_sm;
   info->jit_compile_seconds = P->jit_s;
-  if (P->kernel_last == RAP_KERNEL_ROWS) info->grid = P->rb_last_n_rb * P->rb_last_n_fg;
+  if (P->kernel_last == RAP_KERNEL_ROWS || P->kernel_last == RAP_KERNEL_JIT) info->grid = P->rb_last_grid;
   return RAP_OK;
 }
 
@@ -1555,9 +1558,18 @@ static bool use_rows(const rap_plan* P, int64_t B, const int64_t* nnz) {
 // order, balanced by the cost model, <= kRbMaxFL outputs each), at most the
 // budget's CTA slots.  Large batches: one feature group, one row block per
 // slot.  Small batches: 256-row blocks, the slots left over split the outputs.
-static void rows_geometry(const rap_plan* P, int64_t B, const int64_t* nnz, int ctas_per_sm, RbGeom* g) {
+// n_dense_tiles > 0 (the interpreted form): when the dense blocks are few
+// (<= a quarter of the slots) each gets a dedicated CTA, so small batches run
+// the dense outputs beside the sparse phases rather than after them.
+static void rows_geometry(const rap_plan* P, int64_t B, const int64_t* nnz, int ctas_per_sm, RbGeom* g,
+                          int64_t n_dense_tiles = 0) {
   const int F = (int)P->souts.size();
-  const int64_t slots = std::max<int64_t>(1, std::min<int64_t>((int64_t)P->budget * ctas_per_sm, kMaxCtas));
+  int64_t slots = std::max<int64_t>(1, std::min<int64_t>((int64_t)P->budget * ctas_per_sm, kMaxCtas));
+  g->n_dcta = 0;
+  if (n_dense_tiles > 0 && n_dense_tiles <= slots / 4) {
+    g->n_dcta = (int)n_dense_tiles;
+    slots -= n_dense_tiles;
+  }
   const int fg_min = (F + kRbMaxFL - 1) / kRbMaxFL;
   const int64_t nb256 = (B + kRbChunk - 1) / kRbChunk;
   int64_t n_rb, n_fg;
@@ -1671,8 +1683,8 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
     const bool jit = want_jit && jit_ready(P, small);
     const int iv = small ? 1 : 0;
     rows_geometry(P, B, raw->sp_nnz, jit ? P->jit_occ[iv] : P->rb_ctas_per_sm, &g);
-    if (jit && !(g.n_fg == 1 && drow0 == 0 && drows == B))  // the generated form does not apply: interpreted geometry
-      rows_geometry(P, B, raw->sp_nnz, P->rb_ctas_per_sm, &g);
+    if (!jit || !(g.n_fg == 1 && drow0 == 0 && drows == B))  // interpreted form: its geometry, dense CTAs
+      rows_geometry(P, B, raw->sp_nnz, P->rb_ctas_per_sm, &g, n_dense);
     g.max_fl = P->rb_max_fl;
     g.max_cols = P->rb_max_cols;
     g.dense_bytes = P->rb_dense_bytes;
@@ -1683,11 +1695,13 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
     g.perm = reinterpret_cast<const int32_t*>(P->blob + P->off_perm);
     g.agg = P->d_agg_rb;
     g.tot = P->d_agg_rb + (P->souts.size() + 1) * (size_t)kMaxCtas;
+    g.sup = g.tot + P->souts.size();
     g.sched = P->d_sched + 4;
     // the generated policy covers one group of every output, over the batch's
     // own rows (a sharded plan's dense shard runs the interpreted form)
     const bool gen = jit && g.n_fg == 1 && drow0 == 0 && drows == B;
     if (gen) {
+      g.n_dcta = 0;  // the generated form evaluates the dense outputs itself
       g.len_cache = 0;
       g.n_memo = 0;
       g.dense_bytes = P->jit_dense_bytes;
@@ -1699,6 +1713,7 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
     P->kernel_last = gen ? RAP_KERNEL_JIT : RAP_KERNEL_ROWS;
     P->rb_last_n_rb = g.n_rb;
     P->rb_last_n_fg = g.n_fg;
+    P->rb_last_grid = g.n_rb * g.n_fg + g.n_dcta;
     P->rb_last_rows = g.rows_rb;
     P->n_launches += 1;
     P->last_n_desc = (int64_t)g.n_rb * g.n_fg;

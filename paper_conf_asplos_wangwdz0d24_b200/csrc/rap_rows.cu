@@ -67,7 +67,7 @@ static int launch_rows_t(const Common& c, const RbGeom& g, const LaunchRaw& raw,
     p.svalid[i] = raw.svalid ? raw.svalid[i] : nullptr;
   }
   cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3((unsigned)(g.n_rb * g.n_fg));
+  cfg.gridDim = dim3((unsigned)(g.n_rb * g.n_fg + g.n_dcta));
   cfg.blockDim = dim3(kRbChunk);
   cfg.dynamicSmemBytes = smem;
   cfg.stream = st;

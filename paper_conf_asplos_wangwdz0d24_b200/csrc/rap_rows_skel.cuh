@@ -358,14 +358,18 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
   x.F = c.n_sparse_out;
   const RbSmem s = rb_carve(smem, g, x.F);
   const int n_rb = g.n_rb;
-  x.grp = (int)blockIdx.x / n_rb;
-  x.rb = (int)blockIdx.x - x.grp * n_rb;
-  x.pb = g.fg_off[x.grp];
-  x.pe = g.fg_off[x.grp + 1];
+  // CTAs [n_rb * n_fg, + n_dcta) evaluate only dense blocks (small batches:
+  // the dense work runs beside the sparse phases instead of after them)
+  const int n_sc = n_rb * g.n_fg;
+  const bool dcta = (int)blockIdx.x >= n_sc;
+  x.grp = dcta ? 0 : (int)blockIdx.x / n_rb;
+  x.rb = dcta ? 0 : (int)blockIdx.x - x.grp * n_rb;
+  x.pb = dcta ? 0 : g.fg_off[x.grp];
+  x.pe = dcta ? 0 : g.fg_off[x.grp + 1];
   x.FL = x.pe - x.pb;
   x.B = c.n_rows;
   x.R0 = (int64_t)x.rb * g.rows_rb;
-  x.R1 = min(x.B, x.R0 + (int64_t)g.rows_rb);
+  x.R1 = dcta ? x.R0 : min(x.B, x.R0 + (int64_t)g.rows_rb);
   x.slot = s_slot;
   x.fidx = s_fidx;
   const int FL = x.FL, rb = x.rb;
@@ -446,7 +450,9 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
     const int f = s_fidx[tid];
     g.agg[(int64_t)f * n_rb + rb] = (unsigned long long)tot;  // feature-major: row blocks of f contiguous
     atomicAdd(g.tot + f, (unsigned long long)tot);           // red.add: the output's total over all blocks
+    atomicAdd(g.sup + (int64_t)f * kRbSupMax + rb / kRbSup, (unsigned long long)tot);  // and its super block's
   }
+  trace_stamp(c, 13);
   rb_sync<kDW>();
   if (tid == 0) {
     __threadfence();  // release: the block's totals before the announcement
@@ -463,11 +469,13 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
     if (Pol::kGenDense && all && c.dense_row0 == 0 && c.n_dense_rows == c.n_rows && c.n_groups > 0) {
       Pol::dense(p, s, x);
     } else {
-      for (int64_t d = blockIdx.x; d < c.n_dense_tiles; d += gridDim.x) {
+      const int64_t d0 = g.n_dcta ? (int64_t)blockIdx.x - n_sc : (int64_t)blockIdx.x;
+      const int64_t dstep = g.n_dcta ? (int64_t)g.n_dcta : (int64_t)gridDim.x;
+      for (int64_t d = d0; d >= 0 && d < c.n_dense_tiles; d += dstep) {
         const uint32_t gi = (uint32_t)d % (uint32_t)c.n_groups;
         dense_block(p, (int)gi, (int64_t)((uint32_t)d / (uint32_t)c.n_groups), 0, cs);
         __syncthreads();
-        if (d == (int64_t)blockIdx.x) trace_stamp(c, 9);
+        if (d == d0) trace_stamp(c, 9);
       }
     }
   }
@@ -485,40 +493,51 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
     }
     rb_sync<kDW>();
     trace_stamp(c, 3);
-    // T[f] = the output's total (red.add into g.tot), L[f] = its words of the
-    // row blocks below mine (coalesced; warp w reduces outputs w, w + 8, ...,
-    // two at a time so their loads are in flight together)
+    // T[f] = the output's total (red.add into g.tot), L[f] = its ids in the
+    // row blocks below mine: the super blocks below mine (32 row blocks each,
+    // red.add totals) plus the row blocks of my super block below mine -- one
+    // coalesced load per lane for each, whatever n_rb (warp w reduces
+    // outputs w, w + kWS, ..., four at a time so their loads are in flight together)
     const int fmax = s_fmax;
     long long* sT = reinterpret_cast<long long*>(s.dense);  // [fmax + 1]
     long long* sL = sT + (fmax + 1);                          // [fmax + 1]
     for (int f = tid; f <= fmax; f += kTS) sT[f] = (long long)__ldcg(g.tot + f);
-    for (int f = warp; f <= fmax; f += 2 * kWS) {
-      const int f2 = f + kWS;
-      const unsigned long long* ra = g.agg + (int64_t)f * n_rb;
-      const unsigned long long* rb2 = g.agg + (int64_t)min(f2, fmax) * n_rb;
-      long long la = 0, lb = 0;
-#pragma unroll 4
-      for (int j = lane; j < rb; j += 32) {
-        la += (long long)__ldcg(ra + j);
-        lb += (long long)__ldcg(rb2 + j);
-      }
-      la = rb_warp_sum<kSmall>(la);
-      lb = rb_warp_sum<kSmall>(lb);
-      if (lane == 0) {
-        sL[f] = la;
-        if (f2 <= fmax) sL[f2] = lb;
+    {
+      const int nsb = rb / kRbSup, rb0 = nsb * kRbSup;
+      for (int f0 = warp; f0 <= fmax; f0 += 4 * kWS) {
+        long long v[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const int f = min(f0 + u * kWS, fmax);
+          long long a = 0;
+          if (lane < nsb) a = (long long)__ldcg(g.sup + (int64_t)f * kRbSupMax + lane);
+          if (rb0 + lane < rb) a += (long long)__ldcg(g.agg + (int64_t)f * n_rb + rb0 + lane);
+          v[u] = a;
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const long long t = rb_warp_sum<kSmall>(v[u]);
+          if (lane == 0 && f0 + u * kWS <= fmax) sL[f0 + u * kWS] = t;
+        }
       }
     }
     trace_stamp(c, 10);
     rb_sync<kDW>();
     trace_stamp(c, 11);
     trace_stamp(c, 12);
-    if (tid == 0) {  // exclusive prefix over outputs in feature-major order
+    if (warp == 0) {  // exclusive prefix over outputs in feature-major order (warp scan, 32 at a time)
       long long P = chain0;
-      for (int f = 0; f <= fmax; ++f) {
-        const long long t = sT[f];
-        sT[f] = P;
-        P += t;
+      for (int f0 = 0; f0 <= fmax; f0 += 32) {
+        const int f = f0 + lane;
+        const long long t = f <= fmax ? sT[f] : 0ll;
+        long long x = t;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+          const long long y = __shfl_up_sync(0xffffffffu, x, d);
+          if (lane >= d) x += y;
+        }
+        if (f <= fmax) sT[f] = P + x - t;
+        P += __shfl_sync(0xffffffffu, x, 31);
       }
     }
     rb_sync<kDW>();
@@ -566,6 +585,8 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
   if (s_last) {
     __threadfence();
     for (int f = tid; f < x.F; f += kRbChunk) g.tot[f] = 0ull;
+    const int nsb_all = (n_rb + kRbSup - 1) / kRbSup;
+    for (int i = tid; i < x.F * nsb_all; i += kRbChunk) g.sup[(int64_t)(i / nsb_all) * kRbSupMax + i % nsb_all] = 0ull;
     if (tid == 0) {
       g.sched[0] = 0ull;
       g.sched[2] = 0ull;

@@ -2,7 +2,8 @@
 """Per-CTA phase timing of one row-block launch (rap_debug_trace; dev tool).
 
 Stamps (%globaltimer, ns) of rap_rows.cu: 0 start, 1 totals published,
-2 dense blocks done, 3 all words seen, 4 bases reduced, 5 ids written."""
+2 dense blocks done, 3 all words seen, 4 bases reduced, 5 ids written;
+6-13 finer points of the row-block skeleton (rap_rows_skel.cuh)."""
 import os
 import sys
 
@@ -45,9 +46,9 @@ def main():
               f"(abs end median {np.median(rel[:, k]):7.2f} max {rel[:, k].max():7.2f})")
     print(f"  CTA start: p50 {np.percentile(rel[:, 0], 50):.2f} p90 {np.percentile(rel[:, 0], 90):.2f} "
           f"max {rel[:, 0].max():.2f} us")
-    ex = (tr[:, 6:13] - t0) / 1e3
+    ex = (tr[:, 6:14] - t0) / 1e3
     for k, nm in enumerate(["slots ready", "setup done", "chunk0 staged", "first dense block", "base loads+redux",
-                            "base sync", "base sums"]):
+                            "base sync", "base sums", "totals stored"]):
         v = ex[:, k]
         v = v[v > -1e6]
         if len(v):

@@ -275,3 +275,26 @@ def test_graph_replay_after_partition_evictions(env, kmode):
     torch.cuda.synchronize()
     assert_parity(out.to_numpy(), want, "replay")
     plan.close()
+
+
+@pytest.mark.parametrize("emitter", ["row", "col"])
+def test_ngram_memo_providers_with_multi_id_rows(env, emitter, monkeypatch):
+    """NGram outputs whose sources are memoised by single-id provider outputs
+    (the generated kernel's register/shared memo path), over sources where
+    some rows hold 2-3 ids: those rows leave the memo path for the generic
+    NGram code (rb_fallback), in both generated emitters."""
+    monkeypatch.setenv("RAP_JIT_EMIT", emitter)
+    rng = np.random.default_rng(77)
+    B = 1800
+    sp = [sparse_from_lists(_lists(rng, B, 0, 10**6, max_len=1, p_null=0.1)) for _ in range(3)]
+    # column 3: mostly single ids, a few rows with 2-3
+    rows = _lists(rng, B, 0, 10**6, max_len=1, p_null=0.1)
+    for i in range(0, B, 37):
+        rows[i] = [int(v) for v in rng.integers(0, 10**6, 2 + i % 2)]
+    sp.append(sparse_from_lists(rows))
+    nodes = [node("sigridhash", [("s", i)], salt=20 + i, max_value=10**6 + i) for i in range(4)]
+    nodes.append(node("ngram", [("s", 0), ("s", 1), ("s", 2)], n=3, salt=4, max_value=10**7))
+    nodes.append(node("ngram", [("s", 1), ("s", 3), ("s", 2)], n=2, salt=5, max_value=2**40))
+    nodes.append(node("ngram", [("s", 3), ("s", 0)], n=1, salt=6, max_value=999))
+    s = spec(0, 4, nodes, list(range(7)))
+    run_check(env, 3, s, batch(B, sparse=sp), ctx=emitter)
