@@ -54,6 +54,8 @@ def parse():
     ap.add_argument("--imbalance-tol", type=float, default=0.10, help="N>1: residual move threshold")
     ap.add_argument("--no-c4", action="store_true", help="skip the config-4 (multi-hot) sub-measurement")
     ap.add_argument("--c4-batch", type=int, default=16384, help="rows of the config-4 sub-measurement")
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                    help="N>1: gloo = host-staged exchange (ranks sharing one GPU: tests)")
     return ap.parse_args()
 
 
@@ -568,29 +570,37 @@ def run_sharded(args):
     import torch.distributed as tdist
 
     rank, world, local = dist_env()
+    local = local % max(torch.cuda.device_count(), 1)  # gloo test runs: several ranks may share a GPU
     torch.cuda.set_device(local)
-    tdist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    if args.dist_backend == "nccl":
+        tdist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    else:
+        tdist.init_process_group("gloo")
     dev = torch.device("cuda", local)
     from paper_conf_asplos_wangwdz0d24_b200 import dist, rap, synth
+
+    exchange = None if args.dist_backend == "nccl" else dist.gloo_exchange
 
     wname, B = WORKLOADS[args.workload]
     B = args.batch or B
     w = workload(args.workload)
-    host = synth.make_batch(w, B, seed=1000)  # the same global batch on every rank
-    raw0 = rap.DeviceBatch(host, dev)
-    pl = dist.plan_placement(w.spec, B, raw0.sp_nnz, world, args.placement, args.imbalance_tol, device=local)
-    sp = dist.ShardedPreprocessor(w.spec, pl, rank, world, B, raw0.sp_nnz, device=local, sm_budget=args.budget)
-    props = torch.cuda.get_device_properties(dev)
-    l2 = getattr(props, "L2_cache_size", 126 * 2**20)
+    host = synth.make_batch(w, B, seed=1000)  # the global batch (each rank uploads its own part of it)
+    sp_nnz = np.array([int(o[-1]) - int(o[0]) for o in host["sp_off"]], dtype=np.int64)
+    comm = calibrate_comm(w.spec, host, B, dev, tdist)
+    pl = dist.plan_placement(w.spec, B, sp_nnz, world, args.placement, args.imbalance_tol, device=local, comm=comm)
+    sp = dist.ShardedPreprocessor(w.spec, pl, rank, world, B, sp_nnz, device=local, sm_budget=args.budget)
+    cols = sp.sparse_columns()
     nsets = 1 if args.profile else 4
-    sets = [(raw0, sp.new_output())]
-    for i in range(1, nsets):
-        r = rap.DeviceBatch(synth.make_batch(w, B, seed=1000 + 97 * i), dev)
+    sets = []
+    for i in range(nsets):
+        h = host if i == 0 else synth.make_batch(w, B, seed=1000 + 97 * i)
+        r = rap.DeviceBatch(h, dev, sparse_cols=cols, dense_rows=(sp.row0, sp.dense_rows))
         sets.append((r, sp.new_output()))
+    upload = sets[0][0].uploaded_bytes()
     stream = torch.cuda.current_stream(dev)
     for i in range(args.warmup):
         r, o = sets[i % nsets]
-        sp.preprocess(r, o, stream)
+        sp.preprocess(r, o, stream, exchange=exchange)
     torch.cuda.synchronize()
     tdist.barrier()
     torch.cuda.synchronize()
@@ -601,14 +611,12 @@ def run_sharded(args):
         t0.record(stream)
         for i in range(K):
             r, o = sets[i % nsets]
-            sp.preprocess(r, o, stream)
+            sp.preprocess(r, o, stream, exchange=exchange)
         t1.record(stream)
         t1.synchronize()
     torch.cuda.synchronize()
     tdist.barrier()
-    t = torch.tensor([t0.elapsed_time(t1)], device=dev)
-    tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
-    total_ms = float(t[0])
+    total_ms = allreduce_max(t0.elapsed_time(t1), dev, tdist)
     # my share of the algorithmic bytes: owned tables over the full batch + my dense shard
     o = sets[(K - 1) % nsets][1]
     offs = o.offsets
@@ -617,12 +625,12 @@ def run_sharded(args):
     d_out = sp.d_out
     my_bytes = (4 * sp.dense_rows * d_out + len(sp.features) * B * 20 + 8 * n_vals
                 + (13 * 4.125 * sp.dense_rows if d_out else 0))
-    bt = torch.tensor([my_bytes], device=dev, dtype=torch.float64)
-    tdist.all_reduce(bt, op=tdist.ReduceOp.MAX)
+    bt = [allreduce_max(my_bytes, dev, tdist)]
     peak, peak_kind = measured_peaks()
     ms = total_ms / K
     achieved = float(bt[0]) / (ms / 1e3) / 1e9
     clocks = sampler.summary() if sampler else None
+    c4 = None if (args.no_c4 or args.profile) else c4_sharded_point(args, rank, world, dev, tdist, exchange)
     if rank == 0:
         res = pl.residual
         line = {"metric": METRIC, "value": B / (ms / 1e3), "unit": UNIT, "n_gpus": world, "steps": K,
@@ -631,16 +639,94 @@ def run_sharded(args):
                 "config": {"workload": wname + "_sharded_c3", "batch": B, "parallelism": f"table-wise x{world}",
                            "placement": args.placement, "loads": [round(x) for x in pl.loads],
                            "residual": None if res is None else res.__dict__,
+                           "comm_model": comm.__dict__,
+                           "rank0_upload_bytes": upload, "rank0_sparse_columns": len(cols),
                            "l2_policy": f"rotate {nsets} input/output sets"},
                 "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                              "frac": achieved / peak, "traffic": None, "peak_source": peak_kind,
                              "note": "busiest rank's algorithmic bytes / step time"},
                 "cpu_baseline": None, "e2e": None, "clocks": clocks,
-                "gpu_launches": K * (1 + (0 if res is None else 2))}
+                "gpu_launches": K * (1 + (0 if res is None else 2)), "c4": c4}
         print(json.dumps(line), flush=True)
     sp.close()
     tdist.destroy_process_group()
     return 0
+
+
+def allreduce_max(x: float, dev, tdist) -> float:
+    """Max over ranks of a host scalar (a CUDA tensor over NCCL, a CPU one over gloo)."""
+    import torch
+
+    on_gpu = tdist.get_backend() == "nccl"
+    t = torch.tensor([float(x)], dtype=torch.float64, device=dev if on_gpu else "cpu")
+    tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
+    return float(t[0])
+
+
+def calibrate_comm(spec, host, B, dev, tdist):
+    """rap_comm_model's time scale on this GPU: rank 0 times the full plan on
+    the batch and divides by its predicted cost (broadcast, so every rank
+    computes the same placement)."""
+    import torch
+
+    from paper_conf_asplos_wangwdz0d24_b200 import dist, rap
+
+    t = torch.zeros(1, dtype=torch.float64, device=dev if tdist.get_backend() == "nccl" else "cpu")
+    if tdist.get_rank() == 0:
+        plan = rap.Plan(spec, device=dev.index)
+        raw = rap.DeviceBatch(host, dev)
+        out = rap.DeviceOutput(plan, B, raw.sp_nnz, dev)
+        for _ in range(3):
+            plan.preprocess(raw, out)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for _ in range(10):
+            plan.preprocess(raw, out)
+        e1.record()
+        e1.synchronize()
+        us = e0.elapsed_time(e1) / 10 * 1e3
+        t[0] = us / max(float(sum(plan.output_costs(B, raw.sp_nnz))), 1e-9)
+        plan.close()
+        del raw, out
+    tdist.broadcast(t, 0)
+    return dist.CommModel(us_per_unit=float(t[0]))
+
+
+def c4_sharded_point(args, rank, world, dev, tdist, exchange=None):
+    """Config 4 table-wise over the ranks (512 tables, balanced, no residual):
+    each rank uploads and preprocesses its own tables over the global batch;
+    the step time is the max over ranks."""
+    import torch
+
+    from paper_conf_asplos_wangwdz0d24_b200 import dist, rap, synth
+
+    w = synth.c4_multihot(0)
+    B = args.c4_batch
+    host = synth.make_batch(w, B, seed=700)
+    sp_nnz = np.array([int(o[-1]) - int(o[0]) for o in host["sp_off"]], dtype=np.int64)
+    pl = dist.plan_placement(w.spec, B, sp_nnz, world, "balanced", None, device=dev.index)
+    sp = dist.ShardedPreprocessor(w.spec, pl, rank, world, B, sp_nnz, device=dev.index)
+    raw = rap.DeviceBatch(host, dev, sparse_cols=sp.sparse_columns())
+    out = sp.new_output()
+    stream = torch.cuda.current_stream(dev)
+    for _ in range(3):
+        sp.preprocess(raw, out, stream, exchange=exchange)
+    torch.cuda.synchronize()
+    tdist.barrier()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    steps = 10
+    e0.record(stream)
+    for _ in range(steps):
+        sp.preprocess(raw, out, stream, exchange=exchange)
+    e1.record(stream)
+    e1.synchronize()
+    ms = allreduce_max(e0.elapsed_time(e1) / steps, dev, tdist)
+    sp.close()
+    del raw, out
+    torch.cuda.empty_cache()
+    return {"workload": "multihot_c4_sharded", "batch": B, "tables_per_rank": len(sp.features),
+            "ms_per_step": ms, "value": B / (ms / 1e3), "unit": UNIT, "scaling": "strong",
+            "note": "table-wise over the ranks, global batch fixed; max over ranks"}
 
 
 class _Null:

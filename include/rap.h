@@ -329,6 +329,30 @@ rap_status rap_place(const double* cost, const int32_t* colocate, int32_t n, int
                      int64_t n_rows, double imbalance_tol, int32_t* owner_out, double* load_out,
                      rap_residual* residual);
 
+/* Communication model of a residual move (§7.2: move
+ * only when the balance gain beats the added communication). */
+typedef struct {
+  double us_per_unit;      /* microseconds per cost unit (a measured kernel time / its predicted cost) */
+  double link_gbs;         /* owner <-> helper point-to-point bandwidth, GB/s (NVLink 5 / NVSwitch) */
+  double link_latency_us;  /* fixed cost of one exchange (send/recv launch and synchronisation) */
+  const double* row_bytes; /* HOST double[n]: bytes one row of output j moves (its raw input row to
+                              the helper plus its output row back to the owner) */
+} rap_comm_model;
+
+/* rap_place with a costed residual move: with h the most and l the least
+ * loaded rank (loads L_h > L_l, cost units), f h's costliest output (p cost
+ * units per row) and t(m) = (link_latency_us + m * row_bytes[f] /
+ * (1e3 * link_gbs)) / us_per_unit the exchange of m rows, the helper finishes
+ * the piece at L_l + m p and the owner holds its KJT at
+ * max(L_h - m p, L_l + m p + t(m)).  m balances the two
+ * (m = (L_h - L_l - t(0)) / (2 p + t(1) - t(0))), rounded down to whole
+ * 128-row tiles; the move is made only if that finish time is below L_h
+ * (a gain after communication), whatever imbalance_tol.  comm NULL:
+ * rap_place.  load_out: compute loads after the move. */
+rap_status rap_place_comm(const double* cost, const int32_t* colocate, int32_t n, int32_t world, int32_t mode,
+                          int64_t n_rows, const rap_comm_model* comm, int32_t* owner_out, double* load_out,
+                          rap_residual* residual);
+
 /* A sharded plan: the graph restricted to its dense outputs (evaluated over
  * this rank's batch shard, rap_shard_rows) and the sparse outputs j with
  * sparse_owner[j] == rank (j counts the graph's sparse outputs in order),

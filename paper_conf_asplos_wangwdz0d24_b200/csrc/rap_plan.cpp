@@ -1028,15 +1028,24 @@ static rap_status plan_lower(const rap_graph* graph, const rap_op_param* params,
     const int rows = std::min(kDenseTileBytes / ((max_w | 1) * 4), kDenseInBytes / (max_cols * 4));
     P->rows_dense = std::max(32, std::min(256, rows / 32 * 32));
   }
-  // used raw columns (for the byte model)
+  // raw columns the plan's outputs read (nodes reachable from them): the byte
+  // model, and the columns a batch must supply (a sharded rank's plan reads
+  // only its own tables' columns; the others may be NULL)
   {
-    std::vector<char> ud(graph->n_dense_in, 0), us(graph->n_sparse_in, 0);
-    for (int i = 0; i < graph->n_nodes; ++i)
+    std::vector<char> ud(graph->n_dense_in, 0), us(graph->n_sparse_in, 0), seen(graph->n_nodes, 0);
+    std::vector<int32_t> stack(graph->output_nodes, graph->output_nodes + graph->n_outputs);
+    while (!stack.empty()) {
+      const int32_t i = stack.back();
+      stack.pop_back();
+      if (i < 0 || i >= graph->n_nodes || seen[i]) continue;
+      seen[i] = 1;
       for (int k = 0; k < graph->nodes[i].n_inputs; ++k) {
         int32_t r = graph->nodes[i].inputs[k];
         if (r < 0 && (-r) % 2 == 1) ud[(-r - 1) / 2] = 1;
         if (r < 0 && (-r) % 2 == 0) us[(-r - 2) / 2] = 1;
+        if (r >= 0) stack.push_back(r);
       }
+    }
     for (int c = 0; c < graph->n_dense_in; ++c)
       if (ud[c]) P->used_dense.push_back(c);
     for (int c = 0; c < graph->n_sparse_in; ++c)
@@ -1958,9 +1967,28 @@ rap_status rap_plan_output_costs(const rap_plan* P, int64_t n_rows, const int64_
   return RAP_OK;
 }
 
+static rap_status place_impl(const double* cost, const int32_t* colocate, int32_t n, int32_t world, int32_t mode,
+                             int64_t n_rows, double imbalance_tol, const rap_comm_model* comm, int32_t* owner_out,
+                             double* load_out, rap_residual* residual);
+
 rap_status rap_place(const double* cost, const int32_t* colocate, int32_t n, int32_t world, int32_t mode,
                      int64_t n_rows, double imbalance_tol, int32_t* owner_out, double* load_out,
                      rap_residual* residual) {
+  return place_impl(cost, colocate, n, world, mode, n_rows, imbalance_tol, nullptr, owner_out, load_out, residual);
+}
+
+rap_status rap_place_comm(const double* cost, const int32_t* colocate, int32_t n, int32_t world, int32_t mode,
+                          int64_t n_rows, const rap_comm_model* comm, int32_t* owner_out, double* load_out,
+                          rap_residual* residual) {
+  if (comm && (!(comm->us_per_unit > 0) || !(comm->link_gbs > 0) || !(comm->link_latency_us >= 0) ||
+               (n > 0 && !comm->row_bytes)))
+    return fail(RAP_ERR_INVALID_ARGUMENT, "comm model: us_per_unit, link_gbs > 0, link_latency_us >= 0, row_bytes");
+  return place_impl(cost, colocate, n, world, mode, n_rows, 0.0, comm, owner_out, load_out, residual);
+}
+
+static rap_status place_impl(const double* cost, const int32_t* colocate, int32_t n, int32_t world, int32_t mode,
+                             int64_t n_rows, double imbalance_tol, const rap_comm_model* comm, int32_t* owner_out,
+                             double* load_out, rap_residual* residual) {
   if (n < 0 || world < 1 || n_rows < 0) return fail(RAP_ERR_INVALID_ARGUMENT, "bad size");
   if (n > 0 && (!cost || !owner_out)) return fail(RAP_ERR_INVALID_ARGUMENT, "NULL argument");
   if (mode < RAP_PLACE_BALANCED || mode > RAP_PLACE_SKEWED) return fail(RAP_ERR_INVALID_ARGUMENT, "bad mode");
@@ -2028,20 +2056,33 @@ rap_status rap_place(const double* cost, const int32_t* colocate, int32_t n, int
         if (load[r] < load[l]) l = r;
       }
       const double mean = total / world;
-      if (load[h] > mean * (1.0 + imbalance_tol) && h != l) {
+      if ((comm || load[h] > mean * (1.0 + imbalance_tol)) && h != l) {
         int f = -1;
         for (int j = 0; j < n; ++j)
           if (owner_out[j] == h && (f < 0 || cost[j] > cost[f])) f = j;
         const double per_row = f >= 0 ? cost[f] / (double)n_rows : 0.0;
         if (per_row > 0) {
-          const double delta = 0.5 * (load[h] - load[l]);
+          double want_rows = 0.5 * (load[h] - load[l]) / per_row;
+          double t0 = 0, t1 = 0;  // exchange cost in cost units: t(m) = t0 + m * t1
+          if (comm) {
+            t0 = comm->link_latency_us / comm->us_per_unit;
+            t1 = comm->row_bytes[f] / (1e3 * comm->link_gbs) / comm->us_per_unit;
+            want_rows = (load[h] - load[l] - t0) / (2.0 * per_row + t1);
+          }
           // split row: a multiple of 128 (whole validity words / tiles on both
-          // sides), the owner keeping at least one tile
-          const int64_t want = std::min((int64_t)(delta / per_row), n_rows);
+          // sides), the owner keeping at least one tile; rounded so that at
+          // most want_rows move
+          const int64_t want = std::max<int64_t>(0, std::min((int64_t)std::max(0.0, want_rows), n_rows));
           int64_t split = (n_rows - want + kTileRows - 1) / kTileRows * kTileRows;
           split = std::max<int64_t>(split, kTileRows);
           const int64_t moved = n_rows - split;
-          if (moved > 0) {
+          bool gain = moved > 0;
+          if (comm && gain) {
+            const double m = (double)moved;
+            const double finish = std::max(load[h] - m * per_row, load[l] + m * per_row + t0 + m * t1);
+            gain = finish < load[h];
+          }
+          if (gain) {
             residual->output = f;
             residual->owner = h;
             residual->helper = l;

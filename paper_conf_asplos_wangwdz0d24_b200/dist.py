@@ -43,6 +43,43 @@ def _raw_sparse_source(spec, node):
         node = idx
 
 
+def sparse_sources(spec, node) -> list:
+    """Raw sparse columns a node reads (through every input, sorted)."""
+    seen, out, stack = set(), set(), [node]
+    while stack:
+        n = stack.pop()
+        if n in seen:
+            continue
+        seen.add(n)
+        for kind, idx in spec["nodes"][n]["inputs"]:
+            if kind == "s":
+                out.add(idx)
+            elif kind == "n":
+                stack.append(idx)
+    return sorted(out)
+
+
+def row_bytes(spec, sp_nnz, n_rows: int) -> list:
+    """Bytes one row of each sparse output moves in a residual exchange: its
+    raw input row (offset, validity bit, ids of every source) to the helper and
+    its output row (length, offset, ids -- bounded by the sources' ids) back."""
+    B = max(int(n_rows), 1)
+    out = []
+    for n in sparse_output_nodes(spec):
+        ids = sum(float(sp_nnz[c]) / B for c in sparse_sources(spec, n))
+        srcs = len(sparse_sources(spec, n))
+        out.append(srcs * (4 + 1 / 8) + 8 * ids + 12 + 8 * ids)
+    return out
+
+
+@dataclass
+class CommModel:
+    """rap_comm_model: cost-unit time scale and the owner <-> helper link."""
+    us_per_unit: float
+    link_gbs: float = 700.0        # NVLink 5 / NVSwitch point-to-point, effective
+    link_latency_us: float = 20.0  # one NCCL send/recv pair: launch + synchronisation
+
+
 def colocation(spec) -> list:
     """colocate[j] for the sparse outputs: an NGram table goes with the table
     of its first source column, -1 otherwise."""
@@ -82,20 +119,30 @@ class Placement:
     mode: str
 
 
-def place(costs, colocate, world: int, mode: str = "balanced", n_rows: int = 0, imbalance_tol: float | None = 0.1):
+def place(costs, colocate, world: int, mode: str = "balanced", n_rows: int = 0, imbalance_tol: float | None = 0.1,
+          comm: CommModel | None = None, row_bytes_=None):
     """rap_place (host only): table-wise owner of every sparse output, the
     predicted load per rank and the residual move (imbalance_tol None = never
-    rebalance)."""
+    rebalance).  With a comm model (rap_place_comm) the move is made only when
+    it shortens the owner's finish time after the exchange (L1594-1600)."""
     n = len(costs)
     c = np.ascontiguousarray(costs, dtype=np.float64)
     col = np.ascontiguousarray(colocate if colocate is not None else [-1] * n, dtype=np.int32)
     own = np.zeros(max(n, 1), dtype=np.int32)
     loads = np.zeros(world, dtype=np.float64)
     res = rap.RapResidual()
-    rap._check(rap.load().rap_place(c.ctypes.data if n else None, col.ctypes.data if n else None, n, world,
-                                    rap.PLACE_MODES[mode], n_rows, 0.0 if imbalance_tol is None else imbalance_tol,
-                                    own.ctypes.data, loads.ctypes.data,
-                                    None if imbalance_tol is None else C.byref(res)))
+    L = rap.load()
+    if comm is not None and imbalance_tol is not None:
+        rb = np.ascontiguousarray(row_bytes_ if row_bytes_ is not None else [0.0] * n, dtype=np.float64)
+        cm = rap.RapCommModel(comm.us_per_unit, comm.link_gbs, comm.link_latency_us, rb.ctypes.data if n else None)
+        rap._check(L.rap_place_comm(c.ctypes.data if n else None, col.ctypes.data if n else None, n, world,
+                                    rap.PLACE_MODES[mode], n_rows, C.byref(cm), own.ctypes.data, loads.ctypes.data,
+                                    C.byref(res)))
+    else:
+        rap._check(L.rap_place(c.ctypes.data if n else None, col.ctypes.data if n else None, n, world,
+                               rap.PLACE_MODES[mode], n_rows, 0.0 if imbalance_tol is None else imbalance_tol,
+                               own.ctypes.data, loads.ctypes.data,
+                               None if imbalance_tol is None else C.byref(res)))
     r = None
     if imbalance_tol is not None and res.output >= 0:
         r = Residual(res.output, res.owner, res.helper, res.split_row)
@@ -103,14 +150,16 @@ def place(costs, colocate, world: int, mode: str = "balanced", n_rows: int = 0, 
 
 
 def plan_placement(spec, n_rows: int, sp_nnz, world: int, mode: str = "balanced", imbalance_tol=0.1,
-                   device: int = 0) -> Placement:
-    """Placement from the plan's own cost model (rap_plan_output_costs)."""
+                   device: int = 0, comm: CommModel | None = None) -> Placement:
+    """Placement from the plan's own cost model (rap_plan_output_costs);
+    comm: cost the residual move's exchange (rap_place_comm)."""
     full = rap.Plan(spec, device=device)
     try:
         costs = full.output_costs(n_rows, sp_nnz)
     finally:
         full.close()
-    return place(costs, colocation(spec), world, mode, n_rows, imbalance_tol)
+    return place(costs, colocation(spec), world, mode, n_rows, imbalance_tol, comm,
+                 row_bytes(spec, sp_nnz, n_rows) if comm is not None else None)
 
 
 class RankOutput:
@@ -159,6 +208,24 @@ def nccl_exchange(rank: int, res: Residual, piece, recv_bufs, group=None):
             w.wait()
 
 
+def gloo_exchange(rank: int, res: Residual, piece, recv_bufs, group=None):
+    """The residual exchange staged through host memory over a CPU (gloo)
+    group: ranks sharing one GPU (tests), where NCCL cannot run two ranks on
+    one device.  Same protocol and buffers as nccl_exchange."""
+    import torch
+    import torch.distributed as dist
+
+    if rank == res.helper:
+        torch.cuda.synchronize()
+        for t in piece:
+            dist.send(t.cpu(), res.owner, group=group)
+    elif rank == res.owner:
+        for t in recv_bufs:
+            h = torch.empty(t.shape, dtype=t.dtype)
+            dist.recv(h, res.helper, group=group)
+            t.copy_(h)
+
+
 class ShardedPreprocessor:
     """One rank of the multi-GPU preprocessing."""
 
@@ -199,6 +266,19 @@ class ShardedPreprocessor:
                              torch.empty(n_hi + 1, dtype=torch.int64, device=self.dev),
                              torch.empty(max(self.piece_bound, 1), dtype=torch.int64, device=self.dev)]
         self.values_cap = cap
+
+    def sparse_columns(self) -> list:
+        """Raw sparse columns this rank reads: its own tables' (and the
+        residual output's, on its owner and helper) -- what it uploads."""
+        sp_nodes = sparse_output_nodes(self.spec)
+        outs = list(self.main_features)
+        res = self.pl.residual
+        if res is not None and self.rank in (res.owner, res.helper):
+            outs.append(res.output)
+        cols = set()
+        for j in outs:
+            cols.update(sparse_sources(self.spec, sp_nodes[j]))
+        return sorted(cols)
 
     def new_output(self) -> RankOutput:
         return RankOutput(self.features, self.B, self.dense_rows, self.d_out, self.values_cap, self.dev)

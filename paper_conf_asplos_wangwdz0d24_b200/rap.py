@@ -23,7 +23,7 @@ EXPORTS = ["rap_plan_create", "rap_plan_output_shape", "rap_preprocess", "rap_pr
            "rap_predict_latency_us", "rap_choose_budget", "rap_plan_info_get", "rap_debug_trace", "rap_plan_destroy",
            "rap_status_string", "rap_last_error", "rap_shard_rows", "rap_plan_output_costs", "rap_place",
            "rap_plan_create_sharded", "rap_jagged_append", "rap_set_kernel", "rap_check_overflow",
-           "rap_debug_jit_source"]
+           "rap_debug_jit_source", "rap_place_comm"]
 PLACE_MODES = {"balanced": 0, "round_robin": 1, "skewed": 2}
 RAP_OUT_CHAIN = 1
 
@@ -66,6 +66,11 @@ class RapOutput(C.Structure):
 class RapResidual(C.Structure):
     _fields_ = [("output", C.c_int32), ("owner", C.c_int32), ("helper", C.c_int32), ("pad", C.c_int32),
                 ("split_row", C.c_int64)]
+
+
+class RapCommModel(C.Structure):
+    _fields_ = [("us_per_unit", C.c_double), ("link_gbs", C.c_double), ("link_latency_us", C.c_double),
+                ("row_bytes", C.c_void_p)]
 
 
 class RapPlanInfo(C.Structure):
@@ -143,6 +148,9 @@ def load(build_if_stale: bool = False):
     L.rap_place.restype = C.c_int
     L.rap_place.argtypes = [P, P, C.c_int32, C.c_int32, C.c_int32, C.c_int64, C.c_double, P, P,
                             C.POINTER(RapResidual)]
+    L.rap_place_comm.restype = C.c_int
+    L.rap_place_comm.argtypes = [P, P, C.c_int32, C.c_int32, C.c_int32, C.c_int64, C.POINTER(RapCommModel), P, P,
+                                 C.POINTER(RapResidual)]
     L.rap_plan_create_sharded.restype = C.c_int
     L.rap_plan_create_sharded.argtypes = [C.POINTER(RapGraph), C.POINTER(RapOpParam), C.c_int32, C.c_int32, C.c_int32,
                                           P, C.c_int32, C.c_int32, C.POINTER(P)]
@@ -236,7 +244,12 @@ def _stream_handle(stream):
 class DeviceBatch:
     """A raw batch resident in device memory (torch tensors) + its C struct."""
 
-    def __init__(self, batch, device, pin=False):
+    def __init__(self, batch, device, pin=False, sparse_cols=None, dense_rows=None):
+        """sparse_cols: upload only these raw sparse columns (the others get
+        NULL pointers: a sharded rank's plan reads only its own tables'
+        columns).  dense_rows = (row0, n): upload only those dense rows (a
+        rank's batch shard, row0 a multiple of 128); the column pointers are
+        biased by -row0 so the kernel's global row indices land in the copy."""
         import torch
 
         self.n_rows = int(batch["n_rows"])
@@ -246,19 +259,36 @@ class DeviceBatch:
             x = torch.from_numpy(np.ascontiguousarray(a, dtype=dt))
             return x.pin_memory() if pin else x.to(dev, non_blocking=False)
 
-        self.dense = [t(x, np.float32) for x in batch["dense"]]
-        self.dense_valid = [None if x is None else t(x, np.uint32) for x in batch["dense_valid"]]
-        self.sp_off = [t(x, np.int32) for x in batch["sp_off"]]
-        self.sp_val = [t(x, np.int64) if len(x) else t(np.zeros(1, np.int64), np.int64) for x in batch["sp_val"]]
-        self.sp_valid = [None if x is None else t(x, np.uint32) for x in batch["sp_valid"]]
+        r0, nd = (0, self.n_rows) if dense_rows is None else dense_rows
+        assert r0 % 128 == 0 and 0 <= r0 and r0 + nd <= self.n_rows
+        self._dense_bias = r0
+        self.dense = [t(x[r0:r0 + nd], np.float32) for x in batch["dense"]]
+        w0, w1 = r0 // 32, (r0 + nd + 31) // 32
+        self.dense_valid = [None if x is None else t(x[w0:w1], np.uint32) for x in batch["dense_valid"]]
+        keep = range(len(batch["sp_off"])) if sparse_cols is None else set(sparse_cols)
+        self.sp_off = [t(x, np.int32) if c in keep else None for c, x in enumerate(batch["sp_off"])]
+        self.sp_val = [(t(x, np.int64) if len(x) else t(np.zeros(1, np.int64), np.int64)) if c in keep else None
+                       for c, x in enumerate(batch["sp_val"])]
+        self.sp_valid = [None if (x is None or c not in keep) else t(x, np.uint32)
+                         for c, x in enumerate(batch["sp_valid"])]
         self.sp_nnz = np.array([int(o[-1]) - int(o[0]) for o in batch["sp_off"]] or [0], dtype=np.int64)
         self._build_struct()
+
+    def uploaded_bytes(self) -> int:
+        xs = self.dense + self.dense_valid + self.sp_off + self.sp_val + self.sp_valid
+        return int(sum(x.numel() * x.element_size() for x in xs if x is not None))
 
     def _build_struct(self):
         def ptr(x):
             return None if x is None else x.data_ptr()
 
-        self._arrs = [_ptr_array([ptr(x) for x in self.dense]), _ptr_array([ptr(x) for x in self.dense_valid]),
+        bias = getattr(self, "_dense_bias", 0)
+
+        def dptr(x, elem_rows):  # dense pointers biased to global row 0 (dense_rows shard uploads)
+            return None if x is None else x.data_ptr() - (bias // elem_rows) * 4
+
+        self._arrs = [_ptr_array([dptr(x, 1) for x in self.dense]),
+                      _ptr_array([dptr(x, 32) for x in self.dense_valid]),
                       _ptr_array([ptr(x) for x in self.sp_off]), _ptr_array([ptr(x) for x in self.sp_val]),
                       _ptr_array([ptr(x) for x in self.sp_valid])]
         a = self._arrs
@@ -272,10 +302,12 @@ def row_view(raw: "DeviceBatch", row0: int, n_rows: int) -> "RapRawBatch":
     arithmetic only; row0 a multiple of 32 so validity words stay whole).
     sp_nnz stays the full batch's (an upper bound, used only for capacity)."""
     assert row0 % 32 == 0 and 0 <= row0 and row0 + n_rows <= raw.n_rows
-    def ptrs(xs, elem, scale=1):
-        return _ptr_array([None if x is None else x.data_ptr() + (row0 // scale) * elem for x in xs])
-    arrs = [ptrs(raw.dense, 4), ptrs(raw.dense_valid, 4, 32), ptrs(raw.sp_off, 4),
-            _ptr_array([x.data_ptr() for x in raw.sp_val]), ptrs(raw.sp_valid, 4, 32)]
+    bias = getattr(raw, "_dense_bias", 0)  # a dense_rows upload holds rows [bias, ...)
+
+    def ptrs(xs, elem, scale=1, b=0):
+        return _ptr_array([None if x is None else x.data_ptr() + ((row0 - b) // scale) * elem for x in xs])
+    arrs = [ptrs(raw.dense, 4, 1, bias), ptrs(raw.dense_valid, 4, 32, bias), ptrs(raw.sp_off, 4),
+            _ptr_array([None if x is None else x.data_ptr() for x in raw.sp_val]), ptrs(raw.sp_valid, 4, 32)]
     st = RapRawBatch(n_rows, *[C.cast(a, C.c_void_p) for a in arrs], raw.sp_nnz.ctypes.data)
     st._keep = arrs
     return st

@@ -79,6 +79,49 @@ def test_place_skewed_and_residual():
 
 
 # ------------------------------------------------------- gloo residual protocol
+def test_place_comm_moves_only_when_the_exchange_pays():
+    """rap_place_comm (L1594-1600): a skewed placement moves rows only when the
+    owner's finish time after the exchange beats keeping them; the chosen
+    split balances compute against compute + transfer."""
+    c = np.full(32, 100.0)
+    B = 65536
+    base = dist.place(c, None, 4, "skewed", B, None)
+    L = np.array(base.loads)
+    rb = [64.0] * 32
+    # a fast link with little latency: a move is made, and it beats no move
+    fast = dist.CommModel(us_per_unit=0.01, link_gbs=700.0, link_latency_us=5.0)
+    pf = dist.place(c, None, 4, "skewed", B, 0.0, fast, rb)
+    r = pf.residual
+    assert r is not None and r.owner == 0 and r.split_row % 128 == 0
+    m = B - r.split_row
+    p = c[r.output] / B
+    t = lambda rows: (fast.link_latency_us + rows * rb[r.output] / (1e3 * fast.link_gbs)) / fast.us_per_unit
+    finish = max(L[0] - m * p, L[r.helper] + m * p + t(m))
+    assert finish < L[0]
+    # optimal within one 128-row tile: one tile more or less is not better
+    for d in (-128, 128):
+        m2 = m + d
+        if 0 < m2 < B:
+            assert finish <= max(L[0] - m2 * p, L[r.helper] + m2 * p + t(m2)) + 1e-9
+    # the same imbalance over a link whose latency exceeds the whole gain: no move
+    slow = dist.CommModel(us_per_unit=0.01, link_gbs=700.0, link_latency_us=0.01 * (L[0] - L.min()) * 1.01)
+    assert dist.place(c, None, 4, "skewed", B, 0.0, slow, rb).residual is None
+    # huge rows: the transfer outweighs the compute moved
+    assert dist.place(c, None, 4, "skewed", B, 0.0, fast, [1e9] * 32).residual is None
+
+
+def test_row_bytes_and_sparse_sources_c2():
+    w = synth.c2_terabyte(0)
+    nnz = np.full(26, 65536)
+    rb = dist.row_bytes(w.spec, nnz, 65536)
+    assert len(rb) == 34
+    # a single-id table moves ~ offset + id in, length + offset + id out; a trigram 3 sources
+    assert rb[0] == pytest.approx(4.125 + 8 + 12 + 8)
+    assert rb[26] == pytest.approx(3 * 4.125 + 24 + 12 + 24)
+    nodes = dist.sparse_output_nodes(w.spec)
+    assert dist.sparse_sources(w.spec, nodes[26]) == [0, 1, 2]
+
+
 def _slice_batch(h, r0, n):
     """Rows [r0, r0+n) of a host batch (r0 % 32 == 0); offsets stay absolute."""
     w0, w1 = r0 // 32, (r0 + n + 31) // 32
@@ -227,3 +270,83 @@ def test_sharded_ranks_match_oracle(world, mode):
     for rk in ranks:
         rk.close()
     full.close()
+
+
+# ------------------------------------------- GPU: two processes, one device
+def _gpu_rank_worker(rank, world, port, mode, q):
+    import torch
+    import torch.distributed as tdist
+
+    from oracle import oracle
+    from paper_conf_asplos_wangwdz0d24_b200 import rap
+    from tests.parity import dense_close
+
+    try:
+        os.environ["MASTER_ADDR"] = "127.0.0.1"
+        os.environ["MASTER_PORT"] = str(port)
+        tdist.init_process_group("gloo", rank=rank, world_size=world)
+        torch.cuda.set_device(0)
+        w = synth.c2_terabyte(0)
+        B = 2600
+        h = synth.make_batch(w, B, seed=33)
+        sp_nnz = np.array([int(o[-1]) - int(o[0]) for o in h["sp_off"]], dtype=np.int64)
+        pl = dist.plan_placement(w.spec, B, sp_nnz, world, mode, imbalance_tol=0.05)
+        sp = dist.ShardedPreprocessor(w.spec, pl, rank, world, B, sp_nnz, device=0)
+        # this rank uploads only its own tables' columns and its dense shard
+        raw = rap.DeviceBatch(h, "cuda:0", sparse_cols=sp.sparse_columns(), dense_rows=(sp.row0, sp.dense_rows))
+        full = rap.DeviceBatch(h, "cuda:0")
+        assert raw.uploaded_bytes() < full.uploaded_bytes()
+        del full
+        out = sp.new_output()
+        for _ in range(2):  # twice: the chained launch and the append are re-entrant
+            sp.preprocess(raw, out, exchange=dist.gloo_exchange)
+        torch.cuda.synchronize()
+        got = out.to_numpy()
+        want = oracle.run(w.spec, h)
+        F = len(dist.sparse_output_nodes(w.spec))
+        wl = _feature_lists(want, F, B)
+        gl = _feature_lists(got, len(got["features"]), B)
+        assert dense_close(got["dense"], want["dense"][sp.row0:sp.row0 + sp.dense_rows]).all()
+        for k, j in enumerate(got["features"]):
+            assert all(np.array_equal(a, b) for a, b in zip(gl[k], wl[j])), (rank, j)
+        assert got["offsets"][0] == 0 and np.array_equal(np.diff(got["offsets"]), got["lengths"].reshape(-1))
+        res = pl.residual
+        q.put((rank, {"features": got["features"], "residual": None if res is None else res.__dict__}))
+        sp.close()
+        tdist.destroy_process_group()
+    except Exception as e:  # noqa: BLE001 - reported to the parent
+        import traceback
+
+        q.put((rank, "ERR " + repr(e) + traceback.format_exc()[-1500:]))
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("mode", ["skewed", "balanced"])
+def test_two_processes_one_gpu_vs_oracle(mode):
+    """Two ranks as two processes on one B200 (gloo group, host-staged
+    residual exchange): each uploads only its own columns and dense shard, and
+    its KJT features and dense rows equal the oracle's single-process result."""
+    import multiprocessing as mp
+
+    import torch
+
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_gpu_rank_worker, args=(r, 2, port, mode, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    got = dict(q.get(timeout=600) for _ in range(2))
+    for p in procs:
+        p.join(120)
+    errs = {r: got[r] for r in range(2) if isinstance(got[r], str)}
+    assert not errs, errs
+    assert all(p.exitcode == 0 for p in procs)
+    feats = sorted(got[0]["features"] + got[1]["features"])
+    assert feats == list(range(34))
+    if mode == "skewed":
+        assert got[0]["residual"] is not None
