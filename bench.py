@@ -403,8 +403,22 @@ def run_rap(args):
 
         train = cr.DLRMStep(dev)
         budgets = [int(b) for b in args.corun_budgets.split(",") if b]
-        corun = cr.measure(plan, sets, train, budgets)
+        corun = cr.measure(plan, sets, train, budgets, choose=(B, sets[0][0].sp_nnz))
         corun["training"] = "synthetic DLRM step (DESIGN.md §12): 26 tables x 128 fp32 (TB share at 8 GPUs), batch 8192"
+        # layer-aligned scheduling (Algorithm 1): chunks launched as their layers begin
+        layer_us = train.layer_times_us()
+        alone = corun["train_step_alone_ms"]
+        corun["layer_aligned"] = {"layer_us": layer_us, "per_budget": []}
+        lsets = [r for r, _ in sets[:2]]
+        for lb in (0, 8, 2):
+            lap = cr.LayerAlignedPrep(w.spec, B, sets[0][0].sp_nnz, layer_us, device=dev.index, budget=lb)
+            louts = [lap.output(r.sp_nnz, dev) for r in lsets]
+            t_l, p_l = cr.measure_layer_aligned(lap, lsets, louts, train)
+            corun["layer_aligned"]["per_budget"].append(
+                {"pack_budget": lb, "chunks": lap.describe(), "train_step_corun_ms": t_l, "prep_done_ms": p_l,
+                 "slowdown": t_l / alone - 1.0, "prep_hidden": p_l <= t_l})
+            lap.close()
+            del louts
         del train
         torch.cuda.empty_cache()
     c4 = None

@@ -248,11 +248,23 @@ rap_status rap_set_budget(rap_plan* plan, int32_t sm_budget);
 
 /* Co-running cost model (§5, L871-879 and L1138-1143):
  * predicted standalone latency P (microseconds) of one rap_preprocess for a
- * batch of n_rows under sm_budget, from an analytic roofline predictor
- * (bytes / bandwidth share of the budget + launch cost) that replaces the
- * paper's XGBoost model (L1037-1057).  sp_nnz as in rap_plan_output_shape. */
+ * batch of n_rows under sm_budget, replacing the paper's XGBoost predictor
+ * (L1037-1057) with a structural model of the launch the plan would make:
+ * P = t0[kernel] + c[kernel] * (busiest CTA's predicted work) + bytes / BW,
+ * its constants fitted on B200.  sp_nnz as in
+ * rap_plan_output_shape. */
 rap_status rap_predict_latency_us(const rap_plan* plan, int64_t n_rows, const int64_t* sp_nnz,
                                   int32_t sm_budget, double* latency_us);
+
+/* The latency model's inputs for a launch of n_rows at sm_budget (0 = all
+ * SMs), as rap_predict_latency_us evaluates them: terms[0] the kernel it
+ * takes (RAP_KERNEL_TILED / _ROWS / _JIT), terms[1] its grid (CTAs),
+ * terms[2] the busiest CTA's predicted sparse work (cost units), terms[3]
+ * the algorithmic bytes, terms[4] its dense work (the generated kernel: its
+ * dense warp's), terms[5] its (sparse output, row) pairs.  terms: HOST
+ * double[6].  For refitting the model. */
+rap_status rap_predict_terms(const rap_plan* plan, int64_t n_rows, const int64_t* sp_nnz, int32_t sm_budget,
+                             double* terms);
 
 /* Smallest budget whose predicted exposed latency T_delta = P - OC is <= 0
  * for the given overlapping capacity OC (microseconds of training slack),

@@ -46,35 +46,71 @@ class DLRMStep:
         iu = torch.triu_indices(n_tables + 1, n_tables + 1, 1)
         self.iu = (iu[0].to(device), iu[1].to(device))
 
-    def step(self):
-        """Forward, backward, SGD (MLP weights and the gathered embedding rows)."""
+    LAYERS = ("bottom_mlp", "embedding", "interaction", "top_mlp", "backward", "update")
+
+    def step(self, hook=None):
+        """Forward, backward, SGD (MLP weights and the gathered embedding rows).
+        hook(layer) is called on the training stream as each layer begins
+        (layer-aligned co-run scheduling, §7.1)."""
         import torch
 
+        h = hook or (lambda name: None)
+        h("bottom_mlp")
         x = self.dense
         for i, w in enumerate(self.bot):
             x = x @ w.t()
             x = torch.relu(x) if i < len(self.bot) - 1 else x
+        h("embedding")
         embs = [t.index_select(0, i).to(torch.bfloat16).requires_grad_() for t, i in zip(self.tables, self.idx)]
+        h("interaction")
         feats = torch.stack([x] + embs, dim=1)                        # [B, 27, dim]
         inter = torch.bmm(feats, feats.transpose(1, 2))[:, self.iu[0], self.iu[1]]
         z = torch.cat([x, inter], dim=1)
+        h("top_mlp")
         for i, w in enumerate(self.top):
             z = z @ w.t()
             z = torch.relu(z) if i < len(self.top) - 1 else z
         loss = torch.nn.functional.binary_cross_entropy_with_logits(z.float(), self.label.float())
+        h("backward")
         params = self.bot + self.top
         grads = torch.autograd.grad(loss, params + embs)
+        h("update")
         with torch.no_grad():
             for p, gr in zip(params, grads[: len(params)]):
                 p.sub_(self.lr * gr)
             for t, i, gr in zip(self.tables, self.idx, grads[len(params):]):
                 t.index_add_(0, i, gr.float(), alpha=-self.lr)
+        h(None)
         return loss
 
+    def layer_times_us(self, steps=10):
+        """Median duration of every layer of the step run alone (events on the
+        stream): the windows the layer-aligned schedule fills."""
+        import torch
 
-def measure(plan, sets, train: DLRMStep, budgets, steps=20, warmup=5):
+        per = {n: [] for n in self.LAYERS}
+        for _ in range(steps + 2):
+            evs = []
+
+            def hook(name):
+                e = torch.cuda.Event(enable_timing=True)
+                e.record()
+                evs.append((name, e))
+
+            torch.cuda.synchronize()
+            self.step(hook)
+            torch.cuda.synchronize()
+            for (n, a), (_, b) in zip(evs, evs[1:]):
+                per[n].append(a.elapsed_time(b) * 1e3)
+        return {n: float(np.median(v[2:])) for n, v in per.items()}
+
+
+def measure(plan, sets, train: DLRMStep, budgets, steps=20, warmup=5, choose=None):
     """Per budget: training step alone vs co-run with one preprocessing launch
-    per step (events on each stream), in ms, and the slowdown."""
+    per step (events on each stream), in ms, and the slowdown.  choose =
+    (n_rows, sp_nnz): also the budget rap_choose_budget picks for an overlap
+    capacity OC = the measured training step (the preprocessing of the next
+    batch hides under one step, T_delta = P - OC <= 0, L1138-1152)."""
     import torch
 
     hi = torch.cuda.Stream(priority=-1)  # training: highest priority
@@ -106,6 +142,17 @@ def measure(plan, sets, train: DLRMStep, budgets, steps=20, warmup=5):
     run(warmup, True)
     alone, _ = run(steps, False)
     res = {"train_step_alone_ms": alone, "per_budget": []}
+    budgets = list(budgets)
+    chosen = None
+    if choose is not None:
+        n_rows, nnz = choose
+        oc_us = alone * 1e3
+        b, td = plan.choose_budget(n_rows, nnz, oc_us)
+        chosen = {"sm_budget": b, "overlap_capacity_us": oc_us, "predicted_us": plan.predict_latency_us(n_rows, nnz, b),
+                  "t_delta_us": td}
+        res["chosen"] = chosen
+        if b not in budgets:
+            budgets.append(b)
     for b in budgets:
         plan.set_budget(b)
         run(warmup, True)
@@ -113,6 +160,128 @@ def measure(plan, sets, train: DLRMStep, budgets, steps=20, warmup=5):
         t, p = run(steps, True)
         res["per_budget"].append({"sm_budget": b, "train_step_corun_ms": t, "prep_corun_ms": p,
                                   "prep_alone_ms": prep_alone, "slowdown": t / alone - 1.0,
-                                  "prep_hidden": p <= t})
+                                  "prep_hidden": p <= t, "chosen": chosen is not None and b == chosen["sm_budget"]})
+        if chosen is not None and b == chosen["sm_budget"]:
+            chosen.update({"measured_prep_alone_us": prep_alone * 1e3, "slowdown": t / alone - 1.0})
     plan.set_budget(0)
     return res
+
+
+# ------------------------------------------------- layer-aligned scheduling
+class LayerAlignedPrep:
+    """Layer-aligned co-run scheduling (§5.1, §7.1
+    Algorithm 1): the plan's sparse outputs are cut into chunks
+    (graph pieces, consecutive in output order; the dense outputs ride with
+    the first) and each chunk is launched as its own fused kernel when a
+    chosen training layer begins, on a low-priority stream, under the SM
+    budget rap_choose_budget gives it for that layer's window (its overlap
+    capacity OC_l, the layer's duration alone).  `budget` sets the SM count
+    the greedy packs for (0 = all SMs).  Assignment is Algorithm 1's
+    greedy: walk the layers in step order, give the current layer outputs
+    while their predicted latency fits its remaining capacity, and when an
+    output group does not fit, shard it -- the part that fits stays, the rest
+    starts the next layer.  Chunks chain into ONE output (RAP_OUT_CHAIN), so
+    the result equals the single fused launch (tests/test_gpu_corun.py)."""
+
+    def __init__(self, spec, n_rows, sp_nnz, layer_us, device=0, order=None, min_chunk=2, budget=0):
+        from . import dist, rap, synth
+
+        self.B = n_rows
+        self.layers = list(order or DLRMStep.LAYERS)
+        full = rap.Plan(spec, device=device)
+        types = synth.output_types(spec)
+        sp_outs = [o for o, t in zip(spec["outputs"], types) if t == "I"]
+        dn_outs = [o for o, t in zip(spec["outputs"], types) if t != "I"]
+        costs = full.output_costs(n_rows, sp_nnz)
+        # the greedy packs by the latency at `budget` SMs (0 = all): a small
+        # budget spreads the chunks over more layers, each on fewer SMs
+        p_full = full.predict_latency_us(n_rows, sp_nnz, budget)
+        d_out, f_out, _ = full.output_shape(n_rows, sp_nnz)
+        full.close()
+        total = float(sum(costs)) or 1.0
+        # Algorithm 1 (greedy over layers, shard on overflow): predicted
+        # latency of a group ~ its share of the full plan's at all SMs
+        share = [p_full * c / total for c in costs]
+        cap = [float(layer_us[n]) for n in self.layers]
+        assign, li, cur, used = [], 0, [], 0.0
+        for j in range(len(sp_outs)):
+            if cur and used + share[j] > cap[li] and len(cur) >= min_chunk and li + 1 < len(self.layers):
+                assign.append((self.layers[li], cur))
+                li, cur, used = li + 1, [], 0.0
+            cur.append(j)
+            used += share[j]
+        if cur:
+            assign.append((self.layers[li], cur))
+        self.chunks = []
+        slot = 0
+        for k, (layer, js) in enumerate(assign):
+            sub = dict(spec)
+            sub["outputs"] = (dn_outs if k == 0 else []) + [sp_outs[j] for j in js]
+            plan = rap.Plan(sub, device=device)
+            oc = float(layer_us[layer])
+            b, td = plan.choose_budget(n_rows, sp_nnz, oc)
+            if budget > 0:  # never below the budget the chunk was packed for
+                b = max(b, budget)
+                td = plan.predict_latency_us(n_rows, sp_nnz, b) - oc
+            plan.set_budget(b)
+            self.chunks.append({"layer": layer, "outputs": js, "plan": plan, "slot": slot, "budget": b,
+                                "oc_us": oc, "t_delta_us": td,
+                                "predicted_us": plan.predict_latency_us(n_rows, sp_nnz, b)})
+            slot += len(js)
+        self.d_out, self.f_out = d_out, f_out
+        self.features = list(range(len(sp_outs)))
+        self._dist = dist
+
+    def output(self, sp_nnz, device):
+        vb = sum(c["plan"].output_shape(self.B, sp_nnz)[2] for c in self.chunks)
+        return self._dist.RankOutput(self.features, self.B, self.B, self.d_out, vb, device)
+
+    def launch(self, raw, out, stream, layer=None):
+        """Launch the chunks assigned to `layer` (None: every chunk) on stream."""
+        for c in self.chunks:
+            if layer is None or c["layer"] == layer:
+                c["plan"].preprocess_struct(raw.struct, out.struct(c["slot"], 0, chain=c["slot"] > 0), stream)
+
+    def describe(self):
+        return [{k: v for k, v in c.items() if k != "plan"} for c in self.chunks]
+
+    def close(self):
+        for c in self.chunks:
+            c["plan"].close()
+
+
+def measure_layer_aligned(lap: LayerAlignedPrep, sets_raw, outs, train: DLRMStep, steps=20, warmup=5):
+    """Training step co-run with the layer-aligned chunks: each chunk's launch
+    on the low-priority stream waits for an event recorded when its layer
+    begins on the training stream."""
+    import torch
+
+    hi = torch.cuda.Stream(priority=-1)
+    lo = torch.cuda.Stream(priority=0)
+    t_train, t_prep = [], []
+    assert len(sets_raw) == len(outs)  # output i sized for batch i
+    for i in range(warmup + steps):
+        raw, out = sets_raw[i % len(sets_raw)], outs[i % len(outs)]
+        a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        p0, p1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+
+        def hook(name):
+            if name is None or not any(c["layer"] == name for c in lap.chunks):
+                return
+            e = torch.cuda.Event()
+            e.record(hi)
+            lo.wait_event(e)
+            lap.launch(raw, out, lo, name)
+
+        with torch.cuda.stream(hi):
+            a0.record(hi)
+            p0.record(hi)
+            train.step(hook)
+            a1.record(hi)
+        p1.record(lo)
+        torch.cuda.synchronize()
+        if i >= warmup:
+            t_train.append(a0.elapsed_time(a1))
+            t_prep.append(p0.elapsed_time(p1))
+    return float(np.median(t_train)), float(np.median(t_prep))

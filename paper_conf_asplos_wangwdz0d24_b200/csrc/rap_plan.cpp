@@ -65,6 +65,12 @@ int64_t sat_mul(int64_t a, int64_t b) {
 
 }  // namespace
 
+// Latency-model constants (rap_predict_latency_us): t0/c per kernel family
+// and the HBM bandwidth, fitted on B200 (profiles/r02_cost_model_fit.txt).
+#ifndef RAP_MODEL_FIT
+#define RAP_MODEL_FIT 39.9236, 2.08214e-05, 0, 11.94, 0, 0.0102245, 4.9372, 0, 0.00371049, 6446.6
+#endif
+
 struct rap_plan {
   int device = 0, sm_count = 0, budget = 0, ctas_per_sm = 1, smem = 0;
   int n_dense_in = 0, n_sparse_in = 0;
@@ -1571,9 +1577,10 @@ static bool use_rows(const rap_plan* P, int64_t B, const int64_t* nnz) {
 // (<= a quarter of the slots) each gets a dedicated CTA, so small batches run
 // the dense outputs beside the sparse phases rather than after them.
 static void rows_geometry(const rap_plan* P, int64_t B, const int64_t* nnz, int ctas_per_sm, RbGeom* g,
-                          int64_t n_dense_tiles = 0) {
+                          int64_t n_dense_tiles = 0, int budget = 0) {
   const int F = (int)P->souts.size();
-  int64_t slots = std::max<int64_t>(1, std::min<int64_t>((int64_t)P->budget * ctas_per_sm, kMaxCtas));
+  const int bud = budget > 0 ? budget : P->budget;
+  int64_t slots = std::max<int64_t>(1, std::min<int64_t>((int64_t)bud * ctas_per_sm, kMaxCtas));
   g->n_dcta = 0;
   if (n_dense_tiles > 0 && n_dense_tiles <= slots / 4) {
     g->n_dcta = (int)n_dense_tiles;
@@ -1889,20 +1896,128 @@ rap_status rap_preprocess_host_async(rap_plan* P, const rap_raw_batch* raw, cons
   return preprocess_host_impl(P, raw, out, stream, false);
 }
 
+// ---- latency model (the paper's preprocessing latency predictor, §5.2
+// L1037-1057, for one fused launch at an SM budget) ----
+// The model replays the launch the plan would make (kernel, geometry) and
+// charges a fixed part, the busiest CTA's predicted work and the bytes:
+//   T(b) = t0[k] + c_work[k] * work(b) + c_pair[k] * pairs(b) + bytes / BW
+// with work the CTA's cost units (the tiled kernel's partition model) and
+// pairs its (sparse output, row) pairs (the row-block kernels: whole
+// 224/256-row chunks).  Least-squares fits to B200 kernel times over budgets
+// 8..148 for configs 1, 2 and 4 at several batch sizes (scripts/budget_sweep.py
+// -> scripts/fit_cost_model.py, profiles/r02_cost_model_fit.txt): the tiled
+// kernel is explained by work, the row-block kernels by pairs (a per-output
+// latency, not the op mix).  RAP_MODEL="t0,c_work,c_pair x 3 kernels,bw_gbs"
+// overrides the constants (refitting).
+struct PredTerms {
+  int family;      // RAP_KERNEL_TILED / _ROWS / _JIT
+  int64_t grid;    // CTAs
+  double work;     // sparse cost units of the busiest CTA
+  double bytes;    // algorithmic bytes of the launch
+  double dwork;    // dense cost units of that CTA (the generated kernel: its dense warp's)
+  double pairs;    // (sparse output, row) pairs of that CTA: a per-output latency the cost units miss
+};
+
+static PredTerms predict_terms(const rap_plan* P, int64_t B, const int64_t* nnz, int b) {
+  PredTerms t{RAP_KERNEL_TILED, 0, 0.0, B > 0 ? algorithmic_bytes(P, B, nnz) : 0.0, 0.0, 0.0};
+  if (B <= 0) return t;
+  const int F = (int)P->souts.size();
+  std::vector<double> fc(F);
+  double sparse = 0;
+  for (int f = 0; f < F; ++f) sparse += (fc[f] = sparse_row_cost(P, P->chains[P->souts[f].chain], B, nnz));
+  int64_t drow0 = 0, drows = B;
+  rap_shard_rows(B, P->rank, P->world, &drow0, &drows);
+  double dense = 0;
+  for (const DProg& dp : P->dprogs) dense += dense_row_cost(P, dp);
+  const int64_t n_dense = P->dprogs.empty() ? 0 : (int64_t)P->dprogs.size() * ((drows + kDenseBlockRows - 1) / kDenseBlockRows);
+  if (use_rows(P, B, nnz)) {
+    const bool small = values_bound(P, B, nnz) < (int64_t)INT32_MAX - 1;
+    const int iv = small ? 1 : 0;
+    const bool want_jit = (P->kernel_mode == RAP_KERNEL_JIT || P->kernel_mode == RAP_KERNEL_AUTO) && P->jit_st[iv] != -1;
+    RbGeom g;
+    memset(&g, 0, sizeof(g));
+    const int jocc = P->jit_occ[iv] > 0 ? P->jit_occ[iv] : P->rb_ctas_per_sm;
+    rows_geometry(P, B, nnz, want_jit ? jocc : P->rb_ctas_per_sm, &g, 0, b);
+    const bool jit = want_jit && g.n_fg == 1 && drow0 == 0 && drows == B;
+    if (!jit) rows_geometry(P, B, nnz, P->rb_ctas_per_sm, &g, n_dense, b);
+    const int chunk = jit ? 224 : kRbChunk;
+    const int64_t chunks = (g.rows_rb + chunk - 1) / chunk;
+    double gmax = 0;  // the costliest feature group's cost per row
+    int fmax = 0;
+    for (int k = 0; k < g.n_fg; ++k) {
+      double c = 0;
+      for (int i = g.fg_off[k]; i < g.fg_off[k + 1]; ++i) c += fc[P->rb_perm[i]];
+      if (c > gmax) {
+        gmax = c;
+        fmax = g.fg_off[k + 1] - g.fg_off[k];
+      }
+    }
+    t.pairs = (double)fmax * (double)(chunks * chunk);
+    t.family = jit ? RAP_KERNEL_JIT : RAP_KERNEL_ROWS;
+    t.grid = (int64_t)g.n_rb * g.n_fg + g.n_dcta;
+    t.work = gmax * (double)(chunks * chunk);
+    if (jit) {
+      t.dwork = dense * (double)std::min<int64_t>(g.rows_rb, B);  // the dense warp's rows
+    } else if (g.n_dcta > 0) {
+      t.dwork = dense * (double)kDenseBlockRows;  // one dense block per dedicated CTA
+    } else if (n_dense > 0) {
+      t.dwork = dense * (double)drows / (double)std::max<int64_t>(1, t.grid);  // round robin
+    }
+    return t;
+  }
+  const int64_t T = (B + kTileRows - 1) / kTileRows;
+  const int64_t want = std::max<int64_t>(1, std::max<int64_t>(n_dense, ((int64_t)F * T + kWarpsPerCta - 1) / kWarpsPerCta));
+  t.grid = std::min<int64_t>(std::min<int64_t>((int64_t)b * P->ctas_per_sm, kMaxCtas), want);
+  t.work = sparse * (double)B / (double)t.grid;
+  t.dwork = dense * (double)drows / (double)t.grid;
+  t.pairs = (double)F * (double)B / (double)t.grid;
+  return t;
+}
+
+static void model_constants(double k[10]) {
+  // per kernel (tiled, rows, generated): t0 (us), c_work (us per cost unit),
+  // c_pair (us per (output, row) pair); then the HBM bandwidth (GB/s)
+  static const double fit[10] = {RAP_MODEL_FIT};
+  for (int i = 0; i < 10; ++i) k[i] = fit[i];
+  if (const char* env = getenv("RAP_MODEL")) {
+    double v[10];
+    if (sscanf(env, "%lf,%lf,%lf,%lf,%lf,%lf,%lf,%lf,%lf,%lf", &v[0], &v[1], &v[2], &v[3], &v[4], &v[5], &v[6],
+               &v[7], &v[8], &v[9]) == 10)
+      for (int i = 0; i < 10; ++i) k[i] = v[i];
+  }
+}
+
+rap_status rap_predict_terms(const rap_plan* P, int64_t n_rows, const int64_t* sp_nnz, int32_t sm_budget,
+                             double* terms) {
+  if (!P || !terms) return fail(RAP_ERR_INVALID_ARGUMENT, "NULL argument");
+  if (n_rows < 0 || sm_budget < 0 || sm_budget > P->sm_count) return fail(RAP_ERR_INVALID_ARGUMENT, "bad size");
+  if (n_rows > 0 && P->n_sparse_in > 0 && !sp_nnz) return fail(RAP_ERR_INVALID_ARGUMENT, "sp_nnz NULL");
+  const PredTerms t = predict_terms(P, n_rows, sp_nnz, sm_budget == 0 ? P->sm_count : sm_budget);
+  terms[0] = t.family;
+  terms[1] = (double)t.grid;
+  terms[2] = t.work;
+  terms[3] = t.bytes;
+  terms[4] = t.dwork;
+  terms[5] = t.pairs;
+  return RAP_OK;
+}
+
 rap_status rap_predict_latency_us(const rap_plan* P, int64_t n_rows, const int64_t* sp_nnz, int32_t sm_budget,
                                   double* latency_us) {
   if (!P || !latency_us) return fail(RAP_ERR_INVALID_ARGUMENT, "NULL argument");
-  if (n_rows < 0 || sm_budget < 0 || sm_budget > P->sm_count) return fail(RAP_ERR_INVALID_ARGUMENT, "bad size");
-  const int b = sm_budget == 0 ? P->sm_count : sm_budget;
-  const double bytes = n_rows > 0 ? algorithmic_bytes(P, n_rows, sp_nnz) : 0.0;
-  // Analytic roofline predictor: the fused kernel streams at
-  // HBM bandwidth once ~sat SMs issue loads; fewer SMs get a linear share.
-  const char* env = getenv("RAP_HBM_GBS");
-  const double peak_gbs = env ? atof(env) : 6500.0;
-  const double sat = 0.5 * P->sm_count;
-  const double bw = peak_gbs * 1e9 * std::min(1.0, b / sat);
-  const double launch_us = 5.0;
-  *latency_us = launch_us + bytes / bw * 1e6;
+  double terms[6];
+  rap_status st = rap_predict_terms(P, n_rows, sp_nnz, sm_budget, terms);
+  if (st != RAP_OK) return st;
+  if (n_rows == 0) {
+    *latency_us = 0.0;
+    return RAP_OK;
+  }
+  double k[10];
+  model_constants(k);
+  const int fam = (int)terms[0];
+  const int i = fam == RAP_KERNEL_JIT ? 6 : fam == RAP_KERNEL_ROWS ? 3 : 0;
+  // (the dense work, terms[4], took zero weight in every fit: not modelled)
+  *latency_us = k[i] + k[i + 1] * terms[2] + k[i + 2] * terms[5] + terms[3] / (k[9] * 1e3);
   return RAP_OK;
 }
 

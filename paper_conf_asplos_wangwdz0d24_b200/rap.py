@@ -23,7 +23,7 @@ EXPORTS = ["rap_plan_create", "rap_plan_output_shape", "rap_preprocess", "rap_pr
            "rap_predict_latency_us", "rap_choose_budget", "rap_plan_info_get", "rap_debug_trace", "rap_plan_destroy",
            "rap_status_string", "rap_last_error", "rap_shard_rows", "rap_plan_output_costs", "rap_place",
            "rap_plan_create_sharded", "rap_jagged_append", "rap_set_kernel", "rap_check_overflow",
-           "rap_debug_jit_source", "rap_place_comm"]
+           "rap_debug_jit_source", "rap_place_comm", "rap_predict_terms"]
 PLACE_MODES = {"balanced": 0, "round_robin": 1, "skewed": 2}
 RAP_OUT_CHAIN = 1
 
@@ -122,6 +122,8 @@ def load(build_if_stale: bool = False):
     L.rap_set_budget.argtypes = [P, C.c_int32]
     L.rap_predict_latency_us.restype = C.c_int
     L.rap_predict_latency_us.argtypes = [P, C.c_int64, P, C.c_int32, C.POINTER(C.c_double)]
+    L.rap_predict_terms.restype = C.c_int
+    L.rap_predict_terms.argtypes = [P, C.c_int64, P, C.c_int32, P]
     L.rap_choose_budget.restype = C.c_int
     L.rap_choose_budget.argtypes = [P, C.c_int64, P, C.c_double, C.POINTER(C.c_int32), C.POINTER(C.c_double)]
     L.rap_plan_info_get.restype = C.c_int
@@ -455,6 +457,13 @@ class Plan:
         v = C.c_double()
         _check(load().rap_predict_latency_us(self.handle, n_rows, nnz.ctypes.data, sm_budget, C.byref(v)))
         return v.value
+
+    def predict_terms(self, n_rows, sp_nnz, sm_budget=0):
+        """rap_predict_terms: (kernel, grid, busiest CTA's sparse work, bytes, its dense work, its pairs)."""
+        nnz = np.ascontiguousarray(sp_nnz, dtype=np.int64)
+        t = np.zeros(6, dtype=np.float64)
+        _check(load().rap_predict_terms(self.handle, n_rows, nnz.ctypes.data, sm_budget, t.ctypes.data))
+        return int(t[0]), int(t[1]), float(t[2]), float(t[3]), float(t[4]), float(t[5])
 
     def choose_budget(self, n_rows, sp_nnz, overlap_capacity_us):
         nnz = np.ascontiguousarray(sp_nnz if len(sp_nnz) else [0], dtype=np.int64)

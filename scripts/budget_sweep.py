@@ -28,8 +28,13 @@ def time_plan(plan, sets, steps=50):
 
 def main():
     budgets = [int(b) for b in os.environ.get("BUDGETS", "8,16,37,74,111,148").split(",")]
-    cases = [("c1", synth.c1_kaggle(0), 4096), ("c2", synth.c2_terabyte(0), 65536),
-             ("c2_16k", synth.c2_terabyte(0), 16384), ("c4_16k", synth.c4_multihot(0), 16384)]
+    cases = [("c1", synth.c1_kaggle(0), 4096), ("c1_1k", synth.c1_kaggle(0), 1024),
+             ("c2", synth.c2_terabyte(0), 65536), ("c2_16k", synth.c2_terabyte(0), 16384),
+             ("c2_4k", synth.c2_terabyte(0), 4096), ("c4_16k", synth.c4_multihot(0), 16384),
+             ("c4_4k", synth.c4_multihot(0), 4096)]
+    only = os.environ.get("CASES")
+    if only:
+        cases = [c for c in cases if c[0] in only.split(",")]
     for name, w, B in cases:
         plan = rap.Plan(w.spec, device=0)
         sets = []
@@ -40,11 +45,14 @@ def main():
         nnz = sets[0][0].sp_nnz
         for b in budgets:
             plan.set_budget(b)
-            us = time_plan(plan, sets)
+            us = time_plan(plan, sets, steps=20 if "c4" in name else 50)
             pred = plan.predict_latency_us(B, nnz, b)
+            fam, grid, work, nbytes, dwork, pairs = plan.predict_terms(B, nnz, b)
             info = plan.info()
             print(json.dumps({"workload": name, "B": B, "budget": b, "measured_us": round(us, 2),
-                              "predicted_us": round(pred, 2), "kernel": info["kernel_last"], "grid": info["grid"]}),
+                              "predicted_us": round(pred, 2), "kernel": info["kernel_last"], "grid": info["grid"],
+                              "model_kernel": fam, "model_grid": grid, "work": work, "bytes": nbytes,
+                              "dwork": dwork, "pairs": pairs}),
                   flush=True)
         plan.close()
         del sets
