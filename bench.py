@@ -403,7 +403,7 @@ def run_rap(args):
 
         train = cr.DLRMStep(dev)
         budgets = [int(b) for b in args.corun_budgets.split(",") if b]
-        corun = cr.measure(plan, sets, train, budgets, choose=(B, sets[0][0].sp_nnz))
+        corun = cr.measure(plan, sets, train, budgets, choose=(B, sets[0][0].sp_nnz), partitions=(8, 16, 40))
         corun["training"] = "synthetic DLRM step (DESIGN.md §12): 26 tables x 128 fp32 (TB share at 8 GPUs), batch 8192"
         # layer-aligned scheduling (Algorithm 1): chunks launched as their layers begin
         layer_us = train.layer_times_us()

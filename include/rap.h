@@ -275,6 +275,19 @@ rap_status rap_choose_budget(const rap_plan* plan, int64_t n_rows, const int64_t
 
 rap_status rap_plan_info_get(const rap_plan* plan, rap_plan_info* info);
 
+/* A stream whose kernels run on a dedicated partition of the device's SMs (a
+ * CUDA green context): the SM budget enforced by the hardware instead of by a
+ * CTA-slot cap (§6.2; a capped grid is spread by the block
+ * scheduler over up to ctas_per_sm x budget SMs).  n_sms is rounded up to the
+ * architecture's granularity (sm_100: multiples of 8); *sms_out (HOST, may be
+ * NULL) receives the partition's SM count.  priority as cudaStreamCreateWithPriority.
+ * Launch rap_preprocess on it with the plan's budget set to *sms_out.
+ * RAP_ERR_UNSUPPORTED without driver support.  Destroy with
+ * rap_sm_partition_stream_destroy (after the work on it completed). */
+rap_status rap_sm_partition_stream(int32_t device, int32_t n_sms, int32_t priority, void** stream_out,
+                                   int32_t* sms_out);
+rap_status rap_sm_partition_stream_destroy(void* stream);
+
 /* Select the kernel of the following rap_preprocess calls (RAP_KERNEL_*). */
 rap_status rap_set_kernel(rap_plan* plan, int32_t mode);
 

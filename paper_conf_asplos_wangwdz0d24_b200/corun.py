@@ -105,7 +105,7 @@ class DLRMStep:
         return {n: float(np.median(v[2:])) for n, v in per.items()}
 
 
-def measure(plan, sets, train: DLRMStep, budgets, steps=20, warmup=5, choose=None):
+def measure(plan, sets, train: DLRMStep, budgets, steps=20, warmup=5, choose=None, partitions=()):
     """Per budget: training step alone vs co-run with one preprocessing launch
     per step (events on each stream), in ms, and the slowdown.  choose =
     (n_rows, sp_nnz): also the budget rap_choose_budget picks for an overlap
@@ -117,7 +117,7 @@ def measure(plan, sets, train: DLRMStep, budgets, steps=20, warmup=5, choose=Non
     lo = torch.cuda.Stream(priority=0)   # preprocessing: lowest
     ev = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
 
-    def run(k, with_prep, with_train=True):
+    def run(k, with_prep, with_train=True, lo=lo):
         t_train, t_prep = [], []
         for i in range(k):
             r, o = sets[i % len(sets)]
@@ -163,6 +163,21 @@ def measure(plan, sets, train: DLRMStep, budgets, steps=20, warmup=5, choose=Non
                                   "prep_hidden": p <= t, "chosen": chosen is not None and b == chosen["sm_budget"]})
         if chosen is not None and b == chosen["sm_budget"]:
             chosen.update({"measured_prep_alone_us": prep_alone * 1e3, "slowdown": t / alone - 1.0})
+    # the same launches on a green-context SM partition (rap_sm_partition_stream):
+    # the budget enforced by the hardware, not by the grid size
+    from . import rap
+
+    res["partition"] = []
+    for b in partitions:
+        part = rap.SMPartitionStream(torch.cuda.current_device(), b, priority=0)
+        plan.set_budget(part.sms)
+        run(warmup, True, lo=part.stream)
+        _, prep_alone = run(steps, True, with_train=False, lo=part.stream)
+        t, p = run(steps, True, lo=part.stream)
+        res["partition"].append({"requested_sms": b, "partition_sms": part.sms, "train_step_corun_ms": t,
+                                 "prep_corun_ms": p, "prep_alone_ms": prep_alone, "slowdown": t / alone - 1.0,
+                                 "prep_hidden": p <= t})
+        part.close()
     plan.set_budget(0)
     return res
 

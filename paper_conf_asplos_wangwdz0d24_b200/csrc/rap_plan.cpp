@@ -6,6 +6,7 @@
 // tables, size the (feature, row-range) descriptor geometry and the grid from
 // the SM budget (resource-aware sharding, L1351-1366 §6.2).  rap_preprocess
 // = row a1: one launch, no host sync.
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <math.h>
 #include <stdint.h>
@@ -16,6 +17,8 @@
 #include <cstdio>
 #include <cstdlib>
 #include <limits>
+#include <map>
+#include <mutex>
 #include <numeric>
 #include <string>
 #include <utility>
@@ -2258,3 +2261,99 @@ rap_status rap_jagged_append(const int32_t* lengths, const int64_t* src_offsets,
   if (rc != 0) return cuda_fail((cudaError_t)rc, "jagged append launch");
   return RAP_OK;
 }
+
+// ----------------------------------------------------------------------------
+// SM partition (green context, include/rap.h): a stream whose kernels run on
+// a dedicated set of SMs (§6.2 L1351-1366 resource-aware sharding,
+// enforced by the hardware partition rather than by a CTA-slot cap).  The
+// driver entry points are fetched at run time (no libcuda link dependency).
+namespace {
+struct GreenApi {
+  CUresult (*get_dev)(CUdevice*, int) = nullptr;
+  CUresult (*get_res)(CUdevice, CUdevResource*, CUdevResourceType) = nullptr;
+  CUresult (*split)(CUdevResource*, unsigned int*, const CUdevResource*, CUdevResource*, unsigned int,
+                    unsigned int) = nullptr;
+  CUresult (*gen_desc)(CUdevResourceDesc*, CUdevResource*, unsigned int) = nullptr;
+  CUresult (*create)(CUgreenCtx*, CUdevResourceDesc, CUdevice, unsigned int) = nullptr;
+  CUresult (*destroy)(CUgreenCtx) = nullptr;
+  CUresult (*stream_create)(CUstream*, CUgreenCtx, unsigned int, int) = nullptr;
+  CUresult (*stream_destroy)(CUstream) = nullptr;
+  bool ok = false;
+};
+const GreenApi& green_api() {
+  static GreenApi g;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    auto get = [](const char* name, void** fn) {
+      cudaDriverEntryPointQueryResult q;
+      return cudaGetDriverEntryPoint(name, fn, cudaEnableDefault, &q) == cudaSuccess &&
+             q == cudaDriverEntryPointSuccess && *fn != nullptr;
+    };
+    g.ok = get("cuDeviceGet", reinterpret_cast<void**>(&g.get_dev)) &&
+           get("cuDeviceGetDevResource", reinterpret_cast<void**>(&g.get_res)) &&
+           get("cuDevSmResourceSplitByCount", reinterpret_cast<void**>(&g.split)) &&
+           get("cuDevResourceGenerateDesc", reinterpret_cast<void**>(&g.gen_desc)) &&
+           get("cuGreenCtxCreate", reinterpret_cast<void**>(&g.create)) &&
+           get("cuGreenCtxDestroy", reinterpret_cast<void**>(&g.destroy)) &&
+           get("cuGreenCtxStreamCreate", reinterpret_cast<void**>(&g.stream_create)) &&
+           get("cuStreamDestroy", reinterpret_cast<void**>(&g.stream_destroy));
+  });
+  return g;
+}
+std::mutex g_green_mu;
+std::map<void*, CUgreenCtx>* g_green = nullptr;  // stream -> its green context
+}  // namespace
+
+extern "C" {
+
+rap_status rap_sm_partition_stream(int32_t device, int32_t n_sms, int32_t priority, void** stream_out,
+                                   int32_t* sms_out) {
+  if (!stream_out || n_sms < 1) return fail(RAP_ERR_INVALID_ARGUMENT, "stream_out NULL or n_sms < 1");
+  *stream_out = nullptr;
+  const GreenApi& g = green_api();
+  if (!g.ok) return fail(RAP_ERR_UNSUPPORTED, "green-context driver entry points unavailable");
+  DeviceGuard dg(device);
+  cudaFree(nullptr);  // the runtime's primary context exists (driver initialised)
+  CUdevice dev;
+  if (g.get_dev(&dev, device) != CUDA_SUCCESS) return fail(RAP_ERR_CUDA, "cuDeviceGet");
+  CUdevResource all, part, rest;
+  if (g.get_res(dev, &all, CU_DEV_RESOURCE_TYPE_SM) != CUDA_SUCCESS) return fail(RAP_ERR_CUDA, "cuDeviceGetDevResource");
+  if ((unsigned)n_sms >= all.sm.smCount) return fail(RAP_ERR_INVALID_ARGUMENT, "n_sms >= the device's SMs");
+  unsigned int groups = 1;
+  // one group of at least n_sms SMs (sm_100: multiples of 8, at least 8)
+  if (g.split(&part, &groups, &all, &rest, 0, (unsigned)n_sms) != CUDA_SUCCESS || groups < 1)
+    return fail(RAP_ERR_CUDA, "cuDevSmResourceSplitByCount");
+  CUdevResourceDesc desc;
+  if (g.gen_desc(&desc, &part, 1) != CUDA_SUCCESS) return fail(RAP_ERR_CUDA, "cuDevResourceGenerateDesc");
+  CUgreenCtx gctx;
+  if (g.create(&gctx, desc, dev, CU_GREEN_CTX_DEFAULT_STREAM) != CUDA_SUCCESS) return fail(RAP_ERR_CUDA, "cuGreenCtxCreate");
+  CUstream st;
+  if (g.stream_create(&st, gctx, CU_STREAM_NON_BLOCKING, priority) != CUDA_SUCCESS) {
+    g.destroy(gctx);
+    return fail(RAP_ERR_CUDA, "cuGreenCtxStreamCreate");
+  }
+  {
+    std::lock_guard<std::mutex> lk(g_green_mu);
+    if (!g_green) g_green = new std::map<void*, CUgreenCtx>();
+    (*g_green)[reinterpret_cast<void*>(st)] = gctx;
+  }
+  *stream_out = reinterpret_cast<void*>(st);
+  if (sms_out) *sms_out = (int32_t)part.sm.smCount;
+  return RAP_OK;
+}
+
+rap_status rap_sm_partition_stream_destroy(void* stream) {
+  const GreenApi& g = green_api();
+  CUgreenCtx gctx = nullptr;
+  {
+    std::lock_guard<std::mutex> lk(g_green_mu);
+    if (!g_green || !g_green->count(stream)) return fail(RAP_ERR_INVALID_ARGUMENT, "not a partition stream");
+    gctx = (*g_green)[stream];
+    g_green->erase(stream);
+  }
+  g.stream_destroy(reinterpret_cast<CUstream>(stream));
+  g.destroy(gctx);
+  return RAP_OK;
+}
+
+}  // extern "C"

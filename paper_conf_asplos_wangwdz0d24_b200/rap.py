@@ -23,7 +23,8 @@ EXPORTS = ["rap_plan_create", "rap_plan_output_shape", "rap_preprocess", "rap_pr
            "rap_predict_latency_us", "rap_choose_budget", "rap_plan_info_get", "rap_debug_trace", "rap_plan_destroy",
            "rap_status_string", "rap_last_error", "rap_shard_rows", "rap_plan_output_costs", "rap_place",
            "rap_plan_create_sharded", "rap_jagged_append", "rap_set_kernel", "rap_check_overflow",
-           "rap_debug_jit_source", "rap_place_comm", "rap_predict_terms"]
+           "rap_debug_jit_source", "rap_place_comm", "rap_predict_terms", "rap_sm_partition_stream",
+           "rap_sm_partition_stream_destroy"]
 PLACE_MODES = {"balanced": 0, "round_robin": 1, "skewed": 2}
 RAP_OUT_CHAIN = 1
 
@@ -124,6 +125,10 @@ def load(build_if_stale: bool = False):
     L.rap_predict_latency_us.argtypes = [P, C.c_int64, P, C.c_int32, C.POINTER(C.c_double)]
     L.rap_predict_terms.restype = C.c_int
     L.rap_predict_terms.argtypes = [P, C.c_int64, P, C.c_int32, P]
+    L.rap_sm_partition_stream.restype = C.c_int
+    L.rap_sm_partition_stream.argtypes = [C.c_int32, C.c_int32, C.c_int32, C.POINTER(P), C.POINTER(C.c_int32)]
+    L.rap_sm_partition_stream_destroy.restype = C.c_int
+    L.rap_sm_partition_stream_destroy.argtypes = [P]
     L.rap_choose_budget.restype = C.c_int
     L.rap_choose_budget.argtypes = [P, C.c_int64, P, C.c_double, C.POINTER(C.c_int32), C.POINTER(C.c_double)]
     L.rap_plan_info_get.restype = C.c_int
@@ -471,6 +476,25 @@ class Plan:
         _check(load().rap_choose_budget(self.handle, n_rows, nnz.ctypes.data, overlap_capacity_us, C.byref(b),
                                         C.byref(td)))
         return b.value, td.value
+
+
+class SMPartitionStream:
+    """rap_sm_partition_stream: a CUDA stream (torch.cuda.ExternalStream) on a
+    green-context partition of n_sms SMs (rounded up by the driver)."""
+
+    def __init__(self, device: int, n_sms: int, priority: int = 0):
+        import torch
+
+        h, n = C.c_void_p(), C.c_int32()
+        _check(load().rap_sm_partition_stream(device, n_sms, priority, C.byref(h), C.byref(n)))
+        self.handle, self.sms = h.value, n.value
+        self.stream = torch.cuda.ExternalStream(self.handle, device=torch.device("cuda", device))
+
+    def close(self):
+        if self.handle:
+            self.stream.synchronize()
+            _check(load().rap_sm_partition_stream_destroy(self.handle))
+            self.handle = None
 
 
 def jit_source(spec, compile: bool = False):
