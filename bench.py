@@ -29,7 +29,8 @@ sys.path.insert(0, ROOT)
 
 METRIC = "preprocessed samples/s"
 UNIT = "samples/s"
-WORKLOADS = {"c2": ("criteo_terabyte_c2", 65536), "c1": ("criteo_kaggle_c1", 4096), "c4": ("multihot_c4", 131072)}
+WORKLOADS = {"c2": ("criteo_terabyte_c2", 65536), "c1": ("criteo_kaggle_c1", 4096), "c4": ("multihot_c4", 131072),
+             "plan2": ("table3_plan2", 65536), "plan3": ("table3_plan3", 65536)}
 
 
 def parse():
@@ -54,6 +55,7 @@ def parse():
     ap.add_argument("--imbalance-tol", type=float, default=0.10, help="N>1: residual move threshold")
     ap.add_argument("--no-c4", action="store_true", help="skip the config-4 (multi-hot) sub-measurement")
     ap.add_argument("--c4-batch", type=int, default=16384, help="rows of the config-4 sub-measurement")
+    ap.add_argument("--no-plans", action="store_true", help="skip the Table 3 Plan 2 / 3 sub-measurements")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="N>1: gloo = host-staged exchange (ranks sharing one GPU: tests)")
     return ap.parse_args()
@@ -66,6 +68,8 @@ def workload(name, seed=0):
         return synth.c2_terabyte(seed)
     if name == "c1":
         return synth.c1_kaggle(seed)
+    if name in ("plan2", "plan3"):
+        return synth.plan_graph(int(name[-1]), seed)
     return synth.c4_multihot(seed)
 
 
@@ -397,6 +401,7 @@ def run_rap(args):
     fusion = None
     if world == 1 and not args.no_fusion and not args.profile and args.workload in ("c1", "c2"):
         fusion = fusion_ablation(w, sets, B, dev, stream, kern_ms, steps=min(K, 200))
+        fusion["perop"] = perop_baseline(w, first, dev, kern_ms)
     corun = None
     if world == 1 and not args.no_corun and not args.profile and args.workload == "c2":
         from paper_conf_asplos_wangwdz0d24_b200 import corun as cr
@@ -424,6 +429,9 @@ def run_rap(args):
     c4 = None
     if world == 1 and not args.profile and not args.no_c4 and args.workload != "c4":
         c4 = c4_point(dev, args.c4_batch, steps=20)
+    plans = None
+    if world == 1 and not args.profile and not args.no_plans and args.workload in ("c1", "c2"):
+        plans = [plan_point(dev, p, 65536) for p in (2, 3)]
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": args.warmup,
                 "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
@@ -437,7 +445,7 @@ def run_rap(args):
                            "l2_policy": f"rotate {nsets} distinct input/output sets, {nsets * set_bytes / 2**20:.0f} MB "
                                         f"total vs L2 {l2 / 2**20:.0f} MB"},
                 "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks, "gpu_launches": K,
-                "corun": corun, "fusion": fusion, "graph": graph, "c4": c4}
+                "corun": corun, "fusion": fusion, "graph": graph, "c4": c4, "plans": plans}
         print(json.dumps(line), flush=True)
     plan.close()
     if world > 1:
@@ -488,6 +496,74 @@ def c4_point(dev, B, steps=20):
             "alg_bytes_per_launch": int(alg), "achieved_gbs": gbs, "frac": gbs / peak,
             "kernel": KERNEL_NAMES.get(info["kernel_last"], str(info["kernel_last"])),
             "note": f"config 4 at {B} of its 131072 rows (host generation of the full batch is ~20 GB)"}
+
+
+def perop_baseline(w, host, dev, kern_ms, steps=10):
+    """The paper's Sequential arm on this GPU (baselines/perop_torch.py): every
+    graph node as its own eager PyTorch operation(s), intermediates in HBM;
+    inputs resident, CUDA events around whole-graph evaluations."""
+    import torch
+
+    from baselines.perop_torch import PerOpGraph
+
+    g = PerOpGraph(w.spec, dev)
+    b = g.upload(host)
+    for _ in range(2):
+        g.run(b)
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(steps):
+        g.run(b)
+    e1.record()
+    e1.synchronize()
+    ms = e0.elapsed_time(e1) / steps
+    del b
+    torch.cuda.empty_cache()
+    return {"ms_per_step": ms, "fused_speedup": ms / kern_ms,
+            "note": "one eager PyTorch evaluation per graph node (TorchArrow-style), same batch, "
+                    "outputs equal to the oracle (tests/test_perop_baseline.py)"}
+
+
+def plan_point(dev, plan_id, B, steps=20):
+    """Table 3 Plan 2 / Plan 3-shaped graph (synth.plan_graph, 384 / 1548 ops)
+    at B rows: kernel time (AUTO kernel choice), HBM fraction of the launch."""
+    import torch
+
+    from paper_conf_asplos_wangwdz0d24_b200 import rap, synth
+
+    w = synth.plan_graph(plan_id, 0)
+    plan = rap.Plan(w.spec, device=dev.index)
+    sets = []
+    for i in range(2):
+        h = synth.make_batch(w, B, seed=800 + i)
+        r = rap.DeviceBatch(h, dev)
+        sets.append((h, r, rap.DeviceOutput(plan, B, r.sp_nnz, dev)))
+    stream = torch.cuda.current_stream(dev)
+    for i in range(4):
+        plan.preprocess(sets[i % 2][1], sets[i % 2][2], stream)
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for i in range(steps):
+        plan.preprocess(sets[i % 2][1], sets[i % 2][2], stream)
+    e1.record(stream)
+    e1.synchronize()
+    ms = e0.elapsed_time(e1) / steps
+    last = sets[(steps - 1) % 2]
+    n_vals = int(last[2].offsets[-1].item())
+    alg = synth.algorithmic_bytes(w.spec, last[0], n_vals)
+    peak, _ = measured_peaks()
+    info = plan.info()
+    d_out, f_out = synth.output_dims(w.spec)
+    plan.close()
+    del sets
+    torch.cuda.empty_cache()
+    gbs = alg / (ms / 1e3) / 1e9
+    return {"workload": w.name, "graph_ops": len(w.spec["nodes"]), "dense_out_cols": d_out,
+            "sparse_out_features": f_out, "batch": B, "kernel_ms": ms, "value": B / (ms / 1e3), "unit": UNIT,
+            "alg_bytes_per_launch": int(alg), "achieved_gbs": gbs, "frac": gbs / peak,
+            "kernel": KERNEL_NAMES.get(info["kernel_last"], str(info["kernel_last"]))}
 
 
 def graph_replay(plan, sets, B, dev, steps, alg_bytes):

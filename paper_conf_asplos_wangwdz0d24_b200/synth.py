@@ -248,7 +248,102 @@ def c4_multihot(seed: int = 0, n_features: int = 512, mean_len: float = 20.0, fi
     return Workload("multihot_c4", spec, [], M.copy(), sparse_mean=mu, multi_null=0.05)
 
 
-WORKLOADS = {"c1": c1_kaggle, "c2": c2_terabyte, "c4": c4_multihot}
+# Table 3 (L1616-1621): (dense, sparse) input features and total ops.  Plan 3's
+# "9.80 ops/feature" and "1548 ops" disagree (156 x 9.80 = 1528.8, reading
+# R18); the generator builds 1548.
+PLAN_SHAPES = {2: (26, 52, 384), 3: (52, 104, 1548)}
+
+
+def plan_graph(plan: int, seed: int = 0) -> Workload:
+    """Table 3 Plan 2 / Plan 3-shaped op graph (NEXT-4): the config-2 recipe
+    scaled to the plan's features, extended until it has exactly the plan's
+    op count.  Base chains: dense FillNull -> Logit | BoxCox; sparse FillNull
+    -> Clamp -> SigridHash -> FirstX(1).  Extras, added round robin: MapId
+    before a SigridHash, Bucketize after it, an NGram over three hashed
+    sources, a dense Bucketize -> OneHot(16), and a re-hash (Clamp ->
+    SigridHash) deepening a sparse chain (not the canonical stage order: the
+    kernels' generic paths)."""
+    n_dense, n_sparse, n_ops = PLAN_SHAPES[plan]
+    lambdas = [0.0, 0.25, 0.5, -0.5]
+    mapid = [False] * n_sparse
+    bucket = [False] * n_sparse
+    rehash = [0] * n_sparse
+    onehot = [0] * n_dense
+    ngrams = []
+    remaining = n_ops - (2 * n_dense + 4 * n_sparse)
+    i = 0
+    while remaining > 0:
+        kind = i % 5
+        s, d = (i * 7) % n_sparse, (i * 3) % n_dense
+        if kind == 0 and not mapid[s]:
+            mapid[s] = True
+            remaining -= 1
+        elif kind == 1 and not bucket[s]:
+            bucket[s] = True
+            remaining -= 1
+        elif kind == 2:
+            ngrams.append([s, (s + 1) % n_sparse, (s + 5) % n_sparse])
+            remaining -= 1
+        elif kind == 3 and remaining >= 2 and onehot[d] < 1 and d % 4 == 3:
+            onehot[d] += 1
+            remaining -= 2
+        elif kind == 4 and remaining >= 2 and rehash[s] < 6:
+            rehash[s] += 1
+            remaining -= 2
+        i += 1
+    nodes, outs_dense, outs_vec, outs_sparse = [], [], [], []
+    for c in range(n_dense):
+        nodes.append(_n("fillnull", [("d", c)], f_fill=0.0))
+        f = len(nodes) - 1
+        if c % 2 == 0:
+            nodes.append(_n("logit", [("n", f)], eps=1e-6))
+        else:
+            nodes.append(_n("boxcox", [("n", f)], **{"lambda": lambdas[(c // 2) % 4]}))
+        outs_dense.append(len(nodes) - 1)
+        for k in range(onehot[c]):
+            nodes.append(_n("bucketize", [("n", f)], borders=(DENSE_BORDERS * (1 + k)).astype(np.float32)))
+            nodes.append(_n("onehot", [("n", len(nodes) - 1)], k=16))
+            outs_vec.append(len(nodes) - 1)
+    M = cardinalities(seed, n_sparse, TB_TOTAL)
+    sl = salts(seed, n_sparse, f"plan{plan}_salt")
+    hashed = {}
+    for s in range(n_sparse):
+        nodes.append(_n("fillnull", [("s", s)], i_fill=0))
+        nodes.append(_n("clamp", [("n", len(nodes) - 1)], lo=0, hi=2**32 - 1))
+        if mapid[s]:
+            keys = raw_id(np.arange(1, 1025), s)
+            nodes.append(_n("mapid", [("n", len(nodes) - 1)], keys=keys, vals=np.arange(1, 1025, dtype=np.int64),
+                            map_default=0))
+        nodes.append(_n("sigridhash", [("n", len(nodes) - 1)], salt=sl[s], max_value=int(M[s])))
+        hashed[s] = len(nodes) - 1
+        for r in range(rehash[s]):
+            nodes.append(_n("clamp", [("n", len(nodes) - 1)], lo=0, hi=max(int(M[s]) - 1 - r, 0)))
+            nodes.append(_n("sigridhash", [("n", len(nodes) - 1)], salt=sl[s] ^ (r + 1), max_value=int(M[s])))
+        if bucket[s]:
+            borders = np.unique(np.floor(np.logspace(0, math.log10(max(int(M[s]), 2)), 256))).astype(np.int64)
+            nodes.append(_n("bucketize", [("n", len(nodes) - 1)], borders=borders))
+        nodes.append(_n("firstx", [("n", len(nodes) - 1)], x=1))
+        outs_sparse.append(len(nodes) - 1)
+    ng_salts = salts(seed, max(len(ngrams), 1), f"plan{plan}_ngram")
+    for g, srcs in enumerate(ngrams):
+        nodes.append(_n("ngram", [("n", hashed[x]) for x in srcs], n=3, salt=ng_salts[g], max_value=10_000_000))
+        outs_sparse.append(len(nodes) - 1)
+    assert len(nodes) == n_ops, (len(nodes), n_ops)
+    spec = {"n_dense": n_dense, "n_sparse": n_sparse, "nodes": nodes,
+            "outputs": outs_dense + outs_vec + outs_sparse}
+    kinds = ["unit" if c % 2 == 0 else "count" for c in range(n_dense)]
+    return Workload(f"table3_plan{plan}", spec, kinds, M.copy())
+
+
+def plan2(seed: int = 0) -> Workload:
+    return plan_graph(2, seed)
+
+
+def plan3(seed: int = 0) -> Workload:
+    return plan_graph(3, seed)
+
+
+WORKLOADS = {"c1": c1_kaggle, "c2": c2_terabyte, "c4": c4_multihot, "plan2": plan2, "plan3": plan3}
 
 
 # ----------------------------------------------------------------------------- raw batches

@@ -383,3 +383,16 @@ def test_random_graphs(env, seed):
     sparse = [synth.sparse_column(seed, sc, 5000, B, means[sc], null_p=0.15, null_segments=(sc == 2),
                                   base_offset=sc) for sc in range(n_sparse)]
     check(env, s, batch(B, dense=dense, sparse=sparse))
+
+
+@pytest.mark.parametrize("plan_id", [2, 3])
+def test_table3_plan_graphs(env, plan_id, kernel_mode):
+    """Table 3 Plan 2 (26 dense / 52 sparse features, 384 ops) and Plan 3
+    (52 / 104, 1548 ops) shaped graphs (synth.plan_graph): deep non-canonical
+    chains, hundreds of NGram outputs, > 64 raw sparse columns (Plan 3: the
+    tiled kernel's large template only), ragged batch."""
+    _, synth, _, _ = env
+    if plan_id == 3 and kernel_mode != 1:
+        pytest.skip("Plan 3 reads 104 raw sparse columns: the row-block kernels take <= 64")
+    w = synth.plan_graph(plan_id, 0)
+    check(env, w.spec, synth.make_batch(w, 1111, seed=plan_id))
