@@ -152,6 +152,24 @@ def traffic_from_profile(workload_name):
         return None
 
 
+def issue_roofline(workload_name, kern_ms):
+    """The instruction-issue roofline of the same kernel from the committed ncu
+    capture (profiles/issue.json): its warp instructions at one issue per
+    SMSP per cycle (148 SMs x 4 SMSPs at the max SM clock) against the
+    measured time -- the limiter when the HBM fraction is low."""
+    p = os.path.join(ROOT, "profiles", "issue.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)[workload_name]
+    except Exception:  # noqa: BLE001
+        return None
+    ideal_ms = d["warp_inst_per_launch"] / (148 * 4 * 1.965e9) * 1e3
+    return {"warp_inst_per_launch": d["warp_inst_per_launch"], "ideal_issue_ms": ideal_ms,
+            "frac": ideal_ms / kern_ms, "ncu_issue_active_pct": d["issue_active_pct"],
+            "ncu_warps_active_pct": d["warps_active_pct"], "source": d.get("summary"),
+            "limiter": "latency: few resident warps, dependent id-load -> probe -> hash -> store chains"}
+
+
 def cpu_model():
     try:
         with open("/proc/cpuinfo") as f:
@@ -386,7 +404,10 @@ def run_rap(args):
     traffic = traffic_from_profile(wname)
     roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
             "traffic": traffic, "peak_source": peak_kind, "alg_bytes_per_launch": int(alg_bytes),
-            "kernel_ms": kern_ms}
+            "kernel_ms": kern_ms,
+            "traffic_note": "dram read+write of the committed ncu --set full capture (profiles/traffic.json); "
+                            "output lines still dirty in the 126 MB L2 at kernel end are not counted",
+            "issue": issue_roofline(wname, kern_ms)}
     clocks = sampler.summary() if sampler else None
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline and not args.profile:
@@ -412,16 +433,15 @@ def run_rap(args):
         corun["training"] = "synthetic DLRM step (DESIGN.md §12): 26 tables x 128 fp32 (TB share at 8 GPUs), batch 8192"
         # layer-aligned scheduling (Algorithm 1): chunks launched as their layers begin
         layer_us = train.layer_times_us()
-        alone = corun["train_step_alone_ms"]
         corun["layer_aligned"] = {"layer_us": layer_us, "per_budget": []}
         lsets = [r for r, _ in sets[:2]]
         for lb in (0, 8, 2):
             lap = cr.LayerAlignedPrep(w.spec, B, sets[0][0].sp_nnz, layer_us, device=dev.index, budget=lb)
             louts = [lap.output(r.sp_nnz, dev) for r in lsets]
-            t_l, p_l = cr.measure_layer_aligned(lap, lsets, louts, train)
+            t_l, p_l, a_l = cr.measure_layer_aligned(lap, lsets, louts, train)
             corun["layer_aligned"]["per_budget"].append(
-                {"pack_budget": lb, "chunks": lap.describe(), "train_step_corun_ms": t_l, "prep_done_ms": p_l,
-                 "slowdown": t_l / alone - 1.0, "prep_hidden": p_l <= t_l})
+                {"pack_budget": lb, "chunks": lap.describe(), "train_step_alone_ms": a_l, "train_step_corun_ms": t_l,
+                 "prep_done_ms": p_l, "slowdown": t_l / a_l - 1.0, "prep_hidden": p_l <= t_l})
             lap.close()
             del louts
         del train

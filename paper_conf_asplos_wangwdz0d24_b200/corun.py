@@ -153,16 +153,27 @@ def measure(plan, sets, train: DLRMStep, budgets, steps=20, warmup=5, choose=Non
         res["chosen"] = chosen
         if b not in budgets:
             budgets.append(b)
+    def paired(lo_stream=lo):
+        """Training alone and co-run measured in alternating rounds (medians),
+        so clock / thermal drift over the sweep cancels in the slowdown."""
+        ta, tc, pc = [], [], []
+        for _ in range(4):
+            ta.append(run(max(steps // 4, 3), False)[0])
+            t_, p_ = run(max(steps // 4, 3), True, lo=lo_stream)
+            tc.append(t_)
+            pc.append(p_)
+        return float(np.median(ta)), float(np.median(tc)), float(np.median(pc))
+
     for b in budgets:
         plan.set_budget(b)
         run(warmup, True)
         _, prep_alone = run(steps, True, with_train=False)
-        t, p = run(steps, True)
-        res["per_budget"].append({"sm_budget": b, "train_step_corun_ms": t, "prep_corun_ms": p,
-                                  "prep_alone_ms": prep_alone, "slowdown": t / alone - 1.0,
+        alone_b, t, p = paired()
+        res["per_budget"].append({"sm_budget": b, "train_step_alone_ms": alone_b, "train_step_corun_ms": t,
+                                  "prep_corun_ms": p, "prep_alone_ms": prep_alone, "slowdown": t / alone_b - 1.0,
                                   "prep_hidden": p <= t, "chosen": chosen is not None and b == chosen["sm_budget"]})
         if chosen is not None and b == chosen["sm_budget"]:
-            chosen.update({"measured_prep_alone_us": prep_alone * 1e3, "slowdown": t / alone - 1.0})
+            chosen.update({"measured_prep_alone_us": prep_alone * 1e3, "slowdown": t / alone_b - 1.0})
     # the same launches on a green-context SM partition (rap_sm_partition_stream):
     # the budget enforced by the hardware, not by the grid size
     from . import rap
@@ -173,9 +184,10 @@ def measure(plan, sets, train: DLRMStep, budgets, steps=20, warmup=5, choose=Non
         plan.set_budget(part.sms)
         run(warmup, True, lo=part.stream)
         _, prep_alone = run(steps, True, with_train=False, lo=part.stream)
-        t, p = run(steps, True, lo=part.stream)
-        res["partition"].append({"requested_sms": b, "partition_sms": part.sms, "train_step_corun_ms": t,
-                                 "prep_corun_ms": p, "prep_alone_ms": prep_alone, "slowdown": t / alone - 1.0,
+        alone_b, t, p = paired(part.stream)
+        res["partition"].append({"requested_sms": b, "partition_sms": part.sms, "train_step_alone_ms": alone_b,
+                                 "train_step_corun_ms": t, "prep_corun_ms": p, "prep_alone_ms": prep_alone,
+                                 "slowdown": t / alone_b - 1.0,
                                  "prep_hidden": p <= t})
         part.close()
     plan.set_budget(0)
@@ -268,7 +280,19 @@ class LayerAlignedPrep:
 def measure_layer_aligned(lap: LayerAlignedPrep, sets_raw, outs, train: DLRMStep, steps=20, warmup=5):
     """Training step co-run with the layer-aligned chunks: each chunk's launch
     on the low-priority stream waits for an event recorded when its layer
-    begins on the training stream."""
+    begins on the training stream.  Returns (co-run step, preprocessing done,
+    the step alone measured in alternating rounds), medians in ms."""
+    import torch
+
+    rounds = [(_measure_la(lap, sets_raw, outs, train, max(steps // 4, 3), warmup if r == 0 else 1, False),
+               _measure_la(lap, sets_raw, outs, train, max(steps // 4, 3), 1, True)) for r in range(4)]
+    alone = float(np.median([a[0] for a, _ in rounds]))
+    t = float(np.median([c[0] for _, c in rounds]))
+    p = float(np.median([c[1] for _, c in rounds]))
+    return t, p, alone
+
+
+def _measure_la(lap, sets_raw, outs, train, steps, warmup, with_prep):
     import torch
 
     hi = torch.cuda.Stream(priority=-1)
@@ -282,7 +306,7 @@ def measure_layer_aligned(lap: LayerAlignedPrep, sets_raw, outs, train: DLRMStep
         torch.cuda.synchronize()
 
         def hook(name):
-            if name is None or not any(c["layer"] == name for c in lap.chunks):
+            if not with_prep or name is None or not any(c["layer"] == name for c in lap.chunks):
                 return
             e = torch.cuda.Event()
             e.record(hi)

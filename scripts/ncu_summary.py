@@ -27,7 +27,7 @@ def main():
     txt = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(txt)))
     hdr, units, data = rows[0], rows[1], rows[2:]
-    lines = [f"ncu --set full summary of {os.path.basename(rep)} ({len(data)} launch(es) of rap_fused_kernel)"]
+    lines = [f"ncu --set full summary of {os.path.basename(rep)} ({len(data)} launch(es) of the captured kernel)"]
     vals = {}
     for k in KEYS:
         if k in hdr:
@@ -49,6 +49,14 @@ def main():
         d = json.load(open(p)) if os.path.exists(p) else {}
         d[wl] = int(r + w)
         json.dump(d, open(p, "w"), indent=1)
+        # the issue roofline of the same capture (bench.py roofline.issue)
+        q = os.path.join(root, "profiles", "issue.json")
+        e = json.load(open(q)) if os.path.exists(q) else {}
+        e[wl] = {"warp_inst_per_launch": float(vals["smsp__inst_executed.sum"][0]),
+                 "issue_active_pct": float(vals["smsp__issue_active.avg.pct_of_peak_sustained_active"][0]),
+                 "warps_active_pct": float(vals["sm__warps_active.avg.pct_of_peak_sustained_active"][0]),
+                 "ncu_us": float(vals["gpu__time_duration.sum"][0]), "summary": "profiles/" + os.path.basename(out)}
+        json.dump(e, open(q, "w"), indent=1)
     except Exception as e:  # noqa: BLE001
         print("traffic not recorded:", e)
 
