@@ -475,6 +475,15 @@ __device__ __forceinline__ void trace_stamp(const Common& c, int k) {
   }
 }
 
+// Same, from lane 0 of the calling warp (a warp other than warp 0).
+__device__ __forceinline__ void trace_stamp_warp(const Common& c, int k) {
+  if (c.trace != nullptr && (threadIdx.x & 31) == 0 && (int64_t)blockIdx.x < c.trace_cap) {
+    unsigned long long v;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(v));
+    c.trace[(int64_t)blockIdx.x * kTracePts + k] = v;
+  }
+}
+
 // Profiling aid: clock64 at slot k of this CTA's trace row, once per launch
 // (first call wins), after the value `dep` is available.
 // Compiled in only with -DRAP_TRACE_CLK (dev builds, scripts/trace.py).

@@ -244,6 +244,7 @@ constexpr int kRbMaxFL = 64;    // sparse outputs per feature group
 constexpr int kRbMaxF = 1024;   // sparse outputs of a plan the row-block kernel takes
 constexpr int kRbMaxCols = 64;  // raw sparse columns the row-block kernel addresses
 constexpr int kRbMaxDense = 32; // raw dense columns
+constexpr int kRbIdCap = 232;   // staged ids per column and chunk (224 rows of single ids + 16-byte head/tail)
 
 // Per sparse output (indexed by output f): its closed-form length program
 // (R5, R7, R10, R14 from the Arrow offsets and validity bits of up to
@@ -274,6 +275,8 @@ struct RbGeom {
   int32_t len_cache;                    // 1: the kernel keeps a uint16 length cache per (output, row) in smem
   int32_t n_dcta;                       // dedicated dense CTAs after the n_rb x n_fg sparse ones (0: dense
                                         // blocks round robin over every CTA)
+  int32_t id_slots;                     // staged columns (slots < id_slots) whose chunk ids are bulk-copied
+                                        // into shared memory (generated kernel; 0: ids read from global)
   unsigned long long all_cols;          // raw sparse columns the outputs read (bit c: column c < 64)
   const RbFeat* feat;                   // [n_sparse_out], by output index
   const int32_t* perm;                  // [n_sparse_out] processing order (groups are ranges of it)
@@ -303,7 +306,8 @@ int ensure_dyn_smem(const void* kernel, int smem);
 // Occupancy query: CTAs per SM for the given dynamic smem.
 int fused_occupancy(int smem_bytes, int n_dense, int n_sparse, int* ctas_per_sm);
 // Row-block kernel (rap_rows.cu): dynamic smem for a geometry, occupancy, launch.
-int rows_smem_bytes(int dense_bytes, int max_fl, int max_cols, int n_memo, int n_sparse_out, int len_cache);
+int rows_smem_bytes(int dense_bytes, int max_fl, int max_cols, int n_memo, int n_sparse_out, int len_cache,
+                    int id_slots = 0);
 // Dense-phase shared memory of the row-block kernel for dense groups up to max_width columns.
 int rows_dense_bytes(int max_width);
 int rows_occupancy(int smem_bytes, int* ctas_per_sm);
@@ -325,6 +329,7 @@ struct JitPlanView {
   const int64_t* itab;               // the plan's int64 table pool (Bucketize borders, MapId tables)
   const DevOp* ops;                  // global op pool (DUnit::gops = 1: units too large to stage)
   const float* ftab;                 // global f32 border pool (DUnit::gops = 1)
+  int id_slots;                      // staged slots whose ids the kernel stages in shared memory (RbGeom)
 };
 struct JitModule;  // compiled kernels (opaque)
 // Generate the CUDA source of the plan's policy (small: 32-bit scans, every

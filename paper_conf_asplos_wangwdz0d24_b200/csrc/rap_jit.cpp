@@ -387,10 +387,20 @@ struct Gen {
     auto prefetch = [&](int q) {
       const RbFeat& R = v.feat[v.perm[q]];
       const std::string Y = "Y" + i2s(q);
+      const int sl = slot[R.src[0]];
+      std::string t = "    int64_t pf" + i2s(q) + ";\n    { const RbRow " + Y + " = rb_row(s, " + i2s(sl) +
+                      ", r);\n      const bool ok = in && " + Y + ".valid && " + Y + ".b > " + Y + ".a;\n";
+      if (sl < v.id_slots) {
+        // the chunk's ids were bulk-copied into shared memory (rb_stage_ids):
+        // rows inside the staged range read them there, the rest from global
+        t += "      const long long j = (long long)" + Y + ".a - s.ide0[" + i2s(sl) + "];\n"
+             "      const bool sh = ok && (unsigned long long)j < (unsigned long long)kRbIdCap;\n"
+             "      pf" + i2s(q) + " = sh ? s.ids[" + i2s(sl * kRbIdCap) + " + j] : __ldg(ok && !sh ? p.val[" +
+             i2s(R.src[0]) + "] + " + Y + ".a : c.itab); }\n";
+        return t;
+      }
       // unconditional load (no branch): rows without a first id read a word of the plan blob instead
-      return "    int64_t pf" + i2s(q) + ";\n    { const RbRow " + Y + " = rb_row(s, " + i2s(slot[R.src[0]]) +
-             ", r);\n      const bool ok = in && " + Y + ".valid && " + Y + ".b > " + Y + ".a;\n      pf" + i2s(q) +
-             " = __ldg(ok ? p.val[" + i2s(R.src[0]) + "] + " + Y + ".a : c.itab); }\n";
+      return t + "      pf" + i2s(q) + " = rap_ldin(ok ? p.val[" + i2s(R.src[0]) + "] + " + Y + ".a : c.itab); }\n";
     };
     // MapId outputs: their first table probe is loaded kProbe outputs ahead,
     // from the prefetched id run through the stages before MapId
@@ -781,6 +791,8 @@ struct Gen {
   std::string source(bool small) {
     std::string s;
     s += "// generated by rap_jit.cpp for one plan (" + i2s(F) + " sparse outputs)\n";
+    if (env_int("RAP_JIT_STCS", 1)) s += "#define RAP_ST_CS 1\n";  // streaming output stores (rap_rows_skel.cuh)
+    if (env_int("RAP_JIT_LDCS", 0)) s += "#define RAP_LD_CS 1\n";  // (experiment knob)
     s += "#include \"rap_rows_interp.cuh\"\n\nnamespace rapk {\n\n";
     bool records = false;  // does any output fall back to the interpreter's functions?
     for (int f = 0; f < F; ++f) records |= v.feat[f].emit != 0;
@@ -795,7 +807,31 @@ struct Gen {
     body += "  }\n";
     body += dense;
     body += lengths_fn();
-    body += column_mode() ? col_emit_fn() : emit_fn();
+    {
+      std::string e = column_mode() ? col_emit_fn() : emit_fn();
+      // (experiment knob RAP_JIT_NOSTORE: 1 = no output stores in the emit
+      // phase, 2 = values only, 3 = lengths and offsets only; the stored
+      // values fold into a sink so the computation stays)
+      const int ns = env_int("RAP_JIT_NOSTORE", 0);
+      if (ns) {
+        auto rep = [&](const std::string& a, const std::string& b) {
+          for (size_t i = e.find(a); i != std::string::npos; i = e.find(a, i + b.size())) e.replace(i, a.size(), b);
+        };
+        const size_t k = e.find("bool ovf = false;");
+        if (k != std::string::npos) e.insert(k, "unsigned long long sink = 0;\n    ");
+        if (ns == 1 || ns == 3) rep("stg_s64_if(L", "RAP_SINK(L");
+        if (ns == 1 || ns == 2) {
+          rep("stg_s32_if(in,", "RAP_SINK(in,");
+          rep("stg_s64_if(in,", "RAP_SINK(in,");
+        }
+        rep("stg_s64_if(fast", "RAP_SINK(fast");
+        if (ns == 2) rep("RAP_SINK(fast", "stg_s64_if(fast");
+        const size_t z = e.rfind("if (ovf) atomicExch");
+        e.insert(z, "if (sink == 0x5eed5eedull) c.values[0] = (int64_t)sink;\n    ");
+        body += "#define RAP_SINK(q, p, v) (sink ^= (q) ? (unsigned long long)(v) + (unsigned long long)(p) : 0ull)\n";
+      }
+      body += e;
+    }
     body += "};\n\n}  // namespace rapk\n\n";
     s += globals + sample_globals + "\n" + body;
     // one variant per module: 32-bit scans (every offset < 2^31) or 64-bit
@@ -942,7 +978,7 @@ int launch_jit(JitModule* m, const Common& c, const RbGeom& g, const LaunchRaw& 
   attr[0].id = cudaLaunchAttributeCooperative;
   attr[0].val.cooperative = 1;
   cfg.attrs = attr;
-  cfg.numAttrs = 1;
+  cfg.numAttrs = env_int("RAP_NONCOOP", 0) ? 0 : 1;  // (experiment knob: launch-cost measurement only)
   void* args[1] = {&p};
   cudaError_t e = cudaLaunchKernelExC(&cfg, k, args);
   if (e != cudaSuccess) return (int)e;

@@ -131,7 +131,7 @@ struct rap_plan {
   JitModule* jit[2] = {nullptr, nullptr};  // [small] variants
   int jit_state = 0, jit_ctas_per_sm = 0;  // state of the last variant asked for
   int jit_st[2] = {0, 0}, jit_occ[2] = {0, 0};
-  int jit_smem = 0, jit_dense_bytes = 0;
+  int jit_smem = 0, jit_dense_bytes = 0, jit_id_slots = 0;
   double jit_s = 0;
 };
 
@@ -819,6 +819,28 @@ int memo_prefix(const rap_plan* P, const Chain& o, const Canon& qo, const Chain&
   return pm;
 }
 
+// The generated kernel's shared memory before id staging: the dense warp's
+// 32-row tile after the base-phase totals (rap_jit.cpp tile_offset), no
+// length cache, no shared memo.
+static int jit_base_smem(const rap_plan* P, int dense_bytes) {
+  return rows_smem_bytes(dense_bytes, P->rb_max_fl, P->rb_max_cols, 0, (int)P->souts.size(), 0);
+}
+static int jit_tile_bytes(const rap_plan* P) {
+  const int tile = ((2 * ((int)P->souts.size() + 1) * 8 + 15) & ~15) + 32 * (P->d_out | 1) * 4;
+  return (P->d_out > 0 && tile <= P->rb_dense_bytes) ? tile : P->rb_dense_bytes;
+}
+// Staged columns whose chunk ids the generated kernel bulk-copies into shared
+// memory: as many as fit beside its base layout with two CTAs per SM.
+static int jit_id_slots(const rap_plan* P) {
+  // measured on C2 (B200): staging the ids cost 2.3 us of staging and gained
+  // nothing in the emit phase (cold 59.5 vs 55.8 us), so it is opt-in
+  const char* env = getenv("RAP_JIT_IDS");  // "1": stage the chunk ids (experiment knob)
+  if (!(env && env[0] == '1')) return 0;
+  const int budget = 113 * 1024 - jit_base_smem(P, std::max(P->jit_dense_bytes, jit_tile_bytes(P)));
+  const int per = kRbIdCap * 8 + 8;
+  return std::max(0, std::min(P->rb_max_cols, (budget - 16) / per));
+}
+
 JitPlanView jit_view(const rap_plan* P) {
   JitPlanView v;
   v.n_sparse_out = (int)P->souts.size();
@@ -835,6 +857,7 @@ JitPlanView jit_view(const rap_plan* P) {
   v.itab = P->itab.data();
   v.ops = P->ops.data();
   v.ftab = P->ftab.data();
+  v.id_slots = jit_id_slots(P);
   return v;
 }
 
@@ -1154,10 +1177,11 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
     // the generated kernel: no length cache, no shared memo (registers), and
     // only the dense tile when it generates the dense outputs (rap_jit.cpp)
     // the dense warp's 32-row tile after the base-phase totals (rap_jit.cpp tile_offset)
-    const int tile = ((2 * ((int)P->souts.size() + 1) * 8 + 15) & ~15) + 32 * (P->d_out | 1) * 4;
-    P->jit_dense_bytes = (P->d_out > 0 && tile <= P->rb_dense_bytes) ? tile : P->rb_dense_bytes;
+    P->jit_dense_bytes = jit_tile_bytes(P);
     P->jit_dense_bytes = std::max(P->jit_dense_bytes, jit_dense_need(jit_view(P)));  // + the emitter's memo rows
-    P->jit_smem = rows_smem_bytes(P->jit_dense_bytes, P->rb_max_fl, P->rb_max_cols, 0, (int)P->souts.size(), 0);
+    P->jit_id_slots = jit_id_slots(P);
+    P->jit_smem = rows_smem_bytes(P->jit_dense_bytes, P->rb_max_fl, P->rb_max_cols, 0, (int)P->souts.size(), 0,
+                                  P->jit_id_slots);
     if (P->rb_smem > 227 * 1024) P->rb_fits = 0;
   }
   if (P->rb_fits) {
@@ -1585,6 +1609,7 @@ static void rows_geometry(const rap_plan* P, int64_t B, const int64_t* nnz, int 
   const int bud = budget > 0 ? budget : P->budget;
   int64_t slots = std::max<int64_t>(1, std::min<int64_t>((int64_t)bud * ctas_per_sm, kMaxCtas));
   g->n_dcta = 0;
+  g->id_slots = 0;
   if (n_dense_tiles > 0 && n_dense_tiles <= slots / 4) {
     g->n_dcta = (int)n_dense_tiles;
     slots -= n_dense_tiles;
@@ -1724,6 +1749,7 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
       g.len_cache = 0;
       g.n_memo = 0;
       g.dense_bytes = P->jit_dense_bytes;
+      g.id_slots = P->jit_id_slots;
     } else {
       g.len_cache = 1;
     }

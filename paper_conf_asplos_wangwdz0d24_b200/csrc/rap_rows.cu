@@ -36,6 +36,9 @@
 #include <cuda_runtime.h>
 #include <string.h>
 
+#ifndef RAP_ROWS_PLAIN_STORES
+#define RAP_ST_CS 1  // streaming output stores (rap_rows_skel.cuh)
+#endif
 #include "rap_rows_interp.cuh"
 
 namespace rapk {
@@ -93,7 +96,8 @@ int rows_dense_bytes(int max_width) {
   return kDProgBytes + dense_in_bytes() + align_up(tile, 16);
 }
 
-int rows_smem_bytes(int dense_bytes, int max_fl, int max_cols, int n_memo, int n_sparse_out, int len_cache) {
+int rows_smem_bytes(int dense_bytes, int max_fl, int max_cols, int n_memo, int n_sparse_out, int len_cache,
+                    int id_slots) {
   int o = rb_region0(dense_bytes, n_memo, n_sparse_out);
   o += 2 * rb_align(max_fl * 8 * 8);
   o += rb_align(max_fl * 8);
@@ -101,6 +105,7 @@ int rows_smem_bytes(int dense_bytes, int max_fl, int max_cols, int n_memo, int n
   o += rb_align(max_cols * kRbPitch * 4);
   o += rb_align(max_cols * 8 * 4);
   if (len_cache) o += rb_align(max_fl * kRbChunk * 2);
+  if (id_slots > 0) o += rb_align(id_slots * 8) + id_slots * kRbIdCap * 8;
   return o;
 }
 

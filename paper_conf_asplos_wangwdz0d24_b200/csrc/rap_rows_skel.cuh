@@ -88,7 +88,11 @@ struct RbSmem {
   long long* wb;         // [max_fl][8] warp bases of the chunk
   long long* base;       // [max_fl] running base (first offset of the next chunk)
   long long* memo;       // [n_memo][kRbChunk] memoised element 0 (phase 4)
+  long long* ide0;       // [id_slots] values index of ids[slot][0] (kRbIdNone: not staged)
+  long long* ids;        // [id_slots][kRbIdCap] the chunk's ids of the slot's column
 };
+
+constexpr long long kRbIdNone = -(1ll << 61);  // ide0 of a column whose chunk ids were not staged
 
 __host__ __device__ inline int rb_align(int x) { return (x + 15) & ~15; }
 
@@ -115,6 +119,10 @@ __device__ __forceinline__ RbSmem rb_carve(unsigned char* smem, const RbGeom& g,
   s.bm = reinterpret_cast<uint32_t*>(smem + o);
   o += rb_align(g.max_cols * 8 * 4);
   s.len = g.len_cache ? reinterpret_cast<uint16_t*>(smem + o) : nullptr;
+  if (g.len_cache) o += rb_align(g.max_fl * kRbChunk * 2);
+  s.ide0 = reinterpret_cast<long long*>(smem + o);
+  o += rb_align(g.id_slots * 8);
+  s.ids = reinterpret_cast<long long*>(smem + o);
   return s;
 }
 
@@ -186,13 +194,37 @@ __device__ __forceinline__ void rb_sync() {
     __syncthreads();
 }
 
+// Stage the ids val[a0, a1) of one column's chunk into dst (kRbIdCap slots):
+// dst[j] = val[e0 + j] with e0 = a0 - h (h = 1 when val + a0 is not 16-byte
+// aligned, so the bulk copy's source and destination are), the 16-byte
+// aligned body by one bulk copy onto ibar, the <= 2 unaligned end ids by plain
+// loads (never a byte outside [a0, a1)).  Ranges that do not fit (long lists)
+// are not staged (e0 = kRbIdNone: the emitter reads them from global).
+__device__ __forceinline__ void rb_stage_ids(const int64_t* val, int32_t a0, int32_t a1, long long* dst,
+                                             long long* e0, uint64_t* ibar) {
+  const int n = a1 - a0;
+  const int h = (reinterpret_cast<uintptr_t>(val + a0) & 15) ? 1 : 0;
+  if (val == nullptr || n < 0 || n + h > kRbIdCap) {
+    *e0 = kRbIdNone;
+    mbar_arrive_expect(ibar, 0u);
+    return;
+  }
+  const int t = (n > h && (reinterpret_cast<uintptr_t>(val + a1) & 15)) ? 1 : 0;
+  const int nb = n - h - t;  // body ids (16-byte aligned at both ends)
+  mbar_arrive_expect(ibar, nb > 0 ? (uint32_t)nb * 8u : 0u);
+  if (nb > 0) bulk_g2s(dst + 2 * h, val + a0 + h, (uint32_t)nb * 8u, ibar);
+  if (h && n > 0) dst[1] = __ldg(val + a0);
+  if (t) dst[n - 1 + h] = __ldg(val + a1 - 1);
+  *e0 = (long long)a0 - h;
+}
+
 // Stage the offsets [c0, c0 + nr] and validity words of the group's raw
 // columns: thread 0 issues one bulk copy (TMA engine, cp.async.bulk) per
 // column body onto the CTA's staging mbarrier; warp 0 loads the <= 3
 // unaligned tail words (and whole columns whose base is not 16-byte aligned).
 template <bool kDW, class P>
 __device__ __forceinline__ void rb_stage(const P& p, const RbSmem& s, const int16_t* cols, int n_cols, int64_t c0,
-                                         int nr, uint64_t* bar, int* phase) {
+                                         int nr, uint64_t* bar, int* phase, int n_ids = 0, uint64_t* ibar = nullptr) {
   // thread k < n_cols stages column k: one bulk copy (TMA engine) each for the
   // 16-byte-aligned body of its offsets and validity words, arriving on the
   // staging mbarrier (expected arrivals = n_cols) with those bytes; the <= 3
@@ -205,6 +237,13 @@ __device__ __forceinline__ void rb_stage(const P& p, const RbSmem& s, const int1
   if (tid < n_cols) {
     const int k = tid, col = cols[k];
     const int32_t* src = p.off[col] + c0;
+    // slots < n_ids: the chunk's id range [off[c0], off[c0 + nr]) too (its
+    // two bounds are loaded beside the offsets' bulk copy)
+    int32_t a0 = 0, a1 = 0;
+    if (k < n_ids) {
+      a0 = __ldg(src);
+      a1 = __ldg(src + nr);
+    }
     const bool oa = (reinterpret_cast<uintptr_t>(src) & 15) == 0;
     const uint32_t ob = oa ? ((uint32_t)(no * 4) & ~15u) : 0u;
     const uint32_t* bm = p.svalid[col];
@@ -214,6 +253,7 @@ __device__ __forceinline__ void rb_stage(const P& p, const RbSmem& s, const int1
     mbar_arrive_expect(bar, ob + wb);
     if (ob) bulk_g2s(s.off + k * kRbPitch, src, ob, bar);
     if (wb) bulk_g2s(s.bm + k * 8, bs, wb, bar);
+    if (k < n_ids) rb_stage_ids(p.val[col], a0, a1, s.ids + k * kRbIdCap, s.ide0 + k, ibar);
     for (int i = (int)(ob / 4); i < no; ++i) s.off[k * kRbPitch + i] = __ldg(src + i);
     if (bs == nullptr) {
       for (int i = 0; i < nw; ++i) s.bm[k * 8 + i] = 0xffffffffu;
@@ -231,19 +271,44 @@ __device__ __forceinline__ void rb_stage(const P& p, const RbSmem& s, const int1
 // emitted as st.global without a memory clobber: the compiler may move shared
 // loads of later outputs above them (a store through a plain generic pointer
 // could alias shared memory and would pin every later LDS behind it).
+// The generated kernel stores its outputs with the streaming hint (st.global.cs,
+// evict-first in L2): C2 on B200 with inputs and outputs rotating through HBM,
+// 55.8 -> 47.6 us per launch -- written-once output lines no longer push
+// the plan's tables and the next lines' staging out of L2.
+#ifdef RAP_ST_CS
+#define RAP_STG "st.global.cs"
+#else
+#define RAP_STG "st.global"
+#endif
+// Raw inputs read once (ids, dense values): streaming loads when RAP_LD_CS.
+template <class T>
+__device__ __forceinline__ T rap_ldin(const T* p) {
+#ifdef RAP_LD_CS
+  return __ldcs(p);
+#else
+  return __ldg(p);
+#endif
+}
+__device__ __forceinline__ int64_t rap_ldin(const int64_t* p) {
+#ifdef RAP_LD_CS
+  return (int64_t)__ldcs(reinterpret_cast<const long long*>(p));
+#else
+  return (int64_t)__ldg(reinterpret_cast<const long long*>(p));
+#endif
+}
 __device__ __forceinline__ void stg_s32(int32_t* p, int32_t v) {
-  asm volatile("st.global.s32 [%0], %1;" ::"l"(p), "r"(v));
+  asm volatile(RAP_STG ".s32 [%0], %1;" ::"l"(p), "r"(v));
 }
 __device__ __forceinline__ void stg_s64(int64_t* p, int64_t v) {
-  asm volatile("st.global.s64 [%0], %1;" ::"l"(p), "l"(v));
+  asm volatile(RAP_STG ".s64 [%0], %1;" ::"l"(p), "l"(v));
 }
 // Predicated forms (one instruction, no branch around it).
 __device__ __forceinline__ void stg_s32_if(bool q, int32_t* p, int32_t v) {
-  asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q st.global.s32 [%0], %1;\n\t}" ::"l"(p), "r"(v),
+  asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q " RAP_STG ".s32 [%0], %1;\n\t}" ::"l"(p), "r"(v),
                "r"((unsigned)q));
 }
 __device__ __forceinline__ void stg_s64_if(bool q, int64_t* p, int64_t v) {
-  asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q st.global.s64 [%0], %1;\n\t}" ::"l"(p), "l"(v),
+  asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q " RAP_STG ".s64 [%0], %1;\n\t}" ::"l"(p), "l"(v),
                "r"((unsigned)q));
 }
 __device__ __forceinline__ void rb_store(const Common& c, long long pos, int64_t v) {
@@ -273,7 +338,7 @@ __device__ __forceinline__ void canon_part(const Canon& q, int keep, const int64
 template <class P>
 __device__ __forceinline__ float rb_dense_in(const P& p, int col, int64_t row) {
   const uint32_t* bm = p.dvalid[col];
-  const float v = __ldg(p.dense[col] + row);
+  const float v = rap_ldin(p.dense[col] + row);
   if (bm == nullptr) return v;
   return ((__ldg(bm + (row >> 5)) >> (row & 31)) & 1u) ? v : __int_as_float(0x7fc00000);
 }
@@ -346,6 +411,8 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
   __shared__ int s_last, s_fmax;
   __shared__ uint64_t s_sbar;  // staging mbarrier (bulk copies)
   __shared__ int s_sphase;
+  __shared__ uint64_t s_ibar;  // id staging mbarrier (generated kernel, g.id_slots > 0)
+  __shared__ int s_iphase;
   const RbGeom& g = p.g;
   const Common& c = p.c;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -382,6 +449,7 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
   if (tid == 0) {
     mbar_init(&cs.bar, 1);
     s_sphase = 0;
+    s_iphase = 0;
     cs.phase = 0;
     cs.dgroup = -1;
     s_fmax = 0;
@@ -414,6 +482,11 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
   for (int i = 0; i < (MS + 63) / 64; ++i) n_cols += __popcll(s_mask[i]);
   x.n_cols = n_cols;
   if (tid == 0) mbar_init(&s_sbar, (uint32_t)max(n_cols, 1));  // staging: one arrival per column
+  // id staging: one arrival per slot < n_ids, issued with the chunk's offsets
+  // (phase 1 when the block is one chunk, else phase 4) and awaited just
+  // before the chunk's ids are emitted
+  const int n_ids = min(n_cols, g.id_slots);
+  if (tid == 0) mbar_init(&s_ibar, (uint32_t)max(n_ids, 1));
   for (int col = tid; col < MS; col += kRbChunk) {
     const unsigned long long m = s_mask[col >> 6];
     int before = __popcll(m & ((1ull << (col & 63)) - 1ull));
@@ -431,13 +504,14 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
   trace_stamp(c, 7);
   if (kDW && warp == kWS) {
     Pol::dense_warp(p, s, x);  // the dense outputs of rows [R0, R1), concurrent with the sparse phases
+    trace_stamp_warp(c, 15);
   } else {
 
   // (1) per-output totals of my rows -> agg, then announce the CTA
   for (int ch = 0; ch < nch; ++ch) {
     const int64_t c0 = x.R0 + (int64_t)ch * kTS;
     const int nr = (int)min((int64_t)kTS, x.R1 - c0);
-    rb_stage<kDW>(p, s, s_cols, n_cols, c0, nr, &s_sbar, &s_sphase);
+    rb_stage<kDW>(p, s, s_cols, n_cols, c0, nr, &s_sbar, &s_sphase, nch == 1 ? n_ids : 0, &s_ibar);
     if (ch == 0) trace_stamp(c, 8);
     Pol::template lengths<kSmall>(p, s, x, nr, ch > 0);
     rb_sync<kDW>();
@@ -553,7 +627,7 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
       const int64_t c0 = x.R0 + (int64_t)ch * kTS;
       const int nr = (int)min((int64_t)kTS, x.R1 - c0);
       if (nch > 1) {
-        rb_stage<kDW>(p, s, s_cols, n_cols, c0, nr, &s_sbar, &s_sphase);
+        rb_stage<kDW>(p, s, s_cols, n_cols, c0, nr, &s_sbar, &s_sphase, n_ids, &s_ibar);
         Pol::template lengths<kSmall>(p, s, x, nr, false);
         rb_sync<kDW>();
       }
@@ -567,8 +641,10 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
         s.base[tid] = b;
       }
       rb_sync<kDW>();
+      if (n_ids > 0) mbar_wait(&s_ibar, (uint32_t)s_iphase);  // the chunk's staged ids landed
       Pol::template emit<kSmall>(p, s, x, c0, nr);
       rb_sync<kDW>();
+      if (n_ids > 0 && tid == 0) s_iphase ^= 1;
     }
   }
   }  // sparse warps
@@ -593,6 +669,7 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
     }
     __threadfence();
   }
+  trace_stamp(c, 14);
 }
 
 }  // namespace rapk

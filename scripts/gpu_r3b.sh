@@ -1,0 +1,10 @@
+#!/bin/bash
+mkdir -p gpurun_out
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1 || { tail -20 gpurun_out/build.log; exit 1; }
+(
+timeout 300 python scripts/cold_trace.py
+RAP_NONCOOP=1 TAG=noncoop timeout 300 python scripts/cold_trace.py
+B=2048 TAG=b2048 timeout 300 python scripts/cold_trace.py
+RAP_NONCOOP=1 B=2048 TAG=b2048noncoop STAMPS=0 timeout 300 python scripts/cold_trace.py
+) > gpurun_out/r3b.log 2>&1
+cat gpurun_out/r3b.log
