@@ -162,6 +162,28 @@ __device__ __forceinline__ int count_le8(const int64_t* p, int64_t x) {
 // code computes it from immediates): then the 8 sub-block maxima of block j0
 // (smp8[8 j0 .. 8 j0 + 8), smp8[i] = b[8 i + 7]) and the 8 borders of the
 // chosen sub-block, two bursts (R4; same result as upper_bound).
+// Same search over tables staged in shared memory (the generated kernel
+// copies a plan's Bucketize borders and sub-block maxima there at launch).
+__device__ __forceinline__ int count_le8_s(const int64_t* p, int64_t x) {
+  const longlong2* q = reinterpret_cast<const longlong2*>(p);
+  const longlong2 a0 = q[0], a1 = q[1], a2 = q[2], a3 = q[3];
+  return (a0.x <= x) + (a0.y <= x) + (a1.x <= x) + (a1.y <= x) + (a2.x <= x) + (a2.y <= x) + (a3.x <= x) + (a3.y <= x);
+}
+__device__ __forceinline__ int64_t upper_bound_64s(const int64_t* b, int m, const int64_t* smp8, int j0, int64_t x) {
+  const int nb = m >> 6;
+  const int jc = min(j0, nb - 1);
+  const int j1 = 8 * jc + min(count_le8_s(smp8 + 8 * jc, x), 7);
+  const int64_t r = (int64_t)j1 * 8 + count_le8_s(b + 8 * j1, x);
+  return j0 >= nb ? (int64_t)m : r;
+}
+// Sub-block maxima in shared memory, borders in global.
+__device__ __forceinline__ int64_t upper_bound_64h(const int64_t* b, int m, const int64_t* smp8, int j0, int64_t x) {
+  const int nb = m >> 6;
+  const int jc = min(j0, nb - 1);
+  const int j1 = 8 * jc + min(count_le8_s(smp8 + 8 * jc, x), 7);
+  const int64_t r = (int64_t)j1 * 8 + count_le8(b + 8 * j1, x);
+  return j0 >= nb ? (int64_t)m : r;
+}
 __device__ __forceinline__ int64_t upper_bound_64(const int64_t* b, int m, const int64_t* smp8, int j0, int64_t x) {
   // branch-free: the loads stay in range, the selects pick the answer
   const int nb = m >> 6;
@@ -184,6 +206,39 @@ __device__ __forceinline__ int64_t map_lookup_from(const int64_t* itab, int64_t 
     if (kv.x == INT64_MIN) return dflt;
     i = (i + 1) & mask;
     kv = __ldg(t + i);
+  }
+}
+// The first two probes of x (slots i and i + 1 of the linear-probing table),
+// loaded ahead together: a lookup resolves without a dependent load unless
+// both slots hold other keys (load <= 1/2: rare).
+struct MapProbe2 {
+  longlong2 a, b;
+};
+__device__ __forceinline__ MapProbe2 map_first_probe2(const int64_t* itab, int64_t a, int m, int64_t x) {
+  const longlong2* t = reinterpret_cast<const longlong2*>(itab + a);
+  const uint32_t mask = (1u << m) - 1u;
+  const uint32_t i = (uint32_t)(((uint64_t)x * 0x9E3779B97F4A7C15ull) >> (64 - m));
+  MapProbe2 r;
+  r.a = __ldg(t + i);
+  r.b = __ldg(t + ((i + 1u) & mask));
+  return r;
+}
+__device__ __forceinline__ int64_t map_lookup_from2(const int64_t* itab, int64_t a, int m, int64_t dflt, int64_t x,
+                                                    MapProbe2 kv) {
+  if (x == INT64_MIN) return dflt;
+  if (kv.a.x == x) return kv.a.y;
+  if (kv.a.x == INT64_MIN) return dflt;
+  if (kv.b.x == x) return kv.b.y;
+  if (kv.b.x == INT64_MIN) return dflt;
+  const longlong2* t = reinterpret_cast<const longlong2*>(itab + a);
+  const uint32_t mask = (1u << m) - 1u;
+  uint32_t i = (uint32_t)(((uint64_t)x * 0x9E3779B97F4A7C15ull) >> (64 - m));
+  i = (i + 2u) & mask;
+  while (true) {
+    const longlong2 k = __ldg(t + i);
+    if (k.x == x) return k.y;
+    if (k.x == INT64_MIN) return dflt;
+    i = (i + 1) & mask;
   }
 }
 __device__ __forceinline__ longlong2 map_first_probe(const int64_t* itab, int64_t a, int m, int64_t x) {

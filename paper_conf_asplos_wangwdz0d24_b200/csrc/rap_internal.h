@@ -244,6 +244,7 @@ constexpr int kRbMaxFL = 64;    // sparse outputs per feature group
 constexpr int kRbMaxF = 1024;   // sparse outputs of a plan the row-block kernel takes
 constexpr int kRbMaxCols = 64;  // raw sparse columns the row-block kernel addresses
 constexpr int kRbMaxDense = 32; // raw dense columns
+constexpr int kRbPitchPairs = 132;  // staged offsets per column in warp-pair mode (128-row chunks)
 constexpr int kRbIdCap = 232;   // staged ids per column and chunk (224 rows of single ids + 16-byte head/tail)
 
 // Per sparse output (indexed by output f): its closed-form length program
@@ -277,6 +278,8 @@ struct RbGeom {
                                         // blocks round robin over every CTA)
   int32_t id_slots;                     // staged columns (slots < id_slots) whose chunk ids are bulk-copied
                                         // into shared memory (generated kernel; 0: ids read from global)
+  int32_t pitch;                        // staged offsets per column (0: kRbPitch, 256-row chunks)
+  int32_t feat_recs;                    // 1: the CTA keeps RbF records in shared memory (interpreter)
   unsigned long long all_cols;          // raw sparse columns the outputs read (bit c: column c < 64)
   const RbFeat* feat;                   // [n_sparse_out], by output index
   const int32_t* perm;                  // [n_sparse_out] processing order (groups are ranges of it)
@@ -307,7 +310,7 @@ int ensure_dyn_smem(const void* kernel, int smem);
 int fused_occupancy(int smem_bytes, int n_dense, int n_sparse, int* ctas_per_sm);
 // Row-block kernel (rap_rows.cu): dynamic smem for a geometry, occupancy, launch.
 int rows_smem_bytes(int dense_bytes, int max_fl, int max_cols, int n_memo, int n_sparse_out, int len_cache,
-                    int id_slots = 0);
+                    int id_slots = 0, int pitch = 0, int feat_recs = 1, int tab_bytes = 0);
 // Dense-phase shared memory of the row-block kernel for dense groups up to max_width columns.
 int rows_dense_bytes(int max_width);
 int rows_occupancy(int smem_bytes, int* ctas_per_sm);
@@ -330,8 +333,41 @@ struct JitPlanView {
   const DevOp* ops;                  // global op pool (DUnit::gops = 1: units too large to stage)
   const float* ftab;                 // global f32 border pool (DUnit::gops = 1)
   int id_slots;                      // staged slots whose ids the kernel stages in shared memory (RbGeom)
+  int pairs;                         // warp-pair mode (rap_rows_skel.cuh kPairs)
 };
 struct JitModule;  // compiled kernels (opaque)
+// How the generated kernel evaluates the dense outputs (rap_jit.cpp):
+//   2: every warp evaluates 32-row tiles of its block's dense rows (one
+//      row-major tile per warp in shared memory) after the block's totals
+//      are published, so the work fills the wait for the other CTAs;
+//   1: one dense warp (warp 7) beside the sparse phases (tiles too wide for
+//      eight per CTA);
+//   0: no generated dense code (the interpreted dense blocks).
+// *region0 = the shared-memory bytes of region 0 the mode needs.
+inline int jit_dense_tiles(int pairs) { return pairs ? 4 : 8; }  // mode 2: warps with a tile
+inline int jit_dense_mode(int n_sparse_out, int d_out, int n_dprogs, int rb_dense_bytes, int pairs, int* region0) {
+  const int off = ((2 * (n_sparse_out + 1) * 8) + 15) & ~15;  // after the base phase's T[f], L[f]
+  const int one = 32 * (d_out | 1) * 4;
+  const int nt = jit_dense_tiles(pairs);
+  if (n_dprogs == 0 || d_out <= 0) {
+    *region0 = rb_dense_bytes;
+    return 0;
+  }
+  if (off + nt * one <= (pairs ? 24 : 48) * 1024) {
+    *region0 = off + nt * one;
+    return 2;
+  }
+  if (pairs) {  // the warp-pair form has no dense warp: interpreted dense blocks
+    *region0 = rb_dense_bytes;
+    return 0;
+  }
+  if (off + one <= rb_dense_bytes) {
+    *region0 = off + one;
+    return 1;
+  }
+  *region0 = rb_dense_bytes;
+  return 0;
+}
 // Generate the CUDA source of the plan's policy (small: 32-bit scans, every
 // offset < 2^31; else 64-bit) and compile it with NVRTC for sm_100a (cached
 // per source text in the process).  Returns nullptr and fills *log on failure.
@@ -340,6 +376,9 @@ int jit_occupancy(JitModule* m, int smem_bytes, int* ctas_per_sm);
 // Region-0 shared-memory bytes the generated kernel needs beyond the dense
 // tile (the column emitter's memo rows; 0 if none).
 int jit_dense_need(const JitPlanView& v);
+// Shared-memory bytes of the tables the generated kernel stages at launch
+// (Bucketize borders and sub-block maxima; 0: none).
+int jit_table_bytes(const JitPlanView& v);
 int launch_jit(JitModule* m, const Common& c, const RbGeom& g, const LaunchRaw& raw, int smem_bytes, void* stream);
 double jit_compile_seconds(const JitModule* m);
 #endif

@@ -84,6 +84,67 @@ struct Gen {
     int n = 0;
     for (size_t c = 0; c < used.size(); ++c)
       if (used[c]) slot[c] = n++;
+    plan_tables();
+  }
+
+  // ---- Bucketize tables staged in shared memory at launch ----
+  // The three-level search's two bursts (8 sub-block maxima, then 8 borders)
+  // are dependent L2 round trips on every row's chain; with the tables in
+  // shared memory they are two shared loads.  Sample tables of every 3-level
+  // Bucketize first (1 KB per 1024 borders), then whole border tables while
+  // the budget lasts (the rest keep their borders in global).
+  struct BkTab {
+    int64_t a;
+    int m;
+    int off_s, off_b;  // byte offsets after the 16-byte mbarrier (off_b < 0: borders in global)
+  };
+  std::vector<BkTab> bktabs;
+  int tab_total = 0;  // bytes after the mbarrier
+  static int tab_budget() { return env_int("RAP_JIT_TABS", 1) ? env_int("RAP_JIT_TAB_BYTES", 40 * 1024) : 0; }
+  void plan_tables() {
+    std::vector<std::pair<int64_t, int>> want;
+    for (int f = 0; f < F; ++f) {
+      if (v.feat[f].emit != 0 && v.feat[f].emit != 3) continue;
+      const Canon& q = v.sprogs[f].cn;
+      if (!(q.mask & CB_BUCKET)) continue;
+      if (!(q.bk_m >= 64 && q.bk_m % 64 == 0 && q.bk_a % 2 == 0)) continue;
+      bool seen = false;
+      for (const auto& w : want) seen |= w.first == q.bk_a;
+      if (!seen) want.push_back({q.bk_a, q.bk_m});
+    }
+    const int budget = tab_budget();
+    for (const auto& w : want) {
+      const int sb = (w.second / 8) * 8;
+      if (tab_total + sb > budget) break;
+      bktabs.push_back(BkTab{w.first, w.second, tab_total, -1});
+      tab_total += sb;
+    }
+    for (BkTab& t : bktabs) {
+      const int bb = t.m * 8;
+      if (tab_total + bb > budget) continue;
+      t.off_b = tab_total;
+      tab_total += bb;
+    }
+  }
+  const BkTab* staged_table(int64_t a) const {
+    for (const BkTab& t : bktabs)
+      if (t.a == a) return &t;
+    return nullptr;
+  }
+  int table_bytes() const { return tab_total > 0 ? 16 + tab_total : 0; }
+  std::string setup_tables() {
+    if (tab_total == 0) return "";
+    std::string s = "    if (threadIdx.x == 0 && x.FL > 0 && x.R1 > x.R0) {  // the plan's tables -> shared memory\n"
+                    "      uint64_t* bar = reinterpret_cast<uint64_t*>(s.tabs);\n"
+                    "      mbar_init(bar, 1);\n"
+                    "      mbar_arrive_expect(bar, " + i2s(tab_total) + "u);\n";
+    for (const BkTab& t : bktabs) {
+      s += "      bulk_g2s(s.tabs + " + i2s(16 + t.off_s) + ", " + sample_table(t.a, t.m) + ", " + i2s((t.m / 8) * 8) +
+           "u, bar);\n";
+      if (t.off_b >= 0)
+        s += "      bulk_g2s(s.tabs + " + i2s(16 + t.off_b) + ", p.c.itab + " + lit64(t.a) + ", " + i2s(t.m * 8) + "u, bar);\n";
+    }
+    return s + "    }\n";
   }
 
   static std::string cap_expr(const std::string& X, int cap) {
@@ -100,7 +161,7 @@ struct Gen {
     if (R.kind == 1) return "    const int32_t L" + Q + " = in ? " + i2s(R.out_cap) + " : 0;\n";
     if (R.kind == 0) {
       const std::string X = "X" + Q + "_0";
-      s += "    const RbRow " + X + " = rb_row(s, " + i2s(slot[R.src[0]]) + ", r);\n";
+      s += "    const RbRow " + X + " = " + rbrow() + "(s, " + i2s(slot[R.src[0]]) + ", r);\n";
       s += "    const int32_t L" + Q + " = in ? (" + X + ".valid ? " + cap_expr(X, R.cap[0]) + " : " + i2s(R.ncap[0]) +
            ") : 0;\n";
       return s;
@@ -112,7 +173,7 @@ struct Gen {
         s += "    const int32_t " + l + " = " + i2s(R.cap[i]) + ";\n";
       } else {
         const std::string X = "X" + Q + "_" + i2s(i);
-        s += "    const RbRow " + X + " = rb_row(s, " + i2s(slot[R.src[i]]) + ", r);\n";
+        s += "    const RbRow " + X + " = " + rbrow() + "(s, " + i2s(slot[R.src[i]]) + ", r);\n";
         s += "    const int32_t " + l + " = " + X + ".valid ? " + cap_expr(X, R.cap[i]) + " : " + i2s(R.ncap[i]) +
              ";\n";
       }
@@ -128,6 +189,11 @@ struct Gen {
   std::string stages(const Canon& q, int mask, const std::string& x, const std::string& full, int memo_after,
                      const std::string& mvar, const std::string& probe = "") {
     std::string s;
+    // (experiment knob RAP_JIT_SKIP: bit 1 MapId, 2 SigridHash, 4 Bucketize
+    // stages left out -- wrong outputs, for cost attribution only)
+    mask &= ~(env_int("RAP_JIT_SKIP", 0) & 1 ? CB_MAPID : 0);
+    mask &= ~(env_int("RAP_JIT_SKIP", 0) & 2 ? CB_SIGRID : 0);
+    mask &= ~(env_int("RAP_JIT_SKIP", 0) & 4 ? CB_BUCKET : 0);
     auto cond = [&](int bit) { return (q.null_mask & bit) ? std::string() : "if (" + full + ") "; };
     if (memo_after == 16) s += "        " + mvar + " = " + x + ";\n";
     if (mask & CB_CLAMP) {
@@ -137,7 +203,7 @@ struct Gen {
     }
     if (mask & CB_MAPID) {
       if (!probe.empty())  // first probe loaded ahead
-        s += "        " + cond(CB_MAPID) + x + " = map_lookup_from(c.itab, " + lit64(q.map_a) + ", " + i2s(q.map_m) + ", " +
+        s += "        " + cond(CB_MAPID) + x + " = " + (map2() ? "map_lookup_from2" : "map_lookup_from") + "(c.itab, " + lit64(q.map_a) + ", " + i2s(q.map_m) + ", " +
              lit64(q.map_def) + ", " + x + ", " + probe + ");\n";
       else
         s += "        " + cond(CB_MAPID) + x + " = map_lookup(c.itab, " + lit64(q.map_a) + ", " + i2s(q.map_m) + ", " +
@@ -156,8 +222,14 @@ struct Gen {
         const std::string nm = sample_table(q.bk_a, q.bk_m);
         s += "        " + cond(CB_BUCKET) + "{ const int j0 = 0";
         for (int k = 0; k < q.bk_m / 64; ++k) s += " + (" + x + " >= " + lit64(v.itab[q.bk_a + 64 * k + 63]) + ")";
-        s += "; " + x + " = upper_bound_64(c.itab + " + lit64(q.bk_a) + ", " + i2s(q.bk_m) + ", " + nm + ", j0, " + x +
-             "); }\n";
+        const BkTab* t = staged_table(q.bk_a);
+        const std::string smp =
+            t ? "reinterpret_cast<const int64_t*>(s.tabs + " + i2s(16 + t->off_s) + ")" : nm;
+        const std::string brd = (t && t->off_b >= 0)
+                                    ? "reinterpret_cast<const int64_t*>(s.tabs + " + i2s(16 + t->off_b) + ")"
+                                    : "c.itab + " + lit64(q.bk_a);
+        const std::string fn = !t ? "upper_bound_64" : (t->off_b >= 0 ? "upper_bound_64s" : "upper_bound_64h");
+        s += "; " + x + " = " + fn + "(" + brd + ", " + i2s(q.bk_m) + ", " + smp + ", j0, " + x + "); }\n";
       } else if (q.bk_m >= 64) {  // two-level search over a sample table in the module
         const std::string nm = sample_table(q.bk_a, q.bk_m);
         s += "        " + cond(CB_BUCKET) + x + " = upper_bound_s8(c.itab + " + lit64(q.bk_a) + ", " + i2s(q.bk_m) +
@@ -209,10 +281,11 @@ struct Gen {
   int pitch() const { return v.d_out | 1; }
   // the dense warp's tile sits after the base-phase totals T[f], L[f]
   int tile_offset() const { return ((2 * (F + 1) * 8) + 15) & ~15; }
-  bool gen_dense_ok() const {
-    if (v.n_dprogs == 0 || v.d_out <= 0) return false;
-    return tile_offset() + 32 * pitch() * 4 <= v.dense_bytes;
+  int dense_mode() const {
+    int r0 = 0;
+    return jit_dense_mode(F, v.d_out, v.n_dprogs, v.dense_bytes, v.pairs, &r0);
   }
+  bool gen_dense_ok() const { return dense_mode() == 1; }  // the dense-warp form (kDenseWarp)
   double unit_cost(const DProg& dp, const DUnit& un) const {
     const DevOp* ops = un.gops ? v.ops : dp.ops;
     double c = 8;
@@ -305,12 +378,18 @@ struct Gen {
     // the row (independent loads first), a 32-row tile in shared memory after
     // the base-phase totals, then stored by the warp
     std::string s;
-    const bool ok = gen_dense_ok();
-    s += "  static constexpr bool kGenDense = false;\n";
+    const int mode = dense_mode();
+    const bool ok = mode == 1;
+    s += "  static constexpr bool kGenDense = " + std::string(mode == 2 ? "true" : "false") + ";\n";
     s += "  static constexpr bool kDenseWarp = " + std::string(ok ? "true" : "false") + ";\n";
-    s += "  template <class P>\n  static __device__ __forceinline__ void dense(const P&, const RbSmem&, const RbCtx&) {}\n";
-    s += "  template <class P>\n  static __device__ __forceinline__ void dense_warp(const P& p, const RbSmem& s, const RbCtx& x) {\n";
-    if (!ok) return s + "  }\n";
+    if (mode == 2) {
+      s += "  template <class P>\n  static __device__ __forceinline__ void dense_warp(const P&, const RbSmem&, const RbCtx&) {}\n";
+      s += "  template <class P>\n  static __device__ __forceinline__ void dense(const P& p, const RbSmem& s, const RbCtx& x) {\n";
+    } else {
+      s += "  template <class P>\n  static __device__ __forceinline__ void dense(const P&, const RbSmem&, const RbCtx&) {}\n";
+      s += "  template <class P>\n  static __device__ __forceinline__ void dense_warp(const P& p, const RbSmem& s, const RbCtx& x) {\n";
+      if (!ok) return s + "  }\n";
+    }
     std::vector<std::pair<int, int>> units;
     std::vector<int> cols;
     for (int gi = 0; gi < v.n_dprogs; ++gi)
@@ -321,8 +400,17 @@ struct Gen {
           cols.push_back(un.src_col);
       }
     s += "    const Common& c = p.c;\n    const int lane = threadIdx.x & 31;\n";
-    s += "    float* tile = reinterpret_cast<float*>(s.dense + " + i2s(tile_offset()) + ");  // [32][" + i2s(pitch()) + "]\n";
-    s += "    for (int64_t d0 = x.R0; d0 < x.R1; d0 += 32) {\n";
+    if (mode == 2) {  // warps < nt: their own tile, 32-row tiles of the block round robin over them
+      const int nt = jit_dense_tiles(v.pairs);
+      s += "    const int warp = threadIdx.x >> 5;\n";
+      s += "    float* tile = reinterpret_cast<float*>(s.dense + " + i2s(tile_offset()) + ") + warp * " +
+           i2s(32 * pitch()) + ";  // [" + i2s(nt) + "][32][" + i2s(pitch()) + "]\n";
+      s += "    if (warp < " + i2s(nt) + ")\n";
+      s += "    for (int64_t d0 = x.R0 + 32 * warp; d0 < x.R1; d0 += " + i2s(32 * nt) + ") {\n";
+    } else {
+      s += "    float* tile = reinterpret_cast<float*>(s.dense + " + i2s(tile_offset()) + ");  // [32][" + i2s(pitch()) + "]\n";
+      s += "    for (int64_t d0 = x.R0; d0 < x.R1; d0 += 32) {\n";
+    }
     s += "      const int nr = (int)min((int64_t)32, x.R1 - d0);\n";
     s += "      if (lane < nr) {\n        const int64_t row = d0 + lane;\n";
     s += "        float* trow = tile + lane * " + i2s(pitch()) + ";\n";
@@ -333,27 +421,73 @@ struct Gen {
     return s;
   }
 
+  // Warp-pair mode (rap_rows_skel.cuh kPairs): warps 2w, 2w + 1 take the
+  // outputs [0, split) and [split, F) of the processing order over the same
+  // 32 rows.  split: a unit boundary (no NGram separated from a memo provider)
+  // nearest to half the predicted cost.
+  bool pairs() const { return v.pairs != 0; }
+  // MapId: the first two probe slots loaded ahead (RAP_JIT_MAP1=1: one, experiment knob)
+  static bool map2() { return env_int("RAP_JIT_MAP1", 0) == 0; }
+  std::string rbrow() const { return "rb_row_p<" + i2s(pairs() ? kRbPitchPairs : kRbChunk + 4) + ">"; }
+  std::string thread_vars() const {
+    if (pairs())
+      return "    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, wi = warp >> 1, r = (wi << 5) | lane;\n"
+             "    (void)tid;\n";
+    return "    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, wi = warp, r = tid;\n";
+  }
+  int split_point() const {
+    if (!pairs()) return F;
+    double tot = 0;
+    std::vector<double> pre(F + 1, 0.0);
+    for (int q = 0; q < F; ++q) pre[q + 1] = pre[q] + out_cost(q);
+    tot = pre[F];
+    int best = F;
+    double bd = 1e30;
+    for (int sp = 1; sp < F; ++sp) {
+      bool ok = true;  // no NGram at >= sp reads a memo provider at < sp
+      for (int q = sp; q < F && ok; ++q) {
+        const RbFeat& R = v.feat[v.perm[q]];
+        if (R.emit != 3) continue;
+        for (int i = 0; i < R.k; ++i)
+          if (R.prov[i] >= 0 && R.prov[i] < sp) ok = false;
+      }
+      if (!ok) continue;
+      const double d = std::fabs(pre[sp] - 0.5 * tot);
+      if (d < bd) {
+        bd = d;
+        best = sp;
+      }
+    }
+    return best;
+  }
   std::string lengths_fn() {
     std::string s;
     s += "  template <bool kSmall, class P>\n"
          "  static __device__ __forceinline__ void lengths(const P& p, const RbSmem& s, const RbCtx& x, int nr, "
-         "bool acc) {\n"
-         "    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, r = tid;\n"
-         "    const bool in = tid < nr;\n";
+         "bool acc) {\n" + thread_vars() +
+         "    const bool in = r < nr;\n";
+    const int sp = split_point();
+    if (pairs()) s += "  if ((warp & 1) == 0) {\n";
+    s += lengths_body(0, sp);
+    if (pairs()) s += "  } else {\n" + lengths_body(sp, F) + "  }\n";
+    s += "  }\n";
+    return s;
+  }
+  std::string lengths_body(int qb, int qe) {
+    std::string s;
     // batches of 8 outputs: every staged load of a batch before its warp sums
     // are stored (a shared store would otherwise order the next loads)
-    for (int q0 = 0; q0 < F; q0 += 8) {
-      const int q1 = std::min(F, q0 + 8);
+    for (int q0 = qb; q0 < qe; q0 += 8) {
+      const int q1 = std::min(qe, q0 + 8);
       s += "  {\n";
       for (int q = q0; q < q1; ++q) s += len_code(q);
       for (int q = q0; q < q1; ++q) s += "    const long long w" + i2s(q) + " = rb_warp_sum<kSmall>(L" + i2s(q) + ");\n";
       s += "    if (lane == 0) {\n";
       for (int q = q0; q < q1; ++q)
-        s += "      s.ws[" + i2s(q * 8) + " + warp] = acc ? s.ws[" + i2s(q * 8) + " + warp] + w" + i2s(q) + " : w" + i2s(q) +
+        s += "      s.ws[" + i2s(q * 8) + " + wi] = acc ? s.ws[" + i2s(q * 8) + " + wi] + w" + i2s(q) + " : w" + i2s(q) +
              ";\n";
       s += "    }\n  }\n";
     }
-    s += "  }\n";
     return s;
   }
 
@@ -361,20 +495,31 @@ struct Gen {
     std::string s;
     s += "  template <bool kSmall, class P>\n"
          "  static __device__ __forceinline__ void emit(const P& p, const RbSmem& s, const RbCtx& x, int64_t c0, "
-         "int nr) {\n"
-         "    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, r = tid;\n"
+         "int nr) {\n" + thread_vars() +
          "    const Common& c = p.c;\n"
          "    const int64_t B = x.B;\n"
-         "    const bool in = tid < nr;\n"
-         "    const int64_t row = c0 + tid;\n"
-         "    bool ovf = false;\n"
+         "    const bool in = r < nr;\n"
+         "    const int64_t row = c0 + r;\n";
+    const int sp = split_point();
+    if (tab_total) s += "    mbar_wait(reinterpret_cast<uint64_t*>(s.tabs), 0u);  // staged tables landed\n";
+    if (pairs()) s += "  if ((warp & 1) == 0) {\n";
+    s += emit_body(0, sp);
+    if (pairs()) s += "  } else {\n" + emit_body(sp, F) + "  }\n";
+    s += "  }\n";
+    return s;
+  }
+  std::string emit_body(int qb, int qe) {
+    std::string s;
+    s += "    bool ovf = false;\n"
          "    unsigned late = 0;\n    (void)late;\n";
     std::vector<int> late_q;
     int n_late = 0;
     // memo registers of the providers
     std::vector<char> is_prov(F, 0);
-    for (int f = 0; f < F; ++f)
+    for (int q = qb; q < qe; ++q) {
+      const int f = v.perm[q];
       if (v.feat[f].emit == 0 && v.feat[f].memo_slot >= 0) is_prov[f] = 1;
+    }
     for (int f = 0; f < F; ++f)
       if (is_prov[f]) s += "    int64_t m" + i2s(f) + " = 0;\n    int32_t ml" + i2s(f) + " = 0;\n";
     // first ids of the canonical list outputs, loaded kAhead outputs before
@@ -382,13 +527,13 @@ struct Gen {
     const int kAhead = env_int("RAP_JIT_AHEAD", 4);  // (experiment knob)
     const int kSegment = 1 << 30;  // (barriers every few outputs to keep warps together: measured, no gain)
     std::vector<int> canon_q;
-    for (int q = 0; q < F; ++q)
+    for (int q = qb; q < qe; ++q)
       if (v.feat[v.perm[q]].emit == 0) canon_q.push_back(q);
     auto prefetch = [&](int q) {
       const RbFeat& R = v.feat[v.perm[q]];
       const std::string Y = "Y" + i2s(q);
       const int sl = slot[R.src[0]];
-      std::string t = "    int64_t pf" + i2s(q) + ";\n    { const RbRow " + Y + " = rb_row(s, " + i2s(sl) +
+      std::string t = "    int64_t pf" + i2s(q) + ";\n    { const RbRow " + Y + " = " + rbrow() + "(s, " + i2s(sl) +
                       ", r);\n      const bool ok = in && " + Y + ".valid && " + Y + ".b > " + Y + ".a;\n";
       if (sl < v.id_slots) {
         // the chunk's ids were bulk-copied into shared memory (rb_stage_ids):
@@ -412,17 +557,18 @@ struct Gen {
       const SProg& pg = v.sprogs[f];
       const Canon& cn = pg.cn;
       const std::string Q = i2s(q), Z = "Z" + Q;
-      std::string t = "    longlong2 pk" + Q + ";\n    { const RbRow " + Z + " = rb_row(s, " + i2s(slot[R.src[0]]) +
+      std::string t = std::string(map2() ? "    MapProbe2 pk" : "    longlong2 pk") + Q + ";\n    { const RbRow " + Z + " = " + rbrow() + "(s, " + i2s(slot[R.src[0]]) +
                       ", r);\n      int64_t u = " + Z + ".valid ? pf" + Q + " : " + lit64(pg.ch.fill) + ";\n";
       t += stages(cn, cn.mask & CB_CLAMP, "u", Z + ".valid", -1, "");
-      t += "      pk" + Q + " = map_first_probe(c.itab, " + lit64(cn.map_a) + ", " + i2s(cn.map_m) + ", u); }\n";
+      t += "      pk" + Q + " = " + (map2() ? "map_first_probe2" : "map_first_probe") + "(c.itab, " + lit64(cn.map_a) + ", " + i2s(cn.map_m) + ", u); }\n";
       return t;
     };
+    if (env_int("RAP_JIT_SKIP", 0) & 16) return s + "  }\n";  // (experiment knob: empty emit phase)
     for (int i = 0; i < (int)canon_q.size() && i < kAhead; ++i) s += prefetch(canon_q[i]);
     for (int i = 0; i < (int)canon_q.size() && i < kProbe; ++i)
       if (has_map(canon_q[i])) s += probe(canon_q[i]);
     int canon_i = 0;
-    for (int q = 0; q < F; ++q) {
+    for (int q = qb; q < qe; ++q) {
       const int f = v.perm[q];
       const RbFeat& R = v.feat[f];
       const SProg& pg = v.sprogs[f];
@@ -442,7 +588,7 @@ struct Gen {
       if (q > 0 && q % kSegment == 0)
         s += std::string("    ") + (gen_dense_ok() ? "rb_sync<true>();" : "rb_sync<false>();") + "\n";
       s += "  {  // output " + Fs + "\n" + len_code(q);
-      s += "    const long long P" + Q + " = s.wb[" + i2s(q * 8) + " + warp] + " +
+      s += "    const long long P" + Q + " = s.wb[" + i2s(q * 8) + " + wi] + " +
            (le1 ? "rb_ballot_excl(L" + Q + " != 0, lane)" : "rb_warp_excl<kSmall>(L" + Q + ", lane)") + ";\n";
       if (is_prov[f]) s += "    ml" + Fs + " = L" + Q + ";\n";
       s += "    stg_s32_if(in, c.lengths + ((int64_t)" + Fs + " * B + row), L" + Q + ");\n";
@@ -464,6 +610,8 @@ struct Gen {
           s += "          rb_store(c, P" + Q + " + j, w);\n        }\n";
         }
         s += "    }\n";
+      } else if (R.emit == 3 && (env_int("RAP_JIT_SKIP", 0) & 8)) {
+        // (experiment knob: NGram ids left out)
       } else if (R.emit == 3 && ngram_fast_ok(q)) {
         // every source memoised by an earlier provider: the present elements
         // shift through an n-register window (selects, R7); rows whose sources
@@ -515,12 +663,11 @@ struct Gen {
       const int q = late_q[k];
       const std::string Q = i2s(q), Fs = i2s(v.perm[q]);
       s += "  if (__any_sync(0xffffffffu, (late >> " + i2s(k) + ") & 1u)) {\n" + len_code(q);
-      s += "    const long long P" + Q + " = s.wb[" + i2s(q * 8) + " + warp] + rb_warp_excl<kSmall>(L" + Q + ", lane);\n";
+      s += "    const long long P" + Q + " = s.wb[" + i2s(q * 8) + " + wi] + rb_warp_excl<kSmall>(L" + Q + ", lane);\n";
       s += "    if ((late >> " + i2s(k) + ") & 1u) rb_fallback(p, s, x.slot, " + Fs + ", r, row, L" + Q + ", P" + Q +
            ");\n  }\n";
     }
     s += "    if (ovf) atomicExch(c.err, 1);  // values_capacity understated (sp_nnz): nothing stored past it\n";
-    s += "  }\n";
     return s;
   }
 
@@ -793,6 +940,7 @@ struct Gen {
     s += "// generated by rap_jit.cpp for one plan (" + i2s(F) + " sparse outputs)\n";
     if (env_int("RAP_JIT_STCS", 1)) s += "#define RAP_ST_CS 1\n";  // streaming output stores (rap_rows_skel.cuh)
     if (env_int("RAP_JIT_LDCS", 0)) s += "#define RAP_LD_CS 1\n";  // (experiment knob)
+    if (env_int("RAP_JIT_STPLAIN", 0)) s += "#define RAP_ST_PLAIN 1\n";  // (experiment knob)
     s += "#include \"rap_rows_interp.cuh\"\n\nnamespace rapk {\n\n";
     bool records = false;  // does any output fall back to the interpreter's functions?
     for (int f = 0; f < F; ++f) records |= v.feat[f].emit != 0;
@@ -800,10 +948,14 @@ struct Gen {
     const std::string dense = dense_fn(&globals);
     std::string body;
     body += "struct JitPolicy {\n";
-    body += "  static constexpr bool kSetupEarly = false;  // records only feed the fallbacks of (4)\n";
+    // setup (before phase 1 when tables are staged): the bulk copies of the
+    // Bucketize tables, awaited at the start of the emit phase
+    body += std::string("  static constexpr bool kSetupEarly = ") + (tab_total ? "true" : "false") + ";\n";
+    body += "  static constexpr bool kPairs = " + std::string(pairs() ? "true" : "false") + ";\n";
     body += "  template <class P>\n"
             "  static __device__ __forceinline__ void setup(const P& p, const RbSmem& s, const RbCtx& x) {\n";
     (void)records;  // the fallbacks rebuild their record from the plan blob (rb_fallback)
+    body += setup_tables();
     body += "  }\n";
     body += dense;
     body += lengths_fn();
@@ -835,8 +987,8 @@ struct Gen {
     body += "};\n\n}  // namespace rapk\n\n";
     s += globals + sample_globals + "\n" + body;
     // one variant per module: 32-bit scans (every offset < 2^31) or 64-bit
-    const char* mb = getenv("RAP_JIT_MINB");  // CTAs per SM the register budget targets (default 2)
-    s += "extern \"C\" __global__ void __launch_bounds__(rapk::kRbChunk, " + std::string(mb ? mb : "2") +
+    const char* mb = getenv("RAP_JIT_MINB");  // CTAs per SM the register budget targets (default 2; pairs 4)
+    s += "extern \"C\" __global__ void __launch_bounds__(rapk::kRbChunk, " + std::string(mb ? mb : (pairs() ? "4" : "2")) +
          ") rap_jit_kernel(const __grid_constant__ "
          "rapk::RbParams<rapk::kRbMaxDense, rapk::kRbMaxCols> p) {\n"
          "  rapk::rows_body<rapk::JitPolicy, rapk::kRbMaxDense, rapk::kRbMaxCols, " +
@@ -893,6 +1045,8 @@ bool nvrtc_cubin(const std::string& src, std::vector<char>* cubin, std::string* 
 std::string jit_generate(const JitPlanView& v) { return Gen(v).source(true); }
 
 int jit_dense_need(const JitPlanView& v) { return Gen(v).dense_need(); }
+
+int jit_table_bytes(const JitPlanView& v) { return Gen(v).table_bytes(); }
 
 bool jit_compile_only(const std::string& src, std::string* log) {
   std::vector<char> cubin;

@@ -205,19 +205,23 @@ template <class P>
 __device__ __noinline__ long long value_tile_ngram(const P& p, int f, int64_t rt, int lane, long long base,
                                                    int32_t* scr);
 
+// Output stores are streaming (st.global.cs, evict-first in L2): written once,
+// never read back by the kernel.
+__device__ __forceinline__ void st_cs64(int64_t* p, int64_t v) { __stcs(reinterpret_cast<long long*>(p), (long long)v); }
+
 // Lengths (int4) and offsets (2 x longlong2) of the lane's 4 rows.
 __device__ __forceinline__ void store_quad(int32_t* lp, int64_t* op, int64_t row, int64_t B, const int32_t* l,
                                            long long lb, const int32_t* e) {
   if (row + 4 <= B && (reinterpret_cast<uintptr_t>(lp) & 15) == 0 && (reinterpret_cast<uintptr_t>(op) & 15) == 0) {
-    *reinterpret_cast<int4*>(lp) = make_int4(l[0], l[1], l[2], l[3]);
-    reinterpret_cast<longlong2*>(op)[0] = make_longlong2(lb + e[0], lb + e[1]);
-    reinterpret_cast<longlong2*>(op)[1] = make_longlong2(lb + e[2], lb + e[3]);
+    __stcs(reinterpret_cast<int4*>(lp), make_int4(l[0], l[1], l[2], l[3]));
+    __stcs(reinterpret_cast<longlong2*>(op), make_longlong2(lb + e[0], lb + e[1]));
+    __stcs(reinterpret_cast<longlong2*>(op) + 1, make_longlong2(lb + e[2], lb + e[3]));
   } else {
 #pragma unroll
     for (int k = 0; k < 4; ++k)
       if (row + k < B) {
-        lp[k] = l[k];
-        op[k] = lb + e[k];
+        __stcs(lp + k, l[k]);
+        st_cs64(op + k, lb + e[k]);
       }
   }
 }
@@ -268,7 +272,7 @@ __device__ __noinline__ long long value_tile_canon(const P& p, const FeatCtx& fc
 #pragma unroll
     for (int k = 0; k < 4; ++k) {
       const long long pos = lb + e[k];
-      if (l[k] == 1 && pos < cap) values[pos] = v[k];
+      if (l[k] == 1 && pos < cap) st_cs64(values + (pos), v[k]);
     }
     if (last && lane == 31) {
       p.c.offsets[(int64_t)p.c.n_sparse_out * B] = base + T;  // total, R17
@@ -315,7 +319,7 @@ __device__ __noinline__ long long value_tile_canon(const P& p, const FeatCtx& fc
 #pragma unroll
     for (int u = 0; u < 4; ++u) {
       const long long pos = base + eb + 32 * u + lane;
-      if (((act >> u) & 1u) && pos < cap) values[pos] = x[u];
+      if (((act >> u) & 1u) && pos < cap) st_cs64(values + (pos), x[u]);
     }
   }
   return T;
@@ -422,7 +426,7 @@ __device__ __noinline__ long long value_chunk_canon(const P& p, const FeatCtx& f
 #pragma unroll
         for (int k = 0; k < 4; ++k) {
           const long long pos = lb + e[k];
-          if (l[k] && pos < cap) values[pos] = v[4 * jj + k];
+          if (l[k] && pos < cap) st_cs64(values + (pos), v[4 * jj + k]);
         }
         if (f == p.c.n_sparse_out - 1 && rt == p.c.tiles_per_feature - 1 && lane == 31) {
           p.c.offsets[(int64_t)p.c.n_sparse_out * B] = run + Tj;  // total, R17
@@ -602,7 +606,7 @@ __device__ __noinline__ long long value_tile_multi(const P& p, const FeatCtx& fc
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
         const long long pos = pos0 + 32 * u;
-        if (((act >> u) & 1u) && pos < cap) values[pos] = x[u];
+        if (((act >> u) & 1u) && pos < cap) st_cs64(values + (pos), x[u]);
       }
     }
   }
@@ -668,8 +672,8 @@ __device__ __noinline__ long long value_tile_generic(const P& p, int f, int64_t 
   for (int g = 0; g < kGroups; ++g) {
     const int64_t row = r0 + 32 * g + lane;
     if (row < B) {
-      lengths[row] = len[g];
-      offsets[row] = base + gb[g] + lex[g];
+      __stcs(lengths + row, len[g]);
+      st_cs64(offsets + row, base + gb[g] + lex[g]);
     }
   }
   if (f == p.c.n_sparse_out - 1 && rt == p.c.tiles_per_feature - 1 && lane == 0) {
@@ -680,7 +684,7 @@ __device__ __noinline__ long long value_tile_generic(const P& p, int f, int64_t 
 #pragma unroll
     for (int g = 0; g < kGroups; ++g) {
       const long long pos = base + gb[g] + lex[g];
-      if (len[g] == 1 && pos < cap) values[pos] = v1[g];
+      if (len[g] == 1 && pos < cap) st_cs64(values + (pos), v1[g]);
     }
     return run;
   }
@@ -743,7 +747,7 @@ __device__ __noinline__ void value_group_general(const P& p, int f, int64_t row0
         v = src_value(p, ops, pg.tab_off, ch, st_r, row0 + r, j);
       }
       const long long pos = gbase + e;
-      if (pos < cap) p.c.values[pos] = v;
+      if (pos < cap) st_cs64(p.c.values + (pos), v);
     }
   }
 }
@@ -1071,8 +1075,8 @@ __device__ __noinline__ long long value_tile_ngram(const P& p, int f, int64_t rt
     const int lx = incl - len;
     const int T = __shfl_sync(0xffffffffu, incl, 31);
     if (inr) {
-      lengths[row] = len;
-      offsets[row] = run + lx;
+      __stcs(lengths + row, len);
+      st_cs64(offsets + row, run + lx);
     }
     if (canon_all && __all_sync(0xffffffffu, slmax <= 1)) {
       // single-id sources: run each source's canonical pipeline once per row,
@@ -1101,13 +1105,13 @@ __device__ __noinline__ long long value_tile_ngram(const P& p, int f, int64_t rt
         }
         const int64_t v = canon1(qp, itab, (int64_t)reduce_M(h, pg.ng.M), true);
         const long long pos = run + lx + j;
-        if (pos < cap) values[pos] = v;
+        if (pos < cap) st_cs64(values + (pos), v);
       }
     } else if (__all_sync(0xffffffffu, len <= 1)) {
       if (len == 1) {
         const long long pos = run + lx;
         const int64_t v = ngram_window(p, pg, ops, st_s + lane, sl_s + lane, 32, row, 0);
-        if (pos < cap) values[pos] = v;
+        if (pos < cap) st_cs64(values + (pos), v);
       }
     } else {
       const int mylex = inr ? lx : INT_MAX;
@@ -1123,7 +1127,7 @@ __device__ __noinline__ long long value_tile_ngram(const P& p, int f, int64_t rt
         if (e < T) {
           const int64_t v = ngram_window(p, pg, ops, st_s + r, sl_s + r, 32, r0 + 32 * g + r, e - lex_r);
           const long long pos = run + e;
-          if (pos < cap) values[pos] = v;
+          if (pos < cap) st_cs64(values + (pos), v);
         }
       }
     }

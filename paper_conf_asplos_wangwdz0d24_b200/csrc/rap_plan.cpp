@@ -131,7 +131,7 @@ struct rap_plan {
   JitModule* jit[2] = {nullptr, nullptr};  // [small] variants
   int jit_state = 0, jit_ctas_per_sm = 0;  // state of the last variant asked for
   int jit_st[2] = {0, 0}, jit_occ[2] = {0, 0};
-  int jit_smem = 0, jit_dense_bytes = 0, jit_id_slots = 0;
+  int jit_smem = 0, jit_dense_bytes = 0, jit_id_slots = 0, jit_tab_bytes = 0;
   double jit_s = 0;
 };
 
@@ -822,12 +822,27 @@ int memo_prefix(const rap_plan* P, const Chain& o, const Canon& qo, const Chain&
 // The generated kernel's shared memory before id staging: the dense warp's
 // 32-row tile after the base-phase totals (rap_jit.cpp tile_offset), no
 // length cache, no shared memo.
+// Warp-pair mode of the generated kernel (rap_rows_skel.cuh kPairs): two
+// threads per row, each evaluating half of the outputs.
+static int jit_pairs(const rap_plan* P) {
+  const char* env = getenv("RAP_JIT_PAIRS");  // "0" / "1": force off / on (experiment knob)
+  if (env && env[0] == '0') return 0;
+  if (env && env[0] == '1') return P->souts.size() >= 2 ? 1 : 0;
+  return 0;
+}
+static int64_t jit_min_rows() {
+  const char* env = getenv("RAP_JIT_SMALL_B");  // (experiment knob)
+  return env ? atoll(env) : (int64_t)1 << 62;
+}
+static int jit_pitch(const rap_plan* P) { return jit_pairs(P) ? kRbPitchPairs : 0; }
 static int jit_base_smem(const rap_plan* P, int dense_bytes) {
-  return rows_smem_bytes(dense_bytes, P->rb_max_fl, P->rb_max_cols, 0, (int)P->souts.size(), 0);
+  return rows_smem_bytes(dense_bytes, P->rb_max_fl, P->rb_max_cols, 0, (int)P->souts.size(), 0, 0, jit_pitch(P), 0,
+                         P->jit_tab_bytes);
 }
 static int jit_tile_bytes(const rap_plan* P) {
-  const int tile = ((2 * ((int)P->souts.size() + 1) * 8 + 15) & ~15) + 32 * (P->d_out | 1) * 4;
-  return (P->d_out > 0 && tile <= P->rb_dense_bytes) ? tile : P->rb_dense_bytes;
+  int r0 = 0;
+  jit_dense_mode((int)P->souts.size(), P->d_out, (int)P->dprogs.size(), P->rb_dense_bytes, jit_pairs(P), &r0);
+  return r0;
 }
 // Staged columns whose chunk ids the generated kernel bulk-copies into shared
 // memory: as many as fit beside its base layout with two CTAs per SM.
@@ -858,6 +873,7 @@ JitPlanView jit_view(const rap_plan* P) {
   v.ops = P->ops.data();
   v.ftab = P->ftab.data();
   v.id_slots = jit_id_slots(P);
+  v.pairs = jit_pairs(P);
   return v;
 }
 
@@ -1179,9 +1195,10 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
     // the dense warp's 32-row tile after the base-phase totals (rap_jit.cpp tile_offset)
     P->jit_dense_bytes = jit_tile_bytes(P);
     P->jit_dense_bytes = std::max(P->jit_dense_bytes, jit_dense_need(jit_view(P)));  // + the emitter's memo rows
+    P->jit_tab_bytes = jit_table_bytes(jit_view(P));
     P->jit_id_slots = jit_id_slots(P);
     P->jit_smem = rows_smem_bytes(P->jit_dense_bytes, P->rb_max_fl, P->rb_max_cols, 0, (int)P->souts.size(), 0,
-                                  P->jit_id_slots);
+                                  P->jit_id_slots, jit_pitch(P), 0, P->jit_tab_bytes);
     if (P->rb_smem > 227 * 1024) P->rb_fits = 0;
   }
   if (P->rb_fits) {
@@ -1604,7 +1621,7 @@ static bool use_rows(const rap_plan* P, int64_t B, const int64_t* nnz) {
 // (<= a quarter of the slots) each gets a dedicated CTA, so small batches run
 // the dense outputs beside the sparse phases rather than after them.
 static void rows_geometry(const rap_plan* P, int64_t B, const int64_t* nnz, int ctas_per_sm, RbGeom* g,
-                          int64_t n_dense_tiles = 0, int budget = 0) {
+                          int64_t n_dense_tiles = 0, int budget = 0, bool one_group = false) {
   const int F = (int)P->souts.size();
   const int bud = budget > 0 ? budget : P->budget;
   int64_t slots = std::max<int64_t>(1, std::min<int64_t>((int64_t)bud * ctas_per_sm, kMaxCtas));
@@ -1617,8 +1634,8 @@ static void rows_geometry(const rap_plan* P, int64_t B, const int64_t* nnz, int 
   const int fg_min = (F + kRbMaxFL - 1) / kRbMaxFL;
   const int64_t nb256 = (B + kRbChunk - 1) / kRbChunk;
   int64_t n_rb, n_fg;
-  if (nb256 * fg_min * 2 >= slots) {
-    n_fg = fg_min;
+  if (one_group || nb256 * fg_min * 2 >= slots) {  // one_group: the generated kernel (one group of every output)
+    n_fg = one_group ? 1 : fg_min;
     n_rb = std::max<int64_t>(1, std::min<int64_t>(slots / n_fg, (B + 31) / 32));
   } else {
     n_rb = nb256;
@@ -1726,7 +1743,11 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
     const bool want_jit = P->kernel_mode == RAP_KERNEL_JIT || P->kernel_mode == RAP_KERNEL_AUTO;
     const bool jit = want_jit && jit_ready(P, small);
     const int iv = small ? 1 : 0;
-    rows_geometry(P, B, raw->sp_nnz, jit ? P->jit_occ[iv] : P->rb_ctas_per_sm, &g);
+    // the generated kernel: one group of every output over as many row blocks
+    // as the budget's slots hold (RAP_JIT_SMALL_B: below this batch size the
+    // interpreted form's feature groups fill the slots instead)
+    const bool jit_geo = jit && (B >= jit_min_rows() || jit_pairs(P));
+    rows_geometry(P, B, raw->sp_nnz, jit ? P->jit_occ[iv] : P->rb_ctas_per_sm, &g, 0, 0, jit_geo);
     if (!jit || !(g.n_fg == 1 && drow0 == 0 && drows == B))  // interpreted form: its geometry, dense CTAs
       rows_geometry(P, B, raw->sp_nnz, P->rb_ctas_per_sm, &g, n_dense);
     g.max_fl = P->rb_max_fl;
@@ -1750,8 +1771,12 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
       g.n_memo = 0;
       g.dense_bytes = P->jit_dense_bytes;
       g.id_slots = P->jit_id_slots;
+      g.pitch = jit_pitch(P);
+      g.feat_recs = 0;
     } else {
       g.len_cache = 1;
+      g.pitch = 0;
+      g.feat_recs = 1;
     }
     int rc = gen ? launch_jit(P->jit[iv], c, g, lr, P->jit_smem, stream) : launch_rows(c, g, lr, P->rb_smem, stream);
     if (rc != 0) return cuda_fail((cudaError_t)rc, gen ? "generated kernel launch" : "row-block kernel launch");

@@ -97,15 +97,16 @@ int rows_dense_bytes(int max_width) {
 }
 
 int rows_smem_bytes(int dense_bytes, int max_fl, int max_cols, int n_memo, int n_sparse_out, int len_cache,
-                    int id_slots) {
+                    int id_slots, int pitch, int feat_recs, int tab_bytes) {
   int o = rb_region0(dense_bytes, n_memo, n_sparse_out);
   o += 2 * rb_align(max_fl * 8 * 8);
   o += rb_align(max_fl * 8);
-  o += rb_align(max_fl * (int)sizeof(RbF));
-  o += rb_align(max_cols * kRbPitch * 4);
+  if (feat_recs) o += rb_align(max_fl * (int)sizeof(RbF));
+  o += rb_align(max_cols * (pitch > 0 ? pitch : kRbPitch) * 4);
   o += rb_align(max_cols * 8 * 4);
   if (len_cache) o += rb_align(max_fl * kRbChunk * 2);
   if (id_slots > 0) o += rb_align(id_slots * 8) + id_slots * kRbIdCap * 8;
+  if (tab_bytes > 0) o = rb_align(o) + tab_bytes;
   return o;
 }
 

@@ -56,7 +56,7 @@ __device__ __forceinline__ int64_t rb_prefetch(const P& p, const RbSmem& s, int 
   const RbF& F = s.feat[fl];
   if (F.emit != 0) return 0;
   const int sl = F.slot[0];
-  const int32_t a = s.off[sl * kRbPitch + r];
+  const int32_t a = s.off[sl * s.pitch + r];
   const bool valid = (s.bm[sl * 8 + (r >> 5)] >> (r & 31)) & 1u;
   if (in && valid && s.len[fl * kRbChunk + r] != 0) return __ldg(p.val[F.src0] + a);
   return F.fill;
@@ -139,7 +139,7 @@ __device__ __forceinline__ void emit_canon(const P& p, const RbSmem& s, const Rb
   const int ma = ms >= 0 ? F.memo_after : -1;
   rb_store(p.c, pos, canon_run<MASK>(F.cn, p.c.itab, x0, valid, ma, memo));
   if (len > 1) {  // only a valid row holds more than one id
-    const int32_t a = s.off[sl * kRbPitch + r];
+    const int32_t a = s.off[sl * s.pitch + r];
     const int64_t* vals = p.val[F.src0] + a;
     for (int32_t j = 1; j < len; ++j)
       rb_store(p.c, pos + j, canon_run<MASK>(F.cn, p.c.itab, __ldg(vals + j), true, -1, memo));
@@ -304,6 +304,7 @@ __device__ __noinline__ void rb_fallback(const P& p, const RbSmem s, const int16
 // warp and output.
 struct InterpPolicy {
   static constexpr bool kSetupEarly = true;  // the records drive (1) as well
+  static constexpr bool kPairs = false;
   static constexpr bool kGenDense = false;
   static constexpr bool kDenseWarp = false;
   template <class P>

@@ -90,6 +90,8 @@ struct RbSmem {
   long long* memo;       // [n_memo][kRbChunk] memoised element 0 (phase 4)
   long long* ide0;       // [id_slots] values index of ids[slot][0] (kRbIdNone: not staged)
   long long* ids;        // [id_slots][kRbIdCap] the chunk's ids of the slot's column
+  int pitch;             // staged offsets per column (g.pitch, default kRbPitch)
+  unsigned char* tabs;   // generated kernel: [mbarrier, 16 B][tables staged at launch] (the layout's end)
 };
 
 constexpr long long kRbIdNone = -(1ll << 61);  // ide0 of a column whose chunk ids were not staged
@@ -113,9 +115,10 @@ __device__ __forceinline__ RbSmem rb_carve(unsigned char* smem, const RbGeom& g,
   s.base = reinterpret_cast<long long*>(smem + o);
   o += rb_align(g.max_fl * 8);
   s.feat = reinterpret_cast<RbF*>(smem + o);
-  o += rb_align(g.max_fl * (int)sizeof(RbF));
+  if (g.feat_recs) o += rb_align(g.max_fl * (int)sizeof(RbF));
+  s.pitch = g.pitch > 0 ? g.pitch : kRbPitch;
   s.off = reinterpret_cast<int32_t*>(smem + o);
-  o += rb_align(g.max_cols * kRbPitch * 4);
+  o += rb_align(g.max_cols * s.pitch * 4);
   s.bm = reinterpret_cast<uint32_t*>(smem + o);
   o += rb_align(g.max_cols * 8 * 4);
   s.len = g.len_cache ? reinterpret_cast<uint16_t*>(smem + o) : nullptr;
@@ -123,6 +126,8 @@ __device__ __forceinline__ RbSmem rb_carve(unsigned char* smem, const RbGeom& g,
   s.ide0 = reinterpret_cast<long long*>(smem + o);
   o += rb_align(g.id_slots * 8);
   s.ids = reinterpret_cast<long long*>(smem + o);
+  o += g.id_slots * kRbIdCap * 8;
+  s.tabs = smem + rb_align(o);
   return s;
 }
 
@@ -178,8 +183,17 @@ struct RbRow {
 
 __device__ __forceinline__ RbRow rb_row(const RbSmem& s, int slot, int r) {
   RbRow x;
-  x.a = s.off[slot * kRbPitch + r];
-  x.b = s.off[slot * kRbPitch + r + 1];
+  x.a = s.off[slot * s.pitch + r];
+  x.b = s.off[slot * s.pitch + r + 1];
+  x.valid = (s.bm[slot * 8 + (r >> 5)] >> (r & 31)) & 1u;
+  return x;
+}
+// Same with the pitch a compile-time constant (generated code).
+template <int PITCH>
+__device__ __forceinline__ RbRow rb_row_p(const RbSmem& s, int slot, int r) {
+  RbRow x;
+  x.a = s.off[slot * PITCH + r];
+  x.b = s.off[slot * PITCH + r + 1];
   x.valid = (s.bm[slot * 8 + (r >> 5)] >> (r & 31)) & 1u;
   return x;
 }
@@ -251,10 +265,10 @@ __device__ __forceinline__ void rb_stage(const P& p, const RbSmem& s, const int1
     const bool wa = bs != nullptr && (reinterpret_cast<uintptr_t>(bs) & 15) == 0;
     const uint32_t wb = wa ? ((uint32_t)(nw * 4) & ~15u) : 0u;
     mbar_arrive_expect(bar, ob + wb);
-    if (ob) bulk_g2s(s.off + k * kRbPitch, src, ob, bar);
+    if (ob) bulk_g2s(s.off + k * s.pitch, src, ob, bar);
     if (wb) bulk_g2s(s.bm + k * 8, bs, wb, bar);
     if (k < n_ids) rb_stage_ids(p.val[col], a0, a1, s.ids + k * kRbIdCap, s.ide0 + k, ibar);
-    for (int i = (int)(ob / 4); i < no; ++i) s.off[k * kRbPitch + i] = __ldg(src + i);
+    for (int i = (int)(ob / 4); i < no; ++i) s.off[k * s.pitch + i] = __ldg(src + i);
     if (bs == nullptr) {
       for (int i = 0; i < nw; ++i) s.bm[k * 8 + i] = 0xffffffffu;
     } else {
@@ -302,7 +316,17 @@ __device__ __forceinline__ void stg_s32(int32_t* p, int32_t v) {
 __device__ __forceinline__ void stg_s64(int64_t* p, int64_t v) {
   asm volatile(RAP_STG ".s64 [%0], %1;" ::"l"(p), "l"(v));
 }
-// Predicated forms (one instruction, no branch around it).
+// Predicated forms (one instruction, no branch around it).  RAP_ST_PLAIN:
+// through the st.global.cs intrinsic instead of volatile asm, so the compiler
+// may move them and the loads of later outputs past each other.
+#ifdef RAP_ST_PLAIN
+__device__ __forceinline__ void stg_s32_if(bool q, int32_t* p, int32_t v) {
+  if (q) __stcs(p, v);
+}
+__device__ __forceinline__ void stg_s64_if(bool q, int64_t* p, int64_t v) {
+  if (q) __stcs(reinterpret_cast<long long*>(p), (long long)v);
+}
+#else
 __device__ __forceinline__ void stg_s32_if(bool q, int32_t* p, int32_t v) {
   asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q " RAP_STG ".s32 [%0], %1;\n\t}" ::"l"(p), "r"(v),
                "r"((unsigned)q));
@@ -311,6 +335,7 @@ __device__ __forceinline__ void stg_s64_if(bool q, int64_t* p, int64_t v) {
   asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q " RAP_STG ".s64 [%0], %1;\n\t}" ::"l"(p), "l"(v),
                "r"((unsigned)q));
 }
+#endif
 __device__ __forceinline__ void rb_store(const Common& c, long long pos, int64_t v) {
   if (pos < c.values_cap)
     stg_s64(c.values + pos, v);
@@ -375,13 +400,13 @@ __device__ __forceinline__ void rb_tile_store_warp(const Common& c, const float*
     if ((reinterpret_cast<uintptr_t>(out) & 15) == 0 && (n & 3) == 0) {
       float4* o4 = reinterpret_cast<float4*>(out);
       const float4* t4 = reinterpret_cast<const float4*>(tile);
-      for (int i = lane; i < (n >> 2); i += 32) o4[i] = t4[i];
+      for (int i = lane; i < (n >> 2); i += 32) __stcs(o4 + i, t4[i]);
     } else {
-      for (int i = lane; i < n; i += 32) out[i] = tile[i];
+      for (int i = lane; i < n; i += 32) __stcs(out + i, tile[i]);
     }
   } else {
     for (int r = 0; r < nr; ++r)
-      for (int cc = lane; cc < width; cc += 32) out[r * c.ld + cc] = tile[r * pitch + cc];
+      for (int cc = lane; cc < width; cc += 32) __stcs(out + r * c.ld + cc, tile[r * pitch + cc]);
   }
 }
 
@@ -419,8 +444,13 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
   // generated kernel with a dense warp: warps 0-6 run the sparse phases over
   // 224-row chunks while warp 7 evaluates the dense outputs of the block
   constexpr bool kDW = Pol::kDenseWarp;
-  constexpr int kTS = kDW ? 224 : kRbChunk;  // sparse threads = rows per chunk
-  constexpr int kWS = kTS / 32;               // sparse warps
+  // generated kernel in warp-pair mode (Pol::kPairs): warps 2w and 2w + 1
+  // evaluate two halves of the outputs over the same 32 rows, so a chunk is
+  // 128 rows and each row has two threads (twice the warps per SM at <= 64
+  // registers)
+  constexpr int kTS = Pol::kPairs ? 128 : (kDW ? 224 : kRbChunk);  // rows per chunk
+  constexpr int kWS = kTS / 32;                                    // row warps (s.ws / s.wb columns)
+  constexpr int kNW = kDW ? 7 : kRbChunk / 32;                     // warps running the sparse phases
   RbCtx x;
   x.F = c.n_sparse_out;
   const RbSmem s = rb_carve(smem, g, x.F);
@@ -575,14 +605,14 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
     const int fmax = s_fmax;
     long long* sT = reinterpret_cast<long long*>(s.dense);  // [fmax + 1]
     long long* sL = sT + (fmax + 1);                          // [fmax + 1]
-    for (int f = tid; f <= fmax; f += kTS) sT[f] = (long long)__ldcg(g.tot + f);
+    for (int f = tid; f <= fmax; f += kNW * 32) sT[f] = (long long)__ldcg(g.tot + f);
     {
       const int nsb = rb / kRbSup, rb0 = nsb * kRbSup;
-      for (int f0 = warp; f0 <= fmax; f0 += 4 * kWS) {
+      for (int f0 = warp; f0 <= fmax; f0 += 4 * kNW) {
         long long v[4];
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
-          const int f = min(f0 + u * kWS, fmax);
+          const int f = min(f0 + u * kNW, fmax);
           long long a = 0;
           if (lane < nsb) a = (long long)__ldcg(g.sup + (int64_t)f * kRbSupMax + lane);
           if (rb0 + lane < rb) a += (long long)__ldcg(g.agg + (int64_t)f * n_rb + rb0 + lane);
@@ -591,7 +621,7 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
           const long long t = rb_warp_sum<kSmall>(v[u]);
-          if (lane == 0 && f0 + u * kWS <= fmax) sL[f0 + u * kWS] = t;
+          if (lane == 0 && f0 + u * kNW <= fmax) sL[f0 + u * kNW] = t;
         }
       }
     }

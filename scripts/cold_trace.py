@@ -112,7 +112,8 @@ def main():
     gw = graph_time(plan, sets[:1], 50, stream)
     gc = graph_time(plan, sets, 50, stream)
     print(f"  graph replay per launch: warm {gw:.2f} us, cold {gc:.2f} us")
-    print(f"{wl} B={B} {tag}: kernel {info.get('kernel')} grid {info['grid']} ctas/sm {info.get('rows_ctas_per_sm')} "
+    print(f"{wl} B={B} {tag}: kernel {info.get('kernel_last')} grid {info['grid']} rows {info.get('rb_rows')} "
+          f"groups {info.get('rb_feature_groups')} jit ctas/sm {info.get('jit_ctas_per_sm')} "
           f"smem {info.get('rows_smem_bytes')}: warm {warm:.2f} us, cold ({nsets} sets) {cold:.2f} us")
     if os.environ.get("STAMPS", "1") == "1":
         stamps(plan, sets[:1], stream, "warm")
