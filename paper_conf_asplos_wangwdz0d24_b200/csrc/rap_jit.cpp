@@ -100,7 +100,9 @@ struct Gen {
   };
   std::vector<BkTab> bktabs;
   int tab_total = 0;  // bytes after the mbarrier
-  static int tab_budget() { return env_int("RAP_JIT_TABS", 1) ? env_int("RAP_JIT_TAB_BYTES", 40 * 1024) : 0; }
+  // 8 KB: the sample tables (whole border tables would cost C2 its second
+  // CTA per SM: measured 41 -> 65 us with 36 KB of tables)
+  static int tab_budget() { return env_int("RAP_JIT_TABS", 1) ? env_int("RAP_JIT_TAB_BYTES", 8 * 1024) : 0; }
   void plan_tables() {
     std::vector<std::pair<int64_t, int>> want;
     for (int f = 0; f < F; ++f) {
