@@ -241,6 +241,14 @@ __device__ __forceinline__ int64_t map_lookup_from2(const int64_t* itab, int64_t
     i = (i + 1) & mask;
   }
 }
+// Branch-free MapId from the first two probe slots: *miss = the key is in
+// neither and neither is empty (the row probes further on the generic path).
+__device__ __forceinline__ int64_t map_sel2(MapProbe2 kv, int64_t x, int64_t dflt, bool* miss) {
+  const bool ha = kv.a.x == x, ea = kv.a.x == INT64_MIN, hb = kv.b.x == x, eb = kv.b.x == INT64_MIN;
+  const bool xm = x == INT64_MIN;  // never a key (R8 reading: the table's empty marker)
+  *miss = !xm && !ha && !ea && !hb && !eb;
+  return xm ? dflt : (ha ? kv.a.y : (ea ? dflt : (hb ? kv.b.y : dflt)));
+}
 __device__ __forceinline__ longlong2 map_first_probe(const int64_t* itab, int64_t a, int m, int64_t x) {
   const longlong2* t = reinterpret_cast<const longlong2*>(itab + a);
   return __ldg(t + (uint32_t)(((uint64_t)x * 0x9E3779B97F4A7C15ull) >> (64 - m)));

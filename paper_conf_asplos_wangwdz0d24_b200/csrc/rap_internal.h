@@ -344,7 +344,7 @@ struct JitModule;  // compiled kernels (opaque)
 //      eight per CTA);
 //   0: no generated dense code (the interpreted dense blocks).
 // *region0 = the shared-memory bytes of region 0 the mode needs.
-inline int jit_dense_tiles(int pairs) { return pairs ? 4 : 8; }  // mode 2: warps with a tile
+inline int jit_dense_tiles(int) { return 8; }  // mode 2: warps with a tile
 inline int jit_dense_mode(int n_sparse_out, int d_out, int n_dprogs, int rb_dense_bytes, int pairs, int* region0) {
   const int off = ((2 * (n_sparse_out + 1) * 8) + 15) & ~15;  // after the base phase's T[f], L[f]
   const int one = 32 * (d_out | 1) * 4;
@@ -353,7 +353,7 @@ inline int jit_dense_mode(int n_sparse_out, int d_out, int n_dprogs, int rb_dens
     *region0 = rb_dense_bytes;
     return 0;
   }
-  if (off + nt * one <= (pairs ? 24 : 48) * 1024) {
+  if (off + nt * one <= 48 * 1024) {
     *region0 = off + nt * one;
     return 2;
   }
@@ -372,14 +372,15 @@ inline int jit_dense_mode(int n_sparse_out, int d_out, int n_dprogs, int rb_dens
 // offset < 2^31; else 64-bit) and compile it with NVRTC for sm_100a (cached
 // per source text in the process).  Returns nullptr and fills *log on failure.
 JitModule* jit_build(const JitPlanView& v, bool small, char* log, int log_cap);
-int jit_occupancy(JitModule* m, int smem_bytes, int* ctas_per_sm);
+int jit_occupancy(JitModule* m, int smem_bytes, int threads, int* ctas_per_sm);
 // Region-0 shared-memory bytes the generated kernel needs beyond the dense
 // tile (the column emitter's memo rows; 0 if none).
 int jit_dense_need(const JitPlanView& v);
 // Shared-memory bytes of the tables the generated kernel stages at launch
 // (Bucketize borders and sub-block maxima; 0: none).
 int jit_table_bytes(const JitPlanView& v);
-int launch_jit(JitModule* m, const Common& c, const RbGeom& g, const LaunchRaw& raw, int smem_bytes, void* stream);
+int launch_jit(JitModule* m, const Common& c, const RbGeom& g, const LaunchRaw& raw, int smem_bytes, int threads,
+               void* stream);
 double jit_compile_seconds(const JitModule* m);
 #endif
 }  // namespace rapk

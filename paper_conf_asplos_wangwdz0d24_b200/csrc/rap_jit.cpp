@@ -430,7 +430,7 @@ struct Gen {
   bool pairs() const { return v.pairs != 0; }
   // MapId: the first two probe slots loaded ahead (RAP_JIT_MAP1=1: one, experiment knob)
   static bool map2() { return env_int("RAP_JIT_MAP1", 0) == 0; }
-  std::string rbrow() const { return "rb_row_p<" + i2s(pairs() ? kRbPitchPairs : kRbChunk + 4) + ">"; }
+  std::string rbrow() const { return "rb_row_p<" + i2s(kRbChunk + 4) + ">"; }
   std::string thread_vars() const {
     if (pairs())
       return "    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, wi = warp >> 1, r = (wi << 5) | lane;\n"
@@ -505,11 +505,242 @@ struct Gen {
     const int sp = split_point();
     if (tab_total) s += "    mbar_wait(reinterpret_cast<uint64_t*>(s.tabs), 0u);  // staged tables landed\n";
     if (pairs()) s += "  if ((warp & 1) == 0) {\n";
-    s += emit_body(0, sp);
-    if (pairs()) s += "  } else {\n" + emit_body(sp, F) + "  }\n";
+    s += batch_ok() ? emit_batched(0, sp) : emit_body(0, sp);
+    if (pairs()) s += "  } else {\n" + (batch_ok() ? emit_batched(sp, F) : emit_body(sp, F)) + "  }\n";
     s += "  }\n";
     return s;
   }
+  // ---- batched emitter (default when every output qualifies) ----
+  // Outputs are emitted in batches of kBatch in processing order, stage by
+  // stage across the batch: (1) lengths, positions, length/offset stores and
+  // the pre-MapId stages of every output, (2) every MapId's first two probe
+  // slots, (3) MapId selects and SigridHash, (4) Bucketize, (5) the value
+  // stores, then the batch's NGram outputs.  Each stage's loads are
+  // independent across the batch and the stages are branch-free, so one
+  // warp's L2 round trips of a batch overlap instead of queueing output by
+  // output (measured: the emit phase tracked one warp's serial chain of
+  // ~0.6 us per output).  Rows a MapId resolves only past its first two
+  // slots, and NGram rows whose sources are not on the register path, are
+  // redone by the generic path after the batches (late rows).
+  static int batch_k() { return std::max(1, env_int("RAP_JIT_BATCH", 8)); }
+  bool batch_ok() const {
+    if (env_int("RAP_JIT_BATCH", 8) == 0 || column_mode()) return false;
+    int lates = 0;
+    for (int q = 0; q < F; ++q) {
+      const int f = v.perm[q];
+      const RbFeat& R = v.feat[f];
+      const SProg& pg = v.sprogs[f];
+      if (R.emit == 0) {
+        if (!pg.cn.ok || R.kind != 0 || max_len(f) > 1) return false;
+      } else if (R.emit == 3) {
+        if (!const_cast<Gen*>(this)->ngram_fast_ok(q)) return false;
+        ++lates;
+      } else {
+        return false;
+      }
+    }
+    return lates <= 32;
+  }
+  // one canonical stage on x, branch-free: a stage that does not apply to a
+  // filled null row (null_mask) keeps the row's value by a select
+  std::string sel_stage(const Canon& q, int bit, const std::string& x, const std::string& full,
+                        const std::string& expr) {
+    if (q.null_mask & bit) return "        " + x + " = " + expr + ";\n";
+    return "        " + x + " = " + full + " ? (int64_t)(" + expr + ") : " + x + ";\n";
+  }
+  std::string bucket_expr(const Canon& q, const std::string& x) {
+    if (q.bk_m >= 64 && q.bk_m % 64 == 0 && q.bk_a % 2 == 0) {
+      const std::string nm = sample_table(q.bk_a, q.bk_m);
+      std::string j0 = "(0";
+      for (int k = 0; k < q.bk_m / 64; ++k) j0 += " + (" + x + " >= " + lit64(v.itab[q.bk_a + 64 * k + 63]) + ")";
+      j0 += ")";
+      const BkTab* t = staged_table(q.bk_a);
+      const std::string smp = t ? "reinterpret_cast<const int64_t*>(s.tabs + " + i2s(16 + t->off_s) + ")" : nm;
+      const std::string brd = (t && t->off_b >= 0) ? "reinterpret_cast<const int64_t*>(s.tabs + " + i2s(16 + t->off_b) + ")"
+                                                   : "c.itab + " + lit64(q.bk_a);
+      const std::string fn = !t ? "upper_bound_64" : (t->off_b >= 0 ? "upper_bound_64s" : "upper_bound_64h");
+      return fn + "(" + brd + ", " + i2s(q.bk_m) + ", " + smp + ", " + j0 + ", " + x + ")";
+    }
+    if (q.bk_m >= 64) {
+      const std::string nm = sample_table(q.bk_a, q.bk_m);
+      return "upper_bound_s8(c.itab + " + lit64(q.bk_a) + ", " + i2s(q.bk_m) + ", " + nm + ", " + i2s(q.bk_m / 8) + ", " + x +
+             ")";
+    }
+    return "upper_bound(c.itab + " + lit64(q.bk_a) + ", " + i2s(q.bk_m) + ", " + x + ")";
+  }
+  std::string emit_batched(int qb, int qe) {
+    std::string s;
+    s += "    bool ovf = false;\n    unsigned late = 0;\n    (void)late;\n";
+    std::vector<char> is_prov(F, 0);
+    for (int q = qb; q < qe; ++q) {
+      const int f = v.perm[q];
+      if (v.feat[f].emit == 0 && v.feat[f].memo_slot >= 0) is_prov[f] = 1;
+    }
+    for (int f = 0; f < F; ++f)
+      if (is_prov[f]) s += "    int64_t m" + i2s(f) + " = 0;\n    int32_t ml" + i2s(f) + " = 0;\n";
+    // late slots: every MapId output and every NGram output
+    std::vector<int> late_slot(F, -1), late_q;
+    for (int q = qb; q < qe; ++q) {
+      const int f = v.perm[q];
+      const bool lt = v.feat[f].emit == 3;
+      if (lt) {
+        late_slot[q] = (int)late_q.size();
+        late_q.push_back(q);
+      }
+    }
+    auto prefetch = [&](int q) {
+      const RbFeat& R = v.feat[v.perm[q]];
+      const std::string Y = "Y" + i2s(q);
+      return "    int64_t pf" + i2s(q) + ";\n    { const RbRow " + Y + " = " + rbrow() + "(s, " + i2s(slot[R.src[0]]) +
+             ", r);\n      const bool ok = in && " + Y + ".valid && " + Y + ".b > " + Y + ".a;\n      pf" + i2s(q) +
+             " = rap_ldin(ok ? p.val[" + i2s(R.src[0]) + "] + " + Y + ".a : c.itab); }\n";
+    };
+    const int K = batch_k();
+    std::vector<std::vector<int>> batches;
+    for (int q0 = qb; q0 < qe; q0 += K) {
+      std::vector<int> b;
+      for (int q = q0; q < std::min(qe, q0 + K); ++q) b.push_back(q);
+      batches.push_back(b);
+    }
+    auto pf_batch = [&](const std::vector<int>& b) {
+      std::string t;
+      for (int q : b)
+        if (v.feat[v.perm[q]].emit == 0) t += prefetch(q);
+      return t;
+    };
+    if (!batches.empty()) s += pf_batch(batches[0]);
+    for (size_t bi = 0; bi < batches.size(); ++bi) {
+      const std::vector<int>& b = batches[bi];
+      if (bi + 1 < batches.size()) s += pf_batch(batches[bi + 1]);  // the next batch's ids in flight
+      s += "  {  // batch of outputs";
+      for (int q : b) s += " " + i2s(v.perm[q]);
+      s += "\n";
+      std::vector<int> canon, ngram;
+      for (int q : b) (v.feat[v.perm[q]].emit == 0 ? canon : ngram).push_back(q);
+      // (1) lengths, positions, length/offset stores, fill, Clamp
+      for (int q : canon) {
+        const int f = v.perm[q];
+        const SProg& pg = v.sprogs[f];
+        const Canon& cn = pg.cn;
+        const std::string Q = i2s(q), Fs = i2s(f), X = "X" + Q + "_0";
+        const int ma = is_prov[f] ? memo_point(v.feat[f], cn) : -1;
+        s += len_code(q);
+        s += "    const long long P" + Q + " = s.wb[" + i2s(q * 8) + " + wi] + rb_ballot_excl(L" + Q + " != 0, lane);\n";
+        if (is_prov[f]) s += "    ml" + Fs + " = L" + Q + ";\n";
+        s += "    stg_s32_if(in, c.lengths + ((int64_t)" + Fs + " * B + row), L" + Q + ");\n";
+        s += "    stg_s64_if(in, c.offsets + ((int64_t)" + Fs + " * B + row), P" + Q + ");\n";
+        if (f == F - 1) s += "    stg_s64_if(in && row == B - 1, c.offsets + (int64_t)" + i2s(F) + " * B, P" + Q + " + L" + Q + ");\n";
+        s += "    ovf |= P" + Q + " + L" + Q + " > c.values_cap;\n";
+        s += "    int64_t v" + Q + " = " + X + ".valid ? pf" + Q + " : " + lit64(pg.ch.fill) + ";\n";
+        if (ma == 16) s += "    m" + Fs + " = v" + Q + ";\n";
+        if (cn.mask & CB_CLAMP) {
+          s += sel_stage(cn, CB_CLAMP, "v" + Q, X + ".valid",
+                         "v" + Q + " < " + lit64(cn.lo) + " ? " + lit64(cn.lo) + " : (v" + Q + " > " + lit64(cn.hi) + " ? " +
+                             lit64(cn.hi) + " : v" + Q + ")");
+          if (ma == CB_CLAMP) s += "    m" + Fs + " = v" + Q + ";\n";
+        }
+      }
+      // (2) MapId probes
+      for (int q : canon) {
+        const Canon& cn = v.sprogs[v.perm[q]].cn;
+        if (!(cn.mask & CB_MAPID)) continue;
+        s += "    const MapProbe2 pk" + i2s(q) + " = map_first_probe2(c.itab, " + lit64(cn.map_a) + ", " + i2s(cn.map_m) +
+             ", v" + i2s(q) + ");\n";
+      }
+      // (3) MapId selects, SigridHash
+      for (int q : canon) {
+        const int f = v.perm[q];
+        const Canon& cn = v.sprogs[f].cn;
+        const std::string Q = i2s(q), Fs = i2s(f), X = "X" + Q + "_0";
+        const int ma = is_prov[f] ? memo_point(v.feat[f], cn) : -1;
+        if (cn.mask & CB_MAPID) {
+          s += "    { bool mi;\n      int64_t mv = map_sel2(pk" + Q + ", v" + Q + ", " + lit64(cn.map_def) + ", &mi);\n";
+          const bool all = (cn.null_mask & CB_MAPID) != 0;
+          // rows whose key is past the first two slots probe on (warp-uniform test)
+          s += "      if (__any_sync(0xffffffffu, mi)) mv = mi ? map_lookup_from2(c.itab, " + lit64(cn.map_a) + ", " +
+               i2s(cn.map_m) + ", " + lit64(cn.map_def) + ", v" + Q + ", pk" + Q + ") : mv;\n";
+          s += "      v" + Q + " = " + (all ? "mv" : X + ".valid ? mv : v" + Q) + "; }\n";
+          if (ma == CB_MAPID) s += "    m" + Fs + " = v" + Q + ";\n";
+        }
+        if (cn.mask & CB_SIGRID) {
+          s += sel_stage(cn, CB_SIGRID, "v" + Q, X + ".valid",
+                         "(int64_t)reduce_M(splitmix_H(" + litu64(cn.hs) + " ^ (uint64_t)v" + Q + "), " + lit64(cn.M) + ")");
+          if (ma == CB_SIGRID) s += "    m" + Fs + " = v" + Q + ";\n";
+        }
+      }
+      // (4) Bucketize, (5) value stores
+      for (int q : canon) {
+        const int f = v.perm[q];
+        const Canon& cn = v.sprogs[f].cn;
+        const std::string Q = i2s(q), Fs = i2s(f), X = "X" + Q + "_0";
+        const int ma = is_prov[f] ? memo_point(v.feat[f], cn) : -1;
+        if (cn.mask & CB_BUCKET) {
+          s += sel_stage(cn, CB_BUCKET, "v" + Q, X + ".valid", bucket_expr(cn, "v" + Q));
+          if (ma == CB_BUCKET) s += "    m" + Fs + " = v" + Q + ";\n";
+        }
+      }
+      for (int q : canon) {
+        const std::string Q = i2s(q);
+        s += "    stg_s64_if(L" + Q + " > 0 && P" + Q + " < c.values_cap, c.values + P" + Q + ", v" + Q + ");\n";
+      }
+      // the batch's NGram outputs (their providers' memo words are final)
+      for (int q : ngram) {
+        const int f = v.perm[q];
+        const RbFeat& R = v.feat[f];
+        const SProg& pg = v.sprogs[f];
+        const std::string Q = i2s(q), Fs = i2s(f);
+        const int n = R.n, Kk = R.k;
+        s += "  {  // output " + Fs + " (NGram)\n" + len_code(q);
+        s += "    const long long P" + Q + " = s.wb[" + i2s(q * 8) + " + wi] + " +
+             (max_len(f) <= 1 ? "rb_ballot_excl(L" + Q + " != 0, lane)" : "rb_warp_excl<kSmall>(L" + Q + ", lane)") + ";\n";
+        s += "    stg_s32_if(in, c.lengths + ((int64_t)" + Fs + " * B + row), L" + Q + ");\n";
+        s += "    stg_s64_if(in, c.offsets + ((int64_t)" + Fs + " * B + row), P" + Q + ");\n";
+        if (f == F - 1) s += "    stg_s64_if(in && row == B - 1, c.offsets + (int64_t)" + i2s(F) + " * B, P" + Q + " + L" + Q + ");\n";
+        s += "    ovf |= P" + Q + " + L" + Q + " > c.values_cap;\n";
+        std::string cond;
+        for (int i = 0; i < Kk; ++i) {
+          const int qp = R.prov[i], fp = v.perm[qp];
+          const std::string l = "l" + Q + "_" + i2s(i);
+          if (i) cond += " && ";
+          cond += "(" + l + " <= 1 && (" + l + " == 0 || ml" + i2s(fp) + " >= 1))";
+        }
+        s += "    {\n      const bool fast = " + cond + ";\n      int32_t cnt = 0;\n";
+        for (int j = 0; j < n; ++j) s += "      uint64_t w" + i2s(j) + " = 0;\n";
+        for (int i = 0; i < Kk; ++i) {
+          const int fp = v.perm[R.prov[i]];
+          const std::string pr = "pr" + i2s(i);
+          s += "      const bool " + pr + " = l" + Q + "_" + i2s(i) + " != 0;\n";
+          for (int j = 0; j + 1 < n; ++j) s += "      w" + i2s(j) + " = " + pr + " ? w" + i2s(j + 1) + " : w" + i2s(j) + ";\n";
+          s += "      w" + i2s(n - 1) + " = " + pr + " ? (uint64_t)m" + i2s(fp) + " : w" + i2s(n - 1) + ";\n";
+          s += "      cnt += " + pr + ";\n";
+          if (i + 1 >= n) {
+            s += "      {\n        uint64_t h = " + litu64(pg.ng.hsalt) + ";\n";
+            for (int j = 0; j < n; ++j) s += "        h = splitmix_H(h ^ w" + i2s(j) + ");\n";
+            s += "        int64_t v = (int64_t)reduce_M(h, " + lit64(pg.ng.M) + ");\n";
+            s += stages(pg.cn, pg.cn.mask, "v", "true", -1, "");
+            s += "        const long long at = P" + Q + " + (cnt - " + i2s(n) + ");\n";
+            s += "        stg_s64_if(fast && " + pr + " && cnt >= " + i2s(n) + " && cnt - " + i2s(n) + " < L" + Q +
+                 " && at < c.values_cap, c.values + at, v);\n      }\n";
+          }
+        }
+        s += "      if (!fast && L" + Q + " > 0) late |= 1u << " + i2s(late_slot[q]) + ";\n    }\n  }\n";
+      }
+      s += "  }\n";
+    }
+    // late rows: the generic path (warp-uniform test per output)
+    for (int k = 0; k < (int)late_q.size(); ++k) {
+      const int q = late_q[k];
+      const int f = v.perm[q];
+      const std::string Q = i2s(q), Fs = i2s(f);
+      s += "  if (__any_sync(0xffffffffu, (late >> " + i2s(k) + ") & 1u)) {\n" + len_code(q);
+      s += "    const long long P" + Q + " = s.wb[" + i2s(q * 8) + " + wi] + " +
+           (max_len(f) <= 1 ? "rb_ballot_excl(L" + Q + " != 0, lane)" : "rb_warp_excl<kSmall>(L" + Q + ", lane)") + ";\n";
+      s += "    if ((late >> " + i2s(k) + ") & 1u) rb_fallback(p, s, x.slot, " + Fs + ", r, row, L" + Q + ", P" + Q + ");\n  }\n";
+    }
+    s += "    if (ovf) atomicExch(c.err, 1);  // values_capacity understated (sp_nnz): nothing stored past it\n";
+    return s;
+  }
+
   std::string emit_body(int qb, int qe) {
     std::string s;
     s += "    bool ovf = false;\n"
@@ -954,6 +1185,7 @@ struct Gen {
     // Bucketize tables, awaited at the start of the emit phase
     body += std::string("  static constexpr bool kSetupEarly = ") + (tab_total ? "true" : "false") + ";\n";
     body += "  static constexpr bool kPairs = " + std::string(pairs() ? "true" : "false") + ";\n";
+    body += "  static constexpr int kThreads = " + i2s(pairs() ? 2 * kRbChunk : kRbChunk) + ";\n";
     body += "  template <class P>\n"
             "  static __device__ __forceinline__ void setup(const P& p, const RbSmem& s, const RbCtx& x) {\n";
     (void)records;  // the fallbacks rebuild their record from the plan blob (rb_fallback)
@@ -990,7 +1222,7 @@ struct Gen {
     s += globals + sample_globals + "\n" + body;
     // one variant per module: 32-bit scans (every offset < 2^31) or 64-bit
     const char* mb = getenv("RAP_JIT_MINB");  // CTAs per SM the register budget targets (default 2; pairs 4)
-    s += "extern \"C\" __global__ void __launch_bounds__(rapk::kRbChunk, " + std::string(mb ? mb : (pairs() ? "4" : "2")) +
+    s += "extern \"C\" __global__ void __launch_bounds__(" + i2s(pairs() ? 2 * kRbChunk : kRbChunk) + ", " + std::string(mb ? mb : "2") +
          ") rap_jit_kernel(const __grid_constant__ "
          "rapk::RbParams<rapk::kRbMaxDense, rapk::kRbMaxCols> p) {\n"
          "  rapk::rows_body<rapk::JitPolicy, rapk::kRbMaxDense, rapk::kRbMaxCols, " +
@@ -1089,11 +1321,11 @@ JitModule* jit_build(const JitPlanView& v, bool small, char* log, int log_cap) {
 
 double jit_compile_seconds(const JitModule* m) { return m ? m->compile_s : 0.0; }
 
-int jit_occupancy(JitModule* m, int smem_bytes, int* ctas_per_sm) {
+int jit_occupancy(JitModule* m, int smem_bytes, int threads, int* ctas_per_sm) {
   const void* k = reinterpret_cast<const void*>(m->k);
   const int rc = ensure_dyn_smem(k, smem_bytes);
   if (rc != 0) return rc;
-  return (int)cudaOccupancyMaxActiveBlocksPerMultiprocessor(ctas_per_sm, k, kRbChunk, smem_bytes);
+  return (int)cudaOccupancyMaxActiveBlocksPerMultiprocessor(ctas_per_sm, k, threads, smem_bytes);
 }
 
 // Same parameter block as rap_rows.cu's kernel (RbParams<kRbMaxDense, kRbMaxCols>).
@@ -1107,7 +1339,8 @@ struct JitParams {
   const uint32_t* svalid[kRbMaxCols];
 };
 
-int launch_jit(JitModule* m, const Common& c, const RbGeom& g, const LaunchRaw& raw, int smem_bytes, void* stream) {
+int launch_jit(JitModule* m, const Common& c, const RbGeom& g, const LaunchRaw& raw, int smem_bytes, int threads,
+               void* stream) {
   if (raw.n_dense > kRbMaxDense || raw.n_sparse > kRbMaxCols) return (int)cudaErrorInvalidValue;
   const void* k = reinterpret_cast<const void*>(m->k);
   const int rc = ensure_dyn_smem(k, smem_bytes);
@@ -1127,7 +1360,7 @@ int launch_jit(JitModule* m, const Common& c, const RbGeom& g, const LaunchRaw& 
   }
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)(g.n_rb * g.n_fg + g.n_dcta));
-  cfg.blockDim = dim3(kRbChunk);
+  cfg.blockDim = dim3((unsigned)threads);
   cfg.dynamicSmemBytes = smem_bytes;
   cfg.stream = reinterpret_cast<cudaStream_t>(stream);
   cudaLaunchAttribute attr[1];

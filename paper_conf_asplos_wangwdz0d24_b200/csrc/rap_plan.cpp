@@ -834,7 +834,8 @@ static int64_t jit_min_rows() {
   const char* env = getenv("RAP_JIT_SMALL_B");  // (experiment knob)
   return env ? atoll(env) : (int64_t)1 << 62;
 }
-static int jit_pitch(const rap_plan* P) { return jit_pairs(P) ? kRbPitchPairs : 0; }
+static int jit_pitch(const rap_plan*) { return 0; }
+static int jit_threads(const rap_plan* P) { return jit_pairs(P) ? 2 * kRbChunk : kRbChunk; }
 static int jit_base_smem(const rap_plan* P, int dense_bytes) {
   return rows_smem_bytes(dense_bytes, P->rb_max_fl, P->rb_max_cols, 0, (int)P->souts.size(), 0, 0, jit_pitch(P), 0,
                          P->jit_tab_bytes);
@@ -1584,7 +1585,7 @@ static bool jit_ready(rap_plan* P, bool small) {
       char log[2048] = {0};
       JitModule* m = jit_build(jit_view(P), small, log, (int)sizeof(log));
       int occ = 0;
-      if (m && jit_occupancy(m, P->jit_smem, &occ) == 0 && occ >= 1) {
+      if (m && jit_occupancy(m, P->jit_smem, jit_threads(P), &occ) == 0 && occ >= 1) {
         P->jit[i] = m;
         P->jit_occ[i] = occ;
         P->jit_s += jit_compile_seconds(m);
@@ -1778,7 +1779,8 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
       g.pitch = 0;
       g.feat_recs = 1;
     }
-    int rc = gen ? launch_jit(P->jit[iv], c, g, lr, P->jit_smem, stream) : launch_rows(c, g, lr, P->rb_smem, stream);
+    int rc = gen ? launch_jit(P->jit[iv], c, g, lr, P->jit_smem, jit_threads(P), stream)
+                 : launch_rows(c, g, lr, P->rb_smem, stream);
     if (rc != 0) return cuda_fail((cudaError_t)rc, gen ? "generated kernel launch" : "row-block kernel launch");
     P->kernel_last = gen ? RAP_KERNEL_JIT : RAP_KERNEL_ROWS;
     P->rb_last_n_rb = g.n_rb;

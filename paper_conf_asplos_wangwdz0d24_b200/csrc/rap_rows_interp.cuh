@@ -305,6 +305,7 @@ __device__ __noinline__ void rb_fallback(const P& p, const RbSmem s, const int16
 struct InterpPolicy {
   static constexpr bool kSetupEarly = true;  // the records drive (1) as well
   static constexpr bool kPairs = false;
+  static constexpr int kThreads = kRbChunk;
   static constexpr bool kGenDense = false;
   static constexpr bool kDenseWarp = false;
   template <class P>

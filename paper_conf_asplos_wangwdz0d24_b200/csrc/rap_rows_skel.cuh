@@ -444,13 +444,14 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
   // generated kernel with a dense warp: warps 0-6 run the sparse phases over
   // 224-row chunks while warp 7 evaluates the dense outputs of the block
   constexpr bool kDW = Pol::kDenseWarp;
-  // generated kernel in warp-pair mode (Pol::kPairs): warps 2w and 2w + 1
-  // evaluate two halves of the outputs over the same 32 rows, so a chunk is
-  // 128 rows and each row has two threads (twice the warps per SM at <= 64
-  // registers)
-  constexpr int kTS = Pol::kPairs ? 128 : (kDW ? 224 : kRbChunk);  // rows per chunk
+  // generated kernel in warp-pair mode (Pol::kPairs, 512-thread CTAs): warps
+  // 2w and 2w + 1 evaluate two halves of the outputs over the same 32 rows of
+  // a 224-row chunk, so each row has two threads (twice the warps per SM at
+  // <= 64 registers, the row blocks as in the one-thread-per-row form)
+  constexpr int kT = Pol::kThreads;                                 // threads per CTA
+  constexpr int kTS = Pol::kPairs ? 224 : (kDW ? 224 : kRbChunk);  // rows per chunk
   constexpr int kWS = kTS / 32;                                    // row warps (s.ws / s.wb columns)
-  constexpr int kNW = kDW ? 7 : kRbChunk / 32;                     // warps running the sparse phases
+  constexpr int kNW = kDW ? 7 : kT / 32;                           // warps running the sparse phases
   RbCtx x;
   x.F = c.n_sparse_out;
   const RbSmem s = rb_carve(smem, g, x.F);
@@ -485,7 +486,7 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
     s_fmax = 0;
     if (blockIdx.x == 0 && x.F == 0 && !c.chain && c.offsets) c.offsets[0] = 0;  // no sparse outputs (R17)
   }
-  for (int i = tid; i < (MS + 63) / 64; i += kRbChunk) s_mask[i] = 0ull;
+  for (int i = tid; i < (MS + 63) / 64; i += kT) s_mask[i] = 0ull;
   __syncthreads();
   // the raw columns the group reads -> staged slots (one group of every
   // output: the plan's column mask, no per-output loads)
@@ -517,7 +518,7 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
   // before the chunk's ids are emitted
   const int n_ids = min(n_cols, g.id_slots);
   if (tid == 0) mbar_init(&s_ibar, (uint32_t)max(n_ids, 1));
-  for (int col = tid; col < MS; col += kRbChunk) {
+  for (int col = tid; col < MS; col += kT) {
     const unsigned long long m = s_mask[col >> 6];
     int before = __popcll(m & ((1ull << (col & 63)) - 1ull));
     for (int i = 0; i < (col >> 6); ++i) before += __popcll(s_mask[i]);
@@ -690,9 +691,9 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
   __syncthreads();
   if (s_last) {
     __threadfence();
-    for (int f = tid; f < x.F; f += kRbChunk) g.tot[f] = 0ull;
+    for (int f = tid; f < x.F; f += kT) g.tot[f] = 0ull;
     const int nsb_all = (n_rb + kRbSup - 1) / kRbSup;
-    for (int i = tid; i < x.F * nsb_all; i += kRbChunk) g.sup[(int64_t)(i / nsb_all) * kRbSupMax + i % nsb_all] = 0ull;
+    for (int i = tid; i < x.F * nsb_all; i += kT) g.sup[(int64_t)(i / nsb_all) * kRbSupMax + i % nsb_all] = 0ull;
     if (tid == 0) {
       g.sched[0] = 0ull;
       g.sched[2] = 0ull;
