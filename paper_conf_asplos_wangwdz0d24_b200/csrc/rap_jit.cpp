@@ -504,12 +504,167 @@ struct Gen {
          "    const int64_t row = c0 + r;\n";
     const int sp = split_point();
     if (tab_total) s += "    mbar_wait(reinterpret_cast<uint64_t*>(s.tabs), 0u);  // staged tables landed\n";
+    const LoopPlan lp = loop_plan();
+    if (lp.ok) return s + emit_loop(lp) + "  }\n";
     if (pairs()) s += "  if ((warp & 1) == 0) {\n";
     s += batch_ok() ? emit_batched(0, sp) : emit_body(0, sp);
     if (pairs()) s += "  } else {\n" + (batch_ok() ? emit_batched(sp, F) : emit_body(sp, F)) + "  }\n";
     s += "  }\n";
     return s;
   }
+  // ---- loop emitter (rap_rows_skel.cuh jl_*): the outputs as rows of
+  // __constant__ tables, NGram units (k providers + the NGram) then single
+  // canonical outputs in two loops, so the code a warp streams through in the
+  // emit phase is two short loop bodies (ncu: instruction-fetch stalls were
+  // 40% of the straight-line emitters' warp samples) ----
+  struct LoopPlan {
+    bool ok = false;
+    int K = 0, N = 0;
+    std::vector<int> canon;  // processing indices: unit u's providers at [u*K, u*K+K), then the singles
+    std::vector<int> units;  // processing index of each unit's NGram
+    std::vector<int64_t> bk; // distinct Bucketize border offsets (rows of the level-0 / sample tables)
+  };
+  LoopPlan loop_plan() {
+    LoopPlan L;
+    // opt-in (RAP_JIT_LOOP=1): measured on C2, the loops' serial chains cost
+    // more than the instruction fetches they save (emit phase 19 -> 28 us)
+    if (env_int("RAP_JIT_LOOP", 0) == 0 || pairs() || column_mode()) return L;
+    std::vector<char> used(F, 0);
+    for (int q = 0; q < F; ++q) {
+      const int f = v.perm[q];
+      const RbFeat& R = v.feat[f];
+      const SProg& pg = v.sprogs[f];
+      if (R.emit == 0) {
+        const Canon& cn = pg.cn;
+        if (!cn.ok || R.kind != 0 || max_len(f) > 1) return L;
+        if (cn.mask & CB_BUCKET) {
+          if (!(cn.bk_m >= 64 && cn.bk_m <= 1024 && cn.bk_m % 64 == 0 && cn.bk_a % 2 == 0)) return L;
+          if (std::find(L.bk.begin(), L.bk.end(), cn.bk_a) == L.bk.end()) L.bk.push_back(cn.bk_a);
+        }
+      } else if (R.emit == 3) {
+        if (!ngram_fast_ok(q) || pg.cn.mask != 0 || R.k > kMaxNgramK || R.n > R.k) return L;
+        if (L.K == 0) {
+          L.K = R.k;
+          L.N = R.n;
+        }
+        if (R.k != L.K || R.n != L.N) return L;
+        for (int i = 0; i < R.k; ++i)
+          if (R.prov[i] != q - R.k + i || used[q - R.k + i]) return L;
+        for (int i = 0; i < R.k; ++i) used[q - R.k + i] = 1;
+        L.units.push_back(q);
+      } else {
+        return L;
+      }
+    }
+    if ((int)L.units.size() > 32) return L;
+    for (int u : L.units)
+      for (int i = 0; i < L.K; ++i) L.canon.push_back(u - L.K + i);
+    for (int q = 0; q < F; ++q)
+      if (v.feat[v.perm[q]].emit == 0 && !used[q]) L.canon.push_back(q);
+    L.ok = true;
+    return L;
+  }
+  std::string loop_tables(const LoopPlan& L) {
+    std::string s;
+    s += "__constant__ rapk::JLCanon kJC[" + i2s(std::max<size_t>(1, L.canon.size())) + "] = {\n";
+    for (int q : L.canon) {
+      const int f = v.perm[q];
+      const RbFeat& R = v.feat[f];
+      const SProg& pg = v.sprogs[f];
+      const Canon& cn = pg.cn;
+      int bk_row = 0;
+      if (cn.mask & CB_BUCKET) bk_row = (int)(std::find(L.bk.begin(), L.bk.end(), cn.bk_a) - L.bk.begin());
+      const int mp = R.memo_slot >= 0 ? memo_point(R, cn) : -1;
+      s += "  {" + lit64(pg.ch.fill) + ", " + lit64(cn.lo) + ", " + lit64(cn.hi) + ", " + lit64(cn.map_def) + ", " +
+           lit64(cn.map_a) + ", " + lit64(cn.bk_a) + ", " + lit64(cn.M) + ", " + litu64(cn.hs) + ", " +
+           i2s(slot[R.src[0]]) + ", " + i2s(R.src[0]) + ", " + i2s(f) + ", " + i2s(q) + ", " + i2s(R.cap[0]) + ", " +
+           i2s(R.ncap[0]) + ", " + i2s(cn.mask) + ", " + i2s(cn.null_mask) + ", " + i2s(cn.map_m) + ", " + i2s(cn.bk_m) +
+           ", " + i2s(bk_row) + ", " + i2s(mp < 0 ? 0 : mp) + ", " + i2s(f == F - 1 ? 1 : 0) + ", 0},\n";
+    }
+    if (L.canon.empty()) s += "  {}\n";
+    s += "};\n";
+    const int K = std::max(1, L.K);
+    s += "__constant__ rapk::JLNgram<" + i2s(K) + "> kJN[" + i2s(std::max<size_t>(1, L.units.size())) + "] = {\n";
+    for (int q : L.units) {
+      const int f = v.perm[q];
+      const RbFeat& R = v.feat[f];
+      const SProg& pg = v.sprogs[f];
+      std::string sl, cp, nc;
+      for (int i = 0; i < K; ++i) {
+        sl += (i ? ", " : "") + i2s(slot[R.src[i]]);
+        cp += (i ? ", " : "") + i2s(R.cap[i]);
+        nc += (i ? ", " : "") + i2s(R.ncap[i]);
+      }
+      s += "  {" + litu64(pg.ng.hsalt) + ", " + lit64(pg.ng.M) + ", " + i2s(f) + ", " + i2s(q) + ", " + i2s(R.out_cap) +
+           ", " + i2s(f == F - 1 ? 1 : 0) + ", {" + sl + "}, {" + cp + "}, {" + nc + "}},\n";
+    }
+    if (L.units.empty()) s += "  {}\n";
+    s += "};\n";
+    const int NB = std::max<int>(1, (int)L.bk.size());
+    s += "__constant__ long long kJL0[" + i2s(NB) + " * 16] = {";
+    for (int b = 0; b < NB; ++b)
+      for (int k = 0; k < 16; ++k) {
+        long long x = INT64_MAX;
+        if (b < (int)L.bk.size()) {
+          int m = 0;
+          for (int f = 0; f < F; ++f)
+            if ((v.sprogs[f].cn.mask & CB_BUCKET) && v.sprogs[f].cn.bk_a == L.bk[b]) m = v.sprogs[f].cn.bk_m;
+          if (k < m / 64) x = v.itab[L.bk[b] + 64 * k + 63];
+        }
+        s += (b || k ? ", " : "") + lit64(x);
+      }
+    s += "};\n";
+    s += "__device__ const int64_t* const kJS[" + i2s(NB) + "] = {";
+    for (int b = 0; b < NB; ++b) {
+      std::string nm = "nullptr";
+      if (b < (int)L.bk.size()) {
+        int m = 0;
+        for (int f = 0; f < F; ++f)
+          if ((v.sprogs[f].cn.mask & CB_BUCKET) && v.sprogs[f].cn.bk_a == L.bk[b]) m = v.sprogs[f].cn.bk_m;
+        nm = sample_table(L.bk[b], m);
+      }
+      s += (b ? ", " : "") + nm;
+    }
+    s += "};\n";
+    return s;
+  }
+  std::string emit_loop(const LoopPlan& L) {
+    const int NU = (int)L.units.size(), NC = (int)L.canon.size(), K = L.K, N = L.N;
+    std::string s;
+    s += "    bool ovf = false;\n    unsigned late = 0;\n";
+    if (NU > 0) {
+      const std::string KS = i2s(K), NS = i2s(N);
+      s += "    int64_t pf[" + KS + "];\n#pragma unroll\n    for (int i = 0; i < " + KS +
+           "; ++i) pf[i] = jl_prefetch(p, s, kJC[i], r, in);\n";
+      s += "#pragma unroll 1\n    for (int u = 0; u < " + i2s(NU) + "; ++u) {\n";
+      s += "      int64_t pn[" + KS + "];\n#pragma unroll\n      for (int i = 0; i < " + KS + "; ++i) pn[i] = u + 1 < " +
+           i2s(NU) + " ? jl_prefetch(p, s, kJC[(u + 1) * " + KS + " + i], r, in) : 0;\n";
+      s += "      int64_t mm[" + KS + "];\n      int32_t ml[" + KS + "];\n";
+      s += "#pragma unroll\n      for (int i = 0; i < " + KS + "; ++i) {\n        mm[i] = 0;\n"
+           "        jl_canon<kSmall>(p, s, kJC[u * " + KS + " + i], kJL0, kJS, r, wi, lane, in, row, B, pf[i], &mm[i], &ml[i], ovf);\n      }\n";
+      s += "      if (jl_ngram<" + KS + ", " + NS + ", kSmall>(p, s, kJN[u], mm, ml, r, wi, lane, in, row, B, ovf)) late |= 1u << u;\n";
+      s += "#pragma unroll\n      for (int i = 0; i < " + KS + "; ++i) pf[i] = pn[i];\n    }\n";
+    }
+    if (NC > NU * K) {
+      const std::string b0 = i2s(NU * K);
+      s += "    int64_t p1 = jl_prefetch(p, s, kJC[" + b0 + "], r, in);\n";
+      s += "#pragma unroll 1\n    for (int k = " + b0 + "; k < " + i2s(NC) + "; ++k) {\n";
+      s += "      const int64_t pn = k + 1 < " + i2s(NC) + " ? jl_prefetch(p, s, kJC[k + 1], r, in) : 0;\n";
+      s += "      int64_t mdum = 0;\n      int32_t ldum = 0;\n";
+      s += "      jl_canon<kSmall>(p, s, kJC[k], kJL0, kJS, r, wi, lane, in, row, B, p1, &mdum, &ldum, ovf);\n";
+      s += "      p1 = pn;\n    }\n";
+    }
+    if (NU > 0) {
+      s += "#pragma unroll 1\n    for (int u = 0; u < " + i2s(NU) + "; ++u)\n"
+           "      if (__any_sync(0xffffffffu, (late >> u) & 1u)) {  // NGram rows off the register path\n"
+           "        int32_t L;\n        long long P0;\n"
+           "        jl_ngram_lp<" + i2s(K) + ", " + i2s(N) + ", kSmall>(s, kJN[u], r, wi, lane, in, &L, &P0);\n"
+           "        if ((late >> u) & 1u) rb_fallback(p, s, x.slot, kJN[u].f, r, row, L, P0);\n      }\n";
+    }
+    s += "    if (ovf) atomicExch(c.err, 1);  // values_capacity understated (sp_nnz): nothing stored past it\n";
+    return s;
+  }
+
   // ---- batched emitter (default when every output qualifies) ----
   // Outputs are emitted in batches of kBatch in processing order, stage by
   // stage across the batch: (1) lengths, positions, length/offset stores and
@@ -726,6 +881,10 @@ struct Gen {
         s += "      if (!fast && L" + Q + " > 0) late |= 1u << " + i2s(late_slot[q]) + ";\n    }\n  }\n";
       }
       s += "  }\n";
+      // (experiment knob RAP_JIT_BATCHSYNC: the CTA's warps meet after every
+      // batch, so they stream the same window of straight-line code)
+      if (env_int("RAP_JIT_BATCHSYNC", 0) && bi + 1 < batches.size())
+        s += std::string("    ") + (pairs() ? "__syncthreads();" : (gen_dense_ok() ? "rb_sync<true>();" : "rb_sync<false>();")) + "\n";
     }
     // late rows: the generic path (warp-uniform test per output)
     for (int k = 0; k < (int)late_q.size(); ++k) {
@@ -1219,6 +1378,13 @@ struct Gen {
       body += e;
     }
     body += "};\n\n}  // namespace rapk\n\n";
+    {
+      const LoopPlan lp = loop_plan();
+      if (lp.ok) {  // the tables reference the sample tables: generate them first
+        const std::string t = loop_tables(lp);
+        body = t + body;
+      }
+    }
     s += globals + sample_globals + "\n" + body;
     // one variant per module: 32-bit scans (every offset < 2^31) or 64-bit
     const char* mb = getenv("RAP_JIT_MINB");  // CTAs per SM the register budget targets (default 2; pairs 4)

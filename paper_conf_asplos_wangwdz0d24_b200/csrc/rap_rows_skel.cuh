@@ -410,6 +410,145 @@ __device__ __forceinline__ void rb_tile_store_warp(const Common& c, const float*
   }
 }
 
+// ---- loop emitter of the generated kernel (rap_jit.cpp emit_loop) ----
+// The plan's outputs become rows of __constant__ tables and the emit phase
+// loops over them (NGram units: k providers + their NGram per iteration; then
+// the single canonical outputs), so the code a warp streams is a few short
+// loop bodies instead of one straight-line block per output.
+struct JLCanon {  // a canonical output holding at most one id per row (FirstX <= 1)
+  long long fill, lo, hi, map_def, map_a, bk_a, M;
+  unsigned long long hs;
+  int slot, col, f, q;           // staged slot, raw column, output index, processing index
+  int cap, ncap, flags, nullm;   // flags: CB_* stages of the chain; nullm: stages that apply to filled nulls
+  int map_m, bk_m, bk_row, memo; // bk_row: row of the level-0 / sample tables; memo: stage bit after which the
+                                 // NGram word is taken (16: before any stage, 0: none)
+  int last, pad;                 // last: f == F - 1 (writes offsets[F * B])
+};
+template <int K>
+struct JLNgram {
+  unsigned long long hsalt;
+  long long M;
+  int f, q, out_cap, last;
+  int slot[K], cap[K], ncap[K];
+};
+
+// One canonical output of the loop emitter: lengths, offsets, the value of
+// element 0 (the chain on the prefetched first id) and its NGram word.
+template <bool kSmall, class P>
+__device__ __forceinline__ void jl_canon(const P& p, const RbSmem& s, const JLCanon& Q, const long long* l0,
+                                         const int64_t* const* smp, int r, int wi, int lane, bool in, int64_t row,
+                                         int64_t B, int64_t pf, int64_t* memo, int32_t* len, bool& ovf) {
+  const Common& c = p.c;
+  const RbRow X = rb_row_p<kRbPitch>(s, Q.slot, r);
+  const int32_t L = in ? (X.valid ? min(max(X.b - X.a, 0), Q.cap) : Q.ncap) : 0;
+  *len = L;
+  const long long P0 = s.wb[Q.q * 8 + wi] + rb_ballot_excl(L != 0, lane);
+  stg_s32_if(in, c.lengths + ((int64_t)Q.f * B + row), L);
+  stg_s64_if(in, c.offsets + ((int64_t)Q.f * B + row), P0);
+  if (Q.last) stg_s64_if(in && row == B - 1, c.offsets + (int64_t)(Q.f + 1) * B, P0 + L);
+  ovf |= P0 + L > c.values_cap;
+  const bool valid = X.valid;
+  int64_t v = valid ? pf : Q.fill;
+  if (Q.memo == 16) *memo = v;
+  if (Q.flags & CB_CLAMP) {
+    const int64_t t = v < Q.lo ? Q.lo : (v > Q.hi ? Q.hi : v);
+    v = (valid || (Q.nullm & CB_CLAMP)) ? t : v;
+    if (Q.memo == CB_CLAMP) *memo = v;
+  }
+  if (Q.flags & CB_MAPID) {
+    const MapProbe2 pk = map_first_probe2(c.itab, Q.map_a, Q.map_m, v);
+    bool mi;
+    int64_t mv = map_sel2(pk, v, Q.map_def, &mi);
+    if (__any_sync(0xffffffffu, mi)) mv = mi ? map_lookup_from2(c.itab, Q.map_a, Q.map_m, Q.map_def, v, pk) : mv;
+    v = (valid || (Q.nullm & CB_MAPID)) ? mv : v;
+    if (Q.memo == CB_MAPID) *memo = v;
+  }
+  if (Q.flags & CB_SIGRID) {
+    const int64_t t = (int64_t)reduce_M(splitmix_H(Q.hs ^ (uint64_t)v), Q.M);
+    v = (valid || (Q.nullm & CB_SIGRID)) ? t : v;
+    if (Q.memo == CB_SIGRID) *memo = v;
+  }
+  if (Q.flags & CB_BUCKET) {
+    int j0 = 0;
+    const long long* m0 = l0 + Q.bk_row * 16;
+    for (int k = 0; k < (Q.bk_m >> 6); ++k) j0 += v >= m0[k];
+    const int64_t t = upper_bound_64(c.itab + Q.bk_a, Q.bk_m, smp[Q.bk_row], j0, v);
+    v = (valid || (Q.nullm & CB_BUCKET)) ? t : v;
+    if (Q.memo == CB_BUCKET) *memo = v;
+  }
+  stg_s64_if(L > 0 && P0 < c.values_cap, c.values + P0, v);
+}
+
+// First id of a canonical output's row (0-id rows read a word of the plan blob).
+template <class P>
+__device__ __forceinline__ int64_t jl_prefetch(const P& p, const RbSmem& s, const JLCanon& Q, int r, bool in) {
+  const RbRow Y = rb_row_p<kRbPitch>(s, Q.slot, r);
+  const bool ok = in && Y.valid && Y.b > Y.a;
+  return rap_ldin(ok ? p.val[Q.col] + Y.a : p.c.itab);
+}
+
+// An NGram output (R7) over K memoised provider words, n-windows: returns
+// true when the row needs the generic path (late).
+template <int K, int N, bool kSmall, class P>
+__device__ __forceinline__ bool jl_ngram(const P& p, const RbSmem& s, const JLNgram<K>& G, const int64_t* mm,
+                                         const int32_t* ml, int r, int wi, int lane, bool in, int64_t row, int64_t B,
+                                         bool& ovf) {
+  const Common& c = p.c;
+  int32_t l[K];
+  long long tot = 0;
+#pragma unroll
+  for (int i = 0; i < K; ++i) {
+    const RbRow X = rb_row_p<kRbPitch>(s, G.slot[i], r);
+    l[i] = X.valid ? max(X.b - X.a, 0) : G.ncap[i];
+    l[i] = min(l[i], G.cap[i]);
+    tot += l[i];
+  }
+  const int32_t L = in ? (int32_t)min(max(tot - (long long)N + 1, 0ll), (long long)G.out_cap) : 0;
+  const long long P0 = s.wb[G.q * 8 + wi] + rb_warp_excl<kSmall>(L, lane);
+  stg_s32_if(in, c.lengths + ((int64_t)G.f * B + row), L);
+  stg_s64_if(in, c.offsets + ((int64_t)G.f * B + row), P0);
+  if (G.last) stg_s64_if(in && row == B - 1, c.offsets + (int64_t)(G.f + 1) * B, P0 + L);
+  ovf |= P0 + L > c.values_cap;
+  bool fast = true;
+#pragma unroll
+  for (int i = 0; i < K; ++i) fast = fast && l[i] <= 1 && (l[i] == 0 || ml[i] >= 1);
+  uint64_t w[N];
+#pragma unroll
+  for (int j = 0; j < N; ++j) w[j] = 0;
+  int32_t cnt = 0;
+#pragma unroll
+  for (int i = 0; i < K; ++i) {
+    const bool pr = l[i] != 0;
+#pragma unroll
+    for (int j = 0; j + 1 < N; ++j) w[j] = pr ? w[j + 1] : w[j];
+    w[N - 1] = pr ? (uint64_t)mm[i] : w[N - 1];
+    cnt += pr;
+    if (i + 1 >= N) {
+      uint64_t h = G.hsalt;
+#pragma unroll
+      for (int j = 0; j < N; ++j) h = splitmix_H(h ^ w[j]);
+      const int64_t v = (int64_t)reduce_M(h, G.M);
+      const long long at = P0 + (cnt - N);
+      stg_s64_if(fast && pr && cnt >= N && cnt - N < L && at < c.values_cap, c.values + at, v);
+    }
+  }
+  return !fast && L > 0;
+}
+
+// Length and first position of an NGram row (the late path's recomputation).
+template <int K, int N, bool kSmall>
+__device__ __forceinline__ void jl_ngram_lp(const RbSmem& s, const JLNgram<K>& G, int r, int wi, int lane, bool in,
+                                            int32_t* L, long long* P0) {
+  long long tot = 0;
+#pragma unroll
+  for (int i = 0; i < K; ++i) {
+    const RbRow X = rb_row_p<kRbPitch>(s, G.slot[i], r);
+    tot += min(X.valid ? max(X.b - X.a, 0) : G.ncap[i], G.cap[i]);
+  }
+  *L = in ? (int32_t)min(max(tot - (long long)N + 1, 0ll), (long long)G.out_cap) : 0;
+  *P0 = s.wb[G.q * 8 + wi] + rb_warp_excl<kSmall>(*L, lane);
+}
+
 // Context of one CTA: its feature group (processing indices [pb, pe)) and
 // row block [R0, R1).
 struct RbCtx {
