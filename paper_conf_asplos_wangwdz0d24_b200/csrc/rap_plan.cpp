@@ -69,9 +69,9 @@ int64_t sat_mul(int64_t a, int64_t b) {
 }  // namespace
 
 // Latency-model constants (rap_predict_latency_us): t0/c per kernel family
-// and the HBM bandwidth, fitted on B200 (profiles/r02_cost_model_fit.txt).
+// and the HBM bandwidth, fitted on B200 (profiles/r02b_cost_model_fit.txt).
 #ifndef RAP_MODEL_FIT
-#define RAP_MODEL_FIT 39.9236, 2.08214e-05, 0, 11.94, 0, 0.0102245, 4.9372, 0, 0.00371049, 6446.6
+#define RAP_MODEL_FIT 37.3043, 2.08101e-05, 0, 0, 12.0245, 0, 0.0101371, 0, 10.8344, 0, 0.000840856, 0.000521921, 6446.6
 #endif
 
 struct rap_plan {
@@ -2013,7 +2013,15 @@ static PredTerms predict_terms(const rap_plan* P, int64_t B, const int64_t* nnz,
     t.grid = (int64_t)g.n_rb * g.n_fg + g.n_dcta;
     t.work = gmax * (double)(chunks * chunk);
     if (jit) {
-      t.dwork = dense * (double)std::min<int64_t>(g.rows_rb, B);  // the dense warp's rows
+      int r0 = 0;
+      const int dm = jit_dense_mode((int)P->souts.size(), P->d_out, (int)P->dprogs.size(), P->rb_dense_bytes,
+                                    jit_pairs(P), &r0);
+      const int64_t rows = std::min<int64_t>(g.rows_rb, B);
+      // mode 2: every warp one 32-row tile at a time (the busiest warp's rows,
+      // before the grid wait); mode 1: the dense warp takes the block's rows
+      t.dwork = dm == 2 ? dense * 32.0 * (double)((rows + 32 * jit_dense_tiles(jit_pairs(P)) - 1) /
+                                                  (32 * jit_dense_tiles(jit_pairs(P))))
+                        : dense * (double)rows;
     } else if (g.n_dcta > 0) {
       t.dwork = dense * (double)kDenseBlockRows;  // one dense block per dedicated CTA
     } else if (n_dense > 0) {
@@ -2030,16 +2038,18 @@ static PredTerms predict_terms(const rap_plan* P, int64_t B, const int64_t* nnz,
   return t;
 }
 
-static void model_constants(double k[10]) {
+constexpr int kModelK = 13;
+static void model_constants(double k[kModelK]) {
   // per kernel (tiled, rows, generated): t0 (us), c_work (us per cost unit),
-  // c_pair (us per (output, row) pair); then the HBM bandwidth (GB/s)
-  static const double fit[10] = {RAP_MODEL_FIT};
-  for (int i = 0; i < 10; ++i) k[i] = fit[i];
+  // c_pair (us per (output, row) pair), c_dense (us per dense cost unit of
+  // the busiest CTA's serial dense work); then the HBM bandwidth (GB/s)
+  static const double fit[kModelK] = {RAP_MODEL_FIT};
+  for (int i = 0; i < kModelK; ++i) k[i] = fit[i];
   if (const char* env = getenv("RAP_MODEL")) {
-    double v[10];
-    if (sscanf(env, "%lf,%lf,%lf,%lf,%lf,%lf,%lf,%lf,%lf,%lf", &v[0], &v[1], &v[2], &v[3], &v[4], &v[5], &v[6],
-               &v[7], &v[8], &v[9]) == 10)
-      for (int i = 0; i < 10; ++i) k[i] = v[i];
+    double v[kModelK];
+    if (sscanf(env, "%lf,%lf,%lf,%lf,%lf,%lf,%lf,%lf,%lf,%lf,%lf,%lf,%lf", &v[0], &v[1], &v[2], &v[3], &v[4], &v[5],
+               &v[6], &v[7], &v[8], &v[9], &v[10], &v[11], &v[12]) == kModelK)
+      for (int i = 0; i < kModelK; ++i) k[i] = v[i];
   }
 }
 
@@ -2068,12 +2078,11 @@ rap_status rap_predict_latency_us(const rap_plan* P, int64_t n_rows, const int64
     *latency_us = 0.0;
     return RAP_OK;
   }
-  double k[10];
+  double k[kModelK];
   model_constants(k);
   const int fam = (int)terms[0];
-  const int i = fam == RAP_KERNEL_JIT ? 6 : fam == RAP_KERNEL_ROWS ? 3 : 0;
-  // (the dense work, terms[4], took zero weight in every fit: not modelled)
-  *latency_us = k[i] + k[i + 1] * terms[2] + k[i + 2] * terms[5] + terms[3] / (k[9] * 1e3);
+  const int i = fam == RAP_KERNEL_JIT ? 8 : fam == RAP_KERNEL_ROWS ? 4 : 0;
+  *latency_us = k[i] + k[i + 1] * terms[2] + k[i + 2] * terms[5] + k[i + 3] * terms[4] + terms[3] / (k[12] * 1e3);
   return RAP_OK;
 }
 

@@ -268,11 +268,27 @@ __device__ __forceinline__ void rb_stage(const P& p, const RbSmem& s, const int1
     if (ob) bulk_g2s(s.off + k * s.pitch, src, ob, bar);
     if (wb) bulk_g2s(s.bm + k * 8, bs, wb, bar);
     if (k < n_ids) rb_stage_ids(p.val[col], a0, a1, s.ids + k * kRbIdCap, s.ide0 + k, ibar);
-    for (int i = (int)(ob / 4); i < no; ++i) s.off[k * s.pitch + i] = __ldg(src + i);
-    if (bs == nullptr) {
-      for (int i = 0; i < nw; ++i) s.bm[k * 8 + i] = 0xffffffffu;
-    } else {
-      for (int i = (int)(wb / 4); i < nw; ++i) s.bm[k * 8 + i] = __ldg(bs + i);
+  }
+  // the words outside the bulk copies (an unaligned offsets tail, validity
+  // words of an unaligned bitmap: 3 of 4 row blocks of 224 rows), 8 threads
+  // per column so their loads are in flight together
+  {
+    const int nthr = kDW ? 224 : (int)blockDim.x;
+    for (int t = tid; t < n_cols * 8; t += nthr) {
+      const int k = t >> 3, j = t & 7, col = cols[k];
+      const int32_t* src = p.off[col] + c0;
+      const uint32_t ob = (reinterpret_cast<uintptr_t>(src) & 15) == 0 ? ((uint32_t)(no * 4) & ~15u) : 0u;
+      for (int i = (int)(ob / 4) + j; i < no; i += 8) s.off[k * s.pitch + i] = __ldg(src + i);
+      if (j < nw) {
+        const uint32_t* bm = p.svalid[col];
+        if (bm == nullptr) {
+          s.bm[k * 8 + j] = 0xffffffffu;
+        } else {
+          const uint32_t* bs = bm + (c0 >> 5);
+          const uint32_t wb = (reinterpret_cast<uintptr_t>(bs) & 15) == 0 ? ((uint32_t)(nw * 4) & ~15u) : 0u;
+          if (j >= (int)(wb / 4)) s.bm[k * 8 + j] = __ldg(bs + j);
+        }
+      }
     }
   }
   mbar_wait(bar, (uint32_t)*phase);
