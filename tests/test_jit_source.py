@@ -23,7 +23,13 @@ def test_c2_source_compiles_with_immediates(rap):
     w = synth.c2_terabyte(0)
     st, src, ok, log = rap.jit_source(w.spec, compile=True)
     assert st == "OK" and ok, log
-    assert src.count("// output ") == 34
+    # the batched emitter (rap_jit.cpp emit_batched): every output of the
+    # plan in exactly one batch, in batches of at most 8
+    import re
+
+    listed = [int(f) for b in re.findall(r"// batch of outputs([ 0-9]+)", src) for f in b.split()]
+    assert sorted(listed) == list(range(34))
+    assert all(len(b.split()) <= 8 for b in re.findall(r"// batch of outputs([ 0-9]+)", src))
     # the trigram outputs read their memoised sources from registers
     assert src.count("(uint64_t)m") == 24
     # every SigridHash salt is an immediate H(salt) (R3)
@@ -38,7 +44,10 @@ def test_c1_source_compiles(rap):
     w = synth.c1_kaggle(0)
     st, src, ok, log = rap.jit_source(w.spec, compile=True)
     assert st == "OK" and ok, log
-    assert src.count("// output ") == 26
+    import re
+
+    listed = [int(f) for b in re.findall(r"// batch of outputs([ 0-9]+)", src) for f in b.split()]
+    assert sorted(listed) == list(range(26))
 
 
 @pytest.mark.parametrize("seed", range(3))
