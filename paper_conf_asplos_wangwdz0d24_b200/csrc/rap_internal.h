@@ -29,6 +29,7 @@ typedef unsigned long long uintptr_t;
 #define INT64_MIN (-INT64_MAX - 1LL)
 #else
 #include <stdint.h>
+#include <stdlib.h>
 #endif
 
 #ifdef __CUDACC__
@@ -344,7 +345,12 @@ struct JitModule;  // compiled kernels (opaque)
 //      eight per CTA);
 //   0: no generated dense code (the interpreted dense blocks).
 // *region0 = the shared-memory bytes of region 0 the mode needs.
+//   3: three dense warps (warps 7-9 of a 320-thread CTA) beside the sparse
+//      phases, each with its own tile: the dense work overlaps the emit
+//      phase, whose warps leave most issue slots idle (the default).
 inline int jit_dense_tiles(int) { return 8; }  // mode 2: warps with a tile
+constexpr int kJitDenseWarps = 3;              // mode 3
+inline int jit_dense_warps(int mode) { return mode == 3 ? kJitDenseWarps : mode == 1 ? 1 : 0; }
 inline int jit_dense_mode(int n_sparse_out, int d_out, int n_dprogs, int rb_dense_bytes, int pairs, int* region0) {
   const int off = ((2 * (n_sparse_out + 1) * 8) + 15) & ~15;  // after the base phase's T[f], L[f]
   const int one = 32 * (d_out | 1) * 4;
@@ -353,7 +359,17 @@ inline int jit_dense_mode(int n_sparse_out, int d_out, int n_dprogs, int rb_dens
     *region0 = rb_dense_bytes;
     return 0;
   }
-  if (off + nt * one <= 48 * 1024) {
+#ifndef __CUDACC_RTC__
+  const char* want = getenv("RAP_JIT_DENSE");  // "1" / "2": force that mode (experiment knob)
+  const int wm = want ? atoi(want) : 3;
+#else
+  const int wm = 3;
+#endif
+  if (wm == 3 && !pairs && off + kJitDenseWarps * one <= 48 * 1024) {
+    *region0 = off + kJitDenseWarps * one;
+    return 3;
+  }
+  if (wm != 1 && off + nt * one <= 48 * 1024) {
     *region0 = off + nt * one;
     return 2;
   }
@@ -361,6 +377,7 @@ inline int jit_dense_mode(int n_sparse_out, int d_out, int n_dprogs, int rb_dens
     *region0 = rb_dense_bytes;
     return 0;
   }
+  (void)wm;
   if (off + one <= rb_dense_bytes) {
     *region0 = off + one;
     return 1;

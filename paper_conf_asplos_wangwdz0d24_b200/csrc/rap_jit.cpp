@@ -287,7 +287,12 @@ struct Gen {
     int r0 = 0;
     return jit_dense_mode(F, v.d_out, v.n_dprogs, v.dense_bytes, v.pairs, &r0);
   }
-  bool gen_dense_ok() const { return dense_mode() == 1; }  // the dense-warp form (kDenseWarp)
+  bool gen_dense_ok() const { return dense_mode() == 1 || dense_mode() == 3; }  // the dense-warp forms (kDenseWarp)
+  int threads() const {
+    if (pairs()) return 2 * kRbChunk;
+    const int nd = jit_dense_warps(dense_mode());
+    return nd ? 224 + 32 * nd : kRbChunk;
+  }
   double unit_cost(const DProg& dp, const DUnit& un) const {
     const DevOp* ops = un.gops ? v.ops : dp.ops;
     double c = 8;
@@ -381,7 +386,7 @@ struct Gen {
     // the base-phase totals, then stored by the warp
     std::string s;
     const int mode = dense_mode();
-    const bool ok = mode == 1;
+    const bool ok = mode == 1 || mode == 3;
     s += "  static constexpr bool kGenDense = " + std::string(mode == 2 ? "true" : "false") + ";\n";
     s += "  static constexpr bool kDenseWarp = " + std::string(ok ? "true" : "false") + ";\n";
     if (mode == 2) {
@@ -409,9 +414,12 @@ struct Gen {
            i2s(32 * pitch()) + ";  // [" + i2s(nt) + "][32][" + i2s(pitch()) + "]\n";
       s += "    if (warp < " + i2s(nt) + ")\n";
       s += "    for (int64_t d0 = x.R0 + 32 * warp; d0 < x.R1; d0 += " + i2s(32 * nt) + ") {\n";
-    } else {
-      s += "    float* tile = reinterpret_cast<float*>(s.dense + " + i2s(tile_offset()) + ");  // [32][" + i2s(pitch()) + "]\n";
-      s += "    for (int64_t d0 = x.R0; d0 < x.R1; d0 += 32) {\n";
+    } else {  // dense warps 7 .. 7 + nd - 1: their own tile, the block's 32-row tiles round robin over them
+      const int nd = jit_dense_warps(mode);
+      s += "    const int dw = (threadIdx.x >> 5) - 7;\n";
+      s += "    float* tile = reinterpret_cast<float*>(s.dense + " + i2s(tile_offset()) + ") + dw * " + i2s(32 * pitch()) +
+           ";  // [" + i2s(nd) + "][32][" + i2s(pitch()) + "]\n";
+      s += "    for (int64_t d0 = x.R0 + 32 * dw; d0 < x.R1; d0 += " + i2s(32 * nd) + ") {\n";
     }
     s += "      const int nr = (int)min((int64_t)32, x.R1 - d0);\n";
     s += "      if (lane < nr) {\n        const int64_t row = d0 + lane;\n";
@@ -1344,7 +1352,7 @@ struct Gen {
     // Bucketize tables, awaited at the start of the emit phase
     body += std::string("  static constexpr bool kSetupEarly = ") + (tab_total ? "true" : "false") + ";\n";
     body += "  static constexpr bool kPairs = " + std::string(pairs() ? "true" : "false") + ";\n";
-    body += "  static constexpr int kThreads = " + i2s(pairs() ? 2 * kRbChunk : kRbChunk) + ";\n";
+    body += "  static constexpr int kThreads = " + i2s(threads()) + ";\n";
     body += "  template <class P>\n"
             "  static __device__ __forceinline__ void setup(const P& p, const RbSmem& s, const RbCtx& x) {\n";
     (void)records;  // the fallbacks rebuild their record from the plan blob (rb_fallback)
@@ -1388,7 +1396,7 @@ struct Gen {
     s += globals + sample_globals + "\n" + body;
     // one variant per module: 32-bit scans (every offset < 2^31) or 64-bit
     const char* mb = getenv("RAP_JIT_MINB");  // CTAs per SM the register budget targets (default 2; pairs 4)
-    s += "extern \"C\" __global__ void __launch_bounds__(" + i2s(pairs() ? 2 * kRbChunk : kRbChunk) + ", " + std::string(mb ? mb : "2") +
+    s += "extern \"C\" __global__ void __launch_bounds__(" + i2s(threads()) + ", " + std::string(mb ? mb : "2") +
          ") rap_jit_kernel(const __grid_constant__ "
          "rapk::RbParams<rapk::kRbMaxDense, rapk::kRbMaxCols> p) {\n"
          "  rapk::rows_body<rapk::JitPolicy, rapk::kRbMaxDense, rapk::kRbMaxCols, " +

@@ -71,7 +71,7 @@ int64_t sat_mul(int64_t a, int64_t b) {
 // Latency-model constants (rap_predict_latency_us): t0/c per kernel family
 // and the HBM bandwidth, fitted on B200 (profiles/r02b_cost_model_fit.txt).
 #ifndef RAP_MODEL_FIT
-#define RAP_MODEL_FIT 37.3043, 2.08101e-05, 0, 0, 12.0245, 0, 0.0101371, 0, 10.8344, 0, 0.000840856, 0.000521921, 6446.6
+#define RAP_MODEL_FIT 37.1015, 2.07606e-05, 0, 0, 12.0978, 0, 0.0102007, 0, 10.7953, 0, 0.0030039, 0, 6446.6
 #endif
 
 struct rap_plan {
@@ -835,7 +835,13 @@ static int64_t jit_min_rows() {
   return env ? atoll(env) : (int64_t)1 << 62;
 }
 static int jit_pitch(const rap_plan*) { return 0; }
-static int jit_threads(const rap_plan* P) { return jit_pairs(P) ? 2 * kRbChunk : kRbChunk; }
+static int jit_threads(const rap_plan* P) {
+  if (jit_pairs(P)) return 2 * kRbChunk;
+  int r0 = 0;
+  const int nd = jit_dense_warps(
+      jit_dense_mode((int)P->souts.size(), P->d_out, (int)P->dprogs.size(), P->rb_dense_bytes, 0, &r0));
+  return nd ? 224 + 32 * nd : kRbChunk;  // the generated kernel's CTA (rap_jit.cpp Gen::threads)
+}
 static int jit_base_smem(const rap_plan* P, int dense_bytes) {
   return rows_smem_bytes(dense_bytes, P->rb_max_fl, P->rb_max_cols, 0, (int)P->souts.size(), 0, 0, jit_pitch(P), 0,
                          P->jit_tab_bytes);
@@ -2019,9 +2025,11 @@ static PredTerms predict_terms(const rap_plan* P, int64_t B, const int64_t* nnz,
       const int64_t rows = std::min<int64_t>(g.rows_rb, B);
       // mode 2: every warp one 32-row tile at a time (the busiest warp's rows,
       // before the grid wait); mode 1: the dense warp takes the block's rows
-      t.dwork = dm == 2 ? dense * 32.0 * (double)((rows + 32 * jit_dense_tiles(jit_pairs(P)) - 1) /
-                                                  (32 * jit_dense_tiles(jit_pairs(P))))
-                        : dense * (double)rows;
+      // mode 3: the dense warps run beside the sparse phases (hidden: their
+      // rows per warp stay well below the sparse warps' chain); mode 2 / 1:
+      // the busiest warp's dense rows add to the launch
+      const int nd = dm == 2 ? jit_dense_tiles(jit_pairs(P)) : std::max(1, jit_dense_warps(dm));
+      t.dwork = dm == 3 ? 0.0 : dense * 32.0 * (double)((rows + 32 * nd - 1) / (32 * nd));
     } else if (g.n_dcta > 0) {
       t.dwork = dense * (double)kDenseBlockRows;  // one dense block per dedicated CTA
     } else if (n_dense > 0) {

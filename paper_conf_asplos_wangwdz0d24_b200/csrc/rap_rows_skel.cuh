@@ -688,7 +688,7 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
     __syncthreads();
   }
   trace_stamp(c, 7);
-  if (kDW && warp == kWS) {
+  if (kDW && warp >= kWS) {
     Pol::dense_warp(p, s, x);  // the dense outputs of rows [R0, R1), concurrent with the sparse phases
     trace_stamp_warp(c, 15);
   } else {
