@@ -443,7 +443,8 @@ struct Gen {
     if (pairs())
       return "    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, wi = warp >> 1, r = (wi << 5) | lane;\n"
              "    (void)tid;\n";
-    return "    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, wi = warp, r = tid;\n";
+    return "    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, wi = warp, r = tid;\n"
+           "    (void)lane;\n    (void)wi;\n";
   }
   int split_point() const {
     if (!pairs()) return F;
@@ -505,11 +506,11 @@ struct Gen {
     std::string s;
     s += "  template <bool kSmall, class P>\n"
          "  static __device__ __forceinline__ void emit(const P& p, const RbSmem& s, const RbCtx& x, int64_t c0, "
-         "int nr) {\n" + thread_vars() +
+         "int nr, const PreState& ps, bool use_pre) {\n" + thread_vars() +
          "    const Common& c = p.c;\n"
          "    const int64_t B = x.B;\n"
          "    const bool in = r < nr;\n"
-         "    const int64_t row = c0 + r;\n";
+         "    const int64_t row = c0 + r;\n    (void)ps;\n    (void)use_pre;\n";
     const int sp = split_point();
     if (tab_total) s += "    mbar_wait(reinterpret_cast<uint64_t*>(s.tabs), 0u);  // staged tables landed\n";
     const LoopPlan lp = loop_plan();
@@ -731,6 +732,122 @@ struct Gen {
     }
     return "upper_bound(c.itab + " + lit64(q.bk_a) + ", " + i2s(q.bk_m) + ", " + x + ")";
   }
+  // The value chain of a batch's canonical outputs: v<q> from the prefetched
+  // first id pf<q> and the staged row X<q>_0 (declared by the caller), fill,
+  // Clamp, MapId (two probe slots, warp-uniform continuation), SigridHash,
+  // Bucketize; the NGram word m<f> after the memo stage.
+  std::string value_code(const std::vector<int>& canon, const std::vector<char>& is_prov) {
+    std::string s;
+    for (int q : canon) {
+      const int f = v.perm[q];
+      const SProg& pg = v.sprogs[f];
+      const Canon& cn = pg.cn;
+      const std::string Q = i2s(q), Fs = i2s(f), X = "X" + Q + "_0";
+      const int ma = is_prov[f] ? memo_point(v.feat[f], cn) : -1;
+      s += "    v" + Q + " = " + X + ".valid ? pf" + Q + " : " + lit64(pg.ch.fill) + ";\n";
+      if (ma == 16) s += "    m" + Fs + " = v" + Q + ";\n";
+      if (cn.mask & CB_CLAMP) {
+        s += sel_stage(cn, CB_CLAMP, "v" + Q, X + ".valid",
+                       "v" + Q + " < " + lit64(cn.lo) + " ? " + lit64(cn.lo) + " : (v" + Q + " > " + lit64(cn.hi) + " ? " +
+                           lit64(cn.hi) + " : v" + Q + ")");
+        if (ma == CB_CLAMP) s += "    m" + Fs + " = v" + Q + ";\n";
+      }
+    }
+    for (int q : canon) {
+      const Canon& cn = v.sprogs[v.perm[q]].cn;
+      if (!(cn.mask & CB_MAPID)) continue;
+      s += "    const MapProbe2 pk" + i2s(q) + " = map_first_probe2(c.itab, " + lit64(cn.map_a) + ", " + i2s(cn.map_m) +
+           ", v" + i2s(q) + ");\n";
+    }
+    for (int q : canon) {
+      const int f = v.perm[q];
+      const Canon& cn = v.sprogs[f].cn;
+      const std::string Q = i2s(q), Fs = i2s(f), X = "X" + Q + "_0";
+      const int ma = is_prov[f] ? memo_point(v.feat[f], cn) : -1;
+      if (cn.mask & CB_MAPID) {
+        s += "    { bool mi;\n      int64_t mv = map_sel2(pk" + Q + ", v" + Q + ", " + lit64(cn.map_def) + ", &mi);\n";
+        const bool all = (cn.null_mask & CB_MAPID) != 0;
+        // rows whose key is past the first two slots probe on (warp-uniform test)
+        s += "      if (__any_sync(0xffffffffu, mi)) mv = mi ? map_lookup_from2(c.itab, " + lit64(cn.map_a) + ", " +
+             i2s(cn.map_m) + ", " + lit64(cn.map_def) + ", v" + Q + ", pk" + Q + ") : mv;\n";
+        s += "      v" + Q + " = " + (all ? "mv" : X + ".valid ? mv : v" + Q) + "; }\n";
+        if (ma == CB_MAPID) s += "    m" + Fs + " = v" + Q + ";\n";
+      }
+      if (cn.mask & CB_SIGRID) {
+        s += sel_stage(cn, CB_SIGRID, "v" + Q, X + ".valid",
+                       "(int64_t)reduce_M(splitmix_H(" + litu64(cn.hs) + " ^ (uint64_t)v" + Q + "), " + lit64(cn.M) + ")");
+        if (ma == CB_SIGRID) s += "    m" + Fs + " = v" + Q + ";\n";
+      }
+    }
+    for (int q : canon) {
+      const int f = v.perm[q];
+      const Canon& cn = v.sprogs[f].cn;
+      const std::string Q = i2s(q), Fs = i2s(f), X = "X" + Q + "_0";
+      const int ma = is_prov[f] ? memo_point(v.feat[f], cn) : -1;
+      if (cn.mask & CB_BUCKET) {
+        s += sel_stage(cn, CB_BUCKET, "v" + Q, X + ".valid", bucket_expr(cn, "v" + Q));
+        if (ma == CB_BUCKET) s += "    m" + Fs + " = v" + Q + ";\n";
+      }
+    }
+    return s;
+  }
+  // Batch 0's canonical outputs of the batched emitter (processing indices).
+  std::vector<int> pre_canon() const {
+    std::vector<int> c;
+    for (int q = 0; q < std::min(F, batch_k()); ++q)
+      if (v.feat[v.perm[q]].emit == 0) c.push_back(q);
+    return c;
+  }
+  // pre_emit: batch 0's values before the grid wait (one-chunk blocks), so
+  // the wait for the other CTAs' totals and the base loads overlap them.
+  bool pre_ok() const {
+    return env_int("RAP_JIT_PRE", 1) != 0 && batch_ok() && !pairs() && !pre_canon().empty();
+  }
+  std::vector<char> prov_flags() const {
+    std::vector<char> is_prov(F, 0);
+    for (int f = 0; f < F; ++f)
+      if (v.feat[f].emit == 0 && v.feat[f].memo_slot >= 0) is_prov[f] = 1;
+    return is_prov;
+  }
+  std::string pre_fn() {
+    std::string s;
+    if (!pre_ok()) {
+      s += "  static constexpr bool kPre = false;\n  struct PreState {};\n";
+      s += "  template <class P>\n  static __device__ __forceinline__ PreState pre_emit(const P&, const RbSmem&, const RbCtx&, "
+           "int64_t, int) { return PreState{}; }\n";
+      return s;
+    }
+    const std::vector<int> canon = pre_canon();
+    const std::vector<char> is_prov = prov_flags();
+    s += "  static constexpr bool kPre = true;\n  struct PreState {\n";
+    for (int q : canon) {
+      s += "    int64_t v" + i2s(q) + ";\n";
+      if (is_prov[v.perm[q]]) s += "    int64_t m" + i2s(v.perm[q]) + ";\n";
+    }
+    s += "  };\n";
+    s += "  template <class P>\n  static __device__ __forceinline__ PreState pre_emit(const P& p, const RbSmem& s, "
+         "const RbCtx& x, int64_t c0, int nr) {\n" + thread_vars() +
+         "    const Common& c = p.c;\n    const bool in = r < nr;\n    (void)c0;\n";
+    if (tab_total) s += "    mbar_wait(reinterpret_cast<uint64_t*>(s.tabs), 0u);  // staged tables landed\n";
+    for (int q : canon) {
+      const RbFeat& R = v.feat[v.perm[q]];
+      const std::string Q = i2s(q);
+      s += "    int64_t pf" + Q + ";\n    { const RbRow Y" + Q + " = " + rbrow() + "(s, " + i2s(slot[R.src[0]]) +
+           ", r);\n      const bool ok = in && Y" + Q + ".valid && Y" + Q + ".b > Y" + Q + ".a;\n      pf" + Q +
+           " = rap_ldin(ok ? p.val[" + i2s(R.src[0]) + "] + Y" + Q + ".a : c.itab); }\n";
+      s += "    const RbRow X" + Q + "_0 = " + rbrow() + "(s, " + i2s(slot[R.src[0]]) + ", r);\n";
+      s += "    int64_t v" + Q + ";\n";
+      if (is_prov[v.perm[q]]) s += "    int64_t m" + i2s(v.perm[q]) + " = 0;\n";
+    }
+    s += value_code(canon, is_prov);
+    s += "    PreState ps;\n";
+    for (int q : canon) {
+      s += "    ps.v" + i2s(q) + " = v" + i2s(q) + ";\n";
+      if (is_prov[v.perm[q]]) s += "    ps.m" + i2s(v.perm[q]) + " = m" + i2s(v.perm[q]) + ";\n";
+    }
+    s += "    return ps;\n  }\n";
+    return s;
+  }
   std::string emit_batched(int qb, int qe) {
     std::string s;
     s += "    bool ovf = false;\n    unsigned late = 0;\n    (void)late;\n";
@@ -771,7 +888,24 @@ struct Gen {
         if (v.feat[v.perm[q]].emit == 0) t += prefetch(q);
       return t;
     };
-    if (!batches.empty()) s += pf_batch(batches[0]);
+    if (!batches.empty()) {
+      if (pre_ok() && qb == 0) {  // batch 0's ids only when its values were not carried over
+        for (int q : batches[0])
+          if (v.feat[v.perm[q]].emit == 0) s += "    int64_t pf" + i2s(q) + " = 0;\n";
+        s += "    if (!use_pre) {\n";
+        for (int q : batches[0])
+          if (v.feat[v.perm[q]].emit == 0) {
+            const RbFeat& R = v.feat[v.perm[q]];
+            const std::string Q = i2s(q);
+            s += "    { const RbRow Y" + Q + " = " + rbrow() + "(s, " + i2s(slot[R.src[0]]) + ", r);\n      const bool ok = in && Y" + Q +
+                 ".valid && Y" + Q + ".b > Y" + Q + ".a;\n      pf" + Q + " = rap_ldin(ok ? p.val[" + i2s(R.src[0]) + "] + Y" + Q +
+                 ".a : c.itab); }\n";
+          }
+        s += "    }\n";
+      } else {
+        s += pf_batch(batches[0]);
+      }
+    }
     for (size_t bi = 0; bi < batches.size(); ++bi) {
       const std::vector<int>& b = batches[bi];
       if (bi + 1 < batches.size()) s += pf_batch(batches[bi + 1]);  // the next batch's ids in flight
@@ -780,13 +914,10 @@ struct Gen {
       s += "\n";
       std::vector<int> canon, ngram;
       for (int q : b) (v.feat[v.perm[q]].emit == 0 ? canon : ngram).push_back(q);
-      // (1) lengths, positions, length/offset stores, fill, Clamp
+      // (1) lengths, positions, length/offset stores
       for (int q : canon) {
         const int f = v.perm[q];
-        const SProg& pg = v.sprogs[f];
-        const Canon& cn = pg.cn;
-        const std::string Q = i2s(q), Fs = i2s(f), X = "X" + Q + "_0";
-        const int ma = is_prov[f] ? memo_point(v.feat[f], cn) : -1;
+        const std::string Q = i2s(q), Fs = i2s(f);
         s += len_code(q);
         s += "    const long long P" + Q + " = s.wb[" + i2s(q * 8) + " + wi] + rb_ballot_excl(L" + Q + " != 0, lane);\n";
         if (is_prov[f]) s += "    ml" + Fs + " = L" + Q + ";\n";
@@ -794,54 +925,21 @@ struct Gen {
         s += "    stg_s64_if(in, c.offsets + ((int64_t)" + Fs + " * B + row), P" + Q + ");\n";
         if (f == F - 1) s += "    stg_s64_if(in && row == B - 1, c.offsets + (int64_t)" + i2s(F) + " * B, P" + Q + " + L" + Q + ");\n";
         s += "    ovf |= P" + Q + " + L" + Q + " > c.values_cap;\n";
-        s += "    int64_t v" + Q + " = " + X + ".valid ? pf" + Q + " : " + lit64(pg.ch.fill) + ";\n";
-        if (ma == 16) s += "    m" + Fs + " = v" + Q + ";\n";
-        if (cn.mask & CB_CLAMP) {
-          s += sel_stage(cn, CB_CLAMP, "v" + Q, X + ".valid",
-                         "v" + Q + " < " + lit64(cn.lo) + " ? " + lit64(cn.lo) + " : (v" + Q + " > " + lit64(cn.hi) + " ? " +
-                             lit64(cn.hi) + " : v" + Q + ")");
-          if (ma == CB_CLAMP) s += "    m" + Fs + " = v" + Q + ";\n";
-        }
+        s += "    int64_t v" + Q + ";\n";
       }
-      // (2) MapId probes
-      for (int q : canon) {
-        const Canon& cn = v.sprogs[v.perm[q]].cn;
-        if (!(cn.mask & CB_MAPID)) continue;
-        s += "    const MapProbe2 pk" + i2s(q) + " = map_first_probe2(c.itab, " + lit64(cn.map_a) + ", " + i2s(cn.map_m) +
-             ", v" + i2s(q) + ");\n";
-      }
-      // (3) MapId selects, SigridHash
-      for (int q : canon) {
-        const int f = v.perm[q];
-        const Canon& cn = v.sprogs[f].cn;
-        const std::string Q = i2s(q), Fs = i2s(f), X = "X" + Q + "_0";
-        const int ma = is_prov[f] ? memo_point(v.feat[f], cn) : -1;
-        if (cn.mask & CB_MAPID) {
-          s += "    { bool mi;\n      int64_t mv = map_sel2(pk" + Q + ", v" + Q + ", " + lit64(cn.map_def) + ", &mi);\n";
-          const bool all = (cn.null_mask & CB_MAPID) != 0;
-          // rows whose key is past the first two slots probe on (warp-uniform test)
-          s += "      if (__any_sync(0xffffffffu, mi)) mv = mi ? map_lookup_from2(c.itab, " + lit64(cn.map_a) + ", " +
-               i2s(cn.map_m) + ", " + lit64(cn.map_def) + ", v" + Q + ", pk" + Q + ") : mv;\n";
-          s += "      v" + Q + " = " + (all ? "mv" : X + ".valid ? mv : v" + Q) + "; }\n";
-          if (ma == CB_MAPID) s += "    m" + Fs + " = v" + Q + ";\n";
+      // (2)-(4) the values: computed here, or (batch 0 of a one-chunk block)
+      // before the grid wait by pre_emit and carried over in registers
+      if (bi == 0 && pre_ok()) {
+        s += "    if (use_pre) {\n";
+        for (int q : canon) {
+          s += "      v" + i2s(q) + " = ps.v" + i2s(q) + ";\n";
+          if (is_prov[v.perm[q]]) s += "      m" + i2s(v.perm[q]) + " = ps.m" + i2s(v.perm[q]) + ";\n";
         }
-        if (cn.mask & CB_SIGRID) {
-          s += sel_stage(cn, CB_SIGRID, "v" + Q, X + ".valid",
-                         "(int64_t)reduce_M(splitmix_H(" + litu64(cn.hs) + " ^ (uint64_t)v" + Q + "), " + lit64(cn.M) + ")");
-          if (ma == CB_SIGRID) s += "    m" + Fs + " = v" + Q + ";\n";
-        }
+        s += "    } else {\n" + value_code(canon, is_prov) + "    }\n";
+      } else {
+        s += value_code(canon, is_prov);
       }
-      // (4) Bucketize, (5) value stores
-      for (int q : canon) {
-        const int f = v.perm[q];
-        const Canon& cn = v.sprogs[f].cn;
-        const std::string Q = i2s(q), Fs = i2s(f), X = "X" + Q + "_0";
-        const int ma = is_prov[f] ? memo_point(v.feat[f], cn) : -1;
-        if (cn.mask & CB_BUCKET) {
-          s += sel_stage(cn, CB_BUCKET, "v" + Q, X + ".valid", bucket_expr(cn, "v" + Q));
-          if (ma == CB_BUCKET) s += "    m" + Fs + " = v" + Q + ";\n";
-        }
-      }
+      // (5) value stores
       for (int q : canon) {
         const std::string Q = i2s(q);
         s += "    stg_s64_if(L" + Q + " > 0 && P" + Q + " < c.values_cap, c.values + P" + Q + ", v" + Q + ");\n";
@@ -1293,7 +1391,7 @@ struct Gen {
     std::string s;
     s += "  template <bool kSmall, class P>\n"
          "  static __device__ __forceinline__ void emit(const P& p, const RbSmem& s, const RbCtx& x, int64_t c0, "
-         "int nr) {\n"
+         "int nr, const PreState&, bool) {\n"
          "    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;\n"
          "    const Common& c = p.c;\n"
          "    const int64_t B = x.B;\n"
@@ -1358,6 +1456,7 @@ struct Gen {
     (void)records;  // the fallbacks rebuild their record from the plan blob (rb_fallback)
     body += setup_tables();
     body += "  }\n";
+    body += pre_fn();
     body += dense;
     body += lengths_fn();
     {

@@ -305,6 +305,12 @@ __device__ __noinline__ void rb_fallback(const P& p, const RbSmem s, const int16
 struct InterpPolicy {
   static constexpr bool kSetupEarly = true;  // the records drive (1) as well
   static constexpr bool kPairs = false;
+  static constexpr bool kPre = false;  // (the generated policy's pre_emit: rap_jit.cpp)
+  struct PreState {};
+  template <class P>
+  static __device__ __forceinline__ PreState pre_emit(const P&, const RbSmem&, const RbCtx&, int64_t, int) {
+    return PreState{};
+  }
   static constexpr int kThreads = kRbChunk;
   static constexpr bool kGenDense = false;
   static constexpr bool kDenseWarp = false;
@@ -355,7 +361,8 @@ struct InterpPolicy {
   }
 
   template <bool kSmall, class P>
-  static __device__ __forceinline__ void emit(const P& p, const RbSmem& s, const RbCtx& x, int64_t c0, int nr) {
+  static __device__ __forceinline__ void emit(const P& p, const RbSmem& s, const RbCtx& x, int64_t c0, int nr,
+                                              const PreState&, bool) {
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const Common& c = p.c;
     const int FL = x.FL, pb = x.pb, F = x.F;

@@ -722,6 +722,13 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
 
   if (!Pol::kSetupEarly) Pol::setup(p, s, x);  // records used only in (4)
 
+  // a one-chunk block: the policy's first outputs' values (everything but
+  // their positions) computed now, so the wait below and the base loads
+  // overlap them (the generated policy's pre_emit; carried in registers)
+  typename Pol::PreState pre{};
+  const bool use_pre = Pol::kPre && nch == 1 && FL > 0 && nrows > 0;
+  if (use_pre) pre = Pol::pre_emit(p, s, x, x.R0, nrows);
+
   // (2) dense outputs (independent of the scan): the policy's own rows-of-this-
   // block code when it has one and the dense rows are the batch rows, else the
   // launch's dense blocks round robin over the CTAs (the dense warp took them)
@@ -828,7 +835,7 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
       }
       rb_sync<kDW>();
       if (n_ids > 0) mbar_wait(&s_ibar, (uint32_t)s_iphase);  // the chunk's staged ids landed
-      Pol::template emit<kSmall>(p, s, x, c0, nr);
+      Pol::template emit<kSmall>(p, s, x, c0, nr, pre, use_pre && ch == 0);
       rb_sync<kDW>();
       if (n_ids > 0 && tid == 0) s_iphase ^= 1;
     }
