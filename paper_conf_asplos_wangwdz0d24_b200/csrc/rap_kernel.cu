@@ -601,7 +601,7 @@ __device__ __noinline__ long long value_tile_multi(const P& p, const FeatCtx& fc
     if (act == 15u && pos0 + 96 < cap) {
       int64_t* dst = values + pos0;
 #pragma unroll
-      for (int u = 0; u < 4; ++u) dst[32 * u] = x[u];
+      for (int u = 0; u < 4; ++u) st_cs64(dst + 32 * u, x[u]);
     } else {
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
@@ -1011,7 +1011,7 @@ __device__ __noinline__ long long ngram_tile_fast(const P& p, int f, int64_t rt,
   const long long cap = p.c.values_cap;
 #pragma unroll
   for (int kk = 0; kk < 4; ++kk)
-    if (((act >> kk) & 1u) && lb + e[kk] < cap) p.c.values[lb + e[kk]] = o[kk];
+    if (((act >> kk) & 1u) && lb + e[kk] < cap) st_cs64(p.c.values + (lb + e[kk]), o[kk]);
   if (f == p.c.n_sparse_out - 1 && rt == p.c.tiles_per_feature - 1 && lane == 31) {
     p.c.offsets[(int64_t)p.c.n_sparse_out * B] = base + T;  // total, R17
     if (base + T > cap) atomicExch(p.c.err, 1);
