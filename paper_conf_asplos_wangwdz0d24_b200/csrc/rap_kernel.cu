@@ -393,6 +393,7 @@ __device__ __noinline__ long long value_chunk_canon(const P& p, const FeatCtx& f
   int64_t* values = p.c.values;
   const long long cap = p.c.values_cap;
   long long run = base;
+  const int64_t* const itab_h = p.c.itab;  // hoisted (value_tile_multi)
 #pragma unroll 1
   for (int j0 = 0; j0 < nt; j0 += kVGroup) {
     int64_t v[4 * kVGroup];
@@ -403,7 +404,7 @@ __device__ __noinline__ long long value_chunk_canon(const P& p, const FeatCtx& f
       const int lr = (j0 + (u >> 2)) * kTileRows + 4 * lane + (u & 3);
       v[u] = ((ag & fg) >> u) & 1u ? sid[lr] : fc.fill;
     }
-    canon_apply_n<4 * kVGroup>(fc.q, p.c.itab, v, ag, fg);
+    canon_apply_n<4 * kVGroup>(fc.q, itab_h, v, ag, fg);
     trace_clk(p.c, 11, v[0]);
 #pragma unroll
     for (int jj = 0; jj < kVGroup; ++jj) {
@@ -536,6 +537,11 @@ __device__ __noinline__ long long value_tile_multi(const P& p, const FeatCtx& fc
   const int64_t* val = p.val[src];
   int64_t* values = p.c.values;
   const long long cap = p.c.values_cap;
+  // hoisted: the window loop's stores go through a generic pointer that the
+  // compiler cannot prove disjoint from the parameter block, so a p.c field
+  // read inside the loop is reloaded per window (ncu: a generic 8-byte load
+  // of p.c.itab was the top long-scoreboard stall of C4)
+  const int64_t* const itab = p.c.itab;
   int64_t* ring = reinterpret_cast<int64_t*>(wscr + kMultiRing);  // [4][128]
   uint32_t masks = 0;
   const int nwin = (T + 127) >> 7;
@@ -596,7 +602,7 @@ __device__ __noinline__ long long value_tile_multi(const P& p, const FeatCtx& fc
     int64_t x[4];
 #pragma unroll
     for (int u = 0; u < 4; ++u) x[u] = slot[32 * u + lane];  // this lane's own copies
-    canon_apply_n<4>(fc.q, p.c.itab, x, act, full);
+    canon_apply_n<4>(fc.q, itab, x, act, full);
     const long long pos0 = base + w * 128 + lane;
     if (act == 15u && pos0 + 96 < cap) {
       int64_t* dst = values + pos0;
