@@ -702,11 +702,13 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
     Pol::template lengths<kSmall>(p, s, x, nr, ch > 0);
     rb_sync<kDW>();
   }
+  long long blk_tot = 0;  // thread tid < FL: output tid's ids in this block
   if (tid < FL) {
     long long tot = 0;
     if (nch > 0)
 #pragma unroll
       for (int w = 0; w < kWS; ++w) tot += s.ws[tid * 8 + w];
+    blk_tot = tot;
     const int f = s_fidx[tid];
     g.agg[(int64_t)f * n_rb + rb] = (unsigned long long)tot;  // feature-major: row blocks of f contiguous
     atomicAdd(g.tot + f, (unsigned long long)tot);           // red.add: the output's total over all blocks
@@ -811,6 +813,10 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
     if (tid < FL) {
       const int f = s_fidx[tid];
       s.base[tid] = sT[f] + sL[f];
+      // values_capacity (from sp_nnz) understated: an output's ids of this
+      // block end past it (the emitters store nothing past it; one check per
+      // output and block instead of one per row)
+      if (sT[f] + sL[f] + blk_tot > c.values_cap) atomicExch(c.err, 1);
     }
     rb_sync<kDW>();
     trace_stamp(c, 4);
