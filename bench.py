@@ -471,6 +471,9 @@ def run_rap(args):
             del louts
         del train
         torch.cuda.empty_cache()
+    mapping = None
+    if world == 1 and not args.profile and args.workload in ("c1", "c2"):
+        mapping = mapping_point(plan, w.spec, raw0.sp_nnz, B, kern_ms)
     c4 = None
     if world == 1 and not args.profile and not args.no_c4 and args.workload != "c4":
         c4 = c4_point(dev, args.c4_batch, steps=20)
@@ -490,7 +493,7 @@ def run_rap(args):
                            "l2_policy": f"rotate {nsets} distinct input/output sets, {nsets * set_bytes / 2**20:.0f} MB "
                                         f"total vs L2 {l2 / 2**20:.0f} MB"},
                 "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks, "gpu_launches": K,
-                "corun": corun, "fusion": fusion, "graph": graph, "c4": c4, "plans": plans}
+                "corun": corun, "fusion": fusion, "graph": graph, "c4": c4, "plans": plans, "mapping": mapping}
         print(json.dumps(line), flush=True)
     plan.close()
     if world > 1:
@@ -501,6 +504,42 @@ def run_rap(args):
 
 
 KERNEL_NAMES = {1: "tiled", 2: "rows (interpreted)", 3: "rows (generated, NVRTC sm_100a)"}
+
+
+def mapping_point(plan, spec, sp_nnz, B, kern_ms, world=8, B_eval=None):
+    """Fig 12 analog (§7.2), model-based: the
+    C2 graph's outputs on `world` ranks with a skewed consumer placement (rank
+    0 consumes ~2x the mean, rap_place "skewed"), the per-rank preprocessing
+    time of three mappings under the plan's cost model scaled to this GPU's
+    measured C2 kernel time and a 700 GB/s, 20 us link: data locality (every
+    graph on its consumer), data parallel (every rank the whole graph on its
+    batch shard, outputs all-to-all), and the joint mapping loop
+    (rap_place_joint).  One GPU here: no multi-GPU run behind these numbers."""
+    from paper_conf_asplos_wangwdz0d24_b200 import dist
+
+    import numpy as np
+
+    u = kern_ms * 1e3 / max(float(sum(plan.output_costs(B, sp_nnz))), 1e-9)  # this GPU's scale
+    if B_eval and B_eval != B:  # the config's own batch (ids scale with rows)
+        sp_nnz = (np.asarray(sp_nnz, dtype=np.float64) * (B_eval / B)).astype(np.int64)
+        B = B_eval
+    costs = plan.output_costs(B, sp_nnz)
+    cm = dist.CommModel(us_per_unit=u)
+    col = dist.colocation(spec)
+    rb = dist.row_bytes(spec, sp_nnz, B)
+    home = dist.place(costs, col, world, "skewed", B, None).owner
+    joint = dist.place_joint(costs, col, home, world, B, cm, rb, 0.0)
+    dl = dist.place_joint(costs, col, home, world, B, dist.CommModel(u, 1e-9, 1e12), rb, 0.0)  # no move pays
+    comp = float(sum(costs)) * u / world
+    xfer = cm.link_latency_us + sum(rb) * (B / world) * (world - 1) / world / (1e3 * cm.link_gbs)
+    return {"what": f"model-based per-rank preprocessing time (us), {len(costs)} outputs, B = {B}, {world} ranks, "
+                    "skewed consumers",
+            "us_per_cost_unit": u, "link_gbs": cm.link_gbs, "link_latency_us": cm.link_latency_us,
+            "data_locality": {"max_us": max(dl.times), "times_us": dl.times},
+            "data_parallel": {"max_us": comp + xfer, "compute_us": comp, "all_to_all_us": xfer},
+            "joint": {"max_us": max(joint.times), "times_us": joint.times, "moves": joint.moves},
+            "dl_over_joint": max(dl.times) / max(max(joint.times), 1e-9),
+            "dp_over_joint": (comp + xfer) / max(max(joint.times), 1e-9)}
 
 
 def c4_point(dev, B, steps=20):
@@ -533,6 +572,8 @@ def c4_point(dev, B, steps=20):
     alg = synth.algorithmic_bytes(w.spec, sets[(steps - 1) % 2][0], n_vals)
     peak, _ = measured_peaks()
     info = plan.info()
+    # config 4's 8-GPU mapping (its full 131072-row batch), model-based
+    mapping = mapping_point(plan, w.spec, sets[0][1].sp_nnz, B, ms, world=8, B_eval=131072)
     plan.close()
     del sets
     torch.cuda.empty_cache()
@@ -540,7 +581,8 @@ def c4_point(dev, B, steps=20):
     return {"workload": "multihot_c4", "batch": B, "kernel_ms": ms, "value": B / (ms / 1e3), "unit": UNIT,
             "alg_bytes_per_launch": int(alg), "achieved_gbs": gbs, "frac": gbs / peak,
             "kernel": KERNEL_NAMES.get(info["kernel_last"], str(info["kernel_last"])),
-            "note": f"config 4 at {B} of its 131072 rows (host generation of the full batch is ~20 GB)"}
+            "note": f"config 4 at {B} of its 131072 rows (host generation of the full batch is ~20 GB)",
+            "mapping": mapping}
 
 
 def perop_baseline(w, host, dev, kern_ms, steps=10):

@@ -378,6 +378,33 @@ rap_status rap_place_comm(const double* cost, const int32_t* colocate, int32_t n
                           int64_t n_rows, const rap_comm_model* comm, int32_t* owner_out, double* load_out,
                           rap_residual* residual);
 
+/* Joint preprocessing-graph mapping (§7.2): start from
+ * the data-locality mapping (every output on the rank that consumes it,
+ * home[j]; home[j] = -1: a row-wise sharded table whose input every rank
+ * needs, so its graph is duplicated on every rank, L1526-1533), evaluate it
+ * with the co-running cost model, then repeatedly substitute: move one
+ * preprocessing graph (an output with its colocated outputs) from the rank
+ * with the highest cost to the one with the lowest, when that lowers the
+ * mapping's cost after charging the move's input communication (the raw
+ * rows to the new rank and the output rows back to the consumer,
+ * comm->row_bytes[j] per row over comm->link_gbs plus link_latency_us), until
+ * no substitution helps (L1592-1602).
+ *   cost[n]       HOST, per-output predicted cost units (rap_plan_output_costs)
+ *   colocate[n]   HOST or NULL, as rap_place
+ *   home[n]       HOST, consumer rank of each output, or -1 (duplicated)
+ *   n_rows        batch rows (row_bytes * n_rows = one output's traffic)
+ *   comm          HOST, the link model (us_per_unit converts cost units)
+ *   oc_us         overlap capacity of the training step per rank (us): the
+ *                 cost of a mapping is the largest exposed preprocessing
+ *                 time max_r max(0, T_r - oc_us), ties broken by max_r T_r,
+ *                 with T_r the rank's compute time plus its exchanges
+ *   owner_out[n]  HOST, the rank that evaluates each output (-1: every rank)
+ *   time_out      HOST double[world] or NULL: T_r of the final mapping (us)
+ *   n_moves       HOST or NULL: substitutions made */
+rap_status rap_place_joint(const double* cost, const int32_t* colocate, const int32_t* home, int32_t n,
+                           int32_t world, int64_t n_rows, const rap_comm_model* comm, double oc_us,
+                           int32_t* owner_out, double* time_out, int32_t* n_moves);
+
 /* A sharded plan: the graph restricted to its dense outputs (evaluated over
  * this rank's batch shard, rap_shard_rows) and the sparse outputs j with
  * sparse_owner[j] == rank (j counts the graph's sparse outputs in order),

@@ -2165,6 +2165,103 @@ rap_status rap_place(const double* cost, const int32_t* colocate, int32_t n, int
   return place_impl(cost, colocate, n, world, mode, n_rows, imbalance_tol, nullptr, owner_out, load_out, residual);
 }
 
+// Joint mapping (§7.2; include/rap.h).  A group = an
+// output and the outputs colocated with it (an NGram with its first source's
+// table) moves as one preprocessing graph.
+rap_status rap_place_joint(const double* cost, const int32_t* colocate, const int32_t* home, int32_t n,
+                           int32_t world, int64_t n_rows, const rap_comm_model* comm, double oc_us,
+                           int32_t* owner_out, double* time_out, int32_t* n_moves) {
+  if (n < 0 || world < 1 || n_rows < 0) return fail(RAP_ERR_INVALID_ARGUMENT, "bad size");
+  if (n > 0 && (!cost || !home || !owner_out)) return fail(RAP_ERR_INVALID_ARGUMENT, "NULL argument");
+  if (!comm || !(comm->us_per_unit > 0) || !(comm->link_gbs > 0) || !(comm->link_latency_us >= 0) ||
+      (n > 0 && !comm->row_bytes))
+    return fail(RAP_ERR_INVALID_ARGUMENT, "comm model: us_per_unit, link_gbs > 0, link_latency_us >= 0, row_bytes");
+  std::vector<int> anchor(n);
+  for (int j = 0; j < n; ++j) {
+    if (!(cost[j] >= 0)) return fail(RAP_ERR_INVALID_ARGUMENT, "cost must be >= 0");
+    if (home[j] < -1 || home[j] >= world) return fail(RAP_ERR_INVALID_ARGUMENT, "home[j] must be -1 or a rank");
+    const int c = colocate ? colocate[j] : -1;
+    if (c >= j || c < -1) return fail(RAP_ERR_INVALID_ARGUMENT, "colocate[j] must be -1 or < j");
+    anchor[j] = c < 0 ? j : anchor[c];
+    if (home[j] != home[anchor[j]]) return fail(RAP_ERR_INVALID_ARGUMENT, "colocated outputs must share their home");
+  }
+  // groups: cost (us), exchange time when away from home (us), home
+  std::vector<int> gid(n, -1), ghome;
+  std::vector<double> gus, gxus;
+  for (int j = 0; j < n; ++j) {
+    if (anchor[j] == j) {
+      gid[j] = (int)ghome.size();
+      ghome.push_back(home[j]);
+      gus.push_back(0.0);
+      gxus.push_back(comm->link_latency_us);
+    }
+    const int g = gid[anchor[j]];
+    gid[j] = g;
+    gus[g] += cost[j] * comm->us_per_unit;
+    if (!(comm->row_bytes[j] >= 0)) return fail(RAP_ERR_INVALID_ARGUMENT, "row_bytes must be >= 0");
+    gxus[g] += (double)n_rows * comm->row_bytes[j] / (1e3 * comm->link_gbs);
+  }
+  const int G = (int)ghome.size();
+  std::vector<int> gown(ghome);  // the data-locality mapping (L1524-1529)
+  // rank times: a duplicated graph (home -1, not moved) runs on every rank; a
+  // moved graph costs its compute and its exchange on the rank that runs it
+  auto times = [&](const std::vector<int>& own, std::vector<double>* T) {
+    T->assign(world, 0.0);
+    for (int g = 0; g < G; ++g) {
+      if (own[g] < 0) {
+        for (int r = 0; r < world; ++r) (*T)[r] += gus[g];
+      } else {
+        (*T)[own[g]] += gus[g] + (own[g] != ghome[g] ? gxus[g] : 0.0);
+      }
+    }
+  };
+  auto score = [&](const std::vector<double>& T) {  // (exposed, makespan)
+    double e = 0, m = 0;
+    for (double t : T) {
+      e = std::max(e, std::max(0.0, t - oc_us));
+      m = std::max(m, t);
+    }
+    return std::make_pair(e, m);
+  };
+  std::vector<double> T;
+  times(gown, &T);
+  auto best = score(T);
+  int moves = 0;
+  for (int it = 0; it < 4 * G + 4 && world > 1; ++it) {
+    int h = 0, l = 0;
+    for (int r = 0; r < world; ++r) {
+      if (T[r] > T[h]) h = r;
+      if (T[r] < T[l]) l = r;
+    }
+    if (h == l) break;
+    // substitution: the graph on h whose move to l lowers the cost most
+    int bg = -1;
+    std::pair<double, double> bs = best;
+    for (int g = 0; g < G; ++g) {
+      if (gown[g] != h) continue;
+      std::vector<int> own = gown;
+      own[g] = l;
+      std::vector<double> T2;
+      times(own, &T2);
+      const auto sc = score(T2);
+      if (sc.first < bs.first - 1e-9 || (sc.first <= bs.first + 1e-9 && sc.second < bs.second - 1e-9)) {
+        bs = sc;
+        bg = g;
+      }
+    }
+    if (bg < 0) break;  // no substitution improves the mapping (L1600-1602)
+    gown[bg] = l;
+    times(gown, &T);
+    best = bs;
+    ++moves;
+  }
+  for (int j = 0; j < n; ++j) owner_out[j] = gown[gid[j]];
+  if (time_out)
+    for (int r = 0; r < world; ++r) time_out[r] = T[r];
+  if (n_moves) *n_moves = moves;
+  return RAP_OK;
+}
+
 rap_status rap_place_comm(const double* cost, const int32_t* colocate, int32_t n, int32_t world, int32_t mode,
                           int64_t n_rows, const rap_comm_model* comm, int32_t* owner_out, double* load_out,
                           rap_residual* residual) {

@@ -149,6 +149,35 @@ def place(costs, colocate, world: int, mode: str = "balanced", n_rows: int = 0, 
     return Placement([int(x) for x in own[:n]], [float(x) for x in loads], r, mode)
 
 
+@dataclass
+class JointMapping:
+    owner: list    # rank evaluating each sparse output (-1: every rank, a duplicated graph)
+    times: list    # per-rank time of the mapping (us): compute plus its exchanges
+    moves: int     # substitutions made from the data-locality start
+
+
+def place_joint(costs, colocate, home, world: int, n_rows: int, comm: CommModel, row_bytes_, oc_us: float = 0.0):
+    """rap_place_joint (host only; §7.2): data-locality
+    mapping (home[j]: the consumer rank of output j, -1 = duplicated on every
+    rank), then substitutions of whole preprocessing graphs from the costliest
+    to the cheapest rank while the co-running cost (largest exposed time over
+    the overlap capacity oc_us, then the makespan) falls after charging the
+    moved graph's input communication."""
+    n = len(costs)
+    c = np.ascontiguousarray(costs, dtype=np.float64)
+    col = np.ascontiguousarray(colocate if colocate is not None else [-1] * n, dtype=np.int32)
+    hm = np.ascontiguousarray(home, dtype=np.int32)
+    rb = np.ascontiguousarray(row_bytes_ if row_bytes_ is not None else [0.0] * n, dtype=np.float64)
+    cm = rap.RapCommModel(comm.us_per_unit, comm.link_gbs, comm.link_latency_us, rb.ctypes.data if n else None)
+    own = np.zeros(max(n, 1), dtype=np.int32)
+    times = np.zeros(world, dtype=np.float64)
+    mv = C.c_int32()
+    rap._check(rap.load().rap_place_joint(c.ctypes.data if n else None, col.ctypes.data if n else None,
+                                          hm.ctypes.data if n else None, n, world, n_rows, C.byref(cm), float(oc_us),
+                                          own.ctypes.data, times.ctypes.data, C.byref(mv)))
+    return JointMapping([int(x) for x in own[:n]], [float(x) for x in times], int(mv.value))
+
+
 def plan_placement(spec, n_rows: int, sp_nnz, world: int, mode: str = "balanced", imbalance_tol=0.1,
                    device: int = 0, comm: CommModel | None = None) -> Placement:
     """Placement from the plan's own cost model (rap_plan_output_costs);

@@ -23,7 +23,7 @@ EXPORTS = ["rap_plan_create", "rap_plan_output_shape", "rap_preprocess", "rap_pr
            "rap_predict_latency_us", "rap_choose_budget", "rap_plan_info_get", "rap_debug_trace", "rap_plan_destroy",
            "rap_status_string", "rap_last_error", "rap_shard_rows", "rap_plan_output_costs", "rap_place",
            "rap_plan_create_sharded", "rap_jagged_append", "rap_set_kernel", "rap_check_overflow",
-           "rap_debug_jit_source", "rap_place_comm", "rap_predict_terms", "rap_sm_partition_stream",
+           "rap_debug_jit_source", "rap_place_comm", "rap_place_joint", "rap_predict_terms", "rap_sm_partition_stream",
            "rap_sm_partition_stream_destroy"]
 PLACE_MODES = {"balanced": 0, "round_robin": 1, "skewed": 2}
 RAP_OUT_CHAIN = 1
@@ -158,6 +158,9 @@ def load(build_if_stale: bool = False):
     L.rap_place_comm.restype = C.c_int
     L.rap_place_comm.argtypes = [P, P, C.c_int32, C.c_int32, C.c_int32, C.c_int64, C.POINTER(RapCommModel), P, P,
                                  C.POINTER(RapResidual)]
+    L.rap_place_joint.restype = C.c_int
+    L.rap_place_joint.argtypes = [P, P, P, C.c_int32, C.c_int32, C.c_int64, C.POINTER(RapCommModel), C.c_double, P, P,
+                                  C.POINTER(C.c_int32)]
     L.rap_plan_create_sharded.restype = C.c_int
     L.rap_plan_create_sharded.argtypes = [C.POINTER(RapGraph), C.POINTER(RapOpParam), C.c_int32, C.c_int32, C.c_int32,
                                           P, C.c_int32, C.c_int32, C.POINTER(P)]

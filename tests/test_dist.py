@@ -14,7 +14,7 @@ import socket
 import numpy as np
 import pytest
 
-from paper_conf_asplos_wangwdz0d24_b200 import dist, synth
+from paper_conf_asplos_wangwdz0d24_b200 import dist, rap, synth
 
 
 # ----------------------------------------------------------------- host logic
@@ -350,3 +350,84 @@ def test_two_processes_one_gpu_vs_oracle(mode):
     assert feats == list(range(34))
     if mode == "skewed":
         assert got[0]["residual"] is not None
+
+
+# ---- joint mapping loop (rap_place_joint, §7.2) ----
+def _joint_times(costs, colocate, home, owner, world, n_rows, cm, row_bytes):
+    """Independent restatement of rap_place_joint's cost model: a graph runs
+    on its owner (compute + its exchange when away from home), a duplicated
+    graph (owner -1) on every rank."""
+    T = [0.0] * world
+    for j, c in enumerate(costs):
+        us = c * cm.us_per_unit
+        if owner[j] < 0:
+            for r in range(world):
+                T[r] += us
+            continue
+        T[owner[j]] += us
+        if owner[j] != home[j]:
+            # exchange charged once per colocated group (at its anchor)
+            anchor = j
+            while colocate is not None and colocate[anchor] >= 0:
+                anchor = colocate[anchor]
+            grp = [k for k in range(len(costs)) if _anchor(colocate, k) == anchor]
+            if j == anchor:
+                T[owner[j]] += cm.link_latency_us + sum(n_rows * row_bytes[k] / (1e3 * cm.link_gbs) for k in grp)
+    return T
+
+
+def _anchor(colocate, k):
+    while colocate is not None and colocate[k] >= 0:
+        k = colocate[k]
+    return k
+
+
+def test_joint_mapping_keeps_locality_when_moves_do_not_pay():
+    costs = [100.0] * 8 + [300.0] * 8
+    home = [0] * 8 + [1] * 8
+    slow = dist.CommModel(us_per_unit=0.01, link_gbs=0.001, link_latency_us=1e6)
+    m = dist.place_joint(costs, None, home, 2, 65536, slow, [100.0] * 16)
+    assert m.owner == home and m.moves == 0
+
+
+def test_joint_mapping_balances_a_skewed_home_and_stops_at_a_local_optimum():
+    rng = np.random.default_rng(7)
+    n, world, B = 40, 4, 65536
+    costs = list(rng.uniform(50, 500, n))
+    home = [0 if j < n // 2 else 1 + j % (world - 1) for j in range(n)]  # rank 0: half the graphs (skew)
+    rb = list(rng.uniform(8, 40, n))
+    cm = dist.CommModel(us_per_unit=0.02, link_gbs=700.0, link_latency_us=5.0)
+    m = dist.place_joint(costs, None, home, world, B, cm, rb)
+    T0 = _joint_times(costs, None, home, home, world, B, cm, rb)
+    T = _joint_times(costs, None, home, m.owner, world, B, cm, rb)
+    assert np.allclose(T, m.times, rtol=1e-9)
+    assert m.moves > 0 and max(T) < max(T0)
+    # stopping rule: no single graph of the costliest rank lowers the cost on the cheapest one
+    h, lo = int(np.argmax(T)), int(np.argmin(T))
+    for j in range(n):
+        if m.owner[j] != h:
+            continue
+        o = list(m.owner)
+        o[j] = lo
+        assert max(_joint_times(costs, None, home, o, world, B, cm, rb)) >= max(T) - 1e-9
+
+
+def test_joint_mapping_duplicated_and_colocated_graphs():
+    costs = [200.0, 50.0, 400.0, 100.0, 30.0]
+    colocate = [-1, 0, -1, -1, -1]  # output 1 (an NGram) shares output 0's rank
+    home = [0, 0, 0, -1, 0]         # output 3: a row-wise table, duplicated on every rank
+    cm = dist.CommModel(us_per_unit=0.05, link_gbs=700.0, link_latency_us=1.0)
+    m = dist.place_joint(costs, colocate, home, 3, 4096, cm, [16.0] * 5)
+    assert m.owner[3] == -1
+    assert m.owner[0] == m.owner[1]
+    T = _joint_times(costs, colocate, home, m.owner, 3, 4096, cm, [16.0] * 5)
+    assert np.allclose(T, m.times, rtol=1e-9)
+    assert all(t >= 100.0 * 0.05 for t in T)  # the duplicated graph's compute on every rank
+
+
+def test_joint_mapping_rejects_bad_input():
+    cm = dist.CommModel(us_per_unit=0.05)
+    with pytest.raises(rap.RapError):
+        dist.place_joint([1.0, 2.0], [-1, 0], [0, 1], 2, 128, cm, [1.0, 1.0])  # colocated, different homes
+    with pytest.raises(rap.RapError):
+        dist.place_joint([1.0], None, [5], 2, 128, cm, [1.0])  # home out of range
