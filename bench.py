@@ -56,6 +56,7 @@ def parse():
     ap.add_argument("--no-c4", action="store_true", help="skip the config-4 (multi-hot) sub-measurement")
     ap.add_argument("--c4-batch", type=int, default=16384, help="rows of the config-4 sub-measurement")
     ap.add_argument("--no-plans", action="store_true", help="skip the Table 3 Plan 2 / 3 sub-measurements")
+    ap.add_argument("--ngram-sweep", default="", help="e.g. 8,16,32,64: growing-NGram co-run sweep (Fig 11 analog)")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="N>1: gloo = host-staged exchange (ranks sharing one GPU: tests)")
     return ap.parse_args()
@@ -471,6 +472,9 @@ def run_rap(args):
             del louts
         del train
         torch.cuda.empty_cache()
+    ngram_sweep = None
+    if world == 1 and not args.profile and args.ngram_sweep:
+        ngram_sweep = ngram_sweep_point(dev, B, [int(k) for k in args.ngram_sweep.split(",") if k])
     mapping = None
     if world == 1 and not args.profile and args.workload in ("c1", "c2"):
         mapping = mapping_point(plan, w.spec, raw0.sp_nnz, B, kern_ms)
@@ -493,7 +497,8 @@ def run_rap(args):
                            "l2_policy": f"rotate {nsets} distinct input/output sets, {nsets * set_bytes / 2**20:.0f} MB "
                                         f"total vs L2 {l2 / 2**20:.0f} MB"},
                 "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks, "gpu_launches": K,
-                "corun": corun, "fusion": fusion, "graph": graph, "c4": c4, "plans": plans, "mapping": mapping}
+                "corun": corun, "fusion": fusion, "graph": graph, "c4": c4, "plans": plans, "mapping": mapping,
+                "ngram_sweep": ngram_sweep}
         print(json.dumps(line), flush=True)
     plan.close()
     if world > 1:
@@ -504,6 +509,40 @@ def run_rap(args):
 
 
 KERNEL_NAMES = {1: "tiled", 2: "rows (interpreted)", 3: "rows (generated, NVRTC sm_100a)"}
+
+
+def ngram_sweep_point(dev, B, counts):
+    """Fig 11 analog: the C2 graph with a growing number
+    of trigram features beside the fixed synthetic DLRM training step: per
+    count, the fused launch alone and the training step's slowdown when the
+    launch co-runs on a low-priority stream at the full budget and at the
+    budget rap_choose_budget picks (the paper's turning point: a > 10 % rise)."""
+    import torch
+
+    from paper_conf_asplos_wangwdz0d24_b200 import corun as cr, rap, synth
+
+    train = cr.DLRMStep(dev)
+    out = []
+    for k in counts:
+        w = synth.c2_terabyte(0, n_ngram=k)
+        plan = rap.Plan(w.spec, device=dev.index)
+        sets = []
+        for i in range(2):
+            h = synth.make_batch(w, B, seed=300 + i)
+            r = rap.DeviceBatch(h, dev)
+            sets.append((r, rap.DeviceOutput(plan, B, r.sp_nnz, dev)))
+        m = cr.measure(plan, sets, train, [plan.info()["sm_budget"]], steps=12, warmup=3,
+                       choose=(B, sets[0][0].sp_nnz))
+        full = m["per_budget"][0]
+        out.append({"n_ngram": k, "sparse_outputs": 26 + k, "kernel": KERNEL_NAMES.get(plan.info()["kernel_last"], "?"),
+                    "prep_alone_ms": full["prep_alone_ms"], "slowdown_full_budget": full["slowdown"],
+                    "chosen_budget": m["chosen"]["sm_budget"], "slowdown_chosen": m["chosen"]["slowdown"],
+                    "train_step_alone_ms": m["train_step_alone_ms"]})
+        plan.close()
+        del sets
+        torch.cuda.empty_cache()
+    del train
+    return out
 
 
 def mapping_point(plan, spec, sp_nnz, B, kern_ms, world=8, B_eval=None):

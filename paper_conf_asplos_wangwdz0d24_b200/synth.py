@@ -175,13 +175,15 @@ DENSE_BORDERS = np.array([0.5, 1.5, 2.5, 4.5, 8.5, 16.5, 32.5, 64.5, 128.5, 256.
                           1024.5, 2048.5, 4096.5, 8192.5], dtype=np.float32)
 
 
-def c2_terabyte(seed: int = 0, mapid_size: int = 4096) -> Workload:
+def c2_terabyte(seed: int = 0, mapid_size: int = 4096, n_ngram: int = 8) -> Workload:
     """Config 2: Criteo-Terabyte-shaped full op graph:
     dense: FillNull(0) x13; Logit cols 0-5; BoxCox(lambda cycling) cols 6-12;
     cols 11-12 also Bucketize(15 borders)->OneHot(16).
     sparse x26: FillNull(0)->Clamp(0,2^32-1)->[MapId on 6]->SigridHash->[Bucketize on 4]->FirstX(1).
     NGram: 8 trigram features over 3 post-SigridHash sources each, M=10M.
-    152 ops; 45 dense output columns; 34 sparse output features."""
+    152 ops; 45 dense output columns; 34 sparse output features.
+    n_ngram != 8: that many trigram features (sources cycling over the 26
+    hashed features; the growing-NGram sweep, Fig 11)."""
     nodes, outs_dense, outs_sparse = [], [], []
     lambdas = [0.0, 0.25, 0.5, -0.5]
     fill_node = {}
@@ -219,14 +221,15 @@ def c2_terabyte(seed: int = 0, mapid_size: int = 4096) -> Workload:
             nodes.append(_n("bucketize", [("n", len(nodes) - 1)], borders=borders))
         nodes.append(_n("firstx", [("n", len(nodes) - 1)], x=1))
         outs_sparse.append(len(nodes) - 1)
-    ng_salts = salts(seed, 8, "ngram_salt")
-    for g in range(8):
+    ng_salts = salts(seed, n_ngram, "ngram_salt")
+    for g in range(n_ngram):
         srcs = [(3 * g) % 26, (3 * g + 1) % 26, (3 * g + 2) % 26]
         nodes.append(_n("ngram", [("n", hashed[s]) for s in srcs], n=3, salt=ng_salts[g], max_value=10_000_000))
         outs_sparse.append(len(nodes) - 1)
     spec = {"n_dense": 13, "n_sparse": 26, "nodes": nodes, "outputs": outs_dense + onehots + outs_sparse}
     kinds = ["unit"] * 6 + ["count"] * 7
-    return Workload("criteo_terabyte_c2", spec, kinds, M.copy())
+    name = "criteo_terabyte_c2" if n_ngram == 8 else f"criteo_terabyte_c2_ngram{n_ngram}"
+    return Workload(name, spec, kinds, M.copy())
 
 
 def c4_multihot(seed: int = 0, n_features: int = 512, mean_len: float = 20.0, firstx: int = 32) -> Workload:
