@@ -241,7 +241,8 @@ RAP_HD uint64_t splitmix_H(uint64_t x) {
 // (warp-parallel reductions); (4) lengths, offsets and ids.
 constexpr int kRbChunk = 256;   // rows per chunk (one per thread)
 constexpr int kRbMaxFg = 64;    // feature groups
-constexpr int kRbMaxFL = 64;    // sparse outputs per feature group
+constexpr int kRbMaxFL = 64;    // sparse outputs per feature group (interpreted form)
+constexpr int kJitMaxF = 192;   // sparse outputs of the generated kernel's one group (<= its 224 sparse threads)
 constexpr int kRbMaxF = 1024;   // sparse outputs of a plan the row-block kernel takes
 constexpr int kRbMaxCols = 64;  // raw sparse columns the row-block kernel addresses
 constexpr int kRbMaxDense = 32; // raw dense columns

@@ -132,6 +132,7 @@ struct rap_plan {
   int jit_state = 0, jit_ctas_per_sm = 0;  // state of the last variant asked for
   int jit_st[2] = {0, 0}, jit_occ[2] = {0, 0};
   int jit_smem = 0, jit_dense_bytes = 0, jit_id_slots = 0, jit_tab_bytes = 0;
+  int jit_max_fl = 0;  // the generated kernel's one group: every output (<= kJitMaxF)
   double jit_s = 0;
 };
 
@@ -843,7 +844,7 @@ static int jit_threads(const rap_plan* P) {
   return nd ? 224 + 32 * nd : kRbChunk;  // the generated kernel's CTA (rap_jit.cpp Gen::threads)
 }
 static int jit_base_smem(const rap_plan* P, int dense_bytes) {
-  return rows_smem_bytes(dense_bytes, P->rb_max_fl, P->rb_max_cols, 0, (int)P->souts.size(), 0, 0, jit_pitch(P), 0,
+  return rows_smem_bytes(dense_bytes, P->jit_max_fl, P->rb_max_cols, 0, (int)P->souts.size(), 0, 0, jit_pitch(P), 0,
                          P->jit_tab_bytes);
 }
 static int jit_tile_bytes(const rap_plan* P) {
@@ -1000,6 +1001,7 @@ void build_rows(rap_plan* P) {
   }
   P->rb_fits = P->n_sparse_in <= kRbMaxCols && P->n_dense_in <= kRbMaxDense && F <= kRbMaxF;
   P->rb_max_fl = std::max(1, std::min(F, kRbMaxFL));
+  P->jit_max_fl = std::max(1, std::min(F, kJitMaxF));
   P->rb_max_cols = std::max(1, (int)P->used_sparse.size());
 }
 
@@ -1204,7 +1206,7 @@ rap_status rap_plan_create(const rap_graph* graph, const rap_op_param* params, i
     P->jit_dense_bytes = std::max(P->jit_dense_bytes, jit_dense_need(jit_view(P)));  // + the emitter's memo rows
     P->jit_tab_bytes = jit_table_bytes(jit_view(P));
     P->jit_id_slots = jit_id_slots(P);
-    P->jit_smem = rows_smem_bytes(P->jit_dense_bytes, P->rb_max_fl, P->rb_max_cols, 0, (int)P->souts.size(), 0,
+    P->jit_smem = rows_smem_bytes(P->jit_dense_bytes, P->jit_max_fl, P->rb_max_cols, 0, (int)P->souts.size(), 0,
                                   P->jit_id_slots, jit_pitch(P), 0, P->jit_tab_bytes);
     if (P->rb_smem > 227 * 1024) P->rb_fits = 0;
   }
@@ -1668,7 +1670,7 @@ static void rows_geometry(const rap_plan* P, int64_t B, const int64_t* nnz, int 
   double acc = 0;
   g->fg_off[0] = 0;
   for (int i = 0; i < F; ++i) {
-    const bool full = i - start >= kRbMaxFL;
+    const bool full = !one_group && i - start >= kRbMaxFL;
     const bool due = gcount + 1 < n_fg && acc + 0.5 * cost[i] >= W * (double)(gcount + 1) / (double)n_fg && i > start;
     if ((full || due) && gcount + 1 < kRbMaxFg) {
       g->fg_off[++gcount] = i;
@@ -1753,7 +1755,10 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
     // the generated kernel: one group of every output over as many row blocks
     // as the budget's slots hold (RAP_JIT_SMALL_B: below this batch size the
     // interpreted form's feature groups fill the slots instead)
-    const bool jit_geo = jit && (B >= jit_min_rows() || jit_pairs(P));
+    // (more outputs than an interpreted group holds: the generated kernel's one
+    // group takes up to kJitMaxF of them)
+    const int Fp = (int)P->souts.size();
+    const bool jit_geo = jit && (Fp > kRbMaxFL ? Fp <= kJitMaxF : (B >= jit_min_rows() || jit_pairs(P)));
     rows_geometry(P, B, raw->sp_nnz, jit ? P->jit_occ[iv] : P->rb_ctas_per_sm, &g, 0, 0, jit_geo);
     if (!jit || !(g.n_fg == 1 && drow0 == 0 && drows == B))  // interpreted form: its geometry, dense CTAs
       rows_geometry(P, B, raw->sp_nnz, P->rb_ctas_per_sm, &g, n_dense);
@@ -1777,6 +1782,7 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
       g.len_cache = 0;
       g.n_memo = 0;
       g.dense_bytes = P->jit_dense_bytes;
+      g.max_fl = P->jit_max_fl;
       g.id_slots = P->jit_id_slots;
       g.pitch = jit_pitch(P);
       g.feat_recs = 0;
@@ -1999,7 +2005,8 @@ static PredTerms predict_terms(const rap_plan* P, int64_t B, const int64_t* nnz,
     RbGeom g;
     memset(&g, 0, sizeof(g));
     const int jocc = P->jit_occ[iv] > 0 ? P->jit_occ[iv] : P->rb_ctas_per_sm;
-    rows_geometry(P, B, nnz, want_jit ? jocc : P->rb_ctas_per_sm, &g, 0, b);
+    rows_geometry(P, B, nnz, want_jit ? jocc : P->rb_ctas_per_sm, &g, 0, b,
+                  want_jit && F > kRbMaxFL && F <= kJitMaxF);  // as launch(): one group beyond kRbMaxFL
     const bool jit = want_jit && g.n_fg == 1 && drow0 == 0 && drows == B;
     if (!jit) rows_geometry(P, B, nnz, P->rb_ctas_per_sm, &g, n_dense, b);
     const int chunk = jit ? 224 : kRbChunk;

@@ -587,7 +587,7 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
   __shared__ int16_t s_slot[MS];  // raw sparse column -> staged slot (-1: not staged)
   __shared__ int16_t s_cols[MS];  // staged slot -> raw sparse column
   __shared__ unsigned long long s_mask[(MS + 63) / 64];
-  __shared__ int16_t s_fidx[kRbMaxFL];
+  __shared__ int16_t s_fidx[kJitMaxF > kRbMaxFL ? kJitMaxF : kRbMaxFL];
   __shared__ int s_last, s_fmax;
   __shared__ uint64_t s_sbar;  // staging mbarrier (bulk copies)
   __shared__ int s_sphase;

@@ -75,6 +75,16 @@ def test_c2_terabyte_ragged(env, B):
     check(env, w.spec, synth.make_batch(w, B, seed=B + 7))
 
 
+@pytest.mark.parametrize("n_ngram,B", [(64, 1000), (128, 4099)])
+def test_c2_many_ngram_outputs(env, n_ngram, B):
+    """The growing-NGram graphs (Fig 11 sweep): 90 / 154 sparse outputs, past
+    an interpreted group's 64 -- the generated kernel takes them as one group
+    (kJitMaxF), the others split groups."""
+    _, synth, _, _ = env
+    w = synth.c2_terabyte(0, n_ngram=n_ngram)
+    check(env, w.spec, synth.make_batch(w, B, seed=B + n_ngram))
+
+
 def test_c2_terabyte_full_size(env):
     """BASELINE config 2 at its full batch (65536), the launch bench.py times."""
     _, synth, _, _ = env
