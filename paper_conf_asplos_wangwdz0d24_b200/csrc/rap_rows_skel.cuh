@@ -689,6 +689,10 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
   }
   trace_stamp(c, 7);
   if (kDW && warp >= kWS) {
+    // Pol::kDenseLate: the dense warps start once the sparse warps announced
+    // the block's totals (named barrier 2), so the staging and length phases
+    // on the critical path do not share the SM's issue slots with them
+    if (Pol::kDenseLate) asm volatile("bar.sync 2, %0;" ::"r"(kT) : "memory");
     Pol::dense_warp(p, s, x);  // the dense outputs of rows [R0, R1), concurrent with the sparse phases
     trace_stamp_warp(c, 15);
   } else {
@@ -720,6 +724,7 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
     __threadfence();  // release: the block's totals before the announcement
     atomicAdd(pub, 1ull);
   }
+  if (kDW && Pol::kDenseLate) asm volatile("bar.arrive 2, %0;" ::"r"(kT) : "memory");  // the dense warps may start
   trace_stamp(c, 1);
 
   if (!Pol::kSetupEarly) Pol::setup(p, s, x);  // records used only in (4)
