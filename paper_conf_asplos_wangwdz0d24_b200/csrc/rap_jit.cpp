@@ -1449,6 +1449,8 @@ struct Gen {
     body += std::string("  static constexpr bool kSetupEarly = ") + (tab_total ? "true" : "false") + ";\n";
     body += "  static constexpr bool kPairs = " + std::string(pairs() ? "true" : "false") + ";\n";
     body += "  static constexpr int kThreads = " + i2s(threads()) + ";\n";
+    body += std::string("  static constexpr bool kBasesByDense = ") +
+            (dense_mode() == 3 && env_int("RAP_JIT_BASES_DENSE", 0) ? "true" : "false") + ";\n";
     body += std::string("  static constexpr bool kDenseLate = ") +
             (dense_mode() == 3 && env_int("RAP_JIT_DENSE_LATE", 0) ? "true" : "false") + ";\n";
     body += "  template <class P>\n"

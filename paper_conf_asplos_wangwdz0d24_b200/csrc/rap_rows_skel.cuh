@@ -565,6 +565,67 @@ __device__ __forceinline__ void jl_ngram_lp(const RbSmem& s, const JLNgram<K>& G
   *P0 = s.wb[G.q * 8 + wi] + rb_warp_excl<kSmall>(*L, lane);
 }
 
+// Phase (3) by one warp (the generated kernel's first dense warp, while the
+// sparse warps run pre_emit): wait until every CTA announced its totals,
+// then each output's first offset for the block (as rows_body's phase 3) and
+// the per-block capacity check.  blk totals: the CTA's s.ws sums.
+template <bool kSmall>
+__device__ __forceinline__ void rb_bases_warp(const Common& c, const RbGeom& g, const RbSmem& s, const int16_t* fidx,
+                                              int FL, int fmax, int rb, int n_rb, int kws, long long chain0,
+                                              const unsigned long long* pub, int lane) {
+  if (lane == 0) {
+    int ns = 32;
+    while (ld_acquire(pub) < (unsigned long long)gridDim.x) {
+      __nanosleep(ns);
+      ns = min(ns * 2, 256);
+    }
+  }
+  __syncwarp();
+  long long* sT = reinterpret_cast<long long*>(s.dense);  // [fmax + 1]
+  long long* sL = sT + (fmax + 1);                          // [fmax + 1]
+  for (int f = lane; f <= fmax; f += 32) sT[f] = (long long)__ldcg(g.tot + f);
+  const int nsb = rb / kRbSup, rb0 = nsb * kRbSup;
+  for (int f0 = 0; f0 <= fmax; f0 += 4) {
+    long long v[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const int f = min(f0 + u, fmax);
+      long long a = 0;
+      if (lane < nsb) a = (long long)__ldcg(g.sup + (int64_t)f * kRbSupMax + lane);
+      if (rb0 + lane < rb) a += (long long)__ldcg(g.agg + (int64_t)f * n_rb + rb0 + lane);
+      v[u] = a;
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const long long t = rb_warp_sum<kSmall>(v[u]);
+      if (lane == 0 && f0 + u <= fmax) sL[f0 + u] = t;
+    }
+  }
+  __syncwarp();
+  long long P = chain0;
+  for (int f0 = 0; f0 <= fmax; f0 += 32) {
+    const int f = f0 + lane;
+    const long long t = f <= fmax ? sT[f] : 0ll;
+    long long x = t;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const long long y = __shfl_up_sync(0xffffffffu, x, d);
+      if (lane >= d) x += y;
+    }
+    if (f <= fmax) sT[f] = P + x - t;
+    P += __shfl_sync(0xffffffffu, x, 31);
+  }
+  __syncwarp();
+  for (int fl = lane; fl < FL; fl += 32) {
+    const int f = fidx[fl];
+    long long blk = 0;
+    for (int w = 0; w < kws; ++w) blk += s.ws[fl * 8 + w];
+    s.base[fl] = sT[f] + sL[f];
+    if (sT[f] + sL[f] + blk > c.values_cap) atomicExch(c.err, 1);  // values_capacity understated (sp_nnz)
+  }
+  __syncwarp();
+}
+
 // Context of one CTA: its feature group (processing indices [pb, pe)) and
 // row block [R0, R1).
 struct RbCtx {
@@ -693,6 +754,15 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
     // the block's totals (named barrier 2), so the staging and length phases
     // on the critical path do not share the SM's issue slots with them
     if (Pol::kDenseLate) asm volatile("bar.sync 2, %0;" ::"r"(kT) : "memory");
+    if (Pol::kBasesByDense && warp == kWS && FL > 0 && nrows > 0) {
+      // phase (3) for the sparse warps, while they run pre_emit: their
+      // per-output sums (s.ws) are visible after named barrier 4, the bases
+      // are handed back on named barrier 3
+      asm volatile("bar.sync 4, %0;" ::"r"(kTS + 32) : "memory");
+      rb_bases_warp<kSmall>(c, g, s, s_fidx, FL, s_fmax, rb, n_rb, kWS, chain0, pub, lane);
+      trace_stamp_warp(c, 4);
+      asm volatile("bar.arrive 3, %0;" ::"r"(kTS + 32) : "memory");
+    }
     Pol::dense_warp(p, s, x);  // the dense outputs of rows [R0, R1), concurrent with the sparse phases
     trace_stamp_warp(c, 15);
   } else {
@@ -725,6 +795,8 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
     atomicAdd(pub, 1ull);
   }
   if (kDW && Pol::kDenseLate) asm volatile("bar.arrive 2, %0;" ::"r"(kT) : "memory");  // the dense warps may start
+  constexpr bool kDB = kDW && Pol::kBasesByDense;  // phase (3) by the first dense warp
+  if (kDB && FL > 0 && nrows > 0) asm volatile("bar.arrive 4, %0;" ::"r"(kTS + 32) : "memory");
   trace_stamp(c, 1);
 
   if (!Pol::kSetupEarly) Pol::setup(p, s, x);  // records used only in (4)
@@ -757,6 +829,9 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
   trace_stamp(c, 2);
 
   if (FL > 0 && nrows > 0) {
+    if (kDB) {
+      asm volatile("bar.sync 3, %0;" ::"r"(kTS + 32) : "memory");  // the dense warp's bases
+    } else {
     // (3) wait until every CTA announced its totals (all resident: cooperative launch)
     if (tid == 0) {
       int ns = 32;
@@ -825,6 +900,7 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
     }
     rb_sync<kDW>();
     trace_stamp(c, 4);
+    }  // phase (3) by the sparse warps
 
     // (4) lengths, offsets and ids, chunk by chunk
     for (int ch = 0; ch < nch; ++ch) {
