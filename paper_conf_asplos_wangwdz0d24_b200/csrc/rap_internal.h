@@ -361,8 +361,10 @@ inline int jit_dense_mode(int n_sparse_out, int d_out, int n_dprogs, int rb_dens
     return 0;
   }
 #ifndef __CUDACC_RTC__
-  const char* want = getenv("RAP_JIT_DENSE");  // "1" / "2": force that mode (experiment knob)
-  const int wm = want ? atoi(want) : 3;
+  static const int wm = [] {  // "1" / "2": force that mode (experiment knob; read once per process)
+    const char* want = getenv("RAP_JIT_DENSE");
+    return want ? atoi(want) : 3;
+  }();
 #else
   const int wm = 3;
 #endif

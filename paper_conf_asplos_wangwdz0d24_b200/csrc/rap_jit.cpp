@@ -1642,7 +1642,8 @@ int launch_jit(JitModule* m, const Common& c, const RbGeom& g, const LaunchRaw& 
   attr[0].id = cudaLaunchAttributeCooperative;
   attr[0].val.cooperative = 1;
   cfg.attrs = attr;
-  cfg.numAttrs = env_int("RAP_NONCOOP", 0) ? 0 : 1;  // (experiment knob: launch-cost measurement only)
+  static const int noncoop = env_int("RAP_NONCOOP", 0);  // (experiment knob: launch-cost measurement only)
+  cfg.numAttrs = noncoop ? 0 : 1;
   void* args[1] = {&p};
   cudaError_t e = cudaLaunchKernelExC(&cfg, k, args);
   if (e != cudaSuccess) return (int)e;

@@ -826,14 +826,18 @@ int memo_prefix(const rap_plan* P, const Chain& o, const Canon& qo, const Chain&
 // Warp-pair mode of the generated kernel (rap_rows_skel.cuh kPairs): two
 // threads per row, each evaluating half of the outputs.
 static int jit_pairs(const rap_plan* P) {
-  const char* env = getenv("RAP_JIT_PAIRS");  // "0" / "1": force off / on (experiment knob)
-  if (env && env[0] == '0') return 0;
-  if (env && env[0] == '1') return P->souts.size() >= 2 ? 1 : 0;
-  return 0;
+  static const int knob = [] {  // "0" / "1": force off / on (experiment knob; read once per process)
+    const char* env = getenv("RAP_JIT_PAIRS");
+    return env ? (env[0] == '1' ? 1 : 0) : 0;
+  }();
+  return knob && P->souts.size() >= 2 ? 1 : 0;
 }
 static int64_t jit_min_rows() {
-  const char* env = getenv("RAP_JIT_SMALL_B");  // (experiment knob)
-  return env ? atoll(env) : (int64_t)1 << 62;
+  static const int64_t v = [] {  // (experiment knob; read once per process)
+    const char* env = getenv("RAP_JIT_SMALL_B");
+    return env ? (int64_t)atoll(env) : (int64_t)1 << 62;
+  }();
+  return v;
 }
 static int jit_pitch(const rap_plan*) { return 0; }
 static int jit_threads(const rap_plan* P) {
@@ -1650,8 +1654,11 @@ static void rows_geometry(const rap_plan* P, int64_t B, const int64_t* nnz, int 
     n_rb = nb256;
     n_fg = std::max<int64_t>(fg_min, std::min<int64_t>({(int64_t)F, (int64_t)kRbMaxFg, slots / n_rb}));
   }
-  const char* env = getenv("RAP_RB_ROWS");  // experiment knob: rows per block
-  int64_t rows = env ? std::max<int64_t>(32, atoll(env) / 32 * 32) : 32 * ((B + 32 * n_rb - 1) / (32 * n_rb));
+  static const int64_t knob_rows = [] {  // experiment knob: rows per block (read once per process)
+    const char* env = getenv("RAP_RB_ROWS");
+    return env ? std::max<int64_t>(32, atoll(env) / 32 * 32) : (int64_t)0;
+  }();
+  int64_t rows = knob_rows ? knob_rows : 32 * ((B + 32 * n_rb - 1) / (32 * n_rb));
   n_rb = std::max<int64_t>(1, (B + rows - 1) / rows);
   if (n_rb * n_fg > kMaxCtas) {  // knob out of range: back to the default
     rows = 32 * ((B + 32 * (kMaxCtas / n_fg) - 1) / (32 * (kMaxCtas / n_fg)));
