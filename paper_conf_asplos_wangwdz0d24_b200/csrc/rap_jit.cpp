@@ -436,6 +436,8 @@ struct Gen {
   // 32 rows.  split: a unit boundary (no NGram separated from a memo provider)
   // nearest to half the predicted cost.
   bool pairs() const { return v.pairs != 0; }
+  // programmatic dependent launch of consecutive launches (experiment knob)
+  static bool jit_pdl() { return env_int("RAP_JIT_PDL", 0) != 0; }
   // MapId: the first two probe slots loaded ahead (RAP_JIT_MAP1=1: one, experiment knob)
   static bool map2() { return env_int("RAP_JIT_MAP1", 0) == 0; }
   std::string rbrow() const { return "rb_row_p<" + i2s(kRbChunk + 4) + ">"; }
@@ -1449,6 +1451,7 @@ struct Gen {
     body += std::string("  static constexpr bool kSetupEarly = ") + (tab_total ? "true" : "false") + ";\n";
     body += "  static constexpr bool kPairs = " + std::string(pairs() ? "true" : "false") + ";\n";
     body += "  static constexpr int kThreads = " + i2s(threads()) + ";\n";
+    body += std::string("  static constexpr bool kPDL = ") + (jit_pdl() ? "true" : "false") + ";\n";
     body += std::string("  static constexpr bool kBasesByDense = ") +
             (dense_mode() == 3 && env_int("RAP_JIT_BASES_DENSE", 0) ? "true" : "false") + ";\n";
     body += std::string("  static constexpr bool kDenseLate = ") +
@@ -1643,7 +1646,17 @@ int launch_jit(JitModule* m, const Common& c, const RbGeom& g, const LaunchRaw& 
   attr[0].val.cooperative = 1;
   cfg.attrs = attr;
   static const int noncoop = env_int("RAP_NONCOOP", 0);  // (experiment knob: launch-cost measurement only)
-  cfg.numAttrs = noncoop ? 0 : 1;
+  static const int pdl = env_int("RAP_JIT_PDL", 0);
+  cudaLaunchAttribute attr2[2];
+  attr2[0] = attr[0];
+  attr2[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr2[1].val.programmaticStreamSerializationAllowed = 1;
+  if (pdl && !noncoop) {
+    cfg.attrs = attr2;
+    cfg.numAttrs = 2;
+  } else {
+    cfg.numAttrs = noncoop ? 0 : 1;
+  }
   void* args[1] = {&p};
   cudaError_t e = cudaLaunchKernelExC(&cfg, k, args);
   if (e != cudaSuccess) return (int)e;

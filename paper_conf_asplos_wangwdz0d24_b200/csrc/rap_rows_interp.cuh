@@ -308,6 +308,7 @@ struct InterpPolicy {
   static constexpr bool kPre = false;  // (the generated policy's pre_emit: rap_jit.cpp)
   static constexpr bool kDenseLate = false;
   static constexpr bool kBasesByDense = false;
+  static constexpr bool kPDL = false;
   struct PreState {};
   template <class P>
   static __device__ __forceinline__ PreState pre_emit(const P&, const RbSmem&, const RbCtx&, int64_t, int) {

@@ -689,8 +689,13 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
   const int FL = x.FL, rb = x.rb;
   const int nrows = (int)max((int64_t)0, x.R1 - x.R0);
   const int nch = (nrows + kTS - 1) / kTS;
-  const long long chain0 = c.chain ? (long long)__ldg(c.offsets) : 0ll;
   unsigned long long* const pub = g.sched + 2;  // CTAs whose totals are stored
+  // programmatic dependent launch (Pol::kPDL): the next launch on the stream
+  // may start its CTAs as this one's leave the SMs; before reading any data
+  // a previous launch may have written (its inputs, the chained offsets, the
+  // counters) it waits for the previous grid (griddepcontrol.wait below), so
+  // only the CTA setup overlaps the previous launch's tail
+  if (Pol::kPDL) asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
   trace_stamp(c, 0);
 
   if (tid == 0) {
@@ -743,6 +748,8 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
     if (on) s_cols[before] = (int16_t)col;
   }
   __syncthreads();
+  if (Pol::kPDL) asm volatile("griddepcontrol.wait;" ::: "memory");  // the previous launch's grid is done
+  const long long chain0 = c.chain ? (long long)__ldcg(c.offsets) : 0ll;
   trace_stamp(c, 6);
   if (Pol::kSetupEarly) {
     Pol::setup(p, s, x);
