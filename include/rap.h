@@ -135,7 +135,7 @@ typedef struct {
   int64_t* offsets;
   int64_t* values;
   int64_t values_capacity;
-  int32_t flags;         /* 0, or RAP_OUT_CHAIN */
+  int32_t flags;         /* 0, RAP_OUT_CHAIN, RAP_OUT_VALUES_I32 */
   int32_t reserved;
 } rap_output;
 
@@ -148,6 +148,12 @@ typedef struct {
  * points at the first row slot of this launch.  Used to stitch multi-GPU
  * residual pieces. */
 #define RAP_OUT_CHAIN 1
+/* Cast (Table 1; reading R13): the values are emitted as
+ * int32 -- `values` points to int32[values_capacity] and every id is cast by
+ * two's-complement truncation ((int32_t)id, torch's .to(torch.int32)).
+ * rap_preprocess only (the host-buffer entries and chained launches take
+ * int64 values: RAP_ERR_UNSUPPORTED). */
+#define RAP_OUT_VALUES_I32 2
 
 struct rap_plan;
 typedef struct rap_plan rap_plan;

@@ -193,7 +193,7 @@ struct Common {
   int64_t dense_row0;         // dense outputs cover raw rows [dense_row0, dense_row0 + n_dense_rows)
   int64_t n_dense_rows;       // (a sharded plan's batch shard; else 0 and n_rows)
   int32_t chain;              // 1: offsets/value positions start at offsets[0] (rap_output RAP_OUT_CHAIN)
-  int32_t pad_chain;
+  int32_t vi32;               // 1: values are int32 (rap_output RAP_OUT_VALUES_I32, Cast)
   // sched[0] = CTAs done, sched[1] = launch epoch; the last CTA resets the
   // counter and advances the epoch, so launch parameters are identical from
   // call to call (CUDA-graph replayable).
@@ -391,7 +391,7 @@ inline int jit_dense_mode(int n_sparse_out, int d_out, int n_dprogs, int rb_dens
 // Generate the CUDA source of the plan's policy (small: 32-bit scans, every
 // offset < 2^31; else 64-bit) and compile it with NVRTC for sm_100a (cached
 // per source text in the process).  Returns nullptr and fills *log on failure.
-JitModule* jit_build(const JitPlanView& v, bool small, char* log, int log_cap);
+JitModule* jit_build(const JitPlanView& v, int variant, char* log, int log_cap);  // bit 0 small, bit 1 int32 values
 int jit_occupancy(JitModule* m, int smem_bytes, int threads, int* ctas_per_sm);
 // Region-0 shared-memory bytes the generated kernel needs beyond the dense
 // tile (the column emitter's memo rows; 0 if none).

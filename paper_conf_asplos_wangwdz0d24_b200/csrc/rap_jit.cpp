@@ -943,7 +943,7 @@ struct Gen {
       // (5) value stores
       for (int q : canon) {
         const std::string Q = i2s(q);
-        s += "    stg_s64_if(L" + Q + " > 0 && P" + Q + " < c.values_cap, c.values + P" + Q + ", v" + Q + ");\n";
+        s += "    stv_if(L" + Q + " > 0 && P" + Q + " < c.values_cap, c, P" + Q + ", v" + Q + ");\n";
       }
       // the batch's NGram outputs (their providers' memo words are final)
       for (int q : ngram) {
@@ -980,8 +980,8 @@ struct Gen {
             s += "        int64_t v = (int64_t)reduce_M(h, " + lit64(pg.ng.M) + ");\n";
             s += stages(pg.cn, pg.cn.mask, "v", "true", -1, "");
             s += "        const long long at = P" + Q + " + (cnt - " + i2s(n) + ");\n";
-            s += "        stg_s64_if(fast && " + pr + " && cnt >= " + i2s(n) + " && cnt - " + i2s(n) + " < L" + Q +
-                 " && at < c.values_cap, c.values + at, v);\n      }\n";
+            s += "        stv_if(fast && " + pr + " && cnt >= " + i2s(n) + " && cnt - " + i2s(n) + " < L" + Q +
+                 " && at < c.values_cap, c, at, v);\n      }\n";
           }
         }
         s += "      if (!fast && L" + Q + " > 0) late |= 1u << " + i2s(late_slot[q]) + ";\n    }\n  }\n";
@@ -1100,7 +1100,7 @@ struct Gen {
         s += "    {\n        int64_t v = " + X + ".valid ? pf" + Q + " : " + lit64(pg.ch.fill) + ";\n";
         s += stages(cn, cn.mask, "v", X + ".valid", is_prov[f] ? memo_point(R, cn) : -1, "m" + Fs,
                     (cn.mask & CB_MAPID) ? "pk" + Q : "");
-        s += "        stg_s64_if(L" + Q + " > 0 && P" + Q + " < c.values_cap, c.values + P" + Q + ", v);\n";
+        s += "        stv_if(L" + Q + " > 0 && P" + Q + " < c.values_cap, c, P" + Q + ", v);\n";
         if (R.cap[0] > 1) {
           s += "        for (int32_t j = 1; j < L" + Q + "; ++j) {\n";
           s += "          int64_t w = __ldg(p.val[" + i2s(col) + "] + " + X + ".a + j);\n";
@@ -1138,8 +1138,8 @@ struct Gen {
             s += "        int64_t v = (int64_t)reduce_M(h, " + lit64(pg.ng.M) + ");\n";
             s += stages(pg.cn, pg.cn.mask, "v", "true", -1, "");
             s += "        const long long at = P" + Q + " + (cnt - " + i2s(n) + ");\n";
-            s += "        stg_s64_if(fast && " + pr + " && cnt >= " + i2s(n) + " && cnt - " + i2s(n) + " < L" + Q +
-                 " && at < c.values_cap, c.values + at, v);\n      }\n";
+            s += "        stv_if(fast && " + pr + " && cnt >= " + i2s(n) + " && cnt - " + i2s(n) + " < L" + Q +
+                 " && at < c.values_cap, c, at, v);\n      }\n";
           }
         }
         if (n_late < 32) {  // rows the register path cannot take: after the straight-line code
@@ -1308,7 +1308,7 @@ struct Gen {
       if (prov) s += "        int64_t mv = 0;\n";
       s += stages(cn, cn.mask, "v", X + ".valid", prov ? memo_point(R, cn) : -1, "mv", map ? "pk" + Q : "");
       if (prov) s += "        memo[" + i2s(col_memo[f] * kRbChunk) + " + r] = mv;\n";
-      s += "        stg_s64_if(L" + Q + " > 0 && P" + Q + " < c.values_cap, c.values + P" + Q + ", v);\n";
+      s += "        stv_if(L" + Q + " > 0 && P" + Q + " < c.values_cap, c, P" + Q + ", v);\n";
       if (R.cap[0] > 1) {
         s += "        for (int32_t j = 1; j < L" + Q + "; ++j) {\n";
         s += "          int64_t w = __ldg(p.val[" + i2s(col) + "] + " + X + ".a + j);\n";
@@ -1348,8 +1348,8 @@ struct Gen {
           s += "        int64_t v = (int64_t)reduce_M(h, " + lit64(pg.ng.M) + ");\n";
           s += stages(pg.cn, pg.cn.mask, "v", "true", -1, "");
           s += "        const long long at = P" + Q + " + (cnt - " + i2s(n) + ");\n";
-          s += "        stg_s64_if(fast && " + pr + " && cnt >= " + i2s(n) + " && cnt - " + i2s(n) + " < L" + Q +
-               " && at < c.values_cap, c.values + at, v);\n      }\n";
+          s += "        stv_if(fast && " + pr + " && cnt >= " + i2s(n) + " && cnt - " + i2s(n) + " < L" + Q +
+               " && at < c.values_cap, c, at, v);\n      }\n";
         }
       }
       s += "      const bool late = !fast && L" + Q + " > 0;\n"
@@ -1433,9 +1433,12 @@ struct Gen {
     return true;
   }
 
-  std::string source(bool small) {
+  // variant: bit 0 = 32-bit scans (every offset < 2^31), bit 1 = int32 values (Cast)
+  std::string source(int variant) {
+    const bool small = (variant & 1) != 0;
     std::string s;
     s += "// generated by rap_jit.cpp for one plan (" + i2s(F) + " sparse outputs)\n";
+    s += (variant & 2) ? "#define RAP_VALUES_I32 1\n" : "#define RAP_VALUES_I64 1\n";
     if (env_int("RAP_JIT_STCS", 1)) s += "#define RAP_ST_CS 1\n";  // streaming output stores (rap_rows_skel.cuh)
     if (env_int("RAP_JIT_LDCS", 0)) s += "#define RAP_LD_CS 1\n";  // (experiment knob)
     if (env_int("RAP_JIT_STPLAIN", 0)) s += "#define RAP_ST_PLAIN 1\n";  // (experiment knob)
@@ -1476,16 +1479,17 @@ struct Gen {
         };
         const size_t k = e.find("bool ovf = false;");
         if (k != std::string::npos) e.insert(k, "unsigned long long sink = 0;\n    ");
-        if (ns == 1 || ns == 3) rep("stg_s64_if(L", "RAP_SINK(L");
+        if (ns == 1 || ns == 3) rep("stv_if(L", "RAP_SINKV(L");
         if (ns == 1 || ns == 2) {
           rep("stg_s32_if(in,", "RAP_SINK(in,");
           rep("stg_s64_if(in,", "RAP_SINK(in,");
         }
-        rep("stg_s64_if(fast", "RAP_SINK(fast");
-        if (ns == 2) rep("RAP_SINK(fast", "stg_s64_if(fast");
+        rep("stv_if(fast", "RAP_SINKV(fast");
+        if (ns == 2) rep("RAP_SINKV(fast", "stv_if(fast");
         const size_t z = e.rfind("if (ovf) atomicExch");
         e.insert(z, "if (sink == 0x5eed5eedull) c.values[0] = (int64_t)sink;\n    ");
         body += "#define RAP_SINK(q, p, v) (sink ^= (q) ? (unsigned long long)(v) + (unsigned long long)(p) : 0ull)\n";
+        body += "#define RAP_SINKV(q, c_, p, v) (sink ^= (q) ? (unsigned long long)(v) + (unsigned long long)(p) : 0ull)\n";
       }
       body += e;
     }
@@ -1554,7 +1558,7 @@ bool nvrtc_cubin(const std::string& src, std::vector<char>* cubin, std::string* 
 
 }  // namespace
 
-std::string jit_generate(const JitPlanView& v) { return Gen(v).source(true); }
+std::string jit_generate(const JitPlanView& v) { return Gen(v).source(1); }
 
 int jit_dense_need(const JitPlanView& v) { return Gen(v).dense_need(); }
 
@@ -1565,9 +1569,9 @@ bool jit_compile_only(const std::string& src, std::string* log) {
   return nvrtc_cubin(src, &cubin, log);
 }
 
-JitModule* jit_build(const JitPlanView& v, bool small, char* log, int log_cap) {
+JitModule* jit_build(const JitPlanView& v, int variant, char* log, int log_cap) {
   Gen gen(v);
-  const std::string src = gen.source(small);
+  const std::string src = gen.source(variant);
   {
     std::lock_guard<std::mutex> lk(g_cache_mu);
     if (!g_cache) g_cache = new std::map<std::string, JitModule*>();

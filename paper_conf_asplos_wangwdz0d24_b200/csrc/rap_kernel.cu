@@ -208,6 +208,14 @@ __device__ __noinline__ long long value_tile_ngram(const P& p, int f, int64_t rt
 // Output stores are streaming (st.global.cs, evict-first in L2): written once,
 // never read back by the kernel.
 __device__ __forceinline__ void st_cs64(int64_t* p, int64_t v) { __stcs(reinterpret_cast<long long*>(p), (long long)v); }
+// A value of the jagged output (R17) in the launch's value type: int64, or
+// int32 under Cast (RAP_OUT_VALUES_I32, two's-complement truncation).
+__device__ __forceinline__ void st_val(int64_t* values, bool i32, long long pos, int64_t v) {
+  if (i32)
+    __stcs(reinterpret_cast<int*>(values) + pos, (int)v);
+  else
+    st_cs64(values + pos, v);
+}
 
 // Lengths (int4) and offsets (2 x longlong2) of the lane's 4 rows.
 __device__ __forceinline__ void store_quad(int32_t* lp, int64_t* op, int64_t row, int64_t B, const int32_t* l,
@@ -237,6 +245,7 @@ __device__ __noinline__ long long value_tile_canon(const P& p, const FeatCtx& fc
   const int64_t r0 = rt * kTileRows;
   const int64_t row = r0 + 4 * lane;
   int64_t* values = p.c.values;
+  const bool vi32 = p.c.vi32 != 0;  // Cast: int32 values (RAP_OUT_VALUES_I32)
   const long long cap = p.c.values_cap;
   const int64_t* itab = p.c.itab;
   const int32_t* off = p.off[fc.src];
@@ -272,7 +281,7 @@ __device__ __noinline__ long long value_tile_canon(const P& p, const FeatCtx& fc
 #pragma unroll
     for (int k = 0; k < 4; ++k) {
       const long long pos = lb + e[k];
-      if (l[k] == 1 && pos < cap) st_cs64(values + (pos), v[k]);
+      if (l[k] == 1 && pos < cap) st_val(values, vi32, pos, v[k]);
     }
     if (last && lane == 31) {
       p.c.offsets[(int64_t)p.c.n_sparse_out * B] = base + T;  // total, R17
@@ -319,7 +328,7 @@ __device__ __noinline__ long long value_tile_canon(const P& p, const FeatCtx& fc
 #pragma unroll
     for (int u = 0; u < 4; ++u) {
       const long long pos = base + eb + 32 * u + lane;
-      if (((act >> u) & 1u) && pos < cap) st_cs64(values + (pos), x[u]);
+      if (((act >> u) & 1u) && pos < cap) st_val(values, vi32, pos, x[u]);
     }
   }
   return T;
@@ -391,6 +400,7 @@ __device__ __noinline__ long long value_chunk_canon(const P& p, const FeatCtx& f
   cp_async_wait_all();  // each lane reads only the ids it staged
   trace_clk(p.c, 10, sid[4 * lane]);
   int64_t* values = p.c.values;
+  const bool vi32 = p.c.vi32 != 0;  // Cast: int32 values (RAP_OUT_VALUES_I32)
   const long long cap = p.c.values_cap;
   long long run = base;
   const int64_t* const itab_h = p.c.itab;  // hoisted (value_tile_multi)
@@ -427,7 +437,7 @@ __device__ __noinline__ long long value_chunk_canon(const P& p, const FeatCtx& f
 #pragma unroll
         for (int k = 0; k < 4; ++k) {
           const long long pos = lb + e[k];
-          if (l[k] && pos < cap) st_cs64(values + (pos), v[4 * jj + k]);
+          if (l[k] && pos < cap) st_val(values, vi32, pos, v[4 * jj + k]);
         }
         if (f == p.c.n_sparse_out - 1 && rt == p.c.tiles_per_feature - 1 && lane == 31) {
           p.c.offsets[(int64_t)p.c.n_sparse_out * B] = run + Tj;  // total, R17
@@ -536,6 +546,7 @@ __device__ __noinline__ long long value_tile_multi(const P& p, const FeatCtx& fc
   __syncwarp();
   const int64_t* val = p.val[src];
   int64_t* values = p.c.values;
+  const bool vi32 = p.c.vi32 != 0;  // Cast: int32 values (RAP_OUT_VALUES_I32)
   const long long cap = p.c.values_cap;
   // hoisted: the window loop's stores go through a generic pointer that the
   // compiler cannot prove disjoint from the parameter block, so a p.c field
@@ -605,14 +616,13 @@ __device__ __noinline__ long long value_tile_multi(const P& p, const FeatCtx& fc
     canon_apply_n<4>(fc.q, itab, x, act, full);
     const long long pos0 = base + w * 128 + lane;
     if (act == 15u && pos0 + 96 < cap) {
-      int64_t* dst = values + pos0;
 #pragma unroll
-      for (int u = 0; u < 4; ++u) st_cs64(dst + 32 * u, x[u]);
+      for (int u = 0; u < 4; ++u) st_val(values, vi32, pos0 + 32 * u, x[u]);
     } else {
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
         const long long pos = pos0 + 32 * u;
-        if (((act >> u) & 1u) && pos < cap) st_cs64(values + (pos), x[u]);
+        if (((act >> u) & 1u) && pos < cap) st_val(values, vi32, pos, x[u]);
       }
     }
   }
@@ -631,6 +641,7 @@ __device__ __noinline__ long long value_tile_generic(const P& p, int f, int64_t 
   int64_t* offsets = p.c.offsets + (int64_t)f * B;
   int32_t* lengths = p.c.lengths + (int64_t)f * B;
   int64_t* values = p.c.values;
+  const bool vi32 = p.c.vi32 != 0;  // Cast: int32 values (RAP_OUT_VALUES_I32)
   const long long cap = p.c.values_cap;
   const int64_t* itab = p.c.itab;
   const Chain ch = pg.ch;
@@ -690,7 +701,7 @@ __device__ __noinline__ long long value_tile_generic(const P& p, int f, int64_t 
 #pragma unroll
     for (int g = 0; g < kGroups; ++g) {
       const long long pos = base + gb[g] + lex[g];
-      if (len[g] == 1 && pos < cap) st_cs64(values + (pos), v1[g]);
+      if (len[g] == 1 && pos < cap) st_val(values, vi32, pos, v1[g]);
     }
     return run;
   }
@@ -753,7 +764,7 @@ __device__ __noinline__ void value_group_general(const P& p, int f, int64_t row0
         v = src_value(p, ops, pg.tab_off, ch, st_r, row0 + r, j);
       }
       const long long pos = gbase + e;
-      if (pos < cap) st_cs64(p.c.values + (pos), v);
+      if (pos < cap) st_val(p.c.values, p.c.vi32 != 0, pos, v);
     }
   }
 }
@@ -1017,7 +1028,7 @@ __device__ __noinline__ long long ngram_tile_fast(const P& p, int f, int64_t rt,
   const long long cap = p.c.values_cap;
 #pragma unroll
   for (int kk = 0; kk < 4; ++kk)
-    if (((act >> kk) & 1u) && lb + e[kk] < cap) st_cs64(p.c.values + (lb + e[kk]), o[kk]);
+    if (((act >> kk) & 1u) && lb + e[kk] < cap) st_val(p.c.values, p.c.vi32 != 0, lb + e[kk], o[kk]);
   if (f == p.c.n_sparse_out - 1 && rt == p.c.tiles_per_feature - 1 && lane == 31) {
     p.c.offsets[(int64_t)p.c.n_sparse_out * B] = base + T;  // total, R17
     if (base + T > cap) atomicExch(p.c.err, 1);
@@ -1039,6 +1050,7 @@ __device__ __noinline__ long long value_tile_ngram(const P& p, int f, int64_t rt
   int64_t* offsets = p.c.offsets + (int64_t)f * B;
   int32_t* lengths = p.c.lengths + (int64_t)f * B;
   int64_t* values = p.c.values;
+  const bool vi32 = p.c.vi32 != 0;  // Cast: int32 values (RAP_OUT_VALUES_I32)
   const long long cap = p.c.values_cap;
 
   // NGram feature (R7): per row the k source lists, windows over their
@@ -1111,13 +1123,13 @@ __device__ __noinline__ long long value_tile_ngram(const P& p, int f, int64_t rt
         }
         const int64_t v = canon1(qp, itab, (int64_t)reduce_M(h, pg.ng.M), true);
         const long long pos = run + lx + j;
-        if (pos < cap) st_cs64(values + (pos), v);
+        if (pos < cap) st_val(values, vi32, pos, v);
       }
     } else if (__all_sync(0xffffffffu, len <= 1)) {
       if (len == 1) {
         const long long pos = run + lx;
         const int64_t v = ngram_window(p, pg, ops, st_s + lane, sl_s + lane, 32, row, 0);
-        if (pos < cap) st_cs64(values + (pos), v);
+        if (pos < cap) st_val(values, vi32, pos, v);
       }
     } else {
       const int mylex = inr ? lx : INT_MAX;
@@ -1133,7 +1145,7 @@ __device__ __noinline__ long long value_tile_ngram(const P& p, int f, int64_t rt
         if (e < T) {
           const int64_t v = ngram_window(p, pg, ops, st_s + r, sl_s + r, 32, r0 + 32 * g + r, e - lex_r);
           const long long pos = run + e;
-          if (pos < cap) st_cs64(values + (pos), v);
+          if (pos < cap) st_val(values, vi32, pos, v);
         }
       }
     }

@@ -128,9 +128,9 @@ struct rap_plan {
   unsigned long long* d_agg_rb = nullptr;  // [n_sparse_out][n_rb] row-block totals, then [n_sparse_out] totals
   int rb_last_n_rb = 0, rb_last_n_fg = 0, rb_last_rows = 0;
   // plan-specialised row-block kernel (rap_jit.cpp), built on first use
-  JitModule* jit[2] = {nullptr, nullptr};  // [small] variants
+  JitModule* jit[4] = {nullptr, nullptr, nullptr, nullptr};  // [small | int32 values << 1] variants
   int jit_state = 0, jit_ctas_per_sm = 0;  // state of the last variant asked for
-  int jit_st[2] = {0, 0}, jit_occ[2] = {0, 0};
+  int jit_st[4] = {0, 0, 0, 0}, jit_occ[4] = {0, 0, 0, 0};
   int jit_smem = 0, jit_dense_bytes = 0, jit_id_slots = 0, jit_tab_bytes = 0;
   int jit_max_fl = 0;  // the generated kernel's one group: every output (<= kJitMaxF)
   double jit_s = 0;
@@ -1388,6 +1388,9 @@ rap_status rap_check_overflow(rap_plan* P, int32_t* overflow) {
 
 static rap_status check_batch(const rap_plan* P, const rap_raw_batch* raw, const rap_output* out) {
   if (!P || !raw || !out) return fail(RAP_ERR_INVALID_ARGUMENT, "NULL argument");
+  if (out->flags & ~(RAP_OUT_CHAIN | RAP_OUT_VALUES_I32)) return fail(RAP_ERR_INVALID_ARGUMENT, "unknown output flags");
+  if ((out->flags & RAP_OUT_CHAIN) && (out->flags & RAP_OUT_VALUES_I32))
+    return fail(RAP_ERR_UNSUPPORTED, "RAP_OUT_VALUES_I32 with RAP_OUT_CHAIN");
   if (raw->n_rows < 0) return fail(RAP_ERR_INVALID_ARGUMENT, "n_rows < 0");
   if (raw->n_rows > (int64_t)INT32_MAX - kTileRows) return fail(RAP_ERR_INVALID_ARGUMENT, "n_rows too large");
   const int64_t B = raw->n_rows;
@@ -1587,15 +1590,14 @@ static rap_status update_partition(rap_plan* P, int64_t B, const int64_t* nnz, i
 
 // The generated kernel of this plan (rap_jit.cpp), variant `small`: built on
 // first use; on failure the plan keeps the interpreted row-block kernel.
-static bool jit_ready(rap_plan* P, bool small) {
-  const int i = small ? 1 : 0;
+static bool jit_ready(rap_plan* P, int i) {  // i: variant (bit 0 small, bit 1 int32 values)
   if (P->jit_st[i] == 0) {
     const char* env = getenv("RAP_JIT");
     if (env && env[0] == '0') {
       P->jit_st[i] = -1;
     } else {
       char log[2048] = {0};
-      JitModule* m = jit_build(jit_view(P), small, log, (int)sizeof(log));
+      JitModule* m = jit_build(jit_view(P), i, log, (int)sizeof(log));
       int occ = 0;
       if (m && jit_occupancy(m, P->jit_smem, jit_threads(P), &occ) == 0 && occ >= 1) {
         P->jit[i] = m;
@@ -1732,6 +1734,7 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
   c.dense_row0 = drow0;
   c.n_dense_rows = drows;
   c.chain = (out->flags & RAP_OUT_CHAIN) ? 1 : 0;
+  c.vi32 = (out->flags & RAP_OUT_VALUES_I32) ? 1 : 0;
   c.sched = P->d_sched;
   c.agg = P->d_agg;
   c.dense_out = out->dense_out;
@@ -1757,8 +1760,8 @@ static rap_status launch(rap_plan* P, const rap_raw_batch* raw, const rap_output
     // 32-bit scans when every offset of this launch fits 31 bits
     const bool small = !c.chain && values_bound(P, B, raw->sp_nnz) < (int64_t)INT32_MAX - 1;
     const bool want_jit = P->kernel_mode == RAP_KERNEL_JIT || P->kernel_mode == RAP_KERNEL_AUTO;
-    const bool jit = want_jit && jit_ready(P, small);
-    const int iv = small ? 1 : 0;
+    const int iv = (small ? 1 : 0) | (c.vi32 ? 2 : 0);
+    const bool jit = want_jit && jit_ready(P, iv);
     // the generated kernel: one group of every output over as many row blocks
     // as the budget's slots hold (RAP_JIT_SMALL_B: below this batch size the
     // interpreted form's feature groups fill the slots instead)
@@ -1964,10 +1967,12 @@ static rap_status preprocess_host_impl(rap_plan* P, const rap_raw_batch* raw, co
 }
 
 rap_status rap_preprocess_host(rap_plan* P, const rap_raw_batch* raw, const rap_output* out, void* stream) {
+  if (out && (out->flags & RAP_OUT_VALUES_I32)) return fail(RAP_ERR_UNSUPPORTED, "RAP_OUT_VALUES_I32: rap_preprocess only");
   return preprocess_host_impl(P, raw, out, stream, true);
 }
 
 rap_status rap_preprocess_host_async(rap_plan* P, const rap_raw_batch* raw, const rap_output* out, void* stream) {
+  if (out && (out->flags & RAP_OUT_VALUES_I32)) return fail(RAP_ERR_UNSUPPORTED, "RAP_OUT_VALUES_I32: rap_preprocess only");
   return preprocess_host_impl(P, raw, out, stream, false);
 }
 

@@ -352,11 +352,33 @@ __device__ __forceinline__ void stg_s64_if(bool q, int64_t* p, int64_t v) {
                "r"((unsigned)q));
 }
 #endif
-__device__ __forceinline__ void rb_store(const Common& c, long long pos, int64_t v) {
-  if (pos < c.values_cap)
-    stg_s64(c.values + pos, v);
+// A value store of element pos (R17 values) in the launch's value type:
+// int64, or int32 under Cast (RAP_OUT_VALUES_I32; the generated kernel
+// compiles one variant per type, RAP_VALUES_I32 / RAP_VALUES_I64).
+__device__ __forceinline__ bool values_i32(const Common& c) {
+#if defined(RAP_VALUES_I32)
+  return true;
+#elif defined(RAP_VALUES_I64)
+  return false;
+#else
+  return c.vi32 != 0;
+#endif
+}
+__device__ __forceinline__ void stv_if(bool q, const Common& c, long long pos, int64_t v) {
+  if (values_i32(c))
+    stg_s32_if(q, reinterpret_cast<int32_t*>(c.values) + pos, (int32_t)v);
   else
+    stg_s64_if(q, c.values + pos, v);
+}
+__device__ __forceinline__ void rb_store(const Common& c, long long pos, int64_t v) {
+  if (pos < c.values_cap) {
+    if (values_i32(c))
+      stg_s32(reinterpret_cast<int32_t*>(c.values) + pos, (int32_t)v);
+    else
+      stg_s64(c.values + pos, v);
+  } else {
     atomicExch(c.err, 1);
+  }
 }
 // lengths[oi] and offsets[oi] of one (output, row)
 __device__ __forceinline__ void rb_store_lo(const Common& c, int64_t oi, int32_t len, long long pos) {
@@ -492,7 +514,7 @@ __device__ __forceinline__ void jl_canon(const P& p, const RbSmem& s, const JLCa
     v = (valid || (Q.nullm & CB_BUCKET)) ? t : v;
     if (Q.memo == CB_BUCKET) *memo = v;
   }
-  stg_s64_if(L > 0 && P0 < c.values_cap, c.values + P0, v);
+  stv_if(L > 0 && P0 < c.values_cap, c, P0, v);
 }
 
 // First id of a canonical output's row (0-id rows read a word of the plan blob).
@@ -545,7 +567,7 @@ __device__ __forceinline__ bool jl_ngram(const P& p, const RbSmem& s, const JLNg
       for (int j = 0; j < N; ++j) h = splitmix_H(h ^ w[j]);
       const int64_t v = (int64_t)reduce_M(h, G.M);
       const long long at = P0 + (cnt - N);
-      stg_s64_if(fast && pr && cnt >= N && cnt - N < L && at < c.values_cap, c.values + at, v);
+      stv_if(fast && pr && cnt >= N && cnt - N < L && at < c.values_cap, c, at, v);
     }
   }
   return !fast && L > 0;

@@ -90,6 +90,7 @@ class RapPlanInfo(C.Structure):
 # rap_set_kernel modes (include/rap.h).  DEFAULT_KERNEL is applied to every new
 # Plan (env RAP_KERNEL; tests set it to run each parity case on both kernels).
 KERNEL_AUTO, KERNEL_TILED, KERNEL_ROWS, KERNEL_JIT = 0, 1, 2, 3
+OUT_CHAIN, OUT_VALUES_I32 = 1, 2  # rap_output.flags (include/rap.h)
 DEFAULT_KERNEL = int(os.environ.get("RAP_KERNEL", "0"))
 
 
@@ -326,7 +327,8 @@ def row_view(raw: "DeviceBatch", row0: int, n_rows: int) -> "RapRawBatch":
 class DeviceOutput:
     """Output tensors (device, or pinned host when pin=True) + their C struct."""
 
-    def __init__(self, plan, n_rows, sp_nnz, device, pin=False, dense_ld=None, capacity=None):
+    def __init__(self, plan, n_rows, sp_nnz, device, pin=False, dense_ld=None, capacity=None, values_i32=False):
+        """values_i32: the ids emitted as int32 (Cast, RAP_OUT_VALUES_I32)."""
         import torch
 
         d, f, vb = plan.output_shape(n_rows, sp_nnz)
@@ -337,10 +339,12 @@ class DeviceOutput:
         self.lengths = torch.empty(max(n_rows * f, 1), dtype=torch.int32, **kw)
         self.offsets = torch.empty(n_rows * f + 1, dtype=torch.int64, **kw)
         cap = vb if capacity is None else capacity
-        self.values = torch.empty(max(cap, 1), dtype=torch.int64, **kw)
+        self.values = torch.empty(max(cap, 1), dtype=torch.int32 if values_i32 else torch.int64, **kw)
         self.n_rows, self.ld = n_rows, ld
         self.struct = RapOutput(self.dense.data_ptr(), ld, self.lengths.data_ptr(), self.offsets.data_ptr(),
                                 self.values.data_ptr(), cap)
+        if values_i32:
+            self.struct.flags = OUT_VALUES_I32
 
     def to_numpy(self):
         B, d, f = self.n_rows, self.d_out, self.f_out

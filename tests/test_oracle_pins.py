@@ -412,3 +412,12 @@ def test_spec_goldens_regenerate():
     have = _load("spec_goldens.json")
     want = m.goldens()
     assert have["sigridhash"] == want["sigridhash"] and have["ngram"] == want["ngram"]
+
+
+def test_cast_int32_reading_r13():
+    """Cast (Table 1, reading R13): an id cast to int32 keeps its low 32
+    bits as a two's-complement value -- numpy's astype, checked on hand-worked
+    values (the GPU int32 emission is compared with the oracle's ids cast this way)."""
+    ids = np.array([5, -1, 2**31 - 1, 2**31, 2**31 + 5, 2**32 + 7, -(2**31) - 1, -(2**63)], dtype=np.int64)
+    want = [5, -1, 2147483647, -2147483648, -2147483643, 7, 2147483647, 0]
+    assert ids.astype(np.int32).tolist() == want
