@@ -473,7 +473,7 @@ static_assert(kMultiRing + 4 * 128 * 8 <= kWarpScr, "multi-id tile scratch");
 // before its start, then applies the few change points inside the window;
 // ids are cp.async-staged into a 4-slot ring with kMultiDepth windows in
 // flight.
-template <class P>
+template <bool I32, class P>  // I32: int32 values (Cast), a compile-time branch of the window loop
 __device__ __noinline__ long long value_tile_multi(const P& p, const FeatCtx& fc, int64_t rt, int lane, long long base,
                                                    unsigned char* wscr) {
   int32_t* soff = reinterpret_cast<int32_t*>(wscr);        // [132]
@@ -546,7 +546,7 @@ __device__ __noinline__ long long value_tile_multi(const P& p, const FeatCtx& fc
   __syncwarp();
   const int64_t* val = p.val[src];
   int64_t* values = p.c.values;
-  const bool vi32 = p.c.vi32 != 0;  // Cast: int32 values (RAP_OUT_VALUES_I32)
+  constexpr bool vi32 = I32;  // Cast: int32 values (RAP_OUT_VALUES_I32)
   const long long cap = p.c.values_cap;
   // hoisted: the window loop's stores go through a generic pointer that the
   // compiler cannot prove disjoint from the parameter block, so a p.c field
@@ -1382,7 +1382,9 @@ __global__ void __launch_bounds__(kThreads, RAP_MIN_CTAS) rap_fused_kernel(const
           continue;
         }
         // multi-id rows: element-parallel tiles
-        for (int j = 0; j < nt; ++j) run += value_tile_multi(p, fc, t + j - (int64_t)f * T, lane, run, wscr);
+        for (int j = 0; j < nt; ++j)
+          run += p.c.vi32 ? value_tile_multi<true>(p, fc, t + j - (int64_t)f * T, lane, run, wscr)
+                          : value_tile_multi<false>(p, fc, t + j - (int64_t)f * T, lane, run, wscr);
         t += nt;
         continue;
       }

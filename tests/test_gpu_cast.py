@@ -52,6 +52,8 @@ def run_cast(env, kmode, spec_, host):
 @pytest.mark.parametrize("wl,B", [("c1", 4096), ("c2", 3000), ("c2", 65536), ("c4", 1500), ("plan2", 2000)])
 def test_cast_int32_configs(env, kmode, wl, B):
     _, synth, _, _ = env
+    if wl == "c4" and kmode != 1:
+        pytest.skip("512 raw columns: the tiled kernel only (rap_set_kernel rows / jit: UNSUPPORTED)")
     w = {"c1": synth.c1_kaggle, "c2": synth.c2_terabyte, "c4": synth.c4_multihot,
          "plan2": lambda s: synth.plan_graph(2, s)}[wl](0)
     run_cast(env, kmode, w.spec, synth.make_batch(w, B, seed=B + 3))
