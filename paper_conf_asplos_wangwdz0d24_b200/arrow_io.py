@@ -103,7 +103,9 @@ def write_parquet(batches, path: str):
     import pyarrow.parquet as pq
 
     rbs = [arrow_from_batch(b) for b in batches]
-    pq.write_table(pa.Table.from_batches(rbs), path, row_group_size=max(rb.num_rows for rb in rbs))
+    with pq.ParquetWriter(path, rbs[0].schema) as wr:  # each batch its own row group
+        for rb in rbs:
+            wr.write_table(pa.Table.from_batches([rb]), row_group_size=rb.num_rows)
 
 
 def read_parquet_batches(path: str, n_dense: int, n_sparse: int):

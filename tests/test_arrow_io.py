@@ -53,7 +53,7 @@ def test_arrow_round_trip_and_oracle(wl, B):
 
 def test_parquet_row_groups(tmp_path):
     w = synth.c1_kaggle(0)
-    bs = [synth.make_batch(w, 1024, seed=s) for s in (1, 2, 3)]
+    bs = [synth.make_batch(w, B, seed=s) for s, B in ((1, 1024), (2, 3000), (3, 77))]
     path = os.path.join(tmp_path, "b.parquet")
     arrow_io.write_parquet(bs, path)
     back = list(arrow_io.read_parquet_batches(path, 13, 26))
