@@ -504,24 +504,77 @@ struct Gen {
     return s;
   }
 
+  // ---- dense-warp tail: the last outputs of the processing order (whole
+  // NGram units, ~tail_frac of the predicted cost) are emitted by the dense
+  // warps once their tiles are done, one row warp at a time, so the sparse
+  // warps' chains are that much shorter (one-chunk blocks, dense mode 3) ----
+  int tail_split() const {
+    if (!batch_ok() || pairs() || dense_mode() != 3 || loop_plan_ok()) return F;
+    const double frac = env_int("RAP_JIT_TAIL_PCT", 20) / 100.0;
+    if (frac <= 0) return F;
+    std::vector<double> pre(F + 1, 0.0);
+    for (int q = 0; q < F; ++q) pre[q + 1] = pre[q] + out_cost(q);
+    int best = F;
+    double bd = 1e30;
+    for (int sp = std::min(F, batch_k()); sp < F; ++sp) {  // the tail never takes batch 0 (pre_emit)
+      bool ok = true;
+      for (int q = sp; q < F && ok; ++q) {
+        const RbFeat& R = v.feat[v.perm[q]];
+        if (R.emit != 3) continue;
+        for (int i = 0; i < R.k; ++i)
+          if (R.prov[i] >= 0 && R.prov[i] < sp) ok = false;
+      }
+      if (!ok) continue;
+      const double d = std::fabs((pre[F] - pre[sp]) - frac * pre[F]);
+      if (d < bd) {
+        bd = d;
+        best = sp;
+      }
+    }
+    return best;
+  }
+  bool loop_plan_ok() const { return const_cast<Gen*>(this)->loop_plan().ok; }
   std::string emit_fn() {
     std::string s;
     s += "  template <bool kSmall, class P>\n"
          "  static __device__ __forceinline__ void emit(const P& p, const RbSmem& s, const RbCtx& x, int64_t c0, "
-         "int nr, const PreState& ps, bool use_pre) {\n" + thread_vars() +
+         "int nr, const PreState& ps, bool use_pre, bool tail_by_dense) {\n" + thread_vars() +
          "    const Common& c = p.c;\n"
          "    const int64_t B = x.B;\n"
          "    const bool in = r < nr;\n"
-         "    const int64_t row = c0 + r;\n    (void)ps;\n    (void)use_pre;\n";
+         "    const int64_t row = c0 + r;\n    (void)ps;\n    (void)use_pre;\n    (void)tail_by_dense;\n";
     const int sp = split_point();
     if (tab_total) s += "    mbar_wait(reinterpret_cast<uint64_t*>(s.tabs), 0u);  // staged tables landed\n";
     const LoopPlan lp = loop_plan();
-    if (lp.ok) return s + emit_loop(lp) + "  }\n";
+    if (lp.ok) return s + emit_loop(lp) + "  }\n" + tail_fn(F);
     if (pairs()) s += "  if ((warp & 1) == 0) {\n";
-    s += batch_ok() ? emit_batched(0, sp) : emit_body(0, sp);
+    const int ts = pairs() ? F : tail_split();
+    if (batch_ok() && ts < F) {
+      s += "  {\n" + emit_batched(0, ts) + "  }\n";
+      s += "  if (!tail_by_dense) {\n" + emit_batched(ts, F) + "  }\n";
+    } else {
+      s += batch_ok() ? emit_batched(0, sp) : emit_body(0, sp);
+    }
     if (pairs()) s += "  } else {\n" + (batch_ok() ? emit_batched(sp, F) : emit_body(sp, F)) + "  }\n";
     s += "  }\n";
-    return s;
+    return s + tail_fn(ts);
+  }
+  // emit_tail: the outputs [ts, F) of row warp w of the chunk, by a dense warp
+  std::string tail_fn(int ts) {
+    std::string s = "  static constexpr bool kTail = " + std::string(ts < F ? "true" : "false") + ";\n";
+    s += "  template <bool kSmall, class P>\n"
+         "  static __device__ __forceinline__ void emit_tail(const P& p, const RbSmem& s, const RbCtx& x, int64_t c0, "
+         "int nr, int w) {\n";
+    if (ts >= F) return s + "  }\n";
+    s += "    const int lane = threadIdx.x & 31, wi = w, r = (w << 5) | lane;\n"
+         "    const Common& c = p.c;\n"
+         "    const int64_t B = x.B;\n"
+         "    const bool in = r < nr;\n"
+         "    const int64_t row = c0 + r;\n"
+         "    const bool use_pre = false;\n    (void)use_pre;\n";
+    if (tab_total) s += "    mbar_wait(reinterpret_cast<uint64_t*>(s.tabs), 0u);\n";
+    s += emit_batched(ts, F);
+    return s + "  }\n";
   }
   // ---- loop emitter (rap_rows_skel.cuh jl_*): the outputs as rows of
   // __constant__ tables, NGram units (k providers + the NGram) then single
@@ -930,7 +983,7 @@ struct Gen {
       }
       // (2)-(4) the values: computed here, or (batch 0 of a one-chunk block)
       // before the grid wait by pre_emit and carried over in registers
-      if (bi == 0 && pre_ok()) {
+      if (bi == 0 && qb == 0 && pre_ok()) {
         s += "    if (use_pre) {\n";
         for (int q : canon) {
           s += "      v" + i2s(q) + " = ps.v" + i2s(q) + ";\n";
@@ -1391,7 +1444,7 @@ struct Gen {
     std::string s;
     s += "  template <bool kSmall, class P>\n"
          "  static __device__ __forceinline__ void emit(const P& p, const RbSmem& s, const RbCtx& x, int64_t c0, "
-         "int nr, const PreState&, bool) {\n"
+         "int nr, const PreState&, bool, bool) {\n"
          "    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;\n"
          "    const Common& c = p.c;\n"
          "    const int64_t B = x.B;\n"
@@ -1468,7 +1521,7 @@ struct Gen {
     body += dense;
     body += lengths_fn();
     {
-      std::string e = column_mode() ? col_emit_fn() : emit_fn();
+      std::string e = column_mode() ? col_emit_fn() + tail_fn(F) : emit_fn();
       // (experiment knob RAP_JIT_NOSTORE: 1 = no output stores in the emit
       // phase, 2 = values only, 3 = lengths and offsets only; the stored
       // values fold into a sink so the computation stays)

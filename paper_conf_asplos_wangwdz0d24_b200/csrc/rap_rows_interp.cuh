@@ -309,6 +309,9 @@ struct InterpPolicy {
   static constexpr bool kDenseLate = false;
   static constexpr bool kBasesByDense = false;
   static constexpr bool kPDL = false;
+  static constexpr bool kTail = false;  // (the generated policy's dense-warp tail)
+  template <bool kSmall, class P>
+  static __device__ __forceinline__ void emit_tail(const P&, const RbSmem&, const RbCtx&, int64_t, int, int) {}
   struct PreState {};
   template <class P>
   static __device__ __forceinline__ PreState pre_emit(const P&, const RbSmem&, const RbCtx&, int64_t, int) {
@@ -365,7 +368,7 @@ struct InterpPolicy {
 
   template <bool kSmall, class P>
   static __device__ __forceinline__ void emit(const P& p, const RbSmem& s, const RbCtx& x, int64_t c0, int nr,
-                                              const PreState&, bool) {
+                                              const PreState&, bool, bool) {
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const Common& c = p.c;
     const int FL = x.FL, pb = x.pb, F = x.F;

@@ -794,6 +794,13 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
     }
     Pol::dense_warp(p, s, x);  // the dense outputs of rows [R0, R1), concurrent with the sparse phases
     trace_stamp_warp(c, 15);
+    if (Pol::kTail && nch == 1 && FL > 0 && nrows > 0) {
+      // the tail outputs of every row warp, once the sparse warps set the
+      // chunk's warp bases (named barrier 5)
+      constexpr int kND = kT / 32 - kWS;  // dense warps
+      asm volatile("bar.sync 5, %0;" ::"r"(kT) : "memory");
+      for (int w = warp - kWS; w < kWS; w += kND) Pol::template emit_tail<kSmall>(p, s, x, x.R0, nrows, w);
+    }
   } else {
 
   // (1) per-output totals of my rows -> agg, then announce the CTA
@@ -951,7 +958,9 @@ __device__ __forceinline__ void rows_body(const RbParams<MD, MS>& p) {
       }
       rb_sync<kDW>();
       if (n_ids > 0) mbar_wait(&s_ibar, (uint32_t)s_iphase);  // the chunk's staged ids landed
-      Pol::template emit<kSmall>(p, s, x, c0, nr, pre, use_pre && ch == 0);
+      const bool tail = kDW && Pol::kTail && nch == 1;  // the dense warps emit the tail outputs
+      if (tail) asm volatile("bar.arrive 5, %0;" ::"r"(kT) : "memory");  // (warp bases set above)
+      Pol::template emit<kSmall>(p, s, x, c0, nr, pre, use_pre && ch == 0, tail);
       rb_sync<kDW>();
       if (n_ids > 0 && tid == 0) s_iphase ^= 1;
     }
