@@ -71,7 +71,7 @@ int64_t sat_mul(int64_t a, int64_t b) {
 // Latency-model constants (rap_predict_latency_us): t0/c per kernel family
 // and the HBM bandwidth, fitted on B200 (profiles/r02b_cost_model_fit.txt).
 #ifndef RAP_MODEL_FIT
-#define RAP_MODEL_FIT 37.1015, 2.07606e-05, 0, 0, 12.0978, 0, 0.0102007, 0, 10.7953, 0, 0.0030039, 0, 6446.6
+#define RAP_MODEL_FIT 28.5241, 1.99159e-05, 0, 0, 12.1317, 0, 0.0101896, 0, 12.4147, 0, 0.003001, 0, 6446.6
 #endif
 
 struct rap_plan {
@@ -2034,6 +2034,11 @@ static PredTerms predict_terms(const rap_plan* P, int64_t B, const int64_t* nnz,
       }
     }
     t.pairs = (double)fmax * (double)(chunks * chunk);
+    if (jit && chunks == 1) {  // the dense-warp tail (rap_jit.cpp tail_split) takes ~20 % of the outputs' cost
+      int r0 = 0;
+      if (jit_dense_mode((int)P->souts.size(), P->d_out, (int)P->dprogs.size(), P->rb_dense_bytes, jit_pairs(P), &r0) == 3)
+        t.pairs *= 0.8;
+    }
     t.family = jit ? RAP_KERNEL_JIT : RAP_KERNEL_ROWS;
     t.grid = (int64_t)g.n_rb * g.n_fg + g.n_dcta;
     t.work = gmax * (double)(chunks * chunk);
