@@ -1904,7 +1904,14 @@ static rap_status preprocess_host_impl(rap_plan* P, const rap_raw_batch* raw, co
     }
   }
   const int64_t F = (int64_t)P->souts.size();
-  const int64_t vb = B > 0 ? values_bound(P, B, raw->sp_nnz) : 0;
+  // the staging values buffer is sized from the ids the host offsets hold
+  // (not the caller's sp_nnz, which may understate them)
+  std::vector<int64_t> host_nnz(std::max(P->n_sparse_in, 1), 0);
+  for (int s = 0; s < P->n_sparse_in; ++s)
+    if (raw->sp_offsets && raw->sp_offsets[s] && B > 0)
+      host_nnz[s] = std::max<int64_t>(raw->sp_nnz ? raw->sp_nnz[s] : 0,
+                                      (int64_t)raw->sp_offsets[s][B] - (int64_t)raw->sp_offsets[s][0]);
+  const int64_t vb = B > 0 ? values_bound(P, B, host_nnz.data()) : 0;
   int64_t drow0 = 0, drows = B;
   rap_shard_rows(B, P->rank, P->world, &drow0, &drows);
   void *dd = nullptr, *dl = nullptr, *dof = nullptr, *dv = nullptr;
