@@ -350,8 +350,19 @@ struct JitModule;  // compiled kernels (opaque)
 //      phases, each with its own tile: the dense work overlaps the emit
 //      phase, whose warps leave most issue slots idle (the default).
 inline int jit_dense_tiles(int) { return 8; }  // mode 2: warps with a tile
-constexpr int kJitDenseWarps = 3;              // mode 3
-inline int jit_dense_warps(int mode) { return mode == 3 ? kJitDenseWarps : mode == 1 ? 1 : 0; }
+#ifndef __CUDACC_RTC__
+inline int jit_dense_warps3() {  // mode 3's dense warps (RAP_JIT_DENSE_WARPS: experiment knob, read once)
+  static const int n = [] {
+    const char* e = getenv("RAP_JIT_DENSE_WARPS");
+    const int v = e ? atoi(e) : 3;
+    return v < 1 ? 1 : (v > 8 ? 8 : v);
+  }();
+  return n;
+}
+#else
+inline int jit_dense_warps3() { return 3; }
+#endif
+inline int jit_dense_warps(int mode) { return mode == 3 ? jit_dense_warps3() : mode == 1 ? 1 : 0; }
 inline int jit_dense_mode(int n_sparse_out, int d_out, int n_dprogs, int rb_dense_bytes, int pairs, int* region0) {
   const int off = ((2 * (n_sparse_out + 1) * 8) + 15) & ~15;  // after the base phase's T[f], L[f]
   const int one = 32 * (d_out | 1) * 4;
@@ -368,8 +379,8 @@ inline int jit_dense_mode(int n_sparse_out, int d_out, int n_dprogs, int rb_dens
 #else
   const int wm = 3;
 #endif
-  if (wm == 3 && !pairs && off + kJitDenseWarps * one <= 48 * 1024) {
-    *region0 = off + kJitDenseWarps * one;
+  if (wm == 3 && !pairs && off + jit_dense_warps3() * one <= 48 * 1024) {
+    *region0 = off + jit_dense_warps3() * one;
     return 3;
   }
   if (wm != 1 && off + nt * one <= 48 * 1024) {
