@@ -28,7 +28,10 @@ def test_c2_source_compiles_with_immediates(rap):
     import re
 
     listed = [int(f) for b in re.findall(r"// batch of outputs([ 0-9]+)", src) for f in b.split()]
-    assert sorted(listed) == list(range(34))
+    # every output in a batch; the dense-warp tail's outputs twice (the sparse
+    # warps' copy for multi-chunk blocks, and emit_tail)
+    assert sorted(set(listed)) == list(range(34)) and max(listed.count(f) for f in set(listed)) <= 2
+    assert "kTail = true" in src
     assert all(len(b.split()) <= 8 for b in re.findall(r"// batch of outputs([ 0-9]+)", src))
     # the trigram outputs read their memoised sources from registers
     assert src.count("(uint64_t)m") == 24
@@ -47,7 +50,7 @@ def test_c1_source_compiles(rap):
     import re
 
     listed = [int(f) for b in re.findall(r"// batch of outputs([ 0-9]+)", src) for f in b.split()]
-    assert sorted(listed) == list(range(26))
+    assert sorted(set(listed)) == list(range(26)) and max(listed.count(f) for f in set(listed)) <= 2
 
 
 @pytest.mark.parametrize("seed", range(3))
