@@ -33,8 +33,10 @@ def test_c2_source_compiles_with_immediates(rap):
     assert sorted(set(listed)) == list(range(34)) and max(listed.count(f) for f in set(listed)) <= 2
     assert "kTail = true" in src
     assert all(len(b.split()) <= 8 for b in re.findall(r"// batch of outputs([ 0-9]+)", src))
-    # the trigram outputs read their memoised sources from registers
-    assert src.count("(uint64_t)m") == 24
+    # the trigram outputs read their memoised sources from registers: 3 per
+    # trigram emission (8 trigrams, plus any the dense-warp tail re-emits)
+    n_m = src.count("(uint64_t)m")
+    assert n_m >= 24 and n_m % 3 == 0
     # every SigridHash salt is an immediate H(salt) (R3)
     from oracle import oracle
 
