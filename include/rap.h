@@ -233,7 +233,10 @@ rap_status rap_preprocess(rap_plan* plan, const rap_raw_batch* raw, const rap_ou
 /* Same as rap_preprocess with HOST raw and output buffers (pinned memory makes
  * the copies asynchronous): copies the batch into plan-owned device staging,
  * launches, copies dense/lengths/offsets and the values back, and
- * synchronises `stream` before returning.  When `values` is pinned host
+ * synchronises `stream` before returning.  When every input column is pinned
+ * (device-mapped) host memory, one gather kernel reads all of them across
+ * PCIe into the staging buffers (one launch instead of a copy per column);
+ * otherwise each column is a cudaMemcpyAsync (RAP_H2D_COPIES=1 forces that).  When `values` is pinned host
  * memory, a copy kernel moves exactly offsets[end] ids into it (no host sync,
  * no padding over PCIe); pageable memory receives the first
  * values_upper_bound ids.  Host values beyond offsets[end] are unspecified. */

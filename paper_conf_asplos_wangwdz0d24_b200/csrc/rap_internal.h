@@ -301,6 +301,8 @@ int fused_smem_bytes(int max_width);
 // rap_jagged_append's kernel (rap_kernel.cu).
 int launch_jagged_append(const int32_t* len, const int64_t* so, const int64_t* val, int64_t n, int64_t vb, int32_t* dl,
                          int64_t* dof, int64_t* dv, int64_t cap, void* stream);
+// One launch copying n device-mapped pinned host ranges into device buffers (rap_kernel.cu).
+int launch_gather_h2d(const void* const* src, void* const* dst, const int64_t* bytes, int n, void* stream);
 // Exact-size copy of values[0, *total) into device-mapped pinned host memory (rap_kernel.cu).
 int launch_values_to_host(const int64_t* src, const int64_t* total, int64_t cap, int64_t* dst, void* stream);
 // Raise a kernel's MaxDynamicSharedMemorySize on the current device to at

@@ -1542,6 +1542,79 @@ int launch_values_to_host(const int64_t* src, const int64_t* total, int64_t cap,
   return (int)cudaGetLastError();
 }
 
+// Batched H2D of a host batch's columns (rap_preprocess_host*): every column
+// lives in pinned (device-mapped) host memory, so one launch reads all of them
+// across PCIe into their staging buffers.  One copy engine transfer per column
+// (~100 for C2) costs ~8 us of engine time each and queues behind the other
+// stream's D2H; the SMs' reads overlap it.  A block moves one 32 KB chunk of
+// one copy; units are the widest of 16 / 8 / 4 / 1 bytes both ends allow.
+constexpr int kGatherMax = 192;
+constexpr int64_t kGatherChunk = 32768;
+struct GatherCopy {
+  const void* src;
+  void* dst;
+  int64_t bytes;
+  int64_t blk0;  // first block of this copy
+};
+struct GatherParams {
+  int n;
+  GatherCopy c[kGatherMax];
+};
+
+template <typename T>
+__device__ __forceinline__ void gather_chunk(const GatherCopy& c, int64_t b0, int64_t b1) {
+  const T* __restrict__ s = static_cast<const T*>(c.src);
+  T* __restrict__ d = static_cast<T*>(c.dst);
+  const int64_t u0 = b0 / (int64_t)sizeof(T), u1 = b1 / (int64_t)sizeof(T);
+  for (int64_t u = u0 + threadIdx.x; u < u1; u += 8 * 256) {
+    T v[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k)
+      if (u + k * 256 < u1) v[k] = s[u + k * 256];  // all loads in flight before the stores
+#pragma unroll
+    for (int k = 0; k < 8; ++k)
+      if (u + k * 256 < u1) d[u + k * 256] = v[k];
+  }
+  const int64_t t0 = u1 * (int64_t)sizeof(T);  // bytes past the last whole unit
+  if (threadIdx.x < b1 - t0)
+    static_cast<char*>(c.dst)[t0 + threadIdx.x] = static_cast<const char*>(c.src)[t0 + threadIdx.x];
+}
+
+__global__ void __launch_bounds__(256) gather_h2d_kernel(const __grid_constant__ GatherParams p) {
+  int lo = 0, hi = p.n - 1;  // the copy this block belongs to: last blk0 <= blockIdx.x
+  while (lo < hi) {
+    const int mid = (lo + hi + 1) >> 1;
+    if (p.c[mid].blk0 <= (int64_t)blockIdx.x) lo = mid;
+    else hi = mid - 1;
+  }
+  const GatherCopy& c = p.c[lo];
+  const int64_t b0 = ((int64_t)blockIdx.x - c.blk0) * kGatherChunk;
+  const int64_t b1 = min(c.bytes, b0 + kGatherChunk);
+  const uintptr_t a = reinterpret_cast<uintptr_t>(c.src) | reinterpret_cast<uintptr_t>(c.dst);
+  if ((a & 15) == 0) gather_chunk<int4>(c, b0, b1);
+  else if ((a & 7) == 0) gather_chunk<long long>(c, b0, b1);
+  else if ((a & 3) == 0) gather_chunk<int>(c, b0, b1);
+  else gather_chunk<char>(c, b0, b1);
+}
+
+int launch_gather_h2d(const void* const* src, void* const* dst, const int64_t* bytes, int n, void* stream) {
+  for (int i0 = 0; i0 < n; i0 += kGatherMax) {
+    GatherParams p;
+    p.n = 0;
+    int64_t blocks = 0;
+    for (int i = i0; i < n && i < i0 + kGatherMax; ++i) {
+      if (bytes[i] <= 0) continue;
+      p.c[p.n++] = GatherCopy{src[i], dst[i], bytes[i], blocks};
+      blocks += (bytes[i] + kGatherChunk - 1) / kGatherChunk;
+    }
+    if (!blocks) continue;
+    gather_h2d_kernel<<<(unsigned)blocks, 256, 0, reinterpret_cast<cudaStream_t>(stream)>>>(p);
+    const cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return (int)e;
+  }
+  return 0;
+}
+
 int launch_jagged_append(const int32_t* len, const int64_t* so, const int64_t* val, int64_t n, int64_t vb, int32_t* dl,
                          int64_t* dof, int64_t* dv, int64_t cap, void* stream) {
   const int64_t work = max(n, vb);

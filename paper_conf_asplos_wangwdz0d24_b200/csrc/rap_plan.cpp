@@ -1873,11 +1873,21 @@ static rap_status preprocess_host_impl(rap_plan* P, const rap_raw_batch* raw, co
   std::vector<const uint32_t*> d_svalid(P->n_sparse_in, nullptr);
   size_t slot = 0;
   cudaError_t e = cudaSuccess;
+  // the columns' H2D copies are collected, then issued as one gather launch
+  // when every source is device-mapped pinned memory (launch_gather_h2d), else
+  // one cudaMemcpyAsync each
+  std::vector<const void*> c_src;
+  std::vector<void*> c_dst;
+  std::vector<int64_t> c_bytes;
   auto h2d = [&](const void* src, size_t bytes, void** dst) -> rap_status {
     rap_status s = stage_buf(P, slot++, bytes, dst);
     if (s != RAP_OK) return s;
-    if (bytes) e = cudaMemcpyAsync(*dst, src, bytes, cudaMemcpyHostToDevice, stream);
-    return e == cudaSuccess ? RAP_OK : cuda_fail(e, "H2D copy");
+    if (bytes) {
+      c_src.push_back(src);
+      c_dst.push_back(*dst);
+      c_bytes.push_back((int64_t)bytes);
+    }
+    return RAP_OK;
   };
   if (B > 0) {
     for (int c : P->used_dense) {
@@ -1900,6 +1910,30 @@ static rap_status preprocess_host_impl(rap_plan* P, const rap_raw_batch* raw, co
       if (raw->sp_valid && raw->sp_valid[s]) {
         if ((st = h2d(raw->sp_valid[s], bm_bytes, &d)) != RAP_OK) return st;
         d_svalid[s] = static_cast<const uint32_t*>(d);
+      }
+    }
+  }
+  if (!c_src.empty()) {
+    static const bool copies = [] {  // "1": one cudaMemcpyAsync per column (experiment knob; read once per process)
+      const char* env = getenv("RAP_H2D_COPIES");
+      return env && env[0] == '1';
+    }();
+    std::vector<const void*> mapped(c_src.size(), nullptr);
+    bool all_mapped = !copies;
+    for (size_t i = 0; all_mapped && i < c_src.size(); ++i) {
+      cudaPointerAttributes pa;
+      all_mapped = cudaPointerGetAttributes(&pa, c_src[i]) == cudaSuccess && pa.type == cudaMemoryTypeHost &&
+                   pa.devicePointer != nullptr;
+      if (all_mapped) mapped[i] = pa.devicePointer;
+    }
+    cudaGetLastError();  // pageable pointers leave a sticky-free error behind
+    if (all_mapped) {
+      e = (cudaError_t)launch_gather_h2d(mapped.data(), c_dst.data(), c_bytes.data(), (int)c_src.size(), stream);
+      if (e != cudaSuccess) return cuda_fail(e, "H2D gather");
+    } else {
+      for (size_t i = 0; i < c_src.size(); ++i) {
+        e = cudaMemcpyAsync(c_dst[i], c_src[i], (size_t)c_bytes[i], cudaMemcpyHostToDevice, stream);
+        if (e != cudaSuccess) return cuda_fail(e, "H2D copy");
       }
     }
   }

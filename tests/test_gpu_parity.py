@@ -284,6 +284,23 @@ def test_host_buffers_entry(env):
     plan.close()
 
 
+def test_host_entry_gather_alignments(env):
+    """The host entry's batched H2D (one gather launch over pinned columns):
+    sources only 8- / 4-byte aligned (an odd first offset, a ragged offsets
+    array) and columns smaller than one chunk; pageable columns take the
+    per-column copies.  Every case equal to the oracle."""
+    rap, synth, oracle, torch = env
+    w = synth.c2_terabyte(0)
+    for B, base, where in ((4101, 3, None), (37, 5, None), (70001, 1, None), (1500, 3, "cpu")):
+        host = synth.make_batch(w, B, seed=B, base_offset=base)
+        plan = rap.Plan(w.spec, device=0)
+        raw = rap.DeviceBatch(host, where, pin=where is None)
+        out = rap.DeviceOutput(plan, B, raw.sp_nnz, None, pin=True)
+        plan.preprocess_host(raw, out)
+        assert_parity(out.to_numpy(), oracle.run(w.spec, host), ctx=f"B={B} base={base} {where or 'pinned'}")
+        plan.close()
+
+
 def test_host_async_two_plans_pipelined(env):
     """rap_preprocess_host_async: two plans on two streams, batches alternating,
     each result equal to the oracle once its stream is synchronised."""
