@@ -37,6 +37,9 @@
 // from call to call (CUDA-graph replayable).  The grid is capped by the SM
 // budget (§6.2).
 #pragma once
+#ifndef RAP_BASES_UNROLL
+#define RAP_BASES_UNROLL 4
+#endif
 #ifndef __CUDACC_RTC__
 #include <cuda_runtime.h>
 #include <stdint.h>
@@ -607,10 +610,11 @@ __device__ __forceinline__ void rb_bases_warp(const Common& c, const RbGeom& g, 
   long long* sL = sT + (fmax + 1);                          // [fmax + 1]
   for (int f = lane; f <= fmax; f += 32) sT[f] = (long long)__ldcg(g.tot + f);
   const int nsb = rb / kRbSup, rb0 = nsb * kRbSup;
-  for (int f0 = 0; f0 <= fmax; f0 += 4) {
-    long long v[4];
+  constexpr int kBU = RAP_BASES_UNROLL;  // outputs whose lower-block loads are in flight together
+  for (int f0 = 0; f0 <= fmax; f0 += kBU) {
+    long long v[kBU];
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
+    for (int u = 0; u < kBU; ++u) {
       const int f = min(f0 + u, fmax);
       long long a = 0;
       if (lane < nsb) a = (long long)__ldcg(g.sup + (int64_t)f * kRbSupMax + lane);
@@ -618,7 +622,7 @@ __device__ __forceinline__ void rb_bases_warp(const Common& c, const RbGeom& g, 
       v[u] = a;
     }
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
+    for (int u = 0; u < kBU; ++u) {
       const long long t = rb_warp_sum<kSmall>(v[u]);
       if (lane == 0 && f0 + u <= fmax) sL[f0 + u] = t;
     }
