@@ -1496,6 +1496,7 @@ struct Gen {
     if (env_int("RAP_JIT_LDCS", 0)) s += "#define RAP_LD_CS 1\n";  // (experiment knob)
     if (env_int("RAP_JIT_STPLAIN", 0)) s += "#define RAP_ST_PLAIN 1\n";  // (experiment knob)
     s += "#define RAP_BASES_UNROLL " + i2s(env_int("RAP_JIT_BASES_UNROLL", 4)) + "\n";  // (experiment knob)
+    if (env_int("RAP_JIT_PREFETCH", 0)) s += "#define RAP_PREFETCH_IDS 1\n";  // (experiment knob)
     s += "#include \"rap_rows_interp.cuh\"\n\nnamespace rapk {\n\n";
     bool records = false;  // does any output fall back to the interpreter's functions?
     for (int f = 0; f < F; ++f) records |= v.feat[f].emit != 0;

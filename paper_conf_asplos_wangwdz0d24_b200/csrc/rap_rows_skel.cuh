@@ -271,6 +271,17 @@ __device__ __forceinline__ void rb_stage(const P& p, const RbSmem& s, const int1
     if (ob) bulk_g2s(s.off + k * s.pitch, src, ob, bar);
     if (wb) bulk_g2s(s.bm + k * 8, bs, wb, bar);
     if (k < n_ids) rb_stage_ids(p.val[col], a0, a1, s.ids + k * kRbIdCap, s.ide0 + k, ibar);
+#ifdef RAP_PREFETCH_IDS
+    // the chunk's ids, read only in the emit phase, prefetched into L2 now
+    // (one bulk prefetch of the whole 16-byte units inside the range)
+    if (k >= n_ids) {
+      const int32_t b0 = __ldg(src), b1 = __ldg(src + nr);
+      const uintptr_t lo = (reinterpret_cast<uintptr_t>(p.val[col] + b0) + 15) & ~(uintptr_t)15;
+      const uintptr_t hi = reinterpret_cast<uintptr_t>(p.val[col] + b1) & ~(uintptr_t)15;
+      if (b1 > b0 && hi > lo)
+        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(lo), "r"((uint32_t)(hi - lo)) : "memory");
+    }
+#endif
   }
   // the words outside the bulk copies (an unaligned offsets tail, validity
   // words of an unaligned bitmap: 3 of 4 row blocks of 224 rows), 8 threads
