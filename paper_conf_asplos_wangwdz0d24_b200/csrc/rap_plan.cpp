@@ -1968,7 +1968,40 @@ static rap_status preprocess_host_impl(rap_plan* P, const rap_raw_batch* raw, co
   dout.values_capacity = std::max<int64_t>(vb, 0);
   if ((st = launch(P, &dr, &dout, stream)) != RAP_OK) return st;
   // D2H
-  if (drows > 0 && P->d_out > 0) {
+  static const bool d2h_gather = [] {  // "1": fixed-size outputs by one SM copy launch into mapped host memory (experiment knob)
+    const char* env = getenv("RAP_D2H_GATHER");
+    return env && env[0] == '1';
+  }();
+  bool fixed_done = false;
+  if (d2h_gather && out->dense_ld == P->d_out && !(out->flags & RAP_OUT_CHAIN)) {
+    const void* src[3];
+    void* dst[3];
+    int64_t nb[3];
+    int n = 0;
+    bool ok = true;
+    auto add = [&](const void* d, void* h, int64_t bytes) {
+      if (bytes <= 0 || !ok) return;
+      cudaPointerAttributes pa;
+      if (h == nullptr || cudaPointerGetAttributes(&pa, h) != cudaSuccess || pa.type != cudaMemoryTypeHost ||
+          pa.devicePointer == nullptr) {
+        ok = false;
+        return;
+      }
+      src[n] = d;
+      dst[n] = pa.devicePointer;
+      nb[n++] = bytes;
+    };
+    if (drows > 0 && P->d_out > 0) add(dd, out->dense_out, (int64_t)sizeof(float) * drows * P->d_out);
+    if (F > 0 && B > 0) add(dl, out->lengths, (int64_t)sizeof(int32_t) * B * F);
+    if (F > 0) add(dof, out->offsets, (int64_t)sizeof(int64_t) * (B * F + 1));
+    cudaGetLastError();
+    if (ok && n > 0) {
+      e = (cudaError_t)launch_gather_h2d(src, dst, nb, n, stream);
+      if (e != cudaSuccess) return cuda_fail(e, "D2H gather");
+      fixed_done = true;
+    }
+  }
+  if (!fixed_done && drows > 0 && P->d_out > 0) {
     if (out->dense_ld == P->d_out)
       e = cudaMemcpyAsync(out->dense_out, dd, sizeof(float) * drows * P->d_out, cudaMemcpyDeviceToHost, stream);
     else
@@ -1977,8 +2010,9 @@ static rap_status preprocess_host_impl(rap_plan* P, const rap_raw_batch* raw, co
     if (e != cudaSuccess) return cuda_fail(e, "D2H dense");
   }
   if (F > 0) {
-    if (B > 0) e = cudaMemcpyAsync(out->lengths, dl, sizeof(int32_t) * B * F, cudaMemcpyDeviceToHost, stream);
-    if (e == cudaSuccess)
+    if (B > 0 && !fixed_done)
+      e = cudaMemcpyAsync(out->lengths, dl, sizeof(int32_t) * B * F, cudaMemcpyDeviceToHost, stream);
+    if (e == cudaSuccess && !fixed_done)
       e = cudaMemcpyAsync(out->offsets, dof, sizeof(int64_t) * (B * F + 1), cudaMemcpyDeviceToHost, stream);
     if (e == cudaSuccess && vb > 0) {
       // exact count: pinned host memory is device-mapped (UVA), so a copy
